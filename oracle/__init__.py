@@ -1,0 +1,170 @@
+"""ctypes wrapper of the CPU fp64 oracle (oracle/crocco_oracle.c).
+
+TEST INFRASTRUCTURE ONLY: imported by tests/, __graft_entry__.smoke() and the
+cpu_baseline / ``--impl reference`` legs of bench.py -- never by the product
+package.  No code is shared with paper_conf_ipps_davissngmb23_b200/; the
+arithmetic lives in crocco_oracle.c, this file only marshals numpy arrays.
+
+Arrays are numpy float64, C-contiguous, shape (ncomp, P2, P1, P0) with
+Pd = n[d] + 2*g (g = 4 for state/metrics/rhs, 10 for coordinates): index
+[c, k+g, j+g, i+g] is point (i, j, k).
+"""
+from __future__ import annotations
+
+import ctypes as C
+import os
+import subprocess
+
+import numpy as np
+
+_HERE = os.path.dirname(os.path.abspath(__file__))
+_SRC = os.path.join(_HERE, "crocco_oracle.c")
+_LIB = os.path.join(_HERE, "liboracle.so")
+
+G = 4
+GC = 10
+PERIODIC, EXTRAP, DIRICHLET, WALL = 0, 1, 2, 3
+INVISCID, VISCOUS = 1, 2
+FIELD_STATE, FIELD_METRIC = 0, 1
+MU_CONST, MU_SUTHERLAND = 0, 1
+
+
+def build(force: bool = False) -> str:
+    """Compile the oracle with gcc (-O2, no FMA contraction, OpenMP)."""
+    if force or not os.path.exists(_LIB) or os.path.getmtime(_LIB) < os.path.getmtime(_SRC):
+        cmd = ["gcc", "-O2", "-ffp-contract=off", "-fno-fast-math", "-fopenmp", "-fPIC",
+               "-shared", "-std=c11", "-o", _LIB + ".tmp", _SRC, "-lm"]
+        subprocess.check_call(cmd)
+        os.replace(_LIB + ".tmp", _LIB)
+    return _LIB
+
+
+class Phys(C.Structure):
+    _fields_ = [("gamma", C.c_double), ("R", C.c_double), ("Pr", C.c_double),
+                ("mu_law", C.c_int32), ("mu_ref", C.c_double), ("T_ref", C.c_double),
+                ("S", C.c_double), ("weno_eps", C.c_double), ("terms", C.c_int32),
+                ("dir_mask", C.c_int32), ("weno_linear", C.c_int32)]
+
+
+def phys(gamma=1.4, R=1.0, Pr=0.72, mu_law=MU_CONST, mu_ref=0.0, T_ref=1.0, S=0.0,
+         weno_eps=1e-6, terms=INVISCID | VISCOUS, dir_mask=7, weno_linear=0) -> Phys:
+    return Phys(gamma, R, Pr, mu_law, mu_ref, T_ref, S, weno_eps, terms, dir_mask, weno_linear)
+
+
+_lib = None
+
+
+def lib():
+    global _lib
+    if _lib is None:
+        L = C.CDLL(build())
+        dp = C.POINTER(C.c_double)
+        i64p = C.POINTER(C.c_int64)
+        i32p = C.POINTER(C.c_int32)
+        L.oracle_fill.argtypes = [i64p, i32p, dp, dp, C.c_int32, C.c_int32]
+        L.oracle_metrics.argtypes = [i64p, i32p, dp, dp]
+        L.oracle_weno_symbo.argtypes = [dp, C.c_double, C.c_int]
+        L.oracle_weno_symbo.restype = C.c_double
+        L.oracle_eigvecs.argtypes = [dp, C.c_double, C.c_double, C.c_double, C.c_double,
+                                     C.c_double, C.c_double, dp, dp]
+        L.oracle_interface_flux.argtypes = [C.POINTER(Phys), dp, dp, dp]
+        L.oracle_rhs.argtypes = [i64p, C.POINTER(Phys), dp, dp, dp]
+        L.oracle_rk_update.argtypes = [i64p, C.c_int32, C.c_double, dp, dp, dp, dp]
+        L.oracle_rk_stage.argtypes = [i64p, i32p, dp, C.POINTER(Phys), C.c_int32, C.c_double,
+                                      dp, dp, dp, dp]
+        L.oracle_advance.argtypes = [i64p, i32p, dp, C.POINTER(Phys), C.c_double, C.c_int32,
+                                     dp, dp]
+        L.oracle_set_threads.argtypes = [C.c_int]
+        L.oracle_get_threads.restype = C.c_int
+        _lib = L
+    return _lib
+
+
+def _dp(a: np.ndarray):
+    assert a.dtype == np.float64 and a.flags.c_contiguous
+    return a.ctypes.data_as(C.POINTER(C.c_double))
+
+
+def _n(n):
+    return (C.c_int64 * 3)(*[int(x) for x in n])
+
+
+def _bc(bc):
+    flat = [int(x) for pair in bc for x in pair]
+    return (C.c_int32 * 6)(*flat)
+
+
+def _dir(dirichlet):
+    arr = np.zeros(30) if dirichlet is None else np.ascontiguousarray(dirichlet, dtype=np.float64).reshape(30)
+    return arr
+
+
+def padded(n, ncomp, g=G):
+    return np.zeros((ncomp, n[2] + 2 * g, n[1] + 2 * g, n[0] + 2 * g))
+
+
+def set_threads(k: int):
+    lib().oracle_set_threads(int(k))
+
+
+def get_threads() -> int:
+    return int(lib().oracle_get_threads())
+
+
+def fill(n, bc, f, kind=FIELD_STATE, dirichlet=None):
+    """FillPatch + BC_Fill in place."""
+    d = _dir(dirichlet)
+    lib().oracle_fill(_n(n), _bc(bc), _dp(d), _dp(f), f.shape[0], kind)
+    return f
+
+
+def metrics(n, bc, xyz):
+    """10-component metrics (J, m^d_a) on the padded box from coordinates."""
+    met = padded(n, 10)
+    lib().oracle_metrics(_n(n), _bc(bc), _dp(np.ascontiguousarray(xyz)), _dp(met))
+    return met
+
+
+def weno_symbo(v, eps=1e-6, linear=False) -> float:
+    a = np.ascontiguousarray(v, dtype=np.float64)
+    return float(lib().oracle_weno_symbo(_dp(a), eps, int(linear)))
+
+
+def eigvecs(nrm, rho, u, v, w, c, gamma=1.4):
+    T = np.zeros(25)
+    Ti = np.zeros(25)
+    a = np.ascontiguousarray(nrm, dtype=np.float64)
+    lib().oracle_eigvecs(_dp(a), rho, u, v, w, c, gamma, _dp(T), _dp(Ti))
+    return T.reshape(5, 5), Ti.reshape(5, 5)
+
+
+def interface_flux(ph: Phys, Ul, ml):
+    Ua = np.ascontiguousarray(Ul, dtype=np.float64).reshape(30)
+    ma = np.ascontiguousarray(ml, dtype=np.float64).reshape(18)
+    F = np.zeros(5)
+    lib().oracle_interface_flux(C.byref(ph), _dp(Ua), _dp(ma), _dp(F))
+    return F
+
+
+def rhs(n, ph: Phys, U, met):
+    """rhs = J(-sum delta F_inv + sum D4 F_v) on interior points (ghosts of U must be filled)."""
+    out = padded(n, 5)
+    lib().oracle_rhs(_n(n), C.byref(ph), _dp(U), _dp(met), _dp(out))
+    return out
+
+
+def rk_update(n, stage, dt, Uin, Uout, dU, r):
+    lib().oracle_rk_update(_n(n), stage, dt, _dp(Uin), _dp(Uout), _dp(dU), _dp(r))
+
+
+def rk_stage(n, bc, ph, stage, dt, Uin, Uout, dU, met, dirichlet=None):
+    d = _dir(dirichlet)
+    lib().oracle_rk_stage(_n(n), _bc(bc), _dp(d), C.byref(ph), stage, dt, _dp(Uin), _dp(Uout),
+                          _dp(dU), _dp(met))
+
+
+def advance(n, bc, ph, dt, nsteps, U, met, dirichlet=None):
+    """nsteps RK3 steps in place on U (padded), ghosts filled on return."""
+    d = _dir(dirichlet)
+    lib().oracle_advance(_n(n), _bc(bc), _dp(d), C.byref(ph), dt, nsteps, _dp(U), _dp(met))
+    return U

@@ -1,0 +1,688 @@
+/*
+ * crocco_oracle.c -- CPU fp64 ORACLE for the CRoCCo v2.0 hot path.
+ *
+ * TEST INFRASTRUCTURE ONLY.  Only tests/, __graft_entry__.smoke() and the
+ * cpu_baseline / --impl reference legs of bench.py may load this library.
+ * It shares no source, header, table or helper with the CUDA product path
+ * (paper_conf_ipps_davissngmb23_b200/csrc); the only thing both sides see is
+ * the seeded input generators in synth/.
+ *
+ * What it computes (citations are PAPER.md line numbers, /root/reference;
+ * "reading N" = row N of the readings table in DESIGN.md section 3):
+ *   - conservation laws, single species (Eq. 1-2; reading 1-2)
+ *   - generalised curvilinear strong-conservation form (reading 4)
+ *   - grid metrics from coordinates held in memory (Alg.1 l.2, 139, 149;
+ *     reading 5-6): Thomas-Lombard metrics with the 6th-order central operator D6
+ *   - ghost fill FillPatch + BC_Fill (Alg.2 l.3-4; reading 7,15,16)
+ *   - WENO-SYMBO characteristic inviscid fluxes per direction WENOx/y/z
+ *     (Alg.2 l.5-7; readings 8-11)
+ *   - 4th-order central viscous + heat fluxes "Viscous" (Alg.2 l.8; reading 12)
+ *   - low-storage RK3 "Update" (Alg.2 l.1,9; reading 13, Williamson 1980)
+ *
+ * Style: plain loops, full scratch arrays, one formula per statement, no
+ * blocking, no fusion.  Compile with -O2 -ffp-contract=off (no FMA contraction).
+ * Parity pins for every function are in tests/test_oracle_*.py.
+ *
+ * Array layout (all arrays fp64, component-major SoA, C order):
+ *   a padded box with ghost width g around n[0] x n[1] x n[2] interior points:
+ *   element (c, i, j, k), i in [-g, n0+g) ... , is at
+ *     c*P0*P1*P2 + (i+g) + P0*((j+g) + P1*(k+g)),  Pd = n[d] + 2g.
+ *   state / metric / rhs arrays use g = 4, coordinates use g = 10.
+ *   metric components: 0 = J, 1 + 3*d + a = m^d_a = (d xi_d / d x_a) / J.
+ */
+#include <math.h>
+#include <stdint.h>
+#include <stdlib.h>
+#include <string.h>
+#ifdef _OPENMP
+#include <omp.h>
+#endif
+
+#define OG 4   /* ghost width of state/metric arrays (reading 7) */
+#define OGC 10 /* ghost width of the coordinate array (reading 7) */
+
+enum { O_PERIODIC = 0, O_EXTRAP = 1, O_DIRICHLET = 2, O_WALL = 3 };
+enum { O_INVISCID = 1, O_VISCOUS = 2 };
+enum { O_FIELD_STATE = 0, O_FIELD_METRIC = 1 };
+
+typedef struct {
+    double gamma, R, Pr;
+    int32_t mu_law;
+    double mu_ref, T_ref, S;
+    double weno_eps;
+    int32_t terms, dir_mask;
+    int32_t weno_linear; /* test flag: 1 forces omega_k = C_k (linear stencil) */
+} oracle_phys;
+
+typedef struct {
+    int64_t n[3];
+    int64_t p[3];
+    int64_t g;
+    int64_t cs; /* component stride */
+} obox;
+
+static obox make_box(const int64_t n[3], int64_t g)
+{
+    obox b;
+    for (int d = 0; d < 3; d++) {
+        b.n[d] = n[d];
+        b.p[d] = n[d] + 2 * g;
+    }
+    b.g = g;
+    b.cs = b.p[0] * b.p[1] * b.p[2];
+    return b;
+}
+
+static inline int64_t IX(const obox *b, int64_t i, int64_t j, int64_t k)
+{
+    return (i + b->g) + b->p[0] * ((j + b->g) + b->p[1] * (k + b->g));
+}
+
+static int g_threads = 0;
+void oracle_set_threads(int n) { g_threads = n; }
+int oracle_get_threads(void)
+{
+#ifdef _OPENMP
+    return g_threads > 0 ? g_threads : omp_get_max_threads();
+#else
+    return 1;
+#endif
+}
+#ifdef _OPENMP
+#define OMP_THREADS num_threads(oracle_get_threads())
+#endif
+
+/* ------------------------------------------------------------------ */
+/* 1. Ghost fill: FillPatch (periodic / inter-block copies) + BC_Fill  */
+/*    (readings 15-16).  Three ordered phases    */
+/*    xi -> eta -> zeta; phase d spans the ghosts of directions < d.   */
+/* ------------------------------------------------------------------ */
+void oracle_fill(const int64_t n[3], const int32_t bc[6], const double dirichlet[30],
+                 double *f, int32_t ncomp, int32_t kind)
+{
+    obox b = make_box(n, OG);
+    for (int d = 0; d < 3; d++) {
+        int64_t lo[3], hi[3];
+        for (int e = 0; e < 3; e++) {
+            lo[e] = (e < d) ? -OG : 0;
+            hi[e] = (e < d) ? n[e] + OG : n[e];
+        }
+        for (int side = 0; side < 2; side++) {
+            int kindbc = bc[2 * d + side];
+            if (kind == O_FIELD_METRIC && kindbc != O_PERIODIC)
+                continue; /* metrics: only periodic copies; physical faces keep computed ghosts */
+            for (int64_t gg = 1; gg <= OG; gg++) {
+                int64_t dst = side == 0 ? -gg : n[d] - 1 + gg;
+                int64_t src;
+                double sgn_mom = 1.0;
+                switch (kindbc) {
+                case O_PERIODIC: src = side == 0 ? n[d] - gg : gg - 1; break;
+                case O_EXTRAP: src = side == 0 ? 0 : n[d] - 1; break;
+                case O_WALL:
+                    src = side == 0 ? gg - 1 : n[d] - gg;
+                    sgn_mom = -1.0;
+                    break;
+                default: src = 0; break; /* DIRICHLET: constant state */
+                }
+                for (int64_t c2 = lo[(d + 2) % 3]; c2 < hi[(d + 2) % 3]; c2++)
+                    for (int64_t c1 = lo[(d + 1) % 3]; c1 < hi[(d + 1) % 3]; c1++) {
+                        int64_t id[3], is[3];
+                        id[d] = dst;
+                        is[d] = src;
+                        id[(d + 1) % 3] = is[(d + 1) % 3] = c1;
+                        id[(d + 2) % 3] = is[(d + 2) % 3] = c2;
+                        int64_t pd = IX(&b, id[0], id[1], id[2]);
+                        int64_t ps = IX(&b, is[0], is[1], is[2]);
+                        for (int c = 0; c < ncomp; c++) {
+                            double v;
+                            if (kindbc == O_DIRICHLET)
+                                v = dirichlet[(2 * d + side) * 5 + c];
+                            else
+                                v = f[c * b.cs + ps];
+                            if (kindbc == O_WALL && c >= 1 && c <= 3)
+                                v = sgn_mom * v;
+                            f[c * b.cs + pd] = v;
+                        }
+                    }
+            }
+        }
+    }
+}
+
+/* ------------------------------------------------------------------ */
+/* 2. Grid metrics (readings 5-6).              */
+/*    D6 f_i = [45(f_{i+1}-f_{i-1}) - 9(f_{i+2}-f_{i-2}) + (f_{i+3}-f_{i-3})]/60 */
+/*    dx[a][d] = D6_d x_a ;  1/J = det(dx)                             */
+/*    m^d_a = D6_{d+2}[(D6_{d+1} x_{a+1}) x_{a+2}]                     */
+/*          - D6_{d+1}[(D6_{d+2} x_{a+1}) x_{a+2}]   (indices mod 3)   */
+/* ------------------------------------------------------------------ */
+static double d6(const double *f, int64_t p, int64_t s)
+{
+    return (45.0 * (f[p + s] - f[p - s]) - 9.0 * (f[p + 2 * s] - f[p - 2 * s]) +
+            (f[p + 3 * s] - f[p - 3 * s])) / 60.0;
+}
+
+void oracle_metrics(const int64_t n[3], const int32_t bc[6], const double *xyz, double *met)
+{
+    obox bc_ = make_box(n, OGC); /* coordinate box */
+    obox bm = make_box(n, OG);   /* metric box */
+    int64_t sc[3] = {1, bc_.p[0], bc_.p[0] * bc_.p[1]};
+    const int64_t W1 = OG + 3; /* derivatives needed on interior +-7 */
+
+    /* dx[a][d] on the coordinate layout */
+    double *dx = (double *)calloc((size_t)(9 * bc_.cs), sizeof(double));
+    for (int a = 0; a < 3; a++)
+        for (int d = 0; d < 3; d++) {
+            const double *x = xyz + a * bc_.cs;
+            double *out = dx + (3 * a + d) * bc_.cs;
+#pragma omp parallel for OMP_THREADS
+            for (int64_t k = -W1; k < n[2] + W1; k++)
+                for (int64_t j = -W1; j < n[1] + W1; j++)
+                    for (int64_t i = -W1; i < n[0] + W1; i++) {
+                        int64_t p = IX(&bc_, i, j, k);
+                        out[p] = d6(x, p, sc[d]);
+                    }
+        }
+
+    /* product fields P[a][d][e] = (D6_e x_{a+1}) * x_{a+2}, then outer D6 */
+    double *prod = (double *)calloc((size_t)bc_.cs, sizeof(double));
+    for (int d = 0; d < 3; d++)
+        for (int a = 0; a < 3; a++) {
+            int d1 = (d + 1) % 3, d2 = (d + 2) % 3;
+            int a1 = (a + 1) % 3, a2 = (a + 2) % 3;
+            double *m = met + (1 + 3 * d + a) * bm.cs;
+            /* term 1: D6_{d2}[ (D6_{d1} x_{a1}) x_{a2} ] */
+            const double *x2 = xyz + a2 * bc_.cs;
+            const double *g1 = dx + (3 * a1 + d1) * bc_.cs;
+#pragma omp parallel for OMP_THREADS
+            for (int64_t k = -W1; k < n[2] + W1; k++)
+                for (int64_t j = -W1; j < n[1] + W1; j++)
+                    for (int64_t i = -W1; i < n[0] + W1; i++) {
+                        int64_t p = IX(&bc_, i, j, k);
+                        prod[p] = g1[p] * x2[p];
+                    }
+#pragma omp parallel for OMP_THREADS
+            for (int64_t k = -OG; k < n[2] + OG; k++)
+                for (int64_t j = -OG; j < n[1] + OG; j++)
+                    for (int64_t i = -OG; i < n[0] + OG; i++)
+                        m[IX(&bm, i, j, k)] = d6(prod, IX(&bc_, i, j, k), sc[d2]);
+            /* term 2: - D6_{d1}[ (D6_{d2} x_{a1}) x_{a2} ] */
+            const double *g2 = dx + (3 * a1 + d2) * bc_.cs;
+#pragma omp parallel for OMP_THREADS
+            for (int64_t k = -W1; k < n[2] + W1; k++)
+                for (int64_t j = -W1; j < n[1] + W1; j++)
+                    for (int64_t i = -W1; i < n[0] + W1; i++) {
+                        int64_t p = IX(&bc_, i, j, k);
+                        prod[p] = g2[p] * x2[p];
+                    }
+#pragma omp parallel for OMP_THREADS
+            for (int64_t k = -OG; k < n[2] + OG; k++)
+                for (int64_t j = -OG; j < n[1] + OG; j++)
+                    for (int64_t i = -OG; i < n[0] + OG; i++)
+                        m[IX(&bm, i, j, k)] = m[IX(&bm, i, j, k)] - d6(prod, IX(&bc_, i, j, k), sc[d1]);
+        }
+
+    /* J = 1 / det(dx) */
+#pragma omp parallel for OMP_THREADS
+    for (int64_t k = -OG; k < n[2] + OG; k++)
+        for (int64_t j = -OG; j < n[1] + OG; j++)
+            for (int64_t i = -OG; i < n[0] + OG; i++) {
+                int64_t p = IX(&bc_, i, j, k);
+                double M[3][3];
+                for (int a = 0; a < 3; a++)
+                    for (int d = 0; d < 3; d++)
+                        M[a][d] = dx[(3 * a + d) * bc_.cs + p];
+                double det = M[0][0] * (M[1][1] * M[2][2] - M[1][2] * M[2][1]) -
+                             M[0][1] * (M[1][0] * M[2][2] - M[1][2] * M[2][0]) +
+                             M[0][2] * (M[1][0] * M[2][1] - M[1][1] * M[2][0]);
+                met[IX(&bm, i, j, k)] = 1.0 / det;
+            }
+    free(prod);
+    free(dx);
+    /* periodic ghost metrics are copies from the owners (reading 6) */
+    oracle_fill(n, bc, NULL, met, 10, O_FIELD_METRIC);
+}
+
+/* ------------------------------------------------------------------ */
+/* 3. WENO-SYMBO reconstruction (PAPER.md:50 -> ref [9]; reading 8)   */
+/*    W(v_{-2..3}) reconstructs the value at the +1/2 interface.       */
+/* ------------------------------------------------------------------ */
+static const double C_SYMBO[4] = {0.094647545896, 0.428074212384, 0.408289331408, 0.068988910311};
+
+double oracle_weno_symbo(const double v[6], double eps, int linear)
+{
+    /* v[0..5] = v_{-2}, v_{-1}, v_0, v_1, v_2, v_3 */
+    double q[4], beta[4];
+    q[0] = v[0] / 3.0 - 7.0 * v[1] / 6.0 + 11.0 * v[2] / 6.0;
+    q[1] = -v[1] / 6.0 + 5.0 * v[2] / 6.0 + v[3] / 3.0;
+    q[2] = v[2] / 3.0 + 5.0 * v[3] / 6.0 - v[4] / 6.0;
+    q[3] = 11.0 * v[3] / 6.0 - 7.0 * v[4] / 6.0 + v[5] / 3.0;
+    double t;
+    t = v[0] - 2.0 * v[1] + v[2];
+    beta[0] = 13.0 / 12.0 * t * t;
+    t = v[0] - 4.0 * v[1] + 3.0 * v[2];
+    beta[0] = beta[0] + 0.25 * t * t;
+    t = v[1] - 2.0 * v[2] + v[3];
+    beta[1] = 13.0 / 12.0 * t * t;
+    t = v[1] - v[3];
+    beta[1] = beta[1] + 0.25 * t * t;
+    t = v[2] - 2.0 * v[3] + v[4];
+    beta[2] = 13.0 / 12.0 * t * t;
+    t = 3.0 * v[2] - 4.0 * v[3] + v[4];
+    beta[2] = beta[2] + 0.25 * t * t;
+    t = v[3] - 2.0 * v[4] + v[5];
+    beta[3] = 13.0 / 12.0 * t * t;
+    t = -5.0 * v[3] + 8.0 * v[4] - 3.0 * v[5];
+    beta[3] = beta[3] + 0.25 * t * t;
+    /* the downwind stencil is never the smoothest: beta_3 = max(beta_0..beta_3) */
+    double bmax = beta[0];
+    for (int k = 1; k < 4; k++)
+        if (beta[k] > bmax)
+            bmax = beta[k];
+    beta[3] = bmax;
+    double alpha[4], asum = 0.0, num = 0.0;
+    for (int k = 0; k < 4; k++) {
+        if (linear)
+            alpha[k] = C_SYMBO[k];
+        else
+            alpha[k] = C_SYMBO[k] / ((eps + beta[k]) * (eps + beta[k]));
+        asum = asum + alpha[k];
+    }
+    for (int k = 0; k < 4; k++)
+        num = num + alpha[k] * q[k];
+    return num / asum;
+}
+
+/* ------------------------------------------------------------------ */
+/* 4. Pulliam-Chaussee eigenvectors of A_n = dF_n/dU (reading 9)      */
+/*    Columns of T <-> eigenvalues (theta, theta, theta, theta+c, theta-c). */
+/* ------------------------------------------------------------------ */
+void oracle_eigvecs(const double nrm[3], double rho, double u, double v, double w, double c,
+                    double gamma, double T[25], double Ti[25])
+{
+    double nx = nrm[0], ny = nrm[1], nz = nrm[2];
+    double gm1 = gamma - 1.0;
+    double phi2 = 0.5 * gm1 * (u * u + v * v + w * w);
+    double alpha = rho / (sqrt(2.0) * c);
+    double beta = 1.0 / (sqrt(2.0) * rho * c);
+    double theta = nx * u + ny * v + nz * w;
+    double c2 = c * c;
+    /* right eigenvectors, row-major T[r*5+s] */
+    T[0] = nx;
+    T[1] = ny;
+    T[2] = nz;
+    T[3] = alpha;
+    T[4] = alpha;
+    T[5] = nx * u;
+    T[6] = ny * u - nz * rho;
+    T[7] = nz * u + ny * rho;
+    T[8] = alpha * (u + nx * c);
+    T[9] = alpha * (u - nx * c);
+    T[10] = nx * v + nz * rho;
+    T[11] = ny * v;
+    T[12] = nz * v - nx * rho;
+    T[13] = alpha * (v + ny * c);
+    T[14] = alpha * (v - ny * c);
+    T[15] = nx * w - ny * rho;
+    T[16] = ny * w + nx * rho;
+    T[17] = nz * w;
+    T[18] = alpha * (w + nz * c);
+    T[19] = alpha * (w - nz * c);
+    T[20] = nx * phi2 / gm1 + rho * (nz * v - ny * w);
+    T[21] = ny * phi2 / gm1 + rho * (nx * w - nz * u);
+    T[22] = nz * phi2 / gm1 + rho * (ny * u - nx * v);
+    T[23] = alpha * ((phi2 + c2) / gm1 + c * theta);
+    T[24] = alpha * ((phi2 + c2) / gm1 - c * theta);
+    /* left eigenvectors T^{-1} */
+    Ti[0] = nx * (1.0 - phi2 / c2) - (nz * v - ny * w) / rho;
+    Ti[1] = nx * gm1 * u / c2;
+    Ti[2] = nz / rho + nx * gm1 * v / c2;
+    Ti[3] = -ny / rho + nx * gm1 * w / c2;
+    Ti[4] = -nx * gm1 / c2;
+    Ti[5] = ny * (1.0 - phi2 / c2) - (nx * w - nz * u) / rho;
+    Ti[6] = -nz / rho + ny * gm1 * u / c2;
+    Ti[7] = ny * gm1 * v / c2;
+    Ti[8] = nx / rho + ny * gm1 * w / c2;
+    Ti[9] = -ny * gm1 / c2;
+    Ti[10] = nz * (1.0 - phi2 / c2) - (ny * u - nx * v) / rho;
+    Ti[11] = ny / rho + nz * gm1 * u / c2;
+    Ti[12] = -nx / rho + nz * gm1 * v / c2;
+    Ti[13] = nz * gm1 * w / c2;
+    Ti[14] = -nz * gm1 / c2;
+    Ti[15] = beta * (phi2 - c * theta);
+    Ti[16] = beta * (nx * c - gm1 * u);
+    Ti[17] = beta * (ny * c - gm1 * v);
+    Ti[18] = beta * (nz * c - gm1 * w);
+    Ti[19] = beta * gm1;
+    Ti[20] = beta * (phi2 + c * theta);
+    Ti[21] = -beta * (nx * c + gm1 * u);
+    Ti[22] = -beta * (ny * c + gm1 * v);
+    Ti[23] = -beta * (nz * c + gm1 * w);
+    Ti[24] = beta * gm1;
+}
+
+/* ------------------------------------------------------------------ */
+/* 5. Characteristic WENO interface flux (PAPER.md:50, 110-112;        */
+/*    readings 8-11).  Inputs: the 6 conserved states U_{i-2..i+3} and */
+/*    the metric row m^d at the same 6 points.  Output F^_{i+1/2}.     */
+/* ------------------------------------------------------------------ */
+void oracle_interface_flux(const oracle_phys *ph, const double Ul[30], const double ml[18],
+                           double Fhat[5])
+{
+    const double gam = ph->gamma, gm1 = ph->gamma - 1.0;
+    /* frozen interface metric: R6 reconstruction (reading 6) */
+    double mh[3];
+    for (int a = 0; a < 3; a++)
+        mh[a] = (37.0 * (ml[2 * 3 + a] + ml[3 * 3 + a]) - 8.0 * (ml[1 * 3 + a] + ml[4 * 3 + a]) +
+                 (ml[0 * 3 + a] + ml[5 * 3 + a])) / 60.0;
+    double mag = sqrt(mh[0] * mh[0] + mh[1] * mh[1] + mh[2] * mh[2]);
+    double nrm[3] = {mh[0] / mag, mh[1] / mag, mh[2] / mag};
+
+    /* primitive variables at the 6 points */
+    double rho[6], u[6], v[6], w[6], p[6], c[6], H[6];
+    for (int l = 0; l < 6; l++) {
+        const double *U = Ul + 5 * l;
+        rho[l] = U[0];
+        u[l] = U[1] / U[0];
+        v[l] = U[2] / U[0];
+        w[l] = U[3] / U[0];
+        p[l] = gm1 * (U[4] - 0.5 * rho[l] * (u[l] * u[l] + v[l] * v[l] + w[l] * w[l]));
+        c[l] = sqrt(gam * p[l] / rho[l]);
+        H[l] = (U[4] + p[l]) / rho[l];
+    }
+    /* Roe average of points i (l=2) and i+1 (l=3) */
+    double r = sqrt(rho[3] / rho[2]);
+    double ut = (u[2] + r * u[3]) / (1.0 + r);
+    double vt = (v[2] + r * v[3]) / (1.0 + r);
+    double wt = (w[2] + r * w[3]) / (1.0 + r);
+    double Ht = (H[2] + r * H[3]) / (1.0 + r);
+    double rhot = r * rho[2];
+    double ct = sqrt(gm1 * (Ht - 0.5 * (ut * ut + vt * vt + wt * wt)));
+    double T[25], Ti[25];
+    oracle_eigvecs(nrm, rhot, ut, vt, wt, ct, gam, T, Ti);
+
+    /* projected fluxes and states, characteristic speeds */
+    double g[5][6], wv[5][6], lam[5];
+    for (int s = 0; s < 5; s++)
+        lam[s] = 0.0;
+    for (int l = 0; l < 6; l++) {
+        const double *U = Ul + 5 * l;
+        double th = nrm[0] * u[l] + nrm[1] * v[l] + nrm[2] * w[l];
+        double Fn[5];
+        Fn[0] = rho[l] * th;
+        Fn[1] = U[1] * th + nrm[0] * p[l];
+        Fn[2] = U[2] * th + nrm[1] * p[l];
+        Fn[3] = U[3] * th + nrm[2] * p[l];
+        Fn[4] = (U[4] + p[l]) * th;
+        double eig[5] = {th, th, th, th + c[l], th - c[l]};
+        for (int s = 0; s < 5; s++) {
+            double gs = 0.0, ws = 0.0;
+            for (int q = 0; q < 5; q++) {
+                gs = gs + Ti[5 * s + q] * Fn[q];
+                ws = ws + Ti[5 * s + q] * U[q];
+            }
+            g[s][l] = gs;
+            wv[s][l] = ws;
+            if (fabs(eig[s]) > lam[s])
+                lam[s] = fabs(eig[s]);
+        }
+    }
+    /* local Lax-Friedrichs splitting + WENO-SYMBO per characteristic field */
+    double gh[5];
+    for (int s = 0; s < 5; s++) {
+        double vp[6], vm[6];
+        for (int l = 0; l < 6; l++) {
+            vp[l] = 0.5 * (g[s][l] + lam[s] * wv[s][l]);
+            vm[5 - l] = 0.5 * (g[s][l] - lam[s] * wv[s][l]); /* mirrored: i+3 .. i-2 */
+        }
+        gh[s] = oracle_weno_symbo(vp, ph->weno_eps, ph->weno_linear) +
+                oracle_weno_symbo(vm, ph->weno_eps, ph->weno_linear);
+    }
+    for (int q = 0; q < 5; q++) {
+        double f = 0.0;
+        for (int s = 0; s < 5; s++)
+            f = f + T[5 * q + s] * gh[s];
+        Fhat[q] = mag * f;
+    }
+}
+
+/* ------------------------------------------------------------------ */
+/* 6. Right-hand side (readings 4, 12)        */
+/*    rhs = J ( -sum_d delta_d F^_inv^d + sum_d D4_d F^_v^d )          */
+/*    on interior points; U must have its ghosts filled.               */
+/* ------------------------------------------------------------------ */
+static double mu_of_T(const oracle_phys *ph, double T)
+{
+    if (ph->mu_law == 1) {
+        double t = T / ph->T_ref;
+        return ph->mu_ref * t * sqrt(t) * (ph->T_ref + ph->S) / (T + ph->S);
+    }
+    return ph->mu_ref;
+}
+
+static double d4(const double *f, int64_t p, int64_t s)
+{
+    return (8.0 * (f[p + s] - f[p - s]) - (f[p + 2 * s] - f[p - 2 * s])) / 12.0;
+}
+
+void oracle_rhs(const int64_t n[3], const oracle_phys *ph, const double *U, const double *met,
+                double *rhs)
+{
+    obox b = make_box(n, OG);
+    const int64_t cs = b.cs;
+    int64_t st[3] = {1, b.p[0], b.p[0] * b.p[1]};
+    double *R = (double *)calloc((size_t)(5 * cs), sizeof(double));
+
+    /* --- inviscid: WENOx, WENOy, WENOz (Alg. 2 l.5-7) --- */
+    if (ph->terms & O_INVISCID) {
+        for (int d = 0; d < 3; d++) {
+            if (!(ph->dir_mask & (1 << d)))
+                continue;
+            int e1 = (d + 1) % 3, e2 = (d + 2) % 3;
+            /* F[c][ (i+1) + (n_d+1)*line ] for interfaces i+1/2, i = -1 .. n_d-1 */
+            int64_t nl = n[e1] * n[e2];
+            double *F = (double *)malloc((size_t)(5 * (n[d] + 1) * nl) * sizeof(double));
+#pragma omp parallel for OMP_THREADS
+            for (int64_t line = 0; line < nl; line++) {
+                int64_t idx[3];
+                idx[e1] = line % n[e1];
+                idx[e2] = line / n[e1];
+                for (int64_t i = -1; i < n[d]; i++) {
+                    double Ul[30], ml[18], Fh[5];
+                    for (int l = 0; l < 6; l++) {
+                        idx[d] = i - 2 + l;
+                        int64_t p = IX(&b, idx[0], idx[1], idx[2]);
+                        for (int c = 0; c < 5; c++)
+                            Ul[5 * l + c] = U[c * cs + p];
+                        for (int a = 0; a < 3; a++)
+                            ml[3 * l + a] = met[(1 + 3 * d + a) * cs + p];
+                    }
+                    oracle_interface_flux(ph, Ul, ml, Fh);
+                    for (int c = 0; c < 5; c++)
+                        F[c * (n[d] + 1) * nl + (i + 1) + (n[d] + 1) * line] = Fh[c];
+                }
+            }
+#pragma omp parallel for OMP_THREADS
+            for (int64_t line = 0; line < nl; line++) {
+                int64_t idx[3];
+                idx[e1] = line % n[e1];
+                idx[e2] = line / n[e1];
+                for (int64_t i = 0; i < n[d]; i++) {
+                    idx[d] = i;
+                    int64_t p = IX(&b, idx[0], idx[1], idx[2]);
+                    for (int c = 0; c < 5; c++) {
+                        double fp = F[c * (n[d] + 1) * nl + (i + 1) + (n[d] + 1) * line];
+                        double fm = F[c * (n[d] + 1) * nl + i + (n[d] + 1) * line];
+                        R[c * cs + p] = R[c * cs + p] - (fp - fm);
+                    }
+                }
+            }
+            free(F);
+        }
+    }
+
+    /* --- viscous and heat fluxes (Alg. 2 l.8) --- */
+    if (ph->terms & O_VISCOUS) {
+        const double gm1 = ph->gamma - 1.0;
+        const double cp = ph->gamma * ph->R / gm1;
+        double *pr = (double *)malloc((size_t)(4 * cs) * sizeof(double)); /* u v w T */
+#pragma omp parallel for OMP_THREADS
+        for (int64_t p = 0; p < cs; p++) {
+            double rho = U[p];
+            double u = U[cs + p] / rho, v = U[2 * cs + p] / rho, w = U[3 * cs + p] / rho;
+            double pres = gm1 * (U[4 * cs + p] - 0.5 * rho * (u * u + v * v + w * w));
+            pr[p] = u;
+            pr[cs + p] = v;
+            pr[2 * cs + p] = w;
+            pr[3 * cs + p] = pres / (rho * ph->R);
+        }
+        /* point viscous fluxes Fv[d][q], q = 0..3 -> momentum x,y,z and energy,
+           on the interior +-2 box */
+        double *Fv = (double *)calloc((size_t)(12 * cs), sizeof(double));
+#pragma omp parallel for OMP_THREADS
+        for (int64_t k = -2; k < n[2] + 2; k++)
+            for (int64_t j = -2; j < n[1] + 2; j++)
+                for (int64_t i = -2; i < n[0] + 2; i++) {
+                    int64_t p = IX(&b, i, j, k);
+                    double gc[4][3]; /* d phi / d xi_d */
+                    for (int f = 0; f < 4; f++)
+                        for (int d = 0; d < 3; d++)
+                            gc[f][d] = d4(pr + f * cs, p, st[d]);
+                    double J = met[p];
+                    double m[3][3];
+                    for (int d = 0; d < 3; d++)
+                        for (int a = 0; a < 3; a++)
+                            m[d][a] = met[(1 + 3 * d + a) * cs + p];
+                    double gx[4][3]; /* d phi / d x_a = J sum_d m^d_a phi_,d */
+                    for (int f = 0; f < 4; f++)
+                        for (int a = 0; a < 3; a++) {
+                            double s = 0.0;
+                            for (int d = 0; d < 3; d++)
+                                s = s + m[d][a] * gc[f][d];
+                            gx[f][a] = J * s;
+                        }
+                    double T = pr[3 * cs + p];
+                    double mu = mu_of_T(ph, T);
+                    double kap = mu * cp / ph->Pr;
+                    double div = gx[0][0] + gx[1][1] + gx[2][2];
+                    double tau[3][3], q[3], vel[3];
+                    for (int a = 0; a < 3; a++)
+                        for (int bb = 0; bb < 3; bb++) {
+                            tau[a][bb] = mu * (gx[a][bb] + gx[bb][a]);
+                            if (a == bb)
+                                tau[a][bb] = tau[a][bb] - 2.0 / 3.0 * mu * div;
+                        }
+                    for (int a = 0; a < 3; a++) {
+                        q[a] = -kap * gx[3][a];
+                        vel[a] = pr[a * cs + p];
+                    }
+                    for (int d = 0; d < 3; d++) {
+                        for (int a = 0; a < 3; a++) {
+                            double s = 0.0;
+                            for (int bb = 0; bb < 3; bb++)
+                                s = s + m[d][bb] * tau[a][bb];
+                            Fv[(4 * d + a) * cs + p] = s;
+                        }
+                        double s = 0.0;
+                        for (int bb = 0; bb < 3; bb++) {
+                            double work = 0.0;
+                            for (int a = 0; a < 3; a++)
+                                work = work + vel[a] * tau[a][bb];
+                            s = s + m[d][bb] * (work - q[bb]);
+                        }
+                        Fv[(4 * d + 3) * cs + p] = s;
+                    }
+                }
+#pragma omp parallel for OMP_THREADS
+        for (int64_t k = 0; k < n[2]; k++)
+            for (int64_t j = 0; j < n[1]; j++)
+                for (int64_t i = 0; i < n[0]; i++) {
+                    int64_t p = IX(&b, i, j, k);
+                    for (int q = 0; q < 4; q++)
+                        for (int d = 0; d < 3; d++)
+                            R[(1 + q) * cs + p] = R[(1 + q) * cs + p] + d4(Fv + (4 * d + q) * cs, p, st[d]);
+                }
+        free(Fv);
+        free(pr);
+    }
+
+    /* --- rhs = J * R on interior points --- */
+#pragma omp parallel for OMP_THREADS
+    for (int64_t k = 0; k < n[2]; k++)
+        for (int64_t j = 0; j < n[1]; j++)
+            for (int64_t i = 0; i < n[0]; i++) {
+                int64_t p = IX(&b, i, j, k);
+                for (int c = 0; c < 5; c++)
+                    rhs[c * cs + p] = met[p] * R[c * cs + p];
+            }
+    free(R);
+}
+
+/* ------------------------------------------------------------------ */
+/* 7. Williamson low-storage RK3 stage (PAPER.md:50 ref [10], 106,    */
+/*    114; reading 13):  dU <- A_s dU + dt rhs ;  U_out = U_in + B_s dU */
+/* ------------------------------------------------------------------ */
+static const double RK_A[3] = {0.0, -5.0 / 9.0, -153.0 / 128.0};
+static const double RK_B[3] = {1.0 / 3.0, 15.0 / 16.0, 8.0 / 15.0};
+
+void oracle_rk_update(const int64_t n[3], int32_t stage, double dt, const double *Uin,
+                      double *Uout, double *dU, const double *rhs)
+{
+    obox b = make_box(n, OG);
+    const int64_t cs = b.cs;
+#pragma omp parallel for OMP_THREADS
+    for (int64_t k = 0; k < n[2]; k++)
+        for (int64_t j = 0; j < n[1]; j++)
+            for (int64_t i = 0; i < n[0]; i++) {
+                int64_t p = IX(&b, i, j, k);
+                for (int c = 0; c < 5; c++) {
+                    int64_t q = c * cs + p;
+                    double du;
+                    if (stage == 0)
+                        du = dt * rhs[q];
+                    else
+                        du = RK_A[stage] * dU[q] + dt * rhs[q];
+                    dU[q] = du;
+                    Uout[q] = Uin[q] + RK_B[stage] * du;
+                }
+            }
+}
+
+/* one RK stage = FillPatch/BC_Fill + RHS + Update (Alg. 2 l.3-9) */
+void oracle_rk_stage(const int64_t n[3], const int32_t bc[6], const double dirichlet[30],
+                     const oracle_phys *ph, int32_t stage, double dt, double *Uin, double *Uout,
+                     double *dU, const double *met)
+{
+    obox b = make_box(n, OG);
+    double *rhs = (double *)calloc((size_t)(5 * b.cs), sizeof(double));
+    oracle_fill(n, bc, dirichlet, Uin, 5, O_FIELD_STATE);
+    oracle_rhs(n, ph, Uin, met, rhs);
+    oracle_rk_update(n, stage, dt, Uin, Uout, dU, rhs);
+    free(rhs);
+}
+
+/* nsteps full RK3 steps with a fixed dt (Alg. 1 l.5-10 without Regrid/ComputeDt).
+   U is the state in/out (padded layout); on return its ghosts are filled. */
+void oracle_advance(const int64_t n[3], const int32_t bc[6], const double dirichlet[30],
+                    const oracle_phys *ph, double dt, int32_t nsteps, double *U,
+                    const double *met)
+{
+    obox b = make_box(n, OG);
+    size_t sz = (size_t)(5 * b.cs) * sizeof(double);
+    double *V = (double *)malloc(sz);
+    double *dU = (double *)calloc((size_t)(5 * b.cs), sizeof(double));
+    memcpy(V, U, sz);
+    double *a = U, *o = V;
+    for (int32_t s = 0; s < nsteps; s++)
+        for (int st = 0; st < 3; st++) {
+            oracle_rk_stage(n, bc, dirichlet, ph, st, dt, a, o, dU, met);
+            double *t = a;
+            a = o;
+            o = t;
+        }
+    if (a != U)
+        memcpy(U, a, sz);
+    oracle_fill(n, bc, dirichlet, U, 5, O_FIELD_STATE);
+    free(V);
+    free(dU);
+}

@@ -1,0 +1,327 @@
+"""Seeded synthetic input generators shared by the oracle tests, the GPU
+parity tests and bench.py.
+
+This module holds NONE of the method's arithmetic (no metrics, no fluxes, no
+WENO, no time stepping): it only produces grid coordinates (analytic maps of
+the computational index, evaluated on the padded coordinate band) and
+initial states (closed-form fields converted to conserved variables with the
+perfect-gas equation of state, Eq. 2 single species).  The
+recipes are stated in DESIGN.md section 4 and follow SURVEY.md section 8(d).
+
+Array convention (same as oracle/ and the GPU binding's numpy views):
+shape (ncomp, P2, P1, P0), Pd = n[d] + 2*g, element [c, k+g, j+g, i+g] is
+point (i, j, k) of a block whose first interior point has global index
+``origin``.
+"""
+from __future__ import annotations
+
+import math
+from dataclasses import dataclass, field
+
+import numpy as np
+
+G = 4
+GC = 10
+
+
+# ---------------------------------------------------------------- grids
+
+def _index_grids(n, origin, g):
+    """Global index arrays (float64) for the padded box of a block."""
+    ax = [np.arange(origin[d] - g, origin[d] + n[d] + g, dtype=np.float64) for d in range(3)]
+    K, J, I = np.meshgrid(ax[2], ax[1], ax[0], indexing="ij")
+    return I, J, K
+
+
+@dataclass
+class Cartesian:
+    """x = x0 + (i + 1/2) h  (cell-centred uniform grid, e.g. Sod x_i = (i+1/2)/200)."""
+    h: tuple = (1.0, 1.0, 1.0)
+    x0: tuple = (0.0, 0.0, 0.0)
+    centred: bool = True
+
+    def coords(self, n, origin=(0, 0, 0), g=GC):
+        I, J, K = _index_grids(n, origin, g)
+        off = 0.5 if self.centred else 0.0
+        return np.stack([self.x0[0] + (I + off) * self.h[0],
+                         self.x0[1] + (J + off) * self.h[1],
+                         self.x0[2] + (K + off) * self.h[2]])
+
+
+@dataclass
+class Wavy3D:
+    """Sinusoidally perturbed periodic grid:
+    xi_i = x0 + i L/N,  x = xi + A sin(k eta) sin(k zeta),
+    y = eta + A sin(k zeta) sin(k xi),  z = zeta + A sin(k xi) sin(k eta)."""
+    L: tuple = (10.0, 10.0, 10.0)
+    N: tuple = (64, 64, 64)          # points per length L (global)
+    x0: tuple = (0.0, 0.0, 0.0)
+    k: float = 2 * math.pi * 2 / 10.0
+    A: float = 0.3 / (2 * math.pi * 2 / 10.0)
+
+    def coords(self, n, origin=(0, 0, 0), g=GC):
+        I, J, K = _index_grids(n, origin, g)
+        xi = self.x0[0] + I * self.L[0] / self.N[0]
+        et = self.x0[1] + J * self.L[1] / self.N[1]
+        ze = self.x0[2] + K * self.L[2] / self.N[2]
+        k, A = self.k, self.A
+        return np.stack([xi + A * np.sin(k * et) * np.sin(k * ze),
+                         et + A * np.sin(k * ze) * np.sin(k * xi),
+                         ze + A * np.sin(k * xi) * np.sin(k * et)])
+
+
+@dataclass
+class Wavy2D:
+    """Quasi-2D wavy grid (used for the vortex convergence pin):
+    x = xi + A sin(k eta), y = eta + A sin(k xi), z = zeta."""
+    L: tuple = (10.0, 10.0, 1.0)
+    N: tuple = (32, 32, 4)
+    k: float = 2 * math.pi / 10.0
+    A: float = 0.3 / (2 * math.pi / 10.0)
+
+    def coords(self, n, origin=(0, 0, 0), g=GC):
+        I, J, K = _index_grids(n, origin, g)
+        xi = I * self.L[0] / self.N[0]
+        et = J * self.L[1] / self.N[1]
+        ze = K * self.L[2] / self.N[2]
+        return np.stack([xi + self.A * np.sin(self.k * et),
+                         et + self.A * np.sin(self.k * xi),
+                         ze])
+
+
+@dataclass
+class Ramp:
+    """Compression-ramp grid: x = 4 xi/Nx,
+    wall y_w(x) = tan(24 deg) s ln(1 + exp((x-2)/s)), s = 2 dx,
+    y = y_w(x) + sinh(3 (eta + 1/2)/Ny)/sinh(3), z = zeta/Nz."""
+    N: tuple = (1024, 512, 256)
+    angle_deg: float = 24.0
+
+    def wall(self, x):
+        s = 2.0 * 4.0 / self.N[0]
+        return math.tan(math.radians(self.angle_deg)) * s * np.logaddexp(0.0, (x - 2.0) / s)
+
+    def wall_slope(self, x):
+        s = 2.0 * 4.0 / self.N[0]
+        return math.tan(math.radians(self.angle_deg)) / (1.0 + np.exp(-(x - 2.0) / s))
+
+    def coords(self, n, origin=(0, 0, 0), g=GC):
+        I, J, K = _index_grids(n, origin, g)
+        x = 4.0 * I / self.N[0]
+        y = self.wall(x) + np.sinh(3.0 * (J + 0.5) / self.N[1]) / math.sinh(3.0)
+        z = K / self.N[2]
+        return np.stack([x, y, z])
+
+
+# ---------------------------------------------------------------- states
+
+def prim_to_cons(rho, u, v, w, p, gamma=1.4):
+    """Conserved (rho, rho u, rho v, rho w, E), E = p/(gamma-1) + rho|u|^2/2 (Eq. 2)."""
+    return np.stack([rho, rho * u, rho * v, rho * w,
+                     p / (gamma - 1.0) + 0.5 * rho * (u * u + v * v + w * w)])
+
+
+def interior(a, g=G):
+    return a[:, g:-g, g:-g, g:-g]
+
+
+def pad_state(cons_interior, g=G):
+    nc, n2, n1, n0 = cons_interior.shape
+    out = np.zeros((nc, n2 + 2 * g, n1 + 2 * g, n0 + 2 * g))
+    out[:, g:-g, g:-g, g:-g] = cons_interior
+    return out
+
+
+def _interior_xyz(xyz, gc=GC):
+    return xyz[:, gc:-gc, gc:-gc, gc:-gc]
+
+
+def sod(xyz, gamma=1.4):
+    """Sod (1978): (rho,u,p) = (1,0,1) for x<0.5, (0.125,0,0.1) otherwise."""
+    x = _interior_xyz(xyz)[0]
+    left = x < 0.5
+    rho = np.where(left, 1.0, 0.125)
+    p = np.where(left, 1.0, 0.1)
+    z = np.zeros_like(x)
+    return prim_to_cons(rho, z, z, z, p, gamma)
+
+
+def vortex_prim(x, y, t=0.0, L=10.0, beta=5.0, uinf=(1.0, 1.0), gamma=1.4):
+    """Shu (1998) isentropic vortex centred at (5,5)+t*uinf (periodic images, period L)."""
+    xc = 5.0 + uinf[0] * t
+    yc = 5.0 + uinf[1] * t
+    dx = np.mod(x - xc + L / 2, L) - L / 2
+    dy = np.mod(y - yc + L / 2, L) - L / 2
+    r2 = dx * dx + dy * dy
+    f = np.exp(0.5 * (1.0 - r2))
+    du = -beta / (2 * math.pi) * f * dy
+    dv = beta / (2 * math.pi) * f * dx
+    T = 1.0 - (gamma - 1.0) * beta ** 2 / (8 * gamma * math.pi ** 2) * f * f
+    rho = T ** (1.0 / (gamma - 1.0))
+    p = rho * T
+    return rho, uinf[0] + du, uinf[1] + dv, np.zeros_like(x), p
+
+
+def vortex(xyz, t=0.0, gamma=1.4, **kw):
+    X = _interior_xyz(xyz)
+    rho, u, v, w, p = vortex_prim(X[0], X[1], t=t, gamma=gamma, **kw)
+    return prim_to_cons(rho, u, v, w, p, gamma)
+
+
+def free_stream(xyz, rho=1.0, vel=(0.7, -0.3, 0.4), p=1.0 / 1.4, gamma=1.4):
+    X = _interior_xyz(xyz)
+    o = np.ones_like(X[0])
+    return prim_to_cons(rho * o, vel[0] * o, vel[1] * o, vel[2] * o, p * o, gamma)
+
+
+def tgv(xyz, V0=1.0, rho0=1.0, M0=0.1, gamma=1.4, R=1.0, noise=0.0, seed=5, period=2 * math.pi):
+    """DeBonis (2013) Taylor-Green vortex, T0 = 1/(gamma M0^2) (c0 = 1/M0 for V0 = 1)."""
+    X = _interior_xyz(xyz)
+    s = 2 * math.pi / period
+    x, y, z = X[0] * s, X[1] * s, X[2] * s
+    T0 = V0 ** 2 / (gamma * R * M0 ** 2)
+    p0 = rho0 * R * T0
+    u = V0 * np.sin(x) * np.cos(y) * np.cos(z)
+    v = -V0 * np.cos(x) * np.sin(y) * np.cos(z)
+    w = np.zeros_like(x)
+    p = p0 + rho0 * V0 ** 2 / 16.0 * (np.cos(2 * x) + np.cos(2 * y)) * (np.cos(2 * z) + 2.0)
+    if noise:
+        u = u + noise * V0 * smooth_noise(x, y, z, seed, 0)
+        v = v + noise * V0 * smooth_noise(x, y, z, seed, 1)
+        w = w + noise * V0 * smooth_noise(x, y, z, seed, 2)
+    rho = p / (R * T0)
+    return prim_to_cons(rho, u, v, w, p, gamma)
+
+
+def smooth_noise(x, y, z, seed, comp, modes=4):
+    """Sum of a few 2pi-periodic Fourier modes with seeded random amplitudes/phases, |.| <= 1."""
+    rng = np.random.default_rng([seed, comp])
+    out = np.zeros_like(x)
+    tot = 0.0
+    for _ in range(modes):
+        kx, ky, kz = rng.integers(1, 4, size=3)
+        a = rng.uniform(0.5, 1.0)
+        ph = rng.uniform(0, 2 * math.pi, size=3)
+        out += a * np.sin(kx * x + ph[0]) * np.sin(ky * y + ph[1]) * np.sin(kz * z + ph[2])
+        tot += a
+    return out / tot
+
+
+def shear_wave(xyz, a=0.1, m=1, Lx=1.0, gamma=1.4):
+    """rho = 1, p = 1, u = w = 0, v = a sin(k x), k = 2 pi m / Lx (viscous closed-form pin)."""
+    X = _interior_xyz(xyz)
+    k = 2 * math.pi * m / Lx
+    o = np.ones_like(X[0])
+    z = np.zeros_like(X[0])
+    return prim_to_cons(o, z, a * np.sin(k * X[0]), z, o, gamma)
+
+
+def ramp_state(xyz, grid: Ramp, mach=6.0, delta=0.1, Tw=4.0, gamma=1.4, R=1.0, noise=0.01, seed=4):
+    """Mach-6 free stream + tanh boundary layer, Crocco-Busemann T."""
+    X = _interior_xyz(xyz)
+    x, y, z = X[0], X[1], X[2]
+    Uinf = mach * math.sqrt(gamma * R * 1.0)
+    d = np.maximum(y - grid.wall(x), 0.0)
+    ur = np.tanh(3.0 * d / delta)
+    T = Tw + (1.0 - Tw) * ur + 0.5 * (gamma - 1.0) * mach ** 2 * ur * (1.0 - ur)
+    ang = np.arctan(grid.wall_slope(x))
+    s = 2 * math.pi
+    pert = noise * smooth_noise(x * s / 4.0, y * s, z * s, seed, 0)
+    u = Uinf * ur * np.cos(ang) * (1.0 + pert)
+    v = Uinf * ur * np.sin(ang) * (1.0 + pert)
+    w = Uinf * 0.1 * noise * smooth_noise(x * s / 4.0, y * s, z * s, seed, 1) * ur
+    p = np.ones_like(x) * 1.0 * R * 1.0
+    rho = p / (R * T)
+    return prim_to_cons(rho, u, v, w, p, gamma)
+
+
+def random_state(n, seed=0, amp=0.3, gamma=1.4, mach=0.8):
+    """Random positive state: smooth base + uniform noise (parity inputs, not physics)."""
+    rng = np.random.default_rng(seed)
+    shape = (n[2], n[1], n[0])
+    rho = 1.0 + amp * rng.uniform(-1, 1, shape)
+    p = 1.0 / gamma * (1.0 + amp * rng.uniform(-1, 1, shape))
+    u = mach * rng.uniform(-1, 1, shape)
+    v = mach * rng.uniform(-1, 1, shape)
+    w = mach * rng.uniform(-1, 1, shape)
+    return prim_to_cons(rho, u, v, w, p, gamma)
+
+
+def random_coords_jitter(xyz, seed=0, amp=0.02):
+    """Small smooth perturbation of a grid (keeps it valid) for parity inputs."""
+    rng = np.random.default_rng(seed)
+    out = xyz.copy()
+    _, P2, P1, P0 = xyz.shape
+    I, J, K = np.meshgrid(np.arange(P2), np.arange(P1), np.arange(P0), indexing="ij")
+    for a in range(3):
+        ph = rng.uniform(0, 2 * math.pi, 3)
+        out[a] += amp * np.sin(0.37 * K + ph[0]) * np.sin(0.29 * J + ph[1]) * np.sin(0.23 * I + ph[2])
+    return out
+
+
+# ---------------------------------------------------------------- configs
+
+@dataclass
+class Case:
+    """One BASELINE.json configuration as concrete synthetic input."""
+    name: str
+    n_global: tuple
+    n_blocks: tuple
+    bc: tuple                 # ((xi_lo, xi_hi), (eta_lo, eta_hi), (zeta_lo, zeta_hi))
+    grid: object
+    state: str
+    phys: dict = field(default_factory=dict)
+    dt: float = 1e-3
+    steps: int = 100
+
+
+P, E, D, W = 0, 1, 2, 3
+
+
+def case(name: str, scale: int = 1) -> Case:
+    """Configs of BASELINE.json; ``scale`` divides the grid for parity runs."""
+    if name == "sod":
+        return Case("sod", (200, 4, 4), (1, 1, 1), ((E, E), (P, P), (P, P)),
+                    Cartesian(h=(1 / 200,) * 3), "sod",
+                    dict(gamma=1.4, R=1.0, terms=1), dt=1e-3, steps=100)
+    if name == "vortex":
+        N = 64 // scale
+        return Case("vortex", (N, N, N), (1, 1, 1), ((P, P),) * 3,
+                    Wavy3D(L=(10.0,) * 3, N=(N, N, N)), "vortex",
+                    dict(gamma=1.4, R=1.0, terms=1), dt=0.01 * scale, steps=100)
+    if name == "tgv":
+        N = 256 // scale
+        return Case("tgv", (N, N, N), (1, 1, 1), ((P, P),) * 3,
+                    Wavy3D(L=(2 * math.pi,) * 3, N=(N, N, N), x0=(-math.pi,) * 3, k=2.0, A=0.3 / 2.0),
+                    "tgv", dict(gamma=1.4, R=1.0, Pr=0.71, mu_ref=1.0 / 1600.0),
+                    dt=4e-4 * scale, steps=100)
+    if name == "ramp":
+        N = (1024 // scale, 512 // scale, 256 // scale)
+        return Case("ramp", N, (2, 2, 2), ((E, E), (W, E), (P, P)), Ramp(N=N), "ramp",
+                    dict(gamma=1.4, R=1.0, Pr=0.72, mu_law=1, mu_ref=1e-4, T_ref=1.0, S=0.3),
+                    dt=2e-5 * scale, steps=100)
+    if name == "weak":
+        N = 512 // scale
+        return Case("weak", (N, N, N), (1, 1, 1), ((P, P),) * 3,
+                    Wavy3D(L=(2 * math.pi,) * 3, N=(N, N, N), x0=(-math.pi,) * 3, k=2.0, A=0.3 / 2.0),
+                    "tgv_noise", dict(gamma=1.4, R=1.0, Pr=0.71, mu_ref=1.0 / 1600.0),
+                    dt=2e-4 * scale, steps=100)
+    raise KeyError(name)
+
+
+def block_inputs(c: Case, origin, n, gamma=1.4):
+    """(xyz on the padded coordinate band, conserved interior state) for one block."""
+    xyz = c.grid.coords(n, origin, GC)
+    if c.state == "sod":
+        U = sod(xyz, gamma)
+    elif c.state == "vortex":
+        U = vortex(xyz, gamma=gamma)
+    elif c.state == "tgv":
+        U = tgv(xyz, gamma=gamma)
+    elif c.state == "tgv_noise":
+        U = tgv(xyz, gamma=gamma, noise=0.01, seed=5)
+    elif c.state == "ramp":
+        U = ramp_state(xyz, c.grid, gamma=gamma)
+    else:
+        raise KeyError(c.state)
+    return xyz, U
