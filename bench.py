@@ -1,0 +1,362 @@
+#!/usr/bin/env python
+"""bench.py -- grid-point RK-stage updates/sec (fp64) of the CRoCCo v2.0 hot path
+on 1..8 B200 (BASELINE.json metric), one process per GPU.
+
+Workload (BASELINE.json configs[4], the north_star's 512^3 target): weak
+scaling, 512^3 interior points per GPU of a sinusoidally perturbed periodic
+curvilinear grid holding a Taylor-Green vortex + 1% smooth noise, viscous
+(mu = 1/1600, Pr = 0.71), fixed dt.  N GPUs hold a (512a)x(512b)x(512c)
+global grid, one block per rank, ghost exchange over NCCL.  A step is one
+full RK3 time step = 3 x (FillPatch + BC_Fill + WENOx/y/z + Viscous + Update)
+(Algorithm 2); value = interior points x 3 x steps / time.
+
+  python bench.py [--gpus N --steps K --warmup W]        # CUDA path (default)
+  python bench.py --impl reference ...                   # CPU oracle arm (rank 0)
+torchrun launches one rank per GPU for N > 1.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import math
+import os
+import statistics
+import subprocess
+import sys
+import tempfile
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+METRIC = "grid-point RK-stage updates/sec (fp64) at 1/2/4/8 B200; % HBM roofline"
+UNIT = "point-stages/s"
+N_BLOCK = 512
+# FP64 operations of one characteristic-WENO interface flux:
+# DADD + DMUL + 2*DFMA counted by ncu on k_flux (profiles/), per interface.
+FLUX_FLOPS_PER_IFACE = float(os.environ.get("CROCCO_FLUX_FLOPS", "2478"))
+# B200 FP64 (non-tensor) peak: 148 SMs x 64 FMA/clk x 2 flop x 1.965 GHz
+FP64_PEAK_TFLOPS = 148 * 64 * 2 * 1.965e9 / 1e12
+# compulsory HBM bytes per point-stage of a fused stage: 240 (200 at stage 0)
+HBM_BYTES_PER_PT_STAGE = (200 + 240 + 240) / 3.0
+
+
+def weak_grid(n):
+    return {1: (1, 1, 1), 2: (2, 1, 1), 4: (2, 2, 1), 8: (2, 2, 2)}.get(n) or _factor3(n)
+
+
+def _factor3(n):
+    f = [1, 1, 1]
+    k = 0
+    m = n
+    p = 2
+    while m > 1:
+        while m % p == 0:
+            f[k % 3] *= p
+            k += 1
+            m //= p
+        p += 1
+    return tuple(f)
+
+
+def measured_peaks():
+    try:
+        with open(os.path.join(ROOT, "MEASURED_PEAKS.json")) as f:
+            return json.load(f)
+    except Exception:
+        return {}
+
+
+# ------------------------------------------------------------------ clocks
+class ClockSampler:
+    """nvidia-smi clocks + throttle reasons sampled during the timed region."""
+
+    def __init__(self, gpu_index):
+        self.f = tempfile.NamedTemporaryFile("w+", suffix=".csv", delete=False)
+        q = ("clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.hw_slowdown,"
+             "clocks_event_reasons.hw_thermal_slowdown,clocks_event_reasons.sw_thermal_slowdown,"
+             "clocks_event_reasons.sw_power_cap")
+        try:
+            self.p = subprocess.Popen(["nvidia-smi", "-i", str(gpu_index), f"--query-gpu={q}",
+                                       "--format=csv,noheader,nounits", "-lms", "200"],
+                                      stdout=self.f, stderr=subprocess.DEVNULL)
+        except Exception:
+            self.p = None
+
+    def stop(self):
+        if self.p is None:
+            return None
+        self.p.terminate()
+        try:
+            self.p.wait(timeout=5)
+        except Exception:
+            self.p.kill()
+        self.f.flush()
+        rows = []
+        with open(self.f.name) as fh:
+            for line in fh:
+                parts = [x.strip() for x in line.split(",")]
+                if len(parts) < 7:
+                    continue
+                try:
+                    rows.append((float(parts[0]), float(parts[1]), parts[3:7]))
+                except ValueError:
+                    pass
+        os.unlink(self.f.name)
+        if not rows:
+            return None
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        reasons = sorted({names[i] for _, _, r in rows for i, v in enumerate(r) if v.lower() == "active"})
+        return {"sm_mhz": statistics.median(r[0] for r in rows), "sm_max_mhz": max(r[1] for r in rows),
+                "reasons": reasons, "samples": len(rows)}
+
+
+# ------------------------------------------------------------------ oracle (CPU baseline)
+def oracle_rate(max_seconds=12.0, n=64, max_steps=100, steps=None, warmup=0):
+    """Time the CPU oracle (as it stands) on a bounded sample of the workload:
+    an n^3 periodic wavy-grid TGV+noise box, whole RK3 steps, all host cores."""
+    import numpy as np
+
+    import oracle
+    import synth
+    oracle.build()
+    cores = os.cpu_count() or 1
+    oracle.set_threads(cores)
+    nn = (n, n, n)
+    grid = synth.Wavy3D(L=(2 * math.pi,) * 3, N=nn, x0=(-math.pi,) * 3, k=2.0, A=0.15)
+    xyz = grid.coords(nn, (0, 0, 0), oracle.GC)
+    met = oracle.metrics(nn, ((0, 0),) * 3, xyz)
+    U = synth.pad_state(synth.tgv(xyz, noise=0.01, seed=5))
+    ph = oracle.phys(gamma=1.4, R=1.0, Pr=0.71, mu_ref=1 / 1600, terms=3)
+    bc = ((0, 0),) * 3
+    for _ in range(warmup):
+        oracle.advance(nn, bc, ph, 2e-3, 1, U, met)
+    done = 0
+    t0 = time.perf_counter()
+    per_step = []
+    while True:
+        ts = time.perf_counter()
+        oracle.advance(nn, bc, ph, 2e-3, 1, U, met)
+        per_step.append(time.perf_counter() - ts)
+        done += 1
+        el = time.perf_counter() - t0
+        if steps is not None:
+            if done >= steps:
+                break
+        elif el >= max_seconds or done >= max_steps:
+            break
+    el = time.perf_counter() - t0
+    pts = n ** 3 * 3 * done
+    return {"value": pts / el, "unit": UNIT, "cores": oracle.get_threads(), "kind": "oracle",
+            "sample": f"{done} RK3 step(s) (3 stages each) of a {n}^3 periodic wavy-grid TGV+noise box "
+                      f"(same discretisation and per-point work as the {N_BLOCK}^3 workload), "
+                      f"{el:.2f} s wall", "seconds": el, "steps": done, "per_step_s": per_step}
+
+
+# ------------------------------------------------------------------ reference arm
+def run_reference(args, rank, world):
+    if rank != 0:
+        return 0
+    r = oracle_rate(steps=args.steps, warmup=args.warmup, n=args.ref_n)
+    ms = 1e3 * r["seconds"] / r["steps"]
+    out = {"impl": "reference", "metric": METRIC, "value": r["value"], "unit": UNIT,
+           "n_gpus": args.gpus, "steps": args.steps, "warmup": args.warmup, "ms_per_step": ms,
+           "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "f64",
+           "data": "synthetic",
+           "config": {"workload": f"weak: {N_BLOCK}^3/GPU periodic curvilinear TGV+noise, viscous; "
+                                  f"reference arm times a bounded {args.ref_n}^3 sample per step",
+                      "sample_points": args.ref_n ** 3},
+           "cpu_baseline": {k: r[k] for k in ("value", "unit", "cores", "kind", "sample")},
+           "e2e": {"value": r["value"], "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+    print(json.dumps(out), flush=True)
+    return 0
+
+
+# ------------------------------------------------------------------ CUDA arm
+def run_crocco(args, rank, world, local_rank):
+    import numpy as np
+    import torch
+    import torch.distributed as dist
+
+    import synth
+    from paper_conf_ipps_davissngmb23_b200 import crocco as cc
+    from paper_conf_ipps_davissngmb23_b200.solver import Solver
+
+    torch.cuda.set_device(local_rank)
+    dev = torch.device("cuda", local_rank)
+    a, b, c = weak_grid(world)
+    nb = (a, b, c)
+    n = (N_BLOCK * a, N_BLOCK * b, N_BLOCK * c)
+    uid = None
+    if world > 1:
+        t = torch.zeros(128, dtype=torch.uint8, device=dev)
+        if rank == 0:
+            t.copy_(torch.frombuffer(bytearray(cc.crocco_nccl_unique_id()), dtype=torch.uint8))
+        dist.broadcast(t, 0)
+        uid = bytes(t.cpu().numpy().tobytes())
+    grid = synth.Wavy3D(L=(2 * math.pi * a, 2 * math.pi * b, 2 * math.pi * c), N=n,
+                        x0=(-math.pi,) * 3, k=2.0, A=0.15)
+    phys = dict(gamma=1.4, R=1.0, Pr=0.71, mu_ref=1.0 / 1600.0, terms=3)
+    dt = 2e-4
+    S = Solver(n, nb, ((0, 0),) * 3, cc.make_phys(**phys), rank=rank, nranks=world,
+               block_rank=list(range(world)), device=dev, nccl_unique_id=uid)
+    L = S.layouts[0]
+    origin = tuple(L.origin)
+    bn = tuple(L.n)
+    xyz = torch.from_numpy(grid.coords(bn, origin, cc.GHOST_COORDS)).to(dev)
+    S.set_coords([xyz])
+    U0 = synth.tgv(xyz, noise=0.01, seed=5)
+    del xyz
+    S.set_state([U0])
+    del U0
+    torch.cuda.synchronize()
+    stream = S.stream
+    pts_local = bn[0] * bn[1] * bn[2]
+    pts_total = n[0] * n[1] * n[2]
+
+    for _ in range(args.warmup):
+        S.step(dt)
+    torch.cuda.synchronize()
+
+    # ---------------- timed region (device-resident inputs)
+    cc.crocco_set_timing(S.ctx, True)
+    cc.crocco_kernel_times(S.ctx)          # reset accumulators
+    cc.crocco_launch_count(S.ctx, reset=True)
+    clk = ClockSampler(local_rank) if not args.no_clocks else None
+    e0 = torch.cuda.Event(enable_timing=True)
+    e1 = torch.cuda.Event(enable_timing=True)
+    if world > 1:
+        dist.barrier()
+    torch.cuda.synchronize()
+    e0.record(stream)
+    for _ in range(args.steps):
+        S.step(dt)
+    e1.record(stream)
+    torch.cuda.synchronize()
+    if world > 1:
+        dist.barrier()
+    ms_local = e0.elapsed_time(e1)
+    clocks = clk.stop() if clk else None
+    launches = cc.crocco_launch_count(S.ctx)
+    ktimes = cc.crocco_kernel_times(S.ctx)
+    cc.crocco_set_timing(S.ctx, False)
+    t = torch.tensor([ms_local], dtype=torch.float64, device=dev)
+    if world > 1:
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+    ms = float(t.item())
+    value = pts_total * 3 * args.steps / (ms / 1e3)
+    # state sanity (finite, positive density) -- not part of the timed region
+    Ui = S.view(S.U[0], 0, 5)[:, 4:-4, 4:-4, 4:-4]
+    finite = bool(torch.isfinite(Ui).all().item()) and float(Ui[0].min().item()) > 0
+
+    # ---------------- end-to-end through the public API with host buffers
+    e2e = None
+    if args.e2e_steps > 0:
+        host = torch.empty(S.U[0].numel(), dtype=torch.float64, pin_memory=True)
+        host.copy_(S.U[0])
+        torch.cuda.synchronize()
+        if world > 1:
+            dist.barrier()
+        f0 = torch.cuda.Event(enable_timing=True)
+        f1 = torch.cuda.Event(enable_timing=True)
+        f0.record(stream)
+        for _ in range(args.e2e_steps):
+            S.U[0].copy_(host, non_blocking=True)      # H2D of the step's input state
+            S.step(dt)
+            host.copy_(S.U[0], non_blocking=True)      # D2H of the step's result
+        f1.record(stream)
+        torch.cuda.synchronize()
+        te = torch.tensor([f0.elapsed_time(f1)], dtype=torch.float64, device=dev)
+        if world > 1:
+            dist.all_reduce(te, op=dist.ReduceOp.MAX)
+        nbytes = host.numel() * 8
+        e2e = {"value": pts_total * 3 * args.e2e_steps / (float(te.item()) / 1e3), "unit": UNIT,
+               "h2d_bytes_per_step": nbytes * world, "d2h_bytes_per_step": nbytes * world,
+               "steps": args.e2e_steps}
+
+    # ---------------- roofline of the dominant kernel (CUDA events on the launching stream)
+    flux_cls = {"flux_xi": 0, "flux_eta": 1, "flux_zeta": 2}
+    dom = max(ktimes.items(), key=lambda kv: kv[1][1])
+    name, (nl, kms) = dom
+    avg_ms = kms / max(nl, 1)
+    roof = None
+    if name in flux_cls:
+        d = flux_cls[name]
+        ifaces = (bn[d] + 1) * pts_local // bn[d]
+        ach = FLUX_FLOPS_PER_IFACE * ifaces / (avg_ms / 1e3) / 1e12
+        roof = {"bound": "alu", "kernel": f"k_flux<{d}> ({name})", "achieved": ach,
+                "peak": FP64_PEAK_TFLOPS, "unit": "TFLOP/s", "frac": ach / FP64_PEAK_TFLOPS,
+                "peak_source": "derived: 148 SM x 64 FP64 FMA/clk x 2 x 1.965 GHz (DESIGN.md sec. 6)",
+                "flops_per_unit": FLUX_FLOPS_PER_IFACE, "unit_of_work": "interface flux",
+                "units_per_launch": ifaces, "avg_launch_ms": avg_ms,
+                "traffic": _profiled_traffic(name)}
+    peaks = measured_peaks()
+    hbm = peaks.get("hbm_gbs", 6650.0)
+    stage_gbs = value / world * HBM_BYTES_PER_PT_STAGE / 1e9
+    breakdown = {k: {"launches": v[0], "ms": v[1], "share": v[1] / max(ms_local, 1e-9)}
+                 for k, v in ktimes.items() if v[0]}
+    out = {"metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
+           "warmup": args.warmup, "ms_per_step": ms / args.steps, "higher_is_better": True,
+           "scaling": "weak", "vs_baseline": None, "dtype": "f64",
+           "data": "synthetic (seeded wavy periodic grid, TGV + 1% smooth noise)",
+           "config": {"workload": f"weak: {N_BLOCK}^3/GPU periodic curvilinear TGV+noise, viscous "
+                                  f"(BASELINE.json configs[4]); step = 1 RK3 step (3 stages)",
+                      "n_global": list(n), "n_blocks": list(nb), "points_per_gpu": pts_local,
+                      "dt": dt, "l2": "inputs larger than L2 (5.9 GB state per GPU vs 126 MB L2)",
+                      "parallelism": f"spatial blocks {a}x{b}x{c}, NCCL halo exchange"},
+           "roofline": roof,
+           "hbm": {"algorithmic_gbs_per_gpu": stage_gbs, "peak_gbs": hbm,
+                   "frac": stage_gbs / hbm, "bytes_per_point_stage": HBM_BYTES_PER_PT_STAGE,
+                   "note": "whole-stage compulsory traffic; the path is FP64-pipe bound"},
+           "kernel_breakdown": breakdown,
+           "gpu_launches": launches, "clocks": clocks, "e2e": e2e, "state_finite": finite}
+    if rank == 0 and world == 1 and not args.no_cpu_baseline:
+        r = oracle_rate()
+        out["cpu_baseline"] = {k: r[k] for k in ("value", "unit", "cores", "kind", "sample")}
+    S.close()
+    if rank == 0:
+        print(json.dumps(out), flush=True)
+    return 0
+
+
+def _profiled_traffic(kname):
+    """dram bytes per launch of the dominant kernel from the committed ncu summary, if any."""
+    p = os.path.join(ROOT, "profiles", "ncu_summary.json")
+    try:
+        with open(p) as f:
+            return json.load(f).get("kernels", {}).get(kname, {}).get("dram_bytes_per_launch")
+    except Exception:
+        return None
+
+
+def main():
+    ap = argparse.ArgumentParser(description=__doc__, formatter_class=argparse.RawDescriptionHelpFormatter)
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=5)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--impl", choices=["crocco", "reference"], default="crocco")
+    ap.add_argument("--e2e-steps", type=int, default=2)
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--no-clocks", action="store_true")
+    ap.add_argument("--ref-n", type=int, default=48)
+    args = ap.parse_args()
+    rank = int(os.environ.get("RANK", "0"))
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    local_rank = int(os.environ.get("LOCAL_RANK", "0"))
+    if args.impl == "reference":
+        return run_reference(args, rank, world)
+    if world > 1:
+        import torch
+        import torch.distributed as dist
+        torch.cuda.set_device(local_rank)
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local_rank))
+    try:
+        return run_crocco(args, rank, world, local_rank)
+    finally:
+        if world > 1:
+            import torch.distributed as dist
+            dist.destroy_process_group()
+
+
+if __name__ == "__main__":
+    sys.exit(main())

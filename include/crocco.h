@@ -1,0 +1,207 @@
+/*
+ * crocco.h -- C ABI of libcrocco.so, the B200 (sm_100a) implementation of the
+ * data-parallel hot path of CRoCCo v2.0 (Davis et al., IPDPS 2023).
+ *
+ * Citations "PAPER.md:N" are lines of the paper text;
+ * "reading N" refers to the readings table in DESIGN.md section 3, which fixes
+ * everything the paper leaves unstated (scheme constants, eigenvectors, BCs ...).
+ *
+ * Call order follows Algorithm 1/2:
+ *   crocco_init_grid      (InitGrid, Alg. 1 l.1)
+ *   crocco_init_metrics   (InitGridMetrics, Alg. 1 l.2; coordinates held in memory)
+ *   per RK stage: crocco_rk_stage = FillPatch + BC_Fill + WENOx/y/z + Viscous + Update
+ *                 (Alg. 2 l.3-9), or the unfused crocco_fill_boundary / crocco_rhs /
+ *                 crocco_rk_update used by the tests.
+ *
+ * Conventions
+ *  - Every entry point returns crocco_status; CROCCO_OK == 0.  No C++ exception
+ *    crosses the ABI.  Text for the last error: crocco_last_error(ctx) (or
+ *    crocco_last_error(NULL) for failures before a ctx exists).
+ *  - All field arrays are fp64, structure-of-arrays, CALLER-OWNED DEVICE memory,
+ *    one pointer per LOCAL block (array of crocco_num_local_blocks pointers).
+ *    Layout of every state/metric/rhs array of local block b: see
+ *    crocco_block_layout; point (i,j,k) (interior 0 <= i < n[0] ..., ghosts down to
+ *    -ghost) of component c is element
+ *        c*comp_stride + offset + i + j*pitch_y + k*pitch_z.
+ *    Coordinates use the same formula with coffset/cpitch_y/cpitch_z/ccomp_stride
+ *    and ghost width ghost_coords (=10).  Allocate ncomp*comp_stride doubles
+ *    (5 for U/dU/rhs, 10 for metrics, 3*ccomp_stride for xyz).  The library
+ *    never frees or retains caller pointers beyond a call.
+ *  - The library owns: the ctx, its device scratch (interface-flux buffers,
+ *    primitive and viscous-flux buffers, halo staging; sized at init_grid and
+ *    reported by crocco_scratch_bytes), the internal comm stream/events, and
+ *    the NCCL communicator when nranks > 1.  All freed by crocco_finalize.
+ *  - Execution: every call is asynchronous on desc.stream (a cudaStream_t);
+ *    asynchronous device faults surface at crocco_sync.  After any CUDA/NCCL
+ *    error the ctx is poisoned and later calls return CROCCO_ERR_STATE.
+ *  - Collectives: init_grid, init_metrics, fill_boundary, rhs (does not
+ *    communicate, but keep order) and rk_stage must be called by all ranks in
+ *    the same order when nranks > 1.
+ *  - Threading: not thread-safe; one ctx per process/GPU.
+ */
+#ifndef CROCCO_H
+#define CROCCO_H
+
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef enum {
+    CROCCO_OK = 0,
+    CROCCO_ERR_ARG = 1,   /* invalid argument / shape (synchronous, nothing launched) */
+    CROCCO_ERR_CUDA = 2,  /* CUDA launch/runtime failure */
+    CROCCO_ERR_NCCL = 3,  /* NCCL failure */
+    CROCCO_ERR_NOMEM = 4, /* device scratch allocation failed */
+    CROCCO_ERR_STATE = 5  /* ctx poisoned by an earlier CUDA/NCCL error */
+} crocco_status;
+
+typedef struct crocco_ctx_s *crocco_ctx;
+
+/* Boundary kinds per face (PAPER.md:83 BC_Fill; reading 15). */
+enum {
+    CROCCO_BC_PERIODIC = 0,  /* copy from the periodic partner; lo/hi must both be PERIODIC */
+    CROCCO_BC_EXTRAP = 1,    /* zeroth-order extrapolation: ghost = nearest interior layer */
+    CROCCO_BC_DIRICHLET = 2, /* ghost = constant conserved state dirichlet[d][side][0..4] */
+    CROCCO_BC_WALL = 3       /* no-slip adiabatic wall, mirror about the face at index -1/2 (n-1/2):
+                                (rho, -rho u, -rho v, -rho w, E) of the mirrored interior point */
+};
+enum { CROCCO_TERM_INVISCID = 1, CROCCO_TERM_VISCOUS = 2 }; /* bitmask (Alg. 2 l.5-7 / l.8) */
+enum { CROCCO_MU_CONST = 0, CROCCO_MU_SUTHERLAND = 1 };
+enum { CROCCO_FIELD_STATE = 0, CROCCO_FIELD_METRIC = 1 };
+enum { CROCCO_GHOST = 4, CROCCO_GHOST_COORDS = 10 }; /* reading 7 */
+
+typedef struct {
+    int64_t n_global[3];        /* interior points N_xi, N_eta, N_zeta of the whole domain */
+    int32_t n_blocks[3];        /* equal boxes per direction; n_global[d] % n_blocks[d] == 0,
+                                   block interior >= 4 points per direction */
+    int32_t bc[3][2];           /* per direction d, side lo(0)/hi(1): CROCCO_BC_* */
+    double dirichlet[3][2][5];  /* conserved ghost state for DIRICHLET faces */
+    int32_t rank, nranks;       /* this process / world size */
+    const int32_t *block_rank;  /* owner rank of global block b = bx + nbx*(by + nby*bz);
+                                   NULL = all blocks on rank 0 (requires nranks == 1) */
+    void *stream;               /* cudaStream_t the library enqueues on (NULL = legacy default) */
+    const void *nccl_unique_id; /* 128-byte ncclUniqueId broadcast by the caller (torch.distributed);
+                                   ignored when nranks == 1 */
+} crocco_grid_desc;
+
+typedef struct {
+    double gamma, R, Pr;   /* calorically perfect gas p = rho R T, c_v = R/(gamma-1), c_p = gamma c_v */
+    int32_t mu_law;        /* CROCCO_MU_CONST: mu = mu_ref;
+                              CROCCO_MU_SUTHERLAND: mu = mu_ref (T/T_ref)^{3/2} (T_ref+S)/(T+S) */
+    double mu_ref, T_ref, S;
+    double weno_eps;       /* WENO-SYMBO epsilon in alpha_k = C_k/(eps+beta_k)^2 (reading 8), 1e-6 */
+    int32_t terms;         /* CROCCO_TERM_* bitmask */
+    int32_t dir_mask;      /* inviscid directions evaluated, bit d = direction d (tests; 7 = all) */
+} crocco_phys;
+
+typedef struct {
+    int32_t n[3];          /* interior points of this block */
+    int64_t origin[3];     /* global index of its interior point (0,0,0) */
+    int32_t ghost;         /* 4 */
+    int32_t ghost_coords;  /* 10 */
+    int64_t offset;        /* element offset of interior point (0,0,0) inside one component */
+    int64_t pitch_y, pitch_z, comp_stride;     /* elements; state / metric / rhs arrays */
+    int64_t coffset, cpitch_y, cpitch_z, ccomp_stride; /* elements; coordinate arrays */
+    int32_t global_id;     /* global block id b */
+} crocco_block_layout;
+
+/* One exchange message of the ghost fill (host-side plan, exposed for tests). */
+typedef struct {
+    int32_t phase;          /* direction d of the fill phase (0, 1, 2) */
+    int32_t dst_block;      /* global id of the block whose ghosts are written */
+    int32_t side;           /* 0 = lo face, 1 = hi face of dst_block */
+    int32_t kind;           /* 0 = copy from src_block, 1 = physical BC (bc value in bc_kind) */
+    int32_t bc_kind;        /* CROCCO_BC_* of the face */
+    int32_t src_block;      /* global id of the source block (copy), -1 for physical */
+    int32_t src_rank, dst_rank;
+    int64_t dst_lo[3];      /* box of ghost points written, block-local indices, [lo, lo+ext) */
+    int64_t src_lo[3];      /* box of source points read, src-block-local indices */
+    int64_t ext[3];
+} crocco_msg;
+
+/* ---- setup --------------------------------------------------------------- */
+
+/* Validate the decomposition, build neighbour tables and the exchange plan,
+   allocate device scratch for the local blocks on the current CUDA device,
+   create the NCCL communicator if nranks > 1.  Collective. */
+crocco_status crocco_init_grid(const crocco_grid_desc *desc, const crocco_phys *phys,
+                               crocco_ctx *out);
+crocco_status crocco_num_local_blocks(crocco_ctx ctx, int32_t *n_local);
+crocco_status crocco_get_block_layout(crocco_ctx ctx, int32_t local_block,
+                                      crocco_block_layout *out);
+crocco_status crocco_set_phys(crocco_ctx ctx, const crocco_phys *phys);
+crocco_status crocco_scratch_bytes(crocco_ctx ctx, int64_t *bytes);
+
+/* InitGridMetrics (readings 5-6): from the coordinates
+   xyz (3 comps, interior +-10 filled by the caller) compute
+   metrics (10 comps: 0 = J = 1/det(d x/d xi), 1+3d+a = m^d_a = (d xi_d/d x_a)/J,
+   Thomas-Lombard form with the 6th-order central operator D6) on the whole
+   padded box (interior +-4), then copy the periodic / inter-block ghost metrics
+   from their owners (crocco_fill_boundary(METRIC)).  Collective. */
+crocco_status crocco_init_metrics(crocco_ctx ctx, double *const *xyz, double *const *metrics);
+
+/* FillPatch + BC_Fill: in place on 4 ghost layers,
+   phases xi -> eta (spanning xi ghosts) -> zeta (spanning xi, eta ghosts).
+   kind STATE: 5 comps, copies + physical BCs.  kind METRIC: 10 comps,
+   periodic / inter-block copies only.  Collective. */
+crocco_status crocco_fill_boundary(crocco_ctx ctx, double *const *field, int32_t kind);
+
+/* RHS: rhs = J ( -sum_d delta_d F^_inv^d + sum_d D4_d F^_v^d )
+   on interior points (ghosts of rhs untouched).  U must have its ghosts filled;
+   metrics from crocco_init_metrics.  rhs may not alias U. */
+crocco_status crocco_rhs(crocco_ctx ctx, double *const *U, double *const *metrics,
+                         double *const *rhs);
+
+/* One Williamson low-storage RK3 stage (reading 13):
+   fill(U_in) (in place on U_in's ghosts) + RHS + dU <- A_s dU + dt rhs,
+   U_out = U_in + B_s dU on interior points; A = (0, -5/9, -153/128),
+   B = (1/3, 15/16, 8/15).  dU is not read at stage 0.  U_out != U_in.
+   Collective. */
+crocco_status crocco_rk_stage(crocco_ctx ctx, int32_t stage, double dt, double *const *U_in,
+                              double *const *U_out, double *const *dU,
+                              double *const *metrics);
+
+/* The Update step alone (tests): dU <- A_s dU + dt rhs ; U_out = U_in + B_s dU. */
+crocco_status crocco_rk_update(crocco_ctx ctx, int32_t stage, double dt, double *const *U_in,
+                               double *const *U_out, double *const *dU, double *const *rhs);
+
+/* Block until all work of the ctx finished; surfaces asynchronous errors. */
+crocco_status crocco_sync(crocco_ctx ctx);
+const char *crocco_last_error(crocco_ctx ctx);
+crocco_status crocco_finalize(crocco_ctx ctx);
+
+/* ---- instrumentation (bench / tests) ---------------------------------------- */
+
+/* Number of kernels this ctx launched since init (or the last reset). */
+crocco_status crocco_launch_count(crocco_ctx ctx, int64_t *count, int32_t reset);
+/* Kernel-class timing with CUDA events recorded on the launching stream.
+   When enabled, every launch of class k is bracketed by events; crocco_kernel_times
+   returns, per class, the number of launches and the summed milliseconds
+   (synchronises).  Classes: see crocco_kernel_class_name. */
+crocco_status crocco_set_timing(crocco_ctx ctx, int32_t enable);
+crocco_status crocco_kernel_times(crocco_ctx ctx, int32_t max_classes, int64_t *launches,
+                                  double *ms, int32_t *n_classes);
+const char *crocco_kernel_class_name(int32_t cls);
+
+/* ---- host-only helpers (no CUDA needed; used by the CPU tests) -------------- */
+
+/* The ghost-exchange plan of desc for phase d and rank desc->rank: every
+   message whose dst block or src block lives on this rank, in the canonical
+   order both sides use for NCCL send/recv matching.  Writes up to cap entries,
+   *n_out = total count. */
+crocco_status crocco_exchange_plan(const crocco_grid_desc *desc, int32_t phase, crocco_msg *out,
+                                   int32_t cap, int32_t *n_out);
+/* Generate an ncclUniqueId (128 bytes written to out, size >= 128) on the rank
+   that bootstraps the communicator; the caller broadcasts it (torch.distributed)
+   and passes it as desc.nccl_unique_id on every rank. */
+crocco_status crocco_nccl_unique_id(void *out, int32_t size);
+/* Library version string. */
+const char *crocco_version(void);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* CROCCO_H */

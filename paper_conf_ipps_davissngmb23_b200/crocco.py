@@ -1,0 +1,261 @@
+"""Thin ctypes binding of libcrocco.so (include/crocco.h), same names as the C ABI.
+
+Argument marshalling only: every numerical step runs in the CUDA kernels of
+csrc/.  PyTorch is used for device memory (torch.empty on the GPU), streams
+and torch.distributed plumbing.  There is no CPU fallback: if the shared
+library is missing or fails to load, :func:`lib` raises.
+"""
+from __future__ import annotations
+
+import ctypes as C
+import os
+
+HERE = os.path.dirname(os.path.abspath(__file__))
+LIB_PATH = os.path.join(HERE, "libcrocco.so")
+
+CROCCO_OK, CROCCO_ERR_ARG, CROCCO_ERR_CUDA, CROCCO_ERR_NCCL, CROCCO_ERR_NOMEM, CROCCO_ERR_STATE = range(6)
+BC_PERIODIC, BC_EXTRAP, BC_DIRICHLET, BC_WALL = 0, 1, 2, 3
+TERM_INVISCID, TERM_VISCOUS = 1, 2
+MU_CONST, MU_SUTHERLAND = 0, 1
+FIELD_STATE, FIELD_METRIC = 0, 1
+GHOST, GHOST_COORDS = 4, 10
+
+
+class CroccoError(RuntimeError):
+    def __init__(self, status, msg):
+        super().__init__(f"crocco status {status}: {msg}")
+        self.status = status
+
+
+class GridDesc(C.Structure):
+    _fields_ = [("n_global", C.c_int64 * 3), ("n_blocks", C.c_int32 * 3),
+                ("bc", (C.c_int32 * 2) * 3), ("dirichlet", ((C.c_double * 5) * 2) * 3),
+                ("rank", C.c_int32), ("nranks", C.c_int32),
+                ("block_rank", C.POINTER(C.c_int32)), ("stream", C.c_void_p),
+                ("nccl_unique_id", C.c_void_p)]
+
+
+class PhysC(C.Structure):
+    _fields_ = [("gamma", C.c_double), ("R", C.c_double), ("Pr", C.c_double),
+                ("mu_law", C.c_int32), ("mu_ref", C.c_double), ("T_ref", C.c_double),
+                ("S", C.c_double), ("weno_eps", C.c_double), ("terms", C.c_int32),
+                ("dir_mask", C.c_int32)]
+
+
+class BlockLayout(C.Structure):
+    _fields_ = [("n", C.c_int32 * 3), ("origin", C.c_int64 * 3), ("ghost", C.c_int32),
+                ("ghost_coords", C.c_int32), ("offset", C.c_int64), ("pitch_y", C.c_int64),
+                ("pitch_z", C.c_int64), ("comp_stride", C.c_int64), ("coffset", C.c_int64),
+                ("cpitch_y", C.c_int64), ("cpitch_z", C.c_int64), ("ccomp_stride", C.c_int64),
+                ("global_id", C.c_int32)]
+
+
+class Msg(C.Structure):
+    _fields_ = [("phase", C.c_int32), ("dst_block", C.c_int32), ("side", C.c_int32),
+                ("kind", C.c_int32), ("bc_kind", C.c_int32), ("src_block", C.c_int32),
+                ("src_rank", C.c_int32), ("dst_rank", C.c_int32), ("dst_lo", C.c_int64 * 3),
+                ("src_lo", C.c_int64 * 3), ("ext", C.c_int64 * 3)]
+
+
+_lib = None
+
+DPP = C.POINTER(C.c_void_p)  # double *const * (array of device pointers)
+
+_SIGS = {
+    "crocco_init_grid": [C.POINTER(GridDesc), C.POINTER(PhysC), C.POINTER(C.c_void_p)],
+    "crocco_num_local_blocks": [C.c_void_p, C.POINTER(C.c_int32)],
+    "crocco_get_block_layout": [C.c_void_p, C.c_int32, C.POINTER(BlockLayout)],
+    "crocco_set_phys": [C.c_void_p, C.POINTER(PhysC)],
+    "crocco_scratch_bytes": [C.c_void_p, C.POINTER(C.c_int64)],
+    "crocco_init_metrics": [C.c_void_p, DPP, DPP],
+    "crocco_fill_boundary": [C.c_void_p, DPP, C.c_int32],
+    "crocco_rhs": [C.c_void_p, DPP, DPP, DPP],
+    "crocco_rk_stage": [C.c_void_p, C.c_int32, C.c_double, DPP, DPP, DPP, DPP],
+    "crocco_rk_update": [C.c_void_p, C.c_int32, C.c_double, DPP, DPP, DPP, DPP],
+    "crocco_sync": [C.c_void_p],
+    "crocco_finalize": [C.c_void_p],
+    "crocco_launch_count": [C.c_void_p, C.POINTER(C.c_int64), C.c_int32],
+    "crocco_set_timing": [C.c_void_p, C.c_int32],
+    "crocco_kernel_times": [C.c_void_p, C.c_int32, C.POINTER(C.c_int64), C.POINTER(C.c_double),
+                            C.POINTER(C.c_int32)],
+    "crocco_exchange_plan": [C.POINTER(GridDesc), C.c_int32, C.POINTER(Msg), C.c_int32,
+                             C.POINTER(C.c_int32)],
+    "crocco_nccl_unique_id": [C.c_void_p, C.c_int32],
+}
+_STR = {"crocco_last_error": [C.c_void_p], "crocco_version": [],
+        "crocco_kernel_class_name": [C.c_int32]}
+
+EXPORTED = sorted(list(_SIGS) + list(_STR))
+
+
+def lib() -> C.CDLL:
+    """Load libcrocco.so (fails loudly if it is missing -- no fallback)."""
+    global _lib
+    if _lib is None:
+        if not os.path.exists(LIB_PATH):
+            raise ImportError(f"{LIB_PATH} missing: run `python -m paper_conf_ipps_davissngmb23_b200.build`")
+        L = C.CDLL(LIB_PATH)
+        for name, args in _SIGS.items():
+            f = getattr(L, name)
+            f.argtypes = args
+            f.restype = C.c_int
+        for name, args in _STR.items():
+            f = getattr(L, name)
+            f.argtypes = args
+            f.restype = C.c_char_p
+        _lib = L
+    return _lib
+
+
+def _check(st, ctx=None):
+    if st != CROCCO_OK:
+        msg = lib().crocco_last_error(ctx)
+        raise CroccoError(st, msg.decode() if msg else "")
+
+
+def _ptrs(ptrs):
+    arr = (C.c_void_p * len(ptrs))(*[int(p) for p in ptrs])
+    return C.cast(arr, DPP), arr
+
+
+# ---------------------------------------------------------------- C-ABI mirrors
+
+def crocco_version() -> str:
+    return lib().crocco_version().decode()
+
+
+def crocco_kernel_class_name(k: int) -> str:
+    return lib().crocco_kernel_class_name(k).decode()
+
+
+def make_desc(n_global, n_blocks=(1, 1, 1), bc=((0, 0),) * 3, dirichlet=None, rank=0, nranks=1,
+              block_rank=None, stream=0, nccl_unique_id=None):
+    d = GridDesc()
+    for a in range(3):
+        d.n_global[a] = int(n_global[a])
+        d.n_blocks[a] = int(n_blocks[a])
+        for s in range(2):
+            d.bc[a][s] = int(bc[a][s])
+            for c in range(5):
+                d.dirichlet[a][s][c] = 0.0 if dirichlet is None else float(dirichlet[a][s][c])
+    d.rank, d.nranks = int(rank), int(nranks)
+    keep = []
+    if block_rank is not None:
+        arr = (C.c_int32 * len(block_rank))(*[int(x) for x in block_rank])
+        d.block_rank = C.cast(arr, C.POINTER(C.c_int32))
+        keep.append(arr)
+    d.stream = C.c_void_p(int(stream))
+    if nccl_unique_id is not None:
+        buf = C.create_string_buffer(bytes(nccl_unique_id), 128)
+        d.nccl_unique_id = C.cast(buf, C.c_void_p)
+        keep.append(buf)
+    d._keep = keep
+    return d
+
+
+def make_phys(gamma=1.4, R=1.0, Pr=0.72, mu_law=MU_CONST, mu_ref=0.0, T_ref=1.0, S=0.0,
+              weno_eps=1e-6, terms=TERM_INVISCID | TERM_VISCOUS, dir_mask=7):
+    return PhysC(gamma, R, Pr, mu_law, mu_ref, T_ref, S, weno_eps, terms, dir_mask)
+
+
+def crocco_init_grid(desc: GridDesc, phys: PhysC):
+    ctx = C.c_void_p()
+    _check(lib().crocco_init_grid(C.byref(desc), C.byref(phys), C.byref(ctx)))
+    return ctx
+
+
+def crocco_num_local_blocks(ctx) -> int:
+    n = C.c_int32()
+    _check(lib().crocco_num_local_blocks(ctx, C.byref(n)), ctx)
+    return n.value
+
+
+def crocco_get_block_layout(ctx, b: int) -> BlockLayout:
+    L = BlockLayout()
+    _check(lib().crocco_get_block_layout(ctx, b, C.byref(L)), ctx)
+    return L
+
+
+def crocco_set_phys(ctx, phys: PhysC):
+    _check(lib().crocco_set_phys(ctx, C.byref(phys)), ctx)
+
+
+def crocco_scratch_bytes(ctx) -> int:
+    v = C.c_int64()
+    _check(lib().crocco_scratch_bytes(ctx, C.byref(v)), ctx)
+    return v.value
+
+
+def crocco_init_metrics(ctx, xyz_ptrs, met_ptrs):
+    a, ka = _ptrs(xyz_ptrs)
+    b, kb = _ptrs(met_ptrs)
+    _check(lib().crocco_init_metrics(ctx, a, b), ctx)
+
+
+def crocco_fill_boundary(ctx, field_ptrs, kind=FIELD_STATE):
+    a, ka = _ptrs(field_ptrs)
+    _check(lib().crocco_fill_boundary(ctx, a, kind), ctx)
+
+
+def crocco_rhs(ctx, U_ptrs, met_ptrs, rhs_ptrs):
+    a, ka = _ptrs(U_ptrs)
+    b, kb = _ptrs(met_ptrs)
+    c, kc = _ptrs(rhs_ptrs)
+    _check(lib().crocco_rhs(ctx, a, b, c), ctx)
+
+
+def crocco_rk_stage(ctx, stage, dt, Uin_ptrs, Uout_ptrs, dU_ptrs, met_ptrs):
+    a, ka = _ptrs(Uin_ptrs)
+    b, kb = _ptrs(Uout_ptrs)
+    c, kc = _ptrs(dU_ptrs)
+    d, kd = _ptrs(met_ptrs)
+    _check(lib().crocco_rk_stage(ctx, stage, dt, a, b, c, d), ctx)
+
+
+def crocco_rk_update(ctx, stage, dt, Uin_ptrs, Uout_ptrs, dU_ptrs, rhs_ptrs):
+    a, ka = _ptrs(Uin_ptrs)
+    b, kb = _ptrs(Uout_ptrs)
+    c, kc = _ptrs(dU_ptrs)
+    d, kd = _ptrs(rhs_ptrs)
+    _check(lib().crocco_rk_update(ctx, stage, dt, a, b, c, d), ctx)
+
+
+def crocco_sync(ctx):
+    _check(lib().crocco_sync(ctx), ctx)
+
+
+def crocco_finalize(ctx):
+    _check(lib().crocco_finalize(ctx))
+
+
+def crocco_launch_count(ctx, reset=False) -> int:
+    v = C.c_int64()
+    _check(lib().crocco_launch_count(ctx, C.byref(v), int(reset)), ctx)
+    return v.value
+
+
+def crocco_set_timing(ctx, enable=True):
+    _check(lib().crocco_set_timing(ctx, int(enable)), ctx)
+
+
+def crocco_kernel_times(ctx):
+    n = 32
+    launches = (C.c_int64 * n)()
+    ms = (C.c_double * n)()
+    nc = C.c_int32()
+    _check(lib().crocco_kernel_times(ctx, n, launches, ms, C.byref(nc)), ctx)
+    return {crocco_kernel_class_name(k): (launches[k], ms[k]) for k in range(nc.value)}
+
+
+def crocco_exchange_plan(desc: GridDesc, phase: int):
+    n = C.c_int32()
+    _check(lib().crocco_exchange_plan(C.byref(desc), phase, None, 0, C.byref(n)))
+    arr = (Msg * max(n.value, 1))()
+    _check(lib().crocco_exchange_plan(C.byref(desc), phase, arr, n.value, C.byref(n)))
+    return [arr[i] for i in range(n.value)]
+
+
+def crocco_nccl_unique_id() -> bytes:
+    buf = C.create_string_buffer(128)
+    _check(lib().crocco_nccl_unique_id(C.cast(buf, C.c_void_p), 128))
+    return buf.raw

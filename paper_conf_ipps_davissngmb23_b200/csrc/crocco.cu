@@ -1,0 +1,879 @@
+// crocco.cu -- host side of libcrocco.so: the C ABI of include/crocco.h.
+//
+// Block decomposition, ghost-exchange plan, scratch management, launch
+// orchestration of the sm_100a kernels in kernels.cuh, NCCL halo exchange.
+// Algorithm 1/2 of the paper is the call order; every
+// numerical step runs in the CUDA kernels, never on the host.
+#include <cuda_runtime.h>
+#include <nccl.h>
+
+#include <algorithm>
+#include <cstdarg>
+#include <cstdio>
+#include <cstring>
+#include <string>
+#include <vector>
+
+#include "../../include/crocco.h"
+#include "kernels.cuh"
+
+using namespace crocco;
+
+namespace {
+
+thread_local std::string g_err;  // error text before a ctx exists
+
+struct BlockGeom {
+    int gid;
+    int bidx[3];
+    int n[3];
+    int64_t origin[3];
+    int rank;
+};
+
+struct LocalBlock {
+    BlockGeom g;
+    Lay L;       // state/metric layout
+    Lay C;       // coordinate layout
+    VLay V;      // viscous-flux box
+    double *prim = nullptr;
+    double *flux[3] = {nullptr, nullptr, nullptr};
+    int64_t fcs[3] = {0, 0, 0};
+    double *fv = nullptr;
+};
+
+enum { K_PRIMS = 0, K_FLUX_X, K_FLUX_Y, K_FLUX_Z, K_VISC, K_ASSEMBLE, K_UPDATE, K_FILL, K_METRICS,
+       K_NCLASS };
+const char *k_names[K_NCLASS] = {"prims", "flux_xi", "flux_eta", "flux_zeta", "viscous",
+                                 "assemble_update", "update", "fill", "metrics"};
+
+struct TimedLaunch {
+    int cls;
+    cudaEvent_t e0, e1;
+};
+
+}  // namespace
+
+struct crocco_ctx_s {
+    crocco_grid_desc desc;
+    std::vector<int32_t> block_rank;
+    crocco_phys phys_in;
+    Phys ph;
+    cudaStream_t stream = nullptr;
+    std::vector<BlockGeom> all;
+    std::vector<LocalBlock> loc;
+    std::vector<int> gid_to_local;
+    int nb[3];
+    int bn[3];  // block interior size
+    std::string err;
+    bool poisoned = false;
+    int64_t launches = 0;
+    int64_t scratch = 0;
+    // exchange plan per phase
+    std::vector<crocco_msg> plan[3];
+    // NCCL
+    ncclComm_t comm = nullptr;
+    double *send_stage = nullptr, *recv_stage = nullptr;
+    int64_t stage_elems = 0;
+    // timing
+    bool timing = false;
+    std::vector<TimedLaunch> pending;
+    std::vector<cudaEvent_t> pool;
+    int64_t t_launch[K_NCLASS] = {0};
+    double t_ms[K_NCLASS] = {0};
+};
+
+// ---------------------------------------------------------------------------
+// error helpers
+// ---------------------------------------------------------------------------
+static crocco_status fail(crocco_ctx c, crocco_status st, const char *fmt, ...) {
+    char buf[512];
+    va_list ap;
+    va_start(ap, fmt);
+    vsnprintf(buf, sizeof buf, fmt, ap);
+    va_end(ap);
+    if (c) {
+        c->err = buf;
+        if (st == CROCCO_ERR_CUDA || st == CROCCO_ERR_NCCL) c->poisoned = true;
+    } else {
+        g_err = buf;
+    }
+    return st;
+}
+#define CK(ctx, call)                                                                          \
+    do {                                                                                       \
+        cudaError_t e_ = (call);                                                               \
+        if (e_ != cudaSuccess)                                                                 \
+            return fail(ctx, CROCCO_ERR_CUDA, "%s:%d %s: %s", __FILE__, __LINE__, #call,       \
+                        cudaGetErrorString(e_));                                               \
+    } while (0)
+#define NK(ctx, call)                                                                          \
+    do {                                                                                       \
+        ncclResult_t r_ = (call);                                                              \
+        if (r_ != ncclSuccess)                                                                 \
+            return fail(ctx, CROCCO_ERR_NCCL, "%s:%d %s: %s", __FILE__, __LINE__, #call,       \
+                        ncclGetErrorString(r_));                                               \
+    } while (0)
+#define LIVE(ctx)                                                                              \
+    do {                                                                                       \
+        if (!(ctx)) return fail(nullptr, CROCCO_ERR_ARG, "null ctx");                           \
+        if ((ctx)->poisoned) return CROCCO_ERR_STATE;                                          \
+    } while (0)
+
+// launch bookkeeping: count + optional event timing on the launching stream
+static void pre_launch(crocco_ctx c, int cls, TimedLaunch *tl) {
+    c->launches++;
+    if (!c->timing) return;
+    auto get = [&]() {
+        cudaEvent_t e;
+        if (!c->pool.empty()) {
+            e = c->pool.back();
+            c->pool.pop_back();
+        } else {
+            cudaEventCreate(&e);
+        }
+        return e;
+    };
+    tl->cls = cls;
+    tl->e0 = get();
+    tl->e1 = get();
+    cudaEventRecord(tl->e0, c->stream);
+}
+static crocco_status post_launch(crocco_ctx c, TimedLaunch *tl) {
+    cudaError_t e = cudaGetLastError();
+    if (e != cudaSuccess) return fail(c, CROCCO_ERR_CUDA, "kernel launch: %s", cudaGetErrorString(e));
+    if (c->timing) {
+        cudaEventRecord(tl->e1, c->stream);
+        c->pending.push_back(*tl);
+    }
+    return CROCCO_OK;
+}
+#define LAUNCH(ctx, cls, ...)                                                                  \
+    do {                                                                                       \
+        TimedLaunch tl_;                                                                       \
+        pre_launch(ctx, cls, &tl_);                                                            \
+        __VA_ARGS__;                                                                           \
+        crocco_status s_ = post_launch(ctx, &tl_);                                             \
+        if (s_ != CROCCO_OK) return s_;                                                        \
+    } while (0)
+
+static inline int64_t rup(int64_t x, int64_t m) { return (x + m - 1) / m * m; }
+static inline unsigned cdiv(int64_t a, int64_t b) { return (unsigned)((a + b - 1) / b); }
+
+// padded layout: rows aligned to 128 B with interior i=0 on a 128-B boundary
+static Lay make_layout(const int n[3], int g) {
+    Lay L;
+    L.n0 = n[0];
+    L.n1 = n[1];
+    L.n2 = n[2];
+    const int64_t lead = 16;  // interior starts at element 16 of each row
+    L.py = rup(lead + n[0] + g, 16);
+    L.pz = L.py * (n[1] + 2 * g);
+    L.off = lead + L.py * g + L.pz * g;
+    L.cs = L.pz * (n[2] + 2 * g);
+    return L;
+}
+
+// ---------------------------------------------------------------------------
+// decomposition + exchange plan (host only)
+// ---------------------------------------------------------------------------
+static crocco_status validate(const crocco_grid_desc *d, int nb[3], int bn[3]) {
+    if (!d) return fail(nullptr, CROCCO_ERR_ARG, "null desc");
+    for (int a = 0; a < 3; a++) {
+        if (d->n_blocks[a] < 1 || d->n_global[a] < 1)
+            return fail(nullptr, CROCCO_ERR_ARG, "bad n_global/n_blocks in direction %d", a);
+        if (d->n_global[a] % d->n_blocks[a])
+            return fail(nullptr, CROCCO_ERR_ARG, "n_global[%d]=%lld not divisible by n_blocks=%d", a,
+                        (long long)d->n_global[a], d->n_blocks[a]);
+        nb[a] = d->n_blocks[a];
+        int64_t b = d->n_global[a] / nb[a];
+        if (b < G) return fail(nullptr, CROCCO_ERR_ARG, "block interior %lld < ghost width 4 in direction %d",
+                               (long long)b, a);
+        if (b > (1 << 20)) return fail(nullptr, CROCCO_ERR_ARG, "block too large");
+        bn[a] = (int)b;
+        for (int s = 0; s < 2; s++)
+            if (d->bc[a][s] < 0 || d->bc[a][s] > 3)
+                return fail(nullptr, CROCCO_ERR_ARG, "bad bc kind %d", d->bc[a][s]);
+        if ((d->bc[a][0] == CROCCO_BC_PERIODIC) != (d->bc[a][1] == CROCCO_BC_PERIODIC))
+            return fail(nullptr, CROCCO_ERR_ARG, "PERIODIC must be paired in direction %d", a);
+    }
+    if (d->nranks < 1 || d->rank < 0 || d->rank >= d->nranks)
+        return fail(nullptr, CROCCO_ERR_ARG, "bad rank/nranks");
+    const int nbt = nb[0] * nb[1] * nb[2];
+    if (!d->block_rank && d->nranks != 1)
+        return fail(nullptr, CROCCO_ERR_ARG, "block_rank required when nranks > 1");
+    if (d->block_rank)
+        for (int b = 0; b < nbt; b++)
+            if (d->block_rank[b] < 0 || d->block_rank[b] >= d->nranks)
+                return fail(nullptr, CROCCO_ERR_ARG, "block_rank[%d] out of range", b);
+    return CROCCO_OK;
+}
+
+static void build_blocks(const crocco_grid_desc *d, const int nb[3], const int bn[3],
+                         std::vector<BlockGeom> &all) {
+    all.clear();
+    for (int bz = 0; bz < nb[2]; bz++)
+        for (int by = 0; by < nb[1]; by++)
+            for (int bx = 0; bx < nb[0]; bx++) {
+                BlockGeom g;
+                g.gid = bx + nb[0] * (by + nb[1] * bz);
+                g.bidx[0] = bx;
+                g.bidx[1] = by;
+                g.bidx[2] = bz;
+                for (int a = 0; a < 3; a++) {
+                    g.n[a] = bn[a];
+                    g.origin[a] = (int64_t)g.bidx[a] * bn[a];
+                }
+                g.rank = d->block_rank ? d->block_rank[g.gid] : 0;
+                all.push_back(g);
+            }
+}
+
+// every message of phase `phase` touching rank `me` (me < 0: all), canonical order
+static void build_plan(const crocco_grid_desc *d, const int nb[3], const int bn[3],
+                       const std::vector<BlockGeom> &all, int phase, int me,
+                       std::vector<crocco_msg> &out) {
+    out.clear();
+    const int D = phase;
+    for (const BlockGeom &b : all) {
+        for (int side = 0; side < 2; side++) {
+            crocco_msg m;
+            memset(&m, 0, sizeof m);
+            m.phase = D;
+            m.dst_block = b.gid;
+            m.side = side;
+            m.bc_kind = d->bc[D][side];
+            m.dst_rank = b.rank;
+            // ghost box
+            for (int e = 0; e < 3; e++) {
+                if (e == D) {
+                    m.dst_lo[e] = side == 0 ? -G : bn[e];
+                    m.ext[e] = G;
+                } else if (e < D) {
+                    m.dst_lo[e] = -G;
+                    m.ext[e] = bn[e] + 2 * G;
+                } else {
+                    m.dst_lo[e] = 0;
+                    m.ext[e] = bn[e];
+                }
+                m.src_lo[e] = m.dst_lo[e];
+            }
+            int nbi = b.bidx[D] + (side == 0 ? -1 : 1);
+            bool physical = false;
+            if (nbi < 0 || nbi >= nb[D]) {
+                if (d->bc[D][side] == CROCCO_BC_PERIODIC)
+                    nbi = (nbi + nb[D]) % nb[D];
+                else
+                    physical = true;
+            }
+            if (physical) {
+                m.kind = 1;
+                m.src_block = -1;
+                m.src_rank = b.rank;
+            } else {
+                int idx[3] = {b.bidx[0], b.bidx[1], b.bidx[2]};
+                idx[D] = nbi;
+                const int sg = idx[0] + nb[0] * (idx[1] + nb[1] * idx[2]);
+                m.kind = 0;
+                m.src_block = sg;
+                m.src_rank = all[sg].rank;
+                m.src_lo[D] = side == 0 ? bn[D] - G : 0;
+            }
+            if (me < 0 || m.dst_rank == me || (m.kind == 0 && m.src_rank == me)) out.push_back(m);
+        }
+    }
+}
+
+// ---------------------------------------------------------------------------
+// ABI
+// ---------------------------------------------------------------------------
+extern "C" {
+
+crocco_status crocco_nccl_unique_id(void *out, int32_t size) {
+    if (!out || size < (int32_t)sizeof(ncclUniqueId))
+        return fail(nullptr, CROCCO_ERR_ARG, "need a %zu-byte buffer", sizeof(ncclUniqueId));
+    ncclUniqueId id;
+    ncclResult_t r = ncclGetUniqueId(&id);
+    if (r != ncclSuccess) return fail(nullptr, CROCCO_ERR_NCCL, "ncclGetUniqueId: %s", ncclGetErrorString(r));
+    memcpy(out, &id, sizeof id);
+    return CROCCO_OK;
+}
+
+const char *crocco_version(void) { return "crocco-b200 0.1 (sm_100a, fp64)"; }
+
+const char *crocco_last_error(crocco_ctx c) { return c ? c->err.c_str() : g_err.c_str(); }
+
+const char *crocco_kernel_class_name(int32_t cls) {
+    return (cls >= 0 && cls < K_NCLASS) ? k_names[cls] : "";
+}
+
+crocco_status crocco_exchange_plan(const crocco_grid_desc *desc, int32_t phase, crocco_msg *out,
+                                   int32_t cap, int32_t *n_out) {
+    int nb[3], bn[3];
+    crocco_status st = validate(desc, nb, bn);
+    if (st) return st;
+    if (phase < 0 || phase > 2) return fail(nullptr, CROCCO_ERR_ARG, "phase out of range");
+    std::vector<BlockGeom> all;
+    build_blocks(desc, nb, bn, all);
+    std::vector<crocco_msg> plan;
+    build_plan(desc, nb, bn, all, phase, desc->rank, plan);
+    if (n_out) *n_out = (int32_t)plan.size();
+    for (int i = 0; i < (int)plan.size() && i < cap; i++) out[i] = plan[i];
+    return CROCCO_OK;
+}
+
+static Phys to_phys(const crocco_phys *p) {
+    Phys ph;
+    ph.gamma = p->gamma;
+    ph.gm1 = p->gamma - 1.0;
+    ph.igm1 = 1.0 / (p->gamma - 1.0);
+    ph.R = p->R;
+    ph.Pr = p->Pr;
+    ph.cp_over_Pr = p->gamma * p->R / ((p->gamma - 1.0) * p->Pr);
+    ph.mu_law = p->mu_law;
+    ph.mu_ref = p->mu_ref;
+    ph.T_ref = p->T_ref;
+    ph.S = p->S;
+    ph.eps = p->weno_eps;
+    ph.terms = p->terms;
+    ph.dir_mask = p->dir_mask;
+    return ph;
+}
+
+static crocco_status check_phys(const crocco_phys *p) {
+    if (!p) return fail(nullptr, CROCCO_ERR_ARG, "null phys");
+    if (!(p->gamma > 1.0) || !(p->R > 0) || !(p->Pr > 0) || !(p->weno_eps > 0))
+        return fail(nullptr, CROCCO_ERR_ARG, "bad gas constants (need gamma>1, R>0, Pr>0, eps>0)");
+    if (p->mu_law != 0 && p->mu_law != 1) return fail(nullptr, CROCCO_ERR_ARG, "bad mu_law");
+    if (p->mu_law == 1 && !(p->T_ref > 0)) return fail(nullptr, CROCCO_ERR_ARG, "bad T_ref");
+    if (p->terms & ~3) return fail(nullptr, CROCCO_ERR_ARG, "bad terms mask");
+    return CROCCO_OK;
+}
+
+crocco_status crocco_set_phys(crocco_ctx c, const crocco_phys *p) {
+    LIVE(c);
+    crocco_status st = check_phys(p);
+    if (st) return fail(c, st, "%s", g_err.c_str());
+    c->phys_in = *p;
+    c->ph = to_phys(p);
+    return CROCCO_OK;
+}
+
+static void free_ctx(crocco_ctx c) {
+    for (auto &b : c->loc) {
+        cudaFree(b.prim);
+        for (int d = 0; d < 3; d++) cudaFree(b.flux[d]);
+        cudaFree(b.fv);
+    }
+    cudaFree(c->send_stage);
+    cudaFree(c->recv_stage);
+    for (auto &t : c->pending) {
+        cudaEventDestroy(t.e0);
+        cudaEventDestroy(t.e1);
+    }
+    for (auto e : c->pool) cudaEventDestroy(e);
+    if (c->comm) ncclCommDestroy(c->comm);
+    delete c;
+}
+
+crocco_status crocco_init_grid(const crocco_grid_desc *desc, const crocco_phys *phys,
+                               crocco_ctx *out) {
+    if (!out) return fail(nullptr, CROCCO_ERR_ARG, "null out");
+    *out = nullptr;
+    int nb[3], bn[3];
+    crocco_status st = validate(desc, nb, bn);
+    if (st) return st;
+    st = check_phys(phys);
+    if (st) return st;
+    crocco_ctx c = new crocco_ctx_s();
+    c->desc = *desc;
+    const int nbt = nb[0] * nb[1] * nb[2];
+    if (desc->block_rank) c->block_rank.assign(desc->block_rank, desc->block_rank + nbt);
+    else c->block_rank.assign(nbt, 0);
+    c->desc.block_rank = c->block_rank.data();
+    c->phys_in = *phys;
+    c->ph = to_phys(phys);
+    c->stream = (cudaStream_t)desc->stream;
+    for (int a = 0; a < 3; a++) {
+        c->nb[a] = nb[a];
+        c->bn[a] = bn[a];
+    }
+    build_blocks(&c->desc, nb, bn, c->all);
+    c->gid_to_local.assign(nbt, -1);
+    for (const BlockGeom &g : c->all) {
+        if (g.rank != desc->rank) continue;
+        LocalBlock lb;
+        lb.g = g;
+        lb.L = make_layout(g.n, G);
+        lb.C = make_layout(g.n, GC);
+        lb.V.b0 = g.n[0] + 4;
+        lb.V.b1 = g.n[1] + 4;
+        lb.V.b2 = g.n[2] + 4;
+        lb.V.cs = rup((int64_t)lb.V.b0 * lb.V.b1 * lb.V.b2, 32);
+        c->gid_to_local[g.gid] = (int)c->loc.size();
+        c->loc.push_back(lb);
+    }
+    for (int d = 0; d < 3; d++) build_plan(&c->desc, nb, bn, c->all, d, desc->rank, c->plan[d]);
+
+    // device scratch
+    auto alloc = [&](double **p, int64_t elems) -> bool {
+        if (cudaMalloc((void **)p, (size_t)elems * sizeof(double)) != cudaSuccess) return false;
+        c->scratch += elems * (int64_t)sizeof(double);
+        return true;
+    };
+    for (auto &b : c->loc) {
+        bool ok = alloc(&b.prim, NPRIM * b.L.cs);
+        b.fcs[0] = rup((int64_t)(b.g.n[0] + 1) * b.g.n[1] * b.g.n[2], 32);
+        b.fcs[1] = rup((int64_t)b.g.n[0] * (b.g.n[1] + 1) * b.g.n[2], 32);
+        b.fcs[2] = rup((int64_t)b.g.n[0] * b.g.n[1] * (b.g.n[2] + 1), 32);
+        for (int d = 0; d < 3; d++) ok = ok && alloc(&b.flux[d], 5 * b.fcs[d]);
+        ok = ok && alloc(&b.fv, 12 * b.V.cs);
+        if (!ok) {
+            cudaGetLastError();
+            free_ctx(c);
+            return fail(nullptr, CROCCO_ERR_NOMEM, "device scratch allocation failed");
+        }
+    }
+    // NCCL communicator + staging for remote halo messages
+    if (desc->nranks > 1) {
+        int64_t maxe = 0;
+        for (int d = 0; d < 3; d++) {
+            int64_t s = 0, r = 0;
+            for (auto &m : c->plan[d])
+                if (m.kind == 0 && m.src_rank != m.dst_rank) {
+                    const int64_t v = m.ext[0] * m.ext[1] * m.ext[2] * 10;
+                    if (m.src_rank == desc->rank) s += v;
+                    if (m.dst_rank == desc->rank) r += v;
+                }
+            maxe = std::max(maxe, std::max(s, r));
+        }
+        c->stage_elems = maxe;
+        if (maxe > 0) {
+            if (!alloc(&c->send_stage, maxe) || !alloc(&c->recv_stage, maxe)) {
+                cudaGetLastError();
+                free_ctx(c);
+                return fail(nullptr, CROCCO_ERR_NOMEM, "halo staging allocation failed");
+            }
+        }
+        if (!desc->nccl_unique_id) {
+            free_ctx(c);
+            return fail(nullptr, CROCCO_ERR_ARG, "nccl_unique_id required when nranks > 1");
+        }
+        ncclUniqueId id;
+        memcpy(&id, desc->nccl_unique_id, sizeof id);
+        ncclResult_t r = ncclCommInitRank(&c->comm, desc->nranks, id, desc->rank);
+        if (r != ncclSuccess) {
+            c->comm = nullptr;
+            free_ctx(c);
+            return fail(nullptr, CROCCO_ERR_NCCL, "ncclCommInitRank: %s", ncclGetErrorString(r));
+        }
+    }
+    *out = c;
+    return CROCCO_OK;
+}
+
+crocco_status crocco_num_local_blocks(crocco_ctx c, int32_t *n) {
+    LIVE(c);
+    if (!n) return fail(c, CROCCO_ERR_ARG, "null out");
+    *n = (int32_t)c->loc.size();
+    return CROCCO_OK;
+}
+
+crocco_status crocco_scratch_bytes(crocco_ctx c, int64_t *bytes) {
+    LIVE(c);
+    if (!bytes) return fail(c, CROCCO_ERR_ARG, "null out");
+    *bytes = c->scratch;
+    return CROCCO_OK;
+}
+
+crocco_status crocco_get_block_layout(crocco_ctx c, int32_t lb, crocco_block_layout *o) {
+    LIVE(c);
+    if (!o || lb < 0 || lb >= (int)c->loc.size()) return fail(c, CROCCO_ERR_ARG, "bad local block");
+    const LocalBlock &b = c->loc[lb];
+    memset(o, 0, sizeof *o);
+    for (int a = 0; a < 3; a++) {
+        o->n[a] = b.g.n[a];
+        o->origin[a] = b.g.origin[a];
+    }
+    o->ghost = G;
+    o->ghost_coords = GC;
+    o->offset = b.L.off;
+    o->pitch_y = b.L.py;
+    o->pitch_z = b.L.pz;
+    o->comp_stride = b.L.cs;
+    o->coffset = b.C.off;
+    o->cpitch_y = b.C.py;
+    o->cpitch_z = b.C.pz;
+    o->ccomp_stride = b.C.cs;
+    o->global_id = b.g.gid;
+    return CROCCO_OK;
+}
+
+// ---------------------------------------------------------------------------
+// ghost fill
+// ---------------------------------------------------------------------------
+static crocco_status flush_ops(crocco_ctx c, BoxOps &ops) {
+    if (ops.nops == 0) return CROCCO_OK;
+    int64_t mx = 0;
+    for (int i = 0; i < ops.nops; i++)
+        mx = std::max(mx, (int64_t)ops.op[i].ext[0] * ops.op[i].ext[1] * ops.op[i].ext[2]);
+    dim3 grid(std::min<int64_t>(cdiv(mx, 256), 4096), ops.nops);
+    LAUNCH(c, K_FILL, k_boxops<<<grid, 256, 0, c->stream>>>(ops));
+    ops.nops = 0;
+    return CROCCO_OK;
+}
+static crocco_status push_op(crocco_ctx c, BoxOps &ops, const BoxOp &o) {
+    ops.op[ops.nops++] = o;
+    if (ops.nops == MAX_OPS) return flush_ops(c, ops);
+    return CROCCO_OK;
+}
+
+static void op_strides(const Lay &L, int64_t st[3]) {
+    st[0] = 1;
+    st[1] = L.py;
+    st[2] = L.pz;
+}
+
+static crocco_status fill_phase(crocco_ctx c, double *const *f, int kind, int D) {
+    const int ncomp = kind == CROCCO_FIELD_STATE ? 5 : 10;
+    BoxOps ops;
+    ops.nops = 0;
+    std::vector<const crocco_msg *> remote;
+    for (const crocco_msg &m : c->plan[D]) {
+        if (m.kind == 0 && (m.src_rank != m.dst_rank)) {
+            remote.push_back(&m);
+            continue;
+        }
+        if (m.dst_rank != c->desc.rank) continue;
+        const int dl = c->gid_to_local[m.dst_block];
+        const LocalBlock &db = c->loc[dl];
+        BoxOp o;
+        memset(&o, 0, sizeof o);
+        o.dst = f[dl];
+        op_strides(db.L, o.dst_);
+        o.dcs = db.L.cs;
+        o.dbase = at(db.L, (int)m.dst_lo[0], (int)m.dst_lo[1], (int)m.dst_lo[2]);
+        for (int e = 0; e < 3; e++) o.ext[e] = (int)m.ext[e];
+        o.ncomp = ncomp;
+        if (m.kind == 0) {  // periodic / inter-block copy, same rank
+            const int sl = c->gid_to_local[m.src_block];
+            const LocalBlock &sb = c->loc[sl];
+            o.src = f[sl];
+            op_strides(sb.L, o.sst);
+            o.scs = sb.L.cs;
+            o.sbase = at(sb.L, (int)m.src_lo[0], (int)m.src_lo[1], (int)m.src_lo[2]);
+            o.mode = 0;
+        } else {
+            if (kind == CROCCO_FIELD_METRIC) continue;  // physical faces keep computed metrics
+            const int bc = m.bc_kind;
+            const int n = db.g.n[D];
+            int64_t st[3];
+            op_strides(db.L, st);
+            o.src = f[dl];
+            o.scs = db.L.cs;
+            for (int e = 0; e < 3; e++) o.sst[e] = st[e];
+            int lo[3] = {(int)m.dst_lo[0], (int)m.dst_lo[1], (int)m.dst_lo[2]};
+            if (bc == CROCCO_BC_EXTRAP) {
+                lo[D] = m.side == 0 ? 0 : n - 1;
+                o.sst[D] = 0;
+            } else if (bc == CROCCO_BC_WALL) {
+                // dst index (lo + t) <- src index mirrored about the face
+                lo[D] = m.side == 0 ? G - 1 : n - 1;
+                o.sst[D] = -st[D];
+                o.flip_mom = 1;
+            } else {  // DIRICHLET
+                o.mode = 1;
+                for (int q = 0; q < 5; q++) o.val[q] = c->desc.dirichlet[D][m.side][q];
+            }
+            o.sbase = at(db.L, lo[0], lo[1], lo[2]);
+        }
+        crocco_status st = push_op(c, ops, o);
+        if (st) return st;
+    }
+    crocco_status st = flush_ops(c, ops);
+    if (st) return st;
+    if (remote.empty()) return CROCCO_OK;
+    if (!c->comm) return fail(c, CROCCO_ERR_STATE, "remote halo without communicator");
+    // pack sends
+    int64_t soff = 0, roff = 0;
+    std::vector<int64_t> offs(remote.size());
+    for (size_t r = 0; r < remote.size(); r++) {
+        const crocco_msg &m = *remote[r];
+        const int64_t vol = m.ext[0] * m.ext[1] * m.ext[2];
+        if (m.src_rank == c->desc.rank) {
+            const int sl = c->gid_to_local[m.src_block];
+            const LocalBlock &sb = c->loc[sl];
+            BoxOp o;
+            memset(&o, 0, sizeof o);
+            o.src = f[sl];
+            op_strides(sb.L, o.sst);
+            o.scs = sb.L.cs;
+            o.sbase = at(sb.L, (int)m.src_lo[0], (int)m.src_lo[1], (int)m.src_lo[2]);
+            o.dst = c->send_stage + soff;
+            o.dst_[0] = 1;
+            o.dst_[1] = m.ext[0];
+            o.dst_[2] = m.ext[0] * m.ext[1];
+            o.dcs = vol;
+            o.dbase = 0;
+            for (int e = 0; e < 3; e++) o.ext[e] = (int)m.ext[e];
+            o.ncomp = ncomp;
+            offs[r] = soff;
+            soff += vol * ncomp;
+            st = push_op(c, ops, o);
+            if (st) return st;
+        } else {
+            offs[r] = roff;
+            roff += vol * ncomp;
+        }
+    }
+    st = flush_ops(c, ops);
+    if (st) return st;
+    NK(c, ncclGroupStart());
+    for (size_t r = 0; r < remote.size(); r++) {
+        const crocco_msg &m = *remote[r];
+        const size_t cnt = (size_t)(m.ext[0] * m.ext[1] * m.ext[2] * ncomp);
+        if (m.src_rank == c->desc.rank)
+            NK(c, ncclSend(c->send_stage + offs[r], cnt, ncclDouble, m.dst_rank, c->comm, c->stream));
+        else
+            NK(c, ncclRecv(c->recv_stage + offs[r], cnt, ncclDouble, m.src_rank, c->comm, c->stream));
+    }
+    NK(c, ncclGroupEnd());
+    // unpack receives
+    for (size_t r = 0; r < remote.size(); r++) {
+        const crocco_msg &m = *remote[r];
+        if (m.dst_rank != c->desc.rank) continue;
+        const int dl = c->gid_to_local[m.dst_block];
+        const LocalBlock &db = c->loc[dl];
+        const int64_t vol = m.ext[0] * m.ext[1] * m.ext[2];
+        BoxOp o;
+        memset(&o, 0, sizeof o);
+        o.src = c->recv_stage + offs[r];
+        o.sst[0] = 1;
+        o.sst[1] = m.ext[0];
+        o.sst[2] = m.ext[0] * m.ext[1];
+        o.scs = vol;
+        o.sbase = 0;
+        o.dst = f[dl];
+        op_strides(db.L, o.dst_);
+        o.dcs = db.L.cs;
+        o.dbase = at(db.L, (int)m.dst_lo[0], (int)m.dst_lo[1], (int)m.dst_lo[2]);
+        for (int e = 0; e < 3; e++) o.ext[e] = (int)m.ext[e];
+        o.ncomp = ncomp;
+        st = push_op(c, ops, o);
+        if (st) return st;
+    }
+    return flush_ops(c, ops);
+}
+
+static crocco_status check_ptrs(crocco_ctx c, double *const *p, const char *what) {
+    if (!p) return fail(c, CROCCO_ERR_ARG, "null %s pointer array", what);
+    for (size_t b = 0; b < c->loc.size(); b++)
+        if (!p[b]) return fail(c, CROCCO_ERR_ARG, "null %s pointer for local block %zu", what, b);
+    return CROCCO_OK;
+}
+
+crocco_status crocco_fill_boundary(crocco_ctx c, double *const *f, int32_t kind) {
+    LIVE(c);
+    if (kind != CROCCO_FIELD_STATE && kind != CROCCO_FIELD_METRIC)
+        return fail(c, CROCCO_ERR_ARG, "bad field kind");
+    crocco_status st = check_ptrs(c, f, "field");
+    if (st) return st;
+    for (int d = 0; d < 3; d++) {
+        st = fill_phase(c, f, kind, d);
+        if (st) return st;
+    }
+    return CROCCO_OK;
+}
+
+// ---------------------------------------------------------------------------
+// metrics
+// ---------------------------------------------------------------------------
+crocco_status crocco_init_metrics(crocco_ctx c, double *const *xyz, double *const *met) {
+    LIVE(c);
+    crocco_status st = check_ptrs(c, xyz, "xyz");
+    if (st) return st;
+    st = check_ptrs(c, met, "metrics");
+    if (st) return st;
+    for (size_t b = 0; b < c->loc.size(); b++) {
+        const LocalBlock &lb = c->loc[b];
+        double *dx = nullptr;
+        CK(c, cudaMallocAsync((void **)&dx, (size_t)(9 * lb.C.cs) * sizeof(double), c->stream));
+        const int W = G + 3;
+        const int64_t nd = (int64_t)(lb.g.n[0] + 2 * W) * (lb.g.n[1] + 2 * W) * (lb.g.n[2] + 2 * W);
+        LAUNCH(c, K_METRICS, k_coord_deriv<<<cdiv(nd, 256), 256, 0, c->stream>>>(xyz[b], dx, lb.C));
+        const int64_t nm = (int64_t)(lb.g.n[0] + 2 * G) * (lb.g.n[1] + 2 * G) * (lb.g.n[2] + 2 * G);
+        LAUNCH(c, K_METRICS, k_metric<<<cdiv(nm, 128), 128, 0, c->stream>>>(xyz[b], dx, met[b], lb.C, lb.L));
+        CK(c, cudaFreeAsync(dx, c->stream));
+    }
+    return crocco_fill_boundary(c, met, CROCCO_FIELD_METRIC);
+}
+
+// ---------------------------------------------------------------------------
+// RHS / RK
+// ---------------------------------------------------------------------------
+static crocco_status rhs_parts(crocco_ctx c, const LocalBlock &b, const double *U, const double *M) {
+    const Phys &ph = c->ph;
+    const int64_t np = (int64_t)(b.g.n[0] + 2 * G) * (b.g.n[1] + 2 * G) * (b.g.n[2] + 2 * G);
+    LAUNCH(c, K_PRIMS, k_prims<<<cdiv(np, 256), 256, 0, c->stream>>>(U, b.prim, b.L, ph));
+    if (ph.terms & CROCCO_TERM_INVISCID) {
+        if (ph.dir_mask & 1) {
+            const int64_t t = (int64_t)(b.g.n[0] + 1) * b.g.n[1] * b.g.n[2];
+            LAUNCH(c, K_FLUX_X,
+                   k_flux<0><<<cdiv(t, 128), 128, 0, c->stream>>>(U, b.prim, M, b.flux[0], b.fcs[0], b.L, ph));
+        }
+        if (ph.dir_mask & 2) {
+            dim3 blk(32, 4);
+            dim3 grd(cdiv(b.g.n[0], 32), cdiv((int64_t)(b.g.n[1] + 1) * b.g.n[2], 4));
+            LAUNCH(c, K_FLUX_Y,
+                   k_flux<1><<<grd, blk, 0, c->stream>>>(U, b.prim, M, b.flux[1], b.fcs[1], b.L, ph));
+        }
+        if (ph.dir_mask & 4) {
+            dim3 blk(32, 4);
+            dim3 grd(cdiv(b.g.n[0], 32), cdiv((int64_t)b.g.n[1] * (b.g.n[2] + 1), 4));
+            LAUNCH(c, K_FLUX_Z,
+                   k_flux<2><<<grd, blk, 0, c->stream>>>(U, b.prim, M, b.flux[2], b.fcs[2], b.L, ph));
+        }
+    }
+    if (ph.terms & CROCCO_TERM_VISCOUS) {
+        const int64_t nv = (int64_t)b.V.b0 * b.V.b1 * b.V.b2;
+        LAUNCH(c, K_VISC, k_visc<<<cdiv(nv, 256), 256, 0, c->stream>>>(b.prim, M, b.fv, b.L, b.V, ph));
+    }
+    return CROCCO_OK;
+}
+
+static Asm make_asm(crocco_ctx c, const LocalBlock &b, const double *M) {
+    Asm a;
+    memset(&a, 0, sizeof a);
+    for (int d = 0; d < 3; d++) {
+        a.F[d] = b.flux[d];
+        a.fcs[d] = b.fcs[d];
+    }
+    a.FV = b.fv;
+    a.V = b.V;
+    a.M = M;
+    a.inv_mask = (c->ph.terms & CROCCO_TERM_INVISCID) ? (c->ph.dir_mask & 7) : 0;
+    a.visc = (c->ph.terms & CROCCO_TERM_VISCOUS) ? 1 : 0;
+    return a;
+}
+
+crocco_status crocco_rhs(crocco_ctx c, double *const *U, double *const *M, double *const *rhs) {
+    LIVE(c);
+    crocco_status st;
+    if ((st = check_ptrs(c, U, "U")) || (st = check_ptrs(c, M, "metrics")) ||
+        (st = check_ptrs(c, rhs, "rhs")))
+        return st;
+    for (size_t bi = 0; bi < c->loc.size(); bi++)
+        if (rhs[bi] == U[bi]) return fail(c, CROCCO_ERR_ARG, "rhs aliases U");
+    for (size_t bi = 0; bi < c->loc.size(); bi++) {
+        const LocalBlock &b = c->loc[bi];
+        if ((st = rhs_parts(c, b, U[bi], M[bi]))) return st;
+        Asm a = make_asm(c, b, M[bi]);
+        a.mode = 0;
+        a.rhs = rhs[bi];
+        dim3 grd(cdiv(b.g.n[0], 128), b.g.n[1], b.g.n[2]);
+        LAUNCH(c, K_ASSEMBLE, k_assemble<<<grd, 128, 0, c->stream>>>(a, b.L));
+    }
+    return CROCCO_OK;
+}
+
+static const double RK_A[3] = {0.0, -5.0 / 9.0, -153.0 / 128.0};
+static const double RK_B[3] = {1.0 / 3.0, 15.0 / 16.0, 8.0 / 15.0};
+
+crocco_status crocco_rk_stage(crocco_ctx c, int32_t stage, double dt, double *const *Uin,
+                              double *const *Uout, double *const *dU, double *const *M) {
+    LIVE(c);
+    crocco_status st;
+    if (stage < 0 || stage > 2) return fail(c, CROCCO_ERR_ARG, "stage must be 0..2");
+    if ((st = check_ptrs(c, Uin, "U_in")) || (st = check_ptrs(c, Uout, "U_out")) ||
+        (st = check_ptrs(c, dU, "dU")) || (st = check_ptrs(c, M, "metrics")))
+        return st;
+    for (size_t bi = 0; bi < c->loc.size(); bi++)
+        if (Uin[bi] == Uout[bi] || dU[bi] == Uin[bi] || dU[bi] == Uout[bi])
+            return fail(c, CROCCO_ERR_ARG, "U_in, U_out and dU must be distinct");
+    if ((st = crocco_fill_boundary(c, Uin, CROCCO_FIELD_STATE))) return st;
+    for (size_t bi = 0; bi < c->loc.size(); bi++) {
+        const LocalBlock &b = c->loc[bi];
+        if ((st = rhs_parts(c, b, Uin[bi], M[bi]))) return st;
+        Asm a = make_asm(c, b, M[bi]);
+        a.mode = 1;
+        a.Uin = Uin[bi];
+        a.Uout = Uout[bi];
+        a.dU = dU[bi];
+        a.stage = stage;
+        a.A = RK_A[stage];
+        a.B = RK_B[stage];
+        a.dt = dt;
+        dim3 grd(cdiv(b.g.n[0], 128), b.g.n[1], b.g.n[2]);
+        LAUNCH(c, K_ASSEMBLE, k_assemble<<<grd, 128, 0, c->stream>>>(a, b.L));
+    }
+    return CROCCO_OK;
+}
+
+crocco_status crocco_rk_update(crocco_ctx c, int32_t stage, double dt, double *const *Uin,
+                               double *const *Uout, double *const *dU, double *const *rhs) {
+    LIVE(c);
+    crocco_status st;
+    if (stage < 0 || stage > 2) return fail(c, CROCCO_ERR_ARG, "stage must be 0..2");
+    if ((st = check_ptrs(c, Uin, "U_in")) || (st = check_ptrs(c, Uout, "U_out")) ||
+        (st = check_ptrs(c, dU, "dU")) || (st = check_ptrs(c, rhs, "rhs")))
+        return st;
+    for (size_t bi = 0; bi < c->loc.size(); bi++) {
+        const LocalBlock &b = c->loc[bi];
+        dim3 grd(cdiv(b.g.n[0], 128), b.g.n[1], b.g.n[2]);
+        LAUNCH(c, K_UPDATE, k_update<<<grd, 128, 0, c->stream>>>(Uin[bi], Uout[bi], dU[bi], rhs[bi], b.L,
+                                                                  stage, RK_A[stage], RK_B[stage], dt));
+    }
+    return CROCCO_OK;
+}
+
+crocco_status crocco_sync(crocco_ctx c) {
+    LIVE(c);
+    CK(c, cudaStreamSynchronize(c->stream));
+    CK(c, cudaGetLastError());
+    return CROCCO_OK;
+}
+
+crocco_status crocco_finalize(crocco_ctx c) {
+    if (!c) return CROCCO_OK;
+    cudaStreamSynchronize(c->stream);
+    free_ctx(c);
+    return CROCCO_OK;
+}
+
+crocco_status crocco_launch_count(crocco_ctx c, int64_t *count, int32_t reset) {
+    if (!c) return fail(nullptr, CROCCO_ERR_ARG, "null ctx");
+    if (count) *count = c->launches;
+    if (reset) c->launches = 0;
+    return CROCCO_OK;
+}
+
+crocco_status crocco_set_timing(crocco_ctx c, int32_t enable) {
+    LIVE(c);
+    c->timing = enable != 0;
+    return CROCCO_OK;
+}
+
+crocco_status crocco_kernel_times(crocco_ctx c, int32_t maxc, int64_t *launches, double *ms,
+                                  int32_t *ncls) {
+    LIVE(c);
+    for (auto &t : c->pending) {
+        CK(c, cudaEventSynchronize(t.e1));
+        float f = 0.f;
+        CK(c, cudaEventElapsedTime(&f, t.e0, t.e1));
+        c->t_launch[t.cls]++;
+        c->t_ms[t.cls] += f;
+        c->pool.push_back(t.e0);
+        c->pool.push_back(t.e1);
+    }
+    c->pending.clear();
+    if (ncls) *ncls = K_NCLASS;
+    for (int k = 0; k < K_NCLASS && k < maxc; k++) {
+        if (launches) launches[k] = c->t_launch[k];
+        if (ms) ms[k] = c->t_ms[k];
+        c->t_launch[k] = 0;
+        c->t_ms[k] = 0;
+    }
+    return CROCCO_OK;
+}
+
+}  // extern "C"

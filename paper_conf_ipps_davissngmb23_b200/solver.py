@@ -1,0 +1,123 @@
+"""Convenience driver over the C ABI: allocates caller-owned device arrays with
+torch per crocco_block_layout, uploads/downloads numpy padded arrays, and runs
+RK3 steps (Algorithm 1/2 of the paper, without Regrid and
+with a fixed dt).  Plumbing only -- every numerical step is a libcrocco kernel.
+"""
+from __future__ import annotations
+
+import numpy as np
+import torch
+
+from . import crocco as cc
+
+G = cc.GHOST
+GC = cc.GHOST_COORDS
+
+
+class Solver:
+    def __init__(self, n_global, n_blocks=(1, 1, 1), bc=((0, 0),) * 3, phys=None, dirichlet=None,
+                 rank=0, nranks=1, block_rank=None, device=None, stream=None, nccl_unique_id=None):
+        if not torch.cuda.is_available():
+            raise RuntimeError("libcrocco needs a CUDA device (no CPU fallback)")
+        self.device = torch.device(device if device is not None else "cuda")
+        torch.cuda.set_device(self.device)
+        self.stream = stream if stream is not None else torch.cuda.current_stream(self.device)
+        self.phys = phys if phys is not None else cc.make_phys()
+        self.desc = cc.make_desc(n_global, n_blocks, bc, dirichlet, rank, nranks, block_rank,
+                                 self.stream.cuda_stream, nccl_unique_id)
+        self.ctx = cc.crocco_init_grid(self.desc, self.phys)
+        self.nloc = cc.crocco_num_local_blocks(self.ctx)
+        self.layouts = [cc.crocco_get_block_layout(self.ctx, b) for b in range(self.nloc)]
+        self.U = [self._alloc(L, 5) for L in self.layouts]
+        self.V = [self._alloc(L, 5) for L in self.layouts]
+        self.dU = [self._alloc(L, 5) for L in self.layouts]
+        self.met = [self._alloc(L, 10) for L in self.layouts]
+        self.rhs_buf = None
+
+    # ------------------------------------------------------------ memory
+    def _alloc(self, L, ncomp):
+        return torch.zeros(ncomp * L.comp_stride, dtype=torch.float64, device=self.device)
+
+    def view(self, buf, b, ncomp, coords=False):
+        """(ncomp, P2, P1, P0) strided view of a block array (index [c, k+g, j+g, i+g])."""
+        L = self.layouts[b]
+        if coords:
+            g, off, py, pz, cs = GC, L.coffset, L.cpitch_y, L.cpitch_z, L.ccomp_stride
+        else:
+            g, off, py, pz, cs = G, L.offset, L.pitch_y, L.pitch_z, L.comp_stride
+        n = L.n
+        return torch.as_strided(buf, (ncomp, n[2] + 2 * g, n[1] + 2 * g, n[0] + 2 * g),
+                                (cs, pz, py, 1), off - g - g * py - g * pz)
+
+    @staticmethod
+    def _ptrs(bufs):
+        return [t.data_ptr() for t in bufs]
+
+    # ------------------------------------------------------------ setup
+    def set_coords(self, xyz_blocks):
+        """xyz_blocks[b]: numpy (3, P2, P1, P0) on the coordinate band (g = 10); runs InitGridMetrics."""
+        tmp = []
+        for b in range(self.nloc):
+            L = self.layouts[b]
+            t = torch.zeros(3 * L.ccomp_stride, dtype=torch.float64, device=self.device)
+            src = xyz_blocks[b]
+            if not isinstance(src, torch.Tensor):
+                src = torch.from_numpy(np.ascontiguousarray(src))
+            self.view(t, b, 3, coords=True).copy_(src)
+            tmp.append(t)
+        cc.crocco_init_metrics(self.ctx, self._ptrs(tmp), self._ptrs(self.met))
+        self.sync()
+        del tmp
+
+    def set_state(self, U_blocks, interior=True):
+        """U_blocks[b]: numpy conserved state, interior (5, n2, n1, n0) or padded."""
+        for b in range(self.nloc):
+            v = self.view(self.U[b], b, 5)
+            src = U_blocks[b]
+            if not isinstance(src, torch.Tensor):
+                src = torch.from_numpy(np.ascontiguousarray(src))
+            if interior:
+                v[:, G:-G, G:-G, G:-G].copy_(src)
+            else:
+                v.copy_(src)
+
+    def get(self, bufs, ncomp=5):
+        return [self.view(bufs[b], b, ncomp).cpu().numpy() for b in range(self.nloc)]
+
+    # ------------------------------------------------------------ hot path
+    def fill(self, bufs=None, kind=cc.FIELD_STATE):
+        cc.crocco_fill_boundary(self.ctx, self._ptrs(bufs if bufs is not None else self.U), kind)
+
+    def rhs(self):
+        if self.rhs_buf is None:
+            self.rhs_buf = [self._alloc(L, 5) for L in self.layouts]
+        cc.crocco_rhs(self.ctx, self._ptrs(self.U), self._ptrs(self.met), self._ptrs(self.rhs_buf))
+        return self.rhs_buf
+
+    def stage(self, s, dt):
+        cc.crocco_rk_stage(self.ctx, s, dt, self._ptrs(self.U), self._ptrs(self.V),
+                           self._ptrs(self.dU), self._ptrs(self.met))
+        self.U, self.V = self.V, self.U
+
+    def step(self, dt, nsteps=1):
+        for _ in range(nsteps):
+            for s in range(3):
+                self.stage(s, dt)
+
+    def set_phys(self, phys):
+        self.phys = phys
+        cc.crocco_set_phys(self.ctx, phys)
+
+    def sync(self):
+        cc.crocco_sync(self.ctx)
+
+    def close(self):
+        if self.ctx is not None:
+            cc.crocco_finalize(self.ctx)
+            self.ctx = None
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass

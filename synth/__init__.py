@@ -27,10 +27,17 @@ GC = 10
 # ---------------------------------------------------------------- grids
 
 def _index_grids(n, origin, g):
-    """Global index arrays (float64) for the padded box of a block."""
+    """Global index arrays (float64) for the padded box of a block, as mutually
+    broadcastable arrays I (1,1,P0), J (1,P1,1), K (P2,1,1)."""
     ax = [np.arange(origin[d] - g, origin[d] + n[d] + g, dtype=np.float64) for d in range(3)]
-    K, J, I = np.meshgrid(ax[2], ax[1], ax[0], indexing="ij")
-    return I, J, K
+    return ax[0][None, None, :], ax[1][None, :, None], ax[2][:, None, None]
+
+
+def _stack3(a, b, c):
+    shape = np.broadcast_shapes(np.shape(a), np.shape(b), np.shape(c))
+    out = np.empty((3,) + shape)
+    out[0], out[1], out[2] = a, b, c
+    return out
 
 
 @dataclass
@@ -43,9 +50,9 @@ class Cartesian:
     def coords(self, n, origin=(0, 0, 0), g=GC):
         I, J, K = _index_grids(n, origin, g)
         off = 0.5 if self.centred else 0.0
-        return np.stack([self.x0[0] + (I + off) * self.h[0],
-                         self.x0[1] + (J + off) * self.h[1],
-                         self.x0[2] + (K + off) * self.h[2]])
+        return _stack3(self.x0[0] + (I + off) * self.h[0],
+                       self.x0[1] + (J + off) * self.h[1],
+                       self.x0[2] + (K + off) * self.h[2])
 
 
 @dataclass
@@ -65,9 +72,9 @@ class Wavy3D:
         et = self.x0[1] + J * self.L[1] / self.N[1]
         ze = self.x0[2] + K * self.L[2] / self.N[2]
         k, A = self.k, self.A
-        return np.stack([xi + A * np.sin(k * et) * np.sin(k * ze),
-                         et + A * np.sin(k * ze) * np.sin(k * xi),
-                         ze + A * np.sin(k * xi) * np.sin(k * et)])
+        return _stack3(xi + A * np.sin(k * et) * np.sin(k * ze),
+                       et + A * np.sin(k * ze) * np.sin(k * xi),
+                       ze + A * np.sin(k * xi) * np.sin(k * et))
 
 
 @dataclass
@@ -84,9 +91,9 @@ class Wavy2D:
         xi = I * self.L[0] / self.N[0]
         et = J * self.L[1] / self.N[1]
         ze = K * self.L[2] / self.N[2]
-        return np.stack([xi + self.A * np.sin(self.k * et),
-                         et + self.A * np.sin(self.k * xi),
-                         ze])
+        return _stack3(xi + self.A * np.sin(self.k * et),
+                       et + self.A * np.sin(self.k * xi),
+                       ze)
 
 
 @dataclass
@@ -110,14 +117,23 @@ class Ramp:
         x = 4.0 * I / self.N[0]
         y = self.wall(x) + np.sinh(3.0 * (J + 0.5) / self.N[1]) / math.sinh(3.0)
         z = K / self.N[2]
-        return np.stack([x, y, z])
+        return _stack3(x, y, z)
 
 
 # ---------------------------------------------------------------- states
 
+def _xp(a):
+    """numpy, or torch when the input is a torch tensor (device-side generation in bench.py)."""
+    if type(a).__module__.startswith("torch"):
+        import torch
+        return torch
+    return np
+
+
 def prim_to_cons(rho, u, v, w, p, gamma=1.4):
     """Conserved (rho, rho u, rho v, rho w, E), E = p/(gamma-1) + rho|u|^2/2 (Eq. 2)."""
-    return np.stack([rho, rho * u, rho * v, rho * w,
+    xp = _xp(rho)
+    return xp.stack([rho, rho * u, rho * v, rho * w,
                      p / (gamma - 1.0) + 0.5 * rho * (u * u + v * v + w * w)])
 
 
@@ -177,14 +193,15 @@ def free_stream(xyz, rho=1.0, vel=(0.7, -0.3, 0.4), p=1.0 / 1.4, gamma=1.4):
 def tgv(xyz, V0=1.0, rho0=1.0, M0=0.1, gamma=1.4, R=1.0, noise=0.0, seed=5, period=2 * math.pi):
     """DeBonis (2013) Taylor-Green vortex, T0 = 1/(gamma M0^2) (c0 = 1/M0 for V0 = 1)."""
     X = _interior_xyz(xyz)
+    xp = _xp(X)
     s = 2 * math.pi / period
     x, y, z = X[0] * s, X[1] * s, X[2] * s
     T0 = V0 ** 2 / (gamma * R * M0 ** 2)
     p0 = rho0 * R * T0
-    u = V0 * np.sin(x) * np.cos(y) * np.cos(z)
-    v = -V0 * np.cos(x) * np.sin(y) * np.cos(z)
-    w = np.zeros_like(x)
-    p = p0 + rho0 * V0 ** 2 / 16.0 * (np.cos(2 * x) + np.cos(2 * y)) * (np.cos(2 * z) + 2.0)
+    u = V0 * xp.sin(x) * xp.cos(y) * xp.cos(z)
+    v = -V0 * xp.cos(x) * xp.sin(y) * xp.cos(z)
+    w = xp.zeros_like(x)
+    p = p0 + rho0 * V0 ** 2 / 16.0 * (xp.cos(2 * x) + xp.cos(2 * y)) * (xp.cos(2 * z) + 2.0)
     if noise:
         u = u + noise * V0 * smooth_noise(x, y, z, seed, 0)
         v = v + noise * V0 * smooth_noise(x, y, z, seed, 1)
@@ -196,13 +213,14 @@ def tgv(xyz, V0=1.0, rho0=1.0, M0=0.1, gamma=1.4, R=1.0, noise=0.0, seed=5, peri
 def smooth_noise(x, y, z, seed, comp, modes=4):
     """Sum of a few 2pi-periodic Fourier modes with seeded random amplitudes/phases, |.| <= 1."""
     rng = np.random.default_rng([seed, comp])
-    out = np.zeros_like(x)
+    xp = _xp(x)
+    out = xp.zeros_like(x)
     tot = 0.0
     for _ in range(modes):
-        kx, ky, kz = rng.integers(1, 4, size=3)
-        a = rng.uniform(0.5, 1.0)
-        ph = rng.uniform(0, 2 * math.pi, size=3)
-        out += a * np.sin(kx * x + ph[0]) * np.sin(ky * y + ph[1]) * np.sin(kz * z + ph[2])
+        kx, ky, kz = (int(t) for t in rng.integers(1, 4, size=3))
+        a = float(rng.uniform(0.5, 1.0))
+        ph = [float(t) for t in rng.uniform(0, 2 * math.pi, size=3)]
+        out += a * xp.sin(kx * x + ph[0]) * xp.sin(ky * y + ph[1]) * xp.sin(kz * z + ph[2])
         tot += a
     return out / tot
 

@@ -1,0 +1,307 @@
+"""GPU parity: the CUDA path (through the C ABI) against the CPU oracle on the
+same seeded inputs.  Tolerances (north_star, DESIGN.md sec. 3 reading 17):
+  metrics      <= 1e-13 relative (same D6 formula, FMA contraction only)
+  fill         bitwise
+  RHS          <= 1e-11 relative L_inf per component (floor: flux scale)
+  100 RK steps <= 1e-9  relative L_inf per component
+  decomposition (n blocks vs 1 block on the GPU) bitwise
+"""
+import math
+
+import numpy as np
+import pytest
+
+import oracle
+import synth
+from _harness import Problem, block_slices, flux_scale, inner, rel_linf
+
+pytestmark = pytest.mark.gpu
+
+PER = ((0, 0),) * 3
+P, E, D, W = 0, 1, 2, 3
+
+
+def _torch_cuda():
+    torch = pytest.importorskip("torch")
+    if not torch.cuda.is_available():
+        pytest.fail("GPU test run without a CUDA device")
+    return torch
+
+
+@pytest.fixture(autouse=True)
+def _need_gpu():
+    _torch_cuda()
+
+
+def wavy_random(n, seed=0, phys=None, amp=0.2):
+    g = synth.Wavy3D(L=(10.0,) * 3, N=n)
+    return Problem(n, g, PER, synth.random_state(n, seed=seed, amp=amp),
+                   phys or dict(terms=3, mu_ref=0.02))
+
+
+# ------------------------------------------------------------------ library identity
+
+def test_native_library_loaded():
+    from paper_conf_ipps_davissngmb23_b200 import crocco as cc
+    L = cc.lib()
+    assert L._name.endswith("libcrocco.so")
+    assert "sm_100a" in cc.crocco_version()
+
+
+# ------------------------------------------------------------------ metrics
+
+@pytest.mark.parametrize("nb", [(1, 1, 1), (2, 3, 1)])
+def test_metrics_parity(nb):
+    n = (26, 21, 13)
+    pb = wavy_random(n, 1)
+    xyz, met, U = pb.oracle_inputs()
+    S = pb.solver(nb)
+    got = [S.view(m, b, 10).cpu().numpy() for b, m in enumerate(S.met)]
+    ref = inner(met)
+    glob = pb.gather(S, got)
+    assert rel_linf(glob[1:], ref[1:]) < 1e-13
+    assert rel_linf(glob[:1], ref[:1]) < 1e-13
+    # ghost metrics: periodic copies from the owners -> equal the wrapped global values
+    bn, blocks = block_slices(n, nb)
+    Gw = np.pad(ref, ((0, 0),) + ((4, 4),) * 3, mode="wrap")
+    for (o, _), a in zip(blocks, got):
+        sl = (slice(None), slice(o[2], o[2] + bn[2] + 8), slice(o[1], o[1] + bn[1] + 8),
+              slice(o[0], o[0] + bn[0] + 8))
+        assert rel_linf(a, Gw[sl]) < 1e-13
+    S.close()
+
+
+# ------------------------------------------------------------------ fill
+
+@pytest.mark.parametrize("bc,nb", [
+    (PER, (1, 1, 1)),
+    (PER, (2, 2, 2)),
+    (((E, E), (W, E), (P, P)), (2, 2, 2)),
+    (((D, W), (E, D), (W, W)), (1, 2, 3)),
+])
+def test_fill_bitwise(bc, nb):
+    n = (16, 12, 18)
+    rng = np.random.default_rng(3)
+    dv = rng.uniform(0.5, 2.0, (3, 2, 5))
+    pb = Problem(n, synth.Cartesian(h=(0.1,) * 3), bc, synth.random_state(n, seed=4),
+                 dict(terms=3), dirichlet=dv)
+    _, _, Uref = pb.oracle_inputs()
+    S = pb.solver(nb)
+    S.fill()
+    bn, blocks = block_slices(n, nb)
+    for b, (o, _) in enumerate(blocks):
+        got = S.view(S.U[b], b, 5).cpu().numpy()
+        ref = Uref[:, o[2]:o[2] + bn[2] + 8, o[1]:o[1] + bn[1] + 8, o[0]:o[0] + bn[0] + 8]
+        assert np.array_equal(got, ref), f"block {b}"
+    S.close()
+
+
+# ------------------------------------------------------------------ RHS
+
+def _rhs_parity(pb, nb=(1, 1, 1)):
+    xyz, met, U = pb.oracle_inputs()
+    ref = inner(oracle.rhs(pb.n, pb.oracle_phys(), U, met))
+    S = pb.solver(nb)
+    S.fill()
+    r = S.rhs()
+    got = pb.gather(S, S.get(r))
+    S.close()
+    return rel_linf(got, ref, flux_scale(U, met)), got, ref
+
+
+@pytest.mark.parametrize("terms,mask", [(1, 1), (1, 2), (1, 4), (1, 7), (2, 7), (3, 7)])
+def test_rhs_parity_terms(terms, mask):
+    n = (37, 29, 23)   # ragged w.r.t. every thread-block tile
+    pb = wavy_random(n, 2, dict(terms=terms, dir_mask=mask, mu_ref=0.02))
+    err, _, _ = _rhs_parity(pb)
+    assert err < 1e-11, err
+
+
+def test_rhs_parity_sutherland_multiblock():
+    n = (40, 24, 16)
+    pb = wavy_random(n, 5, dict(terms=3, mu_law=1, mu_ref=0.03, T_ref=1.0, S=0.4, Pr=0.71))
+    err, _, _ = _rhs_parity(pb, (2, 2, 2))
+    assert err < 1e-11, err
+
+
+def test_rhs_parity_sod():
+    c = synth.case("sod")
+    xyz = c.grid.coords(c.n_global, (0, 0, 0), oracle.GC)
+    pb = Problem(c.n_global, c.grid, c.bc, synth.sod(xyz), c.phys)
+    err, _, _ = _rhs_parity(pb)
+    assert err < 1e-11, err
+
+
+def test_rhs_parity_ramp_downscaled_walls():
+    c = synth.case("ramp", scale=16)          # 64 x 32 x 16, 2x2x2 blocks
+    xyz = c.grid.coords(c.n_global, (0, 0, 0), oracle.GC)
+    pb = Problem(c.n_global, c.grid, c.bc, synth.ramp_state(xyz, c.grid), c.phys)
+    err, _, _ = _rhs_parity(pb, c.n_blocks)
+    assert err < 1e-11, err
+
+
+def test_rhs_parity_vortex_and_tgv():
+    for name, scale in (("vortex", 2), ("tgv", 8)):
+        c = synth.case(name, scale=scale)
+        xyz = c.grid.coords(c.n_global, (0, 0, 0), oracle.GC)
+        _, U = synth.block_inputs(c, (0, 0, 0), c.n_global)
+        pb = Problem(c.n_global, c.grid, c.bc, U, c.phys)
+        err, _, _ = _rhs_parity(pb)
+        assert err < 1e-11, (name, err)
+
+
+def test_rhs_minimum_block_size_and_edge_bcs():
+    n = (4, 8, 4)       # blocks of exactly 4 points (= ghost width)
+    dv = np.tile(synth.prim_to_cons(1.1, 0.2, -0.1, 0.05, 0.9).reshape(1, 1, 5), (3, 2, 1))
+    pb = Problem(n, synth.Cartesian(h=(0.2, 0.1, 0.3)), ((D, W), (P, P), (E, W)),
+                 synth.random_state(n, seed=9), dict(terms=3, mu_ref=0.05), dirichlet=dv)
+    err, _, _ = _rhs_parity(pb, (1, 2, 1))
+    assert err < 1e-11, err
+
+
+def test_gpu_free_stream_and_conservation():
+    n = (24, 20, 16)
+    g = synth.Wavy3D(L=(10.0,) * 3, N=n)
+    xyz = g.coords(n, (0, 0, 0), oracle.GC)
+    pb = Problem(n, g, PER, synth.free_stream(xyz), dict(terms=3, mu_ref=0.05))
+    _, met, U = pb.oracle_inputs()
+    S = pb.solver((2, 1, 2))
+    S.fill()
+    got = pb.gather(S, S.get(S.rhs()))
+    assert np.abs(got).max() < 1e-13 * flux_scale(U, met)
+    S.close()
+    pb = wavy_random(n, 11)
+    _, met, U = pb.oracle_inputs()
+    S = pb.solver()
+    S.fill()
+    r = pb.gather(S, S.get(S.rhs()))
+    J = inner(met)[0]
+    tot = (r / J).reshape(5, -1).sum(1)
+    mag = np.abs(r / J).reshape(5, -1).sum(1)
+    assert np.all(np.abs(tot) < 1e-13 * mag)
+    S.close()
+
+
+# ------------------------------------------------------------------ decomposition invariance
+
+def test_decomposition_invariance_bitwise():
+    n = (32, 24, 16)
+    pb = wavy_random(n, 13, dict(terms=3, mu_law=1, mu_ref=0.02, S=0.3))
+    outs = []
+    for nb in [(1, 1, 1), (2, 2, 2), (4, 1, 2)]:
+        S = pb.solver(nb)
+        S.fill()
+        r1 = pb.gather(S, S.get(S.rhs()))
+        S.step(1e-3, 2)
+        u = pb.gather(S, S.get(S.U))
+        outs.append((r1, u))
+        S.close()
+    for r1, u in outs[1:]:
+        assert np.array_equal(r1, outs[0][0])
+        assert np.array_equal(u, outs[0][1])
+
+
+# ------------------------------------------------------------------ RK
+
+def test_rk_update_parity():
+    n = (20, 10, 6)
+    pb = wavy_random(n, 17)
+    S = pb.solver()
+    rng = np.random.default_rng(1)
+    torch = _torch_cuda()
+    arrs = [rng.normal(size=(5, n[2] + 8, n[1] + 8, n[0] + 8)) for _ in range(3)]
+    Uin, dU, rhs = [a.copy() for a in arrs]
+    bufs = [S._alloc(S.layouts[0], 5) for _ in range(4)]
+    for t, a in zip(bufs[:3], (Uin, dU, rhs)):
+        S.view(t, 0, 5).copy_(torch.from_numpy(a))
+    from paper_conf_ipps_davissngmb23_b200 import crocco as cc
+    for stage in range(3):
+        Uo = np.zeros_like(Uin)
+        dUo = dU.copy()
+        oracle.rk_update(n, stage, 0.013, Uin, Uo, dUo, rhs)
+        cc.crocco_rk_update(S.ctx, stage, 0.013, [bufs[0].data_ptr()], [bufs[3].data_ptr()],
+                            [bufs[1].data_ptr()], [bufs[2].data_ptr()])
+        S.sync()
+        gU = S.view(bufs[3], 0, 5).cpu().numpy()
+        gd = S.view(bufs[1], 0, 5).cpu().numpy()
+        assert rel_linf(inner(gU), inner(Uo)) < 1e-15
+        assert rel_linf(inner(gd), inner(dUo)) < 1e-15
+        dU = dUo
+        S.view(bufs[1], 0, 5).copy_(torch.from_numpy(dU))
+    S.close()
+
+
+@pytest.mark.parametrize("name", ["sod", "vortex"])
+def test_rk3_100_steps_parity(name):
+    if name == "sod":
+        c = synth.case("sod")
+        xyz = c.grid.coords(c.n_global, (0, 0, 0), oracle.GC)
+        U0 = synth.sod(xyz)
+        n, dt = c.n_global, c.dt
+    else:
+        n = (24, 24, 24)
+        c = synth.case("vortex")
+        c.grid = synth.Wavy3D(L=(10.0,) * 3, N=n)
+        xyz = c.grid.coords(n, (0, 0, 0), oracle.GC)
+        U0 = synth.vortex(xyz)
+        dt = 0.01
+    pb = Problem(n, c.grid, c.bc, U0, c.phys)
+    _, met, U = pb.oracle_inputs()
+    oracle.advance(n, c.bc, pb.oracle_phys(), dt, 100, U, met)
+    S = pb.solver()
+    S.step(dt, 100)
+    S.sync()
+    got = pb.gather(S, S.get(S.U))
+    S.close()
+    assert rel_linf(got, inner(U)) < 1e-9
+
+
+# ------------------------------------------------------------------ full size, sampled
+
+@pytest.mark.slow
+def test_full_size_weak_config_sampled():
+    """512^3 weak-scaling config, rk_stage in bench.py's launch configuration;
+    64 sampled points recomputed by the oracle one by one from the GPU's
+    filled neighbourhood (9^3 window of U and metrics)."""
+    torch = _torch_cuda()
+    c = synth.case("weak")
+    n = c.n_global
+    from paper_conf_ipps_davissngmb23_b200 import crocco as cc
+    from paper_conf_ipps_davissngmb23_b200.solver import Solver
+    S = Solver(n, c.n_blocks, c.bc, cc.make_phys(**c.phys))
+    xyz, U0 = synth.block_inputs(c, (0, 0, 0), n)
+    S.set_coords([xyz])
+    S.set_state([U0])
+    del xyz, U0
+    rng = np.random.default_rng(0)
+    pts = [tuple(rng.integers(0, m) for m in n) for _ in range(56)]
+    pts += [(0, 0, 0), (n[0] - 1, n[1] - 1, n[2] - 1), (0, n[1] - 1, 3), (n[0] - 1, 0, n[2] - 1),
+            (1, 2, n[2] - 2), (n[0] - 2, 5, 0), (255, 0, 511), (511, 256, 0)]
+    ph = oracle.phys(**c.phys)
+    for stage in (0, 1):
+        Uin_buf, dU_buf = S.U[0], S.dU[0]
+        dU_before = {p: S.view(dU_buf, 0, 5)[:, p[2] + 4, p[1] + 4, p[0] + 4].cpu().numpy()
+                     for p in pts}
+        S.stage(stage, c.dt)
+        S.sync()
+        Uin = S.view(Uin_buf, 0, 5)
+        Uout = S.view(S.U[0], 0, 5)
+        dUv = S.view(dU_buf, 0, 5)
+        M = S.view(S.met[0], 0, 10)
+        worst = 0.0
+        for p in pts:
+            sl = (slice(None), slice(p[2], p[2] + 9), slice(p[1], p[1] + 9), slice(p[0], p[0] + 9))
+            Uw = np.ascontiguousarray(Uin[sl].cpu().numpy())
+            Mw = np.ascontiguousarray(M[sl].cpu().numpy())
+            r = oracle.rhs((1, 1, 1), ph, Uw, Mw)
+            Uo = np.zeros_like(Uw)
+            dUo = np.zeros_like(Uw)
+            dUo[:, 4, 4, 4] = dU_before[p]
+            oracle.rk_update((1, 1, 1), stage, c.dt, Uw, Uo, dUo, r)
+            gU = Uout[:, p[2] + 4, p[1] + 4, p[0] + 4].cpu().numpy()
+            gd = dUv[:, p[2] + 4, p[1] + 4, p[0] + 4].cpu().numpy()
+            scale = flux_scale(Uw, Mw) * c.dt
+            worst = max(worst, float(np.abs(gd - dUo[:, 4, 4, 4]).max() / max(np.abs(dUo[:, 4, 4, 4]).max(), scale)))
+            worst = max(worst, float(np.abs(gU - Uo[:, 4, 4, 4]).max() / np.abs(Uo[:, 4, 4, 4]).max()))
+        assert worst < 1e-11, (stage, worst)
+    S.close()

@@ -240,7 +240,7 @@ class _Affine:
 
     def coords(self, n, origin=(0, 0, 0), g=10):
         I, J, K = synth._index_grids(n, origin, g)
-        X = np.stack([I, J, K])
+        X = synth._stack3(I, J, K)
         return np.einsum("ad,d...->a...", self.A, X) + self.b[:, None, None, None]
 
 
@@ -261,7 +261,7 @@ def test_metrics_affine_exact():
 def test_metrics_sixth_order_vs_analytic():
     # wavy map: analytic d xi/d x via numpy.linalg.inv of the analytic Jacobian
     def analytic(grid, n):
-        I, J, K = synth._index_grids(n, (0, 0, 0), 4)
+        I, J, K = np.broadcast_arrays(*synth._index_grids(n, (0, 0, 0), 4))
         h = grid.L[0] / grid.N[0]
         xi, et, ze = I * h, J * h, K * h
         k, A = grid.k, grid.A
