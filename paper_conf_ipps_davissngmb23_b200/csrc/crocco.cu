@@ -189,7 +189,7 @@ static crocco_status validate(const crocco_grid_desc *d, int nb[3], int bn[3]) {
         int64_t b = d->n_global[a] / nb[a];
         if (b < G) return fail(nullptr, CROCCO_ERR_ARG, "block interior %lld < ghost width 4 in direction %d",
                                (long long)b, a);
-        if (b > (1 << 20)) return fail(nullptr, CROCCO_ERR_ARG, "block too large");
+        if (b > 65535) return fail(nullptr, CROCCO_ERR_ARG, "block interior > 65535 points in direction %d", a);
         bn[a] = (int)b;
         for (int s = 0; s < 2; s++)
             if (d->bc[a][s] < 0 || d->bc[a][s] > 3)
@@ -723,13 +723,13 @@ static crocco_status rhs_parts(crocco_ctx c, const LocalBlock &b, const double *
         }
         if (ph.dir_mask & 2) {
             dim3 blk(32, 4);
-            dim3 grd(cdiv(b.g.n[0], 32), cdiv((int64_t)(b.g.n[1] + 1) * b.g.n[2], 4));
+            dim3 grd(cdiv((int64_t)(b.g.n[1] + 1) * b.g.n[2], 4), cdiv(b.g.n[0], 32));
             LAUNCH(c, K_FLUX_Y,
                    k_flux<1><<<grd, blk, 0, c->stream>>>(U, b.prim, M, b.flux[1], b.fcs[1], b.L, ph));
         }
         if (ph.dir_mask & 4) {
             dim3 blk(32, 4);
-            dim3 grd(cdiv(b.g.n[0], 32), cdiv((int64_t)b.g.n[1] * (b.g.n[2] + 1), 4));
+            dim3 grd(cdiv((int64_t)b.g.n[1] * (b.g.n[2] + 1), 4), cdiv(b.g.n[0], 32));
             LAUNCH(c, K_FLUX_Z,
                    k_flux<2><<<grd, blk, 0, c->stream>>>(U, b.prim, M, b.flux[2], b.fcs[2], b.L, ph));
         }

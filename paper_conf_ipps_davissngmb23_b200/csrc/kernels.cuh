@@ -289,8 +289,8 @@ __global__ void __launch_bounds__(128) k_flux(const double *__restrict__ U,
         i = e - 1;
         out = t;
     } else if (D == 1) {
-        i = blockIdx.x * blockDim.x + threadIdx.x;
-        const int64_t y = (int64_t)blockIdx.y * blockDim.y + threadIdx.y;
+        i = blockIdx.y * blockDim.x + threadIdx.x;
+        const int64_t y = (int64_t)blockIdx.x * blockDim.y + threadIdx.y;
         const int ne = L.n1 + 1;
         if (i >= L.n0 || y >= (int64_t)ne * L.n2) return;
         const int e = (int)(y % ne);
@@ -298,8 +298,8 @@ __global__ void __launch_bounds__(128) k_flux(const double *__restrict__ U,
         j = e - 1;
         out = i + (int64_t)L.n0 * y;
     } else {
-        i = blockIdx.x * blockDim.x + threadIdx.x;
-        const int64_t y = (int64_t)blockIdx.y * blockDim.y + threadIdx.y;
+        i = blockIdx.y * blockDim.x + threadIdx.x;
+        const int64_t y = (int64_t)blockIdx.x * blockDim.y + threadIdx.y;
         if (i >= L.n0 || y >= (int64_t)L.n1 * (L.n2 + 1)) return;
         j = (int)(y % L.n1);
         const int e = (int)(y / L.n1);

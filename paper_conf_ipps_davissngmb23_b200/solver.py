@@ -19,7 +19,11 @@ class Solver:
                  rank=0, nranks=1, block_rank=None, device=None, stream=None, nccl_unique_id=None):
         if not torch.cuda.is_available():
             raise RuntimeError("libcrocco needs a CUDA device (no CPU fallback)")
-        self.device = torch.device(device if device is not None else "cuda")
+        if device is None:
+            device = torch.device("cuda", torch.cuda.current_device())
+        self.device = torch.device(device)
+        if self.device.index is None:
+            self.device = torch.device("cuda", torch.cuda.current_device())
         torch.cuda.set_device(self.device)
         self.stream = stream if stream is not None else torch.cuda.current_stream(self.device)
         self.phys = phys if phys is not None else cc.make_phys()

@@ -42,6 +42,17 @@ def flux_scale(U, met, gamma=1.4):
     return float((J * m * F).max())
 
 
+def state_scale(Ui, gamma=1.4):
+    """max_i rho_i (|u_i| + c_i): the momentum scale used as the parity floor for
+    state comparisons where a component is identically ~0 (e.g. transverse
+    momentum of the 1-D Sod problem)."""
+    rho = Ui[0]
+    vel = Ui[1:4] / rho
+    p = (gamma - 1) * (Ui[4] - 0.5 * rho * (vel ** 2).sum(0))
+    c = np.sqrt(np.abs(gamma * p / rho))
+    return float((rho * (np.sqrt((vel ** 2).sum(0)) + c)).max())
+
+
 def rel_linf(got, ref, floor=0.0):
     """Per component max|got-ref| / max(max|ref|, floor); returns the max over components."""
     got = np.asarray(got)
