@@ -33,8 +33,9 @@ METRIC = "grid-point RK-stage updates/sec (fp64) at 1/2/4/8 B200; % HBM roofline
 UNIT = "point-stages/s"
 N_BLOCK = 512
 # FP64 operations of one characteristic-WENO interface flux:
-# DADD + DMUL + 2*DFMA counted by ncu on k_flux (profiles/), per interface.
-FLUX_FLOPS_PER_IFACE = float(os.environ.get("CROCCO_FLUX_FLOPS", "2478"))
+# hand count of the v1 formulation (FMA = 2, div/sqrt = 1), frozen as the unit of work;
+# ncu executed DADD+DMUL+2*DFMA on v1 = 1951 per interface (profiles/r01_ncu.md).
+FLUX_FLOPS_PER_IFACE = float(os.environ.get("CROCCO_FLUX_FLOPS", "1924"))
 # B200 FP64 (non-tensor) peak: 148 SMs x 64 FMA/clk x 2 flop x 1.965 GHz
 FP64_PEAK_TFLOPS = 148 * 64 * 2 * 1.965e9 / 1e12
 # compulsory HBM bytes per point-stage of a fused stage: 240 (200 at stage 0)

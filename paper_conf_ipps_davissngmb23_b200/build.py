@@ -31,21 +31,24 @@ def needs_build() -> bool:
     return any(os.path.getmtime(p) > t for p in DEPS)
 
 
-def build(force: bool = False, verbose: bool = False) -> str:
-    if not force and not needs_build():
+def build(force: bool = False, verbose: bool = False, defines=(), out: str | None = None) -> str:
+    """Compile libcrocco.so; ``defines``/``out`` build tuning variants (tools/)."""
+    target = out or LIB
+    if not force and out is None and not needs_build():
         return LIB
     inc, lib = nccl_dirs()
     cmd = [NVCC, "-O3", "-std=c++17", "-gencode", "arch=compute_100a,code=sm_100a", "-lineinfo",
            "-Xcompiler", "-fPIC", "-shared", "-fmad=true", "--expt-relaxed-constexpr",
            "-I", os.path.join(ROOT, "include"), "-I", inc,
-           "-o", LIB + ".tmp", *SRC,
+           *[f"-D{d}" for d in defines],
+           "-o", target + ".tmp", *SRC,
            "-L", lib, "-l:libnccl.so.2", "-Xlinker", "-rpath=" + lib, "-lcudart"]
     if verbose:
         cmd.insert(1, "-Xptxas=-v")
     print(" ".join(cmd), file=sys.stderr)
     subprocess.check_call(cmd)
-    os.replace(LIB + ".tmp", LIB)
-    return LIB
+    os.replace(target + ".tmp", target)
+    return target
 
 
 if __name__ == "__main__":

@@ -11,7 +11,7 @@ import ctypes as C
 import os
 
 HERE = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(HERE, "libcrocco.so")
+LIB_PATH = os.environ.get("CROCCO_LIB") or os.path.join(HERE, "libcrocco.so")  # env: variant builds (tools/)
 
 CROCCO_OK, CROCCO_ERR_ARG, CROCCO_ERR_CUDA, CROCCO_ERR_NCCL, CROCCO_ERR_NOMEM, CROCCO_ERR_STATE = range(6)
 BC_PERIODIC, BC_EXTRAP, BC_DIRICHLET, BC_WALL = 0, 1, 2, 3

@@ -89,10 +89,19 @@ __device__ __forceinline__ double weno_symbo(double v0, double v1, double v2, do
 // ---------------------------------------------------------------------------
 enum { PU = 0, PV = 1, PW = 2, PP = 3, PC = 4, PSR = 5, PH = 6, PT = 7, NPRIM = 8 };
 
+#ifndef CROCCO_FLUX_MINB
+#define CROCCO_FLUX_MINB 1   // min resident CTAs/SM for k_flux (register cap)
+#endif
+#ifndef CROCCO_FLUX_USMEM
+#define CROCCO_FLUX_USMEM 0  // 1: keep the 6x5 stencil states in shared memory, not registers
+#endif
+constexpr int FLUX_THREADS = 128;
+
 __device__ __forceinline__ void iface_flux(const double *__restrict__ U,
                                            const double *__restrict__ Pm,
                                            const double *__restrict__ M, int64_t cs, int64_t p0,
-                                           int64_t s, int d, const Phys &ph, double F[5]) {
+                                           int64_t s, int d, const Phys &ph, double F[5],
+                                           double *Us) {
     const double gm1 = ph.gm1;
     // frozen interface metric (reading 6): R6 = (1,-8,37,37,-8,1)/60
     const double *Md = M + (int64_t)(1 + 3 * d) * cs;
@@ -130,13 +139,19 @@ __device__ __forceinline__ void iface_flux(const double *__restrict__ U,
     const double beta = irt * ict * SQ12;  // 1/(sqrt2 rho c)
 
     // stencil points: state, normal velocity, pressure; LLF speeds
-    double Ul[6][5], th[6], pl[6];
+#if CROCCO_FLUX_USMEM
+#define UL(l, c) Us[((l) * 5 + (c)) * FLUX_THREADS]
+#else
+    double Ul[6][5];
+#define UL(l, c) Ul[l][c]
+#endif
+    double th[6], pl[6];
     double lam0 = 0.0, lam3 = 0.0, lam4 = 0.0;
 #pragma unroll
     for (int l = 0; l < 6; l++) {
         const int64_t q = p0 + l * s;
 #pragma unroll
-        for (int c = 0; c < 5; c++) Ul[l][c] = U[c * cs + q];
+        for (int c = 0; c < 5; c++) UL(l, c) = U[c * cs + q];
         const double t = nx * Pm[PU * cs + q] + ny * Pm[PV * cs + q] + nz * Pm[PW * cs + q];
         const double cl = Pm[PC * cs + q];
         th[l] = t;
@@ -213,8 +228,8 @@ __device__ __forceinline__ void iface_flux(const double *__restrict__ U,
         const double hl = 0.5 * lam;
 #pragma unroll
         for (int l = 0; l < 6; l++) {
-            const double w = L0 * Ul[l][0] + L1 * Ul[l][1] + L2 * Ul[l][2] + L3 * Ul[l][3] +
-                             L4 * Ul[l][4];
+            const double w = L0 * UL(l, 0) + L1 * UL(l, 1) + L2 * UL(l, 2) + L3 * UL(l, 3) +
+                             L4 * UL(l, 4);
             const double g = th[l] * w + pl[l] * (kA + kB * th[l]);
             gp[l] = 0.5 * g + hl * w;
             gm[l] = 0.5 * g - hl * w;
@@ -271,7 +286,7 @@ __global__ void __launch_bounds__(256) k_prims(const double *__restrict__ U, dou
 // of the interior lines; written to Fd[c][interface index] (WENOx/y/z,
 // PAPER.md:110-112).  Each interface is computed exactly once.
 template <int D>
-__global__ void __launch_bounds__(128) k_flux(const double *__restrict__ U,
+__global__ void __launch_bounds__(FLUX_THREADS, CROCCO_FLUX_MINB) k_flux(const double *__restrict__ U,
                                               const double *__restrict__ Pm,
                                               const double *__restrict__ M, double *__restrict__ Fd,
                                               int64_t fcs, Lay L, Phys ph) {
@@ -309,9 +324,16 @@ __global__ void __launch_bounds__(128) k_flux(const double *__restrict__ U,
     const int64_t s = (D == 0) ? 1 : (D == 1 ? L.py : L.pz);
     const int64_t p0 = at(L, i, j, k) - 2 * s;
     double F[5];
-    iface_flux(U, Pm, M, L.cs, p0, s, D, ph, F);
+#if CROCCO_FLUX_USMEM
+    __shared__ double sU[30 * FLUX_THREADS];
+    double *Us = sU + threadIdx.x + blockDim.x * threadIdx.y;
+#else
+    double *Us = nullptr;
+#endif
+    iface_flux(U, Pm, M, L.cs, p0, s, D, ph, F, Us);
 #pragma unroll
     for (int c = 0; c < 5; c++) Fd[c * fcs + out] = F[c];
+#undef UL
 }
 
 // Viscous and heat point fluxes F^_v^d (reading 12) on the

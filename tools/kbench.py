@@ -1,0 +1,29 @@
+"""Kernel-variant micro-benchmark: per-kernel-class CUDA-event times of RK stages on
+the bench workload (CROCCO_LIB selects a variant .so).  Not a bench.py number."""
+import json, math, os, sys, time
+sys.path.insert(0, os.getcwd())
+import torch
+import synth
+from paper_conf_ipps_davissngmb23_b200 import crocco as cc
+from paper_conf_ipps_davissngmb23_b200.solver import Solver
+N = int(os.environ.get("KB_N", "512"))
+n = (N, N, N)
+grid = synth.Wavy3D(L=(2 * math.pi,) * 3, N=n, x0=(-math.pi,) * 3, k=2.0, A=0.15)
+S = Solver(n, (1, 1, 1), ((0, 0),) * 3, cc.make_phys(gamma=1.4, R=1.0, Pr=0.71, mu_ref=1 / 1600, terms=3))
+xyz = torch.from_numpy(grid.coords(n, (0, 0, 0), 10)).cuda()
+S.set_coords([xyz]); S.set_state([synth.tgv(xyz, noise=0.01, seed=5)]); del xyz
+for s in range(3): S.stage(s, 2e-4)
+torch.cuda.synchronize()
+cc.crocco_set_timing(S.ctx, True); cc.crocco_kernel_times(S.ctx)
+e0 = torch.cuda.Event(enable_timing=True); e1 = torch.cuda.Event(enable_timing=True)
+e0.record()
+for it in range(2):
+    for s in range(3): S.stage(s, 2e-4)
+e1.record(); torch.cuda.synchronize()
+kt = cc.crocco_kernel_times(S.ctx)
+tot = e0.elapsed_time(e1) / 6
+out = {"lib": os.path.basename(cc.LIB_PATH), "ms_per_stage": tot, "pts_stage_per_s": N ** 3 / tot * 1e3,
+       "kernels_ms": {k: round(v[1] / max(v[0], 1), 3) for k, v in kt.items() if v[0]}}
+U = S.view(S.U[0], 0, 5)[:, 4:-4, 4:-4, 4:-4]
+out["finite"] = bool(torch.isfinite(U).all().item())
+print(json.dumps(out), flush=True)
