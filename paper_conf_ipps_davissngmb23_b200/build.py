@@ -6,6 +6,7 @@ the ones bundled with torch (nvidia-nccl-cu12 2.28.9); the rpath points at them.
 """
 from __future__ import annotations
 
+import glob
 import os
 import subprocess
 import sys
@@ -13,7 +14,7 @@ import sys
 HERE = os.path.dirname(os.path.abspath(__file__))
 ROOT = os.path.dirname(HERE)
 SRC = [os.path.join(HERE, "csrc", "crocco.cu")]
-DEPS = SRC + [os.path.join(HERE, "csrc", "kernels.cuh"), os.path.join(ROOT, "include", "crocco.h")]
+DEPS = SRC + sorted(glob.glob(os.path.join(HERE, "csrc", "*.cuh"))) + [os.path.join(ROOT, "include", "crocco.h")]
 LIB = os.path.join(HERE, "libcrocco.so")
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
 

@@ -1,7 +1,7 @@
 // crocco.cu -- host side of libcrocco.so: the C ABI of include/crocco.h.
 //
 // Block decomposition, ghost-exchange plan, scratch management, launch
-// orchestration of the sm_100a kernels in kernels.cuh, NCCL halo exchange.
+// orchestration of the sm_100a kernels (sweep/pointwise/fill/metrics .cuh), NCCL halo exchange.
 // Algorithm 1/2 of the paper is the call order; every
 // numerical step runs in the CUDA kernels, never on the host.
 #include <cuda_runtime.h>
@@ -15,7 +15,10 @@
 #include <vector>
 
 #include "../../include/crocco.h"
-#include "kernels.cuh"
+#include "fill.cuh"
+#include "metrics.cuh"
+#include "pointwise.cuh"
+#include "sweep.cuh"
 
 using namespace crocco;
 
@@ -37,15 +40,14 @@ struct LocalBlock {
     Lay C;       // coordinate layout
     VLay V;      // viscous-flux box
     double *prim = nullptr;
-    double *flux[3] = {nullptr, nullptr, nullptr};
-    int64_t fcs[3] = {0, 0, 0};
+    double *racc = nullptr;  // RHS accumulator R (5 comps, compact interior)
+    int64_t rcs = 0;
     double *fv = nullptr;
 };
 
-enum { K_PRIMS = 0, K_FLUX_X, K_FLUX_Y, K_FLUX_Z, K_VISC, K_ASSEMBLE, K_UPDATE, K_FILL, K_METRICS,
-       K_NCLASS };
-const char *k_names[K_NCLASS] = {"prims", "flux_xi", "flux_eta", "flux_zeta", "viscous",
-                                 "assemble_update", "update", "fill", "metrics"};
+enum { K_PRIMS = 0, K_FLUX_X, K_FLUX_Y, K_FLUX_Z, K_VISC, K_UPDATE, K_FILL, K_METRICS, K_NCLASS };
+const char *k_names[K_NCLASS] = {"prims", "sweep_xi", "sweep_eta", "sweep_zeta_update", "viscous",
+                                 "update", "fill", "metrics"};
 
 struct TimedLaunch {
     int cls;
@@ -284,6 +286,25 @@ static void build_plan(const crocco_grid_desc *d, const int nb[3], const int bn[
     }
 }
 
+#ifndef CROCCO_SWEEP_SMEM
+#define CROCCO_SWEEP_SMEM 1  // shared-memory staged sweeps (k_sweep_s); 0: global-load sweeps
+#endif
+template <int D>
+static constexpr size_t sweep_smem_bytes() {
+    return (size_t)(SWEEP_THREADS / 32) * RingGeom<D>::PER_WARP * sizeof(double);
+}
+static cudaError_t sweep_attrs() {
+    cudaError_t e = cudaFuncSetAttribute(k_sweep_s<0>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                         (int)sweep_smem_bytes<0>());
+    if (e == cudaSuccess)
+        e = cudaFuncSetAttribute(k_sweep_s<1>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                 (int)sweep_smem_bytes<1>());
+    if (e == cudaSuccess)
+        e = cudaFuncSetAttribute(k_sweep_s<2>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                 (int)sweep_smem_bytes<2>());
+    return e;
+}
+
 // ---------------------------------------------------------------------------
 // ABI
 // ---------------------------------------------------------------------------
@@ -362,7 +383,7 @@ crocco_status crocco_set_phys(crocco_ctx c, const crocco_phys *p) {
 static void free_ctx(crocco_ctx c) {
     for (auto &b : c->loc) {
         cudaFree(b.prim);
-        for (int d = 0; d < 3; d++) cudaFree(b.flux[d]);
+        cudaFree(b.racc);
         cudaFree(b.fv);
     }
     cudaFree(c->send_stage);
@@ -409,7 +430,9 @@ crocco_status crocco_init_grid(const crocco_grid_desc *desc, const crocco_phys *
         lb.V.b0 = g.n[0] + 4;
         lb.V.b1 = g.n[1] + 4;
         lb.V.b2 = g.n[2] + 4;
-        lb.V.cs = rup((int64_t)lb.V.b0 * lb.V.b1 * lb.V.b2, 32);
+        lb.V.py = rup(lb.V.b0, 16);
+        lb.V.pz = lb.V.py * lb.V.b1;
+        lb.V.cs = rup(lb.V.pz * lb.V.b2, 32);
         c->gid_to_local[g.gid] = (int)c->loc.size();
         c->loc.push_back(lb);
     }
@@ -423,15 +446,20 @@ crocco_status crocco_init_grid(const crocco_grid_desc *desc, const crocco_phys *
     };
     for (auto &b : c->loc) {
         bool ok = alloc(&b.prim, NPRIM * b.L.cs);
-        b.fcs[0] = rup((int64_t)(b.g.n[0] + 1) * b.g.n[1] * b.g.n[2], 32);
-        b.fcs[1] = rup((int64_t)b.g.n[0] * (b.g.n[1] + 1) * b.g.n[2], 32);
-        b.fcs[2] = rup((int64_t)b.g.n[0] * b.g.n[1] * (b.g.n[2] + 1), 32);
-        for (int d = 0; d < 3; d++) ok = ok && alloc(&b.flux[d], 5 * b.fcs[d]);
+        b.rcs = rup((int64_t)b.g.n[0] * b.g.n[1] * b.g.n[2], 32);
+        ok = ok && alloc(&b.racc, 5 * b.rcs);
         ok = ok && alloc(&b.fv, 12 * b.V.cs);
         if (!ok) {
             cudaGetLastError();
             free_ctx(c);
             return fail(nullptr, CROCCO_ERR_NOMEM, "device scratch allocation failed");
+        }
+    }
+    {
+        cudaError_t e = sweep_attrs();
+        if (e != cudaSuccess) {
+            free_ctx(c);
+            return fail(nullptr, CROCCO_ERR_CUDA, "cudaFuncSetAttribute: %s", cudaGetErrorString(e));
         }
     }
     // NCCL communicator + staging for remote halo messages
@@ -711,49 +739,69 @@ crocco_status crocco_init_metrics(crocco_ctx c, double *const *xyz, double *cons
 // ---------------------------------------------------------------------------
 // RHS / RK
 // ---------------------------------------------------------------------------
-static crocco_status rhs_parts(crocco_ctx c, const LocalBlock &b, const double *U, const double *M) {
+static const double RK_A[3] = {0.0, -5.0 / 9.0, -153.0 / 128.0};
+static const double RK_B[3] = {1.0 / 3.0, 15.0 / 16.0, 8.0 / 15.0};
+
+// One RHS evaluation of a block (Alg. 2 l.5-9): primitives, viscous point
+// fluxes, then the xi / eta / zeta sweeps; the zeta sweep finishes every point
+// (mode 2: rhs = J R, mode 3: Williamson update).
+static crocco_status rhs_block(crocco_ctx c, const LocalBlock &b, const double *U, const double *M,
+                               int final_mode, double *rhs, const double *Uin, double *Uout,
+                               double *dU, int stage, double dt) {
     const Phys &ph = c->ph;
+    const bool inviscid = (ph.terms & CROCCO_TERM_INVISCID) != 0;
+    const bool viscous = (ph.terms & CROCCO_TERM_VISCOUS) != 0;
     const int64_t np = (int64_t)(b.g.n[0] + 2 * G) * (b.g.n[1] + 2 * G) * (b.g.n[2] + 2 * G);
-    LAUNCH(c, K_PRIMS, k_prims<<<cdiv(np, 256), 256, 0, c->stream>>>(U, b.prim, b.L, ph));
-    if (ph.terms & CROCCO_TERM_INVISCID) {
-        if (ph.dir_mask & 1) {
-            const int64_t t = (int64_t)(b.g.n[0] + 1) * b.g.n[1] * b.g.n[2];
-            LAUNCH(c, K_FLUX_X,
-                   k_flux<0><<<cdiv(t, 128), 128, 0, c->stream>>>(U, b.prim, M, b.flux[0], b.fcs[0], b.L, ph));
-        }
-        if (ph.dir_mask & 2) {
-            dim3 blk(32, 4);
-            dim3 grd(cdiv((int64_t)(b.g.n[1] + 1) * b.g.n[2], 4), cdiv(b.g.n[0], 32));
-            LAUNCH(c, K_FLUX_Y,
-                   k_flux<1><<<grd, blk, 0, c->stream>>>(U, b.prim, M, b.flux[1], b.fcs[1], b.L, ph));
-        }
-        if (ph.dir_mask & 4) {
-            dim3 blk(32, 4);
-            dim3 grd(cdiv((int64_t)b.g.n[1] * (b.g.n[2] + 1), 4), cdiv(b.g.n[0], 32));
-            LAUNCH(c, K_FLUX_Z,
-                   k_flux<2><<<grd, blk, 0, c->stream>>>(U, b.prim, M, b.flux[2], b.fcs[2], b.L, ph));
-        }
-    }
-    if (ph.terms & CROCCO_TERM_VISCOUS) {
+    if (viscous || !CROCCO_SWEEP_SMEM)  // the staged sweeps compute their own primitives
+        LAUNCH(c, K_PRIMS, k_prims<<<cdiv(np, 256), 256, 0, c->stream>>>(U, b.prim, b.L, ph));
+    if (viscous) {
         const int64_t nv = (int64_t)b.V.b0 * b.V.b1 * b.V.b2;
         LAUNCH(c, K_VISC, k_visc<<<cdiv(nv, 256), 256, 0, c->stream>>>(b.prim, M, b.fv, b.L, b.V, ph));
     }
-    return CROCCO_OK;
-}
-
-static Asm make_asm(crocco_ctx c, const LocalBlock &b, const double *M) {
-    Asm a;
-    memset(&a, 0, sizeof a);
     for (int d = 0; d < 3; d++) {
-        a.F[d] = b.flux[d];
-        a.fcs[d] = b.fcs[d];
+        SweepArgs a;
+        memset(&a, 0, sizeof a);
+        a.in.U = U;
+        a.in.P = b.prim;
+        a.in.M = M;
+        a.in.FV = b.fv + (int64_t)4 * d * b.V.cs;
+        a.in.cs = b.L.cs;
+        a.in.vcs = b.V.cs;
+        a.V = b.V;
+        a.R = b.racc;
+        a.rcs = b.rcs;
+        a.inv = inviscid && (ph.dir_mask >> d & 1);
+        a.visc = viscous;
+        a.mode = d == 0 ? 0 : (d == 1 ? 1 : final_mode);
+        a.rhs = rhs;
+        a.Uin = Uin;
+        a.Uout = Uout;
+        a.dU = dU;
+        a.stage = stage;
+        a.A = RK_A[stage];
+        a.B = RK_B[stage];
+        a.dt = dt;
+        // warp tiles: xi 4 lines x 8 interfaces, eta/zeta 8 i x 4 interfaces; lines are
+        // marched whole unless that leaves too few warps for 148 SMs
+        const int64_t nd = b.g.n[d];
+        const int64_t lines = d == 0 ? ((int64_t)b.g.n[1] * b.g.n[2] + 3) / 4
+                                     : (int64_t)((b.g.n[0] + 7) / 8) * (d == 1 ? b.g.n[2] : b.g.n[1]);
+        int64_t seg = nd;
+        while (lines * ((nd + seg - 1) / seg) < 16384 && seg > 32) seg = (seg + 1) / 2;
+        a.seg = (int)seg;
+        const int64_t warps = lines * ((nd + seg - 1) / seg);
+        const unsigned grid = cdiv(warps * 32, SWEEP_THREADS);
+#if CROCCO_SWEEP_SMEM
+        if (d == 0) LAUNCH(c, K_FLUX_X, k_sweep_s<0><<<grid, SWEEP_THREADS, sweep_smem_bytes<0>(), c->stream>>>(a, b.L, ph));
+        else if (d == 1) LAUNCH(c, K_FLUX_Y, k_sweep_s<1><<<grid, SWEEP_THREADS, sweep_smem_bytes<1>(), c->stream>>>(a, b.L, ph));
+        else LAUNCH(c, K_FLUX_Z, k_sweep_s<2><<<grid, SWEEP_THREADS, sweep_smem_bytes<2>(), c->stream>>>(a, b.L, ph));
+#else
+        if (d == 0) LAUNCH(c, K_FLUX_X, k_sweep<0><<<grid, SWEEP_THREADS, 0, c->stream>>>(a, b.L, ph));
+        else if (d == 1) LAUNCH(c, K_FLUX_Y, k_sweep<1><<<grid, SWEEP_THREADS, 0, c->stream>>>(a, b.L, ph));
+        else LAUNCH(c, K_FLUX_Z, k_sweep<2><<<grid, SWEEP_THREADS, 0, c->stream>>>(a, b.L, ph));
+#endif
     }
-    a.FV = b.fv;
-    a.V = b.V;
-    a.M = M;
-    a.inv_mask = (c->ph.terms & CROCCO_TERM_INVISCID) ? (c->ph.dir_mask & 7) : 0;
-    a.visc = (c->ph.terms & CROCCO_TERM_VISCOUS) ? 1 : 0;
-    return a;
+    return CROCCO_OK;
 }
 
 crocco_status crocco_rhs(crocco_ctx c, double *const *U, double *const *M, double *const *rhs) {
@@ -765,19 +813,11 @@ crocco_status crocco_rhs(crocco_ctx c, double *const *U, double *const *M, doubl
     for (size_t bi = 0; bi < c->loc.size(); bi++)
         if (rhs[bi] == U[bi]) return fail(c, CROCCO_ERR_ARG, "rhs aliases U");
     for (size_t bi = 0; bi < c->loc.size(); bi++) {
-        const LocalBlock &b = c->loc[bi];
-        if ((st = rhs_parts(c, b, U[bi], M[bi]))) return st;
-        Asm a = make_asm(c, b, M[bi]);
-        a.mode = 0;
-        a.rhs = rhs[bi];
-        dim3 grd(cdiv(b.g.n[0], 128), b.g.n[1], b.g.n[2]);
-        LAUNCH(c, K_ASSEMBLE, k_assemble<<<grd, 128, 0, c->stream>>>(a, b.L));
+        if ((st = rhs_block(c, c->loc[bi], U[bi], M[bi], 2, rhs[bi], nullptr, nullptr, nullptr, 0, 0.0)))
+            return st;
     }
     return CROCCO_OK;
 }
-
-static const double RK_A[3] = {0.0, -5.0 / 9.0, -153.0 / 128.0};
-static const double RK_B[3] = {1.0 / 3.0, 15.0 / 16.0, 8.0 / 15.0};
 
 crocco_status crocco_rk_stage(crocco_ctx c, int32_t stage, double dt, double *const *Uin,
                               double *const *Uout, double *const *dU, double *const *M) {
@@ -792,19 +832,9 @@ crocco_status crocco_rk_stage(crocco_ctx c, int32_t stage, double dt, double *co
             return fail(c, CROCCO_ERR_ARG, "U_in, U_out and dU must be distinct");
     if ((st = crocco_fill_boundary(c, Uin, CROCCO_FIELD_STATE))) return st;
     for (size_t bi = 0; bi < c->loc.size(); bi++) {
-        const LocalBlock &b = c->loc[bi];
-        if ((st = rhs_parts(c, b, Uin[bi], M[bi]))) return st;
-        Asm a = make_asm(c, b, M[bi]);
-        a.mode = 1;
-        a.Uin = Uin[bi];
-        a.Uout = Uout[bi];
-        a.dU = dU[bi];
-        a.stage = stage;
-        a.A = RK_A[stage];
-        a.B = RK_B[stage];
-        a.dt = dt;
-        dim3 grd(cdiv(b.g.n[0], 128), b.g.n[1], b.g.n[2]);
-        LAUNCH(c, K_ASSEMBLE, k_assemble<<<grd, 128, 0, c->stream>>>(a, b.L));
+        if ((st = rhs_block(c, c->loc[bi], Uin[bi], M[bi], 3, nullptr, Uin[bi], Uout[bi], dU[bi], stage,
+                            dt)))
+            return st;
     }
     return CROCCO_OK;
 }

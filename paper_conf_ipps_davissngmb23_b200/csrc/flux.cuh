@@ -1,0 +1,233 @@
+// flux.cuh -- total interface flux of one direction: characteristic WENO-SYMBO
+// inviscid flux (WENOx/y/z; readings 8-11) minus the
+// viscous interface flux whose difference is the 4th-order central divergence
+// (Viscous; reading 12).
+//
+// Inviscid part at interface i+1/2 of direction d, from the points i-2..i+3:
+//   m^ = R6(m^d) = (m_{i-2} - 8m_{i-1} + 37m_i + 37m_{i+1} - 8m_{i+2} + m_{i+3})/60,
+//   n = m^/|m^|; Roe state of (i, i+1); Pulliam-Chaussee T, T^-1 for n;
+//   g_{s,l} = L_s.F_n(U_l), w_{s,l} = L_s.U_l, lambda_s = max_l |eig_s(l)|,
+//   g^_s = W(g+lambda w) + W_mirror(g-lambda w)  [the 1/2 of the LLF split is
+//   folded: W(v/2; eps) = W(v; 4 eps)/2, so the sum is halved at the end],
+//   F^ = |m^| T g^.
+// L_s.F_n(U_l) is evaluated as theta_l (L_s.U_l) + p_l k_{s,l} using the exact
+// identity F_n(U) = theta U + p (0, n, theta).
+// Viscous part: with the point fluxes f = F^_v^d (k_visc),
+//   h_{i+1/2} = [7(f_i + f_{i+1}) - (f_{i-1} + f_{i+2})]/12,
+//   h_{i+1/2} - h_{i-1/2} = D4 f_i  (exactly, in exact arithmetic).
+#pragma once
+#include "common.cuh"
+#include "weno.cuh"
+
+namespace crocco {
+
+#ifndef CROCCO_FIELD_ROLLED
+#define CROCCO_FIELD_ROLLED 0  // 1: keep the characteristic-field loop rolled (fewer live registers)
+#endif
+#ifndef CROCCO_SWEEP_UREG
+#define CROCCO_SWEEP_UREG 0  // 1: hold the 6x5 stencil states in registers; 0: re-read per field
+#endif
+
+struct FluxIn {
+    const double *__restrict__ U;
+    const double *__restrict__ P;
+    const double *__restrict__ M;
+    const double *__restrict__ FV;  // point viscous fluxes of this direction (4 comps) or null
+    int64_t cs;                     // component stride of U / P / M
+    int64_t vcs;                    // component stride of FV
+};
+
+// Stencil accessors: conserved state U(l, c), primitives P(l, k) (k = PU..PH),
+// the metric row m^d M(l, a) and the point viscous flux of direction d FV(l, q)
+// (q = momentum x, y, z, energy) at stencil point l = 0..5 (points i-2..i+3).
+template <int D>
+struct GAcc {  // straight from the global arrays (L1/L2 cached)
+    const double *__restrict__ u;
+    const double *__restrict__ p;
+    const double *__restrict__ m;   // metric component 1+3D
+    const double *__restrict__ fv;  // FV of direction D
+    int64_t cs, p0, s, vcs, v0, vs; // v0: FV index of point i-2
+    __device__ __forceinline__ double U(int l, int c) const { return u[c * cs + p0 + l * s]; }
+    __device__ __forceinline__ double P(int l, int k) const { return p[k * cs + p0 + l * s]; }
+    __device__ __forceinline__ double M(int l, int a) const { return m[a * cs + p0 + l * s]; }
+    __device__ __forceinline__ double FV(int l, int q) const { return fv[q * vcs + v0 + l * vs]; }
+};
+
+// shared-memory ring of a warp: value v of ring point q in column col at
+// sv[v * VS + (q & (NR-1)) * PS + col]
+enum { SV_U = 0, SV_M = 5, SV_FV = 8, SV_P = 12, SV_N = 19 };
+template <int NR, int PS>
+struct SAcc {
+    const double *sv;
+    int q0, col;
+    static constexpr int VS = NR * PS;
+    __device__ __forceinline__ double at_(int v, int l) const {
+        return sv[v * VS + ((q0 + l) & (NR - 1)) * PS + col];
+    }
+    __device__ __forceinline__ double U(int l, int c) const { return at_(SV_U + c, l); }
+    __device__ __forceinline__ double P(int l, int k) const { return at_(SV_P + k, l); }
+    __device__ __forceinline__ double M(int l, int a) const { return at_(SV_M + a, l); }
+    __device__ __forceinline__ double FV(int l, int q) const { return at_(SV_FV + q, l); }
+};
+
+// Total interface flux F = F^_inv - h_v of direction D at interface i+1/2.
+// A: stencil accessor (flux.cuh GAcc / SAcc).
+template <int D, class Acc>
+__device__ __forceinline__ void total_flux(const Acc &A, bool inv, bool visc, const Phys &ph,
+                                           double F[5]) {
+    F[0] = F[1] = F[2] = F[3] = F[4] = 0.0;
+    if (inv) {
+        const double gm1 = ph.gm1;
+        double mh[3];
+#pragma unroll
+        for (int a = 0; a < 3; a++)
+            mh[a] = fma(37.0, A.M(2, a) + A.M(3, a), fma(-8.0, A.M(1, a) + A.M(4, a), A.M(0, a) + A.M(5, a))) *
+                    (1.0 / 60.0);
+        const double s2 = fma(mh[0], mh[0], fma(mh[1], mh[1], mh[2] * mh[2]));
+        const double imag = rsqrt(s2);
+        const double hmag = 0.5 * s2 * imag;  // |m^|/2 (LLF 1/2 folded here)
+        const double nx = mh[0] * imag, ny = mh[1] * imag, nz = mh[2] * imag;
+
+        // Roe average of points i (l=2), i+1 (l=3), sqrt(rho) weights
+        const double srL = A.P(2, PSR), srR = A.P(3, PSR);
+        const double iden = 1.0 / (srL + srR);
+        const double wL = srL * iden, wR = srR * iden;
+        const double ut = fma(wL, A.P(2, PU), wR * A.P(3, PU));
+        const double vt = fma(wL, A.P(2, PV), wR * A.P(3, PV));
+        const double wt = fma(wL, A.P(2, PW), wR * A.P(3, PW));
+        const double Ht = fma(wL, A.P(2, PH), wR * A.P(3, PH));
+        const double rt = srL * srR;
+        const double q2 = fma(ut, ut, fma(vt, vt, wt * wt));
+        const double c2 = gm1 * fma(-0.5, q2, Ht);
+        const double ict = rsqrt(c2);
+        const double ct = c2 * ict;
+        const double ic2 = ict * ict;
+        const double irt = 1.0 / rt;
+        const double tht = fma(nx, ut, fma(ny, vt, nz * wt));
+        const double phi2 = 0.5 * gm1 * q2;
+        constexpr double SQ12 = 0.70710678118654752440;
+        const double alph = rt * ict * SQ12;   // rho/(sqrt2 c)
+        const double beta = irt * ict * SQ12;  // 1/(sqrt2 rho c)
+
+        // stencil points
+#if CROCCO_SWEEP_UREG
+        double Ul[6][5];
+#define UL(l, c) Ul[l][c]
+#else
+#define UL(l, c) A.U(l, c)
+#endif
+        double th[6], pl[6];
+        double lam0 = 0.0, lam3 = 0.0, lam4 = 0.0;
+#pragma unroll
+        for (int l = 0; l < 6; l++) {
+#if CROCCO_SWEEP_UREG
+#pragma unroll
+            for (int c = 0; c < 5; c++) Ul[l][c] = A.U(l, c);
+#endif
+            const double t = fma(nx, A.P(l, PU), fma(ny, A.P(l, PV), nz * A.P(l, PW)));
+            const double cl = A.P(l, PC);
+            th[l] = t;
+            pl[l] = A.P(l, PP);
+            lam0 = fmax(lam0, fabs(t));
+            lam3 = fmax(lam3, fabs(t + cl));
+            lam4 = fmax(lam4, fabs(t - cl));
+        }
+        const double eps_b = 4.0 * WENO_BSCALE * ph.eps;  // b-units (weno.cuh) x 4 (folded 1/2)
+        const double onemp = fma(-phi2, ic2, 1.0);
+        const double gic2 = gm1 * ic2;
+        const double cx = ny * wt - nz * vt, cy = nz * ut - nx * wt, cz = nx * vt - ny * ut;
+        const double ph1 = phi2 * ph.igm1;
+        double f0 = 0.0, f1 = 0.0, f2 = 0.0, f3 = 0.0, f4 = 0.0;
+#if CROCCO_FIELD_ROLLED
+#pragma unroll 1
+#else
+#pragma unroll
+#endif
+        for (int sf = 0; sf < 5; sf++) {
+            double L0, L1, L2, L3, L4, R0, R1, R2, R3, R4, lam, kA, kB;
+            if (sf < 3) {
+                const double na = sf == 0 ? nx : (sf == 1 ? ny : nz);
+                const double cr = sf == 0 ? cx : (sf == 1 ? cy : cz);
+                const double ng = na * gic2;
+                L0 = fma(na, onemp, cr * irt);
+                if (sf == 0) {
+                    L1 = ng * ut;
+                    L2 = fma(nz, irt, ng * vt);
+                    L3 = fma(-ny, irt, ng * wt);
+                    R1 = na * ut;
+                    R2 = fma(na, vt, nz * rt);
+                    R3 = fma(na, wt, -ny * rt);
+                    R4 = fma(na, ph1, rt * (nz * vt - ny * wt));
+                } else if (sf == 1) {
+                    L1 = fma(-nz, irt, ng * ut);
+                    L2 = ng * vt;
+                    L3 = fma(nx, irt, ng * wt);
+                    R1 = fma(na, ut, -nz * rt);
+                    R2 = na * vt;
+                    R3 = fma(na, wt, nx * rt);
+                    R4 = fma(na, ph1, rt * (nx * wt - nz * ut));
+                } else {
+                    L1 = fma(ny, irt, ng * ut);
+                    L2 = fma(-nx, irt, ng * vt);
+                    L3 = ng * wt;
+                    R1 = fma(na, ut, ny * rt);
+                    R2 = fma(na, vt, -nx * rt);
+                    R3 = na * wt;
+                    R4 = fma(na, ph1, rt * (ny * ut - nx * vt));
+                }
+                L4 = -ng;
+                R0 = na;
+                lam = lam0;
+                kA = ng * tht;
+                kB = -ng;
+            } else {
+                const double sg = (sf == 3) ? 1.0 : -1.0;
+                const double sc = sg * ct;
+                L0 = beta * fma(-sc, tht, phi2);
+                L1 = beta * fma(sc, nx, -gm1 * ut);
+                L2 = beta * fma(sc, ny, -gm1 * vt);
+                L3 = beta * fma(sc, nz, -gm1 * wt);
+                L4 = beta * gm1;
+                R0 = alph;
+                R1 = alph * fma(sc, nx, ut);
+                R2 = alph * fma(sc, ny, vt);
+                R3 = alph * fma(sc, nz, wt);
+                R4 = alph * fma(phi2 + c2, ph.igm1, sc * tht);
+                lam = (sf == 3) ? lam3 : lam4;
+                kA = beta * fma(-gm1, tht, sc);
+                kB = beta * gm1;
+            }
+            double gp[6], gm[6];
+#pragma unroll
+            for (int l = 0; l < 6; l++) {
+                const double w =
+                    fma(L0, UL(l, 0), fma(L1, UL(l, 1), fma(L2, UL(l, 2), fma(L3, UL(l, 3), L4 * UL(l, 4)))));
+                const double g = fma(th[l], w, pl[l] * fma(kB, th[l], kA));
+                gp[l] = fma(lam, w, g);
+                gm[l] = fma(-lam, w, g);
+            }
+            const double gh = weno_pair(gp, gm, eps_b);
+            f0 = fma(R0, gh, f0);
+            f1 = fma(R1, gh, f1);
+            f2 = fma(R2, gh, f2);
+            f3 = fma(R3, gh, f3);
+            f4 = fma(R4, gh, f4);
+        }
+#undef UL
+        F[0] = hmag * f0;
+        F[1] = hmag * f1;
+        F[2] = hmag * f2;
+        F[3] = hmag * f3;
+        F[4] = hmag * f4;
+    }
+    if (visc) {
+        // h_{i+1/2} = [7(f_i + f_{i+1}) - (f_{i-1} + f_{i+2})]/12 for momentum x,y,z and energy
+#pragma unroll
+        for (int q = 0; q < 4; q++) {
+            const double h = fma(7.0, A.FV(2, q) + A.FV(3, q), -(A.FV(1, q) + A.FV(4, q))) * (1.0 / 12.0);
+            F[1 + q] -= h;
+        }
+    }
+}
+
+}  // namespace crocco

@@ -1,0 +1,403 @@
+// sweep.cuh -- directional sweeps (WENOx, WENOy, WENOz + Viscous)
+// fused with the RHS assembly and the RK Update.
+//
+// Work decomposition (one warp = 32 interfaces per step, each interface flux
+// evaluated exactly once; the point difference uses the neighbour interface
+// exchanged by warp shuffle, the step-to-step carry stays in registers):
+//   D = 0 (xi, contiguous): a warp holds 4 lines x 8 consecutive interfaces and
+//     advances 8 interfaces per step.
+//   D = 1, 2 (eta, zeta): a warp holds 8 consecutive i (64-B coalesced rows) x 4
+//     consecutive interfaces and advances 4 per step.
+//   A line is marched over segments of `seg` points; each segment recomputes
+//   the one interface it shares with the previous segment.
+// Every interface, in any decomposition and any lane, runs the same code
+// (total_flux), so an n-block run equals the 1-block run bit for bit.
+//
+// Accumulation of R = -sum_d (F_{i+1/2} - F_{i-1/2}) per point in fixed order
+// xi, eta, zeta (mode 0 writes, mode 1 adds); the zeta sweep finishes the point:
+//   mode 2: rhs = J R ;  mode 3: dU <- A dU + dt J R, U_out = U_in + B dU.
+#pragma once
+#include "common.cuh"
+#include "flux.cuh"
+
+namespace crocco {
+
+#ifndef CROCCO_SWEEP_MINB
+#define CROCCO_SWEEP_MINB 1  // min CTAs/SM (register cap); the staged ring allows 2 CTAs x 4 warps
+#endif
+constexpr int SWEEP_THREADS = 128;
+
+struct SweepArgs {
+    FluxIn in;
+    VLay V;
+    double *R;          // accumulator, compact interior layout i + n0 (j + n1 k)
+    int64_t rcs;        // its component stride
+    int inv, visc;      // terms evaluated in this direction
+    int mode;           // 0 write R, 1 add to R, 2 rhs = J R, 3 RK update
+    int seg;            // march segment (D = 1, 2)
+    double *rhs;        // mode 2 (padded layout)
+    const double *Uin;  // mode 3 (padded layout)
+    double *Uout, *dU;
+    double A, B, dt;
+    int stage;
+};
+
+// finish / accumulate the contribution dF = F_{i-1/2} - F_{i+1/2} at interior point (i,j,k)
+__device__ __forceinline__ void contribute(const SweepArgs &a, const Lay &L, int i, int j, int k,
+                                           const double dF[5]) {
+    const int64_t r = (int64_t)i + (int64_t)L.n0 * (j + (int64_t)L.n1 * k);
+    if (a.mode == 0) {
+#pragma unroll
+        for (int c = 0; c < 5; c++) a.R[c * a.rcs + r] = dF[c];
+        return;
+    }
+    double Rt[5];
+#pragma unroll
+    for (int c = 0; c < 5; c++) Rt[c] = a.R[c * a.rcs + r] + dF[c];
+    if (a.mode == 1) {
+#pragma unroll
+        for (int c = 0; c < 5; c++) a.R[c * a.rcs + r] = Rt[c];
+        return;
+    }
+    const int64_t p = at(L, i, j, k);
+    const double J = a.in.M[p];
+    if (a.mode == 2) {
+#pragma unroll
+        for (int c = 0; c < 5; c++) a.rhs[c * L.cs + p] = J * Rt[c];
+        return;
+    }
+#pragma unroll
+    for (int c = 0; c < 5; c++) {
+        const int64_t q = c * L.cs + p;
+        const double rr = J * Rt[c];
+        const double du = (a.stage == 0) ? a.dt * rr : fma(a.A, a.dU[q], a.dt * rr);
+        a.dU[q] = du;
+        a.Uout[q] = fma(a.B, du, a.Uin[q]);
+    }
+}
+
+template <int D>
+__global__ void __launch_bounds__(SWEEP_THREADS, CROCCO_SWEEP_MINB) k_sweep(const __grid_constant__ SweepArgs a,
+                                                                        const Lay L, const Phys ph) {
+    // warp tile: D = 0: 4 lines x 8 consecutive interfaces (lane = 8*line + offset);
+    //            D = 1, 2: 8 consecutive i x 4 consecutive interfaces (lane = 8*offset + i).
+    constexpr int WS = (D == 0) ? 8 : 4;  // interfaces per step along the sweep
+    constexpr int WT = 32 / WS;           // transverse lines per warp
+    const int lane = threadIdx.x & 31;
+    const int ls = (D == 0) ? (lane & 7) : (lane >> 3);  // sweep offset
+    const int lt = (D == 0) ? (lane >> 3) : (lane & 7);  // transverse offset
+    const int64_t gw = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+    const bool inv = a.inv != 0, visc = a.visc != 0;
+    // swept extent and segments of the march
+    const int nd = D == 0 ? L.n0 : (D == 1 ? L.n1 : L.n2);
+    const int nseg = (nd + a.seg - 1) / a.seg;
+    bool lvalid;
+    int ci = 0, cj = 0, ck = 0;  // point coordinates of the line (swept one unused)
+    int sg;
+    if (D == 0) {
+        const int64_t ntl = ((int64_t)L.n1 * L.n2 + WT - 1) / WT;
+        if (gw >= ntl * nseg) return;
+        sg = (int)(gw / ntl);
+        const int64_t tline = (gw % ntl) * WT + lt;  // j + n1 k
+        lvalid = tline < (int64_t)L.n1 * L.n2;
+        if (lvalid) {
+            cj = (int)(tline % L.n1);
+            ck = (int)(tline / L.n1);
+        }
+    } else {
+        const int tiles = (L.n0 + WT - 1) / WT;
+        const int nother = (D == 1) ? L.n2 : L.n1;
+        const int64_t ntl = (int64_t)tiles * nother;
+        if (gw >= ntl * nseg) return;
+        sg = (int)(gw / ntl);
+        const int64_t r = gw % ntl;
+        const int iv = (int)(r % tiles) * WT + lt;
+        const int oo = (int)(r / tiles);
+        lvalid = iv < L.n0;
+        if (lvalid) {
+            ci = iv;
+            if (D == 1) ck = oo;
+            else cj = oo;
+        }
+    }
+    const int e0 = sg * a.seg, e1 = min(nd, e0 + a.seg);
+    const int64_t s = (D == 0) ? 1 : (D == 1 ? L.py : L.pz);
+    const int64_t vs = (D == 0) ? 1 : (D == 1 ? a.V.py : a.V.pz);
+    const int nsteps = (e1 - e0 + 1 + WS - 1) / WS;  // interfaces e0-1 .. e1-1
+    double F[5], Fc[5];
+#pragma unroll
+    for (int c = 0; c < 5; c++) Fc[c] = 0.0;
+    for (int st = 0; st < nsteps; st++) {
+        const int e = e0 - 1 + WS * st + ls;  // this lane's interface e+1/2
+        const bool act = lvalid && e <= e1 - 1;
+        const int pi = D == 0 ? e : ci, pj = D == 1 ? e : cj, pk = D == 2 ? e : ck;
+        if (act) {
+            // the single call site of the flux for every interface (bitwise decomposition invariance)
+            const int qi = D == 0 ? e - 2 : pi, qj = D == 1 ? e - 2 : pj, qk = D == 2 ? e - 2 : pk;
+            const int vi = D == 0 ? e - 1 : pi, vj = D == 1 ? e - 1 : pj, vk = D == 2 ? e - 1 : pk;
+            const GAcc<D> A{a.in.U, a.in.P, a.in.M + (int64_t)(1 + 3 * D) * a.in.cs, a.in.FV,
+                            a.in.cs, at(L, qi, qj, qk), s, a.in.vcs, vat(a.V, vi, vj, vk) - vs, vs};
+            total_flux<D>(A, inv, visc, ph, F);
+        } else {
+#pragma unroll
+            for (int c = 0; c < 5; c++) F[c] = 0.0;
+        }
+        double dF[5];
+#pragma unroll
+        for (int c = 0; c < 5; c++) {
+            double Fm;
+            if (D == 0) {
+                Fm = __shfl_up_sync(0xffffffffu, F[c], 1, 8);
+                if (ls == 0) Fm = Fc[c];
+                Fc[c] = __shfl_sync(0xffffffffu, F[c], 7, 8);
+            } else {
+                Fm = __shfl_up_sync(0xffffffffu, F[c], 8);
+                if (ls == 0) Fm = Fc[c];
+                Fc[c] = __shfl_sync(0xffffffffu, F[c], 24 + lt);
+            }
+            dF[c] = Fm - F[c];
+        }
+        if (act && e >= e0) contribute(a, L, pi, pj, pk, dF);
+    }
+}
+
+// ---------------------------------------------------------------------------
+// Shared-memory staged sweep (same tiles and arithmetic as k_sweep): each warp
+// keeps a ring of its stencil window in shared memory -- conserved state and
+// metric row copied with cp.async one step ahead of use, primitives computed
+// once per point when it enters the ring -- so the characteristic WENO reads
+// only shared memory.  Warps are independent (no block barriers).
+// ---------------------------------------------------------------------------
+__device__ __forceinline__ void cp_async8(double *dst, const double *src) {
+    const unsigned d = (unsigned)__cvta_generic_to_shared(dst);
+    asm volatile("cp.async.ca.shared.global [%0], [%1], 8;\n" ::"r"(d), "l"(src) : "memory");
+}
+__device__ __forceinline__ void cp_async16(double *dst, const double *src) {
+    const unsigned d = (unsigned)__cvta_generic_to_shared(dst);
+    asm volatile("cp.async.cg.shared.global [%0], [%1], 16;\n" ::"r"(d), "l"(src) : "memory");
+}
+__device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commit_group;\n" ::: "memory"); }
+__device__ __forceinline__ void cp_async_wait_all() { asm volatile("cp.async.wait_group 0;\n" ::: "memory"); }
+
+template <int D>
+struct RingGeom {
+    static constexpr int WS = (D == 0) ? 8 : 4;    // interfaces per step
+    static constexpr int C = 32 / WS;              // columns (lines) per warp
+    static constexpr int LA = (D == 0) ? 1 : 2;    // chunks ahead needed by a step
+    static constexpr int NR = (D == 0) ? 32 : 16;  // ring points (>= (LA + 2) * WS, power of 2)
+    static constexpr int NCB = 16;                 // prefetched accumulate/update operands per lane
+    static constexpr int PER_WARP = SV_N * NR * C + NCB * 32;  // doubles
+};
+
+// accumulate / finish with operands prefetched into shared memory:
+// cb[0..4] = R, cb[5] = J, cb[6..10] = dU, cb[11..15] = U_in  (stride 32 doubles)
+__device__ __forceinline__ void contribute_pre(const SweepArgs &a, const Lay &L, int i, int j, int k,
+                                               const double dF[5], const double *cb) {
+    const int64_t r = (int64_t)i + (int64_t)L.n0 * (j + (int64_t)L.n1 * k);
+    if (a.mode == 0) {
+#pragma unroll
+        for (int c = 0; c < 5; c++) a.R[c * a.rcs + r] = dF[c];
+        return;
+    }
+    double Rt[5];
+#pragma unroll
+    for (int c = 0; c < 5; c++) Rt[c] = cb[32 * c] + dF[c];
+    if (a.mode == 1) {
+#pragma unroll
+        for (int c = 0; c < 5; c++) a.R[c * a.rcs + r] = Rt[c];
+        return;
+    }
+    const int64_t p = at(L, i, j, k);
+    const double J = cb[32 * 5];
+    if (a.mode == 2) {
+#pragma unroll
+        for (int c = 0; c < 5; c++) a.rhs[c * L.cs + p] = J * Rt[c];
+        return;
+    }
+#pragma unroll
+    for (int c = 0; c < 5; c++) {
+        const int64_t q = c * L.cs + p;
+        const double rr = J * Rt[c];
+        const double du = (a.stage == 0) ? a.dt * rr : fma(a.A, cb[32 * (6 + c)], a.dt * rr);
+        a.dU[q] = du;
+        a.Uout[q] = fma(a.B, du, cb[32 * (11 + c)]);
+    }
+}
+
+template <int D>
+__global__ void __launch_bounds__(SWEEP_THREADS, CROCCO_SWEEP_MINB) k_sweep_s(const __grid_constant__ SweepArgs a,
+                                                                          const Lay L, const Phys ph) {
+    using RG = RingGeom<D>;
+    constexpr int WS = RG::WS, C = RG::C, LA = RG::LA, NR = RG::NR;
+    constexpr int VS = NR * C;
+    extern __shared__ double smem_dyn[];
+    const int lane = threadIdx.x & 31;
+    double *sv = smem_dyn + (threadIdx.x >> 5) * RG::PER_WARP;
+    double *cb = sv + SV_N * VS + lane;  // this lane's prefetched operands
+    const int ls = (D == 0) ? (lane & 7) : (lane >> 3);  // sweep offset of this lane
+    const int lt = (D == 0) ? (lane >> 3) : (lane & 7);  // column of this lane
+    const int64_t gw = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+    const bool inv = a.inv != 0, visc = a.visc != 0;
+    const int nvl = visc ? 12 : 8;  // values copied per point: U, metric row (, FV)
+    const int nd = D == 0 ? L.n0 : (D == 1 ? L.n1 : L.n2);
+    const int nseg = (nd + a.seg - 1) / a.seg;
+    int64_t ntl;
+    if (D == 0) ntl = ((int64_t)L.n1 * L.n2 + C - 1) / C;
+    else ntl = (int64_t)((L.n0 + C - 1) / C) * ((D == 1) ? L.n2 : L.n1);
+    if (gw >= ntl * nseg) return;
+    const int sg = (int)(gw / ntl);
+    const int64_t r = gw % ntl;
+    int colbase = 0, oo = 0;
+    if (D != 0) {
+        const int tiles = (L.n0 + C - 1) / C;
+        colbase = (int)(r % tiles) * C;
+        oo = (int)(r / tiles);
+    }
+    // line coordinates of column `col` (swept coordinate left 0)
+    auto line_of = [&](int col, int &ci, int &cj, int &ck) -> bool {
+        if (D == 0) {
+            const int64_t t = r * C + col;
+            ci = cj = ck = 0;
+            if (t >= (int64_t)L.n1 * L.n2) return false;
+            cj = (int)(t % L.n1);
+            ck = (int)(t / L.n1);
+            return true;
+        } else {
+            ci = colbase + col;
+            cj = D == 1 ? 0 : oo;
+            ck = D == 1 ? oo : 0;
+            return ci < L.n0;
+        }
+    };
+    int ci, cj, ck;
+    const bool lvalid = line_of(lt, ci, cj, ck);
+    const int e0 = sg * a.seg, e1 = min(nd, e0 + a.seg);
+    const int qbase = e0 - 3;                        // swept index of ring point q = 0
+    const int nsteps = (e1 - e0 + 1 + WS - 1) / WS;  // interfaces e0-1 .. e1-1
+    const int qmax = nd + G - 1 - qbase;             // last ring point inside the padded box
+    const double *Mrow = a.in.M + (int64_t)(1 + 3 * D) * L.cs;
+
+    // source of value v (0..11) at point (gi, gj, gk); FV only on the interior +-2 box
+    auto src_of = [&](int v, int gi, int gj, int gk) -> const double * {
+        if (v < 5) return a.in.U + (int64_t)v * L.cs + at(L, gi, gj, gk);
+        if (v < 8) return Mrow + (int64_t)(v - 5) * L.cs + at(L, gi, gj, gk);
+        return a.in.FV + (int64_t)(v - 8) * a.in.vcs + vat(a.V, gi, gj, gk);
+    };
+    // issue the copies of chunk `ch` (WS points x C columns x nvl values)
+    auto issue = [&](int ch) {
+        if (D == 0) {
+            // 8 consecutive points x 4 lines, 8-B copies, one value per iteration
+            const int pt = lane & 7, col = lane >> 3;
+            const int q = ch * WS + pt, gq = qbase + q;
+            int li, lj, lk;
+            const bool ok = q <= qmax && line_of(col, li, lj, lk);
+            for (int v = 0; v < nvl; v++) {
+                if (ok && (v < 8 || (gq >= -2 && gq <= nd + 1)))
+                    cp_async8(sv + v * VS + (q & (NR - 1)) * C + col, src_of(v, gq, lj, lk));
+            }
+        } else {
+            // 4 points x nvl values x 8 columns (64-B rows), 16-B copies
+            const int pair = lane & 3;
+            const int gi = colbase + 2 * pair;
+            for (int t = lane >> 2; t < WS * nvl; t += 8) {
+                const int v = t % nvl, pt = t / nvl;
+                const int q = ch * WS + pt, gq = qbase + q;
+                if (q <= qmax && (v < 8 || (gq >= -2 && gq <= nd + 1))) {
+                    const double *src = D == 1 ? src_of(v, gi, gq, oo) : src_of(v, gi, oo, gq);
+                    cp_async16(sv + v * VS + (q & (NR - 1)) * C + 2 * pair, src);
+                }
+            }
+        }
+        cp_async_commit();
+    };
+    // primitives of chunk `ch` (one point per lane), from the staged state
+    auto prims = [&](int ch) {
+        const int q = ch * WS + ls;
+        if (q > qmax) return;
+        double *b = sv + (q & (NR - 1)) * C + lt;
+        const double rho = b[0], ru = b[VS], rv = b[2 * VS], rw = b[3 * VS], E = b[4 * VS];
+        const double ir = 1.0 / rho;
+        const double u = ru * ir, v = rv * ir, w = rw * ir;
+        const double pr = ph.gm1 * fma(-0.5, fma(ru, u, fma(rv, v, rw * w)), E);
+        b[(SV_P + PU) * VS] = u;
+        b[(SV_P + PV) * VS] = v;
+        b[(SV_P + PW) * VS] = w;
+        b[(SV_P + PP) * VS] = pr;
+        b[(SV_P + PC) * VS] = sqrt(ph.gamma * pr * ir);
+        b[(SV_P + PSR) * VS] = sqrt(rho);
+        b[(SV_P + PH) * VS] = (E + pr) * ir;
+    };
+    // accumulate / update operands of this lane's point of step st (own slots only)
+    auto prefetch_ops = [&](int pi, int pj, int pk) {
+        if (a.mode == 0) return;
+        const int64_t rr = (int64_t)pi + (int64_t)L.n0 * (pj + (int64_t)L.n1 * pk);
+#pragma unroll
+        for (int c = 0; c < 5; c++) cp_async8(cb + 32 * c, a.R + c * a.rcs + rr);
+        if (a.mode >= 2) {
+            const int64_t p = at(L, pi, pj, pk);
+            cp_async8(cb + 32 * 5, a.in.M + p);
+            if (a.mode == 3) {
+#pragma unroll
+                for (int c = 0; c < 5; c++) {
+                    if (a.stage != 0) cp_async8(cb + 32 * (6 + c), a.dU + c * L.cs + p);
+                    cp_async8(cb + 32 * (11 + c), a.Uin + c * L.cs + p);
+                }
+            }
+        }
+    };
+
+    // prologue: chunks 0 .. LA staged with primitives, chunk LA+1 in flight
+    for (int ch = 0; ch <= LA; ch++) issue(ch);
+    cp_async_wait_all();
+    __syncwarp();
+    for (int ch = 0; ch <= LA; ch++) prims(ch);
+    __syncwarp();
+
+    double F[5], Fc[5];
+#pragma unroll
+    for (int c = 0; c < 5; c++) Fc[c] = 0.0;
+    for (int st = 0; st < nsteps; st++) {
+        if (st > 0) {
+            // chunk st+LA landed -> primitives (its slot was consumed at step st-2..)
+            cp_async_wait_all();
+            __syncwarp();
+            prims(st + LA);
+            __syncwarp();
+        }
+        const int e = e0 - 1 + WS * st + ls;  // this lane's interface e+1/2
+        const bool act = lvalid && e <= e1 - 1;
+        const int pi = D == 0 ? e : ci, pj = D == 1 ? e : cj, pk = D == 2 ? e : ck;
+        const bool own = act && e >= e0;      // this lane finishes point e
+        if (own) prefetch_ops(pi, pj, pk);
+        cp_async_commit();                    // group A: operands of step st
+        issue(st + LA + 1);                   // group B: chunk st+LA+1 (slot of chunk st-1)
+        if (act) {
+            const SAcc<NR, C> A{sv, WS * st + ls, lt};  // ring point of stencil point i-2
+            total_flux<D>(A, inv, visc, ph, F);
+        } else {
+#pragma unroll
+            for (int c = 0; c < 5; c++) F[c] = 0.0;
+        }
+        double dF[5];
+#pragma unroll
+        for (int c = 0; c < 5; c++) {
+            double Fm;
+            if (D == 0) {
+                Fm = __shfl_up_sync(0xffffffffu, F[c], 1, 8);
+                if (ls == 0) Fm = Fc[c];
+                Fc[c] = __shfl_sync(0xffffffffu, F[c], 7, 8);
+            } else {
+                Fm = __shfl_up_sync(0xffffffffu, F[c], 8);
+                if (ls == 0) Fm = Fc[c];
+                Fc[c] = __shfl_sync(0xffffffffu, F[c], 24 + lt);
+            }
+            dF[c] = Fm - F[c];
+        }
+        asm volatile("cp.async.wait_group 1;\n" ::: "memory");  // group A landed (own data)
+        if (own) contribute_pre(a, L, pi, pj, pk, dF, cb);
+        __syncwarp();
+    }
+    cp_async_wait_all();
+}
+
+}  // namespace crocco

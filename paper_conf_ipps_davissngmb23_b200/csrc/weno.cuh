@@ -1,0 +1,73 @@
+// weno.cuh -- WENO-SYMBO reconstruction (PAPER.md:50 -> ref [9]; reading 8).
+//
+// W(v_{-2..3}) reconstructs the value at the +1/2 interface from 4 candidate
+// 3-point stencils (the 4th one downwind), Jiang-Shu smoothness indicators with
+// beta_3 <- max(beta_0..beta_3), weights alpha_k = C_k/(eps+beta_k)^2.
+//
+// Evaluated in difference form (algebraically identical):
+//   d_m = v_{m-1} - v_{m-2}  (d0 = v_{-1}-v_{-2}, ..., d4 = v_3-v_2)
+//   q_k = v_0 + r_k/6, r = (5d1-2d0, d1+2d2, 4d2-d3, 6d2-5d3+2d4)
+//   (12/13) beta_k = b_k = s_k^2 + (3/13) f_k^2, s = second differences,
+//   f = one-sided first differences (3d1-d0, d1+d2, d3-3d2, 5d3-3d4)
+//   alpha_k ~ C_k prod_{m != k} (lam eps + b_m)^2 with lam = 12/13   (one division)
+// so W = v_0 + num/(6 den), num = sum alpha_k r_k, den = sum alpha_k.
+// Callers pass eps_b = the epsilon in the units of b (see flux.cuh).
+#pragma once
+#include "common.cuh"
+
+namespace crocco {
+
+constexpr double WENO_BSCALE = 12.0 / 13.0;  // b_k = WENO_BSCALE * beta_k
+
+struct WenoFrac {
+    double base, num, den;  // W = base + num/(6 den)
+};
+
+__device__ __forceinline__ WenoFrac weno_symbo_frac(double v0, double v1, double v2, double v3,
+                                                    double v4, double v5, double eps_b) {
+    constexpr double C0 = 0.094647545896, C1 = 0.428074212384, C2 = 0.408289331408,
+                     C3 = 0.068988910311;
+    constexpr double K3 = 3.0 / 13.0;
+    const double d0 = v1 - v0, d1 = v2 - v1, d2 = v3 - v2, d3 = v4 - v3, d4 = v5 - v4;
+    const double r0 = fma(5.0, d1, -2.0 * d0);
+    const double r1 = fma(2.0, d2, d1);
+    const double r2 = fma(4.0, d2, -d3);
+    const double r3 = fma(6.0, d2, fma(-5.0, d3, 2.0 * d4));
+    const double s0 = d1 - d0, s1 = d2 - d1, s2 = d3 - d2, s3 = d4 - d3;
+    const double f0 = fma(3.0, d1, -d0);
+    const double f1 = d1 + d2;
+    const double f2 = fma(-3.0, d2, d3);
+    const double f3 = fma(5.0, d3, -3.0 * d4);
+    const double b0 = fma(K3 * f0, f0, s0 * s0);
+    const double b1 = fma(K3 * f1, f1, s1 * s1);
+    const double b2 = fma(K3 * f2, f2, s2 * s2);
+    double b3 = fma(K3 * f3, f3, s3 * s3);
+    // downwind stencil never preferred (continuous max, parity-safe)
+    const double m01 = b0 > b1 ? b0 : b1;
+    const double m23 = b2 > b3 ? b2 : b3;
+    b3 = m01 > m23 ? m01 : m23;
+    double e0 = eps_b + b0, e1 = eps_b + b1, e2 = eps_b + b2, e3 = eps_b + b3;
+    e0 *= e0;
+    e1 *= e1;
+    e2 *= e2;
+    e3 *= e3;
+    // alpha_0 = C0 e1 e2 e3, alpha_1 = C1 e0 e2 e3, alpha_2 = C2 e0 e1 e3, alpha_3 = C3 e0 e1 e2
+    const double e01 = e0 * e1, e23 = e2 * e3;
+    const double x0 = C0 * e1, x1 = C1 * e0, x2 = C2 * e3, x3 = C3 * e2;
+    WenoFrac w;
+    w.base = v2;
+    w.num = fma(e23, fma(x0, r0, x1 * r1), e01 * fma(x2, r2, x3 * r3));
+    w.den = fma(e23, x0 + x1, e01 * (x2 + x3));
+    return w;
+}
+
+// W^+ of (vp0..vp5) plus W^- of the mirrored (vm5..vm0), as one fraction:
+// (b+ + b-) + (n+ d- + n- d+)/(6 d+ d-)  -- one division per characteristic field.
+// Range: the alpha products stay inside fp64 for |v| up to ~1e9.
+__device__ __forceinline__ double weno_pair(const double vp[6], const double vm[6], double eps_b) {
+    const WenoFrac a = weno_symbo_frac(vp[0], vp[1], vp[2], vp[3], vp[4], vp[5], eps_b);
+    const WenoFrac b = weno_symbo_frac(vm[5], vm[4], vm[3], vm[2], vm[1], vm[0], eps_b);
+    return (a.base + b.base) + fma(a.num, b.den, b.num * a.den) / (6.0 * (a.den * b.den));
+}
+
+}  // namespace crocco
