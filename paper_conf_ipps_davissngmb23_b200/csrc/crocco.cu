@@ -169,7 +169,7 @@ static Lay make_layout(const int n[3], int g) {
     L.n1 = n[1];
     L.n2 = n[2];
     const int64_t lead = 16;  // interior starts at element 16 of each row
-    L.py = rup(lead + n[0] + g, 16);
+    L.py = rup(lead + n[0] + g + 8, 16);  // +8: whole 8-column tiles of the sweeps stay in the row
     L.pz = L.py * (n[1] + 2 * g);
     L.off = lead + L.py * g + L.pz * g;
     L.cs = L.pz * (n[2] + 2 * g);
@@ -293,15 +293,20 @@ template <int D>
 static constexpr size_t sweep_smem_bytes() {
     return (size_t)(SWEEP_THREADS / 32) * RingGeom<D>::PER_WARP * sizeof(double);
 }
+template <int D, bool V>
+static cudaError_t sweep_attr1() {
+    return cudaFuncSetAttribute(k_sweep_s<D, V>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                (int)sweep_smem_bytes<D>());
+}
 static cudaError_t sweep_attrs() {
-    cudaError_t e = cudaFuncSetAttribute(k_sweep_s<0>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                         (int)sweep_smem_bytes<0>());
+    cudaError_t e = sweep_attr1<0, false>();
+    if (e == cudaSuccess) e = sweep_attr1<1, false>();
+    if (e == cudaSuccess) e = sweep_attr1<2, false>();
+    if (e == cudaSuccess) e = sweep_attr1<0, true>();
+    if (e == cudaSuccess) e = sweep_attr1<1, true>();
+    if (e == cudaSuccess) e = sweep_attr1<2, true>();
     if (e == cudaSuccess)
-        e = cudaFuncSetAttribute(k_sweep_s<1>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                 (int)sweep_smem_bytes<1>());
-    if (e == cudaSuccess)
-        e = cudaFuncSetAttribute(k_sweep_s<2>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                 (int)sweep_smem_bytes<2>());
+        e = cudaFuncSetAttribute(k_visc_tiled, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)VISC_SMEM);
     return e;
 }
 
@@ -430,7 +435,7 @@ crocco_status crocco_init_grid(const crocco_grid_desc *desc, const crocco_phys *
         lb.V.b0 = g.n[0] + 4;
         lb.V.b1 = g.n[1] + 4;
         lb.V.b2 = g.n[2] + 4;
-        lb.V.py = rup(lb.V.b0, 16);
+        lb.V.py = rup(lb.V.b0 + 8, 16);
         lb.V.pz = lb.V.py * lb.V.b1;
         lb.V.cs = rup(lb.V.pz * lb.V.b2, 32);
         c->gid_to_local[g.gid] = (int)c->loc.size();
@@ -752,11 +757,17 @@ static crocco_status rhs_block(crocco_ctx c, const LocalBlock &b, const double *
     const bool inviscid = (ph.terms & CROCCO_TERM_INVISCID) != 0;
     const bool viscous = (ph.terms & CROCCO_TERM_VISCOUS) != 0;
     const int64_t np = (int64_t)(b.g.n[0] + 2 * G) * (b.g.n[1] + 2 * G) * (b.g.n[2] + 2 * G);
-    if (viscous || !CROCCO_SWEEP_SMEM)  // the staged sweeps compute their own primitives
+    if (!CROCCO_SWEEP_SMEM)  // the staged sweeps and the tiled viscous kernel compute their own primitives
         LAUNCH(c, K_PRIMS, k_prims<<<cdiv(np, 256), 256, 0, c->stream>>>(U, b.prim, b.L, ph));
     if (viscous) {
+#if CROCCO_SWEEP_SMEM
+        const unsigned nt = (unsigned)(((b.V.b0 + VTX - 1) / VTX) * ((b.V.b1 + VTY - 1) / VTY) *
+                                       ((b.V.b2 + VK - 1) / VK));
+        LAUNCH(c, K_VISC, k_visc_tiled<<<nt, VTX * VTY, VISC_SMEM, c->stream>>>(U, M, b.fv, b.L, b.V, ph));
+#else
         const int64_t nv = (int64_t)b.V.b0 * b.V.b1 * b.V.b2;
         LAUNCH(c, K_VISC, k_visc<<<cdiv(nv, 256), 256, 0, c->stream>>>(b.prim, M, b.fv, b.L, b.V, ph));
+#endif
     }
     for (int d = 0; d < 3; d++) {
         SweepArgs a;
@@ -792,9 +803,12 @@ static crocco_status rhs_block(crocco_ctx c, const LocalBlock &b, const double *
         const int64_t warps = lines * ((nd + seg - 1) / seg);
         const unsigned grid = cdiv(warps * 32, SWEEP_THREADS);
 #if CROCCO_SWEEP_SMEM
-        if (d == 0) LAUNCH(c, K_FLUX_X, k_sweep_s<0><<<grid, SWEEP_THREADS, sweep_smem_bytes<0>(), c->stream>>>(a, b.L, ph));
-        else if (d == 1) LAUNCH(c, K_FLUX_Y, k_sweep_s<1><<<grid, SWEEP_THREADS, sweep_smem_bytes<1>(), c->stream>>>(a, b.L, ph));
-        else LAUNCH(c, K_FLUX_Z, k_sweep_s<2><<<grid, SWEEP_THREADS, sweep_smem_bytes<2>(), c->stream>>>(a, b.L, ph));
+#define SWEEP_LAUNCH(DD, VV) \
+        k_sweep_s<DD, VV><<<grid, SWEEP_THREADS, sweep_smem_bytes<DD>(), c->stream>>>(a, b.L, ph)
+        if (d == 0) LAUNCH(c, K_FLUX_X, if (viscous) SWEEP_LAUNCH(0, true); else SWEEP_LAUNCH(0, false));
+        else if (d == 1) LAUNCH(c, K_FLUX_Y, if (viscous) SWEEP_LAUNCH(1, true); else SWEEP_LAUNCH(1, false));
+        else LAUNCH(c, K_FLUX_Z, if (viscous) SWEEP_LAUNCH(2, true); else SWEEP_LAUNCH(2, false));
+#undef SWEEP_LAUNCH
 #else
         if (d == 0) LAUNCH(c, K_FLUX_X, k_sweep<0><<<grid, SWEEP_THREADS, 0, c->stream>>>(a, b.L, ph));
         else if (d == 1) LAUNCH(c, K_FLUX_Y, k_sweep<1><<<grid, SWEEP_THREADS, 0, c->stream>>>(a, b.L, ph));

@@ -109,6 +109,113 @@ __global__ void __launch_bounds__(256) k_visc(const double *__restrict__ Pm,
     }
 }
 
+// Same viscous point fluxes, fused with the primitive recovery and tiled in
+// shared memory: a CTA owns 32 (i) x 8 (j) columns of the interior +-2 box and
+// marches a slab of VK planes in k, keeping u, v, w, T of planes k-2..k+2 (with
+// a 2-point i/j halo) in a rolling shared-memory window; every primitive is
+// computed once per slab from U.
+constexpr int VTX = 32, VTY = 8, VK = 32;           // tile and slab
+constexpr int VHX = VTX + 4, VHY = VTY + 4;          // with halo
+constexpr int VPL = VHX * VHY;                       // points per plane
+constexpr size_t VISC_SMEM = (size_t)5 * 4 * VPL * sizeof(double);
+
+__global__ void __launch_bounds__(VTX * VTY) k_visc_tiled(const double *__restrict__ U,
+                                                          const double *__restrict__ M,
+                                                          double *__restrict__ FV, Lay L, VLay V,
+                                                          Phys ph) {
+    extern __shared__ double vsm[];  // [plane slot 5][value 4][VPL]
+    const int tx = threadIdx.x % VTX, ty = threadIdx.x / VTX;
+    const int tilesx = (V.b0 + VTX - 1) / VTX, tilesy = (V.b1 + VTY - 1) / VTY;
+    int b = blockIdx.x;
+    const int bx = b % tilesx;
+    b /= tilesx;
+    const int by = b % tilesy;
+    const int bz = b / tilesy;
+    const int i0 = bx * VTX - 2, j0 = by * VTY - 2;      // first output point of the tile
+    const int k0 = bz * VK - 2, k1 = min(k0 + VK, V.b2 - 2);
+    const double iR = 1.0 / ph.R;
+    // primitives u v w T of plane kk into slot (kk mod 5); halo points clamped to the padded box
+    auto load_plane = [&](int kk) {
+        double *pl = vsm + ((kk + 10) % 5) * 4 * VPL;
+        for (int t = threadIdx.x; t < VPL; t += VTX * VTY) {
+            const int hi = t % VHX, hj = t / VHX;
+            const int gi = min(i0 - 2 + hi, L.n0 + G - 1), gj = min(j0 - 2 + hj, L.n1 + G - 1);
+            const int64_t p = at(L, gi, gj, kk);
+            const double rho = U[p], ru = U[L.cs + p], rv = U[2 * L.cs + p], rw = U[3 * L.cs + p],
+                         E = U[4 * L.cs + p];
+            const double ir = 1.0 / rho;
+            const double u = ru * ir, v = rv * ir, w = rw * ir;
+            const double pr = ph.gm1 * fma(-0.5, fma(ru, u, fma(rv, v, rw * w)), E);
+            pl[t] = u;
+            pl[VPL + t] = v;
+            pl[2 * VPL + t] = w;
+            pl[3 * VPL + t] = pr * ir * iR;
+        }
+    };
+    for (int kk = k0 - 2; kk < k0 + 2; kk++) load_plane(kk);
+    const int i = i0 + tx, j = j0 + ty;
+    const bool own = i < V.b0 - 2 && j < V.b1 - 2;
+    const int c0 = (ty + 2) * VHX + (tx + 2);  // this thread's point in a plane
+    for (int k = k0; k < k1; k++) {
+        load_plane(k + 2);
+        __syncthreads();
+        if (own) {
+            const double *pk[5];
+#pragma unroll
+            for (int o = 0; o < 5; o++) pk[o] = vsm + ((k - 2 + o + 10) % 5) * 4 * VPL;
+            double gc[4][3];
+#pragma unroll
+            for (int f = 0; f < 4; f++) {
+                const double *c = pk[2] + f * VPL + c0;
+                gc[f][0] = fma(8.0, c[1] - c[-1], -(c[2] - c[-2])) * (1.0 / 12.0);
+                gc[f][1] = fma(8.0, c[VHX] - c[-VHX], -(c[2 * VHX] - c[-2 * VHX])) * (1.0 / 12.0);
+                gc[f][2] = fma(8.0, pk[3][f * VPL + c0] - pk[1][f * VPL + c0],
+                               -(pk[4][f * VPL + c0] - pk[0][f * VPL + c0])) * (1.0 / 12.0);
+            }
+            const int64_t p = at(L, i, j, k);
+            const double J = M[p];
+            double m[3][3];
+#pragma unroll
+            for (int d = 0; d < 3; d++)
+#pragma unroll
+                for (int a = 0; a < 3; a++) m[d][a] = M[(1 + 3 * d + a) * L.cs + p];
+            double gx[4][3];
+#pragma unroll
+            for (int f = 0; f < 4; f++)
+#pragma unroll
+                for (int a = 0; a < 3; a++)
+                    gx[f][a] = J * fma(m[0][a], gc[f][0], fma(m[1][a], gc[f][1], m[2][a] * gc[f][2]));
+            const double T = pk[2][3 * VPL + c0];
+            const double mu = mu_of_T(ph, T);
+            const double kap = mu * ph.cp_over_Pr;
+            const double div = gx[0][0] + gx[1][1] + gx[2][2];
+            double tau[3][3];
+#pragma unroll
+            for (int a = 0; a < 3; a++)
+#pragma unroll
+                for (int bb = 0; bb < 3; bb++) tau[a][bb] = mu * (gx[a][bb] + gx[bb][a]);
+            const double dterm = (2.0 / 3.0) * mu * div;
+            tau[0][0] -= dterm;
+            tau[1][1] -= dterm;
+            tau[2][2] -= dterm;
+            const double vel[3] = {pk[2][c0], pk[2][VPL + c0], pk[2][2 * VPL + c0]};
+            double hb[3];
+#pragma unroll
+            for (int bb = 0; bb < 3; bb++)
+                hb[bb] = fma(vel[0], tau[0][bb], fma(vel[1], tau[1][bb], fma(vel[2], tau[2][bb], kap * gx[3][bb])));
+            const int64_t o = vat(V, i, j, k);
+#pragma unroll
+            for (int d = 0; d < 3; d++) {
+#pragma unroll
+                for (int a = 0; a < 3; a++)
+                    FV[(4 * d + a) * V.cs + o] = fma(m[d][0], tau[a][0], fma(m[d][1], tau[a][1], m[d][2] * tau[a][2]));
+                FV[(4 * d + 3) * V.cs + o] = fma(m[d][0], hb[0], fma(m[d][1], hb[1], m[d][2] * hb[2]));
+            }
+        }
+        __syncthreads();
+    }
+}
+
 // Update alone, from a materialised rhs (crocco_rk_update).
 __global__ void __launch_bounds__(256) k_update(const double *__restrict__ Uin,
                                                 double *__restrict__ Uout, double *__restrict__ dU,

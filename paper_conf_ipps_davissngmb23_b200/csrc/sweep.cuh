@@ -189,42 +189,7 @@ struct RingGeom {
     static constexpr int PER_WARP = SV_N * NR * C + NCB * 32;  // doubles
 };
 
-// accumulate / finish with operands prefetched into shared memory:
-// cb[0..4] = R, cb[5] = J, cb[6..10] = dU, cb[11..15] = U_in  (stride 32 doubles)
-__device__ __forceinline__ void contribute_pre(const SweepArgs &a, const Lay &L, int i, int j, int k,
-                                               const double dF[5], const double *cb) {
-    const int64_t r = (int64_t)i + (int64_t)L.n0 * (j + (int64_t)L.n1 * k);
-    if (a.mode == 0) {
-#pragma unroll
-        for (int c = 0; c < 5; c++) a.R[c * a.rcs + r] = dF[c];
-        return;
-    }
-    double Rt[5];
-#pragma unroll
-    for (int c = 0; c < 5; c++) Rt[c] = cb[32 * c] + dF[c];
-    if (a.mode == 1) {
-#pragma unroll
-        for (int c = 0; c < 5; c++) a.R[c * a.rcs + r] = Rt[c];
-        return;
-    }
-    const int64_t p = at(L, i, j, k);
-    const double J = cb[32 * 5];
-    if (a.mode == 2) {
-#pragma unroll
-        for (int c = 0; c < 5; c++) a.rhs[c * L.cs + p] = J * Rt[c];
-        return;
-    }
-#pragma unroll
-    for (int c = 0; c < 5; c++) {
-        const int64_t q = c * L.cs + p;
-        const double rr = J * Rt[c];
-        const double du = (a.stage == 0) ? a.dt * rr : fma(a.A, cb[32 * (6 + c)], a.dt * rr);
-        a.dU[q] = du;
-        a.Uout[q] = fma(a.B, du, cb[32 * (11 + c)]);
-    }
-}
-
-template <int D>
+template <int D, bool VISC>
 __global__ void __launch_bounds__(SWEEP_THREADS, CROCCO_SWEEP_MINB) k_sweep_s(const __grid_constant__ SweepArgs a,
                                                                           const Lay L, const Phys ph) {
     using RG = RingGeom<D>;
@@ -237,8 +202,7 @@ __global__ void __launch_bounds__(SWEEP_THREADS, CROCCO_SWEEP_MINB) k_sweep_s(co
     const int ls = (D == 0) ? (lane & 7) : (lane >> 3);  // sweep offset of this lane
     const int lt = (D == 0) ? (lane >> 3) : (lane & 7);  // column of this lane
     const int64_t gw = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
-    const bool inv = a.inv != 0, visc = a.visc != 0;
-    const int nvl = visc ? 12 : 8;  // values copied per point: U, metric row (, FV)
+    const bool inv = a.inv != 0;
     const int nd = D == 0 ? L.n0 : (D == 1 ? L.n1 : L.n2);
     const int nseg = (nd + a.seg - 1) / a.seg;
     int64_t ntl;
@@ -247,64 +211,78 @@ __global__ void __launch_bounds__(SWEEP_THREADS, CROCCO_SWEEP_MINB) k_sweep_s(co
     if (gw >= ntl * nseg) return;
     const int sg = (int)(gw / ntl);
     const int64_t r = gw % ntl;
-    int colbase = 0, oo = 0;
-    if (D != 0) {
-        const int tiles = (L.n0 + C - 1) / C;
-        colbase = (int)(r % tiles) * C;
-        oo = (int)(r / tiles);
-    }
-    // line coordinates of column `col` (swept coordinate left 0)
-    auto line_of = [&](int col, int &ci, int &cj, int &ck) -> bool {
-        if (D == 0) {
-            const int64_t t = r * C + col;
-            ci = cj = ck = 0;
-            if (t >= (int64_t)L.n1 * L.n2) return false;
-            cj = (int)(t % L.n1);
-            ck = (int)(t / L.n1);
-            return true;
-        } else {
-            ci = colbase + col;
-            cj = D == 1 ? 0 : oo;
-            ck = D == 1 ? oo : 0;
-            return ci < L.n0;
-        }
-    };
-    int ci, cj, ck;
-    const bool lvalid = line_of(lt, ci, cj, ck);
     const int e0 = sg * a.seg, e1 = min(nd, e0 + a.seg);
     const int qbase = e0 - 3;                        // swept index of ring point q = 0
     const int nsteps = (e1 - e0 + 1 + WS - 1) / WS;  // interfaces e0-1 .. e1-1
     const int qmax = nd + G - 1 - qbase;             // last ring point inside the padded box
+    const int64_t sst = D == 0 ? 1 : (D == 1 ? L.py : L.pz);  // swept strides
+    const int64_t vst = D == 0 ? 1 : (D == 1 ? a.V.py : a.V.pz);
+
+    // this lane's own line (for its interfaces) ...
+    int ci = 0, cj = 0, ck = 0;
+    bool lvalid;
+    // ... and the line / column it copies for the ring (D = 0: column lane>>3; D != 0: pair lane&3)
+    int64_t cpo = 0, cpv = 0;  // padded / FV-box index of the copy column at swept index 0
+    bool cvalid;
+    if (D == 0) {
+        const int64_t t = r * C + lt, nl = (int64_t)L.n1 * L.n2;
+        lvalid = cvalid = t < nl;
+        if (lvalid) {
+            cj = (int)(t % L.n1);
+            ck = (int)(t / L.n1);
+        }
+        cpo = at(L, 0, cj, ck);
+        cpv = vat(a.V, 0, cj, ck);
+    } else {
+        const int tiles = (L.n0 + C - 1) / C;
+        const int colbase = (int)(r % tiles) * C, oo = (int)(r / tiles);
+        ci = colbase + lt;
+        lvalid = ci < L.n0;
+        if (D == 1) ck = oo;
+        else cj = oo;
+        cvalid = true;  // whole 8-column rows are copied (columns past n0 stay in the row padding)
+        const int gi = colbase + 2 * (lane & 3);
+        cpo = D == 1 ? at(L, gi, 0, oo) : at(L, gi, oo, 0);
+        cpv = D == 1 ? vat(a.V, gi, 0, oo) : vat(a.V, gi, oo, 0);
+    }
     const double *Mrow = a.in.M + (int64_t)(1 + 3 * D) * L.cs;
 
-    // source of value v (0..11) at point (gi, gj, gk); FV only on the interior +-2 box
-    auto src_of = [&](int v, int gi, int gj, int gk) -> const double * {
-        if (v < 5) return a.in.U + (int64_t)v * L.cs + at(L, gi, gj, gk);
-        if (v < 8) return Mrow + (int64_t)(v - 5) * L.cs + at(L, gi, gj, gk);
-        return a.in.FV + (int64_t)(v - 8) * a.in.vcs + vat(a.V, gi, gj, gk);
-    };
-    // issue the copies of chunk `ch` (WS points x C columns x nvl values)
+    // issue the copies of chunk `ch`: U (5) + metric row (3) [+ FV (4)] of WS points x C columns
     auto issue = [&](int ch) {
         if (D == 0) {
-            // 8 consecutive points x 4 lines, 8-B copies, one value per iteration
-            const int pt = lane & 7, col = lane >> 3;
-            const int q = ch * WS + pt, gq = qbase + q;
-            int li, lj, lk;
-            const bool ok = q <= qmax && line_of(col, li, lj, lk);
-            for (int v = 0; v < nvl; v++) {
-                if (ok && (v < 8 || (gq >= -2 && gq <= nd + 1)))
-                    cp_async8(sv + v * VS + (q & (NR - 1)) * C + col, src_of(v, gq, lj, lk));
+            // lane: point lane&7 of column lane>>3, all values, 8-B copies
+            const int q = ch * WS + (lane & 7), gq = qbase + q;
+            if (cvalid && q <= qmax) {
+                double *dst = sv + (q & (NR - 1)) * C + lt;
+                const int64_t o = cpo + gq;
+#pragma unroll
+                for (int v = 0; v < 5; v++) cp_async8(dst + v * VS, a.in.U + v * L.cs + o);
+#pragma unroll
+                for (int v = 0; v < 3; v++) cp_async8(dst + (SV_M + v) * VS, Mrow + v * L.cs + o);
+                if (VISC && gq >= -2 && gq <= nd + 1) {
+                    const int64_t ov = cpv + gq;
+#pragma unroll
+                    for (int v = 0; v < 4; v++) cp_async8(dst + (SV_FV + v) * VS, a.in.FV + v * a.in.vcs + ov);
+                }
             }
         } else {
-            // 4 points x nvl values x 8 columns (64-B rows), 16-B copies
-            const int pair = lane & 3;
-            const int gi = colbase + 2 * pair;
-            for (int t = lane >> 2; t < WS * nvl; t += 8) {
-                const int v = t % nvl, pt = t / nvl;
+            // lane: value lane>>2 (U0-4, M0-2) [and FV lane>>2 for lanes < 16] of the
+            // column pair lane&3, all WS points, 16-B copies
+            const int v = lane >> 2;
+            const double *src0 = v < 5 ? a.in.U + v * L.cs + cpo : Mrow + (v - 5) * L.cs + cpo;
+            double *dst0 = sv + v * VS + 2 * (lane & 3);
+#pragma unroll
+            for (int pt = 0; pt < WS; pt++) {
                 const int q = ch * WS + pt, gq = qbase + q;
-                if (q <= qmax && (v < 8 || (gq >= -2 && gq <= nd + 1))) {
-                    const double *src = D == 1 ? src_of(v, gi, gq, oo) : src_of(v, gi, oo, gq);
-                    cp_async16(sv + v * VS + (q & (NR - 1)) * C + 2 * pair, src);
+                if (q <= qmax) cp_async16(dst0 + (q & (NR - 1)) * C, src0 + gq * sst);
+            }
+            if (VISC && v < 4) {
+                const double *srcf = a.in.FV + v * a.in.vcs + cpv;
+                double *dstf = sv + (SV_FV + v) * VS + 2 * (lane & 3);
+#pragma unroll
+                for (int pt = 0; pt < WS; pt++) {
+                    const int q = ch * WS + pt, gq = qbase + q;
+                    if (q <= qmax && gq >= -2 && gq <= nd + 1) cp_async16(dstf + (q & (NR - 1)) * C, srcf + gq * vst);
                 }
             }
         }
@@ -314,51 +292,43 @@ __global__ void __launch_bounds__(SWEEP_THREADS, CROCCO_SWEEP_MINB) k_sweep_s(co
     auto prims = [&](int ch) {
         const int q = ch * WS + ls;
         if (q > qmax) return;
-        double *b = sv + (q & (NR - 1)) * C + lt;
-        const double rho = b[0], ru = b[VS], rv = b[2 * VS], rw = b[3 * VS], E = b[4 * VS];
+        double *bq = sv + (q & (NR - 1)) * C + lt;
+        const double rho = bq[0], ru = bq[VS], rv = bq[2 * VS], rw = bq[3 * VS], E = bq[4 * VS];
         const double ir = 1.0 / rho;
         const double u = ru * ir, v = rv * ir, w = rw * ir;
         const double pr = ph.gm1 * fma(-0.5, fma(ru, u, fma(rv, v, rw * w)), E);
-        b[(SV_P + PU) * VS] = u;
-        b[(SV_P + PV) * VS] = v;
-        b[(SV_P + PW) * VS] = w;
-        b[(SV_P + PP) * VS] = pr;
-        b[(SV_P + PC) * VS] = sqrt(ph.gamma * pr * ir);
-        b[(SV_P + PSR) * VS] = sqrt(rho);
-        b[(SV_P + PH) * VS] = (E + pr) * ir;
-    };
-    // accumulate / update operands of this lane's point of step st (own slots only)
-    auto prefetch_ops = [&](int pi, int pj, int pk) {
-        if (a.mode == 0) return;
-        const int64_t rr = (int64_t)pi + (int64_t)L.n0 * (pj + (int64_t)L.n1 * pk);
-#pragma unroll
-        for (int c = 0; c < 5; c++) cp_async8(cb + 32 * c, a.R + c * a.rcs + rr);
-        if (a.mode >= 2) {
-            const int64_t p = at(L, pi, pj, pk);
-            cp_async8(cb + 32 * 5, a.in.M + p);
-            if (a.mode == 3) {
-#pragma unroll
-                for (int c = 0; c < 5; c++) {
-                    if (a.stage != 0) cp_async8(cb + 32 * (6 + c), a.dU + c * L.cs + p);
-                    cp_async8(cb + 32 * (11 + c), a.Uin + c * L.cs + p);
-                }
-            }
-        }
+        bq[(SV_P + PU) * VS] = u;
+        bq[(SV_P + PV) * VS] = v;
+        bq[(SV_P + PW) * VS] = w;
+        bq[(SV_P + PP) * VS] = pr;
+        bq[(SV_P + PC) * VS] = sqrt(ph.gamma * pr * ir);
+        bq[(SV_P + PSR) * VS] = sqrt(rho);
+        bq[(SV_P + PH) * VS] = (E + pr) * ir;
     };
 
-    // prologue: chunks 0 .. LA staged with primitives, chunk LA+1 in flight
+    // prologue: chunks 0 .. LA staged with primitives
     for (int ch = 0; ch <= LA; ch++) issue(ch);
     cp_async_wait_all();
     __syncwarp();
     for (int ch = 0; ch <= LA; ch++) prims(ch);
     __syncwarp();
 
+    // this lane's point at step 0 (interface e = e0-1+ls finishes point e) and its indices
+    const int64_t rstep = (D == 0 ? 1 : (D == 1 ? (int64_t)L.n0 : (int64_t)L.n0 * L.n1)) * WS;
+    const int64_t pstep = sst * WS;
+    int64_t rr, pp;
+    {
+        const int e = e0 - 1 + ls;
+        const int pi = D == 0 ? e : ci, pj = D == 1 ? e : cj, pk = D == 2 ? e : ck;
+        rr = (int64_t)pi + (int64_t)L.n0 * (pj + (int64_t)L.n1 * pk);
+        pp = at(L, pi, pj, pk);
+    }
     double F[5], Fc[5];
 #pragma unroll
     for (int c = 0; c < 5; c++) Fc[c] = 0.0;
-    for (int st = 0; st < nsteps; st++) {
+    for (int st = 0; st < nsteps; st++, rr += rstep, pp += pstep) {
         if (st > 0) {
-            // chunk st+LA landed -> primitives (its slot was consumed at step st-2..)
+            // chunk st+LA landed -> primitives
             cp_async_wait_all();
             __syncwarp();
             prims(st + LA);
@@ -366,14 +336,26 @@ __global__ void __launch_bounds__(SWEEP_THREADS, CROCCO_SWEEP_MINB) k_sweep_s(co
         }
         const int e = e0 - 1 + WS * st + ls;  // this lane's interface e+1/2
         const bool act = lvalid && e <= e1 - 1;
-        const int pi = D == 0 ? e : ci, pj = D == 1 ? e : cj, pk = D == 2 ? e : ck;
         const bool own = act && e >= e0;      // this lane finishes point e
-        if (own) prefetch_ops(pi, pj, pk);
-        cp_async_commit();                    // group A: operands of step st
+        if (own && a.mode != 0) {             // group A: accumulate / update operands
+#pragma unroll
+            for (int c = 0; c < 5; c++) cp_async8(cb + 32 * c, a.R + c * a.rcs + rr);
+            if (a.mode >= 2) {
+                cp_async8(cb + 32 * 5, a.in.M + pp);
+                if (a.mode == 3) {
+#pragma unroll
+                    for (int c = 0; c < 5; c++) {
+                        if (a.stage != 0) cp_async8(cb + 32 * (6 + c), a.dU + c * L.cs + pp);
+                        cp_async8(cb + 32 * (11 + c), a.Uin + c * L.cs + pp);
+                    }
+                }
+            }
+        }
+        cp_async_commit();
         issue(st + LA + 1);                   // group B: chunk st+LA+1 (slot of chunk st-1)
         if (act) {
             const SAcc<NR, C> A{sv, WS * st + ls, lt};  // ring point of stencil point i-2
-            total_flux<D>(A, inv, visc, ph, F);
+            total_flux<D>(A, inv, VISC, ph, F);
         } else {
 #pragma unroll
             for (int c = 0; c < 5; c++) F[c] = 0.0;
@@ -394,7 +376,33 @@ __global__ void __launch_bounds__(SWEEP_THREADS, CROCCO_SWEEP_MINB) k_sweep_s(co
             dF[c] = Fm - F[c];
         }
         asm volatile("cp.async.wait_group 1;\n" ::: "memory");  // group A landed (own data)
-        if (own) contribute_pre(a, L, pi, pj, pk, dF, cb);
+        if (own) {
+            if (a.mode == 0) {
+#pragma unroll
+                for (int c = 0; c < 5; c++) a.R[c * a.rcs + rr] = dF[c];
+            } else {
+                double Rt[5];
+#pragma unroll
+                for (int c = 0; c < 5; c++) Rt[c] = cb[32 * c] + dF[c];
+                if (a.mode == 1) {
+#pragma unroll
+                    for (int c = 0; c < 5; c++) a.R[c * a.rcs + rr] = Rt[c];
+                } else if (a.mode == 2) {
+                    const double J = cb[32 * 5];
+#pragma unroll
+                    for (int c = 0; c < 5; c++) a.rhs[c * L.cs + pp] = J * Rt[c];
+                } else {
+                    const double J = cb[32 * 5];
+#pragma unroll
+                    for (int c = 0; c < 5; c++) {
+                        const double rv = J * Rt[c];
+                        const double du = (a.stage == 0) ? a.dt * rv : fma(a.A, cb[32 * (6 + c)], a.dt * rv);
+                        a.dU[c * L.cs + pp] = du;
+                        a.Uout[c * L.cs + pp] = fma(a.B, du, cb[32 * (11 + c)]);
+                    }
+                }
+            }
+        }
         __syncwarp();
     }
     cp_async_wait_all();
