@@ -36,6 +36,37 @@ __host__ __device__ inline int64_t vat(const VLay &V, int i, int j, int k) {
     return (int64_t)(i + 2) + V.py * (j + 2) + V.pz * (k + 2);
 }
 
+// Branch-free reciprocal / reciprocal square root: hardware approximation
+// (MUFU.RCP64H / MUFU.RSQ64H) + 2 Newton steps + (for x/y) one residual
+// correction -- within ~1 ulp for the positive, normal-range operands of this
+// path (densities, sound speeds, metric norms, WENO weight sums); used instead
+// of the IEEE div/sqrt sequences, whose slow-path branches cost issue slots.
+__device__ __forceinline__ double rcp_nr(double y) {
+    double r;
+    asm("rcp.approx.ftz.f64 %0, %1;" : "=d"(r) : "d"(y));
+    double e = fma(-y, r, 1.0);
+    r = fma(r, e, r);
+    e = fma(-y, r, 1.0);
+    return fma(r, e, r);
+}
+__device__ __forceinline__ double div_nr(double x, double y) {
+    const double r = rcp_nr(y);
+    const double q = x * r;
+    return fma(r, fma(-y, q, x), q);
+}
+__device__ __forceinline__ double rsqrt_nr(double x) {
+    double r;
+    asm("rsqrt.approx.ftz.f64 %0, %1;" : "=d"(r) : "d"(x));
+    const double h = 0.5 * x;
+    r = r * fma(-h * r, r, 1.5);
+    return r * fma(-h * r, r, 1.5);
+}
+__device__ __forceinline__ double sqrt_nr(double x) {  // x > 0
+    const double r = rsqrt_nr(x);
+    const double s = x * r;
+    return fma(0.5 * r, fma(-s, s, x), s);  // one Newton correction of s
+}
+
 // primitive buffer components (k_prims)
 enum { PU = 0, PV = 1, PW = 2, PP = 3, PC = 4, PSR = 5, PH = 6, PT = 7, NPRIM = 8 };
 

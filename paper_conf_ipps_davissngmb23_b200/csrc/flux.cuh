@@ -84,13 +84,13 @@ __device__ __forceinline__ void total_flux(const Acc &A, bool inv, bool visc, co
             mh[a] = fma(37.0, A.M(2, a) + A.M(3, a), fma(-8.0, A.M(1, a) + A.M(4, a), A.M(0, a) + A.M(5, a))) *
                     (1.0 / 60.0);
         const double s2 = fma(mh[0], mh[0], fma(mh[1], mh[1], mh[2] * mh[2]));
-        const double imag = rsqrt(s2);
+        const double imag = rsqrt_nr(s2);
         const double hmag = 0.5 * s2 * imag;  // |m^|/2 (LLF 1/2 folded here)
         const double nx = mh[0] * imag, ny = mh[1] * imag, nz = mh[2] * imag;
 
         // Roe average of points i (l=2), i+1 (l=3), sqrt(rho) weights
         const double srL = A.P(2, PSR), srR = A.P(3, PSR);
-        const double iden = 1.0 / (srL + srR);
+        const double iden = rcp_nr(srL + srR);
         const double wL = srL * iden, wR = srR * iden;
         const double ut = fma(wL, A.P(2, PU), wR * A.P(3, PU));
         const double vt = fma(wL, A.P(2, PV), wR * A.P(3, PV));
@@ -99,10 +99,10 @@ __device__ __forceinline__ void total_flux(const Acc &A, bool inv, bool visc, co
         const double rt = srL * srR;
         const double q2 = fma(ut, ut, fma(vt, vt, wt * wt));
         const double c2 = gm1 * fma(-0.5, q2, Ht);
-        const double ict = rsqrt(c2);
+        const double ict = rsqrt_nr(c2);
         const double ct = c2 * ict;
         const double ic2 = ict * ict;
-        const double irt = 1.0 / rt;
+        const double irt = rcp_nr(rt);
         const double tht = fma(nx, ut, fma(ny, vt, nz * wt));
         const double phi2 = 0.5 * gm1 * q2;
         constexpr double SQ12 = 0.70710678118654752440;

@@ -294,15 +294,15 @@ __global__ void __launch_bounds__(SWEEP_THREADS, CROCCO_SWEEP_MINB) k_sweep_s(co
         if (q > qmax) return;
         double *bq = sv + (q & (NR - 1)) * C + lt;
         const double rho = bq[0], ru = bq[VS], rv = bq[2 * VS], rw = bq[3 * VS], E = bq[4 * VS];
-        const double ir = 1.0 / rho;
+        const double ir = rcp_nr(rho);
         const double u = ru * ir, v = rv * ir, w = rw * ir;
         const double pr = ph.gm1 * fma(-0.5, fma(ru, u, fma(rv, v, rw * w)), E);
         bq[(SV_P + PU) * VS] = u;
         bq[(SV_P + PV) * VS] = v;
         bq[(SV_P + PW) * VS] = w;
         bq[(SV_P + PP) * VS] = pr;
-        bq[(SV_P + PC) * VS] = sqrt(ph.gamma * pr * ir);
-        bq[(SV_P + PSR) * VS] = sqrt(rho);
+        bq[(SV_P + PC) * VS] = sqrt_nr(ph.gamma * pr * ir);
+        bq[(SV_P + PSR) * VS] = sqrt_nr(rho);
         bq[(SV_P + PH) * VS] = (E + pr) * ir;
     };
 

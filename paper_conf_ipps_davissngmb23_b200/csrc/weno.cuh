@@ -67,7 +67,7 @@ __device__ __forceinline__ WenoFrac weno_symbo_frac(double v0, double v1, double
 __device__ __forceinline__ double weno_pair(const double vp[6], const double vm[6], double eps_b) {
     const WenoFrac a = weno_symbo_frac(vp[0], vp[1], vp[2], vp[3], vp[4], vp[5], eps_b);
     const WenoFrac b = weno_symbo_frac(vm[5], vm[4], vm[3], vm[2], vm[1], vm[0], eps_b);
-    return (a.base + b.base) + fma(a.num, b.den, b.num * a.den) / (6.0 * (a.den * b.den));
+    return (a.base + b.base) + div_nr(fma(a.num, b.den, b.num * a.den), 6.0 * (a.den * b.den));
 }
 
 }  // namespace crocco
