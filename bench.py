@@ -276,7 +276,7 @@ def run_crocco(args, rank, world, local_rank):
                "steps": args.e2e_steps}
 
     # ---------------- roofline of the dominant kernel (CUDA events on the launching stream)
-    flux_cls = {"flux_xi": 0, "flux_eta": 1, "flux_zeta": 2}
+    flux_cls = {"sweep_xi": 0, "sweep_eta": 1, "sweep_zeta_update": 2}
     dom = max(ktimes.items(), key=lambda kv: kv[1][1])
     name, (nl, kms) = dom
     avg_ms = kms / max(nl, 1)
@@ -285,12 +285,13 @@ def run_crocco(args, rank, world, local_rank):
         d = flux_cls[name]
         ifaces = (bn[d] + 1) * pts_local // bn[d]
         ach = FLUX_FLOPS_PER_IFACE * ifaces / (avg_ms / 1e3) / 1e12
-        roof = {"bound": "alu", "kernel": f"k_flux<{d}> ({name})", "achieved": ach,
+        roof = {"bound": "alu", "kernel": f"k_sweep_s<{d}> ({name})", "achieved": ach,
                 "peak": FP64_PEAK_TFLOPS, "unit": "TFLOP/s", "frac": ach / FP64_PEAK_TFLOPS,
                 "peak_source": "derived: 148 SM x 64 FP64 FMA/clk x 2 x 1.965 GHz (DESIGN.md sec. 6)",
                 "flops_per_unit": FLUX_FLOPS_PER_IFACE, "unit_of_work": "interface flux",
                 "units_per_launch": ifaces, "avg_launch_ms": avg_ms,
-                "traffic": _profiled_traffic(name)}
+                "traffic": _profiled_traffic(f"k_sweep_s<{d}, 1>"),
+                "traffic_source": "profiles/ncu_summary.json (ncu --set full, dram__bytes_read+write per launch)"}
     peaks = measured_peaks()
     hbm = peaks.get("hbm_gbs", 6650.0)
     stage_gbs = value / world * HBM_BYTES_PER_PT_STAGE / 1e9
@@ -339,7 +340,7 @@ def main():
     ap.add_argument("--e2e-steps", type=int, default=2)
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-clocks", action="store_true")
-    ap.add_argument("--ref-n", type=int, default=48)
+    ap.add_argument("--ref-n", type=int, default=64)
     args = ap.parse_args()
     rank = int(os.environ.get("RANK", "0"))
     world = int(os.environ.get("WORLD_SIZE", "1"))
