@@ -109,22 +109,37 @@ __global__ void __launch_bounds__(256) k_visc(const double *__restrict__ Pm,
     }
 }
 
-// Same viscous point fluxes, fused with the primitive recovery and tiled in
-// shared memory: a CTA owns 32 (i) x 8 (j) columns of the interior +-2 box and
-// marches a slab of VK planes in k, keeping u, v, w, T of planes k-2..k+2 (with
-// a 2-point i/j halo) in a rolling shared-memory window; every primitive is
-// computed once per slab from U.
+// Same viscous point fluxes, fused with the primitive recovery: a CTA owns
+// 32 (i) x 8 (j) columns of the interior +-2 box and marches a slab of VK
+// planes in k.  Each thread keeps u, v, w, T of its own column for planes
+// k-2..k+2 in registers (k-derivatives), and only the current plane k (with a
+// 2-point i/j halo) is staged in shared memory (i/j-derivatives), double
+// buffered so one barrier per plane suffices.
 constexpr int VTX = 32, VTY = 8, VK = 32;           // tile and slab
 constexpr int VHX = VTX + 4, VHY = VTY + 4;          // with halo
-constexpr int VPL = VHX * VHY;                       // points per plane
-constexpr size_t VISC_SMEM = (size_t)5 * 4 * VPL * sizeof(double);
+constexpr int VPL = VHX * VHY;                       // points per staged plane
+constexpr int VHALO = VPL - VTX * VTY;               // halo points per plane
+constexpr size_t VISC_SMEM = (size_t)2 * 4 * VPL * sizeof(double);
+
+__device__ __forceinline__ void prim4(const double *__restrict__ U, int64_t cs, int64_t p, double gm1,
+                                      double iR, double out[4]) {
+    const double rho = U[p], ru = U[cs + p], rv = U[2 * cs + p], rw = U[3 * cs + p], E = U[4 * cs + p];
+    const double ir = rcp_nr(rho);
+    const double u = ru * ir, v = rv * ir, w = rw * ir;
+    const double pr = gm1 * fma(-0.5, fma(ru, u, fma(rv, v, rw * w)), E);
+    out[0] = u;
+    out[1] = v;
+    out[2] = w;
+    out[3] = pr * ir * iR;
+}
 
 __global__ void __launch_bounds__(VTX * VTY) k_visc_tiled(const double *__restrict__ U,
                                                           const double *__restrict__ M,
                                                           double *__restrict__ FV, Lay L, VLay V,
                                                           Phys ph) {
-    extern __shared__ double vsm[];  // [plane slot 5][value 4][VPL]
-    const int tx = threadIdx.x % VTX, ty = threadIdx.x / VTX;
+    extern __shared__ double vsm[];  // [buffer 2][value 4][VPL]
+    const int tid = threadIdx.x;
+    const int tx = tid % VTX, ty = tid / VTX;
     const int tilesx = (V.b0 + VTX - 1) / VTX, tilesy = (V.b1 + VTY - 1) / VTY;
     int b = blockIdx.x;
     const int bx = b % tilesx;
@@ -134,43 +149,63 @@ __global__ void __launch_bounds__(VTX * VTY) k_visc_tiled(const double *__restri
     const int i0 = bx * VTX - 2, j0 = by * VTY - 2;      // first output point of the tile
     const int k0 = bz * VK - 2, k1 = min(k0 + VK, V.b2 - 2);
     const double iR = 1.0 / ph.R;
-    // primitives u v w T of plane kk into slot (kk mod 5); halo points clamped to the padded box
-    auto load_plane = [&](int kk) {
-        double *pl = vsm + ((kk + 10) % 5) * 4 * VPL;
-        for (int t = threadIdx.x; t < VPL; t += VTX * VTY) {
-            const int hi = t % VHX, hj = t / VHX;
-            const int gi = min(i0 - 2 + hi, L.n0 + G - 1), gj = min(j0 - 2 + hj, L.n1 + G - 1);
-            const int64_t p = at(L, gi, gj, kk);
-            const double rho = U[p], ru = U[L.cs + p], rv = U[2 * L.cs + p], rw = U[3 * L.cs + p],
-                         E = U[4 * L.cs + p];
-            const double ir = 1.0 / rho;
-            const double u = ru * ir, v = rv * ir, w = rw * ir;
-            const double pr = ph.gm1 * fma(-0.5, fma(ru, u, fma(rv, v, rw * w)), E);
-            pl[t] = u;
-            pl[VPL + t] = v;
-            pl[2 * VPL + t] = w;
-            pl[3 * VPL + t] = pr * ir * iR;
-        }
-    };
-    for (int kk = k0 - 2; kk < k0 + 2; kk++) load_plane(kk);
+    // own column (clamped into the padded box for the idle threads of edge tiles)
     const int i = i0 + tx, j = j0 + ty;
     const bool own = i < V.b0 - 2 && j < V.b1 - 2;
-    const int c0 = (ty + 2) * VHX + (tx + 2);  // this thread's point in a plane
+    const int gi = min(i, L.n0 + G - 1), gj = min(j, L.n1 + G - 1);
+    // halo point handled by this thread (tid < VHALO): rows j0-2, j0-1, j0+8, j0+9 (36 each),
+    // then columns i0-2, i0-1, i0+32, i0+33 of rows j0..j0+7
+    int hx = 0, hy = 0;
+    if (tid < 4 * VHX) {
+        hx = tid % VHX;
+        const int r = tid / VHX;
+        hy = r < 2 ? r : VTY + r;        // 0,1 | 10,11
+    } else if (tid < VHALO) {
+        const int t = tid - 4 * VHX;      // 0..31
+        const int c = t % 4;
+        hy = 2 + t / 4;
+        hx = c < 2 ? c : VTX + c;         // 0,1 | 34,35
+    }
+    const int hgi = min(i0 - 2 + hx, L.n0 + G - 1), hgj = min(j0 - 2 + hy, L.n1 + G - 1);
+    const int hidx = hy * VHX + hx;
+    const int oidx = (ty + 2) * VHX + (tx + 2);
+
+    double win[4][5];  // own u v w T at planes k-2 .. k+2
+    for (int o = 0; o < 4; o++) {
+        double q[4];
+        prim4(U, L.cs, at(L, gi, gj, k0 - 2 + o), ph.gm1, iR, q);
+#pragma unroll
+        for (int f = 0; f < 4; f++) win[f][o + 1] = q[f];  // shifted into 0..3 by the first step
+    }
     for (int k = k0; k < k1; k++) {
-        load_plane(k + 2);
+        {   // own primitives of plane k+2, shift the window
+            double q[4];
+            prim4(U, L.cs, at(L, gi, gj, k + 2), ph.gm1, iR, q);
+#pragma unroll
+            for (int f = 0; f < 4; f++) {
+#pragma unroll
+                for (int o = 0; o < 4; o++) win[f][o] = win[f][o + 1];
+                win[f][4] = q[f];
+            }
+        }
+        double *pl = vsm + (k & 1) * 4 * VPL;
+#pragma unroll
+        for (int f = 0; f < 4; f++) pl[f * VPL + oidx] = win[f][2];
+        if (tid < VHALO) {
+            double q[4];
+            prim4(U, L.cs, at(L, hgi, hgj, k), ph.gm1, iR, q);
+#pragma unroll
+            for (int f = 0; f < 4; f++) pl[f * VPL + hidx] = q[f];
+        }
         __syncthreads();
         if (own) {
-            const double *pk[5];
-#pragma unroll
-            for (int o = 0; o < 5; o++) pk[o] = vsm + ((k - 2 + o + 10) % 5) * 4 * VPL;
             double gc[4][3];
 #pragma unroll
             for (int f = 0; f < 4; f++) {
-                const double *c = pk[2] + f * VPL + c0;
+                const double *c = pl + f * VPL + oidx;
                 gc[f][0] = fma(8.0, c[1] - c[-1], -(c[2] - c[-2])) * (1.0 / 12.0);
                 gc[f][1] = fma(8.0, c[VHX] - c[-VHX], -(c[2 * VHX] - c[-2 * VHX])) * (1.0 / 12.0);
-                gc[f][2] = fma(8.0, pk[3][f * VPL + c0] - pk[1][f * VPL + c0],
-                               -(pk[4][f * VPL + c0] - pk[0][f * VPL + c0])) * (1.0 / 12.0);
+                gc[f][2] = fma(8.0, win[f][3] - win[f][1], -(win[f][4] - win[f][0])) * (1.0 / 12.0);
             }
             const int64_t p = at(L, i, j, k);
             const double J = M[p];
@@ -185,7 +220,7 @@ __global__ void __launch_bounds__(VTX * VTY) k_visc_tiled(const double *__restri
 #pragma unroll
                 for (int a = 0; a < 3; a++)
                     gx[f][a] = J * fma(m[0][a], gc[f][0], fma(m[1][a], gc[f][1], m[2][a] * gc[f][2]));
-            const double T = pk[2][3 * VPL + c0];
+            const double T = win[3][2];
             const double mu = mu_of_T(ph, T);
             const double kap = mu * ph.cp_over_Pr;
             const double div = gx[0][0] + gx[1][1] + gx[2][2];
@@ -198,7 +233,7 @@ __global__ void __launch_bounds__(VTX * VTY) k_visc_tiled(const double *__restri
             tau[0][0] -= dterm;
             tau[1][1] -= dterm;
             tau[2][2] -= dterm;
-            const double vel[3] = {pk[2][c0], pk[2][VPL + c0], pk[2][2 * VPL + c0]};
+            const double vel[3] = {win[0][2], win[1][2], win[2][2]};
             double hb[3];
 #pragma unroll
             for (int bb = 0; bb < 3; bb++)
@@ -212,7 +247,6 @@ __global__ void __launch_bounds__(VTX * VTY) k_visc_tiled(const double *__restri
                 FV[(4 * d + 3) * V.cs + o] = fma(m[d][0], hb[0], fma(m[d][1], hb[1], m[d][2] * hb[2]));
             }
         }
-        __syncthreads();
     }
 }
 
