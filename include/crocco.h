@@ -168,6 +168,14 @@ crocco_status crocco_rk_stage(crocco_ctx ctx, int32_t stage, double dt, double *
 crocco_status crocco_rk_update(crocco_ctx ctx, int32_t stage, double dt, double *const *U_in,
                                double *const *U_out, double *const *dU, double *const *rhs);
 
+/* ComputeDt (Eq. 3, 95 Alg. 1 l.9, 131 ReduceRealMin):
+   *dt = cfl / max_i sum_d J_i (|m^d_i . u_i| + c_i |m^d_i|) over the interior points of
+   all blocks of all ranks (global reduction with ncclAllReduce(max) when nranks > 1).
+   U: conserved state (ghosts not read); metrics from crocco_init_metrics; dt: HOST
+   pointer.  Synchronises the stream.  Collective. */
+crocco_status crocco_compute_dt(crocco_ctx ctx, double *const *U, double *const *metrics,
+                                double cfl, double *dt);
+
 /* Block until all work of the ctx finished; surfaces asynchronous errors. */
 crocco_status crocco_sync(crocco_ctx ctx);
 const char *crocco_last_error(crocco_ctx ctx);

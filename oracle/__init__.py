@@ -74,6 +74,8 @@ def lib():
                                       dp, dp, dp, dp]
         L.oracle_advance.argtypes = [i64p, i32p, dp, C.POINTER(Phys), C.c_double, C.c_int32,
                                      dp, dp]
+        L.oracle_compute_dt.argtypes = [i64p, C.POINTER(Phys), dp, dp, C.c_double]
+        L.oracle_compute_dt.restype = C.c_double
         L.oracle_set_threads.argtypes = [C.c_int]
         L.oracle_get_threads.restype = C.c_int
         _lib = L
@@ -168,3 +170,8 @@ def advance(n, bc, ph, dt, nsteps, U, met, dirichlet=None):
     d = _dir(dirichlet)
     lib().oracle_advance(_n(n), _bc(bc), _dp(d), C.byref(ph), dt, nsteps, _dp(U), _dp(met))
     return U
+
+
+def compute_dt(n, ph: Phys, U, met, cfl):
+    """ComputeDt: CFL / max_i sum_d J(|m^d.u| + c|m^d|) (Eq. 3, 95, 131)."""
+    return float(lib().oracle_compute_dt(_n(n), C.byref(ph), _dp(U), _dp(met), float(cfl)))

@@ -686,3 +686,40 @@ void oracle_advance(const int64_t n[3], const int32_t bc[6], const double dirich
     free(V);
     free(dU);
 }
+
+/* ------------------------------------------------------------------ */
+/* 8. ComputeDt (Eq. 3, 95 Alg. 1 l.9, 131, 169;       */
+/*    SURVEY 8(f) NEXT-1): the 1-D CFL condition (|u| + a) dt/dx <= CFL */
+/*    generalised to the curvilinear grid and summed over directions:   */
+/*    dt = CFL / max_i sum_d J_i ( |m^d_i . u_i| + c_i |m^d_i| ).       */
+/*    Interior points only; a global minimum of dt (ReduceRealMin).    */
+/* ------------------------------------------------------------------ */
+double oracle_compute_dt(const int64_t n[3], const oracle_phys *ph, const double *U,
+                         const double *met, double cfl)
+{
+    obox b = make_box(n, OG);
+    const int64_t cs = b.cs;
+    double lam_max = 0.0;
+    for (int64_t k = 0; k < n[2]; k++)
+        for (int64_t j = 0; j < n[1]; j++)
+            for (int64_t i = 0; i < n[0]; i++) {
+                int64_t p = IX(&b, i, j, k);
+                double rho = U[p];
+                double u = U[cs + p] / rho, v = U[2 * cs + p] / rho, w = U[3 * cs + p] / rho;
+                double pres = (ph->gamma - 1.0) * (U[4 * cs + p] - 0.5 * rho * (u * u + v * v + w * w));
+                double c = sqrt(ph->gamma * pres / rho);
+                double s = 0.0;
+                for (int d = 0; d < 3; d++) {
+                    double mx = met[(1 + 3 * d) * cs + p];
+                    double my = met[(2 + 3 * d) * cs + p];
+                    double mz = met[(3 + 3 * d) * cs + p];
+                    double mu = mx * u + my * v + mz * w;
+                    double mm = sqrt(mx * mx + my * my + mz * mz);
+                    s = s + fabs(mu) + c * mm;
+                }
+                s = met[p] * s;
+                if (s > lam_max)
+                    lam_max = s;
+            }
+    return cfl / lam_max;
+}

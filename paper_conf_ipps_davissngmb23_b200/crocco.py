@@ -81,6 +81,7 @@ _SIGS = {
     "crocco_exchange_plan": [C.POINTER(GridDesc), C.c_int32, C.POINTER(Msg), C.c_int32,
                              C.POINTER(C.c_int32)],
     "crocco_nccl_unique_id": [C.c_void_p, C.c_int32],
+    "crocco_compute_dt": [C.c_void_p, DPP, DPP, C.c_double, C.POINTER(C.c_double)],
 }
 _STR = {"crocco_last_error": [C.c_void_p], "crocco_version": [],
         "crocco_kernel_class_name": [C.c_int32]}
@@ -259,3 +260,11 @@ def crocco_nccl_unique_id() -> bytes:
     buf = C.create_string_buffer(128)
     _check(lib().crocco_nccl_unique_id(C.cast(buf, C.c_void_p), 128))
     return buf.raw
+
+
+def crocco_compute_dt(ctx, U_ptrs, met_ptrs, cfl) -> float:
+    a, ka = _ptrs(U_ptrs)
+    b, kb = _ptrs(met_ptrs)
+    dt = C.c_double()
+    _check(lib().crocco_compute_dt(ctx, a, b, float(cfl), C.byref(dt)), ctx)
+    return dt.value

@@ -45,9 +45,10 @@ struct LocalBlock {
     double *fv = nullptr;
 };
 
-enum { K_PRIMS = 0, K_FLUX_X, K_FLUX_Y, K_FLUX_Z, K_VISC, K_UPDATE, K_FILL, K_METRICS, K_NCLASS };
+enum { K_PRIMS = 0, K_FLUX_X, K_FLUX_Y, K_FLUX_Z, K_VISC, K_UPDATE, K_FILL, K_METRICS, K_CFL,
+       K_NCLASS };
 const char *k_names[K_NCLASS] = {"prims", "sweep_xi", "sweep_eta", "sweep_zeta_update", "viscous",
-                                 "update", "fill", "metrics"};
+                                 "update", "fill", "metrics", "compute_dt"};
 
 struct TimedLaunch {
     int cls;
@@ -76,6 +77,7 @@ struct crocco_ctx_s {
     // NCCL
     ncclComm_t comm = nullptr;
     double *send_stage = nullptr, *recv_stage = nullptr;
+    unsigned long long *dmax = nullptr;  // ComputeDt reduction cell
     int64_t stage_elems = 0;
     // timing
     bool timing = false;
@@ -392,6 +394,7 @@ static void free_ctx(crocco_ctx c) {
         cudaFree(b.fv);
     }
     cudaFree(c->send_stage);
+    cudaFree(c->dmax);
     cudaFree(c->recv_stage);
     for (auto &t : c->pending) {
         cudaEventDestroy(t.e0);
@@ -867,6 +870,32 @@ crocco_status crocco_rk_update(crocco_ctx c, int32_t stage, double dt, double *c
         LAUNCH(c, K_UPDATE, k_update<<<grd, 128, 0, c->stream>>>(Uin[bi], Uout[bi], dU[bi], rhs[bi], b.L,
                                                                   stage, RK_A[stage], RK_B[stage], dt));
     }
+    return CROCCO_OK;
+}
+
+crocco_status crocco_compute_dt(crocco_ctx c, double *const *U, double *const *M, double cfl,
+                                double *dt) {
+    LIVE(c);
+    crocco_status st;
+    if ((st = check_ptrs(c, U, "U")) || (st = check_ptrs(c, M, "metrics"))) return st;
+    if (!dt || !(cfl > 0)) return fail(c, CROCCO_ERR_ARG, "need cfl > 0 and a dt pointer");
+    if (!c->dmax) CK(c, cudaMalloc((void **)&c->dmax, sizeof(unsigned long long)));
+    CK(c, cudaMemsetAsync(c->dmax, 0, sizeof(unsigned long long), c->stream));
+    for (size_t bi = 0; bi < c->loc.size(); bi++) {
+        const LocalBlock &b = c->loc[bi];
+        const int64_t tot = (int64_t)b.g.n[0] * b.g.n[1] * b.g.n[2];
+        const unsigned grid = (unsigned)std::min<int64_t>(cdiv(tot, 256), 148 * 8);
+        LAUNCH(c, K_CFL, k_cfl<<<grid, 256, 0, c->stream>>>(U[bi], M[bi], b.L, c->ph, c->dmax));
+    }
+    if (c->comm)  // global max over ranks (the bit pattern is the double itself)
+        NK(c, ncclAllReduce(c->dmax, c->dmax, 1, ncclFloat64, ncclMax, c->comm, c->stream));
+    unsigned long long h = 0;
+    CK(c, cudaMemcpyAsync(&h, c->dmax, sizeof h, cudaMemcpyDeviceToHost, c->stream));
+    CK(c, cudaStreamSynchronize(c->stream));
+    double lam;
+    memcpy(&lam, &h, sizeof lam);
+    if (!(lam > 0)) return fail(c, CROCCO_ERR_ARG, "non-positive spectral radius (state not set?)");
+    *dt = cfl / lam;
     return CROCCO_OK;
 }
 

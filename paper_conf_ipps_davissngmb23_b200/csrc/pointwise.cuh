@@ -250,6 +250,47 @@ __global__ void __launch_bounds__(VTX * VTY) k_visc_tiled(const double *__restri
     }
 }
 
+// ComputeDt (Eq. 3, 95 Alg. 1 l.9, 131, 169):
+// lambda_i = J_i sum_d (|m^d_i . u_i| + c_i |m^d_i|) on interior points, maximum
+// over the block by warp shuffles + shared memory, over blocks/launches by
+// atomicMax on the 64-bit pattern (non-negative doubles order like their bit
+// patterns, so the result is exact and independent of the reduction order).
+__global__ void __launch_bounds__(256) k_cfl(const double *__restrict__ U, const double *__restrict__ M,
+                                             Lay L, Phys ph, unsigned long long *__restrict__ out) {
+    __shared__ double red[8];
+    const int64_t tot = (int64_t)L.n0 * L.n1 * L.n2;
+    double lmax = 0.0;
+    for (int64_t t = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; t < tot;
+         t += (int64_t)gridDim.x * blockDim.x) {
+        const int i = (int)(t % L.n0);
+        const int64_t r = t / L.n0;
+        const int j = (int)(r % L.n1), k = (int)(r / L.n1);
+        const int64_t p = at(L, i, j, k);
+        const double rho = U[p];
+        const double ir = 1.0 / rho;
+        const double u = U[L.cs + p] * ir, v = U[2 * L.cs + p] * ir, w = U[3 * L.cs + p] * ir;
+        const double pr = ph.gm1 * (U[4 * L.cs + p] - 0.5 * rho * fma(u, u, fma(v, v, w * w)));
+        const double c = sqrt(ph.gamma * pr * ir);
+        double sum = 0.0;
+#pragma unroll
+        for (int d = 0; d < 3; d++) {
+            const double mx = M[(1 + 3 * d) * L.cs + p], my = M[(2 + 3 * d) * L.cs + p],
+                         mz = M[(3 + 3 * d) * L.cs + p];
+            sum += fabs(fma(mx, u, fma(my, v, mz * w))) + c * sqrt(fma(mx, mx, fma(my, my, mz * mz)));
+        }
+        lmax = fmax(lmax, M[p] * sum);
+    }
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) lmax = fmax(lmax, __shfl_xor_sync(0xffffffffu, lmax, o));
+    if ((threadIdx.x & 31) == 0) red[threadIdx.x >> 5] = lmax;
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        double m = red[0];
+        for (int w = 1; w < (int)(blockDim.x >> 5); w++) m = fmax(m, red[w]);
+        atomicMax(out, (unsigned long long)__double_as_longlong(m));
+    }
+}
+
 // Update alone, from a materialised rhs (crocco_rk_update).
 __global__ void __launch_bounds__(256) k_update(const double *__restrict__ Uin,
                                                 double *__restrict__ Uout, double *__restrict__ dU,

@@ -108,6 +108,10 @@ class Solver:
             for s in range(3):
                 self.stage(s, dt)
 
+    def compute_dt(self, cfl):
+        """ComputeDt (Alg. 1 l.9): CFL time step of the current state (synchronises)."""
+        return cc.crocco_compute_dt(self.ctx, self._ptrs(self.U), self._ptrs(self.met), cfl)
+
     def set_phys(self, phys):
         self.phys = phys
         cc.crocco_set_phys(self.ctx, phys)

@@ -305,3 +305,30 @@ def test_full_size_weak_config_sampled():
             worst = max(worst, float(np.abs(gU - Uo[:, 4, 4, 4]).max() / np.abs(Uo[:, 4, 4, 4]).max()))
         assert worst < 1e-11, (stage, worst)
     S.close()
+
+
+# ------------------------------------------------------------------ ComputeDt (NEXT-1)
+
+@pytest.mark.parametrize("nb", [(1, 1, 1), (2, 3, 2)])
+def test_compute_dt_parity(nb):
+    n = (36, 30, 20)
+    pb = wavy_random(n, 23)
+    _, met, U = pb.oracle_inputs()
+    ref = oracle.compute_dt(n, pb.oracle_phys(), U, met, 0.7)
+    S = pb.solver(nb)
+    got = S.compute_dt(0.7)
+    S.close()
+    assert abs(got - ref) <= 1e-13 * ref, (got, ref)
+
+
+def test_compute_dt_sod_closed_form():
+    # Sod initial state on the Cartesian 1/200 grid: max over the two states of
+    # sum_d (|u_d| + c)/h = 3 c_L / h (u = 0), c_L = sqrt(1.4)
+    c = synth.case("sod")
+    xyz = c.grid.coords(c.n_global, (0, 0, 0), oracle.GC)
+    pb = Problem(c.n_global, c.grid, c.bc, synth.sod(xyz), c.phys)
+    S = pb.solver()
+    got = S.compute_dt(0.9)
+    S.close()
+    expect = 0.9 / (3 * math.sqrt(1.4) * 200)
+    assert abs(got - expect) < 1e-12 * expect

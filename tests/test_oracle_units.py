@@ -417,3 +417,42 @@ def test_williamson_stage_times_second_order_conditions():
             oracle.rk_update(n, s, dt, a, o, dU, r)
             a, o = o, a
         assert abs(a[0, 4, 4, 4] - dt ** (deg + 1) / (deg + 1)) < 1e-15
+
+
+# ------------------------------------------------------------------ ComputeDt (Eq. 3; NEXT-1)
+
+def test_compute_dt_cartesian_closed_form():
+    # uniform state on a Cartesian grid: dt = CFL / sum_d (|u_d| + c)/h_d  (Eq. 3 per direction)
+    n = (6, 5, 4)
+    h = (0.1, 0.2, 0.05)
+    grid = synth.Cartesian(h=h)
+    xyz = grid.coords(n, (0, 0, 0), 10)
+    met = oracle.metrics(n, ((0, 0),) * 3, xyz)
+    vel = (0.3, -0.7, 0.2)
+    U = synth.pad_state(synth.free_stream(xyz, rho=1.3, vel=vel, p=0.9))
+    c = math.sqrt(1.4 * 0.9 / 1.3)
+    expect = 0.8 / sum((abs(vel[d]) + c) / h[d] for d in range(3))
+    got = oracle.compute_dt(n, oracle.phys(), U, met, 0.8)
+    assert abs(got - expect) < 1e-13 * expect
+
+
+def test_compute_dt_affine_grid_via_matrix_inverse():
+    # affine grid x = A xi: d xi_d/d x_a = inv(A)[d, a]; the spectral radius of
+    # the contravariant flux Jacobian of direction d is |grad xi_d . u| + c |grad xi_d|
+    A = np.array([[0.9, 0.2, -0.1], [0.15, 1.1, 0.05], [-0.2, 0.1, 0.8]])
+    n = (5, 5, 5)
+    xyz = _Affine(A, [0.0, 0.0, 0.0]).coords(n, (0, 0, 0), 10)
+    met = oracle.metrics(n, ((1, 1),) * 3, xyz)
+    rng = np.random.default_rng(11)
+    Ui = synth.random_state(n, seed=12)
+    U = synth.pad_state(Ui)
+    gradxi = np.linalg.inv(A)                      # rows: grad xi_d
+    rho = Ui[0]
+    vel = Ui[1:4] / rho
+    p = 0.4 * (Ui[4] - 0.5 * rho * (vel ** 2).sum(0))
+    c = np.sqrt(1.4 * p / rho)
+    lam = sum(np.abs(np.einsum("a,a...->...", gradxi[d], vel)) + c * np.linalg.norm(gradxi[d])
+              for d in range(3))
+    expect = 0.5 / lam.max()
+    got = oracle.compute_dt(n, oracle.phys(), U, met, 0.5)
+    assert abs(got - expect) < 1e-13 * expect
