@@ -51,11 +51,16 @@ struct GAcc {  // straight from the global arrays (L1/L2 cached)
     __device__ __forceinline__ double P(int l, int k) const { return p[k * cs + p0 + l * s]; }
     __device__ __forceinline__ double M(int l, int a) const { return m[a * cs + p0 + l * s]; }
     __device__ __forceinline__ double FV(int l, int q) const { return fv[q * vcs + v0 + l * vs]; }
+    __device__ __forceinline__ double SR(int l) const { return P(l, PSR); }  // sqrt(rho)
+    __device__ __forceinline__ double H(int l) const { return P(l, PH); }    // total enthalpy
 };
 
 // shared-memory ring of a warp: value v of ring point q in column col at
 // sv[v * VS + (q & (NR-1)) * PS + col]
-enum { SV_U = 0, SV_M = 5, SV_FV = 8, SV_P = 12, SV_N = 19 };
+#ifndef CROCCO_RING_LEAN
+#define CROCCO_RING_LEAN 0  // 1: stage u v w p c only; sqrt(rho), H derived per interface
+#endif
+enum { SV_U = 0, SV_M = 5, SV_FV = 8, SV_P = 12, SV_N = CROCCO_RING_LEAN ? 17 : 19 };
 template <int NR, int PS>
 struct SAcc {
     const double *sv;
@@ -68,6 +73,13 @@ struct SAcc {
     __device__ __forceinline__ double P(int l, int k) const { return at_(SV_P + k, l); }
     __device__ __forceinline__ double M(int l, int a) const { return at_(SV_M + a, l); }
     __device__ __forceinline__ double FV(int l, int q) const { return at_(SV_FV + q, l); }
+#if CROCCO_RING_LEAN
+    __device__ __forceinline__ double SR(int l) const { return U(l, 0) * rsqrt_nr(U(l, 0)); }
+    __device__ __forceinline__ double H(int l) const { return (U(l, 4) + P(l, PP)) * rcp_nr(U(l, 0)); }
+#else
+    __device__ __forceinline__ double SR(int l) const { return P(l, PSR); }
+    __device__ __forceinline__ double H(int l) const { return P(l, PH); }
+#endif
 };
 
 // Total interface flux F = F^_inv - h_v of direction D at interface i+1/2.
@@ -89,13 +101,13 @@ __device__ __forceinline__ void total_flux(const Acc &A, bool inv, bool visc, co
         const double nx = mh[0] * imag, ny = mh[1] * imag, nz = mh[2] * imag;
 
         // Roe average of points i (l=2), i+1 (l=3), sqrt(rho) weights
-        const double srL = A.P(2, PSR), srR = A.P(3, PSR);
+        const double srL = A.SR(2), srR = A.SR(3);
         const double iden = rcp_nr(srL + srR);
         const double wL = srL * iden, wR = srR * iden;
         const double ut = fma(wL, A.P(2, PU), wR * A.P(3, PU));
         const double vt = fma(wL, A.P(2, PV), wR * A.P(3, PV));
         const double wt = fma(wL, A.P(2, PW), wR * A.P(3, PW));
-        const double Ht = fma(wL, A.P(2, PH), wR * A.P(3, PH));
+        const double Ht = fma(wL, A.H(2), wR * A.H(3));
         const double rt = srL * srR;
         const double q2 = fma(ut, ut, fma(vt, vt, wt * wt));
         const double c2 = gm1 * fma(-0.5, q2, Ht);

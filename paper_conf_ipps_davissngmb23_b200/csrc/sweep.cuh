@@ -25,7 +25,10 @@ namespace crocco {
 #ifndef CROCCO_SWEEP_MINB
 #define CROCCO_SWEEP_MINB 1  // min CTAs/SM (register cap); the staged ring allows 2 CTAs x 4 warps
 #endif
-constexpr int SWEEP_THREADS = 128;
+#ifndef CROCCO_SWEEP_THREADS
+#define CROCCO_SWEEP_THREADS 128
+#endif
+constexpr int SWEEP_THREADS = CROCCO_SWEEP_THREADS;
 
 struct SweepArgs {
     FluxIn in;
@@ -302,8 +305,10 @@ __global__ void __launch_bounds__(SWEEP_THREADS, CROCCO_SWEEP_MINB) k_sweep_s(co
         bq[(SV_P + PW) * VS] = w;
         bq[(SV_P + PP) * VS] = pr;
         bq[(SV_P + PC) * VS] = sqrt_nr(ph.gamma * pr * ir);
+#if !CROCCO_RING_LEAN
         bq[(SV_P + PSR) * VS] = sqrt_nr(rho);
         bq[(SV_P + PH) * VS] = (E + pr) * ir;
+#endif
     };
 
     // prologue: chunks 0 .. LA staged with primitives

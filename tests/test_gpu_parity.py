@@ -258,52 +258,69 @@ def test_rk3_100_steps_parity(name):
 
 # ------------------------------------------------------------------ full size, sampled
 
+def _block_points(bn, rng, k_random):
+    """Sampled interior points of a block: random ones plus corners, edges and faces."""
+    pts = [tuple(int(rng.integers(0, m)) for m in bn) for _ in range(k_random)]
+    hi = [m - 1 for m in bn]
+    pts += [(0, 0, 0), tuple(hi), (0, hi[1], 3 % bn[2]), (hi[0], 0, hi[2]), (1, 2, hi[2] - 1),
+            (hi[0] - 1, 5 % bn[1], 0), (bn[0] // 2, 0, hi[2]), (hi[0], bn[1] // 2, 0)]
+    return pts
+
+
 @pytest.mark.slow
-def test_full_size_weak_config_sampled():
-    """512^3 weak-scaling config, rk_stage in bench.py's launch configuration;
-    64 sampled points recomputed by the oracle one by one from the GPU's
-    filled neighbourhood (9^3 window of U and metrics)."""
-    torch = _torch_cuda()
-    c = synth.case("weak")
+@pytest.mark.parametrize("name", ["weak", "ramp"])
+def test_full_size_config_sampled(name):
+    """BASELINE.json full sizes in bench.py's launch configuration (crocco_rk_stage):
+    weak = 512^3 periodic wavy TGV (configs[4]); ramp = 1024 x 512 x 256 Mach-6
+    ramp in 2 x 2 x 2 blocks with walls (configs[3]).  Stages 0 and 1; sampled
+    points recomputed by the oracle one by one from the GPU's filled 9^3
+    neighbourhood of U and metrics (plus the stage-1 dU)."""
+    _torch_cuda()
+    c = synth.case(name)
     n = c.n_global
     from paper_conf_ipps_davissngmb23_b200 import crocco as cc
     from paper_conf_ipps_davissngmb23_b200.solver import Solver
     S = Solver(n, c.n_blocks, c.bc, cc.make_phys(**c.phys))
-    xyz, U0 = synth.block_inputs(c, (0, 0, 0), n)
-    S.set_coords([xyz])
-    S.set_state([U0])
+    bn, blocks = block_slices(n, c.n_blocks)
+    xyz = []
+    U0 = []
+    for o, _ in blocks:
+        x, u = synth.block_inputs(c, o, bn)
+        xyz.append(x)
+        U0.append(u)
+    S.set_coords(xyz)
+    S.set_state(U0)
     del xyz, U0
     rng = np.random.default_rng(0)
-    pts = [tuple(rng.integers(0, m) for m in n) for _ in range(56)]
-    pts += [(0, 0, 0), (n[0] - 1, n[1] - 1, n[2] - 1), (0, n[1] - 1, 3), (n[0] - 1, 0, n[2] - 1),
-            (1, 2, n[2] - 2), (n[0] - 2, 5, 0), (255, 0, 511), (511, 256, 0)]
+    per_block = max(8, 64 // len(blocks))
+    pts = [(b, p) for b in range(len(blocks)) for p in _block_points(bn, rng, per_block)]
     ph = oracle.phys(**c.phys)
     for stage in (0, 1):
-        Uin_buf, dU_buf = S.U[0], S.dU[0]
-        dU_before = {p: S.view(dU_buf, 0, 5)[:, p[2] + 4, p[1] + 4, p[0] + 4].cpu().numpy()
-                     for p in pts}
+        Uin_bufs, dU_bufs = list(S.U), list(S.dU)
+        dU_before = {(b, p): S.view(dU_bufs[b], b, 5)[:, p[2] + 4, p[1] + 4, p[0] + 4].cpu().numpy()
+                     for b, p in pts}
         S.stage(stage, c.dt)
         S.sync()
-        Uin = S.view(Uin_buf, 0, 5)
-        Uout = S.view(S.U[0], 0, 5)
-        dUv = S.view(dU_buf, 0, 5)
-        M = S.view(S.met[0], 0, 10)
         worst = 0.0
-        for p in pts:
+        for b, p in pts:
+            Uin = S.view(Uin_bufs[b], b, 5)
+            Uout = S.view(S.U[b], b, 5)
+            dUv = S.view(dU_bufs[b], b, 5)
+            M = S.view(S.met[b], b, 10)
             sl = (slice(None), slice(p[2], p[2] + 9), slice(p[1], p[1] + 9), slice(p[0], p[0] + 9))
             Uw = np.ascontiguousarray(Uin[sl].cpu().numpy())
             Mw = np.ascontiguousarray(M[sl].cpu().numpy())
             r = oracle.rhs((1, 1, 1), ph, Uw, Mw)
             Uo = np.zeros_like(Uw)
             dUo = np.zeros_like(Uw)
-            dUo[:, 4, 4, 4] = dU_before[p]
+            dUo[:, 4, 4, 4] = dU_before[(b, p)]
             oracle.rk_update((1, 1, 1), stage, c.dt, Uw, Uo, dUo, r)
             gU = Uout[:, p[2] + 4, p[1] + 4, p[0] + 4].cpu().numpy()
             gd = dUv[:, p[2] + 4, p[1] + 4, p[0] + 4].cpu().numpy()
             scale = flux_scale(Uw, Mw) * c.dt
             worst = max(worst, float(np.abs(gd - dUo[:, 4, 4, 4]).max() / max(np.abs(dUo[:, 4, 4, 4]).max(), scale)))
             worst = max(worst, float(np.abs(gU - Uo[:, 4, 4, 4]).max() / np.abs(Uo[:, 4, 4, 4]).max()))
-        assert worst < 1e-11, (stage, worst)
+        assert worst < 1e-11, (name, stage, worst)
     S.close()
 
 
