@@ -42,6 +42,15 @@ FP64_PEAK_TFLOPS = 148 * 64 * 2 * 1.965e9 / 1e12
 HBM_BYTES_PER_PT_STAGE = (200 + 240 + 240) / 3.0
 
 
+WORKLOADS = {
+    "weak": f"weak: {N_BLOCK}^3/GPU periodic curvilinear TGV+noise, viscous (BASELINE.json configs[4])",
+    "ramp": "ramp: Mach-6 compression ramp 1024x512x256 in 2x2x2 blocks, walls, Sutherland (configs[3])",
+    "tgv": "tgv: Taylor-Green vortex 256^3 on the wavy grid, viscous (configs[2])",
+    "vortex": "vortex: isentropic vortex on the wavy periodic 64^3 grid, inviscid (configs[1])",
+    "sod": "sod: Sod shock tube 200x4x4, inviscid (configs[0])",
+}
+
+
 def weak_grid(n):
     return {1: (1, 1, 1), 2: (2, 1, 1), 4: (2, 2, 1), 8: (2, 2, 2)}.get(n) or _factor3(n)
 
@@ -185,9 +194,6 @@ def run_crocco(args, rank, world, local_rank):
 
     torch.cuda.set_device(local_rank)
     dev = torch.device("cuda", local_rank)
-    a, b, c = weak_grid(world)
-    nb = (a, b, c)
-    n = (N_BLOCK * a, N_BLOCK * b, N_BLOCK * c)
     uid = None
     if world > 1:
         t = torch.zeros(128, dtype=torch.uint8, device=dev)
@@ -195,50 +201,86 @@ def run_crocco(args, rank, world, local_rank):
             t.copy_(torch.frombuffer(bytearray(cc.crocco_nccl_unique_id()), dtype=torch.uint8))
         dist.broadcast(t, 0)
         uid = bytes(t.cpu().numpy().tobytes())
-    grid = synth.Wavy3D(L=(2 * math.pi * a, 2 * math.pi * b, 2 * math.pi * c), N=n,
-                        x0=(-math.pi,) * 3, k=2.0, A=0.15)
-    phys = dict(gamma=1.4, R=1.0, Pr=0.71, mu_ref=1.0 / 1600.0, terms=3)
-    dt = 2e-4
-    S = Solver(n, nb, ((0, 0),) * 3, cc.make_phys(**phys), rank=rank, nranks=world,
-               block_rank=list(range(world)), device=dev, nccl_unique_id=uid)
-    L = S.layouts[0]
-    origin = tuple(L.origin)
-    bn = tuple(L.n)
-    xyz = torch.from_numpy(grid.coords(bn, origin, cc.GHOST_COORDS)).to(dev)
-    S.set_coords([xyz])
-    U0 = synth.tgv(xyz, noise=0.01, seed=5)
-    del xyz
-    S.set_state([U0])
-    del U0
+    if args.config == "weak":
+        # weak scaling: 512^3 per GPU, one block per rank (BASELINE.json configs[4])
+        a, b, c = weak_grid(world)
+        nb = (a, b, c)
+        n = (N_BLOCK * a, N_BLOCK * b, N_BLOCK * c)
+        grid = synth.Wavy3D(L=(2 * math.pi * a, 2 * math.pi * b, 2 * math.pi * c), N=n,
+                            x0=(-math.pi,) * 3, k=2.0, A=0.15)
+        phys = dict(gamma=1.4, R=1.0, Pr=0.71, mu_ref=1.0 / 1600.0, terms=3)
+        dt, bc, state = 2e-4, ((0, 0),) * 3, "tgv_noise"
+        block_rank = list(range(world))
+        case = synth.Case("weak", n, nb, bc, grid, state, phys, dt)
+    else:
+        # fixed global problem (strong scaling for N > 1): configs[0..3]
+        case = synth.case(args.config)
+        n, nb, bc, grid, phys, dt = case.n_global, case.n_blocks, case.bc, case.grid, case.phys, case.dt
+        nbt = nb[0] * nb[1] * nb[2]
+        block_rank = [bb * world // nbt for bb in range(nbt)]
+    S = Solver(n, nb, bc, cc.make_phys(**phys), rank=rank, nranks=world,
+               block_rank=block_rank, device=dev, nccl_unique_id=uid)
+    for bl in range(S.nloc):
+        L = S.layouts[bl]
+        origin, bn = tuple(L.origin), tuple(L.n)
+        if case.state in ("tgv", "tgv_noise"):
+            # generated on the device (torch ops on the synth formulas) -- input setup only
+            xyz = torch.from_numpy(grid.coords(bn, origin, cc.GHOST_COORDS)).to(dev)
+            U0 = synth.tgv(xyz, noise=0.01 if case.state == "tgv_noise" else 0.0, seed=5)
+        else:
+            xyz, U0 = synth.block_inputs(case, origin, bn)
+        S.set_coords_block(bl, xyz)
+        S.set_state_block(bl, U0)
+        del xyz, U0
+    pts_local = sum(L.n[0] * L.n[1] * L.n[2] for L in S.layouts)
+    pts_total = n[0] * n[1] * n[2]
+    bn = tuple(S.layouts[0].n)
     torch.cuda.synchronize()
     stream = S.stream
-    pts_local = bn[0] * bn[1] * bn[2]
-    pts_total = n[0] * n[1] * n[2]
 
     for _ in range(args.warmup):
         S.step(dt)
     torch.cuda.synchronize()
 
     # ---------------- timed region (device-resident inputs)
-    cc.crocco_set_timing(S.ctx, True)
+    state_bytes = sum(u.numel() for u in S.U) * 8
+    flush = state_bytes < 4 * 126e6  # small configs: flush L2 between timed steps
+    # kernel-class CUDA events inside the timed region for the large (non-graph) workloads;
+    # small launch-bound configs run CUDA-graph steps and get their breakdown afterwards
+    cc.crocco_set_timing(S.ctx, not flush)
     cc.crocco_kernel_times(S.ctx)          # reset accumulators
     cc.crocco_launch_count(S.ctx, reset=True)
     clk = ClockSampler(local_rank) if not args.no_clocks else None
-    e0 = torch.cuda.Event(enable_timing=True)
-    e1 = torch.cuda.Event(enable_timing=True)
+    scratch = torch.empty(int(256e6) // 8, dtype=torch.float64, device=dev) if flush else None
+    evs = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True))
+           for _ in range(args.steps if flush else 1)]
     if world > 1:
         dist.barrier()
     torch.cuda.synchronize()
-    e0.record(stream)
-    for _ in range(args.steps):
-        S.step(dt)
-    e1.record(stream)
+    if flush:
+        for e0, e1 in evs:
+            scratch.fill_(1.0)               # 256 MB write evicts L2 (outside the timed events)
+            e0.record(stream)
+            S.step(dt)
+            e1.record(stream)
+    else:
+        e0, e1 = evs[0]
+        e0.record(stream)
+        for _ in range(args.steps):
+            S.step(dt)
+        e1.record(stream)
     torch.cuda.synchronize()
     if world > 1:
         dist.barrier()
-    ms_local = e0.elapsed_time(e1)
+    ms_local = sum(a_.elapsed_time(b_) for a_, b_ in evs)
     clocks = clk.stop() if clk else None
     launches = cc.crocco_launch_count(S.ctx)
+    if flush:  # breakdown pass (eager launches with events) after the graph-timed region
+        cc.crocco_set_timing(S.ctx, True)
+        cc.crocco_kernel_times(S.ctx)
+        for _ in range(args.steps):
+            S.step(dt)
+        torch.cuda.synchronize()
     ktimes = cc.crocco_kernel_times(S.ctx)
     cc.crocco_set_timing(S.ctx, False)
     t = torch.tensor([ms_local], dtype=torch.float64, device=dev)
@@ -247,14 +289,17 @@ def run_crocco(args, rank, world, local_rank):
     ms = float(t.item())
     value = pts_total * 3 * args.steps / (ms / 1e3)
     # state sanity (finite, positive density) -- not part of the timed region
-    Ui = S.view(S.U[0], 0, 5)[:, 4:-4, 4:-4, 4:-4]
-    finite = bool(torch.isfinite(Ui).all().item()) and float(Ui[0].min().item()) > 0
+    finite = True
+    for bl in range(S.nloc):
+        Ui = S.view(S.U[bl], bl, 5)[:, 4:-4, 4:-4, 4:-4]
+        finite = finite and bool(torch.isfinite(Ui).all().item()) and float(Ui[0].min().item()) > 0
 
     # ---------------- end-to-end through the public API with host buffers
     e2e = None
     if args.e2e_steps > 0:
-        host = torch.empty(S.U[0].numel(), dtype=torch.float64, pin_memory=True)
-        host.copy_(S.U[0])
+        hosts = [torch.empty(u.numel(), dtype=torch.float64, pin_memory=True) for u in S.U]
+        for h, u in zip(hosts, S.U):
+            h.copy_(u)
         torch.cuda.synchronize()
         if world > 1:
             dist.barrier()
@@ -262,17 +307,23 @@ def run_crocco(args, rank, world, local_rank):
         f1 = torch.cuda.Event(enable_timing=True)
         f0.record(stream)
         for _ in range(args.e2e_steps):
-            S.U[0].copy_(host, non_blocking=True)      # H2D of the step's input state
+            for h, u in zip(hosts, S.U):
+                u.copy_(h, non_blocking=True)      # H2D of the step's input state
             S.step(dt)
-            host.copy_(S.U[0], non_blocking=True)      # D2H of the step's result
+            for h, u in zip(hosts, S.U):
+                h.copy_(u, non_blocking=True)      # D2H of the step's result
         f1.record(stream)
         torch.cuda.synchronize()
         te = torch.tensor([f0.elapsed_time(f1)], dtype=torch.float64, device=dev)
         if world > 1:
             dist.all_reduce(te, op=dist.ReduceOp.MAX)
-        nbytes = host.numel() * 8
+        nbytes = sum(h.numel() for h in hosts) * 8
+        if world > 1:
+            tb = torch.tensor([nbytes], dtype=torch.float64, device=dev)
+            dist.all_reduce(tb)
+            nbytes = int(tb.item())
         e2e = {"value": pts_total * 3 * args.e2e_steps / (float(te.item()) / 1e3), "unit": UNIT,
-               "h2d_bytes_per_step": nbytes * world, "d2h_bytes_per_step": nbytes * world,
+               "h2d_bytes_per_step": nbytes, "d2h_bytes_per_step": nbytes,
                "steps": args.e2e_steps}
 
     # ---------------- roofline of the dominant kernel (CUDA events on the launching stream)
@@ -283,7 +334,7 @@ def run_crocco(args, rank, world, local_rank):
     roof = None
     if name in flux_cls:
         d = flux_cls[name]
-        ifaces = (bn[d] + 1) * pts_local // bn[d]
+        ifaces = (bn[d] + 1) * (bn[0] * bn[1] * bn[2]) // bn[d]  # per launch (one block)
         ach = FLUX_FLOPS_PER_IFACE * ifaces / (avg_ms / 1e3) / 1e12
         roof = {"bound": "alu", "kernel": f"k_sweep_s<{d}> ({name})", "achieved": ach,
                 "peak": FP64_PEAK_TFLOPS, "unit": "TFLOP/s", "frac": ach / FP64_PEAK_TFLOPS,
@@ -295,17 +346,20 @@ def run_crocco(args, rank, world, local_rank):
     peaks = measured_peaks()
     hbm = peaks.get("hbm_gbs", 6650.0)
     stage_gbs = value / world * HBM_BYTES_PER_PT_STAGE / 1e9
-    breakdown = {k: {"launches": v[0], "ms": v[1], "share": v[1] / max(ms_local, 1e-9)}
+    ktot = sum(v[1] for v in ktimes.values())
+    breakdown = {k: {"launches": v[0], "ms": v[1], "share_of_kernel_time": v[1] / max(ktot, 1e-9)}
                  for k, v in ktimes.items() if v[0]}
     out = {"metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
            "warmup": args.warmup, "ms_per_step": ms / args.steps, "higher_is_better": True,
-           "scaling": "weak", "vs_baseline": None, "dtype": "f64",
-           "data": "synthetic (seeded wavy periodic grid, TGV + 1% smooth noise)",
-           "config": {"workload": f"weak: {N_BLOCK}^3/GPU periodic curvilinear TGV+noise, viscous "
-                                  f"(BASELINE.json configs[4]); step = 1 RK3 step (3 stages)",
+           "scaling": "weak" if args.config == "weak" else "strong", "vs_baseline": None, "dtype": "f64",
+           "data": "synthetic (seeded, " + WORKLOADS[args.config].split(":")[0] + " recipe of DESIGN.md sec. 4)",
+           "config": {"workload": WORKLOADS[args.config] + "; step = 1 RK3 step (3 stages)",
                       "n_global": list(n), "n_blocks": list(nb), "points_per_gpu": pts_local,
-                      "dt": dt, "l2": "inputs larger than L2 (5.9 GB state per GPU vs 126 MB L2)",
-                      "parallelism": f"spatial blocks {a}x{b}x{c}, NCCL halo exchange"},
+                      "dt": dt,
+                      "l2": ("L2 flushed (256 MB write) between timed steps" if flush else
+                             f"inputs larger than L2 ({state_bytes / 1e9:.1f} GB state vs 126 MB L2)"),
+                      "parallelism": f"spatial blocks {nb[0]}x{nb[1]}x{nb[2]} over {world} GPU(s), "
+                                     "NCCL halo exchange"},
            "roofline": roof,
            "hbm": {"algorithmic_gbs_per_gpu": stage_gbs, "peak_gbs": hbm,
                    "frac": stage_gbs / hbm, "bytes_per_point_stage": HBM_BYTES_PER_PT_STAGE,
@@ -337,6 +391,8 @@ def main():
     ap.add_argument("--steps", type=int, default=5)
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--impl", choices=["crocco", "reference"], default="crocco")
+    ap.add_argument("--config", choices=["weak", "ramp", "tgv", "vortex", "sod"], default="weak",
+                    help="weak (default, the north_star 512^3/GPU workload) or a fixed BASELINE config")
     ap.add_argument("--e2e-steps", type=int, default=2)
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-clocks", action="store_true")

@@ -164,6 +164,15 @@ crocco_status crocco_rk_stage(crocco_ctx ctx, int32_t stage, double dt, double *
                               double *const *U_out, double *const *dU,
                               double *const *metrics);
 
+/* One full RK3 time step (Alg. 2 l.1: stages 1..3) = crocco_rk_stage(0: U -> V),
+   (1: V -> U), (2: U -> V): the new state is in V, U was used for the middle stage.
+   use_graph != 0: the three stages (fills, sweeps, update: ~20 kernels) are captured
+   once per (U, V, dU, metrics, dt) into a CUDA graph and replayed with one launch
+   (at most 4 graphs cached per ctx; eager launches when kernel timing is on or
+   nranks > 1).  Collective. */
+crocco_status crocco_rk3_step(crocco_ctx ctx, double dt, double *const *U, double *const *V,
+                              double *const *dU, double *const *metrics, int32_t use_graph);
+
 /* The Update step alone (tests): dU <- A_s dU + dt rhs ; U_out = U_in + B_s dU. */
 crocco_status crocco_rk_update(crocco_ctx ctx, int32_t stage, double dt, double *const *U_in,
                                double *const *U_out, double *const *dU, double *const *rhs);

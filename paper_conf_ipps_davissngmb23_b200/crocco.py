@@ -82,6 +82,7 @@ _SIGS = {
                              C.POINTER(C.c_int32)],
     "crocco_nccl_unique_id": [C.c_void_p, C.c_int32],
     "crocco_compute_dt": [C.c_void_p, DPP, DPP, C.c_double, C.POINTER(C.c_double)],
+    "crocco_rk3_step": [C.c_void_p, C.c_double, DPP, DPP, DPP, DPP, C.c_int32],
 }
 _STR = {"crocco_last_error": [C.c_void_p], "crocco_version": [],
         "crocco_kernel_class_name": [C.c_int32]}
@@ -268,3 +269,11 @@ def crocco_compute_dt(ctx, U_ptrs, met_ptrs, cfl) -> float:
     dt = C.c_double()
     _check(lib().crocco_compute_dt(ctx, a, b, float(cfl), C.byref(dt)), ctx)
     return dt.value
+
+
+def crocco_rk3_step(ctx, dt, U_ptrs, V_ptrs, dU_ptrs, met_ptrs, use_graph=True):
+    a, ka = _ptrs(U_ptrs)
+    b, kb = _ptrs(V_ptrs)
+    c, kc = _ptrs(dU_ptrs)
+    d, kd = _ptrs(met_ptrs)
+    _check(lib().crocco_rk3_step(ctx, float(dt), a, b, c, d, int(use_graph)), ctx)

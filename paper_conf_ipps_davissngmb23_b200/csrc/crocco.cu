@@ -78,6 +78,15 @@ struct crocco_ctx_s {
     ncclComm_t comm = nullptr;
     double *send_stage = nullptr, *recv_stage = nullptr;
     unsigned long long *dmax = nullptr;  // ComputeDt reduction cell
+    // CUDA graphs of full RK3 steps, keyed by (buffers, dt)
+    struct StepGraph {
+        std::vector<const void *> key;
+        double dt;
+        cudaGraphExec_t exec;
+        int64_t nodes;
+    };
+    std::vector<StepGraph> graphs;
+    cudaStream_t cap_stream = nullptr;
     int64_t stage_elems = 0;
     // timing
     bool timing = false;
@@ -401,6 +410,8 @@ static void free_ctx(crocco_ctx c) {
         cudaEventDestroy(t.e1);
     }
     for (auto e : c->pool) cudaEventDestroy(e);
+    for (auto &g : c->graphs) cudaGraphExecDestroy(g.exec);
+    if (c->cap_stream) cudaStreamDestroy(c->cap_stream);
     if (c->comm) ncclCommDestroy(c->comm);
     delete c;
 }
@@ -853,6 +864,68 @@ crocco_status crocco_rk_stage(crocco_ctx c, int32_t stage, double dt, double *co
                             dt)))
             return st;
     }
+    return CROCCO_OK;
+}
+
+static crocco_status rk3_eager(crocco_ctx c, double dt, double *const *U, double *const *V,
+                               double *const *dU, double *const *M) {
+    crocco_status st;
+    if ((st = crocco_rk_stage(c, 0, dt, U, V, dU, M))) return st;
+    if ((st = crocco_rk_stage(c, 1, dt, V, U, dU, M))) return st;
+    return crocco_rk_stage(c, 2, dt, U, V, dU, M);
+}
+
+crocco_status crocco_rk3_step(crocco_ctx c, double dt, double *const *U, double *const *V,
+                              double *const *dU, double *const *M, int32_t use_graph) {
+    LIVE(c);
+    crocco_status st;
+    if ((st = check_ptrs(c, U, "U")) || (st = check_ptrs(c, V, "V")) || (st = check_ptrs(c, dU, "dU")) ||
+        (st = check_ptrs(c, M, "metrics")))
+        return st;
+    if (!use_graph || c->timing || c->desc.nranks > 1 || c->stream == nullptr)
+        return rk3_eager(c, dt, U, V, dU, M);
+    std::vector<const void *> key;
+    for (size_t b = 0; b < c->loc.size(); b++) {
+        key.push_back(U[b]);
+        key.push_back(V[b]);
+        key.push_back(dU[b]);
+        key.push_back(M[b]);
+    }
+    crocco_ctx_s::StepGraph *g = nullptr;
+    for (auto &x : c->graphs)
+        if (x.key == key && x.dt == dt) g = &x;
+    if (!g) {
+        if (!c->cap_stream) CK(c, cudaStreamCreateWithFlags(&c->cap_stream, cudaStreamNonBlocking));
+        // capture on a private stream ordered after the caller's stream, then restore
+        cudaEvent_t ev;
+        CK(c, cudaEventCreateWithFlags(&ev, cudaEventDisableTiming));
+        CK(c, cudaEventRecord(ev, c->stream));
+        CK(c, cudaStreamWaitEvent(c->cap_stream, ev, 0));
+        cudaStream_t orig = c->stream;
+        const int64_t l0 = c->launches;
+        c->stream = c->cap_stream;
+        CK(c, cudaStreamBeginCapture(c->cap_stream, cudaStreamCaptureModeThreadLocal));
+        st = rk3_eager(c, dt, U, V, dU, M);
+        cudaGraph_t graph;
+        cudaError_t e = cudaStreamEndCapture(c->cap_stream, &graph);
+        c->stream = orig;
+        cudaEventDestroy(ev);
+        if (st) return st;
+        if (e != cudaSuccess) return fail(c, CROCCO_ERR_CUDA, "graph capture: %s", cudaGetErrorString(e));
+        cudaGraphExec_t exec;
+        e = cudaGraphInstantiate(&exec, graph, 0);
+        cudaGraphDestroy(graph);
+        if (e != cudaSuccess) return fail(c, CROCCO_ERR_CUDA, "graph instantiate: %s", cudaGetErrorString(e));
+        if (c->graphs.size() >= 4) {
+            cudaGraphExecDestroy(c->graphs.front().exec);
+            c->graphs.erase(c->graphs.begin());
+        }
+        c->graphs.push_back({key, dt, exec, c->launches - l0});
+        c->launches = l0;  // captured, not launched
+        g = &c->graphs.back();
+    }
+    CK(c, cudaGraphLaunch(g->exec, c->stream));
+    c->launches += g->nodes;
     return CROCCO_OK;
 }
 

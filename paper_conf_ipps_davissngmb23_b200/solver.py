@@ -59,31 +59,43 @@ class Solver:
 
     # ------------------------------------------------------------ setup
     def set_coords(self, xyz_blocks):
-        """xyz_blocks[b]: numpy (3, P2, P1, P0) on the coordinate band (g = 10); runs InitGridMetrics."""
-        tmp = []
+        """xyz_blocks[b]: (3, P2, P1, P0) numpy/torch on the coordinate band (g = 10); runs InitGridMetrics."""
         for b in range(self.nloc):
-            L = self.layouts[b]
-            t = torch.zeros(3 * L.ccomp_stride, dtype=torch.float64, device=self.device)
-            src = xyz_blocks[b]
-            if not isinstance(src, torch.Tensor):
-                src = torch.from_numpy(np.ascontiguousarray(src))
-            self.view(t, b, 3, coords=True).copy_(src)
-            tmp.append(t)
-        cc.crocco_init_metrics(self.ctx, self._ptrs(tmp), self._ptrs(self.met))
+            self._stage_coords(b, xyz_blocks[b])
+        self._init_metrics()
+
+    def set_coords_block(self, b, xyz):
+        """Stage one block's coordinates; InitGridMetrics runs once all blocks are staged."""
+        self._stage_coords(b, xyz)
+        if all(t is not None for t in self._coords):
+            self._init_metrics()
+
+    def _stage_coords(self, b, xyz):
+        if not hasattr(self, "_coords") or self._coords is None:
+            self._coords = [None] * self.nloc
+        L = self.layouts[b]
+        t = torch.zeros(3 * L.ccomp_stride, dtype=torch.float64, device=self.device)
+        src = xyz if isinstance(xyz, torch.Tensor) else torch.from_numpy(np.ascontiguousarray(xyz))
+        self.view(t, b, 3, coords=True).copy_(src)
+        self._coords[b] = t
+
+    def _init_metrics(self):
+        cc.crocco_init_metrics(self.ctx, self._ptrs(self._coords), self._ptrs(self.met))
         self.sync()
-        del tmp
+        self._coords = None
 
     def set_state(self, U_blocks, interior=True):
-        """U_blocks[b]: numpy conserved state, interior (5, n2, n1, n0) or padded."""
+        """U_blocks[b]: numpy/torch conserved state, interior (5, n2, n1, n0) or padded."""
         for b in range(self.nloc):
-            v = self.view(self.U[b], b, 5)
-            src = U_blocks[b]
-            if not isinstance(src, torch.Tensor):
-                src = torch.from_numpy(np.ascontiguousarray(src))
-            if interior:
-                v[:, G:-G, G:-G, G:-G].copy_(src)
-            else:
-                v.copy_(src)
+            self.set_state_block(b, U_blocks[b], interior)
+
+    def set_state_block(self, b, U, interior=True):
+        v = self.view(self.U[b], b, 5)
+        src = U if isinstance(U, torch.Tensor) else torch.from_numpy(np.ascontiguousarray(U))
+        if interior:
+            v[:, G:-G, G:-G, G:-G].copy_(src)
+        else:
+            v.copy_(src)
 
     def get(self, bufs, ncomp=5):
         return [self.view(bufs[b], b, ncomp).cpu().numpy() for b in range(self.nloc)]
@@ -103,10 +115,12 @@ class Solver:
                            self._ptrs(self.dU), self._ptrs(self.met))
         self.U, self.V = self.V, self.U
 
-    def step(self, dt, nsteps=1):
+    def step(self, dt, nsteps=1, graph=True):
+        """nsteps full RK3 steps (crocco_rk3_step; one CUDA-graph launch per step)."""
         for _ in range(nsteps):
-            for s in range(3):
-                self.stage(s, dt)
+            cc.crocco_rk3_step(self.ctx, dt, self._ptrs(self.U), self._ptrs(self.V),
+                               self._ptrs(self.dU), self._ptrs(self.met), graph)
+            self.U, self.V = self.V, self.U
 
     def compute_dt(self, cfl):
         """ComputeDt (Alg. 1 l.9): CFL time step of the current state (synchronises)."""

@@ -324,6 +324,25 @@ def test_full_size_config_sampled(name):
     S.close()
 
 
+# ------------------------------------------------------------------ CUDA-graph RK3 steps
+
+def test_rk3_step_graph_equals_eager_bitwise():
+    n = (40, 16, 12)
+    pb = wavy_random(n, 29, dict(terms=3, mu_ref=0.02))
+    outs = []
+    for graph in (False, True):
+        S = pb.solver((2, 1, 1))
+        for _ in range(5):                       # 5 steps: both cached buffer orders replayed
+            S.step(1e-3, graph=graph)
+        S.sync()
+        outs.append(pb.gather(S, S.get(S.U)))
+        from paper_conf_ipps_davissngmb23_b200 import crocco as cc
+        nl = cc.crocco_launch_count(S.ctx)
+        S.close()
+        assert nl > 0
+    assert np.array_equal(outs[0], outs[1])
+
+
 # ------------------------------------------------------------------ ComputeDt (NEXT-1)
 
 @pytest.mark.parametrize("nb", [(1, 1, 1), (2, 3, 2)])
