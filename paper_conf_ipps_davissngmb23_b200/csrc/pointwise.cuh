@@ -115,6 +115,9 @@ __global__ void __launch_bounds__(256) k_visc(const double *__restrict__ Pm,
 // k-2..k+2 in registers (k-derivatives), and only the current plane k (with a
 // 2-point i/j halo) is staged in shared memory (i/j-derivatives), double
 // buffered so one barrier per plane suffices.
+#ifndef CROCCO_VISC_PREFETCH
+#define CROCCO_VISC_PREFETCH 1  // load the next plane's U / metrics one step ahead (registers)
+#endif
 constexpr int VTX = 32, VTY = 8, VK = 32;           // tile and slab
 constexpr int VHX = VTX + 4, VHY = VTY + 4;          // with halo
 constexpr int VPL = VHX * VHY;                       // points per staged plane
@@ -177,7 +180,67 @@ __global__ void __launch_bounds__(VTX * VTY) k_visc_tiled(const double *__restri
 #pragma unroll
         for (int f = 0; f < 4; f++) win[f][o + 1] = q[f];  // shifted into 0..3 by the first step
     }
+#if CROCCO_VISC_PREFETCH
+    // global operands of the step, loaded one step ahead: own U at plane k+2,
+    // halo U at plane k, own metrics at plane k
+    double cO[5], cH[5], cM[10];
+    auto ld_own = [&](int kk, double o5[5]) {
+        const int64_t q = at(L, gi, gj, kk);
+#pragma unroll
+        for (int c = 0; c < 5; c++) o5[c] = U[c * L.cs + q];
+    };
+    auto ld_halo = [&](int kk, double o5[5]) {
+        if (tid < VHALO) {
+            const int64_t q = at(L, hgi, hgj, kk);
+#pragma unroll
+            for (int c = 0; c < 5; c++) o5[c] = U[c * L.cs + q];
+        }
+    };
+    auto ld_met = [&](int kk, double o10[10]) {
+        const int64_t q = at(L, gi, gj, kk);
+#pragma unroll
+        for (int c = 0; c < 10; c++) o10[c] = M[c * L.cs + q];
+    };
+    auto prim_of = [&](const double u5[5], double q[4]) {
+        const double ir = rcp_nr(u5[0]);
+        const double u = u5[1] * ir, v = u5[2] * ir, w = u5[3] * ir;
+        const double pr = ph.gm1 * fma(-0.5, fma(u5[1], u, fma(u5[2], v, u5[3] * w)), u5[4]);
+        q[0] = u;
+        q[1] = v;
+        q[2] = w;
+        q[3] = pr * ir * iR;
+    };
+    ld_own(k0 + 2, cO);
+    ld_halo(k0, cH);
+    ld_met(k0, cM);
+#endif
     for (int k = k0; k < k1; k++) {
+#if CROCCO_VISC_PREFETCH
+        double nO[5], nH[5], nM[10];
+        const int kn = min(k + 1, k1 - 1);  // clamp: the last step reloads its own plane
+        ld_own(kn + 2, nO);
+        ld_halo(kn, nH);
+        ld_met(kn, nM);
+        {
+            double q[4];
+            prim_of(cO, q);
+#pragma unroll
+            for (int f = 0; f < 4; f++) {
+#pragma unroll
+                for (int o = 0; o < 4; o++) win[f][o] = win[f][o + 1];
+                win[f][4] = q[f];
+            }
+        }
+        double *pl = vsm + (k & 1) * 4 * VPL;
+#pragma unroll
+        for (int f = 0; f < 4; f++) pl[f * VPL + oidx] = win[f][2];
+        if (tid < VHALO) {
+            double q[4];
+            prim_of(cH, q);
+#pragma unroll
+            for (int f = 0; f < 4; f++) pl[f * VPL + hidx] = q[f];
+        }
+#else
         {   // own primitives of plane k+2, shift the window
             double q[4];
             prim4(U, L.cs, at(L, gi, gj, k + 2), ph.gm1, iR, q);
@@ -197,6 +260,7 @@ __global__ void __launch_bounds__(VTX * VTY) k_visc_tiled(const double *__restri
 #pragma unroll
             for (int f = 0; f < 4; f++) pl[f * VPL + hidx] = q[f];
         }
+#endif
         __syncthreads();
         if (own) {
             double gc[4][3];
@@ -207,6 +271,14 @@ __global__ void __launch_bounds__(VTX * VTY) k_visc_tiled(const double *__restri
                 gc[f][1] = fma(8.0, c[VHX] - c[-VHX], -(c[2 * VHX] - c[-2 * VHX])) * (1.0 / 12.0);
                 gc[f][2] = fma(8.0, win[f][3] - win[f][1], -(win[f][4] - win[f][0])) * (1.0 / 12.0);
             }
+#if CROCCO_VISC_PREFETCH
+            const double J = cM[0];
+            double m[3][3];
+#pragma unroll
+            for (int d = 0; d < 3; d++)
+#pragma unroll
+                for (int a = 0; a < 3; a++) m[d][a] = cM[1 + 3 * d + a];
+#else
             const int64_t p = at(L, i, j, k);
             const double J = M[p];
             double m[3][3];
@@ -214,6 +286,7 @@ __global__ void __launch_bounds__(VTX * VTY) k_visc_tiled(const double *__restri
             for (int d = 0; d < 3; d++)
 #pragma unroll
                 for (int a = 0; a < 3; a++) m[d][a] = M[(1 + 3 * d + a) * L.cs + p];
+#endif
             double gx[4][3];
 #pragma unroll
             for (int f = 0; f < 4; f++)
@@ -247,6 +320,15 @@ __global__ void __launch_bounds__(VTX * VTY) k_visc_tiled(const double *__restri
                 FV[(4 * d + 3) * V.cs + o] = fma(m[d][0], hb[0], fma(m[d][1], hb[1], m[d][2] * hb[2]));
             }
         }
+#if CROCCO_VISC_PREFETCH
+#pragma unroll
+        for (int c = 0; c < 5; c++) {
+            cO[c] = nO[c];
+            cH[c] = nH[c];
+        }
+#pragma unroll
+        for (int c = 0; c < 10; c++) cM[c] = nM[c];
+#endif
     }
 }
 
