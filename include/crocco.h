@@ -65,13 +65,29 @@ enum {
     CROCCO_BC_PERIODIC = 0,  /* copy from the periodic partner; lo/hi must both be PERIODIC */
     CROCCO_BC_EXTRAP = 1,    /* zeroth-order extrapolation: ghost = nearest interior layer */
     CROCCO_BC_DIRICHLET = 2, /* ghost = constant conserved state dirichlet[d][side][0..4] */
-    CROCCO_BC_WALL = 3       /* no-slip adiabatic wall, mirror about the face at index -1/2 (n-1/2):
+    CROCCO_BC_WALL = 3,      /* no-slip adiabatic wall, mirror about the face at index -1/2 (n-1/2):
                                 (rho, -rho u, -rho v, -rho w, E) of the mirrored interior point */
+    CROCCO_BC_SLIPWALL = 4,  /* inviscid reflecting wall (DMR; reading 19): mirror, the
+                                momentum reflected about the plane normal to n = m^d/|m^d| of the
+                                mirrored point (needs the metrics in the fill) */
+    CROCCO_BC_SPLIT = 5      /* boundary data switching at a moving index (DMR bottom/top, reading 20):
+                                see crocco_split; the right part may be DIRICHLET or SLIPWALL */
 };
 enum { CROCCO_TERM_INVISCID = 1, CROCCO_TERM_VISCOUS = 2 }; /* bitmask (Alg. 2 l.5-7 / l.8) */
 enum { CROCCO_MU_CONST = 0, CROCCO_MU_SUTHERLAND = 1 };
 enum { CROCCO_FIELD_STATE = 0, CROCCO_FIELD_METRIC = 1 };
 enum { CROCCO_GHOST = 4, CROCCO_GHOST_COORDS = 10 }; /* reading 7 */
+
+/* SPLIT face data: ghost point with global index g along `axis` (a tangential axis
+   of the face) takes the DIRICHLET state `left` if g + 1/2 < s(t) = i0 + di_dt * t,
+   else `right_kind` (CROCCO_BC_DIRICHLET with state `right`, or CROCCO_BC_SLIPWALL). */
+typedef struct {
+    int32_t axis;
+    double i0, di_dt;
+    double left[5];
+    int32_t right_kind;
+    double right[5];
+} crocco_split;
 
 typedef struct {
     int64_t n_global[3];        /* interior points N_xi, N_eta, N_zeta of the whole domain */
@@ -85,6 +101,7 @@ typedef struct {
     void *stream;               /* cudaStream_t the library enqueues on (NULL = legacy default) */
     const void *nccl_unique_id; /* 128-byte ncclUniqueId broadcast by the caller (torch.distributed);
                                    ignored when nranks == 1 */
+    crocco_split split[3][2];   /* data of CROCCO_BC_SPLIT faces (ignored elsewhere) */
 } crocco_grid_desc;
 
 typedef struct {
@@ -145,9 +162,16 @@ crocco_status crocco_init_metrics(crocco_ctx ctx, double *const *xyz, double *co
 
 /* FillPatch + BC_Fill: in place on 4 ghost layers,
    phases xi -> eta (spanning xi ghosts) -> zeta (spanning xi, eta ghosts).
-   kind STATE: 5 comps, copies + physical BCs.  kind METRIC: 10 comps,
-   periodic / inter-block copies only.  Collective. */
-crocco_status crocco_fill_boundary(crocco_ctx ctx, double *const *field, int32_t kind);
+   kind STATE: 5 comps, copies + physical BCs at the ctx time (crocco_set_time).
+   kind METRIC: 10 comps, periodic / inter-block copies only.  metrics: required
+   for STATE fills when a face is SLIPWALL or SPLIT, else may be NULL.  Collective. */
+crocco_status crocco_fill_boundary(crocco_ctx ctx, double *const *field, int32_t kind,
+                                   double *const *metrics);
+/* Simulation time t_n of the start of the current step (time-dependent SPLIT faces).
+   crocco_rk_stage evaluates the boundary data of stage s at t_n + c_s dt,
+   c = (0, 1/3, 3/4); crocco_rk3_step advances it by dt (t <- t + dt). */
+crocco_status crocco_set_time(crocco_ctx ctx, double t);
+crocco_status crocco_get_time(crocco_ctx ctx, double *t);
 
 /* RHS: rhs = J ( -sum_d delta_d F^_inv^d + sum_d D4_d F^_v^d )
    on interior points (ghosts of rhs untouched).  U must have its ghosts filled;
@@ -168,8 +192,8 @@ crocco_status crocco_rk_stage(crocco_ctx ctx, int32_t stage, double dt, double *
    (1: V -> U), (2: U -> V): the new state is in V, U was used for the middle stage.
    use_graph != 0: the three stages (fills, sweeps, update: ~20 kernels) are captured
    once per (U, V, dU, metrics, dt) into a CUDA graph and replayed with one launch
-   (at most 4 graphs cached per ctx; eager launches when kernel timing is on or
-   nranks > 1).  Collective. */
+   (at most 4 graphs cached per ctx; eager launches when kernel timing is on,
+   nranks > 1 or a SPLIT face moves in time).  Advances the ctx time by dt.  Collective. */
 crocco_status crocco_rk3_step(crocco_ctx ctx, double dt, double *const *U, double *const *V,
                               double *const *dU, double *const *metrics, int32_t use_graph);
 

@@ -23,7 +23,7 @@ _LIB = os.path.join(_HERE, "liboracle.so")
 
 G = 4
 GC = 10
-PERIODIC, EXTRAP, DIRICHLET, WALL = 0, 1, 2, 3
+PERIODIC, EXTRAP, DIRICHLET, WALL, SLIPWALL, SPLIT = 0, 1, 2, 3, 4, 5
 INVISCID, VISCOUS = 1, 2
 FIELD_STATE, FIELD_METRIC = 0, 1
 MU_CONST, MU_SUTHERLAND = 0, 1
@@ -44,6 +44,24 @@ class Phys(C.Structure):
                 ("mu_law", C.c_int32), ("mu_ref", C.c_double), ("T_ref", C.c_double),
                 ("S", C.c_double), ("weno_eps", C.c_double), ("terms", C.c_int32),
                 ("dir_mask", C.c_int32), ("weno_linear", C.c_int32)]
+
+
+class Split(C.Structure):
+    """Moving split of boundary data along a tangential axis (SPLIT faces, DMR)."""
+    _fields_ = [("axis", C.c_int32), ("i0", C.c_double), ("di_dt", C.c_double),
+                ("left", C.c_double * 5), ("right_kind", C.c_int32), ("right", C.c_double * 5)]
+
+
+def splits(spec=None):
+    """spec: {(d, side): dict(axis, i0, di_dt, left, right_kind, right)} -> Split[6]."""
+    arr = (Split * 6)()
+    for (d, side), v in (spec or {}).items():
+        s = arr[2 * d + side]
+        s.axis, s.i0, s.di_dt, s.right_kind = int(v["axis"]), float(v["i0"]), float(v["di_dt"]), int(v["right_kind"])
+        for c in range(5):
+            s.left[c] = float(v["left"][c])
+            s.right[c] = float(v.get("right", [0.0] * 5)[c])
+    return arr
 
 
 def phys(gamma=1.4, R=1.0, Pr=0.72, mu_law=MU_CONST, mu_ref=0.0, T_ref=1.0, S=0.0,
@@ -74,6 +92,12 @@ def lib():
                                       dp, dp, dp, dp]
         L.oracle_advance.argtypes = [i64p, i32p, dp, C.POINTER(Phys), C.c_double, C.c_int32,
                                      dp, dp]
+        sp = C.POINTER(Split)
+        L.oracle_fill_ex.argtypes = [i64p, i32p, dp, sp, C.c_double, dp, dp, C.c_int32, C.c_int32]
+        L.oracle_rk_stage_ex.argtypes = [i64p, i32p, dp, sp, C.c_double, C.POINTER(Phys), C.c_int32,
+                                         C.c_double, dp, dp, dp, dp]
+        L.oracle_advance_ex.argtypes = [i64p, i32p, dp, sp, C.c_double, C.POINTER(Phys), C.c_double,
+                                        C.c_int32, dp, dp]
         L.oracle_compute_dt.argtypes = [i64p, C.POINTER(Phys), dp, dp, C.c_double]
         L.oracle_compute_dt.restype = C.c_double
         L.oracle_set_threads.argtypes = [C.c_int]
@@ -113,10 +137,12 @@ def get_threads() -> int:
     return int(lib().oracle_get_threads())
 
 
-def fill(n, bc, f, kind=FIELD_STATE, dirichlet=None):
-    """FillPatch + BC_Fill in place (PAPER.md:83, 108-109)."""
+def fill(n, bc, f, kind=FIELD_STATE, dirichlet=None, split=None, t=0.0, met=None):
+    """FillPatch + BC_Fill in place; split/t/met for SPLIT and SLIPWALL faces."""
     d = _dir(dirichlet)
-    lib().oracle_fill(_n(n), _bc(bc), _dp(d), _dp(f), f.shape[0], kind)
+    sp = split if split is not None else splits()
+    mp = _dp(met) if met is not None else None
+    lib().oracle_fill_ex(_n(n), _bc(bc), _dp(d), sp, float(t), mp, _dp(f), f.shape[0], kind)
     return f
 
 
@@ -165,10 +191,11 @@ def rk_stage(n, bc, ph, stage, dt, Uin, Uout, dU, met, dirichlet=None):
                           _dp(dU), _dp(met))
 
 
-def advance(n, bc, ph, dt, nsteps, U, met, dirichlet=None):
-    """nsteps RK3 steps in place on U (padded), ghosts filled on return."""
+def advance(n, bc, ph, dt, nsteps, U, met, dirichlet=None, split=None, t0=0.0):
+    """nsteps RK3 steps in place on U (padded) from time t0, ghosts filled on return."""
     d = _dir(dirichlet)
-    lib().oracle_advance(_n(n), _bc(bc), _dp(d), C.byref(ph), dt, nsteps, _dp(U), _dp(met))
+    sp = split if split is not None else splits()
+    lib().oracle_advance_ex(_n(n), _bc(bc), _dp(d), sp, float(t0), C.byref(ph), dt, nsteps, _dp(U), _dp(met))
     return U
 
 

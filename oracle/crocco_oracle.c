@@ -94,11 +94,35 @@ int oracle_get_threads(void)
 
 /* ------------------------------------------------------------------ */
 /* 1. Ghost fill: FillPatch (periodic / inter-block copies) + BC_Fill  */
-/*    (readings 15-16).  Three ordered phases    */
-/*    xi -> eta -> zeta; phase d spans the ghosts of directions < d.   */
+/*    (readings 15-16, 19-20).  Three ordered    */
+/*    phases xi -> eta -> zeta; phase d spans the ghosts of directions */
+/*    < d.  Kinds:                                                     */
+/*      PERIODIC  copy from the periodic partner                       */
+/*      EXTRAP    copy of the nearest interior layer                   */
+/*      DIRICHLET constant conserved state                             */
+/*      WALL      no-slip adiabatic: mirror, momentum negated          */
+/*      SLIPWALL  inviscid reflecting wall (DMR): mirror,*/
+/*                momentum reflected about the plane normal to         */
+/*                n = m^d/|m^d| of the mirrored interior point         */
+/*      SPLIT     boundary data switching at a moving index along a    */
+/*                tangential axis (DMR bottom/top, reading 20): ghost  */
+/*                points with g + 1/2 < s(t) = i0 + di_dt t take the   */
+/*                left state, the others the right kind (DIRICHLET     */
+/*                right state or SLIPWALL).                            */
 /* ------------------------------------------------------------------ */
-void oracle_fill(const int64_t n[3], const int32_t bc[6], const double dirichlet[30],
-                 double *f, int32_t ncomp, int32_t kind)
+enum { O_SLIPWALL = 4, O_SPLIT = 5 };
+
+typedef struct {
+    int32_t axis;       /* tangential axis of the split (0..2) */
+    double i0, di_dt;   /* split position s(t) = i0 + di_dt t, in global index units */
+    double left[5];     /* conserved state where g + 1/2 < s(t) */
+    int32_t right_kind; /* O_DIRICHLET or O_SLIPWALL elsewhere */
+    double right[5];
+} oracle_split;
+
+void oracle_fill_ex(const int64_t n[3], const int32_t bc[6], const double dirichlet[30],
+                    const oracle_split *split, double t, const double *met, double *f,
+                    int32_t ncomp, int32_t kind)
 {
     obox b = make_box(n, OG);
     for (int d = 0; d < 3; d++) {
@@ -111,17 +135,17 @@ void oracle_fill(const int64_t n[3], const int32_t bc[6], const double dirichlet
             int kindbc = bc[2 * d + side];
             if (kind == O_FIELD_METRIC && kindbc != O_PERIODIC)
                 continue; /* metrics: only periodic copies; physical faces keep computed ghosts */
+            const oracle_split *sp = (kindbc == O_SPLIT) ? &split[2 * d + side] : NULL;
+            const double s_t = sp ? sp->i0 + sp->di_dt * t : 0.0;
             for (int64_t gg = 1; gg <= OG; gg++) {
                 int64_t dst = side == 0 ? -gg : n[d] - 1 + gg;
                 int64_t src;
-                double sgn_mom = 1.0;
                 switch (kindbc) {
                 case O_PERIODIC: src = side == 0 ? n[d] - gg : gg - 1; break;
                 case O_EXTRAP: src = side == 0 ? 0 : n[d] - 1; break;
                 case O_WALL:
-                    src = side == 0 ? gg - 1 : n[d] - gg;
-                    sgn_mom = -1.0;
-                    break;
+                case O_SLIPWALL:
+                case O_SPLIT: src = side == 0 ? gg - 1 : n[d] - gg; break; /* mirror */
                 default: src = 0; break; /* DIRICHLET: constant state */
                 }
                 for (int64_t c2 = lo[(d + 2) % 3]; c2 < hi[(d + 2) % 3]; c2++)
@@ -133,20 +157,50 @@ void oracle_fill(const int64_t n[3], const int32_t bc[6], const double dirichlet
                         id[(d + 2) % 3] = is[(d + 2) % 3] = c2;
                         int64_t pd = IX(&b, id[0], id[1], id[2]);
                         int64_t ps = IX(&b, is[0], is[1], is[2]);
-                        for (int c = 0; c < ncomp; c++) {
-                            double v;
-                            if (kindbc == O_DIRICHLET)
-                                v = dirichlet[(2 * d + side) * 5 + c];
-                            else
-                                v = f[c * b.cs + ps];
-                            if (kindbc == O_WALL && c >= 1 && c <= 3)
-                                v = sgn_mom * v;
-                            f[c * b.cs + pd] = v;
+                        /* effective kind of this ghost point */
+                        int k = kindbc;
+                        const double *cst = dirichlet + (2 * d + side) * 5;
+                        if (sp) {
+                            if ((double)id[sp->axis] + 0.5 < s_t) {
+                                k = O_DIRICHLET;
+                                cst = sp->left;
+                            } else {
+                                k = sp->right_kind;
+                                cst = sp->right;
+                            }
                         }
+                        double v[5];
+                        for (int c = 0; c < ncomp; c++)
+                            v[c] = (k == O_DIRICHLET) ? cst[c] : f[c * b.cs + ps];
+                        if (k == O_WALL)
+                            for (int c = 1; c <= 3; c++)
+                                v[c] = -v[c];
+                        if (k == O_SLIPWALL) {
+                            double m[3], mm = 0.0, mdot = 0.0;
+                            for (int a = 0; a < 3; a++) {
+                                m[a] = met[(1 + 3 * d + a) * b.cs + ps];
+                                mm = mm + m[a] * m[a];
+                            }
+                            mm = sqrt(mm);
+                            for (int a = 0; a < 3; a++) {
+                                m[a] = m[a] / mm;
+                                mdot = mdot + v[1 + a] * m[a];
+                            }
+                            for (int a = 0; a < 3; a++)
+                                v[1 + a] = v[1 + a] - 2.0 * mdot * m[a];
+                        }
+                        for (int c = 0; c < ncomp; c++)
+                            f[c * b.cs + pd] = v[c];
                     }
             }
         }
     }
+}
+
+void oracle_fill(const int64_t n[3], const int32_t bc[6], const double dirichlet[30],
+                 double *f, int32_t ncomp, int32_t kind)
+{
+    oracle_fill_ex(n, bc, dirichlet, NULL, 0.0, NULL, f, ncomp, kind);
 }
 
 /* ------------------------------------------------------------------ */
@@ -648,24 +702,35 @@ void oracle_rk_update(const int64_t n[3], int32_t stage, double dt, const double
             }
 }
 
-/* one RK stage = FillPatch/BC_Fill + RHS + Update (Alg. 2 l.3-9) */
-void oracle_rk_stage(const int64_t n[3], const int32_t bc[6], const double dirichlet[30],
-                     const oracle_phys *ph, int32_t stage, double dt, double *Uin, double *Uout,
-                     double *dU, const double *met)
+/* one RK stage = FillPatch/BC_Fill + RHS + Update (Alg. 2 l.3-9); the boundary
+   data of stage s are evaluated at t + c_s dt, c = (0, 1/3, 3/4) (reading 13) */
+static const double RK_C[3] = {0.0, 1.0 / 3.0, 3.0 / 4.0};
+
+void oracle_rk_stage_ex(const int64_t n[3], const int32_t bc[6], const double dirichlet[30],
+                        const oracle_split *split, double t, const oracle_phys *ph, int32_t stage,
+                        double dt, double *Uin, double *Uout, double *dU, const double *met)
 {
     obox b = make_box(n, OG);
     double *rhs = (double *)calloc((size_t)(5 * b.cs), sizeof(double));
-    oracle_fill(n, bc, dirichlet, Uin, 5, O_FIELD_STATE);
+    oracle_fill_ex(n, bc, dirichlet, split, t + RK_C[stage] * dt, met, Uin, 5, O_FIELD_STATE);
     oracle_rhs(n, ph, Uin, met, rhs);
     oracle_rk_update(n, stage, dt, Uin, Uout, dU, rhs);
     free(rhs);
 }
 
-/* nsteps full RK3 steps with a fixed dt (Alg. 1 l.5-10 without Regrid/ComputeDt).
-   U is the state in/out (padded layout); on return its ghosts are filled. */
-void oracle_advance(const int64_t n[3], const int32_t bc[6], const double dirichlet[30],
-                    const oracle_phys *ph, double dt, int32_t nsteps, double *U,
-                    const double *met)
+void oracle_rk_stage(const int64_t n[3], const int32_t bc[6], const double dirichlet[30],
+                     const oracle_phys *ph, int32_t stage, double dt, double *Uin, double *Uout,
+                     double *dU, const double *met)
+{
+    oracle_rk_stage_ex(n, bc, dirichlet, NULL, 0.0, ph, stage, dt, Uin, Uout, dU, met);
+}
+
+/* nsteps full RK3 steps with a fixed dt from time t0 (Alg. 1 l.5-10 without
+   Regrid/ComputeDt).  U is the state in/out (padded layout); on return its
+   ghosts are filled at t0 + nsteps dt. */
+void oracle_advance_ex(const int64_t n[3], const int32_t bc[6], const double dirichlet[30],
+                       const oracle_split *split, double t0, const oracle_phys *ph, double dt,
+                       int32_t nsteps, double *U, const double *met)
 {
     obox b = make_box(n, OG);
     size_t sz = (size_t)(5 * b.cs) * sizeof(double);
@@ -673,18 +738,28 @@ void oracle_advance(const int64_t n[3], const int32_t bc[6], const double dirich
     double *dU = (double *)calloc((size_t)(5 * b.cs), sizeof(double));
     memcpy(V, U, sz);
     double *a = U, *o = V;
-    for (int32_t s = 0; s < nsteps; s++)
+    double t = t0; /* step start time, advanced by repeated addition t <- t + dt */
+    for (int32_t s = 0; s < nsteps; s++) {
         for (int st = 0; st < 3; st++) {
-            oracle_rk_stage(n, bc, dirichlet, ph, st, dt, a, o, dU, met);
-            double *t = a;
+            oracle_rk_stage_ex(n, bc, dirichlet, split, t, ph, st, dt, a, o, dU, met);
+            double *tmp = a;
             a = o;
-            o = t;
+            o = tmp;
         }
+        t = t + dt;
+    }
     if (a != U)
         memcpy(U, a, sz);
-    oracle_fill(n, bc, dirichlet, U, 5, O_FIELD_STATE);
+    oracle_fill_ex(n, bc, dirichlet, split, t, met, U, 5, O_FIELD_STATE);
     free(V);
     free(dU);
+}
+
+void oracle_advance(const int64_t n[3], const int32_t bc[6], const double dirichlet[30],
+                    const oracle_phys *ph, double dt, int32_t nsteps, double *U,
+                    const double *met)
+{
+    oracle_advance_ex(n, bc, dirichlet, NULL, 0.0, ph, dt, nsteps, U, met);
 }
 
 /* ------------------------------------------------------------------ */

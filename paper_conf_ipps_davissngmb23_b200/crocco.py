@@ -14,7 +14,7 @@ HERE = os.path.dirname(os.path.abspath(__file__))
 LIB_PATH = os.environ.get("CROCCO_LIB") or os.path.join(HERE, "libcrocco.so")  # env: variant builds (tools/)
 
 CROCCO_OK, CROCCO_ERR_ARG, CROCCO_ERR_CUDA, CROCCO_ERR_NCCL, CROCCO_ERR_NOMEM, CROCCO_ERR_STATE = range(6)
-BC_PERIODIC, BC_EXTRAP, BC_DIRICHLET, BC_WALL = 0, 1, 2, 3
+BC_PERIODIC, BC_EXTRAP, BC_DIRICHLET, BC_WALL, BC_SLIPWALL, BC_SPLIT = 0, 1, 2, 3, 4, 5
 TERM_INVISCID, TERM_VISCOUS = 1, 2
 MU_CONST, MU_SUTHERLAND = 0, 1
 FIELD_STATE, FIELD_METRIC = 0, 1
@@ -27,12 +27,17 @@ class CroccoError(RuntimeError):
         self.status = status
 
 
+class Split(C.Structure):
+    _fields_ = [("axis", C.c_int32), ("i0", C.c_double), ("di_dt", C.c_double),
+                ("left", C.c_double * 5), ("right_kind", C.c_int32), ("right", C.c_double * 5)]
+
+
 class GridDesc(C.Structure):
     _fields_ = [("n_global", C.c_int64 * 3), ("n_blocks", C.c_int32 * 3),
                 ("bc", (C.c_int32 * 2) * 3), ("dirichlet", ((C.c_double * 5) * 2) * 3),
                 ("rank", C.c_int32), ("nranks", C.c_int32),
                 ("block_rank", C.POINTER(C.c_int32)), ("stream", C.c_void_p),
-                ("nccl_unique_id", C.c_void_p)]
+                ("nccl_unique_id", C.c_void_p), ("split", (Split * 2) * 3)]
 
 
 class PhysC(C.Structure):
@@ -68,7 +73,9 @@ _SIGS = {
     "crocco_set_phys": [C.c_void_p, C.POINTER(PhysC)],
     "crocco_scratch_bytes": [C.c_void_p, C.POINTER(C.c_int64)],
     "crocco_init_metrics": [C.c_void_p, DPP, DPP],
-    "crocco_fill_boundary": [C.c_void_p, DPP, C.c_int32],
+    "crocco_fill_boundary": [C.c_void_p, DPP, C.c_int32, DPP],
+    "crocco_set_time": [C.c_void_p, C.c_double],
+    "crocco_get_time": [C.c_void_p, C.POINTER(C.c_double)],
     "crocco_rhs": [C.c_void_p, DPP, DPP, DPP],
     "crocco_rk_stage": [C.c_void_p, C.c_int32, C.c_double, DPP, DPP, DPP, DPP],
     "crocco_rk_update": [C.c_void_p, C.c_int32, C.c_double, DPP, DPP, DPP, DPP],
@@ -131,7 +138,8 @@ def crocco_kernel_class_name(k: int) -> str:
 
 
 def make_desc(n_global, n_blocks=(1, 1, 1), bc=((0, 0),) * 3, dirichlet=None, rank=0, nranks=1,
-              block_rank=None, stream=0, nccl_unique_id=None):
+              block_rank=None, stream=0, nccl_unique_id=None, split=None):
+    """split: {(d, side): dict(axis, i0, di_dt, left, right_kind, right)} for SPLIT faces."""
     d = GridDesc()
     for a in range(3):
         d.n_global[a] = int(n_global[a])
@@ -151,6 +159,13 @@ def make_desc(n_global, n_blocks=(1, 1, 1), bc=((0, 0),) * 3, dirichlet=None, ra
         buf = C.create_string_buffer(bytes(nccl_unique_id), 128)
         d.nccl_unique_id = C.cast(buf, C.c_void_p)
         keep.append(buf)
+    for (a, sd), v in (split or {}).items():
+        sp = d.split[a][sd]
+        sp.axis, sp.i0, sp.di_dt = int(v["axis"]), float(v["i0"]), float(v["di_dt"])
+        sp.right_kind = int(v["right_kind"])
+        for c in range(5):
+            sp.left[c] = float(v["left"][c])
+            sp.right[c] = float(v.get("right", [0.0] * 5)[c])
     d._keep = keep
     return d
 
@@ -194,9 +209,23 @@ def crocco_init_metrics(ctx, xyz_ptrs, met_ptrs):
     _check(lib().crocco_init_metrics(ctx, a, b), ctx)
 
 
-def crocco_fill_boundary(ctx, field_ptrs, kind=FIELD_STATE):
+def crocco_fill_boundary(ctx, field_ptrs, kind=FIELD_STATE, met_ptrs=None):
     a, ka = _ptrs(field_ptrs)
-    _check(lib().crocco_fill_boundary(ctx, a, kind), ctx)
+    if met_ptrs is None:
+        _check(lib().crocco_fill_boundary(ctx, a, kind, None), ctx)
+    else:
+        b, kb = _ptrs(met_ptrs)
+        _check(lib().crocco_fill_boundary(ctx, a, kind, b), ctx)
+
+
+def crocco_set_time(ctx, t):
+    _check(lib().crocco_set_time(ctx, float(t)), ctx)
+
+
+def crocco_get_time(ctx) -> float:
+    v = C.c_double()
+    _check(lib().crocco_get_time(ctx, C.byref(v)), ctx)
+    return v.value
 
 
 def crocco_rhs(ctx, U_ptrs, met_ptrs, rhs_ptrs):

@@ -87,6 +87,7 @@ struct crocco_ctx_s {
     };
     std::vector<StepGraph> graphs;
     cudaStream_t cap_stream = nullptr;
+    double time = 0.0;  // start of the current step (time-dependent SPLIT faces)
     int64_t stage_elems = 0;
     // timing
     bool timing = false;
@@ -205,8 +206,16 @@ static crocco_status validate(const crocco_grid_desc *d, int nb[3], int bn[3]) {
         if (b > 65535) return fail(nullptr, CROCCO_ERR_ARG, "block interior > 65535 points in direction %d", a);
         bn[a] = (int)b;
         for (int s = 0; s < 2; s++)
-            if (d->bc[a][s] < 0 || d->bc[a][s] > 3)
+            if (d->bc[a][s] < 0 || d->bc[a][s] > 5)
                 return fail(nullptr, CROCCO_ERR_ARG, "bad bc kind %d", d->bc[a][s]);
+        for (int s = 0; s < 2; s++)
+            if (d->bc[a][s] == CROCCO_BC_SPLIT) {
+                const crocco_split &sp = d->split[a][s];
+                if (sp.axis < 0 || sp.axis > 2 || sp.axis == a)
+                    return fail(nullptr, CROCCO_ERR_ARG, "SPLIT face %d/%d: axis must be tangential", a, s);
+                if (sp.right_kind != CROCCO_BC_DIRICHLET && sp.right_kind != CROCCO_BC_SLIPWALL)
+                    return fail(nullptr, CROCCO_ERR_ARG, "SPLIT face %d/%d: right_kind must be DIRICHLET or SLIPWALL", a, s);
+            }
         if ((d->bc[a][0] == CROCCO_BC_PERIODIC) != (d->bc[a][1] == CROCCO_BC_PERIODIC))
             return fail(nullptr, CROCCO_ERR_ARG, "PERIODIC must be paired in direction %d", a);
     }
@@ -581,7 +590,8 @@ static void op_strides(const Lay &L, int64_t st[3]) {
     st[2] = L.pz;
 }
 
-static crocco_status fill_phase(crocco_ctx c, double *const *f, int kind, int D) {
+static crocco_status fill_phase(crocco_ctx c, double *const *f, int kind, int D,
+                                double *const *met, double t) {
     const int ncomp = kind == CROCCO_FIELD_STATE ? 5 : 10;
     BoxOps ops;
     ops.nops = 0;
@@ -609,7 +619,7 @@ static crocco_status fill_phase(crocco_ctx c, double *const *f, int kind, int D)
             op_strides(sb.L, o.sst);
             o.scs = sb.L.cs;
             o.sbase = at(sb.L, (int)m.src_lo[0], (int)m.src_lo[1], (int)m.src_lo[2]);
-            o.mode = 0;
+            o.mode = BOX_COPY;
         } else {
             if (kind == CROCCO_FIELD_METRIC) continue;  // physical faces keep computed metrics
             const int bc = m.bc_kind;
@@ -623,14 +633,30 @@ static crocco_status fill_phase(crocco_ctx c, double *const *f, int kind, int D)
             if (bc == CROCCO_BC_EXTRAP) {
                 lo[D] = m.side == 0 ? 0 : n - 1;
                 o.sst[D] = 0;
-            } else if (bc == CROCCO_BC_WALL) {
-                // dst index (lo + t) <- src index mirrored about the face
+                o.mode = BOX_COPY;
+            } else if (bc == CROCCO_BC_DIRICHLET) {
+                o.mode = BOX_CONST;
+                for (int q = 0; q < 5; q++) o.val[q] = c->desc.dirichlet[D][m.side][q];
+            } else {
+                // WALL / SLIPWALL / SPLIT: dst index (lo + t) <- src index mirrored about the face
                 lo[D] = m.side == 0 ? G - 1 : n - 1;
                 o.sst[D] = -st[D];
-                o.flip_mom = 1;
-            } else {  // DIRICHLET
-                o.mode = 1;
-                for (int q = 0; q < 5; q++) o.val[q] = c->desc.dirichlet[D][m.side][q];
+                o.mode = bc == CROCCO_BC_WALL ? BOX_WALL : (bc == CROCCO_BC_SLIPWALL ? BOX_SLIP : BOX_SPLIT);
+                if (bc != CROCCO_BC_WALL) {
+                    if (!met || !met[dl])
+                        return fail(c, CROCCO_ERR_ARG, "SLIPWALL/SPLIT faces need the metrics in the fill");
+                    o.met = met[dl] + (int64_t)(1 + 3 * D) * db.L.cs;
+                    o.mcs = db.L.cs;
+                }
+                if (bc == CROCCO_BC_SPLIT) {
+                    const crocco_split &sp = c->desc.split[D][m.side];
+                    o.axis = sp.axis;
+                    o.g0 = db.g.origin[sp.axis] + m.dst_lo[sp.axis];
+                    o.s = sp.i0 + sp.di_dt * t;
+                    for (int q = 0; q < 5; q++) o.val[q] = sp.left[q];
+                    o.right_mode = sp.right_kind == CROCCO_BC_SLIPWALL ? BOX_SLIP : BOX_CONST;
+                    for (int q = 0; q < 5; q++) o.rval[q] = sp.right[q];
+                }
             }
             o.sbase = at(db.L, lo[0], lo[1], lo[2]);
         }
@@ -719,16 +745,33 @@ static crocco_status check_ptrs(crocco_ctx c, double *const *p, const char *what
     return CROCCO_OK;
 }
 
-crocco_status crocco_fill_boundary(crocco_ctx c, double *const *f, int32_t kind) {
-    LIVE(c);
+static crocco_status fill_all(crocco_ctx c, double *const *f, int32_t kind, double *const *met, double t) {
     if (kind != CROCCO_FIELD_STATE && kind != CROCCO_FIELD_METRIC)
         return fail(c, CROCCO_ERR_ARG, "bad field kind");
     crocco_status st = check_ptrs(c, f, "field");
     if (st) return st;
     for (int d = 0; d < 3; d++) {
-        st = fill_phase(c, f, kind, d);
+        st = fill_phase(c, f, kind, d, met, t);
         if (st) return st;
     }
+    return CROCCO_OK;
+}
+
+crocco_status crocco_fill_boundary(crocco_ctx c, double *const *f, int32_t kind, double *const *met) {
+    LIVE(c);
+    return fill_all(c, f, kind, met, c->time);
+}
+
+crocco_status crocco_set_time(crocco_ctx c, double t) {
+    LIVE(c);
+    c->time = t;
+    return CROCCO_OK;
+}
+
+crocco_status crocco_get_time(crocco_ctx c, double *t) {
+    LIVE(c);
+    if (!t) return fail(c, CROCCO_ERR_ARG, "null out");
+    *t = c->time;
     return CROCCO_OK;
 }
 
@@ -752,13 +795,14 @@ crocco_status crocco_init_metrics(crocco_ctx c, double *const *xyz, double *cons
         LAUNCH(c, K_METRICS, k_metric<<<cdiv(nm, 128), 128, 0, c->stream>>>(xyz[b], dx, met[b], lb.C, lb.L));
         CK(c, cudaFreeAsync(dx, c->stream));
     }
-    return crocco_fill_boundary(c, met, CROCCO_FIELD_METRIC);
+    return fill_all(c, met, CROCCO_FIELD_METRIC, nullptr, 0.0);
 }
 
 // ---------------------------------------------------------------------------
 // RHS / RK
 // ---------------------------------------------------------------------------
 static const double RK_A[3] = {0.0, -5.0 / 9.0, -153.0 / 128.0};
+static const double RK_C[3] = {0.0, 1.0 / 3.0, 3.0 / 4.0};  // stage times (reading 13)
 static const double RK_B[3] = {1.0 / 3.0, 15.0 / 16.0, 8.0 / 15.0};
 
 // One RHS evaluation of a block (Alg. 2 l.5-9): primitives, viscous point
@@ -858,7 +902,7 @@ crocco_status crocco_rk_stage(crocco_ctx c, int32_t stage, double dt, double *co
     for (size_t bi = 0; bi < c->loc.size(); bi++)
         if (Uin[bi] == Uout[bi] || dU[bi] == Uin[bi] || dU[bi] == Uout[bi])
             return fail(c, CROCCO_ERR_ARG, "U_in, U_out and dU must be distinct");
-    if ((st = crocco_fill_boundary(c, Uin, CROCCO_FIELD_STATE))) return st;
+    if ((st = fill_all(c, Uin, CROCCO_FIELD_STATE, M, c->time + RK_C[stage] * dt))) return st;
     for (size_t bi = 0; bi < c->loc.size(); bi++) {
         if ((st = rhs_block(c, c->loc[bi], Uin[bi], M[bi], 3, nullptr, Uin[bi], Uout[bi], dU[bi], stage,
                             dt)))
@@ -882,8 +926,15 @@ crocco_status crocco_rk3_step(crocco_ctx c, double dt, double *const *U, double 
     if ((st = check_ptrs(c, U, "U")) || (st = check_ptrs(c, V, "V")) || (st = check_ptrs(c, dU, "dU")) ||
         (st = check_ptrs(c, M, "metrics")))
         return st;
-    if (!use_graph || c->timing || c->desc.nranks > 1 || c->stream == nullptr)
-        return rk3_eager(c, dt, U, V, dU, M);
+    bool moving = false;
+    for (int d = 0; d < 3; d++)
+        for (int sd = 0; sd < 2; sd++)
+            moving = moving || (c->desc.bc[d][sd] == CROCCO_BC_SPLIT && c->desc.split[d][sd].di_dt != 0.0);
+    if (!use_graph || c->timing || c->desc.nranks > 1 || c->stream == nullptr || moving) {
+        st = rk3_eager(c, dt, U, V, dU, M);
+        if (st == CROCCO_OK) c->time = c->time + dt;
+        return st;
+    }
     std::vector<const void *> key;
     for (size_t b = 0; b < c->loc.size(); b++) {
         key.push_back(U[b]);
@@ -926,6 +977,7 @@ crocco_status crocco_rk3_step(crocco_ctx c, double dt, double *const *U, double 
     }
     CK(c, cudaGraphLaunch(g->exec, c->stream));
     c->launches += g->nodes;
+    c->time = c->time + dt;
     return CROCCO_OK;
 }
 

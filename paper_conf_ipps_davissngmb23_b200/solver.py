@@ -16,7 +16,8 @@ GC = cc.GHOST_COORDS
 
 class Solver:
     def __init__(self, n_global, n_blocks=(1, 1, 1), bc=((0, 0),) * 3, phys=None, dirichlet=None,
-                 rank=0, nranks=1, block_rank=None, device=None, stream=None, nccl_unique_id=None):
+                 rank=0, nranks=1, block_rank=None, device=None, stream=None, nccl_unique_id=None,
+                 split=None):
         if not torch.cuda.is_available():
             raise RuntimeError("libcrocco needs a CUDA device (no CPU fallback)")
         if device is None:
@@ -28,7 +29,7 @@ class Solver:
         self.stream = stream if stream is not None else torch.cuda.current_stream(self.device)
         self.phys = phys if phys is not None else cc.make_phys()
         self.desc = cc.make_desc(n_global, n_blocks, bc, dirichlet, rank, nranks, block_rank,
-                                 self.stream.cuda_stream, nccl_unique_id)
+                                 self.stream.cuda_stream, nccl_unique_id, split)
         self.ctx = cc.crocco_init_grid(self.desc, self.phys)
         self.nloc = cc.crocco_num_local_blocks(self.ctx)
         self.layouts = [cc.crocco_get_block_layout(self.ctx, b) for b in range(self.nloc)]
@@ -102,7 +103,15 @@ class Solver:
 
     # ------------------------------------------------------------ hot path
     def fill(self, bufs=None, kind=cc.FIELD_STATE):
-        cc.crocco_fill_boundary(self.ctx, self._ptrs(bufs if bufs is not None else self.U), kind)
+        cc.crocco_fill_boundary(self.ctx, self._ptrs(bufs if bufs is not None else self.U), kind,
+                                self._ptrs(self.met) if kind == cc.FIELD_STATE else None)
+
+    def set_time(self, t):
+        cc.crocco_set_time(self.ctx, t)
+
+    @property
+    def time(self):
+        return cc.crocco_get_time(self.ctx)
 
     def rhs(self):
         if self.rhs_buf is None:

@@ -293,7 +293,43 @@ class Case:
     steps: int = 100
 
 
-P, E, D, W = 0, 1, 2, 3
+P, E, D, W, SW, SPL = 0, 1, 2, 3, 4, 5
+
+
+# ---------------------------------------------------------------- double Mach reflection
+
+DMR_PRE = (1.4, 0.0, 0.0, 0.0, 1.0)          # rho, u, v, w, p ahead of the shock (c = 1)
+DMR_POST = (8.0, 8.25 * math.cos(math.pi / 6), -8.25 * math.sin(math.pi / 6), 0.0, 116.5)
+DMR_X0 = 1.0 / 6.0                           # shock foot on the bottom wall at t = 0
+
+
+def dmr_shock_x(y, t):
+    """Woodward & Colella (1984): Mach-10 shock at 60 deg to the wall, x_s = 1/6 + (y + 20 t)/sqrt(3)."""
+    return DMR_X0 + (y + 20.0 * t) / math.sqrt(3.0)
+
+
+def dmr_state(xyz, gamma=1.4):
+    """Post-shock state left of the inclined shock, pre-shock state right of it."""
+    X = _interior_xyz(xyz)
+    post = X[0] < DMR_X0 + X[1] / math.sqrt(3.0)
+    q = [np.where(post, b, a) for a, b in zip(DMR_PRE, DMR_POST)]
+    return prim_to_cons(*q, gamma=gamma)
+
+
+def dmr_bc(h, gamma=1.4):
+    """BCs of the DMR on a Cartesian grid of spacing h (x_i = (i+1/2) h), as
+    (bc, dirichlet, split spec): xi lo post-shock inflow, xi hi extrapolation,
+    eta lo: post-shock for x < 1/6 then reflecting (slip) wall, eta hi: the exact
+    shock motion x_s(1, t) (post-shock behind, pre-shock ahead), zeta periodic."""
+    pre = [float(v) for v in prim_to_cons(*[np.float64(a) for a in DMR_PRE], gamma=gamma)]
+    post = [float(v) for v in prim_to_cons(*[np.float64(a) for a in DMR_POST], gamma=gamma)]
+    bc = ((D, E), (SPL, SPL), (P, P))
+    dirichlet = np.zeros((3, 2, 5))
+    dirichlet[0, 0] = post
+    split = {(1, 0): dict(axis=0, i0=DMR_X0 / h, di_dt=0.0, left=post, right_kind=SW),
+             (1, 1): dict(axis=0, i0=(DMR_X0 + 1.0 / math.sqrt(3.0)) / h,
+                          di_dt=20.0 / (math.sqrt(3.0) * h), left=post, right_kind=D, right=pre)}
+    return bc, dirichlet, split
 
 
 def case(name: str, scale: int = 1) -> Case:
@@ -318,6 +354,14 @@ def case(name: str, scale: int = 1) -> Case:
         return Case("ramp", N, (2, 2, 2), ((E, E), (W, E), (P, P)), Ramp(N=N), "ramp",
                     dict(gamma=1.4, R=1.0, Pr=0.72, mu_law=1, mu_ref=1e-4, T_ref=1.0, S=0.3),
                     dt=2e-5 * scale, steps=100)
+    if name == "dmr":
+        # the paper's test case on a uniform grid, no AMR:
+        # [0,4] x [0,1] x [0,Lz], 2048 x 512 x 128 in 2 x 2 x 1 blocks (scale divides)
+        N = (2048 // scale, 512 // scale, 128 // scale)
+        h = 1.0 / N[1]
+        bc, _, _ = dmr_bc(h)
+        return Case("dmr", N, (2, 2, 1) if scale < 8 else (1, 1, 1), bc, Cartesian(h=(h, h, h)), "dmr",
+                    dict(gamma=1.4, R=1.0, terms=1), dt=0.2 * h / 13.0, steps=100)
     if name == "weak":
         N = 512 // scale
         return Case("weak", (N, N, N), (1, 1, 1), ((P, P),) * 3,
@@ -340,6 +384,8 @@ def block_inputs(c: Case, origin, n, gamma=1.4):
         U = tgv(xyz, gamma=gamma, noise=0.01, seed=5)
     elif c.state == "ramp":
         U = ramp_state(xyz, c.grid, gamma=gamma)
+    elif c.state == "dmr":
+        U = dmr_state(xyz, gamma=gamma)
     else:
         raise KeyError(c.state)
     return xyz, U

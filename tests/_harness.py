@@ -67,21 +67,25 @@ def rel_linf(got, ref, floor=0.0):
 class Problem:
     """A global problem: grid object, BCs, initial interior state (global)."""
 
-    def __init__(self, n, grid, bc, U_interior, phys_kw=None, dirichlet=None):
+    def __init__(self, n, grid, bc, U_interior, phys_kw=None, dirichlet=None, split=None):
         self.n = tuple(n)
         self.grid = grid
         self.bc = bc
         self.U0 = U_interior
         self.phys_kw = dict(phys_kw or {})
         self.dirichlet = dirichlet
+        self.split = split  # {(d, side): spec} for SPLIT faces
 
     # ---------------- oracle side (global single block)
     def oracle_inputs(self):
         xyz = self.grid.coords(self.n, (0, 0, 0), oracle.GC)
         met = oracle.metrics(self.n, self.bc, xyz)
         U = synth.pad_state(self.U0)
-        oracle.fill(self.n, self.bc, U, dirichlet=self.dirichlet)
+        oracle.fill(self.n, self.bc, U, dirichlet=self.dirichlet, split=self.oracle_split(), met=met)
         return xyz, met, U
+
+    def oracle_split(self):
+        return oracle.splits(self.split) if self.split else None
 
     def oracle_phys(self):
         return oracle.phys(**self.phys_kw)
@@ -92,7 +96,8 @@ class Problem:
         from paper_conf_ipps_davissngmb23_b200.solver import Solver
         kw = dict(self.phys_kw)
         kw.pop("weno_linear", None)
-        S = Solver(self.n, n_blocks, self.bc, cc.make_phys(**kw), dirichlet=self.dirichlet)
+        S = Solver(self.n, n_blocks, self.bc, cc.make_phys(**kw), dirichlet=self.dirichlet,
+                   split=self.split)
         bn, blocks = block_slices(self.n, n_blocks)
         xyz = [self.grid.coords(bn, o, oracle.GC) for o, _ in blocks]
         S.set_coords(xyz)

@@ -324,6 +324,55 @@ def test_full_size_config_sampled(name):
     S.close()
 
 
+# ------------------------------------------------------------------ DMR (NEXT-2): SLIPWALL / SPLIT faces
+
+def _dmr_problem(scale=16):
+    c = synth.case("dmr", scale=scale)
+    h = 1.0 / c.n_global[1]
+    bc, dv, spec = synth.dmr_bc(h)
+    xyz = c.grid.coords(c.n_global, (0, 0, 0), oracle.GC)
+    return c, Problem(c.n_global, c.grid, bc, synth.dmr_state(xyz), c.phys, dirichlet=dv, split=spec)
+
+
+@pytest.mark.parametrize("nb", [(1, 1, 1), (2, 2, 1)])
+def test_fill_slipwall_split_parity(nb):
+    c, pb = _dmr_problem()
+    # random state so every ghost value is distinguishable; move the top split with t
+    pb.U0 = synth.random_state(pb.n, seed=31)
+    t = 0.0123
+    xyz, met, Uref = pb.oracle_inputs()
+    oracle.fill(pb.n, pb.bc, Uref, dirichlet=pb.dirichlet, split=pb.oracle_split(), t=t, met=met)
+    S = pb.solver(nb)
+    S.set_time(t)
+    S.fill()
+    bn, blocks = block_slices(pb.n, nb)
+    for b, (o, _) in enumerate(blocks):
+        got = S.view(S.U[b], b, 5).cpu().numpy()
+        ref = Uref[:, o[2]:o[2] + bn[2] + 8, o[1]:o[1] + bn[1] + 8, o[0]:o[0] + bn[0] + 8]
+        # copies and constants are exact; slip-wall reflections round differently (FMA)
+        assert np.abs(got - ref).max() <= 1e-14 * np.abs(ref).max(), b
+    S.close()
+
+
+def test_dmr_rk3_parity_and_decomposition():
+    c, pb = _dmr_problem()
+    n = pb.n
+    _, met, U = pb.oracle_inputs()
+    steps = 40
+    oracle.advance(n, pb.bc, pb.oracle_phys(), c.dt, steps, U, met, dirichlet=pb.dirichlet,
+                   split=pb.oracle_split())
+    outs = []
+    for nb in [(1, 1, 1), (2, 2, 1)]:
+        S = pb.solver(nb)
+        S.step(c.dt, steps)
+        S.sync()
+        assert abs(S.time - steps * c.dt) < 1e-15
+        outs.append(pb.gather(S, S.get(S.U)))
+        S.close()
+    assert np.array_equal(outs[0], outs[1])
+    assert rel_linf(outs[0], inner(U), state_scale(inner(U))) < 1e-9
+
+
 # ------------------------------------------------------------------ CUDA-graph RK3 steps
 
 def test_rk3_step_graph_equals_eager_bitwise():
