@@ -48,6 +48,8 @@ WORKLOADS = {
     "tgv": "tgv: Taylor-Green vortex 256^3 on the wavy grid, viscous (configs[2])",
     "vortex": "vortex: isentropic vortex on the wavy periodic 64^3 grid, inviscid (configs[1])",
     "sod": "sod: Sod shock tube 200x4x4, inviscid (configs[0])",
+    "dmr": "dmr: double Mach reflection 2048x512x128 in 2x2x1 blocks, slip wall + moving shock BCs "
+           "(the paper's case, PAPER.md:183-185; SURVEY NEXT-2)",
 }
 
 
@@ -218,8 +220,11 @@ def run_crocco(args, rank, world, local_rank):
         n, nb, bc, grid, phys, dt = case.n_global, case.n_blocks, case.bc, case.grid, case.phys, case.dt
         nbt = nb[0] * nb[1] * nb[2]
         block_rank = [bb * world // nbt for bb in range(nbt)]
-    S = Solver(n, nb, bc, cc.make_phys(**phys), rank=rank, nranks=world,
-               block_rank=block_rank, device=dev, nccl_unique_id=uid)
+    dirichlet, split = None, None
+    if args.config == "dmr":
+        bc, dirichlet, split = synth.dmr_bc(1.0 / n[1])
+    S = Solver(n, nb, bc, cc.make_phys(**phys), rank=rank, nranks=world, dirichlet=dirichlet,
+               block_rank=block_rank, device=dev, nccl_unique_id=uid, split=split)
     for bl in range(S.nloc):
         L = S.layouts[bl]
         origin, bn = tuple(L.origin), tuple(L.n)
@@ -391,7 +396,7 @@ def main():
     ap.add_argument("--steps", type=int, default=5)
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--impl", choices=["crocco", "reference"], default="crocco")
-    ap.add_argument("--config", choices=["weak", "ramp", "tgv", "vortex", "sod"], default="weak",
+    ap.add_argument("--config", choices=["weak", "ramp", "tgv", "vortex", "sod", "dmr"], default="weak",
                     help="weak (default, the north_star 512^3/GPU workload) or a fixed BASELINE config")
     ap.add_argument("--e2e-steps", type=int, default=2)
     ap.add_argument("--no-cpu-baseline", action="store_true")
