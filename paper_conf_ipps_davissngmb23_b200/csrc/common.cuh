@@ -67,6 +67,13 @@ __device__ __forceinline__ double sqrt_nr(double x) {  // x > 0
     return fma(0.5 * r, fma(-s, s, x), s);  // one Newton correction of s
 }
 
+// max of two NON-NEGATIVE doubles by their bit patterns (IEEE order = integer order
+// for x >= 0): compare on the integer pipe instead of DSETP on the FP64 pipe.
+__device__ __forceinline__ double maxnn(double a, double b) {
+    const long long x = __double_as_longlong(a), y = __double_as_longlong(b);
+    return __longlong_as_double(x > y ? x : y);
+}
+
 // primitive buffer components (k_prims)
 enum { PU = 0, PV = 1, PW = 2, PP = 3, PC = 4, PSR = 5, PH = 6, PT = 7, NPRIM = 8 };
 

@@ -140,9 +140,9 @@ __device__ __forceinline__ void total_flux(const Acc &A, bool inv, bool visc, co
             const double cl = A.P(l, PC);
             th[l] = t;
             pl[l] = A.P(l, PP);
-            lam0 = fmax(lam0, fabs(t));
-            lam3 = fmax(lam3, fabs(t + cl));
-            lam4 = fmax(lam4, fabs(t - cl));
+            lam0 = maxnn(lam0, fabs(t));
+            lam3 = maxnn(lam3, fabs(t + cl));
+            lam4 = maxnn(lam4, fabs(t - cl));
         }
         const double eps_b = 4.0 * WENO_BSCALE * ph.eps;  // b-units (weno.cuh) x 4 (folded 1/2)
         const double onemp = fma(-phi2, ic2, 1.0);

@@ -29,23 +29,21 @@ __device__ __forceinline__ WenoFrac weno_symbo_frac(double v0, double v1, double
                      C3 = 0.068988910311;
     constexpr double K3 = 3.0 / 13.0;
     const double d0 = v1 - v0, d1 = v2 - v1, d2 = v3 - v2, d3 = v4 - v3, d4 = v5 - v4;
-    const double r0 = fma(5.0, d1, -2.0 * d0);
-    const double r1 = fma(2.0, d2, d1);
-    const double r2 = fma(4.0, d2, -d3);
-    const double r3 = fma(6.0, d2, fma(-5.0, d3, 2.0 * d4));
     const double s0 = d1 - d0, s1 = d2 - d1, s2 = d3 - d2, s3 = d4 - d3;
     const double f0 = fma(3.0, d1, -d0);
     const double f1 = d1 + d2;
     const double f2 = fma(-3.0, d2, d3);
     const double f3 = fma(5.0, d3, -3.0 * d4);
+    const double r0 = fma(2.0, f0, -d1);         // 5 d1 - 2 d0
+    const double r1 = fma(2.0, d2, d1);
+    const double r2 = fma(4.0, d2, -d3);
+    const double r3 = fma(6.0, d2, -f3) - d4;    // 6 d2 - 5 d3 + 2 d4
     const double b0 = fma(K3 * f0, f0, s0 * s0);
     const double b1 = fma(K3 * f1, f1, s1 * s1);
     const double b2 = fma(K3 * f2, f2, s2 * s2);
     double b3 = fma(K3 * f3, f3, s3 * s3);
     // downwind stencil never preferred (continuous max, parity-safe)
-    const double m01 = b0 > b1 ? b0 : b1;
-    const double m23 = b2 > b3 ? b2 : b3;
-    b3 = m01 > m23 ? m01 : m23;
+    b3 = maxnn(maxnn(b0, b1), maxnn(b2, b3));
     double e0 = eps_b + b0, e1 = eps_b + b1, e2 = eps_b + b2, e3 = eps_b + b3;
     e0 *= e0;
     e1 *= e1;

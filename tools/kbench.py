@@ -14,16 +14,25 @@ xyz = torch.from_numpy(grid.coords(n, (0, 0, 0), 10)).cuda()
 S.set_coords([xyz]); S.set_state([synth.tgv(xyz, noise=0.01, seed=5)]); del xyz
 for s in range(3): S.stage(s, 2e-4)
 torch.cuda.synchronize()
-cc.crocco_set_timing(S.ctx, True); cc.crocco_kernel_times(S.ctx)
-e0 = torch.cuda.Event(enable_timing=True); e1 = torch.cuda.Event(enable_timing=True)
-e0.record()
-for it in range(2):
-    for s in range(3): S.stage(s, 2e-4)
-e1.record(); torch.cuda.synchronize()
-kt = cc.crocco_kernel_times(S.ctx)
-tot = e0.elapsed_time(e1) / 6
+REPS = int(os.environ.get("KB_REPS", "3"))
+best = None
+best_k = {}
+for rep in range(REPS):
+    cc.crocco_set_timing(S.ctx, True); cc.crocco_kernel_times(S.ctx)
+    e0 = torch.cuda.Event(enable_timing=True); e1 = torch.cuda.Event(enable_timing=True)
+    e0.record()
+    for it in range(2):
+        for s in range(3): S.stage(s, 2e-4)
+    e1.record(); torch.cuda.synchronize()
+    kt = cc.crocco_kernel_times(S.ctx)
+    tot = e0.elapsed_time(e1) / 6
+    best = tot if best is None else min(best, tot)
+    for k, v in kt.items():
+        if v[0]:
+            best_k[k] = min(best_k.get(k, 1e30), v[1] / v[0])
+tot = best
 out = {"lib": os.path.basename(cc.LIB_PATH), "ms_per_stage": tot, "pts_stage_per_s": N ** 3 / tot * 1e3,
-       "kernels_ms": {k: round(v[1] / max(v[0], 1), 3) for k, v in kt.items() if v[0]}}
+       "kernels_ms": {k: round(v, 3) for k, v in best_k.items()}}
 U = S.view(S.U[0], 0, 5)[:, 4:-4, 4:-4, 4:-4]
 out["finite"] = bool(torch.isfinite(U).all().item())
 print(json.dumps(out), flush=True)
