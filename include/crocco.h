@@ -112,6 +112,9 @@ typedef struct {
     double weno_eps;       /* WENO-SYMBO epsilon in alpha_k = C_k/(eps+beta_k)^2 (reading 8), 1e-6 */
     int32_t terms;         /* CROCCO_TERM_* bitmask */
     int32_t dir_mask;      /* inviscid directions evaluated, bit d = direction d (tests; 7 = all) */
+    int32_t weno_weights;  /* optimal weights: 0 = SYMBO (bandwidth-optimised, Martin et al. 2006),
+                              1 = SYMOO (1/20, 9/20, 9/20, 1/20: 6th-order central linear stencil);
+                              reading 22, SURVEY NEXT-3 */
 } crocco_phys;
 
 typedef struct {

@@ -52,6 +52,7 @@ typedef struct {
     double weno_eps;
     int32_t terms, dir_mask;
     int32_t weno_linear; /* test flag: 1 forces omega_k = C_k (linear stencil) */
+    int32_t weno_weights; /* 0: SYMBO (Martin et al. 2006), 1: SYMOO (reading 22, NEXT-3) */
 } oracle_phys;
 
 typedef struct {
@@ -302,9 +303,11 @@ void oracle_metrics(const int64_t n[3], const int32_t bc[6], const double *xyz, 
 /*    W(v_{-2..3}) reconstructs the value at the +1/2 interface.       */
 /* ------------------------------------------------------------------ */
 static const double C_SYMBO[4] = {0.094647545896, 0.428074212384, 0.408289331408, 0.068988910311};
+static const double C_SYMOO[4] = {1.0 / 20.0, 9.0 / 20.0, 9.0 / 20.0, 1.0 / 20.0};
 
-double oracle_weno_symbo(const double v[6], double eps, int linear)
+double oracle_weno(const double v[6], double eps, int linear, int weights)
 {
+    const double *Cw = weights == 1 ? C_SYMOO : C_SYMBO;
     /* v[0..5] = v_{-2}, v_{-1}, v_0, v_1, v_2, v_3 */
     double q[4], beta[4];
     q[0] = v[0] / 3.0 - 7.0 * v[1] / 6.0 + 11.0 * v[2] / 6.0;
@@ -337,14 +340,19 @@ double oracle_weno_symbo(const double v[6], double eps, int linear)
     double alpha[4], asum = 0.0, num = 0.0;
     for (int k = 0; k < 4; k++) {
         if (linear)
-            alpha[k] = C_SYMBO[k];
+            alpha[k] = Cw[k];
         else
-            alpha[k] = C_SYMBO[k] / ((eps + beta[k]) * (eps + beta[k]));
+            alpha[k] = Cw[k] / ((eps + beta[k]) * (eps + beta[k]));
         asum = asum + alpha[k];
     }
     for (int k = 0; k < 4; k++)
         num = num + alpha[k] * q[k];
     return num / asum;
+}
+
+double oracle_weno_symbo(const double v[6], double eps, int linear)
+{
+    return oracle_weno(v, eps, linear, 0);
 }
 
 /* ------------------------------------------------------------------ */
@@ -489,8 +497,8 @@ void oracle_interface_flux(const oracle_phys *ph, const double Ul[30], const dou
             vp[l] = 0.5 * (g[s][l] + lam[s] * wv[s][l]);
             vm[5 - l] = 0.5 * (g[s][l] - lam[s] * wv[s][l]); /* mirrored: i+3 .. i-2 */
         }
-        gh[s] = oracle_weno_symbo(vp, ph->weno_eps, ph->weno_linear) +
-                oracle_weno_symbo(vm, ph->weno_eps, ph->weno_linear);
+        gh[s] = oracle_weno(vp, ph->weno_eps, ph->weno_linear, ph->weno_weights) +
+                oracle_weno(vm, ph->weno_eps, ph->weno_linear, ph->weno_weights);
     }
     for (int q = 0; q < 5; q++) {
         double f = 0.0;

@@ -16,6 +16,7 @@ struct Phys {
     double mu_ref, T_ref, S;
     double eps;
     int terms, dir_mask;
+    double wC[4];  // WENO optimal weights (SYMBO or SYMOO)
 };
 
 struct Lay {  // padded block layout (elements)

@@ -383,6 +383,9 @@ static Phys to_phys(const crocco_phys *p) {
     ph.eps = p->weno_eps;
     ph.terms = p->terms;
     ph.dir_mask = p->dir_mask;
+    static const double SYMBO[4] = {0.094647545896, 0.428074212384, 0.408289331408, 0.068988910311};
+    static const double SYMOO[4] = {1.0 / 20.0, 9.0 / 20.0, 9.0 / 20.0, 1.0 / 20.0};
+    for (int k = 0; k < 4; k++) ph.wC[k] = p->weno_weights == 1 ? SYMOO[k] : SYMBO[k];
     return ph;
 }
 
@@ -393,6 +396,7 @@ static crocco_status check_phys(const crocco_phys *p) {
     if (p->mu_law != 0 && p->mu_law != 1) return fail(nullptr, CROCCO_ERR_ARG, "bad mu_law");
     if (p->mu_law == 1 && !(p->T_ref > 0)) return fail(nullptr, CROCCO_ERR_ARG, "bad T_ref");
     if (p->terms & ~3) return fail(nullptr, CROCCO_ERR_ARG, "bad terms mask");
+    if (p->weno_weights != 0 && p->weno_weights != 1) return fail(nullptr, CROCCO_ERR_ARG, "bad weno_weights");
     return CROCCO_OK;
 }
 

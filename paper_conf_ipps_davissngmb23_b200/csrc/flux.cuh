@@ -218,7 +218,7 @@ __device__ __forceinline__ void total_flux(const Acc &A, bool inv, bool visc, co
                 gp[l] = fma(lam, w, g);
                 gm[l] = fma(-lam, w, g);
             }
-            const double gh = weno_pair(gp, gm, eps_b);
+            const double gh = weno_pair(gp, gm, eps_b, ph.wC);
             f0 = fma(R0, gh, f0);
             f1 = fma(R1, gh, f1);
             f2 = fma(R2, gh, f2);

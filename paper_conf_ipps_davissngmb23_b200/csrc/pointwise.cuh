@@ -115,6 +115,9 @@ __global__ void __launch_bounds__(256) k_visc(const double *__restrict__ Pm,
 // k-2..k+2 in registers (k-derivatives), and only the current plane k (with a
 // 2-point i/j halo) is staged in shared memory (i/j-derivatives), double
 // buffered so one barrier per plane suffices.
+#ifndef CROCCO_VISC_MINB
+#define CROCCO_VISC_MINB 1
+#endif
 #ifndef CROCCO_VISC_PREFETCH
 #define CROCCO_VISC_PREFETCH 1  // load the next plane's U / metrics one step ahead (registers)
 #endif
@@ -136,7 +139,7 @@ __device__ __forceinline__ void prim4(const double *__restrict__ U, int64_t cs, 
     out[3] = pr * ir * iR;
 }
 
-__global__ void __launch_bounds__(VTX * VTY) k_visc_tiled(const double *__restrict__ U,
+__global__ void __launch_bounds__(VTX * VTY, CROCCO_VISC_MINB) k_visc_tiled(const double *__restrict__ U,
                                                           const double *__restrict__ M,
                                                           double *__restrict__ FV, Lay L, VLay V,
                                                           Phys ph) {

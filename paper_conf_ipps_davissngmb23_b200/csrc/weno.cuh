@@ -1,6 +1,7 @@
 // weno.cuh -- WENO-SYMBO reconstruction (PAPER.md:50 -> ref [9]; reading 8).
 //
 // W(v_{-2..3}) reconstructs the value at the +1/2 interface from 4 candidate
+// (optimal weights C: SYMBO by default, SYMOO selectable, reading 22)
 // 3-point stencils (the 4th one downwind), Jiang-Shu smoothness indicators with
 // beta_3 <- max(beta_0..beta_3), weights alpha_k = C_k/(eps+beta_k)^2.
 //
@@ -24,9 +25,9 @@ struct WenoFrac {
 };
 
 __device__ __forceinline__ WenoFrac weno_symbo_frac(double v0, double v1, double v2, double v3,
-                                                    double v4, double v5, double eps_b) {
-    constexpr double C0 = 0.094647545896, C1 = 0.428074212384, C2 = 0.408289331408,
-                     C3 = 0.068988910311;
+                                                    double v4, double v5, double eps_b,
+                                                    const double C[4]) {
+    const double C0 = C[0], C1 = C[1], C2 = C[2], C3 = C[3];
     constexpr double K3 = 3.0 / 13.0;
     const double d0 = v1 - v0, d1 = v2 - v1, d2 = v3 - v2, d3 = v4 - v3, d4 = v5 - v4;
     const double s0 = d1 - d0, s1 = d2 - d1, s2 = d3 - d2, s3 = d4 - d3;
@@ -62,9 +63,10 @@ __device__ __forceinline__ WenoFrac weno_symbo_frac(double v0, double v1, double
 // W^+ of (vp0..vp5) plus W^- of the mirrored (vm5..vm0), as one fraction:
 // (b+ + b-) + (n+ d- + n- d+)/(6 d+ d-)  -- one division per characteristic field.
 // Range: the alpha products stay inside fp64 for |v| up to ~1e9.
-__device__ __forceinline__ double weno_pair(const double vp[6], const double vm[6], double eps_b) {
-    const WenoFrac a = weno_symbo_frac(vp[0], vp[1], vp[2], vp[3], vp[4], vp[5], eps_b);
-    const WenoFrac b = weno_symbo_frac(vm[5], vm[4], vm[3], vm[2], vm[1], vm[0], eps_b);
+__device__ __forceinline__ double weno_pair(const double vp[6], const double vm[6], double eps_b,
+                                            const double C[4]) {
+    const WenoFrac a = weno_symbo_frac(vp[0], vp[1], vp[2], vp[3], vp[4], vp[5], eps_b, C);
+    const WenoFrac b = weno_symbo_frac(vm[5], vm[4], vm[3], vm[2], vm[1], vm[0], eps_b, C);
     return (a.base + b.base) + div_nr(fma(a.num, b.den, b.num * a.den), 6.0 * (a.den * b.den));
 }
 

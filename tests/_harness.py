@@ -95,7 +95,7 @@ class Problem:
         from paper_conf_ipps_davissngmb23_b200 import crocco as cc
         from paper_conf_ipps_davissngmb23_b200.solver import Solver
         kw = dict(self.phys_kw)
-        kw.pop("weno_linear", None)
+        kw.pop("weno_linear", None)  # oracle-only test flag
         S = Solver(self.n, n_blocks, self.bc, cc.make_phys(**kw), dirichlet=self.dirichlet,
                    split=self.split)
         bn, blocks = block_slices(self.n, n_blocks)

@@ -109,10 +109,11 @@ def _rhs_parity(pb, nb=(1, 1, 1)):
     return rel_linf(got, ref, flux_scale(U, met)), got, ref
 
 
-@pytest.mark.parametrize("terms,mask", [(1, 1), (1, 2), (1, 4), (1, 7), (2, 7), (3, 7)])
-def test_rhs_parity_terms(terms, mask):
+@pytest.mark.parametrize("terms,mask,weights", [(1, 1, 0), (1, 2, 0), (1, 4, 0), (1, 7, 0), (2, 7, 0),
+                                                (3, 7, 0), (3, 7, 1)])
+def test_rhs_parity_terms(terms, mask, weights):
     n = (37, 29, 23)   # ragged w.r.t. every thread-block tile
-    pb = wavy_random(n, 2, dict(terms=terms, dir_mask=mask, mu_ref=0.02))
+    pb = wavy_random(n, 2, dict(terms=terms, dir_mask=mask, mu_ref=0.02, weno_weights=weights))
     err, _, _ = _rhs_parity(pb)
     assert err < 1e-11, err
 

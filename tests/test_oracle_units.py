@@ -456,3 +456,25 @@ def test_compute_dt_affine_grid_via_matrix_inverse():
     expect = 0.5 / lam.max()
     got = oracle.compute_dt(n, oracle.phys(), U, met, 0.5)
     assert abs(got - expect) < 1e-13 * expect
+
+
+# ------------------------------------------------------------------ SYMOO weights (NEXT-3, reading 22)
+
+def test_symoo_linear_stencil_is_sixth_order_central():
+    # C = (1, 9, 9, 1)/20 turns the 4 candidate stencils into the 6th-order central
+    # interface reconstruction (1, -8, 37, 37, -8, 1)/60
+    got = np.array([oracle.weno_symbo(np.eye(6)[l], linear=True, weights=1) for l in range(6)])
+    np.testing.assert_allclose(got, np.array([1, -8, 37, 37, -8, 1]) / 60.0, rtol=0, atol=1e-15)
+
+
+def test_symoo_exact_for_quintic_cell_averages_in_linear_mode():
+    rng = np.random.default_rng(8)
+    for _ in range(20):
+        coef = rng.normal(size=6)
+        v = _cell_avgs(coef, np.arange(-2, 4))
+        exact = np.polynomial.Polynomial(coef)(0.5)
+        assert abs(oracle.weno_symbo(v, linear=True, weights=1) - exact) < 1e-12 * (1 + abs(exact))
+
+
+def test_symoo_nonlinear_still_nonoscillatory():
+    assert abs(oracle.weno_symbo([0, 0, 0, 0, 1, 1], weights=1)) < 1e-9
