@@ -473,6 +473,8 @@ crocco_status crocco_init_grid(const crocco_grid_desc *desc, const crocco_phys *
     // device scratch
     auto alloc = [&](double **p, int64_t elems) -> bool {
         if (cudaMalloc((void **)p, (size_t)elems * sizeof(double)) != cudaSuccess) return false;
+        // defined padding: whole-tile copies of the sweeps read (and discard) row padding
+        if (cudaMemset(*p, 0, (size_t)elems * sizeof(double)) != cudaSuccess) return false;
         c->scratch += elems * (int64_t)sizeof(double);
         return true;
     };

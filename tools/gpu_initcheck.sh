@@ -1,0 +1,5 @@
+cd "${GRAFT_REPO_ROOT:-/root/repo}"; mkdir -p gpurun_out
+SEL="rhs_parity_terms or fill_bitwise or dmr or rk3_step_graph or compute_dt or minimum_block"
+timeout 1200 compute-sanitizer --tool initcheck --target-processes all --print-limit 20 \
+     python -m pytest tests/test_gpu_parity.py -q -x -k "$SEL" > gpurun_out/sanitize_initcheck.log 2>&1
+echo "exit $?" >> gpurun_out/sanitize_initcheck.log
