@@ -110,7 +110,7 @@ __global__ void __launch_bounds__(256) k_visc(const double *__restrict__ Pm,
 }
 
 // Same viscous point fluxes, fused with the primitive recovery: a CTA owns
-// 32 (i) x 8 (j) columns of the interior +-2 box and marches a slab of VK
+// VTX (i) x 8 (j) columns of the interior +-2 box and marches a slab of VK
 // planes in k.  Each thread keeps u, v, w, T of its own column for planes
 // k-2..k+2 in registers (k-derivatives), and only the current plane k (with a
 // 2-point i/j halo) is staged in shared memory (i/j-derivatives), double
@@ -121,7 +121,10 @@ __global__ void __launch_bounds__(256) k_visc(const double *__restrict__ Pm,
 #ifndef CROCCO_VISC_PREFETCH
 #define CROCCO_VISC_PREFETCH 1  // load the next plane's U / metrics one step ahead (registers)
 #endif
-constexpr int VTX = 32, VTY = 8, VK = 32;           // tile and slab
+#ifndef CROCCO_VISC_TX
+#define CROCCO_VISC_TX 16  // 16 x 8 tiles: two 4-warp CTAs per SM (measured 3 % faster than 32 x 8)
+#endif
+constexpr int VTX = CROCCO_VISC_TX, VTY = 8, VK = 32;  // tile and slab
 constexpr int VHX = VTX + 4, VHY = VTY + 4;          // with halo
 constexpr int VPL = VHX * VHY;                       // points per staged plane
 constexpr int VHALO = VPL - VTX * VTY;               // halo points per plane
@@ -170,7 +173,7 @@ __global__ void __launch_bounds__(VTX * VTY, CROCCO_VISC_MINB) k_visc_tiled(cons
         const int t = tid - 4 * VHX;      // 0..31
         const int c = t % 4;
         hy = 2 + t / 4;
-        hx = c < 2 ? c : VTX + c;         // 0,1 | 34,35
+        hx = c < 2 ? c : VTX + c;         // 0,1 | VTX+2, VTX+3
     }
     const int hgi = min(i0 - 2 + hx, L.n0 + G - 1), hgj = min(j0 - 2 + hy, L.n1 + G - 1);
     const int hidx = hy * VHX + hx;
