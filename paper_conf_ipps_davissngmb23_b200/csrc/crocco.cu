@@ -386,6 +386,11 @@ static Phys to_phys(const crocco_phys *p) {
     static const double SYMBO[4] = {0.094647545896, 0.428074212384, 0.408289331408, 0.068988910311};
     static const double SYMOO[4] = {1.0 / 20.0, 9.0 / 20.0, 9.0 / 20.0, 1.0 / 20.0};
     for (int k = 0; k < 4; k++) ph.wC[k] = p->weno_weights == 1 ? SYMOO[k] : SYMBO[k];
+#if CROCCO_WENO_FOLD
+    // only the ratios C_k / C_0 enter W (weno.cuh); alpha_0 then needs no multiply
+    const double c0 = ph.wC[0];
+    for (int k = 0; k < 4; k++) ph.wC[k] = k == 0 ? 1.0 : ph.wC[k] / c0;
+#endif
     return ph;
 }
 

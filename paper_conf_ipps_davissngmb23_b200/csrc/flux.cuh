@@ -24,6 +24,9 @@ namespace crocco {
 #ifndef CROCCO_FIELD_ROLLED
 #define CROCCO_FIELD_ROLLED 0  // 1: keep the characteristic-field loop rolled (fewer live registers)
 #endif
+#ifndef CROCCO_DEFER_DIV
+#define CROCCO_DEFER_DIV 1  // 1: the five WENO-pair divisions after the field loop (independent chains)
+#endif
 #ifndef CROCCO_SWEEP_UREG
 #define CROCCO_SWEEP_UREG 0  // 1: hold the 6x5 stencil states in registers; 0: re-read per field
 #endif
@@ -150,6 +153,9 @@ __device__ __forceinline__ void total_flux(const Acc &A, bool inv, bool visc, co
         const double cx = ny * wt - nz * vt, cy = nz * ut - nx * wt, cz = nx * vt - ny * ut;
         const double ph1 = phi2 * ph.igm1;
         double f0 = 0.0, f1 = 0.0, f2 = 0.0, f3 = 0.0, f4 = 0.0;
+#if CROCCO_DEFER_DIV
+        double gb[5], gn[5], gd[5];
+#endif
 #if CROCCO_FIELD_ROLLED
 #pragma unroll 1
 #else
@@ -218,7 +224,47 @@ __device__ __forceinline__ void total_flux(const Acc &A, bool inv, bool visc, co
                 gp[l] = fma(lam, w, g);
                 gm[l] = fma(-lam, w, g);
             }
+#if CROCCO_DEFER_DIV
+            const WenoFrac wf = weno_pair_frac(gp, gm, eps_b, ph.wC);
+            gb[sf] = wf.base;
+            gn[sf] = wf.num;
+            gd[sf] = wf.den;
+            (void)R0; (void)R1; (void)R2; (void)R3; (void)R4;
+        }
+#pragma unroll
+        for (int sf = 0; sf < 5; sf++) {
+            const double gh = gb[sf] + div_nr(gn[sf], gd[sf]);
+            double R0, R1, R2, R3, R4;
+            if (sf < 3) {
+                const double na = sf == 0 ? nx : (sf == 1 ? ny : nz);
+                R0 = na;
+                if (sf == 0) {
+                    R1 = na * ut;
+                    R2 = fma(na, vt, nz * rt);
+                    R3 = fma(na, wt, -ny * rt);
+                    R4 = fma(na, ph1, rt * (nz * vt - ny * wt));
+                } else if (sf == 1) {
+                    R1 = fma(na, ut, -nz * rt);
+                    R2 = na * vt;
+                    R3 = fma(na, wt, nx * rt);
+                    R4 = fma(na, ph1, rt * (nx * wt - nz * ut));
+                } else {
+                    R1 = fma(na, ut, ny * rt);
+                    R2 = fma(na, vt, -nx * rt);
+                    R3 = na * wt;
+                    R4 = fma(na, ph1, rt * (ny * ut - nx * vt));
+                }
+            } else {
+                const double sc = (sf == 3) ? ct : -ct;
+                R0 = alph;
+                R1 = alph * fma(sc, nx, ut);
+                R2 = alph * fma(sc, ny, vt);
+                R3 = alph * fma(sc, nz, wt);
+                R4 = alph * fma(phi2 + c2, ph.igm1, sc * tht);
+            }
+#else
             const double gh = weno_pair(gp, gm, eps_b, ph.wC);
+#endif
             f0 = fma(R0, gh, f0);
             f1 = fma(R1, gh, f1);
             f2 = fma(R2, gh, f2);

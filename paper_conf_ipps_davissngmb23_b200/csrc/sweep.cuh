@@ -25,6 +25,9 @@ namespace crocco {
 #ifndef CROCCO_SWEEP_MINB
 #define CROCCO_SWEEP_MINB 1  // min CTAs/SM (register cap); the staged ring allows 2 CTAs x 4 warps
 #endif
+#ifndef CROCCO_PRIMS_LATE
+#define CROCCO_PRIMS_LATE 0  // 1: next chunk's primitives computed at the end of the step (registers)
+#endif
 #ifndef CROCCO_SWEEP_THREADS
 #define CROCCO_SWEEP_THREADS 128
 #endif
@@ -291,25 +294,39 @@ __global__ void __launch_bounds__(SWEEP_THREADS, CROCCO_SWEEP_MINB) k_sweep_s(co
         }
         cp_async_commit();
     };
-    // primitives of chunk `ch` (one point per lane), from the staged state
-    auto prims = [&](int ch) {
+    // primitives of chunk `ch` (one point per lane), from the staged state:
+    // prim_calc into registers, prim_store into the ring
+    auto prim_calc = [&](int ch, double pv[7]) {
         const int q = ch * WS + ls;
         if (q > qmax) return;
-        double *bq = sv + (q & (NR - 1)) * C + lt;
+        const double *bq = sv + (q & (NR - 1)) * C + lt;
         const double rho = bq[0], ru = bq[VS], rv = bq[2 * VS], rw = bq[3 * VS], E = bq[4 * VS];
         const double ir = rcp_nr(rho);
         const double u = ru * ir, v = rv * ir, w = rw * ir;
         const double pr = ph.gm1 * fma(-0.5, fma(ru, u, fma(rv, v, rw * w)), E);
-        bq[(SV_P + PU) * VS] = u;
-        bq[(SV_P + PV) * VS] = v;
-        bq[(SV_P + PW) * VS] = w;
-        bq[(SV_P + PP) * VS] = pr;
-        bq[(SV_P + PC) * VS] = sqrt_nr(ph.gamma * pr * ir);
-#if !CROCCO_RING_LEAN
-        bq[(SV_P + PSR) * VS] = sqrt_nr(rho);
-        bq[(SV_P + PH) * VS] = (E + pr) * ir;
-#endif
+        pv[PU] = u;
+        pv[PV] = v;
+        pv[PW] = w;
+        pv[PP] = pr;
+        pv[PC] = sqrt_nr(ph.gamma * pr * ir);
+        pv[PSR] = sqrt_nr(rho);
+        pv[PH] = (E + pr) * ir;
     };
+    auto prim_store = [&](int ch, const double pv[7]) {
+        const int q = ch * WS + ls;
+        if (q > qmax) return;
+        double *bq = sv + (q & (NR - 1)) * C + lt;
+#pragma unroll
+        for (int k = 0; k < (CROCCO_RING_LEAN ? 5 : 7); k++) bq[(SV_P + k) * VS] = pv[k];
+    };
+    auto prims = [&](int ch) {
+        double pv[7];
+        prim_calc(ch, pv);
+        prim_store(ch, pv);
+    };
+#if CROCCO_PRIMS_LATE
+    double pnext[7];  // primitives of chunk st+LA, computed at the end of step st-1
+#endif
 
     // prologue: chunks 0 .. LA staged with primitives
     for (int ch = 0; ch <= LA; ch++) issue(ch);
@@ -333,10 +350,14 @@ __global__ void __launch_bounds__(SWEEP_THREADS, CROCCO_SWEEP_MINB) k_sweep_s(co
     for (int c = 0; c < 5; c++) Fc[c] = 0.0;
     for (int st = 0; st < nsteps; st++, rr += rstep, pp += pstep) {
         if (st > 0) {
+#if CROCCO_PRIMS_LATE
+            prim_store(st + LA, pnext);
+#else
             // chunk st+LA landed -> primitives
             cp_async_wait_all();
             __syncwarp();
             prims(st + LA);
+#endif
             __syncwarp();
         }
         const int e = e0 - 1 + WS * st + ls;  // this lane's interface e+1/2
@@ -408,7 +429,15 @@ __global__ void __launch_bounds__(SWEEP_THREADS, CROCCO_SWEEP_MINB) k_sweep_s(co
                 }
             }
         }
+#if CROCCO_PRIMS_LATE
+        // chunk st+LA+1 (issued at the top of this step) landed -> its primitives, kept in
+        // registers so their latency chain overlaps the tail of this step's flux
+        cp_async_wait_all();
         __syncwarp();
+        if (st + 1 < nsteps) prim_calc(st + 1 + LA, pnext);
+#else
+        __syncwarp();
+#endif
     }
     cp_async_wait_all();
 }

@@ -9,7 +9,7 @@ from paper_conf_ipps_davissngmb23_b200.solver import Solver
 N = int(os.environ.get("KB_N", "512"))
 n = (N, N, N)
 grid = synth.Wavy3D(L=(2 * math.pi,) * 3, N=n, x0=(-math.pi,) * 3, k=2.0, A=0.15)
-S = Solver(n, (1, 1, 1), ((0, 0),) * 3, cc.make_phys(gamma=1.4, R=1.0, Pr=0.71, mu_ref=1 / 1600, terms=3))
+S = Solver(n, (1, 1, 1), ((0, 0),) * 3, cc.make_phys(gamma=1.4, R=1.0, Pr=0.71, mu_ref=1 / 1600, terms=int(os.environ.get("KB_TERMS", "3"))))
 xyz = torch.from_numpy(grid.coords(n, (0, 0, 0), 10)).cuda()
 S.set_coords([xyz]); S.set_state([synth.tgv(xyz, noise=0.01, seed=5)]); del xyz
 for s in range(3): S.stage(s, 2e-4)
