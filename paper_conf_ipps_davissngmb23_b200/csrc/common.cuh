@@ -13,7 +13,7 @@ constexpr int GC = 10;  // coordinate ghost width (reading 7)
 struct Phys {
     double gamma, gm1, igm1, R, Pr, cp_over_Pr;  // cp/Pr = gamma R /((gamma-1) Pr)
     int mu_law;
-    double mu_ref, T_ref, S;
+    double mu_ref, T_ref, S, iT_ref;
     double eps;
     int terms, dir_mask;
     double wC[4];  // WENO optimal weights (SYMBO or SYMOO)

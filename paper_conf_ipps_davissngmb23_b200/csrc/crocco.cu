@@ -327,6 +327,8 @@ static cudaError_t sweep_attrs() {
     if (e == cudaSuccess) e = sweep_attr1<2, true>();
     if (e == cudaSuccess)
         e = cudaFuncSetAttribute(k_visc_tiled, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)VISC_SMEM);
+    if (e == cudaSuccess)
+        e = cudaFuncSetAttribute(k_visc_div, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)VDIV_SMEM);
     return e;
 }
 
@@ -379,6 +381,7 @@ static Phys to_phys(const crocco_phys *p) {
     ph.mu_law = p->mu_law;
     ph.mu_ref = p->mu_ref;
     ph.T_ref = p->T_ref;
+    ph.iT_ref = p->T_ref > 0 ? 1.0 / p->T_ref : 0.0;
     ph.S = p->S;
     ph.eps = p->weno_eps;
     ph.terms = p->terms;
@@ -484,10 +487,12 @@ crocco_status crocco_init_grid(const crocco_grid_desc *desc, const crocco_phys *
         return true;
     };
     for (auto &b : c->loc) {
-        bool ok = alloc(&b.prim, NPRIM * b.L.cs);
+        // primitives are only materialised by the global-load sweeps; point viscous fluxes only
+        // when the divergence is not fused (k_visc_div keeps them on chip)
+        bool ok = CROCCO_SWEEP_SMEM || alloc(&b.prim, NPRIM * b.L.cs);
         b.rcs = rup((int64_t)b.g.n[0] * b.g.n[1] * b.g.n[2], 32);
         ok = ok && alloc(&b.racc, 5 * b.rcs);
-        ok = ok && alloc(&b.fv, 12 * b.V.cs);
+        ok = ok && ((CROCCO_SWEEP_SMEM && CROCCO_VISC_DIV) || alloc(&b.fv, 12 * b.V.cs));
         if (!ok) {
             cudaGetLastError();
             free_ctx(c);
@@ -828,7 +833,12 @@ static crocco_status rhs_block(crocco_ctx c, const LocalBlock &b, const double *
     const int64_t np = (int64_t)(b.g.n[0] + 2 * G) * (b.g.n[1] + 2 * G) * (b.g.n[2] + 2 * G);
     if (!CROCCO_SWEEP_SMEM)  // the staged sweeps and the tiled viscous kernel compute their own primitives
         LAUNCH(c, K_PRIMS, k_prims<<<cdiv(np, 256), 256, 0, c->stream>>>(U, b.prim, b.L, ph));
-    if (viscous) {
+    const bool vdiv = viscous && CROCCO_SWEEP_SMEM && CROCCO_VISC_DIV;  // fused viscous divergence -> R
+    if (vdiv) {
+        const unsigned nt = (unsigned)(((b.g.n[0] + DTX - 1) / DTX) * ((b.g.n[1] + DTY - 1) / DTY) *
+                                       ((b.g.n[2] + DK - 1) / DK));
+        LAUNCH(c, K_VISC, k_visc_div<<<nt, DNT, VDIV_SMEM, c->stream>>>(U, M, b.racc, b.rcs, b.L, ph));
+    } else if (viscous) {
 #if CROCCO_SWEEP_SMEM
         const unsigned nt = (unsigned)(((b.V.b0 + VTX - 1) / VTX) * ((b.V.b1 + VTY - 1) / VTY) *
                                        ((b.V.b2 + VK - 1) / VK));
@@ -851,8 +861,8 @@ static crocco_status rhs_block(crocco_ctx c, const LocalBlock &b, const double *
         a.R = b.racc;
         a.rcs = b.rcs;
         a.inv = inviscid && (ph.dir_mask >> d & 1);
-        a.visc = viscous;
-        a.mode = d == 0 ? 0 : (d == 1 ? 1 : final_mode);
+        a.visc = viscous && !vdiv;
+        a.mode = d == 0 ? (vdiv ? 4 : 0) : (d == 1 ? 1 : final_mode);
         a.rhs = rhs;
         a.Uin = Uin;
         a.Uout = Uout;
@@ -874,9 +884,9 @@ static crocco_status rhs_block(crocco_ctx c, const LocalBlock &b, const double *
 #if CROCCO_SWEEP_SMEM
 #define SWEEP_LAUNCH(DD, VV) \
         k_sweep_s<DD, VV><<<grid, SWEEP_THREADS, sweep_smem_bytes<DD>(), c->stream>>>(a, b.L, ph)
-        if (d == 0) LAUNCH(c, K_FLUX_X, if (viscous) SWEEP_LAUNCH(0, true); else SWEEP_LAUNCH(0, false));
-        else if (d == 1) LAUNCH(c, K_FLUX_Y, if (viscous) SWEEP_LAUNCH(1, true); else SWEEP_LAUNCH(1, false));
-        else LAUNCH(c, K_FLUX_Z, if (viscous) SWEEP_LAUNCH(2, true); else SWEEP_LAUNCH(2, false));
+        if (d == 0) LAUNCH(c, K_FLUX_X, if (a.visc) SWEEP_LAUNCH(0, true); else SWEEP_LAUNCH(0, false));
+        else if (d == 1) LAUNCH(c, K_FLUX_Y, if (a.visc) SWEEP_LAUNCH(1, true); else SWEEP_LAUNCH(1, false));
+        else LAUNCH(c, K_FLUX_Z, if (a.visc) SWEEP_LAUNCH(2, true); else SWEEP_LAUNCH(2, false));
 #undef SWEEP_LAUNCH
 #else
         if (d == 0) LAUNCH(c, K_FLUX_X, k_sweep<0><<<grid, SWEEP_THREADS, 0, c->stream>>>(a, b.L, ph));

@@ -3,6 +3,7 @@
 // read in DESIGN.md sec. 3 (citations: PAPER.md line numbers); no code is
 // shared with oracle/.
 #pragma once
+#include <type_traits>
 #include "common.cuh"
 
 namespace crocco {
@@ -335,6 +336,290 @@ __global__ void __launch_bounds__(VTX * VTY, CROCCO_VISC_MINB) k_visc_tiled(cons
 #pragma unroll
         for (int c = 0; c < 10; c++) cM[c] = nM[c];
 #endif
+    }
+}
+
+// ---------------------------------------------------------------------------
+// Viscous divergence (Viscous; reading 12), fused end to end:
+//   R_visc(i,j,k) = sum_d D4_d F^_v^d   (momentum x, y, z and energy)
+// with the point fluxes F^_v^d of the same D4-gradient / Stokes / Fourier
+// construction as k_visc_tiled, evaluated where the divergence needs them and
+// never stored to HBM.  A CTA owns DTX (i) x DTY (j) interior columns and
+// marches a slab of DK output planes in k; per gradient plane g:
+//   phase 1: u, v, w, T of plane g+2 on the tile + 2-point halo (5-plane ring
+//            in shared memory) and of plane g on the 4-point i / j arms;
+//   phase 2: full gradients at plane g on the own points and on the 2-point
+//            i-arm / j-arm points; F^_v^xi (own + i-arm) and F^_v^eta (own +
+//            j-arm) to shared memory, F^_v^zeta of the own column to a 5-plane
+//            register queue;
+//   phase 3: D4_xi + D4_eta of plane g (3-plane register queue); plane g-2 is
+//            complete once D4_zeta of the queue is added -> R comps 1..4.
+// The point flux of a point is computed by one function with explicitly
+// rounded operations, so a point evaluated as a halo point of one tile equals
+// the same point evaluated as an own point of its neighbour tile bit for bit
+// (decomposition invariance).
+// ---------------------------------------------------------------------------
+#ifndef CROCCO_VISC_DIV
+#define CROCCO_VISC_DIV 0  // 1: fused viscous divergence (k_visc_div, measured slower: smem-bound); 0: point fluxes
+#endif
+#ifndef CROCCO_VDIV_MINB
+#define CROCCO_VDIV_MINB 2
+#endif
+#ifndef CROCCO_VDIV_TY
+#define CROCCO_VDIV_TY 8
+#endif
+#ifndef CROCCO_VDIV_TX
+#define CROCCO_VDIV_TX 16
+#endif
+#ifndef CROCCO_VDIV_K
+#define CROCCO_VDIV_K 64
+#endif
+constexpr int DTX = CROCCO_VDIV_TX, DTY = CROCCO_VDIV_TY, DK = CROCCO_VDIV_K;  // tile (i x j), slab (k)
+constexpr int DNT = DTX * DTY;                  // threads (one own column each)
+constexpr int DBW = DTX + 4;                    // ring rows: tile + 2-point halo
+constexpr int DNB = DBW * (DTY + 4);            // ring points per plane
+constexpr int DNA = 4 * DTY + 4 * DTX;          // 4-point arm points (current plane only)
+constexpr int DXW = DTX + 4;                    // F^xi rows: own + i-arm
+constexpr int DYH = DTY + 4;                    // F^eta columns: own + j-arm
+constexpr int DNX = DXW * DTY, DNY = DTX * DYH;
+constexpr size_t VDIV_SMEM = (size_t)(5 * 4 * DNB + 4 * DNA + 5 * 4 * DNT + 4 * DNX + 4 * DNY) * sizeof(double);
+
+// stress tensor / energy flux of a point from its computational-space gradient
+// gc[f][d] = D4_d f (f = u, v, w, T), metrics Mp[0..9] = (J, m^xi, m^eta, m^zeta)
+// and its u, v, w, T: returns tau (symmetric, 6) and hb = u_a tau_ab - q_b.
+// Every operation is an explicit rounding (no contraction freedom).
+__device__ __forceinline__ void visc_point(const double gc[4][3], const double Mp[10], double u, double v,
+                                           double w, double T, const Phys &ph, double tau[6], double hb[3]) {
+    double gx[4][3];
+#pragma unroll
+    for (int f = 0; f < 4; f++)
+#pragma unroll
+        for (int a = 0; a < 3; a++)
+            gx[f][a] = __dmul_rn(Mp[0], fma(Mp[1 + a], gc[f][0], fma(Mp[4 + a], gc[f][1], __dmul_rn(Mp[7 + a], gc[f][2]))));
+    double mu = ph.mu_ref;
+    if (ph.mu_law == 1) {
+        const double t = __dmul_rn(T, ph.iT_ref);
+        mu = __dmul_rn(__dmul_rn(__dmul_rn(ph.mu_ref, t), sqrt_nr(t)), div_nr(ph.T_ref + ph.S, __dadd_rn(T, ph.S)));
+    }
+    const double kap = __dmul_rn(mu, ph.cp_over_Pr);
+    const double dv = __dmul_rn(__dmul_rn(2.0 / 3.0, mu), __dadd_rn(__dadd_rn(gx[0][0], gx[1][1]), gx[2][2]));
+    const double m2 = __dmul_rn(2.0, mu);
+    tau[0] = __dsub_rn(__dmul_rn(m2, gx[0][0]), dv);                 // xx
+    tau[1] = __dsub_rn(__dmul_rn(m2, gx[1][1]), dv);                 // yy
+    tau[2] = __dsub_rn(__dmul_rn(m2, gx[2][2]), dv);                 // zz
+    tau[3] = __dmul_rn(mu, __dadd_rn(gx[0][1], gx[1][0]));           // xy
+    tau[4] = __dmul_rn(mu, __dadd_rn(gx[0][2], gx[2][0]));           // xz
+    tau[5] = __dmul_rn(mu, __dadd_rn(gx[1][2], gx[2][1]));           // yz
+    hb[0] = fma(u, tau[0], fma(v, tau[3], fma(w, tau[4], __dmul_rn(kap, gx[3][0]))));
+    hb[1] = fma(u, tau[3], fma(v, tau[1], fma(w, tau[5], __dmul_rn(kap, gx[3][1]))));
+    hb[2] = fma(u, tau[4], fma(v, tau[5], fma(w, tau[2], __dmul_rn(kap, gx[3][2]))));
+}
+// F^_v^d = m^d_b (tau_xb, tau_yb, tau_zb, hb_b), m^d = Mp[1+3d .. 3+3d]
+__device__ __forceinline__ void visc_proj(const double *md, const double tau[6], const double hb[3],
+                                          double out[4]) {
+    out[0] = fma(md[0], tau[0], fma(md[1], tau[3], __dmul_rn(md[2], tau[4])));
+    out[1] = fma(md[0], tau[3], fma(md[1], tau[1], __dmul_rn(md[2], tau[5])));
+    out[2] = fma(md[0], tau[4], fma(md[1], tau[5], __dmul_rn(md[2], tau[2])));
+    out[3] = fma(md[0], hb[0], fma(md[1], hb[1], __dmul_rn(md[2], hb[2])));
+}
+__device__ __forceinline__ double d4v(double fm2, double fm1, double fp1, double fp2) {
+    return __dmul_rn(fma(8.0, __dsub_rn(fp1, fm1), -__dsub_rn(fp2, fm2)), 1.0 / 12.0);
+}
+
+__global__ void __launch_bounds__(DNT, CROCCO_VDIV_MINB) k_visc_div(const double *__restrict__ U,
+                                                                   const double *__restrict__ M,
+                                                                   double *__restrict__ R, int64_t rcs,
+                                                                   Lay L, Phys ph) {
+    extern __shared__ double dsm[];
+    double *ring = dsm;                   // u v w T, tile + 2 halo: [plane mod 5][4][DNB]
+    double *arms = ring + 5 * 4 * DNB;    // u v w T of the 4-point arms, current plane: [4][DNA]
+    double *fz = arms + 4 * DNA;          // F^zeta of the own columns: [plane mod 5][4][DNT]
+    double *fx = fz + 5 * 4 * DNT;        // F^xi  [4][DNX], index (a+2) + DXW b
+    double *fy = fx + 4 * DNX;            // F^eta [4][DNY], index a + DTX (b+2)
+    constexpr int NSB = (DNB + DNT - 1) / DNT;  // ring points per thread and plane
+    static_assert(DNA <= DNT, "one arm point per thread");
+    const int tid = threadIdx.x;
+    const int tilesx = (L.n0 + DTX - 1) / DTX, tilesy = (L.n1 + DTY - 1) / DTY;
+    int bb = blockIdx.x;
+    const int bx = bb % tilesx;
+    bb /= tilesx;
+    const int by = bb % tilesy;
+    const int bz = bb / tilesy;
+    const int i0 = bx * DTX, j0 = by * DTY, k0 = bz * DK, k1 = min(k0 + DK, L.n2);
+    const double iR = 1.0 / ph.R;
+    auto ci = [&](int a) { return min(max(i0 + a, -G), L.n0 + G - 1); };
+    auto cj = [&](int b) { return min(max(j0 + b, -G), L.n1 + G - 1); };
+    auto slot = [](int k) { return ((k + 10) % 5); };
+    auto rb = [](int a, int b) { return (a + 2) + DBW * (b + 2); };
+    // arm point (a, b) outside the ring rectangle -> index in `arms`
+    auto ai = [](int a, int b) {
+        return (b >= 0 && b < DTY) ? (a < 0 ? a + 4 : a - DTX) + 4 * b
+                                   : 4 * DTY + a + DTX * (b < 0 ? b + 4 : b - DTY);
+    };
+    // this thread's arm points (tid < DNA): the 4-point arm point it stages and the
+    // 2-point arm point whose gradient / flux it evaluates; xarm: along i (F^xi) else j (F^eta)
+    const bool xarm = tid < 4 * DTY;
+    int sa, sb, ga, gb;
+    if (xarm) {
+        const int c = tid & 3;
+        sa = c < 2 ? c - 4 : DTX + c;
+        ga = c < 2 ? c - 2 : DTX + c - 2;
+        sb = gb = tid >> 2;
+    } else {
+        const int u = tid - 4 * DTY, r = u / DTX;
+        sa = ga = u % DTX;
+        sb = r < 2 ? r - 4 : DTY + r;
+        gb = r < 2 ? r - 2 : DTY + r - 2;
+    }
+    const bool arm = tid < DNA;
+    const int oa = tid % DTX, ob = tid / DTX;  // own column
+    const bool own = i0 + oa < L.n0 && j0 + ob < L.n1;
+
+    auto ld5 = [&](int a, int b, int k, double o[5]) {
+        const int64_t p = at(L, ci(a), cj(b), k);
+#pragma unroll
+        for (int c = 0; c < 5; c++) o[c] = U[c * L.cs + p];
+    };
+    auto ld10 = [&](int a, int b, int k, double o[10]) {
+        const int64_t p = at(L, ci(a), cj(b), k);
+#pragma unroll
+        for (int c = 0; c < 10; c++) o[c] = M[c * L.cs + p];
+    };
+    // u, v, w, T of a conserved state into d[0], d[st], d[2 st], d[3 st]
+    auto put = [&](const double u5[5], double *d, int st) {
+        const double ir = rcp_nr(u5[0]);
+        const double u = __dmul_rn(u5[1], ir), v = __dmul_rn(u5[2], ir), w = __dmul_rn(u5[3], ir);
+        const double pr = __dmul_rn(ph.gm1, fma(-0.5, fma(u5[1], u, fma(u5[2], v, __dmul_rn(u5[3], w))), u5[4]));
+        d[0] = u;
+        d[st] = v;
+        d[2 * st] = w;
+        d[3 * st] = __dmul_rn(__dmul_rn(pr, ir), iR);
+    };
+    // gradient of u, v, w, T at (a, b) of plane k -> tau, hb.  ARM: the point is a
+    // 2-point arm point whose i- or j-stencil reaches into the 4-point arms.
+    auto grad = [&](auto armc, int a, int b, int k, const double Mp[10], double tau[6], double hb[3]) {
+        constexpr bool ARM = std::decay_t<decltype(armc)>::value;
+        const double *pl = ring + slot(k) * 4 * DNB;
+        const int ix = rb(a, b);
+        const double *cm1 = ring + slot(k - 1) * 4 * DNB + ix, *cp1 = ring + slot(k + 1) * 4 * DNB + ix;
+        const double *cm2 = ring + slot(k - 2) * 4 * DNB + ix, *cp2 = ring + slot(k + 2) * 4 * DNB + ix;
+        auto cur = [&](int f, int a2, int b2) -> double {
+            if (ARM && (a2 < -2 || a2 > DTX + 1 || b2 < -2 || b2 > DTY + 1)) return arms[f * DNA + ai(a2, b2)];
+            return pl[f * DNB + rb(a2, b2)];
+        };
+        double gc[4][3];
+#pragma unroll
+        for (int f = 0; f < 4; f++) {
+            gc[f][0] = d4v(cur(f, a - 2, b), cur(f, a - 1, b), cur(f, a + 1, b), cur(f, a + 2, b));
+            gc[f][1] = d4v(cur(f, a, b - 2), cur(f, a, b - 1), cur(f, a, b + 1), cur(f, a, b + 2));
+            gc[f][2] = d4v(cm2[f * DNB], cm1[f * DNB], cp1[f * DNB], cp2[f * DNB]);
+        }
+        const double *c0 = pl + ix;
+        visc_point(gc, Mp, c0[0], c0[DNB], c0[2 * DNB], c0[3 * DNB], ph, tau, hb);
+    };
+
+    double xq[3][4];  // D4_xi F^xi + D4_eta F^eta of the own column, planes g-2 .. g
+#pragma unroll
+    for (int o = 0; o < 3; o++)
+#pragma unroll
+        for (int q = 0; q < 4; q++) xq[o][q] = 0.0;
+
+    // prologue: ring planes k0-4 .. k0-1
+    for (int t = tid; t < 4 * DNB; t += DNT) {
+        const int k = k0 - 4 + t / DNB, r = t % DNB;
+        double u5[5];
+        ld5(r % DBW - 2, r / DBW - 2, k, u5);
+        put(u5, ring + slot(k) * 4 * DNB + r, DNB);
+    }
+    // global operands of step g, loaded one step ahead: ring points of plane g+2, the
+    // arm point of plane g, the metrics of the own and the arm gradient point
+    double nU[NSB + 1][5], nM[2][10];
+    auto prefetch = [&](int g) {
+        const bool xy = g >= k0 && g < k1;
+#pragma unroll
+        for (int s2 = 0; s2 < NSB; s2++) {
+            const int t = tid + s2 * DNT;
+            if (t < DNB) ld5(t % DBW - 2, t / DBW - 2, g + 2, nU[s2]);
+        }
+        if (xy && arm) ld5(sa, sb, g, nU[NSB]);
+        ld10(oa, ob, g, nM[0]);
+        if (xy && arm) ld10(ga, gb, g, nM[1]);
+    };
+    prefetch(k0 - 2);
+    for (int g = k0 - 2; g <= k1 + 1; g++) {
+        const bool xy = g >= k0 && g < k1;  // F^xi / F^eta of plane g needed
+        double cU[NSB + 1][5], cM[2][10];
+#pragma unroll
+        for (int s2 = 0; s2 <= NSB; s2++)
+#pragma unroll
+            for (int c = 0; c < 5; c++) cU[s2][c] = nU[s2][c];
+#pragma unroll
+        for (int s2 = 0; s2 < 2; s2++)
+#pragma unroll
+            for (int c = 0; c < 10; c++) cM[s2][c] = nM[s2][c];
+        if (g < k1 + 1) prefetch(g + 1);
+        // phase 1
+#pragma unroll
+        for (int s2 = 0; s2 < NSB; s2++) {
+            const int t = tid + s2 * DNT;
+            if (t < DNB) put(cU[s2], ring + slot(g + 2) * 4 * DNB + t, DNB);
+        }
+        if (xy && arm) put(cU[NSB], arms + tid, DNA);
+        __syncthreads();
+        // phase 2: own point
+        {
+            double tau[6], hb[3], f[4];
+            grad(std::false_type{}, oa, ob, g, cM[0], tau, hb);
+            visc_proj(cM[0] + 7, tau, hb, f);
+#pragma unroll
+            for (int q = 0; q < 4; q++) fz[(slot(g) * 4 + q) * DNT + tid] = f[q];
+            if (xy) {
+                visc_proj(cM[0] + 1, tau, hb, f);
+#pragma unroll
+                for (int q = 0; q < 4; q++) fx[q * DNX + (oa + 2) + DXW * ob] = f[q];
+                visc_proj(cM[0] + 4, tau, hb, f);
+#pragma unroll
+                for (int q = 0; q < 4; q++) fy[q * DNY + oa + DTX * (ob + 2)] = f[q];
+            }
+        }
+        // phase 2: arm point (2-point halo of F^xi along i, of F^eta along j)
+        if (xy && arm) {
+            double tau[6], hb[3], f[4];
+            grad(std::true_type{}, ga, gb, g, cM[1], tau, hb);
+            visc_proj(xarm ? cM[1] + 1 : cM[1] + 4, tau, hb, f);
+            if (xarm) {
+#pragma unroll
+                for (int q = 0; q < 4; q++) fx[q * DNX + (ga + 2) + DXW * gb] = f[q];
+            } else {
+#pragma unroll
+                for (int q = 0; q < 4; q++) fy[q * DNY + ga + DTX * (gb + 2)] = f[q];
+            }
+        }
+        __syncthreads();
+        // phase 3
+#pragma unroll
+        for (int o = 0; o < 2; o++)
+#pragma unroll
+            for (int q = 0; q < 4; q++) xq[o][q] = xq[o + 1][q];
+        if (xy) {
+#pragma unroll
+            for (int q = 0; q < 4; q++) {
+                const double *x = fx + q * DNX + (oa + 2) + DXW * ob;
+                const double *y = fy + q * DNY + oa + DTX * (ob + 2);
+                xq[2][q] = __dadd_rn(d4v(x[-2], x[-1], x[1], x[2]), d4v(y[-2 * DTX], y[-DTX], y[DTX], y[2 * DTX]));
+            }
+        }
+        const int k = g - 2;
+        if (k >= k0 && own) {
+            const int64_t r = (int64_t)(i0 + oa) + (int64_t)L.n0 * ((j0 + ob) + (int64_t)L.n1 * k);
+#pragma unroll
+            for (int q = 0; q < 4; q++) {
+                const double *z = fz + q * DNT + tid;
+                const double zd = d4v(z[slot(k - 2) * 4 * DNT], z[slot(k - 1) * 4 * DNT], z[slot(k + 1) * 4 * DNT],
+                                      z[slot(k + 2) * 4 * DNT]);
+                R[(1 + q) * rcs + r] = __dadd_rn(xq[0][q], zd);
+            }
+        }
     }
 }
 

@@ -39,7 +39,8 @@ struct SweepArgs {
     double *R;          // accumulator, compact interior layout i + n0 (j + n1 k)
     int64_t rcs;        // its component stride
     int inv, visc;      // terms evaluated in this direction
-    int mode;           // 0 write R, 1 add to R, 2 rhs = J R, 3 RK update
+    int mode;           // 0 write R, 1 add to R, 2 rhs = J R, 3 RK update,
+                        // 4 add to the viscous divergence in R comps 1..4 (k_visc_div), write comp 0
     int seg;            // march segment (D = 1, 2)
     double *rhs;        // mode 2 (padded layout)
     const double *Uin;  // mode 3 (padded layout)
@@ -365,7 +366,8 @@ __global__ void __launch_bounds__(SWEEP_THREADS, CROCCO_SWEEP_MINB) k_sweep_s(co
         const bool own = act && e >= e0;      // this lane finishes point e
         if (own && a.mode != 0) {             // group A: accumulate / update operands
 #pragma unroll
-            for (int c = 0; c < 5; c++) cp_async8(cb + 32 * c, a.R + c * a.rcs + rr);
+            for (int c = 0; c < 5; c++)
+                if (c > 0 || a.mode != 4) cp_async8(cb + 32 * c, a.R + c * a.rcs + rr);
             if (a.mode >= 2) {
                 cp_async8(cb + 32 * 5, a.in.M + pp);
                 if (a.mode == 3) {
@@ -409,8 +411,8 @@ __global__ void __launch_bounds__(SWEEP_THREADS, CROCCO_SWEEP_MINB) k_sweep_s(co
             } else {
                 double Rt[5];
 #pragma unroll
-                for (int c = 0; c < 5; c++) Rt[c] = cb[32 * c] + dF[c];
-                if (a.mode == 1) {
+                for (int c = 0; c < 5; c++) Rt[c] = (c == 0 && a.mode == 4) ? dF[0] : cb[32 * c] + dF[c];
+                if (a.mode == 1 || a.mode == 4) {
 #pragma unroll
                     for (int c = 0; c < 5; c++) a.R[c * a.rcs + rr] = Rt[c];
                 } else if (a.mode == 2) {
