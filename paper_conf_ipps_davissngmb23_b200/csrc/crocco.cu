@@ -43,6 +43,7 @@ struct LocalBlock {
     double *racc = nullptr;  // RHS accumulator R (5 comps, compact interior)
     int64_t rcs = 0;
     double *fv = nullptr;
+    double *rv = nullptr;    // viscous D4_zeta term (CROCCO_ZDIV_SWEEP != 0)
 };
 
 enum { K_PRIMS = 0, K_FLUX_X, K_FLUX_Y, K_FLUX_Z, K_VISC, K_UPDATE, K_FILL, K_METRICS, K_CFL,
@@ -306,6 +307,9 @@ static void build_plan(const crocco_grid_desc *d, const int nb[3], const int bn[
     }
 }
 
+#ifndef CROCCO_ZDIV_SWEEP
+#define CROCCO_ZDIV_SWEEP 0  // 0: k_visc_tiled writes R, the xi sweep adds (measured equal to 1 / 2, no extra buffer)
+#endif
 #ifndef CROCCO_SWEEP_SMEM
 #define CROCCO_SWEEP_SMEM 1  // shared-memory staged sweeps (k_sweep_s); 0: global-load sweeps
 #endif
@@ -422,6 +426,7 @@ static void free_ctx(crocco_ctx c) {
         cudaFree(b.prim);
         cudaFree(b.racc);
         cudaFree(b.fv);
+        cudaFree(b.rv);
     }
     cudaFree(c->send_stage);
     cudaFree(c->dmax);
@@ -492,7 +497,10 @@ crocco_status crocco_init_grid(const crocco_grid_desc *desc, const crocco_phys *
         bool ok = CROCCO_SWEEP_SMEM || alloc(&b.prim, NPRIM * b.L.cs);
         b.rcs = rup((int64_t)b.g.n[0] * b.g.n[1] * b.g.n[2], 32);
         ok = ok && alloc(&b.racc, 5 * b.rcs);
-        ok = ok && ((CROCCO_SWEEP_SMEM && CROCCO_VISC_DIV) || alloc(&b.fv, 12 * b.V.cs));
+        ok = ok && (!(CROCCO_SWEEP_SMEM && !CROCCO_VISC_DIV && CROCCO_VISC_ZDIV && CROCCO_ZDIV_SWEEP) ||
+                    alloc(&b.rv, 5 * b.rcs));
+        ok = ok && ((CROCCO_SWEEP_SMEM && CROCCO_VISC_DIV) ||
+                    alloc(&b.fv, (CROCCO_SWEEP_SMEM && CROCCO_VISC_ZDIV ? 8 : 12) * b.V.cs));
         if (!ok) {
             cudaGetLastError();
             free_ctx(c);
@@ -834,15 +842,22 @@ static crocco_status rhs_block(crocco_ctx c, const LocalBlock &b, const double *
     if (!CROCCO_SWEEP_SMEM)  // the staged sweeps and the tiled viscous kernel compute their own primitives
         LAUNCH(c, K_PRIMS, k_prims<<<cdiv(np, 256), 256, 0, c->stream>>>(U, b.prim, b.L, ph));
     const bool vdiv = viscous && CROCCO_SWEEP_SMEM && CROCCO_VISC_DIV;  // fused viscous divergence -> R
+    // D4_zeta of the zeta point flux inside k_visc_tiled -> R (the zeta sweep carries no viscous term)
+    const bool zdiv = viscous && CROCCO_SWEEP_SMEM && !CROCCO_VISC_DIV && CROCCO_VISC_ZDIV;
+    // where the D4_zeta term is added: 0 -> k_visc_tiled writes R and the xi sweep adds to it;
+    // 1 / 2 -> separate buffer added by the eta / zeta sweep
+    const int zsw = CROCCO_ZDIV_SWEEP;
+    double *rvz = (zdiv && zsw != 0) ? b.rv : b.racc;
     if (vdiv) {
         const unsigned nt = (unsigned)(((b.g.n[0] + DTX - 1) / DTX) * ((b.g.n[1] + DTY - 1) / DTY) *
                                        ((b.g.n[2] + DK - 1) / DK));
         LAUNCH(c, K_VISC, k_visc_div<<<nt, DNT, VDIV_SMEM, c->stream>>>(U, M, b.racc, b.rcs, b.L, ph));
     } else if (viscous) {
 #if CROCCO_SWEEP_SMEM
-        const unsigned nt = (unsigned)(((b.V.b0 + VTX - 1) / VTX) * ((b.V.b1 + VTY - 1) / VTY) *
-                                       ((b.V.b2 + VK - 1) / VK));
-        LAUNCH(c, K_VISC, k_visc_tiled<<<nt, VTX * VTY, VISC_SMEM, c->stream>>>(U, M, b.fv, b.L, b.V, ph));
+        const int nz = zdiv ? b.g.n[2] : b.V.b2;
+        const unsigned nt = (unsigned)(((b.V.b0 + VTX - 1) / VTX) * ((b.V.b1 + VTY - 1) / VTY) * ((nz + VK - 1) / VK));
+        LAUNCH(c, K_VISC, k_visc_tiled<<<nt, VTX * VTY, VISC_SMEM, c->stream>>>(U, M, b.fv, b.L, b.V, ph,
+                                                                                 rvz, b.rcs));
 #else
         const int64_t nv = (int64_t)b.V.b0 * b.V.b1 * b.V.b2;
         LAUNCH(c, K_VISC, k_visc<<<cdiv(nv, 256), 256, 0, c->stream>>>(b.prim, M, b.fv, b.L, b.V, ph));
@@ -861,8 +876,9 @@ static crocco_status rhs_block(crocco_ctx c, const LocalBlock &b, const double *
         a.R = b.racc;
         a.rcs = b.rcs;
         a.inv = inviscid && (ph.dir_mask >> d & 1);
-        a.visc = viscous && !vdiv;
-        a.mode = d == 0 ? (vdiv ? 4 : 0) : (d == 1 ? 1 : final_mode);
+        a.visc = viscous && !vdiv && !(zdiv && d == 2);
+        a.mode = d == 0 ? ((vdiv || (zdiv && zsw == 0)) ? 4 : 0) : (d == 1 ? 1 : final_mode);
+        a.RV = (zdiv && zsw != 0 && d == zsw) ? b.rv : nullptr;
         a.rhs = rhs;
         a.Uin = Uin;
         a.Uout = Uout;

@@ -122,10 +122,16 @@ __global__ void __launch_bounds__(256) k_visc(const double *__restrict__ Pm,
 #ifndef CROCCO_VISC_PREFETCH
 #define CROCCO_VISC_PREFETCH 1  // load the next plane's U / metrics one step ahead (registers)
 #endif
+#ifndef CROCCO_VISC_ZDIV
+#define CROCCO_VISC_ZDIV 1  // 1: D4_zeta of F^_v^zeta folded into k_visc_tiled (own-column queue) -> R
+#endif
 #ifndef CROCCO_VISC_TX
 #define CROCCO_VISC_TX 16  // 16 x 8 tiles: two 4-warp CTAs per SM (measured 3 % faster than 32 x 8)
 #endif
-constexpr int VTX = CROCCO_VISC_TX, VTY = 8, VK = 32;  // tile and slab
+#ifndef CROCCO_VISC_VK
+#define CROCCO_VISC_VK (CROCCO_VISC_ZDIV ? 64 : 32)  // slab depth (ZDIV recomputes 4 planes per slab)
+#endif
+constexpr int VTX = CROCCO_VISC_TX, VTY = 8, VK = CROCCO_VISC_VK;  // tile and slab
 constexpr int VHX = VTX + 4, VHY = VTY + 4;          // with halo
 constexpr int VPL = VHX * VHY;                       // points per staged plane
 constexpr int VHALO = VPL - VTX * VTY;               // halo points per plane
@@ -146,7 +152,7 @@ __device__ __forceinline__ void prim4(const double *__restrict__ U, int64_t cs, 
 __global__ void __launch_bounds__(VTX * VTY, CROCCO_VISC_MINB) k_visc_tiled(const double *__restrict__ U,
                                                           const double *__restrict__ M,
                                                           double *__restrict__ FV, Lay L, VLay V,
-                                                          Phys ph) {
+                                                          Phys ph, double *__restrict__ R, int64_t rcs) {
     extern __shared__ double vsm[];  // [buffer 2][value 4][VPL]
     const int tid = threadIdx.x;
     const int tx = tid % VTX, ty = tid / VTX;
@@ -157,7 +163,18 @@ __global__ void __launch_bounds__(VTX * VTY, CROCCO_VISC_MINB) k_visc_tiled(cons
     const int by = b % tilesy;
     const int bz = b / tilesy;
     const int i0 = bx * VTX - 2, j0 = by * VTY - 2;      // first output point of the tile
+#if CROCCO_VISC_ZDIV
+    // slab of interior output planes [z0, z1); gradients / point fluxes on planes z0-2 .. z1+1
+    const int z0 = bz * VK, z1 = min(z0 + VK, L.n2);
+    const int k0 = z0 - 2, k1 = z1 + 2;
+    double zq[5][4];  // F^zeta of the own column, planes k-4 .. k
+#pragma unroll
+    for (int o = 0; o < 5; o++)
+#pragma unroll
+        for (int q = 0; q < 4; q++) zq[o][q] = 0.0;
+#else
     const int k0 = bz * VK - 2, k1 = min(k0 + VK, V.b2 - 2);
+#endif
     const double iR = 1.0 / ph.R;
     // own column (clamped into the padded box for the idle threads of edge tiles)
     const int i = i0 + tx, j = j0 + ty;
@@ -319,6 +336,33 @@ __global__ void __launch_bounds__(VTX * VTY, CROCCO_VISC_MINB) k_visc_tiled(cons
             for (int bb = 0; bb < 3; bb++)
                 hb[bb] = fma(vel[0], tau[0][bb], fma(vel[1], tau[1][bb], fma(vel[2], tau[2][bb], kap * gx[3][bb])));
             const int64_t o = vat(V, i, j, k);
+#if CROCCO_VISC_ZDIV
+            // F^xi, F^eta of the interior planes to HBM (the xi / eta sweeps difference them);
+            // F^zeta stays in the own column's queue and is differenced here (D4_zeta)
+            if (k >= z0 && k < z1) {
+#pragma unroll
+                for (int d = 0; d < 2; d++) {
+#pragma unroll
+                    for (int a = 0; a < 3; a++)
+                        FV[(4 * d + a) * V.cs + o] = fma(m[d][0], tau[a][0], fma(m[d][1], tau[a][1], m[d][2] * tau[a][2]));
+                    FV[(4 * d + 3) * V.cs + o] = fma(m[d][0], hb[0], fma(m[d][1], hb[1], m[d][2] * hb[2]));
+                }
+            }
+#pragma unroll
+            for (int oq = 0; oq < 4; oq++)
+#pragma unroll
+                for (int q = 0; q < 4; q++) zq[oq][q] = zq[oq + 1][q];
+#pragma unroll
+            for (int a = 0; a < 3; a++) zq[4][a] = fma(m[2][0], tau[a][0], fma(m[2][1], tau[a][1], m[2][2] * tau[a][2]));
+            zq[4][3] = fma(m[2][0], hb[0], fma(m[2][1], hb[1], m[2][2] * hb[2]));
+            if (k - 2 >= z0 && i >= 0 && i < L.n0 && j >= 0 && j < L.n1) {
+                const int64_t r = (int64_t)i + (int64_t)L.n0 * (j + (int64_t)L.n1 * (k - 2));
+#pragma unroll
+                for (int q = 0; q < 4; q++)
+                    R[(1 + q) * rcs + r] =
+                        fma(8.0, zq[3][q] - zq[1][q], -(zq[4][q] - zq[0][q])) * (1.0 / 12.0);
+            }
+#else
 #pragma unroll
             for (int d = 0; d < 3; d++) {
 #pragma unroll
@@ -326,6 +370,7 @@ __global__ void __launch_bounds__(VTX * VTY, CROCCO_VISC_MINB) k_visc_tiled(cons
                     FV[(4 * d + a) * V.cs + o] = fma(m[d][0], tau[a][0], fma(m[d][1], tau[a][1], m[d][2] * tau[a][2]));
                 FV[(4 * d + 3) * V.cs + o] = fma(m[d][0], hb[0], fma(m[d][1], hb[1], m[d][2] * hb[2]));
             }
+#endif
         }
 #if CROCCO_VISC_PREFETCH
 #pragma unroll

@@ -42,6 +42,7 @@ struct SweepArgs {
     int mode;           // 0 write R, 1 add to R, 2 rhs = J R, 3 RK update,
                         // 4 add to the viscous divergence in R comps 1..4 (k_visc_div), write comp 0
     int seg;            // march segment (D = 1, 2)
+    const double *RV;   // viscous D4_zeta term (comps 1..4, R layout) added by this sweep, or null
     double *rhs;        // mode 2 (padded layout)
     const double *Uin;  // mode 3 (padded layout)
     double *Uout, *dU;
@@ -192,7 +193,7 @@ struct RingGeom {
     static constexpr int C = 32 / WS;              // columns (lines) per warp
     static constexpr int LA = (D == 0) ? 1 : 2;    // chunks ahead needed by a step
     static constexpr int NR = (D == 0) ? 32 : 16;  // ring points (>= (LA + 2) * WS, power of 2)
-    static constexpr int NCB = 16;                 // prefetched accumulate/update operands per lane
+    static constexpr int NCB = 20;                 // prefetched accumulate/update operands per lane
     static constexpr int PER_WARP = SV_N * NR * C + NCB * 32;  // doubles
 };
 
@@ -368,6 +369,10 @@ __global__ void __launch_bounds__(SWEEP_THREADS, CROCCO_SWEEP_MINB) k_sweep_s(co
 #pragma unroll
             for (int c = 0; c < 5; c++)
                 if (c > 0 || a.mode != 4) cp_async8(cb + 32 * c, a.R + c * a.rcs + rr);
+            if (a.RV) {
+#pragma unroll
+                for (int c = 1; c < 5; c++) cp_async8(cb + 32 * (15 + c), a.RV + c * a.rcs + rr);
+            }
             if (a.mode >= 2) {
                 cp_async8(cb + 32 * 5, a.in.M + pp);
                 if (a.mode == 3) {
@@ -412,6 +417,10 @@ __global__ void __launch_bounds__(SWEEP_THREADS, CROCCO_SWEEP_MINB) k_sweep_s(co
                 double Rt[5];
 #pragma unroll
                 for (int c = 0; c < 5; c++) Rt[c] = (c == 0 && a.mode == 4) ? dF[0] : cb[32 * c] + dF[c];
+                if (a.RV) {
+#pragma unroll
+                    for (int c = 1; c < 5; c++) Rt[c] += cb[32 * (15 + c)];
+                }
                 if (a.mode == 1 || a.mode == 4) {
 #pragma unroll
                     for (int c = 0; c < 5; c++) a.R[c * a.rcs + rr] = Rt[c];
