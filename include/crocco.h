@@ -186,7 +186,10 @@ crocco_status crocco_rhs(crocco_ctx ctx, double *const *U, double *const *metric
    fill(U_in) (in place on U_in's ghosts) + RHS + dU <- A_s dU + dt rhs,
    U_out = U_in + B_s dU on interior points; A = (0, -5/9, -153/128),
    B = (1/3, 15/16, 8/15).  dU is not read at stage 0.  U_out != U_in.
-   Collective. */
+   Collective.  With viscous terms the ghost fill (local copies, physical BCs and
+   the NCCL send/recv of remote faces) runs on an internal comm stream while the
+   viscous tiles that read no ghost point run on `stream`; the rest of the stage
+   waits for the fill (SURVEY 8(e) overlap; see crocco_set_overlap). */
 crocco_status crocco_rk_stage(crocco_ctx ctx, int32_t stage, double dt, double *const *U_in,
                               double *const *U_out, double *const *dU,
                               double *const *metrics);
@@ -216,6 +219,14 @@ crocco_status crocco_compute_dt(crocco_ctx ctx, double *const *U, double *const 
 crocco_status crocco_sync(crocco_ctx ctx);
 const char *crocco_last_error(crocco_ctx ctx);
 crocco_status crocco_finalize(crocco_ctx ctx);
+
+/* Overlap of the ghost exchange with interior compute inside crocco_rk_stage /
+   crocco_rk3_step: 1 on, 0 off, -1 auto (default: on when nranks > 1, i.e. when
+   the fill has NCCL faces; a purely local fill is too short to hide and the split
+   viscous launch costs more than it saves -- measured on one B200).  Results are
+   bitwise identical either way: the fill writes only ghost points, the overlapped
+   tiles read only interior points.  CROCCO_ERR_ARG for other values. */
+crocco_status crocco_set_overlap(crocco_ctx ctx, int32_t enable);
 
 /* ---- instrumentation (bench / tests) ---------------------------------------- */
 

@@ -83,6 +83,7 @@ _SIGS = {
     "crocco_finalize": [C.c_void_p],
     "crocco_launch_count": [C.c_void_p, C.POINTER(C.c_int64), C.c_int32],
     "crocco_set_timing": [C.c_void_p, C.c_int32],
+    "crocco_set_overlap": [C.c_void_p, C.c_int32],
     "crocco_kernel_times": [C.c_void_p, C.c_int32, C.POINTER(C.c_int64), C.POINTER(C.c_double),
                             C.POINTER(C.c_int32)],
     "crocco_exchange_plan": [C.POINTER(GridDesc), C.c_int32, C.POINTER(Msg), C.c_int32,
@@ -263,6 +264,11 @@ def crocco_launch_count(ctx, reset=False) -> int:
     v = C.c_int64()
     _check(lib().crocco_launch_count(ctx, C.byref(v), int(reset)), ctx)
     return v.value
+
+
+def crocco_set_overlap(ctx, enable=True):
+    """1 / True on, 0 / False off, -1 auto (on when nranks > 1)."""
+    _check(lib().crocco_set_overlap(ctx, int(enable)), ctx)
 
 
 def crocco_set_timing(ctx, enable=True):

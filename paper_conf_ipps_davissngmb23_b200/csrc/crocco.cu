@@ -88,6 +88,10 @@ struct crocco_ctx_s {
     };
     std::vector<StepGraph> graphs;
     cudaStream_t cap_stream = nullptr;
+    // overlapped stage: ghost fill / exchange on comm_stream beside the interior viscous tiles
+    int overlap = -1;  // -1 auto (on when the fill has remote faces, nranks > 1), 0 off, 1 on
+    cudaStream_t comm_stream = nullptr;
+    cudaEvent_t ev_fork = nullptr, ev_join = nullptr;
     double time = 0.0;  // start of the current step (time-dependent SPLIT faces)
     int64_t stage_elems = 0;
     // timing
@@ -438,6 +442,9 @@ static void free_ctx(crocco_ctx c) {
     for (auto e : c->pool) cudaEventDestroy(e);
     for (auto &g : c->graphs) cudaGraphExecDestroy(g.exec);
     if (c->cap_stream) cudaStreamDestroy(c->cap_stream);
+    if (c->comm_stream) cudaStreamDestroy(c->comm_stream);
+    if (c->ev_fork) cudaEventDestroy(c->ev_fork);
+    if (c->ev_join) cudaEventDestroy(c->ev_join);
     if (c->comm) ncclCommDestroy(c->comm);
     delete c;
 }
@@ -832,9 +839,30 @@ static const double RK_B[3] = {1.0 / 3.0, 15.0 / 16.0, 8.0 / 15.0};
 // One RHS evaluation of a block (Alg. 2 l.5-9): primitives, viscous point
 // fluxes, then the xi / eta / zeta sweeps; the zeta sweep finishes every point
 // (mode 2: rhs = J R, mode 3: Williamson update).
+// ghost-free interior tiles of the viscous kernel (k_visc_tiled sel 1) of one block;
+// returns false if the block has none or the configuration has no such split
+static bool visc_overlap_possible(crocco_ctx c) {
+    const bool viscous = (c->ph.terms & CROCCO_TERM_VISCOUS) != 0;
+    if (!(viscous && CROCCO_SWEEP_SMEM && !CROCCO_VISC_DIV && CROCCO_VISC_ZDIV && CROCCO_ZDIV_SWEEP == 0))
+        return false;
+    for (const auto &b : c->loc) {
+        const VTiles t = visc_interior_tiles(b.L);
+        if (t.x1 > t.x0 && t.y1 > t.y0 && t.z1 > t.z0) return true;
+    }
+    return false;
+}
+static crocco_status visc_interior(crocco_ctx c, const LocalBlock &b, const double *U, const double *M) {
+    const VTiles t = visc_interior_tiles(b.L);
+    const int64_t nt = (int64_t)(t.x1 - t.x0) * (t.y1 - t.y0) * (t.z1 - t.z0);
+    if (nt == 0) return CROCCO_OK;
+    LAUNCH(c, K_VISC, k_visc_tiled<<<(unsigned)nt, VTX * VTY, VISC_SMEM, c->stream>>>(U, M, b.fv, b.L, b.V,
+                                                                                     c->ph, b.racc, b.rcs, 1));
+    return CROCCO_OK;
+}
+
 static crocco_status rhs_block(crocco_ctx c, const LocalBlock &b, const double *U, const double *M,
                                int final_mode, double *rhs, const double *Uin, double *Uout,
-                               double *dU, int stage, double dt) {
+                               double *dU, int stage, double dt, int visc_sel = 0) {
     const Phys &ph = c->ph;
     const bool inviscid = (ph.terms & CROCCO_TERM_INVISCID) != 0;
     const bool viscous = (ph.terms & CROCCO_TERM_VISCOUS) != 0;
@@ -854,10 +882,17 @@ static crocco_status rhs_block(crocco_ctx c, const LocalBlock &b, const double *
         LAUNCH(c, K_VISC, k_visc_div<<<nt, DNT, VDIV_SMEM, c->stream>>>(U, M, b.racc, b.rcs, b.L, ph));
     } else if (viscous) {
 #if CROCCO_SWEEP_SMEM
-        const int nz = zdiv ? b.g.n[2] : b.V.b2;
-        const unsigned nt = (unsigned)(((b.V.b0 + VTX - 1) / VTX) * ((b.V.b1 + VTY - 1) / VTY) * ((nz + VK - 1) / VK));
-        LAUNCH(c, K_VISC, k_visc_tiled<<<nt, VTX * VTY, VISC_SMEM, c->stream>>>(U, M, b.fv, b.L, b.V, ph,
-                                                                                 rvz, b.rcs));
+        if (visc_sel != 1) {  // sel 1 (interior tiles) was launched by visc_interior() beside the fill
+            const int nz = zdiv ? b.g.n[2] : b.V.b2;
+            int64_t nt = (int64_t)((b.V.b0 + VTX - 1) / VTX) * ((b.V.b1 + VTY - 1) / VTY) * ((nz + VK - 1) / VK);
+            if (visc_sel == 2) {
+                const VTiles t = visc_interior_tiles(b.L);
+                nt -= (int64_t)(t.x1 - t.x0) * (t.y1 - t.y0) * (t.z1 - t.z0);
+            }
+            if (nt > 0)
+                LAUNCH(c, K_VISC, k_visc_tiled<<<(unsigned)nt, VTX * VTY, VISC_SMEM, c->stream>>>(
+                                      U, M, b.fv, b.L, b.V, ph, rvz, b.rcs, visc_sel));
+        }
 #else
         const int64_t nv = (int64_t)b.V.b0 * b.V.b1 * b.V.b2;
         LAUNCH(c, K_VISC, k_visc<<<cdiv(nv, 256), 256, 0, c->stream>>>(b.prim, M, b.fv, b.L, b.V, ph));
@@ -939,10 +974,41 @@ crocco_status crocco_rk_stage(crocco_ctx c, int32_t stage, double dt, double *co
     for (size_t bi = 0; bi < c->loc.size(); bi++)
         if (Uin[bi] == Uout[bi] || dU[bi] == Uin[bi] || dU[bi] == Uout[bi])
             return fail(c, CROCCO_ERR_ARG, "U_in, U_out and dU must be distinct");
-    if ((st = fill_all(c, Uin, CROCCO_FIELD_STATE, M, c->time + RK_C[stage] * dt))) return st;
+    const double ts = c->time + RK_C[stage] * dt;
+    const bool ov = c->overlap < 0 ? c->desc.nranks > 1 : c->overlap != 0;
+    if (!(ov && visc_overlap_possible(c))) {
+        if ((st = fill_all(c, Uin, CROCCO_FIELD_STATE, M, ts))) return st;
+        for (size_t bi = 0; bi < c->loc.size(); bi++) {
+            if ((st = rhs_block(c, c->loc[bi], Uin[bi], M[bi], 3, nullptr, Uin[bi], Uout[bi], dU[bi], stage,
+                                dt)))
+                return st;
+        }
+        return CROCCO_OK;
+    }
+    // Overlapped stage: the ghost fill -- local copies, BCs and the NCCL
+    // exchange -- runs on the comm stream while the viscous tiles that read no ghost point
+    // run on the compute stream; the remaining tiles and the sweeps follow the fill.
+    // Disjoint memory: the fill writes only ghost points of U_in, the interior tiles read
+    // only interior points; the result is bitwise that of the serial stage.
+    if (!c->comm_stream) CK(c, cudaStreamCreateWithFlags(&c->comm_stream, cudaStreamNonBlocking));
+    if (!c->ev_fork) CK(c, cudaEventCreateWithFlags(&c->ev_fork, cudaEventDisableTiming));
+    if (!c->ev_join) CK(c, cudaEventCreateWithFlags(&c->ev_join, cudaEventDisableTiming));
+    CK(c, cudaEventRecord(c->ev_fork, c->stream));
+    CK(c, cudaStreamWaitEvent(c->comm_stream, c->ev_fork, 0));
+    {
+        cudaStream_t comp = c->stream;
+        c->stream = c->comm_stream;
+        st = fill_all(c, Uin, CROCCO_FIELD_STATE, M, ts);
+        c->stream = comp;
+        if (st) return st;
+    }
+    CK(c, cudaEventRecord(c->ev_join, c->comm_stream));
+    for (size_t bi = 0; bi < c->loc.size(); bi++)
+        if ((st = visc_interior(c, c->loc[bi], Uin[bi], M[bi]))) return st;
+    CK(c, cudaStreamWaitEvent(c->stream, c->ev_join, 0));
     for (size_t bi = 0; bi < c->loc.size(); bi++) {
-        if ((st = rhs_block(c, c->loc[bi], Uin[bi], M[bi], 3, nullptr, Uin[bi], Uout[bi], dU[bi], stage,
-                            dt)))
+        if ((st = rhs_block(c, c->loc[bi], Uin[bi], M[bi], 3, nullptr, Uin[bi], Uout[bi], dU[bi], stage, dt,
+                            2)))
             return st;
     }
     return CROCCO_OK;
@@ -1079,6 +1145,13 @@ crocco_status crocco_launch_count(crocco_ctx c, int64_t *count, int32_t reset) {
     if (!c) return fail(nullptr, CROCCO_ERR_ARG, "null ctx");
     if (count) *count = c->launches;
     if (reset) c->launches = 0;
+    return CROCCO_OK;
+}
+
+crocco_status crocco_set_overlap(crocco_ctx c, int32_t enable) {
+    LIVE(c);
+    if (enable < -1 || enable > 1) return fail(c, CROCCO_ERR_ARG, "overlap must be -1, 0 or 1");
+    c->overlap = enable;
     return CROCCO_OK;
 }
 

@@ -149,19 +149,82 @@ __device__ __forceinline__ void prim4(const double *__restrict__ U, int64_t cs, 
     out[3] = pr * ir * iR;
 }
 
+// Tiles of k_visc_tiled whose loads stay inside the interior [0, n) in every
+// direction (no ghost point read): with ZDIV they may run while the ghost
+// exchange is in flight (SURVEY 8(e) overlap).  Half-open ranges of tile indices.
+struct VTiles {
+    int x0, x1, y0, y1, z0, z1;
+};
+__host__ __device__ inline VTiles visc_interior_tiles(const Lay &L) {
+    VTiles t;
+    // x: loads i0-2 .. i0+VTX+1 with i0 = bx VTX - 2; y likewise; z: planes z0-4 .. z1+3
+    t.x0 = (4 + VTX - 1) / VTX;
+    t.x1 = (L.n0 - VTX) >= 0 ? (L.n0 - VTX) / VTX + 1 : 0;
+    t.y0 = (4 + VTY - 1) / VTY;
+    t.y1 = (L.n1 - VTY) >= 0 ? (L.n1 - VTY) / VTY + 1 : 0;
+    t.z0 = (4 + VK - 1) / VK;
+    t.z1 = (L.n2 - 4) / VK;
+    if (t.x1 < t.x0) t.x1 = t.x0;
+    if (t.y1 < t.y0) t.y1 = t.y0;
+    if (t.z1 < t.z0) t.z1 = t.z0;
+    return t;
+}
+
+// sel: 0 every tile, 1 the ghost-free interior tiles only, 2 every other tile
 __global__ void __launch_bounds__(VTX * VTY, CROCCO_VISC_MINB) k_visc_tiled(const double *__restrict__ U,
                                                           const double *__restrict__ M,
                                                           double *__restrict__ FV, Lay L, VLay V,
-                                                          Phys ph, double *__restrict__ R, int64_t rcs) {
+                                                          Phys ph, double *__restrict__ R, int64_t rcs,
+                                                          int sel) {
     extern __shared__ double vsm[];  // [buffer 2][value 4][VPL]
     const int tid = threadIdx.x;
     const int tx = tid % VTX, ty = tid / VTX;
     const int tilesx = (V.b0 + VTX - 1) / VTX, tilesy = (V.b1 + VTY - 1) / VTY;
     int b = blockIdx.x;
-    const int bx = b % tilesx;
-    b /= tilesx;
-    const int by = b % tilesy;
-    const int bz = b / tilesy;
+    int bx, by, bz;
+    const VTiles it = visc_interior_tiles(L);
+    if (sel == 1) {
+        const int nx = it.x1 - it.x0, ny = it.y1 - it.y0;
+        bx = it.x0 + b % nx;
+        b /= nx;
+        by = it.y0 + b % ny;
+        bz = it.z0 + b / ny;
+    } else if (sel == 2) {
+        // the complement of the interior box, enumerated compactly: whole tile planes of the
+        // slabs outside [z0, z1), then the xy ring around [x0, x1) x [y0, y1) of the others
+        const int nx = it.x1 - it.x0, ny = it.y1 - it.y0, nzi = it.z1 - it.z0;
+        const int plane = tilesx * tilesy;
+        const int tz = (L.n2 + VK - 1) / VK;
+        const int nzs = tz - nzi;
+        if (b < nzs * plane) {
+            const int sl = b / plane, r = b % plane;
+            bz = sl < it.z0 ? sl : sl + nzi;
+            bx = r % tilesx;
+            by = r / tilesx;
+        } else {
+            b -= nzs * plane;
+            const int ring = plane - nx * ny;
+            bz = it.z0 + b / ring;
+            int r = b % ring;
+            if (r < it.y0 * tilesx) {
+                by = r / tilesx;
+                bx = r % tilesx;
+            } else if ((r -= it.y0 * tilesx) < ny * (tilesx - nx)) {
+                by = it.y0 + r / (tilesx - nx);
+                const int c = r % (tilesx - nx);
+                bx = c < it.x0 ? c : c + nx;
+            } else {
+                r -= ny * (tilesx - nx);
+                by = it.y1 + r / tilesx;
+                bx = r % tilesx;
+            }
+        }
+    } else {
+        bx = b % tilesx;
+        b /= tilesx;
+        by = b % tilesy;
+        bz = b / tilesy;
+    }
     const int i0 = bx * VTX - 2, j0 = by * VTY - 2;      // first output point of the tile
 #if CROCCO_VISC_ZDIV
     // slab of interior output planes [z0, z1); gradients / point fluxes on planes z0-2 .. z1+1

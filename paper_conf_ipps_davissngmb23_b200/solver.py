@@ -131,6 +131,48 @@ class Solver:
                                self._ptrs(self.dU), self._ptrs(self.met), graph)
             self.U, self.V = self.V, self.U
 
+    def steps_from_host(self, h_in, h_out, dt):
+        """Independent RK3 steps streamed through pinned host memory: job n's padded state is
+        uploaded from h_in[n] (list over local blocks of flat pinned float64 tensors sized like
+        the state arrays), advanced one RK3 step and downloaded into h_out[n].  Uploads and
+        downloads run on their own copy streams, so job n's download and job n+1's upload
+        overlap the compute of the neighbouring jobs (two device state pairs alternate).
+        Plumbing only: the step itself is crocco_rk3_step."""
+        if not hasattr(self, "_pairs"):
+            self._pairs = [(self.U, self.V), ([self._alloc(L, 5) for L in self.layouts],
+                                              [self._alloc(L, 5) for L in self.layouts])]
+            self._h2d = torch.cuda.Stream(self.device)
+            self._d2h = torch.cuda.Stream(self.device)
+        comp = self.stream
+        e0 = torch.cuda.Event()
+        e0.record(comp)                                        # earlier work on the buffers
+        self._h2d.wait_event(e0)
+        self._d2h.wait_event(e0)
+        ev_c, ev_d = {}, {}
+        for n in range(len(h_in)):
+            X, Y = self._pairs[n % 2]
+            with torch.cuda.stream(self._h2d):
+                if n - 2 in ev_c:
+                    self._h2d.wait_event(ev_c[n - 2])          # X clobbered by job n-2's stages
+                for h, x in zip(h_in[n], X):
+                    x.copy_(h, non_blocking=True)
+                eh = torch.cuda.Event()
+                eh.record(self._h2d)
+            comp.wait_event(eh)
+            if n - 2 in ev_d:
+                comp.wait_event(ev_d[n - 2])                   # Y still being downloaded
+            cc.crocco_rk3_step(self.ctx, dt, self._ptrs(X), self._ptrs(Y), self._ptrs(self.dU),
+                               self._ptrs(self.met), True)
+            ev_c[n] = torch.cuda.Event()
+            ev_c[n].record(comp)
+            with torch.cuda.stream(self._d2h):
+                self._d2h.wait_event(ev_c[n])
+                for h, y in zip(h_out[n], Y):
+                    h.copy_(y, non_blocking=True)
+                ev_d[n] = torch.cuda.Event()
+                ev_d[n].record(self._d2h)
+        comp.wait_stream(self._d2h)
+
     def compute_dt(self, cfl):
         """ComputeDt (Alg. 1 l.9): CFL time step of the current state (synchronises)."""
         return cc.crocco_compute_dt(self.ctx, self._ptrs(self.U), self._ptrs(self.met), cfl)

@@ -393,6 +393,54 @@ def test_rk3_step_graph_equals_eager_bitwise():
     assert np.array_equal(outs[0], outs[1])
 
 
+@pytest.mark.parametrize("nb,n", [((1, 1, 1), (40, 40, 140)), ((2, 1, 2), (72, 36, 264))])
+def test_overlapped_stage_equals_serial_bitwise(nb, n):
+    """crocco_rk_stage with the ghost fill on the comm stream beside the ghost-free viscous
+    tiles equals the serial stage bit for bit; sizes with interior tiles."""
+    from paper_conf_ipps_davissngmb23_b200 import crocco as cc
+    pb = wavy_random(n, 37, dict(terms=3, mu_law=1, mu_ref=0.02, S=0.3))
+    outs = []
+    for ov in (False, True):
+        S = pb.solver(nb)
+        cc.crocco_set_overlap(S.ctx, ov)
+        S.step(1e-3, 2, graph=False)
+        S.step(1e-3, 1, graph=True)
+        S.sync()
+        outs.append(pb.gather(S, S.get(S.U)))
+        S.close()
+    assert np.array_equal(outs[0], outs[1])
+
+
+def test_steps_from_host_equals_resident_steps_bitwise():
+    """Solver.steps_from_host (bench e2e: independent jobs through pinned host memory, copies
+    overlapped with compute on two streams) gives each job exactly the resident RK3 step."""
+    import torch
+    n = (32, 16, 12)
+    pb = wavy_random(n, 31, dict(terms=3, mu_ref=0.02))
+    S = pb.solver((2, 1, 1))
+    jobs = []
+    for j in range(5):                           # 5 distinct inputs: state after j resident steps
+        jobs.append([u.detach().cpu().pin_memory() for u in S.U])
+        S.step(1e-3)
+    S.sync()
+    ref = []
+    for j in range(5):                           # resident reference: one step from each input
+        for u, h in zip(S.U, jobs[j]):
+            u.copy_(h)
+        S.step(1e-3)
+        S.sync()
+        ref.append([u.detach().cpu().clone() for u in S.U])
+    outs = [[torch.empty_like(h).pin_memory() for h in jobs[0]] for _ in range(5)]
+    S.steps_from_host(jobs, outs, 1e-3)
+    torch.cuda.synchronize()
+    for j in range(5):
+        for b in range(S.nloc):
+            v = S.view(outs[j][b], b, 5)[:, 4:-4, 4:-4, 4:-4]
+            r = S.view(ref[j][b], b, 5)[:, 4:-4, 4:-4, 4:-4]
+            assert torch.equal(v, r), (j, b)
+    S.close()
+
+
 # ------------------------------------------------------------------ ComputeDt (NEXT-1)
 
 @pytest.mark.parametrize("nb", [(1, 1, 1), (2, 3, 2)])
