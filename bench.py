@@ -383,7 +383,7 @@ def run_crocco(args, rank, world, local_rank):
                 "peak_source": "derived: 148 SM x 64 FP64 FMA/clk x 2 x 1.965 GHz (DESIGN.md sec. 6)",
                 "flops_per_unit": FLUX_FLOPS_PER_IFACE, "unit_of_work": "interface flux",
                 "units_per_launch": ifaces, "avg_launch_ms": avg_ms,
-                "traffic": _profiled_traffic(f"k_sweep_s<{d}, 1>"),
+                "traffic": _profiled_traffic(f"k_sweep_s<{d},"),
                 "traffic_source": "profiles/ncu_summary.json (ncu --set full, dram__bytes_read+write per launch)"}
     peaks = measured_peaks()
     hbm = peaks.get("hbm_gbs", 6650.0)
@@ -423,7 +423,11 @@ def _profiled_traffic(kname):
     p = os.path.join(ROOT, "profiles", "ncu_summary.json")
     try:
         with open(p) as f:
-            return json.load(f).get("kernels", {}).get(kname, {}).get("dram_bytes_per_launch")
+            ks = json.load(f).get("kernels", {})
+        for k, v in ks.items():  # kname: full kernel name or a prefix of it
+            if k.startswith(kname) and "dram_bytes_per_launch" in v:
+                return v["dram_bytes_per_launch"]
+        return None
     except Exception:
         return None
 
