@@ -24,6 +24,9 @@ namespace crocco {
 #ifndef CROCCO_FIELD_ROLLED
 #define CROCCO_FIELD_ROLLED 0  // 1: keep the characteristic-field loop rolled (fewer live registers)
 #endif
+#ifndef CROCCO_PL_SMEM
+#define CROCCO_PL_SMEM 0  // 1: stencil pressures re-read from the ring per field (fewer live registers)
+#endif
 #ifndef CROCCO_DEFER_DIV
 #define CROCCO_DEFER_DIV 1  // 1: the five WENO-pair divisions after the field loop (independent chains)
 #endif
@@ -142,7 +145,9 @@ __device__ __forceinline__ void total_flux(const Acc &A, bool inv, bool visc, co
             const double t = fma(nx, A.P(l, PU), fma(ny, A.P(l, PV), nz * A.P(l, PW)));
             const double cl = A.P(l, PC);
             th[l] = t;
+#if !CROCCO_PL_SMEM
             pl[l] = A.P(l, PP);
+#endif
             lam0 = maxnn(lam0, fabs(t));
             lam3 = maxnn(lam3, fabs(t + cl));
             lam4 = maxnn(lam4, fabs(t - cl));
@@ -220,7 +225,11 @@ __device__ __forceinline__ void total_flux(const Acc &A, bool inv, bool visc, co
             for (int l = 0; l < 6; l++) {
                 const double w =
                     fma(L0, UL(l, 0), fma(L1, UL(l, 1), fma(L2, UL(l, 2), fma(L3, UL(l, 3), L4 * UL(l, 4)))));
+#if CROCCO_PL_SMEM
+                const double g = fma(th[l], w, A.P(l, PP) * fma(kB, th[l], kA));
+#else
                 const double g = fma(th[l], w, pl[l] * fma(kB, th[l], kA));
+#endif
                 gp[l] = fma(lam, w, g);
                 gm[l] = fma(-lam, w, g);
             }
