@@ -43,7 +43,8 @@ class Phys(C.Structure):
     _fields_ = [("gamma", C.c_double), ("R", C.c_double), ("Pr", C.c_double),
                 ("mu_law", C.c_int32), ("mu_ref", C.c_double), ("T_ref", C.c_double),
                 ("S", C.c_double), ("weno_eps", C.c_double), ("terms", C.c_int32),
-                ("dir_mask", C.c_int32), ("weno_linear", C.c_int32), ("weno_weights", C.c_int32)]
+                ("dir_mask", C.c_int32), ("weno_linear", C.c_int32), ("weno_weights", C.c_int32),
+                ("weno_limiter", C.c_int32), ("weno_alpha_rl", C.c_double), ("weno_alpha_al", C.c_double)]
 
 
 class Split(C.Structure):
@@ -65,8 +66,10 @@ def splits(spec=None):
 
 
 def phys(gamma=1.4, R=1.0, Pr=0.72, mu_law=MU_CONST, mu_ref=0.0, T_ref=1.0, S=0.0,
-         weno_eps=1e-6, terms=INVISCID | VISCOUS, dir_mask=7, weno_linear=0, weno_weights=0) -> Phys:
-    return Phys(gamma, R, Pr, mu_law, mu_ref, T_ref, S, weno_eps, terms, dir_mask, weno_linear, weno_weights)
+         weno_eps=1e-6, terms=INVISCID | VISCOUS, dir_mask=7, weno_linear=0, weno_weights=0,
+         weno_limiter=0, weno_alpha_rl=0.0, weno_alpha_al=0.0) -> Phys:
+    return Phys(gamma, R, Pr, mu_law, mu_ref, T_ref, S, weno_eps, terms, dir_mask, weno_linear, weno_weights,
+                weno_limiter, weno_alpha_rl, weno_alpha_al)
 
 
 _lib = None
@@ -85,6 +88,8 @@ def lib():
         L.oracle_weno_symbo.restype = C.c_double
         L.oracle_weno.argtypes = [dp, C.c_double, C.c_int, C.c_int]
         L.oracle_weno.restype = C.c_double
+        L.oracle_weno_lim.argtypes = [dp, C.c_double, C.c_int, C.c_int, C.c_int, C.c_double, C.c_double]
+        L.oracle_weno_lim.restype = C.c_double
         L.oracle_eigvecs.argtypes = [dp, C.c_double, C.c_double, C.c_double, C.c_double,
                                      C.c_double, C.c_double, dp, dp]
         L.oracle_interface_flux.argtypes = [C.POINTER(Phys), dp, dp, dp]
@@ -159,6 +164,13 @@ def weno_symbo(v, eps=1e-6, linear=False, weights=0) -> float:
     """W(v_{-2..3}) at the +1/2 interface; weights 0 = SYMBO, 1 = SYMOO."""
     a = np.ascontiguousarray(v, dtype=np.float64)
     return float(lib().oracle_weno(_dp(a), eps, int(linear), int(weights)))
+
+
+def weno_limited(v, eps=1e-6, limiter=0, alpha_rl=0.0, alpha_al=0.0, weights=0, linear=False) -> float:
+    """W with the relative (bit 0) / absolute (bit 1) limiters of reading 23."""
+    a = np.ascontiguousarray(v, dtype=np.float64)
+    return float(lib().oracle_weno_lim(_dp(a), eps, int(linear), int(weights), int(limiter),
+                                        float(alpha_rl), float(alpha_al)))
 
 
 def eigvecs(nrm, rho, u, v, w, c, gamma=1.4):

@@ -53,6 +53,8 @@ typedef struct {
     int32_t terms, dir_mask;
     int32_t weno_linear; /* test flag: 1 forces omega_k = C_k (linear stencil) */
     int32_t weno_weights; /* 0: SYMBO (Martin et al. 2006), 1: SYMOO (reading 22, NEXT-3) */
+    int32_t weno_limiter; /* bit 0: relative, bit 1: absolute limiter (reading 23, NEXT-3); 0 = off */
+    double weno_alpha_rl, weno_alpha_al; /* thresholds of the two limiters */
 } oracle_phys;
 
 typedef struct {
@@ -305,7 +307,21 @@ void oracle_metrics(const int64_t n[3], const int32_t bc[6], const double *xyz, 
 static const double C_SYMBO[4] = {0.094647545896, 0.428074212384, 0.408289331408, 0.068988910311};
 static const double C_SYMOO[4] = {1.0 / 20.0, 9.0 / 20.0, 9.0 / 20.0, 1.0 / 20.0};
 
+/* WENO limiters (reading 23; [lit] Taylor, Wu & Martin 2007, not in the
+   paper): after the downwind substitution, the reconstruction falls back to the linear
+   optimal weights omega_k = C_k when
+     (limiter & 1) and max_k beta_k < alpha_rl * min_k beta_k   (relative limiter), or
+     (limiter & 2) and max_k beta_k < alpha_al                  (absolute limiter).      */
+double oracle_weno_lim(const double v[6], double eps, int linear, int weights, int limiter,
+                       double alpha_rl, double alpha_al);
+
 double oracle_weno(const double v[6], double eps, int linear, int weights)
+{
+    return oracle_weno_lim(v, eps, linear, weights, 0, 0.0, 0.0);
+}
+
+double oracle_weno_lim(const double v[6], double eps, int linear, int weights, int limiter,
+                       double alpha_rl, double alpha_al)
 {
     const double *Cw = weights == 1 ? C_SYMOO : C_SYMBO;
     /* v[0..5] = v_{-2}, v_{-1}, v_0, v_1, v_2, v_3 */
@@ -337,6 +353,16 @@ double oracle_weno(const double v[6], double eps, int linear, int weights)
         if (beta[k] > bmax)
             bmax = beta[k];
     beta[3] = bmax;
+    if (limiter) {
+        double bmin = beta[0];
+        for (int k = 1; k < 4; k++)
+            if (beta[k] < bmin)
+                bmin = beta[k];
+        if ((limiter & 1) && bmax < alpha_rl * bmin)
+            linear = 1;
+        if ((limiter & 2) && bmax < alpha_al)
+            linear = 1;
+    }
     double alpha[4], asum = 0.0, num = 0.0;
     for (int k = 0; k < 4; k++) {
         if (linear)
@@ -497,8 +523,10 @@ void oracle_interface_flux(const oracle_phys *ph, const double Ul[30], const dou
             vp[l] = 0.5 * (g[s][l] + lam[s] * wv[s][l]);
             vm[5 - l] = 0.5 * (g[s][l] - lam[s] * wv[s][l]); /* mirrored: i+3 .. i-2 */
         }
-        gh[s] = oracle_weno(vp, ph->weno_eps, ph->weno_linear, ph->weno_weights) +
-                oracle_weno(vm, ph->weno_eps, ph->weno_linear, ph->weno_weights);
+        gh[s] = oracle_weno_lim(vp, ph->weno_eps, ph->weno_linear, ph->weno_weights, ph->weno_limiter,
+                                ph->weno_alpha_rl, ph->weno_alpha_al) +
+                oracle_weno_lim(vm, ph->weno_eps, ph->weno_linear, ph->weno_weights, ph->weno_limiter,
+                                ph->weno_alpha_rl, ph->weno_alpha_al);
     }
     for (int q = 0; q < 5; q++) {
         double f = 0.0;

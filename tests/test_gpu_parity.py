@@ -269,7 +269,7 @@ def _block_points(bn, rng, k_random):
 
 
 @pytest.mark.slow
-@pytest.mark.parametrize("name", ["weak", "ramp"])
+@pytest.mark.parametrize("name", ["weak", "ramp", "tgv"])
 def test_full_size_config_sampled(name):
     """BASELINE.json full sizes in bench.py's launch configuration (crocco_rk_stage):
     weak = 512^3 periodic wavy TGV (configs[4]); ramp = 1024 x 512 x 256 Mach-6

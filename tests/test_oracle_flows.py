@@ -54,12 +54,13 @@ def test_free_stream_preserved_on_wavy_grid(terms):
 
 # ------------------------------------------------------------------ conservation (periodic)
 
-def test_periodic_conservation_of_sum_U_over_J():
+@pytest.mark.parametrize("lim", [{}, dict(weno_limiter=3, weno_alpha_rl=5.0, weno_alpha_al=1e-3)])
+def test_periodic_conservation_of_sum_U_over_J(lim):
     n = (16, 14, 12)
     grid = synth.Wavy3D(L=(10.0,) * 3, N=n)
     Ui = synth.random_state(n, seed=7, amp=0.2)
     xyz, met, U = _setup(grid, n, PER, Ui)
-    ph = oracle.phys(terms=3, mu_law=1, mu_ref=0.02, S=0.5)
+    ph = oracle.phys(terms=3, mu_law=1, mu_ref=0.02, S=0.5, **lim)
     r = _inner(oracle.rhs(n, ph, U, met))
     J = _inner(met)[0]
     tot = (r / J).reshape(5, -1).sum(1)
@@ -220,13 +221,14 @@ def test_exact_riemann_solver_matches_toro_table():
     assert abs(rsR - gold["rho_star_R"]) < 1e-5
 
 
-def test_sod_shock_tube_vs_exact():
+@pytest.mark.parametrize("lim", [{}, dict(weno_limiter=1, weno_alpha_rl=5.0)])
+def test_sod_shock_tube_vs_exact(lim):
     c = synth.case("sod")
     n = c.n_global
     xyz = c.grid.coords(n, (0, 0, 0), oracle.GC)
     met = oracle.metrics(n, c.bc, xyz)
     U = synth.pad_state(synth.sod(xyz))
-    ph = oracle.phys(terms=1)
+    ph = oracle.phys(terms=1, **lim)
     oracle.advance(n, c.bc, ph, c.dt, c.steps, U, met)
     rho = _inner(U)[0]
     x = synth._interior_xyz(xyz)[0][0, 0]

@@ -478,3 +478,46 @@ def test_symoo_exact_for_quintic_cell_averages_in_linear_mode():
 
 def test_symoo_nonlinear_still_nonoscillatory():
     assert abs(oracle.weno_symbo([0, 0, 0, 0, 1, 1], weights=1)) < 1e-9
+
+
+# ------------------------------------------------------------------ WENO limiters (reading 23, NEXT-3)
+
+# v_i = i^3 at i = -2..3.  Jiang-Shu indicators by hand (App. A.3 definitions):
+#   beta_0 = 13/12 (-6)^2 + 1/4 (-4)^2 = 43,  beta_1 = 0 + 1/4 (-2)^2 = 1,
+#   beta_2 = 13/12 6^2 + 1/4 4^2 = 43,        beta_3 = 13/12 12^2 + 1/4 (-22)^2 = 277
+# so max/min = 277 and max = 277 (the downwind beta_3 is already the largest).
+CUBIC = [-8.0, -1.0, 0.0, 1.0, 8.0, 27.0]
+
+
+def test_limiter_thresholds_on_hand_computed_indicators():
+    lin = oracle.weno_symbo(CUBIC, linear=True)
+    non = oracle.weno_symbo(CUBIC)
+    assert abs(lin - non) > 1e-2                       # the two branches are distinguishable
+    lim = lambda **kw: oracle.weno_limited(CUBIC, **kw)
+    assert lim(limiter=1, alpha_rl=278.0) == lin       # 277 < 278 * 1: relative fires
+    assert lim(limiter=1, alpha_rl=276.0) == non
+    assert lim(limiter=2, alpha_al=278.0) == lin       # 277 < 278: absolute fires
+    assert lim(limiter=2, alpha_al=276.0) == non
+    assert lim(limiter=3, alpha_rl=276.0, alpha_al=278.0) == lin   # either limiter suffices
+    assert lim(limiter=3, alpha_rl=278.0, alpha_al=276.0) == lin
+    assert lim(limiter=3, alpha_rl=276.0, alpha_al=276.0) == non
+    assert lim(limiter=0, alpha_rl=1e300, alpha_al=1e300) == non   # flags off
+
+
+def test_limiter_limits_reduce_to_linear_and_plain_weno():
+    rng = np.random.default_rng(23)
+    for _ in range(200):
+        v = rng.normal(size=6) * 10.0 ** rng.uniform(-3, 3)
+        # thresholds that always / never fire (beta >= 0, so max < 0 * min is never true)
+        assert oracle.weno_limited(v, limiter=1, alpha_rl=1e300) == oracle.weno_symbo(v, linear=True)
+        assert oracle.weno_limited(v, limiter=3, alpha_rl=0.0, alpha_al=0.0) == oracle.weno_symbo(v)
+
+
+def test_limiter_keeps_step_nonoscillatory_and_smooth_data_linear():
+    # at a jump the indicators differ by orders of magnitude -> nonlinear weights stay;
+    # on a gentle sine they are within a factor ~1.5 -> relative limiter (5) goes linear
+    step = [0.0, 0.0, 0.0, 1.0, 1.0, 1.0]
+    assert oracle.weno_limited(step, limiter=1, alpha_rl=5.0) == oracle.weno_symbo(step)
+    x = np.arange(-2, 4) * 0.05
+    s = np.sin(x + 0.3)
+    assert oracle.weno_limited(s, limiter=1, alpha_rl=5.0) == oracle.weno_symbo(s, linear=True)
