@@ -115,6 +115,12 @@ typedef struct {
     int32_t weno_weights;  /* optimal weights: 0 = SYMBO (bandwidth-optimised, Martin et al. 2006),
                               1 = SYMOO (1/20, 9/20, 9/20, 1/20: 6th-order central linear stencil);
                               reading 22, SURVEY NEXT-3 */
+    int32_t weno_limiter;  /* WENO limiters (reading 23), bitmask, 0 = off: after
+                              beta_3 <- max(beta), use the linear weights omega = C when
+                              bit 0: max beta < weno_alpha_rl * min beta (relative limiter),
+                              bit 1: max beta < weno_alpha_al (absolute limiter; beta of the
+                              reconstructed characteristic flux (g +- lambda w)/2) */
+    double weno_alpha_rl, weno_alpha_al;  /* thresholds, >= 0 */
 } crocco_phys;
 
 typedef struct {

@@ -44,7 +44,8 @@ class PhysC(C.Structure):
     _fields_ = [("gamma", C.c_double), ("R", C.c_double), ("Pr", C.c_double),
                 ("mu_law", C.c_int32), ("mu_ref", C.c_double), ("T_ref", C.c_double),
                 ("S", C.c_double), ("weno_eps", C.c_double), ("terms", C.c_int32),
-                ("dir_mask", C.c_int32), ("weno_weights", C.c_int32)]
+                ("dir_mask", C.c_int32), ("weno_weights", C.c_int32), ("weno_limiter", C.c_int32),
+                ("weno_alpha_rl", C.c_double), ("weno_alpha_al", C.c_double)]
 
 
 class BlockLayout(C.Structure):
@@ -172,8 +173,10 @@ def make_desc(n_global, n_blocks=(1, 1, 1), bc=((0, 0),) * 3, dirichlet=None, ra
 
 
 def make_phys(gamma=1.4, R=1.0, Pr=0.72, mu_law=MU_CONST, mu_ref=0.0, T_ref=1.0, S=0.0,
-              weno_eps=1e-6, terms=TERM_INVISCID | TERM_VISCOUS, dir_mask=7, weno_weights=0):
-    return PhysC(gamma, R, Pr, mu_law, mu_ref, T_ref, S, weno_eps, terms, dir_mask, weno_weights)
+              weno_eps=1e-6, terms=TERM_INVISCID | TERM_VISCOUS, dir_mask=7, weno_weights=0,
+              weno_limiter=0, weno_alpha_rl=0.0, weno_alpha_al=0.0):
+    return PhysC(gamma, R, Pr, mu_law, mu_ref, T_ref, S, weno_eps, terms, dir_mask, weno_weights,
+                 weno_limiter, weno_alpha_rl, weno_alpha_al)
 
 
 def crocco_init_grid(desc: GridDesc, phys: PhysC):

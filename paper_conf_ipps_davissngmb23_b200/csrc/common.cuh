@@ -17,6 +17,9 @@ struct Phys {
     double eps;
     int terms, dir_mask;
     double wC[4];  // WENO optimal weights (SYMBO or SYMOO)
+    int lim;       // WENO limiters (reading 23): bit 0 relative, bit 1 absolute
+    double arl;    // relative threshold (scale-free)
+    double aal_b;  // absolute threshold in the units of the kernels' b_k (weno.cuh)
 };
 
 struct Lay {  // padded block layout (elements)
@@ -78,6 +81,10 @@ __device__ __forceinline__ double sqrt_nr(double x) {  // x > 0
 __device__ __forceinline__ double maxnn(double a, double b) {
     const long long x = __double_as_longlong(a), y = __double_as_longlong(b);
     return __longlong_as_double(x > y ? x : y);
+}
+__device__ __forceinline__ double minnn(double a, double b) {
+    const long long x = __double_as_longlong(a), y = __double_as_longlong(b);
+    return __longlong_as_double(x < y ? x : y);
 }
 
 // primitive buffer components (k_prims)

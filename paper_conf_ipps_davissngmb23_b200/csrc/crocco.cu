@@ -323,8 +323,12 @@ static constexpr size_t sweep_smem_bytes() {
 }
 template <int D, bool V>
 static cudaError_t sweep_attr1() {
-    return cudaFuncSetAttribute(k_sweep_s<D, V>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                (int)sweep_smem_bytes<D>());
+    cudaError_t e = cudaFuncSetAttribute(k_sweep_s<D, V, false>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                         (int)sweep_smem_bytes<D>());
+    if (e == cudaSuccess)
+        e = cudaFuncSetAttribute(k_sweep_s<D, V, true>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                 (int)sweep_smem_bytes<D>());
+    return e;
 }
 static cudaError_t sweep_attrs() {
     cudaError_t e = sweep_attr1<0, false>();
@@ -397,6 +401,11 @@ static Phys to_phys(const crocco_phys *p) {
     static const double SYMBO[4] = {0.094647545896, 0.428074212384, 0.408289331408, 0.068988910311};
     static const double SYMOO[4] = {1.0 / 20.0, 9.0 / 20.0, 9.0 / 20.0, 1.0 / 20.0};
     for (int k = 0; k < 4; k++) ph.wC[k] = p->weno_weights == 1 ? SYMOO[k] : SYMBO[k];
+    ph.lim = p->weno_limiter;
+    ph.arl = p->weno_alpha_rl;
+    // b_k of the kernels = (12/13) beta_k of the reconstructed values, which carry a factor 2
+    // (LLF 1/2 folded, flux.cuh): b = (48/13) beta of (g +- lambda w)/2
+    ph.aal_b = p->weno_alpha_al * (4.0 * WENO_BSCALE);
 #if CROCCO_WENO_FOLD
     // only the ratios C_k / C_0 enter W (weno.cuh); alpha_0 then needs no multiply
     const double c0 = ph.wC[0];
@@ -413,6 +422,9 @@ static crocco_status check_phys(const crocco_phys *p) {
     if (p->mu_law == 1 && !(p->T_ref > 0)) return fail(nullptr, CROCCO_ERR_ARG, "bad T_ref");
     if (p->terms & ~3) return fail(nullptr, CROCCO_ERR_ARG, "bad terms mask");
     if (p->weno_weights != 0 && p->weno_weights != 1) return fail(nullptr, CROCCO_ERR_ARG, "bad weno_weights");
+    if (p->weno_limiter & ~3) return fail(nullptr, CROCCO_ERR_ARG, "bad weno_limiter mask");
+    if (!(p->weno_alpha_rl >= 0) || !(p->weno_alpha_al >= 0))
+        return fail(nullptr, CROCCO_ERR_ARG, "WENO limiter thresholds must be >= 0");
     return CROCCO_OK;
 }
 
@@ -933,8 +945,13 @@ static crocco_status rhs_block(crocco_ctx c, const LocalBlock &b, const double *
         const int64_t warps = lines * ((nd + seg - 1) / seg);
         const unsigned grid = cdiv(warps * 32, SWEEP_THREADS);
 #if CROCCO_SWEEP_SMEM
-#define SWEEP_LAUNCH(DD, VV) \
-        k_sweep_s<DD, VV><<<grid, SWEEP_THREADS, sweep_smem_bytes<DD>(), c->stream>>>(a, b.L, ph)
+#define SWEEP_LAUNCH(DD, VV)                                                                              \
+    do {                                                                                                  \
+        if (ph.lim)                                                                                       \
+            k_sweep_s<DD, VV, true><<<grid, SWEEP_THREADS, sweep_smem_bytes<DD>(), c->stream>>>(a, b.L, ph);  \
+        else                                                                                              \
+            k_sweep_s<DD, VV, false><<<grid, SWEEP_THREADS, sweep_smem_bytes<DD>(), c->stream>>>(a, b.L, ph); \
+    } while (0)
         if (d == 0) LAUNCH(c, K_FLUX_X, if (a.visc) SWEEP_LAUNCH(0, true); else SWEEP_LAUNCH(0, false));
         else if (d == 1) LAUNCH(c, K_FLUX_Y, if (a.visc) SWEEP_LAUNCH(1, true); else SWEEP_LAUNCH(1, false));
         else LAUNCH(c, K_FLUX_Z, if (a.visc) SWEEP_LAUNCH(2, true); else SWEEP_LAUNCH(2, false));

@@ -90,7 +90,7 @@ struct SAcc {
 
 // Total interface flux F = F^_inv - h_v of direction D at interface i+1/2.
 // A: stencil accessor (flux.cuh GAcc / SAcc).
-template <int D, class Acc>
+template <int D, class Acc, bool LIM = false>
 __device__ __forceinline__ void total_flux(const Acc &A, bool inv, bool visc, const Phys &ph,
                                            double F[5]) {
     F[0] = F[1] = F[2] = F[3] = F[4] = 0.0;
@@ -234,7 +234,7 @@ __device__ __forceinline__ void total_flux(const Acc &A, bool inv, bool visc, co
                 gm[l] = fma(-lam, w, g);
             }
 #if CROCCO_DEFER_DIV
-            const WenoFrac wf = weno_pair_frac(gp, gm, eps_b, ph.wC);
+            const WenoFrac wf = weno_pair_frac<LIM>(gp, gm, eps_b, ph.wC, &ph);
             gb[sf] = wf.base;
             gn[sf] = wf.num;
             gd[sf] = wf.den;
@@ -272,7 +272,7 @@ __device__ __forceinline__ void total_flux(const Acc &A, bool inv, bool visc, co
                 R4 = alph * fma(phi2 + c2, ph.igm1, sc * tht);
             }
 #else
-            const double gh = weno_pair(gp, gm, eps_b, ph.wC);
+            const double gh = weno_pair<LIM>(gp, gm, eps_b, ph.wC, &ph);
 #endif
             f0 = fma(R0, gh, f0);
             f1 = fma(R1, gh, f1);

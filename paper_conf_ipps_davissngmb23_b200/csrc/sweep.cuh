@@ -149,7 +149,8 @@ __global__ void __launch_bounds__(SWEEP_THREADS, CROCCO_SWEEP_MINB) k_sweep(cons
             const int vi = D == 0 ? e - 1 : pi, vj = D == 1 ? e - 1 : pj, vk = D == 2 ? e - 1 : pk;
             const GAcc<D> A{a.in.U, a.in.P, a.in.M + (int64_t)(1 + 3 * D) * a.in.cs, a.in.FV,
                             a.in.cs, at(L, qi, qj, qk), s, a.in.vcs, vat(a.V, vi, vj, vk) - vs, vs};
-            total_flux<D>(A, inv, visc, ph, F);
+            if (ph.lim) total_flux<D, GAcc<D>, true>(A, inv, visc, ph, F);
+            else total_flux<D, GAcc<D>, false>(A, inv, visc, ph, F);
         } else {
 #pragma unroll
             for (int c = 0; c < 5; c++) F[c] = 0.0;
@@ -203,7 +204,7 @@ struct RingGeom {
     static constexpr int PER_WARP = SV_N * NR * C + NCB * 32 + NFC;  // doubles
 };
 
-template <int D, bool VISC>
+template <int D, bool VISC, bool LIM>
 __global__ void __launch_bounds__(SWEEP_THREADS, CROCCO_SWEEP_MINB) k_sweep_s(const __grid_constant__ SweepArgs a,
                                                                           const Lay L, const Phys ph) {
     using RG = RingGeom<D>;
@@ -394,7 +395,7 @@ __global__ void __launch_bounds__(SWEEP_THREADS, CROCCO_SWEEP_MINB) k_sweep_s(co
         issue(st + LA + 1);                   // group B: chunk st+LA+1 (slot of chunk st-1)
         if (act) {
             const SAcc<NR, C> A{sv, WS * st + ls, lt};  // ring point of stencil point i-2
-            total_flux<D>(A, inv, VISC, ph, F);
+            total_flux<D, SAcc<NR, C>, LIM>(A, inv, VISC, ph, F);
         } else {
 #pragma unroll
             for (int c = 0; c < 5; c++) F[c] = 0.0;

@@ -32,9 +32,13 @@ struct WenoFrac {
 // enter W), so alpha_0 needs no multiply, and e_k = eps + b_k is formed inside the
 // FMA chain of b_k; max_k(eps + b_k) = eps + max_k b_k (monotone), so the
 // downwind-stencil rule is unchanged.
+// LIM: the limiters of reading 23 (ph.lim / ph.arl / ph.aal_b, common.cuh): linear weights
+// alpha_k = C_k when max b < arl min b (bit 0) or max b < aal_b (bit 1), b after the
+// downwind substitution
+template <bool LIM = false>
 __device__ __forceinline__ WenoFrac weno_symbo_frac(double v0, double v1, double v2, double v3,
                                                     double v4, double v5, double eps_b,
-                                                    const double C[4]) {
+                                                    const double C[4], const Phys *lp = nullptr) {
     const double C0 = C[0], C1 = C[1], C2 = C[2], C3 = C[3];
     constexpr double K3 = 3.0 / 13.0;
     const double d0 = v1 - v0, d1 = v2 - v1, d2 = v3 - v2, d3 = v4 - v3, d4 = v5 - v4;
@@ -47,11 +51,26 @@ __device__ __forceinline__ WenoFrac weno_symbo_frac(double v0, double v1, double
     const double r1 = fma(2.0, d2, d1);
     const double r2 = fma(4.0, d2, -d3);
     const double r3 = fma(6.0, d2, -f3) - d4;    // 6 d2 - 5 d3 + 2 d4
+    bool lin = false;
+    double e0, e1, e2, e3;
+    if constexpr (LIM) {
+        const double b0 = fma(K3 * f0, f0, s0 * s0);
+        const double b1 = fma(K3 * f1, f1, s1 * s1);
+        const double b2 = fma(K3 * f2, f2, s2 * s2);
+        double b3 = fma(K3 * f3, f3, s3 * s3);
+        b3 = maxnn(maxnn(b0, b1), maxnn(b2, b3));
+        const double bmin = minnn(minnn(b0, b1), b2);  // b3 is the maximum
+        lin = ((lp->lim & 1) && b3 < lp->arl * bmin) || ((lp->lim & 2) && b3 < lp->aal_b);
+        e0 = eps_b + b0;
+        e1 = eps_b + b1;
+        e2 = eps_b + b2;
+        e3 = eps_b + b3;
+    } else {
 #if CROCCO_WENO_FOLD
-    double e0 = fma(s0, s0, fma(K3 * f0, f0, eps_b));
-    double e1 = fma(s1, s1, fma(K3 * f1, f1, eps_b));
-    double e2 = fma(s2, s2, fma(K3 * f2, f2, eps_b));
-    double e3 = fma(s3, s3, fma(K3 * f3, f3, eps_b));
+    e0 = fma(s0, s0, fma(K3 * f0, f0, eps_b));
+    e1 = fma(s1, s1, fma(K3 * f1, f1, eps_b));
+    e2 = fma(s2, s2, fma(K3 * f2, f2, eps_b));
+    e3 = fma(s3, s3, fma(K3 * f3, f3, eps_b));
     // downwind stencil never preferred (continuous max, parity-safe)
     e3 = maxnn(maxnn(e0, e1), maxnn(e2, e3));
 #else
@@ -61,21 +80,30 @@ __device__ __forceinline__ WenoFrac weno_symbo_frac(double v0, double v1, double
     double b3 = fma(K3 * f3, f3, s3 * s3);
     // downwind stencil never preferred (continuous max, parity-safe)
     b3 = maxnn(maxnn(b0, b1), maxnn(b2, b3));
-    double e0 = eps_b + b0, e1 = eps_b + b1, e2 = eps_b + b2, e3 = eps_b + b3;
+    e0 = eps_b + b0, e1 = eps_b + b1, e2 = eps_b + b2, e3 = eps_b + b3;
 #endif
+    }
     e0 *= e0;
     e1 *= e1;
     e2 *= e2;
     e3 *= e3;
     // alpha_0 = C0 e1 e2 e3, alpha_1 = C1 e0 e2 e3, alpha_2 = C2 e0 e1 e3, alpha_3 = C3 e0 e1 e2
-    const double e01 = e0 * e1, e23 = e2 * e3;
+    double e01 = e0 * e1, e23 = e2 * e3;
 #if CROCCO_WENO_FOLD
-    const double x0 = e1;  // C0 = 1
-    (void)C0;
+    double x0 = e1;  // C0 = 1
 #else
-    const double x0 = C0 * e1;
+    double x0 = C0 * e1;
 #endif
-    const double x1 = C1 * e0, x2 = C2 * e3, x3 = C3 * e2;
+    double x1 = C1 * e0, x2 = C2 * e3, x3 = C3 * e2;
+    if constexpr (LIM) {
+        if (lin) {  // linear optimal weights: alpha_k = C_k
+            x0 = C0;
+            x1 = C1;
+            x2 = C2;
+            x3 = C3;
+            e01 = e23 = 1.0;
+        }
+    }
     WenoFrac w;
     w.base = v2;
     w.num = fma(e23, fma(x0, r0, x1 * r1), e01 * fma(x2, r2, x3 * r3));
@@ -86,19 +114,21 @@ __device__ __forceinline__ WenoFrac weno_symbo_frac(double v0, double v1, double
 // W^+ of (vp0..vp5) plus W^- of the mirrored (vm5..vm0), as one fraction:
 // (b+ + b-) + (n+ d- + n- d+)/(6 d+ d-)  -- one division per characteristic field.
 // Range: the alpha products stay inside fp64 for |v| up to ~1e9.
+template <bool LIM = false>
 __device__ __forceinline__ WenoFrac weno_pair_frac(const double vp[6], const double vm[6], double eps_b,
-                                                   const double C[4]) {
-    const WenoFrac a = weno_symbo_frac(vp[0], vp[1], vp[2], vp[3], vp[4], vp[5], eps_b, C);
-    const WenoFrac b = weno_symbo_frac(vm[5], vm[4], vm[3], vm[2], vm[1], vm[0], eps_b, C);
+                                                   const double C[4], const Phys *lp = nullptr) {
+    const WenoFrac a = weno_symbo_frac<LIM>(vp[0], vp[1], vp[2], vp[3], vp[4], vp[5], eps_b, C, lp);
+    const WenoFrac b = weno_symbo_frac<LIM>(vm[5], vm[4], vm[3], vm[2], vm[1], vm[0], eps_b, C, lp);
     WenoFrac w;
     w.base = a.base + b.base;
     w.num = fma(a.num, b.den, b.num * a.den);
     w.den = 6.0 * (a.den * b.den);
     return w;
 }
+template <bool LIM = false>
 __device__ __forceinline__ double weno_pair(const double vp[6], const double vm[6], double eps_b,
-                                            const double C[4]) {
-    const WenoFrac w = weno_pair_frac(vp, vm, eps_b, C);
+                                            const double C[4], const Phys *lp = nullptr) {
+    const WenoFrac w = weno_pair_frac<LIM>(vp, vm, eps_b, C, lp);
     return w.base + div_nr(w.num, w.den);
 }
 

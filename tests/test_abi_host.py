@@ -64,11 +64,18 @@ def test_invalid_desc_is_err_arg(kw, frag):
     assert frag in str(ei.value)
 
 
-def test_invalid_phys_is_err_arg():
+@pytest.mark.parametrize("kw,frag", [
+    (dict(gamma=1.0), "gas constants"),
+    (dict(weno_limiter=4), "weno_limiter"),
+    (dict(weno_limiter=1, weno_alpha_rl=-1.0), "thresholds"),
+    (dict(weno_weights=2), "weno_weights"),
+])
+def test_invalid_phys_is_err_arg(kw, frag):
     d = cc.make_desc((8, 8, 8))
     with pytest.raises(cc.CroccoError) as ei:
-        cc.crocco_init_grid(d, cc.make_phys(gamma=1.0))
+        cc.crocco_init_grid(d, cc.make_phys(**kw))
     assert ei.value.status == cc.CROCCO_ERR_ARG
+    assert frag in str(ei.value)
 
 
 def _plan_all(n, nb, bc, nranks=1, block_rank=None):

@@ -118,6 +118,33 @@ def test_rhs_parity_terms(terms, mask, weights):
     assert err < 1e-11, err
 
 
+@pytest.mark.parametrize("lim,arl,aal", [(1, 5.0, 0.0), (2, 0.0, 2e-3), (3, 3.0, 1e-4)])
+def test_rhs_parity_weno_limiters(lim, arl, aal):
+    """Reading 23 limiters (NEXT-3): random wavy state (both branches taken) and the smooth
+    vortex (relative limiter mostly linear), against the oracle."""
+    n = (37, 29, 23)
+    kw = dict(terms=3, mu_ref=0.02, weno_limiter=lim, weno_alpha_rl=arl, weno_alpha_al=aal)
+    err, _, _ = _rhs_parity(wavy_random(n, 41, kw))
+    assert err < 1e-11, err
+    c = synth.case("vortex", scale=2)
+    _, U = synth.block_inputs(c, (0, 0, 0), c.n_global)
+    pb = Problem(c.n_global, c.grid, c.bc, U, dict(c.phys, weno_limiter=lim, weno_alpha_rl=arl,
+                                                     weno_alpha_al=aal))
+    err, _, _ = _rhs_parity(pb)
+    assert err < 1e-11, err
+
+
+def test_weno_limiter_changes_the_result():
+    """The limited GPU RHS differs from the plain one (the switch is live) and matches the
+    oracle's limited RHS, not its plain one."""
+    n = (24, 20, 16)
+    base = dict(terms=1)
+    _, plain, ref_plain = _rhs_parity(wavy_random(n, 43, base))
+    err, lim, ref_lim = _rhs_parity(wavy_random(n, 43, dict(base, weno_limiter=1, weno_alpha_rl=5.0)))
+    assert err < 1e-11, err
+    assert np.abs(lim - plain).max() > 1e3 * np.abs(lim - ref_lim).max()
+
+
 def test_rhs_parity_sutherland_multiblock():
     n = (40, 24, 16)
     pb = wavy_random(n, 5, dict(terms=3, mu_law=1, mu_ref=0.03, T_ref=1.0, S=0.4, Pr=0.71))
