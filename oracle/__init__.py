@@ -23,7 +23,7 @@ _LIB = os.path.join(_HERE, "liboracle.so")
 
 G = 4
 GC = 10
-PERIODIC, EXTRAP, DIRICHLET, WALL, SLIPWALL, SPLIT = 0, 1, 2, 3, 4, 5
+PERIODIC, EXTRAP, DIRICHLET, WALL, SLIPWALL, SPLIT, COARSE_FINE = 0, 1, 2, 3, 4, 5, 6
 INVISCID, VISCOUS = 1, 2
 FIELD_STATE, FIELD_METRIC = 0, 1
 MU_CONST, MU_SUTHERLAND = 0, 1
@@ -107,6 +107,10 @@ def lib():
                                         C.c_int32, dp, dp]
         L.oracle_compute_dt.argtypes = [i64p, C.POINTER(Phys), dp, dp, C.c_double]
         L.oracle_compute_dt.restype = C.c_double
+        L.oracle_fill_two_levels.argtypes = [i64p, i32p, dp, dp, dp, i64p, i64p, dp]
+        L.oracle_average_down.argtypes = [i64p, i32p, dp, dp, i64p, i64p, dp]
+        L.oracle_amr_advance.argtypes = [i64p, i32p, dp, i64p, i32p, dp, i64p, C.POINTER(Phys),
+                                         C.c_double, C.c_int32, dp, dp, dp, dp]
         L.oracle_set_threads.argtypes = [C.c_int]
         L.oracle_get_threads.restype = C.c_int
         _lib = L
@@ -217,3 +221,29 @@ def advance(n, bc, ph, dt, nsteps, U, met, dirichlet=None, split=None, t0=0.0):
 def compute_dt(n, ph: Phys, U, met, cfl):
     """ComputeDt: CFL / max_i sum_d J(|m^d.u| + c|m^d|) (Eq. 3, 95, 131)."""
     return float(lib().oracle_compute_dt(_n(n), C.byref(ph), _dp(U), _dp(met), float(cfl)))
+
+
+# ---- two-level AMR (SURVEY 8(f) NEXT-4; oracle section 9, readings 24-26) ----
+def fill_two_levels(nf, bcf, Uf, nc, c0, Uc, dirichlet=None, met=None):
+    """FillPatchTwoLevels in place on the fine state Uf: the three-phase fill with COARSE_FINE
+    faces interpolated (trilinear, ratio 2, node-centred) from the coarse state Uc (ghosts filled)."""
+    d = _dir(dirichlet)
+    mp = _dp(met) if met is not None else None
+    lib().oracle_fill_two_levels(_n(nf), _bc(bcf), _dp(d), mp, _dp(Uf), _n(nc), _n(c0), _dp(Uc))
+    return Uf
+
+
+def average_down(nf, bcf, Uf, nc, c0, Uc, dirichlet=None):
+    """AverageDown in place on Uc (covered coarse nodes = trapezoid average of the fine data over
+    the coarse cell); refills the same-level ghosts of Uf first."""
+    d = _dir(dirichlet)
+    lib().oracle_average_down(_n(nf), _bc(bcf), _dp(d), _dp(Uf), _n(nc), _n(c0), _dp(Uc))
+    return Uc
+
+
+def amr_advance(nc, bcc, nf, bcf, c0, ph, dt, nsteps, Uc, metc, Uf, metf, dirc=None, dirf=None):
+    """nsteps two-level RK3 steps (Alg. 2 with levels 0, 1 and AverageDown), in place on Uc, Uf."""
+    lib().oracle_amr_advance(_n(nc), _bc(bcc), _dp(_dir(dirc)), _n(nf), _bc(bcf), _dp(_dir(dirf)),
+                             _n(c0), C.byref(ph), float(dt), int(nsteps), _dp(Uc), _dp(metc),
+                             _dp(Uf), _dp(metf))
+    return Uc, Uf

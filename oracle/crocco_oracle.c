@@ -123,9 +123,31 @@ typedef struct {
     double right[5];
 } oracle_split;
 
+/* COARSE_FINE faces (two-level AMR, section 9): the ghosts of a fine-level
+   face inside the coarse domain are interpolated from the coarse level (FillPatchTwoLevels,
+   PAPER.md:83, 129).  Without a coarse level (amr == NULL) they are left untouched. */
+enum { O_COARSE_FINE = 6 };
+typedef struct {
+    int64_t nc[3];    /* coarse-level interior size (one global box, ghost width 4) */
+    int64_t c0[3];    /* coarse node index of fine node 0 (refinement ratio 2) */
+    const double *Uc; /* coarse state, padded, ghosts filled */
+} oracle_amr;
+static void cf_interp(const oracle_amr *a, const int64_t f[3], double v[5]);
+
+static void fill_core(const int64_t n[3], const int32_t bc[6], const double dirichlet[30],
+                      const oracle_split *split, double t, const double *met, double *f,
+                      int32_t ncomp, int32_t kind, const oracle_amr *amr);
+
 void oracle_fill_ex(const int64_t n[3], const int32_t bc[6], const double dirichlet[30],
                     const oracle_split *split, double t, const double *met, double *f,
                     int32_t ncomp, int32_t kind)
+{
+    fill_core(n, bc, dirichlet, split, t, met, f, ncomp, kind, NULL);
+}
+
+static void fill_core(const int64_t n[3], const int32_t bc[6], const double dirichlet[30],
+                      const oracle_split *split, double t, const double *met, double *f,
+                      int32_t ncomp, int32_t kind, const oracle_amr *amr)
 {
     obox b = make_box(n, OG);
     for (int d = 0; d < 3; d++) {
@@ -138,6 +160,8 @@ void oracle_fill_ex(const int64_t n[3], const int32_t bc[6], const double dirich
             int kindbc = bc[2 * d + side];
             if (kind == O_FIELD_METRIC && kindbc != O_PERIODIC)
                 continue; /* metrics: only periodic copies; physical faces keep computed ghosts */
+            if (kindbc == O_COARSE_FINE && (amr == NULL || kind != O_FIELD_STATE))
+                continue; /* no coarse level given: C/F ghosts untouched */
             const oracle_split *sp = (kindbc == O_SPLIT) ? &split[2 * d + side] : NULL;
             const double s_t = sp ? sp->i0 + sp->di_dt * t : 0.0;
             for (int64_t gg = 1; gg <= OG; gg++) {
@@ -173,6 +197,12 @@ void oracle_fill_ex(const int64_t n[3], const int32_t bc[6], const double dirich
                             }
                         }
                         double v[5];
+                        if (k == O_COARSE_FINE) {
+                            cf_interp(amr, id, v);
+                            for (int c = 0; c < 5; c++)
+                                f[c * b.cs + pd] = v[c];
+                            continue;
+                        }
                         for (int c = 0; c < ncomp; c++)
                             v[c] = (k == O_DIRICHLET) ? cst[c] : f[c * b.cs + ps];
                         if (k == O_WALL)
@@ -833,4 +863,153 @@ double oracle_compute_dt(const int64_t n[3], const oracle_phys *ph, const double
                     lam_max = s;
             }
     return cfl / lam_max;
+}
+
+/* ------------------------------------------------------------------ */
+/* 9. Two-level block-structured AMR (the paper's  */
+/*    v2.1 path with AMReX's trilinear interpolator,  */
+/*    115-117, 129, 141, 258; readings 24-26).                         */
+/*    Refinement ratio 2, node-centred: fine node f (fine-level index) */
+/*    sits at coarse index c0 + f/2, so even fine nodes coincide with  */
+/*    coarse nodes and odd ones lie halfway between two (*/
+/*    "fine points are always physically located halfway between      */
+/*    coarse points ... coefficients always a multiple of 1/2").       */
+/*    All levels advance with the same dt, stage by stage (Alg. 2:     */
+/*    the level loop sits inside the stage loop).    */
+/* ------------------------------------------------------------------ */
+
+/* floor(h / 2) for any sign of h */
+static int64_t floor_half(int64_t h)
+{
+    return h >= 0 ? h / 2 : -((-h + 1) / 2);
+}
+
+/* FillPatchTwoLevels value of the fine point f ("the eight neighboring
+   coarse vertices"): trilinear interpolation in index space,
+   U_f(f) = sum over the 8 corners (I + e), e in {0,1}^3, of prod_d w_d(e_d) U_c(I + e),
+   h_d = 2 c0_d + f_d, I_d = floor(h_d / 2), t_d = (h_d - 2 I_d) / 2 in {0, 1/2},
+   w_d(0) = 1 - t_d, w_d(1) = t_d.  Corner order e = (e0, e1, e2) with e0 fastest. */
+static void cf_interp(const oracle_amr *a, const int64_t f[3], double v[5])
+{
+    obox cb = make_box(a->nc, OG);
+    int64_t I[3];
+    double tt[3];
+    for (int d = 0; d < 3; d++) {
+        int64_t h = 2 * a->c0[d] + f[d];
+        I[d] = floor_half(h);
+        tt[d] = (double)(h - 2 * I[d]) * 0.5;
+    }
+    for (int c = 0; c < 5; c++)
+        v[c] = 0.0;
+    for (int e = 0; e < 8; e++) {
+        int e0 = e & 1, e1 = (e >> 1) & 1, e2 = (e >> 2) & 1;
+        double w0 = e0 ? tt[0] : 1.0 - tt[0];
+        double w1 = e1 ? tt[1] : 1.0 - tt[1];
+        double w2 = e2 ? tt[2] : 1.0 - tt[2];
+        double w = w0 * w1 * w2;
+        int64_t p = IX(&cb, I[0] + e0, I[1] + e1, I[2] + e2);
+        for (int c = 0; c < 5; c++)
+            v[c] = v[c] + w * a->Uc[c * cb.cs + p];
+    }
+}
+
+/* FillPatch of a fine level (Alg. 2 l.3-4 at level 1): the three-phase fill of section 1
+   with COARSE_FINE faces interpolated from the coarse state Uc (ghosts filled). */
+void oracle_fill_two_levels(const int64_t nf[3], const int32_t bcf[6], const double dirichlet[30],
+                            const double *metf, double *Uf, const int64_t nc[3],
+                            const int64_t c0[3], const double *Uc)
+{
+    oracle_amr a;
+    for (int d = 0; d < 3; d++) {
+        a.nc[d] = nc[d];
+        a.c0[d] = c0[d];
+    }
+    a.Uc = Uc;
+    fill_core(nf, bcf, dirichlet, NULL, 0.0, metf, Uf, 5, O_FIELD_STATE, &a);
+}
+
+/* AverageDown (Alg. 2 l.10-12; "sets covered coarse AMR cells to be equal to the
+   average of the covering fine cells"; reading 25): a coarse node I is covered when, in every
+   direction, the fine level is PERIODIC (spans the whole periodic domain) or the fine nodes
+   2(I - c0) - 1 .. 2(I - c0) + 1 are fine interior nodes.  Its new value is the average of
+   the fine data over its cell [I - 1/2, I + 1/2]^3 by the trapezoid rule on the fine nodes:
+   U_c(I) = sum_{c,b,a in {-1,0,1}} w_a w_b w_c U_f(2(I - c0) + (a, b, c)), w_0 = 1/2,
+   w_{+-1} = 1/4 (sum order: c outer, a inner).  The fine ghosts are first refilled in place
+   (same-level periodic / inter-block copies and physical BCs; C/F ghosts are not read). */
+void oracle_average_down(const int64_t nf[3], const int32_t bcf[6], const double dirichlet[30],
+                         double *Uf, const int64_t nc[3], const int64_t c0[3], double *Uc)
+{
+    static const double wt[3] = {0.25, 0.5, 0.25};
+    obox fb = make_box(nf, OG), cb = make_box(nc, OG);
+    fill_core(nf, bcf, dirichlet, NULL, 0.0, NULL, Uf, 5, O_FIELD_STATE, NULL);
+    for (int64_t k = 0; k < nc[2]; k++)
+        for (int64_t j = 0; j < nc[1]; j++)
+            for (int64_t i = 0; i < nc[0]; i++) {
+                int64_t I[3] = {i, j, k}, fc[3];
+                int covered = 1;
+                for (int d = 0; d < 3; d++) {
+                    fc[d] = 2 * (I[d] - c0[d]);
+                    if (bcf[2 * d] != O_PERIODIC && (fc[d] < 1 || fc[d] > nf[d] - 2))
+                        covered = 0;
+                }
+                if (!covered)
+                    continue;
+                int64_t pc = IX(&cb, i, j, k);
+                for (int q = 0; q < 5; q++) {
+                    double s = 0.0;
+                    for (int c = -1; c <= 1; c++)
+                        for (int bb = -1; bb <= 1; bb++)
+                            for (int a = -1; a <= 1; a++) {
+                                double w = wt[a + 1] * wt[bb + 1] * wt[c + 1];
+                                int64_t pf = IX(&fb, fc[0] + a, fc[1] + bb, fc[2] + c);
+                                s = s + w * Uf[q * fb.cs + pf];
+                            }
+                    Uc[q * cb.cs + pc] = s;
+                }
+            }
+}
+
+/* nsteps two-level RK3 steps with a fixed dt (Alg. 1 l.10 with Alg. 2): per stage, level 0
+   (fill, RHS, update), then level 1 (FillPatchTwoLevels from level 0's stage input, whose
+   ghosts that fill has just set; RHS; update), then at the third stage AverageDown of the
+   new fine state onto the new coarse state.  Uc, Uf in/out (padded). */
+void oracle_amr_advance(const int64_t nc[3], const int32_t bcc[6], const double dirc[30],
+                        const int64_t nf[3], const int32_t bcf[6], const double dirf[30],
+                        const int64_t c0[3], const oracle_phys *ph, double dt, int32_t nsteps,
+                        double *Uc, const double *metc, double *Uf, const double *metf)
+{
+    obox cb = make_box(nc, OG), fb = make_box(nf, OG);
+    size_t szc = (size_t)(5 * cb.cs) * sizeof(double), szf = (size_t)(5 * fb.cs) * sizeof(double);
+    double *Vc = (double *)malloc(szc), *Vf = (double *)malloc(szf);
+    double *dUc = (double *)calloc((size_t)(5 * cb.cs), sizeof(double));
+    double *dUf = (double *)calloc((size_t)(5 * fb.cs), sizeof(double));
+    double *rf = (double *)calloc((size_t)(5 * fb.cs), sizeof(double));
+    memcpy(Vc, Uc, szc);
+    memcpy(Vf, Uf, szf);
+    double *ac = Uc, *oc = Vc, *af = Uf, *of = Vf;
+    for (int32_t s = 0; s < nsteps; s++) {
+        for (int st = 0; st < 3; st++) {
+            oracle_rk_stage_ex(nc, bcc, dirc, NULL, 0.0, ph, st, dt, ac, oc, dUc, metc);
+            oracle_fill_two_levels(nf, bcf, dirf, metf, af, nc, c0, ac);
+            oracle_rhs(nf, ph, af, metf, rf);
+            oracle_rk_update(nf, st, dt, af, of, dUf, rf);
+            if (st == 2)
+                oracle_average_down(nf, bcf, dirf, of, nc, c0, oc);
+            double *tmp = ac;
+            ac = oc;
+            oc = tmp;
+            tmp = af;
+            af = of;
+            of = tmp;
+        }
+    }
+    if (ac != Uc)
+        memcpy(Uc, ac, szc);
+    if (af != Uf)
+        memcpy(Uf, af, szf);
+    free(Vc);
+    free(Vf);
+    free(dUc);
+    free(dUf);
+    free(rf);
 }

@@ -48,7 +48,9 @@ class Cartesian:
     centred: bool = True
 
     def coords(self, n, origin=(0, 0, 0), g=GC):
-        I, J, K = _index_grids(n, origin, g)
+        return self.map(*_index_grids(n, origin, g))
+
+    def map(self, I, J, K):
         off = 0.5 if self.centred else 0.0
         return _stack3(self.x0[0] + (I + off) * self.h[0],
                        self.x0[1] + (J + off) * self.h[1],
@@ -67,7 +69,9 @@ class Wavy3D:
     A: float = 0.3 / (2 * math.pi * 2 / 10.0)
 
     def coords(self, n, origin=(0, 0, 0), g=GC):
-        I, J, K = _index_grids(n, origin, g)
+        return self.map(*_index_grids(n, origin, g))
+
+    def map(self, I, J, K):
         xi = self.x0[0] + I * self.L[0] / self.N[0]
         et = self.x0[1] + J * self.L[1] / self.N[1]
         ze = self.x0[2] + K * self.L[2] / self.N[2]
@@ -87,7 +91,9 @@ class Wavy2D:
     A: float = 0.3 / (2 * math.pi / 10.0)
 
     def coords(self, n, origin=(0, 0, 0), g=GC):
-        I, J, K = _index_grids(n, origin, g)
+        return self.map(*_index_grids(n, origin, g))
+
+    def map(self, I, J, K):
         xi = I * self.L[0] / self.N[0]
         et = J * self.L[1] / self.N[1]
         ze = K * self.L[2] / self.N[2]
@@ -113,11 +119,29 @@ class Ramp:
         return math.tan(math.radians(self.angle_deg)) / (1.0 + np.exp(-(x - 2.0) / s))
 
     def coords(self, n, origin=(0, 0, 0), g=GC):
-        I, J, K = _index_grids(n, origin, g)
+        return self.map(*_index_grids(n, origin, g))
+
+    def map(self, I, J, K):
         x = 4.0 * I / self.N[0]
         y = self.wall(x) + np.sinh(3.0 * (J + 0.5) / self.N[1]) / math.sinh(3.0)
         z = K / self.N[2]
         return _stack3(x, y, z)
+
+
+@dataclass
+class Refined:
+    """Fine level of a two-level hierarchy (DESIGN reading 24): refinement ratio 2,
+    node-centred, fine node f at coarse index c0 + f/2, coordinates from the coarse level's
+    analytic map (the in-memory whole-grid coordinate store)."""
+    base: object
+    c0: tuple = (0, 0, 0)
+
+    def coords(self, n, origin=(0, 0, 0), g=GC):
+        I, J, K = _index_grids(n, origin, g)
+        return self.base.map(self.c0[0] + 0.5 * I, self.c0[1] + 0.5 * J, self.c0[2] + 0.5 * K)
+
+    def map(self, I, J, K):
+        return self.base.map(self.c0[0] + 0.5 * I, self.c0[1] + 0.5 * J, self.c0[2] + 0.5 * K)
 
 
 # ---------------------------------------------------------------- states

@@ -1,0 +1,210 @@
+"""Pins of the oracle's two-level AMR functions (oracle section 9;
+DESIGN.md readings 24-26) against what the paper and the mathematics fix:
+
+- FillPatchTwoLevels (trilinear, ratio 2, node-centred): reproduces every
+  multilinear field exactly (with dyadic data the fp result is exact), interpolates x^2 at a
+  halfway point to x^2 + 1/4 (linear, not higher order), copies coincident nodes, leaves the
+  fine interior untouched;
+- AverageDown ("average of the covering fine cells"): exact for linear fields,
+  x^2 -> x^2 + 1/8 per direction (trapezoid rule over the coarse cell), the covered set, and the
+  periodic conservation identity sum_c = sum_f / 8;
+- the two-level RK3 advance: free-stream preservation across the coarse/fine interface on a
+  wavy grid; with a fine level covering the whole periodic domain it reduces exactly to the
+  single-level advance of the fine grid (and the coarse level to its full-weighting average);
+  an isentropic vortex is resolved more accurately on the fine patch than on the coarse grid.
+CPU only.
+"""
+import numpy as np
+import pytest
+
+import oracle
+import synth
+
+G = 4
+CF = oracle.COARSE_FINE
+PER = ((0, 0),) * 3
+
+
+def _pad_index(n, origin, scale=1.0):
+    """Index arrays over the padded box (ghost 4) at positions origin + scale * local."""
+    ax = [origin[d] + scale * np.arange(-G, n[d] + G, dtype=np.float64) for d in range(3)]
+    return ax[0][None, None, :], ax[1][None, :, None], ax[2][:, None, None]
+
+
+def _multilinear(X, Y, Z, coef):
+    a, b, c, d, e, f, g, h = coef
+    return a + b * X + c * Y + d * Z + e * X * Y + f * Y * Z + g * X * Z + h * X * Y * Z
+
+
+def _coarse_field(nc, fn):
+    X, Y, Z = _pad_index(nc, (0, 0, 0))
+    U = np.zeros((5, nc[2] + 2 * G, nc[1] + 2 * G, nc[0] + 2 * G))
+    for q in range(5):
+        U[q] = np.broadcast_to(fn(q, X, Y, Z), U[q].shape)
+    return U
+
+
+def _ghost_mask(nf):
+    m = np.ones((nf[2] + 2 * G, nf[1] + 2 * G, nf[0] + 2 * G), bool)
+    m[G:-G, G:-G, G:-G] = False
+    return m
+
+
+COEF = [(3, 1, -2, 1, 1, -1, 2, 1), (1, 0, 0, 0, 0, 0, 0, 0), (-2, 2, 1, 3, 0, 1, -1, 0),
+        (5, -1, 1, 1, 2, 0, 0, -1), (0, 0, 0, 1, 1, 1, 1, 1)]
+
+
+@pytest.mark.parametrize("c0", [(3, 2, 4), (2, 3, 2)])
+def test_interp_reproduces_multilinear_fields(c0):
+    nc = (14, 12, 13)
+    nf = (10, 12, 8)
+    Uc = _coarse_field(nc, lambda q, X, Y, Z: _multilinear(X, Y, Z, COEF[q]))
+    Uf = np.full((5, nf[2] + 2 * G, nf[1] + 2 * G, nf[0] + 2 * G), 7.25)
+    oracle.fill_two_levels(nf, ((CF, CF),) * 3, Uf, nc, c0, Uc)
+    Xf, Yf, Zf = _pad_index(nf, c0, 0.5)
+    m = _ghost_mask(nf)
+    for q in range(5):
+        exact = np.broadcast_to(_multilinear(Xf, Yf, Zf, COEF[q]), m.shape)
+        assert np.array_equal(Uf[q][m], exact[m]), q           # every ghost, edges and corners
+        assert np.all(Uf[q][~m] == 7.25)                          # interior untouched
+
+
+def test_interp_is_linear_halfway():
+    """x^2 at a fine node halfway between two coarse nodes -> x^2 + 1/4 (coarse index units);
+    coincident nodes are copies.  A cubic or WENO interpolant would give x^2 exactly."""
+    nc = (16, 10, 10)
+    c0 = (4, 3, 3)
+    nf = (8, 8, 6)
+    Uc = _coarse_field(nc, lambda q, X, Y, Z: X * X + 0 * Y * Z + q)
+    Uf = np.zeros((5, nf[2] + 2 * G, nf[1] + 2 * G, nf[0] + 2 * G))
+    oracle.fill_two_levels(nf, ((CF, CF), (0, 0), (0, 0)), Uf, nc, c0, Uc)
+    # xi ghosts at interior j, k (periodic eta/zeta phases copy them further)
+    for gi, f in [(0, -4), (1, -3), (2, -2), (3, -1)]:
+        X = c0[0] + 0.5 * f
+        want = X * X + (0.25 if f % 2 else 0.0)
+        assert np.all(Uf[2, G:-G, G:-G, gi] == want + 2)
+
+
+@pytest.mark.parametrize("c0", [(2, 3, 1), (3, 2, 2)])
+def test_average_down_linear_exact_and_covered_set(c0):
+    nc = (12, 12, 10)
+    nf = (12, 10, 11)
+    bcf = ((CF, CF),) * 3
+    Xf, Yf, Zf = _pad_index(nf, c0, 0.5)
+    Uf = np.zeros((5, nf[2] + 2 * G, nf[1] + 2 * G, nf[0] + 2 * G))
+    for q in range(5):
+        Uf[q] = np.broadcast_to(1.0 + 2 * Xf - Yf + 3 * Zf + q * Xf * Xf * 0, Uf[q].shape)
+    Uf[3] = np.broadcast_to(Xf * Xf + Yf * Yf + Zf * Zf, Uf[3].shape)
+    Uc = np.full((5, nc[2] + 2 * G, nc[1] + 2 * G, nc[0] + 2 * G), -99.0)
+    oracle.average_down(nf, bcf, Uf, nc, c0, Uc)
+    X, Y, Z = _pad_index(nc, (0, 0, 0))
+    cov = np.zeros(Uc.shape[1:], bool)
+    rng = [range(c0[d] + 1, c0[d] + (nf[d] - 2) // 2 + 1) for d in range(3)]
+    for k in rng[2]:
+        for j in rng[1]:
+            for i in rng[0]:
+                cov[k + G, j + G, i + G] = True
+    assert cov.sum() == np.prod([len(r) for r in rng]) > 0
+    lin = np.broadcast_to(1.0 + 2 * X - Y + 3 * Z, cov.shape)
+    assert np.array_equal(Uc[0][cov], lin[cov])
+    quad = np.broadcast_to(X * X + Y * Y + Z * Z + 3.0 / 8.0, cov.shape)   # trapezoid: +1/8 per direction
+    assert np.array_equal(Uc[3][cov], quad[cov])
+    assert np.all(Uc[:, ~cov] == -99.0)
+
+
+def test_average_down_periodic_conservation():
+    nc = (8, 6, 10)
+    nf = tuple(2 * x for x in nc)
+    rng = np.random.default_rng(11)
+    Uf = synth.pad_state(rng.uniform(0.5, 1.5, (5, nf[2], nf[1], nf[0])))
+    Uc = np.zeros((5, nc[2] + 2 * G, nc[1] + 2 * G, nc[0] + 2 * G))
+    oracle.average_down(nf, PER, Uf, nc, (0, 0, 0), Uc)
+    ci = Uc[:, G:-G, G:-G, G:-G]
+    fi = Uf[:, G:-G, G:-G, G:-G]
+    assert np.all(ci != 0.0)                                      # every coarse node covered
+    np.testing.assert_allclose(ci.sum(axis=(1, 2, 3)), fi.sum(axis=(1, 2, 3)) / 8.0, rtol=1e-13)
+    # the coarse node coincident with fine node (2, 4, 6): explicit 27-point average
+    i, j, k = 1, 2, 3
+    w = np.array([0.25, 0.5, 0.25])
+    blk = Uf[:, G + 2 * k - 1:G + 2 * k + 2, G + 2 * j - 1:G + 2 * j + 2, G + 2 * i - 1:G + 2 * i + 2]
+    want = np.einsum("qcba,c,b,a->q", blk, w, w, w)
+    np.testing.assert_allclose(Uc[:, G + k, G + j, G + i], want, rtol=1e-15)
+
+
+def _two_level(grid_c, nc, bcc, c0, nf, bcf, state_fn, ph):
+    xc = grid_c.coords(nc, (0, 0, 0), oracle.GC)
+    metc = oracle.metrics(nc, bcc, xc)
+    Uc = synth.pad_state(state_fn(xc))
+    gf = synth.Refined(grid_c, c0)
+    xf = gf.coords(nf, (0, 0, 0), oracle.GC)
+    metf = oracle.metrics(nf, bcf, xf)
+    Uf = synth.pad_state(state_fn(xf))
+    return xc, metc, Uc, xf, metf, Uf
+
+
+def test_two_level_free_stream_preserved():
+    nc = (16, 16, 16)
+    grid = synth.Wavy3D(L=(10.0,) * 3, N=nc)
+    c0 = (4, 5, 3)
+    nf = (14, 12, 16)
+    bcf = ((CF, CF),) * 3
+    ph = oracle.phys(terms=3, mu_ref=0.01)
+    xc, metc, Uc, xf, metf, Uf = _two_level(grid, nc, PER, c0, nf, bcf, synth.free_stream, ph)
+    U0 = synth.free_stream(xc)[:, 0, 0, 0]
+    oracle.amr_advance(nc, PER, nf, bcf, c0, ph, 0.02, 2, Uc, metc, Uf, metf)
+    for U in (Uc, Uf):
+        dev = np.abs(U[:, G:-G, G:-G, G:-G] - U0[:, None, None, None]).max(axis=(1, 2, 3))
+        assert np.all(dev <= 1e-12 * np.abs(U0).max()), dev
+
+
+def test_two_level_full_cover_reduces_to_single_level():
+    """Fine level = the whole periodic domain: no C/F faces, so its evolution is the
+    single-level advance of the fine grid bit for bit, and the coarse level ends as the
+    full-weighting average of the fine state."""
+    nc = (8, 8, 6)
+    nf = tuple(2 * x for x in nc)
+    grid = synth.Wavy3D(L=(10.0,) * 3, N=nc)
+    ph = oracle.phys(terms=3, mu_ref=0.02)
+    st = lambda x: synth.vortex(x)
+    xc, metc, Uc, xf, metf, Uf = _two_level(grid, nc, PER, (0, 0, 0), nf, PER, st, ph)
+    Uf1 = Uf.copy()
+    oracle.amr_advance(nc, PER, nf, PER, (0, 0, 0), ph, 0.01, 2, Uc, metc, Uf, metf)
+    oracle.advance(nf, PER, ph, 0.01, 2, Uf1, metf)
+    assert np.array_equal(Uf[:, G:-G, G:-G, G:-G], Uf1[:, G:-G, G:-G, G:-G])
+    Uc2 = np.zeros_like(Uc)
+    oracle.average_down(nf, PER, Uf1, nc, (0, 0, 0), Uc2)
+    assert np.array_equal(Uc[:, G:-G, G:-G, G:-G], Uc2[:, G:-G, G:-G, G:-G])
+
+
+def test_two_level_vortex_more_accurate_on_fine_patch():
+    """Shu vortex (quasi-2D wavy grid, periodic) advected to t = 1 with a fine patch around its
+    path: the fine-level error against the translated closed form is well below the error of
+    the same coarse grid run without refinement, at the same (coincident) points."""
+    nc = (32, 32, 4)
+    grid = synth.Wavy2D(N=nc)
+    c0 = (8, 8, 0)
+    nf = (34, 34, 8)
+    bcf = ((CF, CF), (CF, CF), (0, 0))
+    ph = oracle.phys(terms=1)
+    dt, nsteps = 0.025, 40
+    st = lambda x: synth.vortex(x)
+    xc, metc, Uc, xf, metf, Uf = _two_level(grid, nc, PER, c0, nf, bcf, st, ph)
+    Uc1 = Uc.copy()
+    oracle.amr_advance(nc, PER, nf, bcf, c0, ph, dt, nsteps, Uc, metc, Uf, metf)
+    oracle.fill(nc, PER, Uc1)
+    oracle.advance(nc, PER, ph, dt, nsteps, Uc1, metc)
+    t = dt * nsteps
+    fi = range(2, nf[0] - 2, 2)                       # even fine interior nodes away from the C/F faces
+    fj = range(2, nf[1] - 2, 2)
+    ci = slice(c0[0] + fi[0] // 2, c0[0] + fi[-1] // 2 + 1)   # the coincident coarse nodes
+    cj = slice(c0[1] + fj[0] // 2, c0[1] + fj[-1] // 2 + 1)
+    fsl = (0, slice(None, None, 2), slice(fj[0], fj[-1] + 1, 2), slice(fi[0], fi[-1] + 1, 2))
+    csl = (0, slice(None), cj, ci)
+    exf = synth.vortex(xf, t=t)
+    exc = synth.vortex(xc, t=t)
+    err_fine = np.abs(Uf[:, G:-G, G:-G, G:-G][fsl] - exf[fsl]).max()
+    err_coarse = np.abs(Uc1[:, G:-G, G:-G, G:-G][csl] - exc[csl]).max()
+    err_comp = np.abs(Uc[:, G:-G, G:-G, G:-G][csl] - exc[csl]).max()
+    assert exf[fsl].shape == exc[csl].shape
+    assert err_fine < 0.5 * err_coarse, (err_fine, err_coarse)
+    assert err_comp < err_coarse, (err_comp, err_coarse)
