@@ -70,8 +70,12 @@ enum {
     CROCCO_BC_SLIPWALL = 4,  /* inviscid reflecting wall (DMR; reading 19): mirror, the
                                 momentum reflected about the plane normal to n = m^d/|m^d| of the
                                 mirrored point (needs the metrics in the fill) */
-    CROCCO_BC_SPLIT = 5      /* boundary data switching at a moving index (DMR bottom/top, reading 20):
+    CROCCO_BC_SPLIT = 5,     /* boundary data switching at a moving index (DMR bottom/top, reading 20):
                                 see crocco_split; the right part may be DIRICHLET or SLIPWALL */
+    CROCCO_BC_COARSE_FINE = 6 /* face of a fine AMR level inside the coarse domain (SURVEY NEXT-4,
+                                readings 24-25): its ghosts are interpolated from the coarse level by
+                                crocco_fill_patch_two_levels / crocco_amr_rk_stage; crocco_fill_boundary
+                                leaves them untouched, crocco_rk_stage / rk3_step refuse the ctx */
 };
 enum { CROCCO_TERM_INVISCID = 1, CROCCO_TERM_VISCOUS = 2 }; /* bitmask (Alg. 2 l.5-7 / l.8) */
 enum { CROCCO_MU_CONST = 0, CROCCO_MU_SUTHERLAND = 1 };
@@ -220,6 +224,41 @@ crocco_status crocco_rk_update(crocco_ctx ctx, int32_t stage, double dt, double 
    pointer.  Synchronises the stream.  Collective. */
 crocco_status crocco_compute_dt(crocco_ctx ctx, double *const *U, double *const *metrics,
                                 double cfl, double *dt);
+
+/* ---- two-level block-structured AMR (PAPER.md:56, 75, 83, 102-119,
+   129, 141, 258; readings 24-26) --------------------------------------------
+   A fine level is its own ctx (crocco_init_grid over the fine region, any equal-block
+   decomposition) whose faces inside the coarse domain are CROCCO_BC_COARSE_FINE.  Refinement
+   ratio 2, node-centred: fine node f (fine-level global index) lies at coarse index c0 + f/2.
+   All levels take the same dt; per RK stage the coarse level runs first (Alg. 2 l.2 level loop
+   inside the stage loop), then the fine level with its C/F ghosts interpolated from the coarse
+   stage INPUT, then at stage 2 (the third) AverageDown.  Both ctx must enqueue on the same
+   stream (or the caller orders them).  No inter-level communication: every coarse block a fine
+   block reads (and every fine block a covered coarse node reads) must be local to the rank. */
+
+/* Declare `fine` a refinement of `coarse` with fine node 0 at coarse node c0[3].  Checks:
+   per direction either the fine level is PERIODIC and spans the periodic coarse domain
+   (N_f = 2 N_c, c0 = 0), or 0 <= c0 and 2 c0 + N_f - 1 <= 2 (N_c - 1) with physical (non-C/F)
+   faces only on the domain boundary; <= 64 local / 512 blocks per level; locality as above.
+   CROCCO_ERR_ARG otherwise.  The ctx keep no reference beyond the pair (finalize the fine
+   level first or relink). */
+crocco_status crocco_amr_link(crocco_ctx fine, crocco_ctx coarse, const int64_t c0[3]);
+/* FillPatch of the fine level (FillPatchTwoLevels + BC_Fill; reading 25):
+   the 3-phase fill of U_fine in place, COARSE_FINE ghosts = trilinear interpolation from the
+   coarse state U_coarse (one device pointer per coarse local block; its ghosts must be filled,
+   e.g. by the coarse level's own fill of this stage).  metrics_fine as crocco_fill_boundary.
+   Collective over the fine level. */
+crocco_status crocco_fill_patch_two_levels(crocco_ctx fine, double *const *U_fine,
+                                           double *const *metrics_fine, double *const *U_coarse);
+/* crocco_rk_stage of the fine level with its C/F ghosts interpolated from U_coarse_in, the
+   coarse level's input state of the same stage (ghosts filled). */
+crocco_status crocco_amr_rk_stage(crocco_ctx fine, int32_t stage, double dt, double *const *U_in,
+                                  double *const *U_out, double *const *dU, double *const *metrics,
+                                  double *const *U_coarse_in);
+/* AverageDown (Alg. 2 l.10-12; reading 26): refills the same-level ghosts of U_fine
+   (periodic / inter-block copies only), then every covered coarse node of U_coarse (interior
+   points only) becomes the full-weighting (trapezoid) average of the fine data over its cell. */
+crocco_status crocco_average_down(crocco_ctx fine, double *const *U_fine, double *const *U_coarse);
 
 /* Block until all work of the ctx finished; surfaces asynchronous errors. */
 crocco_status crocco_sync(crocco_ctx ctx);

@@ -934,14 +934,15 @@ void oracle_fill_two_levels(const int64_t nf[3], const int32_t bcf[6], const dou
    2(I - c0) - 1 .. 2(I - c0) + 1 are fine interior nodes.  Its new value is the average of
    the fine data over its cell [I - 1/2, I + 1/2]^3 by the trapezoid rule on the fine nodes:
    U_c(I) = sum_{c,b,a in {-1,0,1}} w_a w_b w_c U_f(2(I - c0) + (a, b, c)), w_0 = 1/2,
-   w_{+-1} = 1/4 (sum order: c outer, a inner).  The fine ghosts are first refilled in place
-   (same-level periodic / inter-block copies and physical BCs; C/F ghosts are not read). */
+   w_{+-1} = 1/4 (sum order: c outer, a inner).  The fine ghosts are first refilled in place by
+   the same-level periodic copies only (the METRIC kind of fill_core skips every non-periodic
+   face): physical and C/F ghosts are never read by a covered node. */
 void oracle_average_down(const int64_t nf[3], const int32_t bcf[6], const double dirichlet[30],
                          double *Uf, const int64_t nc[3], const int64_t c0[3], double *Uc)
 {
     static const double wt[3] = {0.25, 0.5, 0.25};
     obox fb = make_box(nf, OG), cb = make_box(nc, OG);
-    fill_core(nf, bcf, dirichlet, NULL, 0.0, NULL, Uf, 5, O_FIELD_STATE, NULL);
+    fill_core(nf, bcf, dirichlet, NULL, 0.0, NULL, Uf, 5, O_FIELD_METRIC, NULL);
     for (int64_t k = 0; k < nc[2]; k++)
         for (int64_t j = 0; j < nc[1]; j++)
             for (int64_t i = 0; i < nc[0]; i++) {

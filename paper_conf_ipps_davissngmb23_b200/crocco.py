@@ -14,7 +14,7 @@ HERE = os.path.dirname(os.path.abspath(__file__))
 LIB_PATH = os.environ.get("CROCCO_LIB") or os.path.join(HERE, "libcrocco.so")  # env: variant builds (tools/)
 
 CROCCO_OK, CROCCO_ERR_ARG, CROCCO_ERR_CUDA, CROCCO_ERR_NCCL, CROCCO_ERR_NOMEM, CROCCO_ERR_STATE = range(6)
-BC_PERIODIC, BC_EXTRAP, BC_DIRICHLET, BC_WALL, BC_SLIPWALL, BC_SPLIT = 0, 1, 2, 3, 4, 5
+BC_PERIODIC, BC_EXTRAP, BC_DIRICHLET, BC_WALL, BC_SLIPWALL, BC_SPLIT, BC_COARSE_FINE = 0, 1, 2, 3, 4, 5, 6
 TERM_INVISCID, TERM_VISCOUS = 1, 2
 MU_CONST, MU_SUTHERLAND = 0, 1
 FIELD_STATE, FIELD_METRIC = 0, 1
@@ -92,6 +92,10 @@ _SIGS = {
     "crocco_nccl_unique_id": [C.c_void_p, C.c_int32],
     "crocco_compute_dt": [C.c_void_p, DPP, DPP, C.c_double, C.POINTER(C.c_double)],
     "crocco_rk3_step": [C.c_void_p, C.c_double, DPP, DPP, DPP, DPP, C.c_int32],
+    "crocco_amr_link": [C.c_void_p, C.c_void_p, C.POINTER(C.c_int64)],
+    "crocco_fill_patch_two_levels": [C.c_void_p, DPP, DPP, DPP],
+    "crocco_amr_rk_stage": [C.c_void_p, C.c_int32, C.c_double, DPP, DPP, DPP, DPP, DPP],
+    "crocco_average_down": [C.c_void_p, DPP, DPP],
 }
 _STR = {"crocco_last_error": [C.c_void_p], "crocco_version": [],
         "crocco_kernel_class_name": [C.c_int32]}
@@ -315,3 +319,31 @@ def crocco_rk3_step(ctx, dt, U_ptrs, V_ptrs, dU_ptrs, met_ptrs, use_graph=True):
     c, kc = _ptrs(dU_ptrs)
     d, kd = _ptrs(met_ptrs)
     _check(lib().crocco_rk3_step(ctx, float(dt), a, b, c, d, int(use_graph)), ctx)
+
+
+# ---- two-level AMR (include/crocco.h) ----
+def crocco_amr_link(fine, coarse, c0):
+    arr = (C.c_int64 * 3)(*[int(x) for x in c0])
+    _check(lib().crocco_amr_link(fine, coarse, arr), fine)
+
+
+def crocco_fill_patch_two_levels(fine, Uf_ptrs, metf_ptrs, Uc_ptrs):
+    a, ka = _ptrs(Uf_ptrs)
+    b, kb = _ptrs(metf_ptrs) if metf_ptrs is not None else (None, None)
+    c, kc = _ptrs(Uc_ptrs)
+    _check(lib().crocco_fill_patch_two_levels(fine, a, b, c), fine)
+
+
+def crocco_amr_rk_stage(fine, stage, dt, Uin_ptrs, Uout_ptrs, dU_ptrs, met_ptrs, Uc_in_ptrs):
+    a, ka = _ptrs(Uin_ptrs)
+    b, kb = _ptrs(Uout_ptrs)
+    c, kc = _ptrs(dU_ptrs)
+    d, kd = _ptrs(met_ptrs)
+    e, ke = _ptrs(Uc_in_ptrs)
+    _check(lib().crocco_amr_rk_stage(fine, stage, dt, a, b, c, d, e), fine)
+
+
+def crocco_average_down(fine, Uf_ptrs, Uc_ptrs):
+    a, ka = _ptrs(Uf_ptrs)
+    b, kb = _ptrs(Uc_ptrs)
+    _check(lib().crocco_average_down(fine, a, b), fine)

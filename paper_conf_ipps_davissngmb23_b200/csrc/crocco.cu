@@ -15,6 +15,7 @@
 #include <vector>
 
 #include "../../include/crocco.h"
+#include "amr.cuh"
 #include "fill.cuh"
 #include "metrics.cuh"
 #include "pointwise.cuh"
@@ -46,10 +47,12 @@ struct LocalBlock {
     double *rv = nullptr;    // viscous D4_zeta term (CROCCO_ZDIV_SWEEP != 0)
 };
 
-enum { K_PRIMS = 0, K_FLUX_X, K_FLUX_Y, K_FLUX_Z, K_VISC, K_UPDATE, K_FILL, K_METRICS, K_CFL,
+enum { K_PRIMS = 0, K_FLUX_X, K_FLUX_Y, K_FLUX_Z, K_VISC, K_UPDATE, K_FILL, K_METRICS, K_CFL, K_AMR,
        K_NCLASS };
 const char *k_names[K_NCLASS] = {"prims", "sweep_xi", "sweep_eta", "sweep_zeta_update", "viscous",
-                                 "update", "fill", "metrics", "compute_dt"};
+                                 "update", "fill", "metrics", "compute_dt", "amr"};
+// internal fill kind: 5-component state, periodic / inter-block copies only (AverageDown)
+enum { FILL_STATE_COPIES = 100 };
 
 struct TimedLaunch {
     int cls;
@@ -93,6 +96,11 @@ struct crocco_ctx_s {
     cudaStream_t comm_stream = nullptr;
     cudaEvent_t ev_fork = nullptr, ev_join = nullptr;
     double time = 0.0;  // start of the current step (time-dependent SPLIT faces)
+    // two-level AMR (NEXT-4): this ctx as the fine level of `amr_coarse`
+    bool has_cf = false;                 // some face is CROCCO_BC_COARSE_FINE
+    crocco_ctx amr_coarse = nullptr;     // set by crocco_amr_link
+    int64_t amr_c0[3] = {0, 0, 0};       // coarse index of fine node 0
+    double *const *amr_Uc = nullptr;     // coarse state of the current two-level call only
     int64_t stage_elems = 0;
     // timing
     bool timing = false;
@@ -211,7 +219,7 @@ static crocco_status validate(const crocco_grid_desc *d, int nb[3], int bn[3]) {
         if (b > 65535) return fail(nullptr, CROCCO_ERR_ARG, "block interior > 65535 points in direction %d", a);
         bn[a] = (int)b;
         for (int s = 0; s < 2; s++)
-            if (d->bc[a][s] < 0 || d->bc[a][s] > 5)
+            if (d->bc[a][s] < 0 || d->bc[a][s] > CROCCO_BC_COARSE_FINE)
                 return fail(nullptr, CROCCO_ERR_ARG, "bad bc kind %d", d->bc[a][s]);
         for (int s = 0; s < 2; s++)
             if (d->bc[a][s] == CROCCO_BC_SPLIT) {
@@ -478,6 +486,8 @@ crocco_status crocco_init_grid(const crocco_grid_desc *desc, const crocco_phys *
     c->desc.block_rank = c->block_rank.data();
     c->phys_in = *phys;
     c->ph = to_phys(phys);
+    for (int d = 0; d < 3; d++)
+        for (int sd = 0; sd < 2; sd++) c->has_cf = c->has_cf || desc->bc[d][sd] == CROCCO_BC_COARSE_FINE;
     c->stream = (cudaStream_t)desc->stream;
     for (int a = 0; a < 3; a++) {
         c->nb[a] = nb[a];
@@ -633,11 +643,47 @@ static void op_strides(const Lay &L, int64_t st[3]) {
     st[2] = L.pz;
 }
 
+static crocco_status flush_cf(crocco_ctx c, CFOps &cf, const LevelTab &ct) {
+    if (cf.nops == 0) return CROCCO_OK;
+    int64_t mx = 0;
+    for (int i = 0; i < cf.nops; i++)
+        mx = std::max(mx, (int64_t)cf.op[i].ext[0] * cf.op[i].ext[1] * cf.op[i].ext[2]);
+    dim3 grid(std::min<int64_t>(cdiv(mx, 256), 4096), cf.nops);
+    LAUNCH(c, K_AMR, k_cf_interp<<<grid, 256, 0, c->stream>>>(cf, ct));
+    cf.nops = 0;
+    return CROCCO_OK;
+}
+
+// table of one level's local blocks for the AMR kernels
+static void level_tab(const crocco_ctx_s *lv, double *const *ptr, LevelTab &t) {
+    memset(&t, 0, sizeof t);
+    for (size_t b = 0; b < lv->loc.size(); b++) t.p[b] = ptr[b];
+    for (int g = 0; g < AMR_MAX_BLOCKS; g++)
+        t.g2l[g] = g < (int)lv->gid_to_local.size() ? (int16_t)lv->gid_to_local[g] : (int16_t)-1;
+    t.L = lv->loc[0].L;
+    for (int d = 0; d < 3; d++) {
+        t.bn[d] = lv->bn[d];
+        t.nb[d] = lv->nb[d];
+        t.N[d] = lv->desc.n_global[d];
+    }
+}
+
 static crocco_status fill_phase(crocco_ctx c, double *const *f, int kind, int D,
                                 double *const *met, double t) {
+    const bool copies_only = kind == FILL_STATE_COPIES;
+    if (copies_only) kind = CROCCO_FIELD_STATE;
     const int ncomp = kind == CROCCO_FIELD_STATE ? 5 : 10;
     BoxOps ops;
     ops.nops = 0;
+    CFOps cf;
+    cf.nops = 0;
+    LevelTab ct;
+    const bool interp = kind == CROCCO_FIELD_STATE && !copies_only && c->amr_Uc && c->amr_coarse;
+    if (interp) {
+        level_tab(c->amr_coarse, c->amr_Uc, ct);
+        cf.Lf = c->loc.empty() ? Lay{} : c->loc[0].L;
+        for (int e = 0; e < 3; e++) cf.c0[e] = c->amr_c0[e];
+    }
     std::vector<const crocco_msg *> remote;
     for (const crocco_msg &m : c->plan[D]) {
         if (m.kind == 0 && (m.src_rank != m.dst_rank)) {
@@ -664,8 +710,24 @@ static crocco_status fill_phase(crocco_ctx c, double *const *f, int kind, int D,
             o.sbase = at(sb.L, (int)m.src_lo[0], (int)m.src_lo[1], (int)m.src_lo[2]);
             o.mode = BOX_COPY;
         } else {
-            if (kind == CROCCO_FIELD_METRIC) continue;  // physical faces keep computed metrics
+            if (kind == CROCCO_FIELD_METRIC || copies_only) continue;  // physical faces keep computed metrics
             const int bc = m.bc_kind;
+            if (bc == CROCCO_BC_COARSE_FINE) {  // FillPatchTwoLevels (reading 25); untouched without a coarse level
+                if (!interp) continue;
+                CFOp q;
+                q.dst = f[dl];
+                q.dbase = o.dbase;
+                for (int e = 0; e < 3; e++) {
+                    q.ext[e] = o.ext[e];
+                    q.fo[e] = db.g.origin[e] + m.dst_lo[e];
+                }
+                cf.op[cf.nops++] = q;
+                if (cf.nops == CF_MAX_OPS) {
+                    crocco_status s2 = flush_cf(c, cf, ct);
+                    if (s2) return s2;
+                }
+                continue;
+            }
             const int n = db.g.n[D];
             int64_t st[3];
             op_strides(db.L, st);
@@ -708,6 +770,7 @@ static crocco_status fill_phase(crocco_ctx c, double *const *f, int kind, int D,
     }
     crocco_status st = flush_ops(c, ops);
     if (st) return st;
+    if (interp && (st = flush_cf(c, cf, ct))) return st;
     if (remote.empty()) return CROCCO_OK;
     if (!c->comm) return fail(c, CROCCO_ERR_STATE, "remote halo without communicator");
     // pack sends
@@ -789,7 +852,7 @@ static crocco_status check_ptrs(crocco_ctx c, double *const *p, const char *what
 }
 
 static crocco_status fill_all(crocco_ctx c, double *const *f, int32_t kind, double *const *met, double t) {
-    if (kind != CROCCO_FIELD_STATE && kind != CROCCO_FIELD_METRIC)
+    if (kind != CROCCO_FIELD_STATE && kind != CROCCO_FIELD_METRIC && kind != FILL_STATE_COPIES)
         return fail(c, CROCCO_ERR_ARG, "bad field kind");
     crocco_status st = check_ptrs(c, f, "field");
     if (st) return st;
@@ -802,6 +865,7 @@ static crocco_status fill_all(crocco_ctx c, double *const *f, int32_t kind, doub
 
 crocco_status crocco_fill_boundary(crocco_ctx c, double *const *f, int32_t kind, double *const *met) {
     LIVE(c);
+    if (kind != CROCCO_FIELD_STATE && kind != CROCCO_FIELD_METRIC) return fail(c, CROCCO_ERR_ARG, "bad field kind");
     return fill_all(c, f, kind, met, c->time);
 }
 
@@ -991,6 +1055,8 @@ crocco_status crocco_rk_stage(crocco_ctx c, int32_t stage, double dt, double *co
     for (size_t bi = 0; bi < c->loc.size(); bi++)
         if (Uin[bi] == Uout[bi] || dU[bi] == Uin[bi] || dU[bi] == Uout[bi])
             return fail(c, CROCCO_ERR_ARG, "U_in, U_out and dU must be distinct");
+    if (c->has_cf && !c->amr_Uc)
+        return fail(c, CROCCO_ERR_ARG, "COARSE_FINE faces need the coarse level: use crocco_amr_rk_stage");
     const double ts = c->time + RK_C[stage] * dt;
     const bool ov = c->overlap < 0 ? c->desc.nranks > 1 : c->overlap != 0;
     if (!(ov && visc_overlap_possible(c))) {
@@ -1046,6 +1112,8 @@ crocco_status crocco_rk3_step(crocco_ctx c, double dt, double *const *U, double 
     if ((st = check_ptrs(c, U, "U")) || (st = check_ptrs(c, V, "V")) || (st = check_ptrs(c, dU, "dU")) ||
         (st = check_ptrs(c, M, "metrics")))
         return st;
+    if (c->has_cf)
+        return fail(c, CROCCO_ERR_ARG, "COARSE_FINE faces: step the hierarchy with crocco_amr_rk_stage");
     bool moving = false;
     for (int d = 0; d < 3; d++)
         for (int sd = 0; sd < 2; sd++)
@@ -1142,6 +1210,173 @@ crocco_status crocco_compute_dt(crocco_ctx c, double *const *U, double *const *M
     if (!(lam > 0)) return fail(c, CROCCO_ERR_ARG, "non-positive spectral radius (state not set?)");
     *dt = cfl / lam;
     return CROCCO_OK;
+}
+
+// ---------------------------------------------------------------------------
+// two-level AMR (readings 24-26)
+// ---------------------------------------------------------------------------
+static int64_t floor_half_h(int64_t h) { return h >= 0 ? h / 2 : -((-h + 1) / 2); }
+
+// coarse nodes I in [lo, hi] along d of the covered set (reading 26); empty when lo > hi
+static void covered_range(const crocco_ctx_s *f, int d, int64_t &lo, int64_t &hi) {
+    const int64_t nf = f->desc.n_global[d], c0 = f->amr_c0[d];
+    if (f->desc.bc[d][0] == CROCCO_BC_PERIODIC) {
+        lo = 0;
+        hi = nf / 2 - 1;
+    } else {
+        lo = c0 + 1;
+        hi = c0 + (nf - 2) / 2;
+    }
+}
+
+crocco_status crocco_amr_link(crocco_ctx f, crocco_ctx c, const int64_t c0[3]) {
+    LIVE(f);
+    LIVE(c);
+    if (!c0 || f == c) return fail(f, CROCCO_ERR_ARG, "need distinct fine / coarse ctx and c0");
+    if (f->desc.nranks != c->desc.nranks || f->desc.rank != c->desc.rank)
+        return fail(f, CROCCO_ERR_ARG, "fine and coarse levels must share the process group");
+    if (f->loc.size() > AMR_MAX_LOCAL || c->loc.size() > AMR_MAX_LOCAL || f->all.size() > AMR_MAX_BLOCKS ||
+        c->all.size() > AMR_MAX_BLOCKS)
+        return fail(f, CROCCO_ERR_ARG, "two-level AMR: at most %d local / %d blocks per level", AMR_MAX_LOCAL,
+                    AMR_MAX_BLOCKS);
+    for (int d = 0; d < 3; d++) {
+        const int64_t nf = f->desc.n_global[d], nc = c->desc.n_global[d];
+        const int *bf = f->desc.bc[d], *bcc = c->desc.bc[d];
+        if (bf[0] == CROCCO_BC_PERIODIC) {
+            if (bcc[0] != CROCCO_BC_PERIODIC || nf != 2 * nc || c0[d] != 0)
+                return fail(f, CROCCO_ERR_ARG,
+                            "direction %d: a PERIODIC fine level must span the periodic coarse domain "
+                            "(N_f = 2 N_c, c0 = 0)", d);
+            continue;
+        }
+        if (c0[d] < 0 || 2 * c0[d] + nf - 1 > 2 * (nc - 1))
+            return fail(f, CROCCO_ERR_ARG, "direction %d: fine level outside the coarse domain", d);
+        if (bf[0] != CROCCO_BC_COARSE_FINE && c0[d] != 0)
+            return fail(f, CROCCO_ERR_ARG, "direction %d: a physical lo face must lie on the domain boundary", d);
+        if (bf[1] != CROCCO_BC_COARSE_FINE && 2 * c0[d] + nf - 1 != 2 * (nc - 1))
+            return fail(f, CROCCO_ERR_ARG, "direction %d: a physical hi face must lie on the domain boundary", d);
+        if (nf < 3) return fail(f, CROCCO_ERR_ARG, "direction %d: fine level needs >= 3 points", d);
+    }
+    for (int d = 0; d < 3; d++) f->amr_c0[d] = c0[d];
+    // locality: every coarse block a fine ghost interpolates from, and every fine block a
+    // covered coarse node averages, lives on this rank (no inter-level communication)
+    for (const LocalBlock &b : f->loc) {
+        int64_t lo[3], hi[3];
+        for (int d = 0; d < 3; d++) {
+            lo[d] = floor_half_h(2 * c0[d] + b.g.origin[d] - G);
+            hi[d] = floor_half_h(2 * c0[d] + b.g.origin[d] + b.g.n[d] + G - 1);
+            lo[d] = std::min<int64_t>(std::max<int64_t>(lo[d], 0), c->desc.n_global[d] - 1) / c->bn[d];
+            hi[d] = std::min<int64_t>(std::max<int64_t>(hi[d], 0), c->desc.n_global[d] - 1) / c->bn[d];
+        }
+        for (int64_t z = lo[2]; z <= hi[2]; z++)
+            for (int64_t y = lo[1]; y <= hi[1]; y++)
+                for (int64_t x = lo[0]; x <= hi[0]; x++)
+                    if (c->gid_to_local[x + c->nb[0] * (y + c->nb[1] * z)] < 0)
+                        return fail(f, CROCCO_ERR_ARG,
+                                    "fine block %d interpolates from a coarse block on another rank", b.g.gid);
+    }
+    for (const LocalBlock &b : c->loc) {
+        int64_t lo[3], hi[3];
+        bool empty = false;
+        for (int d = 0; d < 3; d++) {
+            covered_range(f, d, lo[d], hi[d]);
+            lo[d] = std::max<int64_t>(lo[d], b.g.origin[d]);
+            hi[d] = std::min<int64_t>(hi[d], b.g.origin[d] + b.g.n[d] - 1);
+            empty = empty || lo[d] > hi[d];
+            if (!empty) {
+                lo[d] = 2 * (lo[d] - c0[d]) / f->bn[d];
+                hi[d] = 2 * (hi[d] - c0[d]) / f->bn[d];
+            }
+        }
+        if (empty) continue;
+        for (int64_t z = lo[2]; z <= hi[2]; z++)
+            for (int64_t y = lo[1]; y <= hi[1]; y++)
+                for (int64_t x = lo[0]; x <= hi[0]; x++)
+                    if (f->gid_to_local[x + f->nb[0] * (y + f->nb[1] * z)] < 0)
+                        return fail(f, CROCCO_ERR_ARG,
+                                    "coarse block %d averages down from a fine block on another rank", b.g.gid);
+    }
+    f->amr_coarse = c;
+    return CROCCO_OK;
+}
+
+static crocco_status amr_ready(crocco_ctx f, double *const *Uc) {
+    if (!f->amr_coarse) return fail(f, CROCCO_ERR_ARG, "fine level not linked (crocco_amr_link)");
+    if (f->amr_coarse->poisoned) return CROCCO_ERR_STATE;
+    if (!Uc) return fail(f, CROCCO_ERR_ARG, "null coarse pointer array");
+    for (size_t b = 0; b < f->amr_coarse->loc.size(); b++)
+        if (!Uc[b]) return fail(f, CROCCO_ERR_ARG, "null coarse pointer for local block %zu", b);
+    return CROCCO_OK;
+}
+
+crocco_status crocco_fill_patch_two_levels(crocco_ctx f, double *const *Uf, double *const *Mf,
+                                           double *const *Uc) {
+    LIVE(f);
+    crocco_status st = amr_ready(f, Uc);
+    if (st) return st;
+    f->amr_Uc = Uc;
+    st = fill_all(f, Uf, CROCCO_FIELD_STATE, Mf, f->time);
+    f->amr_Uc = nullptr;
+    return st;
+}
+
+crocco_status crocco_amr_rk_stage(crocco_ctx f, int32_t stage, double dt, double *const *Uin,
+                                  double *const *Uout, double *const *dU, double *const *M,
+                                  double *const *Uc_in) {
+    LIVE(f);
+    crocco_status st = amr_ready(f, Uc_in);
+    if (st) return st;
+    f->amr_Uc = Uc_in;
+    st = crocco_rk_stage(f, stage, dt, Uin, Uout, dU, M);
+    f->amr_Uc = nullptr;
+    return st;
+}
+
+crocco_status crocco_average_down(crocco_ctx f, double *const *Uf, double *const *Uc) {
+    LIVE(f);
+    crocco_status st = amr_ready(f, Uc);
+    if (st) return st;
+    if ((st = check_ptrs(f, Uf, "U_fine"))) return st;
+    // same-level ghosts of the fine state (copies only; C/F and physical ghosts are not read)
+    if ((st = fill_all(f, Uf, FILL_STATE_COPIES, nullptr, f->time))) return st;
+    const crocco_ctx_s *c = f->amr_coarse;
+    LevelTab ft;
+    level_tab(f, Uf, ft);
+    ADOps ops;
+    memset(&ops, 0, sizeof ops);
+    ops.Lc = c->loc.empty() ? Lay{} : c->loc[0].L;
+    for (int d = 0; d < 3; d++) ops.c0[d] = f->amr_c0[d];
+    int64_t mx = 0;
+    auto flush = [&]() -> crocco_status {
+        if (ops.nops == 0) return CROCCO_OK;
+        dim3 grid(std::min<int64_t>(cdiv(mx, 256), 4096), ops.nops);
+        LAUNCH(f, K_AMR, k_average_down<<<grid, 256, 0, f->stream>>>(ops, ft));
+        ops.nops = 0;
+        mx = 0;
+        return CROCCO_OK;
+    };
+    for (size_t bi = 0; bi < c->loc.size(); bi++) {
+        const LocalBlock &b = c->loc[bi];
+        int64_t lo[3], hi[3];
+        bool empty = false;
+        for (int d = 0; d < 3; d++) {
+            covered_range(f, d, lo[d], hi[d]);
+            lo[d] = std::max<int64_t>(lo[d], b.g.origin[d]);
+            hi[d] = std::min<int64_t>(hi[d], b.g.origin[d] + b.g.n[d] - 1);
+            empty = empty || lo[d] > hi[d];
+        }
+        if (empty) continue;
+        ADOp &o = ops.op[ops.nops++];
+        o.dst = Uc[bi];
+        o.dbase = at(b.L, (int)(lo[0] - b.g.origin[0]), (int)(lo[1] - b.g.origin[1]), (int)(lo[2] - b.g.origin[2]));
+        for (int d = 0; d < 3; d++) {
+            o.ext[d] = (int)(hi[d] - lo[d] + 1);
+            o.Io[d] = lo[d];
+        }
+        mx = std::max<int64_t>(mx, (int64_t)o.ext[0] * o.ext[1] * o.ext[2]);
+        if (ops.nops == CF_MAX_OPS && (st = flush())) return st;
+    }
+    return flush();
 }
 
 crocco_status crocco_sync(crocco_ctx c) {

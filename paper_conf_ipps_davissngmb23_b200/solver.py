@@ -194,3 +194,44 @@ class Solver:
             self.close()
         except Exception:
             pass
+
+
+class AmrSolver:
+    """Two-level hierarchy (DESIGN readings 24-26): a coarse Solver and a fine
+    Solver whose faces inside the coarse domain are BC_COARSE_FINE, fine node 0 at coarse node
+    c0 (ratio 2, node-centred).  step() follows Algorithm 2: per stage the
+    coarse level, then the fine level with its C/F ghosts interpolated from the coarse stage
+    input, then AverageDown at the third stage.  Plumbing only -- the C ABI does every step."""
+
+    def __init__(self, coarse: Solver, fine: Solver, c0):
+        self.coarse, self.fine, self.c0 = coarse, fine, tuple(int(x) for x in c0)
+        cc.crocco_amr_link(fine.ctx, coarse.ctx, self.c0)
+
+    def fill_fine(self):
+        """FillPatchTwoLevels of the current fine state from the current coarse state."""
+        cc.crocco_fill_patch_two_levels(self.fine.ctx, self.fine._ptrs(self.fine.U),
+                                        self.fine._ptrs(self.fine.met), self.coarse._ptrs(self.coarse.U))
+
+    def average_down(self):
+        cc.crocco_average_down(self.fine.ctx, self.fine._ptrs(self.fine.U), self.coarse._ptrs(self.coarse.U))
+
+    def stage(self, s, dt):
+        C, F = self.coarse, self.fine
+        Uc_in = C.U
+        C.stage(s, dt)                                   # fills Uc_in's ghosts, writes C.V; swaps
+        cc.crocco_amr_rk_stage(F.ctx, s, dt, F._ptrs(F.U), F._ptrs(F.V), F._ptrs(F.dU), F._ptrs(F.met),
+                               C._ptrs(Uc_in))
+        F.U, F.V = F.V, F.U
+        if s == 2:
+            self.average_down()
+
+    def step(self, dt, nsteps=1):
+        for _ in range(nsteps):
+            for s in range(3):
+                self.stage(s, dt)
+            self.coarse.set_time(self.coarse.time + dt)
+            self.fine.set_time(self.fine.time + dt)
+
+    def sync(self):
+        self.coarse.sync()
+        self.fine.sync()

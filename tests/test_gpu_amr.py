@@ -1,0 +1,182 @@
+"""GPU parity of the two-level AMR path (readings 24-26)
+through the C ABI against the oracle (oracle section 9) on the same seeded inputs:
+  FillPatchTwoLevels (C/F ghosts)   bitwise (dyadic weights, same corner order)
+  AverageDown                       bitwise (same 27-term order, exact products)
+  two-level RK3 steps               <= 1e-9 relative L_inf per component
+for single- and multi-block coarse and fine levels, plus the ABI's refusals.
+"""
+import numpy as np
+import pytest
+
+import oracle
+import synth
+from _harness import block_slices, rel_linf, state_scale
+
+pytestmark = pytest.mark.gpu
+
+G = 4
+CF = oracle.COARSE_FINE
+PER = ((0, 0),) * 3
+
+
+@pytest.fixture(autouse=True)
+def _need_gpu():
+    torch = pytest.importorskip("torch")
+    if not torch.cuda.is_available():
+        pytest.fail("GPU test run without a CUDA device")
+
+
+def _blocks_of(a_glob_padded, n, nb):
+    """Per-block padded views (ghost 4) cut out of a global padded array."""
+    bn, blocks = block_slices(n, nb)
+    out = []
+    for o, _ in blocks:
+        out.append(a_glob_padded[:, o[2]:o[2] + bn[2] + 2 * G, o[1]:o[1] + bn[1] + 2 * G,
+                                 o[0]:o[0] + bn[0] + 2 * G])
+    return bn, blocks, out
+
+
+class Hier:
+    """One two-level problem, built identically for the oracle (global single boxes) and the GPU
+    (any block decomposition of either level)."""
+
+    def __init__(self, nc, c0, nf, bcf, grid, phys_kw, seed=3, state="random"):
+        self.nc, self.c0, self.nf, self.bcf, self.grid = nc, c0, nf, bcf, grid
+        self.phys_kw = phys_kw
+        self.fgrid = synth.Refined(grid, c0)
+        if state == "random":
+            self.Uc0 = synth.random_state(nc, seed=seed, amp=0.2)
+            self.Uf0 = synth.random_state(nf, seed=seed + 1, amp=0.2)
+        else:
+            self.Uc0 = synth.vortex(grid.coords(nc, (0, 0, 0), oracle.GC))
+            self.Uf0 = synth.vortex(self.fgrid.coords(nf, (0, 0, 0), oracle.GC))
+
+    def oracle(self):
+        xc = self.grid.coords(self.nc, (0, 0, 0), oracle.GC)
+        xf = self.fgrid.coords(self.nf, (0, 0, 0), oracle.GC)
+        metc = oracle.metrics(self.nc, PER, xc)
+        metf = oracle.metrics(self.nf, self.bcf, xf)
+        Uc = synth.pad_state(self.Uc0)
+        Uf = synth.pad_state(self.Uf0)
+        oracle.fill(self.nc, PER, Uc)
+        return metc, Uc, metf, Uf
+
+    def gpu(self, nbc, nbf):
+        from paper_conf_ipps_davissngmb23_b200 import crocco as cc
+        from paper_conf_ipps_davissngmb23_b200.solver import AmrSolver, Solver
+        kw = dict(self.phys_kw)
+        C = Solver(self.nc, nbc, PER, cc.make_phys(**kw))
+        F = Solver(self.nf, nbf, self.bcf, cc.make_phys(**kw))
+        for S, n, nb, g, U0 in ((C, self.nc, nbc, self.grid, self.Uc0), (F, self.nf, nbf, self.fgrid, self.Uf0)):
+            bn, blocks = block_slices(n, nb)
+            S.set_coords([g.coords(bn, o, oracle.GC) for o, _ in blocks])
+            S.set_state([np.ascontiguousarray(U0[(slice(None),) + sl]) for _, sl in blocks])
+            S.blocks = blocks
+        C.fill()
+        return C, F, AmrSolver(C, F, self.c0)
+
+
+def _check_padded(S, bufs, ref_glob, n, nb, exact=True, tol=0.0, floor=0.0):
+    bn, blocks, refs = _blocks_of(ref_glob, n, nb)
+    got = S.get(bufs)
+    for g, r in zip(got, refs):
+        if exact:
+            assert np.array_equal(g, r)
+        else:
+            assert rel_linf(g[:, G:-G, G:-G, G:-G], r[:, G:-G, G:-G, G:-G], floor) <= tol
+
+
+@pytest.mark.parametrize("nbc,nbf", [((1, 1, 1), (1, 1, 1)), ((2, 2, 2), (2, 2, 1)), ((3, 1, 2), (1, 2, 3))])
+def test_fill_patch_two_levels_bitwise(nbc, nbf):
+    nc, c0, nf = (24, 20, 16), (3, 4, 2), (20, 16, 12)
+    h = Hier(nc, c0, nf, ((CF, CF),) * 3, synth.Wavy3D(L=(10.0,) * 3, N=nc), dict(terms=3, mu_ref=0.02))
+    metc, Uc, metf, Uf = h.oracle()
+    oracle.fill_two_levels(nf, h.bcf, Uf, nc, c0, Uc)
+    C, F, A = h.gpu(nbc, nbf)
+    A.fill_fine()
+    _check_padded(F, F.U, Uf, nf, nbf)                    # interior, inter-block and C/F ghosts
+    C.close()
+    F.close()
+
+
+def test_fill_patch_two_levels_mixed_faces_bitwise():
+    """Fine level spanning the periodic zeta direction (PERIODIC) and touching the xi-lo domain
+    boundary (EXTRAP there), C/F elsewhere."""
+    nc, c0 = (20, 16, 8), (0, 3, 0)
+    nf = (24, 16, 16)
+    bcf = ((1, CF), (CF, CF), (0, 0))
+    h = Hier(nc, c0, nf, bcf, synth.Wavy3D(L=(10.0,) * 3, N=nc), dict(terms=3, mu_ref=0.02))
+    metc, Uc, metf, Uf = h.oracle()
+    oracle.fill_two_levels(nf, bcf, Uf, nc, c0, Uc)
+    C, F, A = h.gpu((2, 2, 2), (2, 2, 2))
+    A.fill_fine()
+    _check_padded(F, F.U, Uf, nf, (2, 2, 2))
+    C.close()
+    F.close()
+
+
+@pytest.mark.parametrize("bcf,nf,c0", [(((CF, CF),) * 3, (18, 14, 12), (2, 3, 1)),
+                                       (((CF, CF), (CF, CF), (0, 0)), (18, 14, 16), (2, 3, 0))])
+def test_average_down_bitwise(bcf, nf, c0):
+    nc = (16, 12, 8)
+    h = Hier(nc, c0, nf, bcf, synth.Wavy3D(L=(10.0,) * 3, N=nc), dict(terms=3, mu_ref=0.02))
+    metc, Uc, metf, Uf = h.oracle()
+    oracle.average_down(nf, bcf, Uf, nc, c0, Uc)
+    C, F, A = h.gpu((2, 2, 1), (2, 1, 2))
+    A.average_down()
+    bn, blocks, refs = _blocks_of(Uc, nc, (2, 2, 1))
+    for g, r in zip(C.get(C.U), refs):
+        assert np.array_equal(g[:, G:-G, G:-G, G:-G], r[:, G:-G, G:-G, G:-G])
+    C.close()
+    F.close()
+
+
+@pytest.mark.parametrize("nbc,nbf,state", [((1, 1, 1), (1, 1, 1), "vortex"), ((2, 2, 1), (2, 1, 2), "random")])
+def test_two_level_rk3_parity(nbc, nbf, state):
+    nc, c0, nf = (24, 24, 16), (5, 6, 3), (24, 20, 16)
+    bcf = ((CF, CF),) * 3
+    h = Hier(nc, c0, nf, bcf, synth.Wavy3D(L=(10.0,) * 3, N=nc), dict(terms=3, mu_ref=0.01),
+             state=state)
+    metc, Uc, metf, Uf = h.oracle()
+    dt, nsteps = 0.01, 10
+    oracle.amr_advance(nc, PER, nf, bcf, c0, oracle.phys(terms=3, mu_ref=0.01), dt, nsteps, Uc, metc, Uf, metf)
+    C, F, A = h.gpu(nbc, nbf)
+    A.step(dt, nsteps)
+    A.sync()
+    for S, n, nb, ref in ((C, nc, nbc, Uc), (F, nf, nbf, Uf)):
+        bn, blocks, refs = _blocks_of(ref, n, nb)
+        for g, r in zip(S.get(S.U), refs):
+            ri = r[:, G:-G, G:-G, G:-G]
+            assert rel_linf(g[:, G:-G, G:-G, G:-G], ri, state_scale(ri)) <= 1e-9
+    C.close()
+    F.close()
+
+
+def test_amr_abi_refusals():
+    from paper_conf_ipps_davissngmb23_b200 import crocco as cc
+    from paper_conf_ipps_davissngmb23_b200.solver import AmrSolver, Solver
+    nc = (16, 16, 16)
+    grid = synth.Wavy3D(L=(10.0,) * 3, N=nc)
+    C = Solver(nc, (1, 1, 1), PER)
+    F = Solver((12, 12, 12), (1, 1, 1), ((CF, CF),) * 3)
+    for S, g, n in ((C, grid, nc), (F, synth.Refined(grid, (2, 2, 2)), (12, 12, 12))):
+        S.set_coords([g.coords(n, (0, 0, 0), oracle.GC)])
+        S.set_state([synth.random_state(n, seed=1)])
+    with pytest.raises(cc.CroccoError):          # C/F faces without a coarse level
+        F.stage(0, 0.01)
+    with pytest.raises(cc.CroccoError):          # RK3 graph step on a fine level
+        F.step(0.01)
+    with pytest.raises(cc.CroccoError):          # fine level leaves the coarse domain
+        AmrSolver(C, F, (10, 2, 2))
+    with pytest.raises(cc.CroccoError):          # periodic fine level must span the domain
+        F2 = Solver((16, 16, 16), (1, 1, 1), PER)
+        try:
+            AmrSolver(C, F2, (0, 0, 0))
+        finally:
+            F2.close()
+    A = AmrSolver(C, F, (2, 2, 2))
+    C.fill()
+    A.step(0.01, 1)
+    A.sync()
+    C.close()
+    F.close()
