@@ -50,6 +50,8 @@ WORKLOADS = {
     "sod": "sod: Sod shock tube 200x4x4, inviscid (configs[0])",
     "dmr": "dmr: double Mach reflection 2048x512x128 in 2x2x1 blocks, slip wall + moving shock BCs "
            "(the paper's case, PAPER.md:183-185; SURVEY NEXT-2)",
+    "amr": "amr: two-level hierarchy (SURVEY NEXT-4): TGV 256^3 coarse level on the wavy grid + a "
+           "256^3-node fine level (ratio 2) over its central 128^3 region, C/F faces all round, viscous",
 }
 
 
@@ -418,6 +420,79 @@ def run_crocco(args, rank, world, local_rank):
     return 0
 
 
+def run_amr(args):
+    """--config amr (one GPU): Algorithm 2 with two levels -- per stage the coarse level, the fine
+    level with its C/F ghosts interpolated from the coarse stage input (k_cf_interp), AverageDown
+    (k_average_down) at the third stage.  value = (coarse + fine interior points) x 3 x steps / time."""
+    import torch
+
+    import synth
+    from paper_conf_ipps_davissngmb23_b200 import crocco as cc
+    from paper_conf_ipps_davissngmb23_b200.solver import AmrSolver, Solver
+
+    dev = torch.device("cuda", 0)
+    torch.cuda.set_device(dev)
+    nc, c0, nf = (256, 256, 256), (64, 64, 64), (256, 256, 256)
+    grid = synth.Wavy3D(L=(2 * math.pi,) * 3, N=nc, x0=(-math.pi,) * 3, k=2.0, A=0.15)
+    fgrid = synth.Refined(grid, c0)
+    phys = cc.make_phys(gamma=1.4, R=1.0, Pr=0.71, mu_ref=1.0 / 1600.0, terms=3)
+    CF = cc.BC_COARSE_FINE
+    C = Solver(nc, (1, 1, 1), ((0, 0),) * 3, phys, device=dev)
+    F = Solver(nf, (1, 1, 1), ((CF, CF),) * 3, phys, device=dev)
+    for S, g, n in ((C, grid, nc), (F, fgrid, nf)):
+        xyz = torch.from_numpy(g.coords(n, (0, 0, 0), cc.GHOST_COORDS)).to(dev)
+        S.set_coords_block(0, xyz)
+        S.set_state_block(0, synth.tgv(xyz, noise=0.01, seed=5))
+        del xyz
+    A = AmrSolver(C, F, c0)
+    dt = 2e-4
+    for _ in range(args.warmup):
+        A.step(dt)
+    torch.cuda.synchronize()
+    for S in (C, F):
+        cc.crocco_set_timing(S.ctx, True)
+        cc.crocco_kernel_times(S.ctx)
+        cc.crocco_launch_count(S.ctx, reset=True)
+    clk = ClockSampler(0) if not args.no_clocks else None
+    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    torch.cuda.synchronize()
+    e0.record(C.stream)
+    A.step(dt, args.steps)
+    e1.record(C.stream)
+    torch.cuda.synchronize()
+    ms = e0.elapsed_time(e1)
+    clocks = clk.stop() if clk else None
+    launches = cc.crocco_launch_count(C.ctx) + cc.crocco_launch_count(F.ctx)
+    kt = {}
+    for lv, S in (("coarse", C), ("fine", F)):
+        for k, (nl, kms) in cc.crocco_kernel_times(S.ctx).items():
+            if nl:
+                kt[f"{lv}:{k}"] = {"launches": nl, "ms": kms}
+    ktot = sum(v["ms"] for v in kt.values())
+    for v in kt.values():
+        v["share_of_kernel_time"] = v["ms"] / max(ktot, 1e-9)
+    pts = nc[0] * nc[1] * nc[2] + nf[0] * nf[1] * nf[2]
+    value = pts * 3 * args.steps / (ms / 1e3)
+    amr_ms = sum(v["ms"] for k, v in kt.items() if k.endswith(":amr"))
+    finite = all(bool(torch.isfinite(S.view(S.U[0], 0, 5)[:, 4:-4, 4:-4, 4:-4]).all().item()) for S in (C, F))
+    # C/F interpolation and AverageDown: HBM gathers; algorithmic bytes = 5 comps x 8 B written per
+    # C/F ghost point (+ the coarse corners read once, 1/8 of that) and 27+1 fine/coarse values per
+    # covered coarse point -- reported as a share of the step, not as a roofline (they are < 1 %)
+    out = {"metric": METRIC, "value": value, "unit": UNIT, "n_gpus": 1, "steps": args.steps,
+           "warmup": args.warmup, "ms_per_step": ms / args.steps, "higher_is_better": True,
+           "scaling": "strong", "vs_baseline": None, "dtype": "f64",
+           "data": "synthetic (seeded TGV + 1 % noise on both levels, DESIGN.md sec. 4)",
+           "config": {"workload": WORKLOADS["amr"] + "; step = 1 RK3 step (3 stages x 2 levels + AverageDown)",
+                      "n_coarse": list(nc), "n_fine": list(nf), "c0": list(c0), "points": pts, "dt": dt,
+                      "l2": "inputs larger than L2 (1.5 GB state per level)", "parallelism": "1 GPU"},
+           "amr_kernels_share": amr_ms / max(ktot, 1e-9), "kernel_breakdown": kt,
+           "gpu_launches": launches, "clocks": clocks, "state_finite": finite, "impl": "crocco"}
+    C.close()
+    F.close()
+    print(json.dumps(out), flush=True)
+    return 0
+
+
 def _profiled_traffic(kname):
     """dram bytes per launch of the dominant kernel from the committed ncu summary, if any."""
     p = os.path.join(ROOT, "profiles", "ncu_summary.json")
@@ -438,7 +513,7 @@ def main():
     ap.add_argument("--steps", type=int, default=5)
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--impl", choices=["crocco", "reference"], default="crocco")
-    ap.add_argument("--config", choices=["weak", "ramp", "tgv", "vortex", "sod", "dmr"], default="weak",
+    ap.add_argument("--config", choices=["weak", "ramp", "tgv", "vortex", "sod", "dmr", "amr"], default="weak",
                     help="weak (default, the north_star 512^3/GPU workload) or a fixed BASELINE config")
     ap.add_argument("--e2e-steps", type=int, default=4)
     ap.add_argument("--no-cpu-baseline", action="store_true")
@@ -450,6 +525,10 @@ def main():
     local_rank = int(os.environ.get("LOCAL_RANK", "0"))
     if args.impl == "reference":
         return run_reference(args, rank, world)
+    if args.config == "amr":
+        if world > 1:
+            raise SystemExit("--config amr runs on one GPU")
+        return run_amr(args)
     if world > 1:
         import torch
         import torch.distributed as dist
