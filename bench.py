@@ -515,7 +515,8 @@ def main():
     ap.add_argument("--impl", choices=["crocco", "reference"], default="crocco")
     ap.add_argument("--config", choices=["weak", "ramp", "tgv", "vortex", "sod", "dmr", "amr"], default="weak",
                     help="weak (default, the north_star 512^3/GPU workload) or a fixed BASELINE config")
-    ap.add_argument("--e2e-steps", type=int, default=4)
+    ap.add_argument("--e2e-steps", type=int, default=16,
+                    help="independent jobs streamed through host memory for e2e (pipeline fill + drain amortised)")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-clocks", action="store_true")
     ap.add_argument("--ref-n", type=int, default=64)
