@@ -40,11 +40,14 @@ class Hier:
     """One two-level problem, built identically for the oracle (global single boxes) and the GPU
     (any block decomposition of either level)."""
 
-    def __init__(self, nc, c0, nf, bcf, grid, phys_kw, seed=3, state="random"):
-        self.nc, self.c0, self.nf, self.bcf, self.grid = nc, c0, nf, bcf, grid
+    def __init__(self, nc, c0, nf, bcf, grid, phys_kw, seed=3, state="random", bcc=PER):
+        self.nc, self.c0, self.nf, self.bcf, self.grid, self.bcc = nc, c0, nf, bcf, grid, bcc
         self.phys_kw = phys_kw
         self.fgrid = synth.Refined(grid, c0)
-        if state == "random":
+        if callable(state):
+            self.Uc0 = state(grid.coords(nc, (0, 0, 0), oracle.GC))
+            self.Uf0 = state(self.fgrid.coords(nf, (0, 0, 0), oracle.GC))
+        elif state == "random":
             self.Uc0 = synth.random_state(nc, seed=seed, amp=0.2)
             self.Uf0 = synth.random_state(nf, seed=seed + 1, amp=0.2)
         else:
@@ -54,18 +57,18 @@ class Hier:
     def oracle(self):
         xc = self.grid.coords(self.nc, (0, 0, 0), oracle.GC)
         xf = self.fgrid.coords(self.nf, (0, 0, 0), oracle.GC)
-        metc = oracle.metrics(self.nc, PER, xc)
+        metc = oracle.metrics(self.nc, self.bcc, xc)
         metf = oracle.metrics(self.nf, self.bcf, xf)
         Uc = synth.pad_state(self.Uc0)
         Uf = synth.pad_state(self.Uf0)
-        oracle.fill(self.nc, PER, Uc)
+        oracle.fill(self.nc, self.bcc, Uc)
         return metc, Uc, metf, Uf
 
     def gpu(self, nbc, nbf):
         from paper_conf_ipps_davissngmb23_b200 import crocco as cc
         from paper_conf_ipps_davissngmb23_b200.solver import AmrSolver, Solver
         kw = dict(self.phys_kw)
-        C = Solver(self.nc, nbc, PER, cc.make_phys(**kw))
+        C = Solver(self.nc, nbc, self.bcc, cc.make_phys(**kw))
         F = Solver(self.nf, nbf, self.bcf, cc.make_phys(**kw))
         for S, n, nb, g, U0 in ((C, self.nc, nbc, self.grid, self.Uc0), (F, self.nf, nbf, self.fgrid, self.Uf0)):
             bn, blocks = block_slices(n, nb)
@@ -144,6 +147,32 @@ def test_two_level_rk3_parity(nbc, nbf, state):
     A.step(dt, nsteps)
     A.sync()
     for S, n, nb, ref in ((C, nc, nbc, Uc), (F, nf, nbf, Uf)):
+        bn, blocks, refs = _blocks_of(ref, n, nb)
+        for g, r in zip(S.get(S.U), refs):
+            ri = r[:, G:-G, G:-G, G:-G]
+            assert rel_linf(g[:, G:-G, G:-G, G:-G], ri, state_scale(ri)) <= 1e-9
+    C.close()
+    F.close()
+
+
+def test_two_level_ramp_wall_parity():
+    """Compression-ramp flow (walls, Sutherland, Mach 6) with a fine level on the no-slip wall:
+    eta-lo WALL on both levels, zeta spanned periodically, xi and eta-hi C/F; multi-block levels."""
+    E, W = 1, 3
+    nc = (64, 32, 16)
+    grid = synth.Ramp(N=nc)
+    bcc = ((E, E), (W, E), (0, 0))
+    c0, nf = (16, 0, 0), (40, 32, 32)
+    bcf = ((CF, CF), (W, CF), (0, 0))
+    phys = dict(gamma=1.4, R=1.0, Pr=0.72, mu_law=1, mu_ref=1e-3, T_ref=1.0, S=0.3, terms=3)
+    h = Hier(nc, c0, nf, bcf, grid, phys, state=lambda x: synth.ramp_state(x, grid), bcc=bcc)
+    metc, Uc, metf, Uf = h.oracle()
+    dt, nsteps = 2e-4, 5
+    oracle.amr_advance(nc, bcc, nf, bcf, c0, oracle.phys(**phys), dt, nsteps, Uc, metc, Uf, metf)
+    C, F, A = h.gpu((2, 2, 1), (2, 2, 2))
+    A.step(dt, nsteps)
+    A.sync()
+    for S, n, nb, ref in ((C, nc, (2, 2, 1), Uc), (F, nf, (2, 2, 2), Uf)):
         bn, blocks, refs = _blocks_of(ref, n, nb)
         for g, r in zip(S.get(S.U), refs):
             ri = r[:, G:-G, G:-G, G:-G]
