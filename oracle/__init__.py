@@ -44,7 +44,8 @@ class Phys(C.Structure):
                 ("mu_law", C.c_int32), ("mu_ref", C.c_double), ("T_ref", C.c_double),
                 ("S", C.c_double), ("weno_eps", C.c_double), ("terms", C.c_int32),
                 ("dir_mask", C.c_int32), ("weno_linear", C.c_int32), ("weno_weights", C.c_int32),
-                ("weno_limiter", C.c_int32), ("weno_alpha_rl", C.c_double), ("weno_alpha_al", C.c_double)]
+                ("weno_limiter", C.c_int32), ("weno_alpha_rl", C.c_double), ("weno_alpha_al", C.c_double),
+                ("visc_form", C.c_int32)]
 
 
 class Split(C.Structure):
@@ -67,9 +68,9 @@ def splits(spec=None):
 
 def phys(gamma=1.4, R=1.0, Pr=0.72, mu_law=MU_CONST, mu_ref=0.0, T_ref=1.0, S=0.0,
          weno_eps=1e-6, terms=INVISCID | VISCOUS, dir_mask=7, weno_linear=0, weno_weights=0,
-         weno_limiter=0, weno_alpha_rl=0.0, weno_alpha_al=0.0) -> Phys:
+         weno_limiter=0, weno_alpha_rl=0.0, weno_alpha_al=0.0, visc_form=0) -> Phys:
     return Phys(gamma, R, Pr, mu_law, mu_ref, T_ref, S, weno_eps, terms, dir_mask, weno_linear, weno_weights,
-                weno_limiter, weno_alpha_rl, weno_alpha_al)
+                weno_limiter, weno_alpha_rl, weno_alpha_al, visc_form)
 
 
 _lib = None
@@ -111,6 +112,8 @@ def lib():
         L.oracle_average_down.argtypes = [i64p, i32p, dp, dp, i64p, i64p, dp]
         L.oracle_amr_advance.argtypes = [i64p, i32p, dp, i64p, i32p, dp, i64p, C.POINTER(Phys),
                                          C.c_double, C.c_int32, dp, dp, dp, dp]
+        L.oracle_metrics2.argtypes = [i64p, dp, dp]
+        L.oracle_rhs_ex.argtypes = [i64p, C.POINTER(Phys), dp, dp, dp, dp]
         L.oracle_set_threads.argtypes = [C.c_int]
         L.oracle_get_threads.restype = C.c_int
         _lib = L
@@ -197,6 +200,14 @@ def rhs(n, ph: Phys, U, met):
     """rhs = J(-sum delta F_inv + sum D4 F_v) on interior points (ghosts of U must be filled)."""
     out = padded(n, 5)
     lib().oracle_rhs(_n(n), C.byref(ph), _dp(U), _dp(met), _dp(out))
+    return out
+
+
+def metrics2(n, met):
+    """18 second metrics xi_{a,jk} (j <= k; component 6a + pair) on interior points from the
+    10-component metrics (PAPER.md:139's 27-component set = these + the 9 first metrics)."""
+    out = padded(n, 18)
+    lib().oracle_metrics2(_n(n), _dp(met), _dp(out))
     return out
 
 

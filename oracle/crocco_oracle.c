@@ -55,6 +55,8 @@ typedef struct {
     int32_t weno_weights; /* 0: SYMBO (Martin et al. 2006), 1: SYMOO (reading 22, NEXT-3) */
     int32_t weno_limiter; /* bit 0: relative, bit 1: absolute limiter (reading 23, NEXT-3); 0 = off */
     double weno_alpha_rl, weno_alpha_al; /* thresholds of the two limiters */
+    int32_t visc_form; /* 0: conservative point-flux form (reading 12), 1: expanded form with the
+                          27-component metrics (readings 27-28, NEXT-3) */
 } oracle_phys;
 
 typedef struct {
@@ -585,8 +587,36 @@ static double d4(const double *f, int64_t p, int64_t s)
     return (8.0 * (f[p + s] - f[p - s]) - (f[p + 2 * s] - f[p - 2 * s])) / 12.0;
 }
 
+static void rhs_core(const int64_t n[3], const oracle_phys *ph, const double *U, const double *met,
+                     const double *met2, double *rhs);
+
+void oracle_metrics2(const int64_t n[3], const double *met, double *met2);
+
 void oracle_rhs(const int64_t n[3], const oracle_phys *ph, const double *U, const double *met,
                 double *rhs)
+{
+    if (ph->visc_form == 1 && (ph->terms & O_VISCOUS)) {
+        obox b = make_box(n, OG);
+        double *met2 = (double *)calloc((size_t)(18 * b.cs), sizeof(double));
+        oracle_metrics2(n, met, met2);
+        rhs_core(n, ph, U, met, met2, rhs);
+        free(met2);
+        return;
+    }
+    rhs_core(n, ph, U, met, NULL, rhs);
+}
+
+void oracle_rhs_ex(const int64_t n[3], const oracle_phys *ph, const double *U, const double *met,
+                   const double *met2, double *rhs)
+{
+    rhs_core(n, ph, U, met, met2, rhs);
+}
+
+static void visc_expanded(const int64_t n[3], const oracle_phys *ph, const double *U,
+                          const double *met, const double *met2, double *V);
+
+static void rhs_core(const int64_t n[3], const oracle_phys *ph, const double *U, const double *met,
+                     const double *met2, double *rhs)
 {
     obox b = make_box(n, OG);
     const int64_t cs = b.cs;
@@ -642,7 +672,11 @@ void oracle_rhs(const int64_t n[3], const oracle_phys *ph, const double *U, cons
     }
 
     /* --- viscous and heat fluxes (Alg. 2 l.8) --- */
-    if (ph->terms & O_VISCOUS) {
+    double *Vx = NULL; /* expanded form: physical-space viscous divergence at interior points */
+    if ((ph->terms & O_VISCOUS) && ph->visc_form == 1) {
+        Vx = (double *)calloc((size_t)(5 * cs), sizeof(double));
+        visc_expanded(n, ph, U, met, met2, Vx);
+    } else if (ph->terms & O_VISCOUS) {
         const double gm1 = ph->gamma - 1.0;
         const double cp = ph->gamma * ph->R / gm1;
         double *pr = (double *)malloc((size_t)(4 * cs) * sizeof(double)); /* u v w T */
@@ -732,10 +766,193 @@ void oracle_rhs(const int64_t n[3], const oracle_phys *ph, const double *U, cons
         for (int64_t j = 0; j < n[1]; j++)
             for (int64_t i = 0; i < n[0]; i++) {
                 int64_t p = IX(&b, i, j, k);
-                for (int c = 0; c < 5; c++)
+                for (int c = 0; c < 5; c++) {
                     rhs[c * cs + p] = met[p] * R[c * cs + p];
+                    if (Vx)
+                        rhs[c * cs + p] = rhs[c * cs + p] + Vx[c * cs + p];
+                }
             }
     free(R);
+    free(Vx);
+}
+
+/* ------------------------------------------------------------------ */
+/* 6b. The paper's 27-component metric set and the expanded viscous    */
+/*     form ("first and second order grid metrics ... a    */
+/*     27-component MultiFab"; readings 27-28).          */
+/*     First metrics xi_{a,j} = d xi_a / d x_j = J m^a_j (9, from the   */
+/*     10-component set); second metrics                                */
+/*       xi_{a,jk} = d/dx_k (xi_{a,j}) = sum_b xi_{b,k} D6_b(xi_{a,j})   */
+/*     for j <= k (18): component 6a + P(j,k), pairs P = (00, 01, 02,   */
+/*     11, 12, 22).  Interior points only.                              */
+/* ------------------------------------------------------------------ */
+static const int PJ[6] = {0, 0, 0, 1, 1, 2}, PK[6] = {0, 1, 2, 1, 2, 2};
+static int pair_of(int j, int k)
+{
+    int lo = j < k ? j : k, hi = j < k ? k : j;
+    return lo == 0 ? hi : (lo == 1 ? 2 + hi : 5);
+}
+
+void oracle_metrics2(const int64_t n[3], const double *met, double *met2)
+{
+    obox b = make_box(n, OG);
+    const int64_t cs = b.cs;
+    int64_t st[3] = {1, b.p[0], b.p[0] * b.p[1]};
+    /* xi_{a,j} on the whole padded box */
+    double *xi = (double *)malloc((size_t)(9 * cs) * sizeof(double));
+    for (int a = 0; a < 3; a++)
+        for (int j = 0; j < 3; j++)
+            for (int64_t p = 0; p < cs; p++)
+                xi[(3 * a + j) * cs + p] = met[p] * met[(1 + 3 * a + j) * cs + p];
+#pragma omp parallel for OMP_THREADS
+    for (int64_t k = 0; k < n[2]; k++)
+        for (int64_t j = 0; j < n[1]; j++)
+            for (int64_t i = 0; i < n[0]; i++) {
+                int64_t p = IX(&b, i, j, k);
+                for (int a = 0; a < 3; a++)
+                    for (int q = 0; q < 6; q++) {
+                        int jj = PJ[q], kk = PK[q];
+                        double s = 0.0;
+                        for (int bb = 0; bb < 3; bb++)
+                            s = s + xi[(3 * bb + kk) * cs + p] * d6(xi + (3 * a + jj) * cs, p, st[bb]);
+                        met2[(6 * a + q) * cs + p] = s;
+                    }
+            }
+    free(xi);
+}
+
+/* d mu / d T of the viscosity law (reading 2) */
+static double dmu_dT(const oracle_phys *ph, double T)
+{
+    if (ph->mu_law == 1)
+        return mu_of_T(ph, T) * (1.5 / T - 1.0 / (T + ph->S));
+    return 0.0;
+}
+
+/* 4th-order central second derivative (5 points) */
+static double d2(const double *f, int64_t p, int64_t s)
+{
+    return (16.0 * (f[p + s] + f[p - s]) - (f[p + 2 * s] + f[p - 2 * s]) - 30.0 * f[p]) / 12.0;
+}
+
+/* Expanded viscous form (reading 28): V = div F_v evaluated pointwise with the chain rule,
+     G_ij = d u_i/d x_j = sum_a xi_{a,j} D4_a u_i,   g_j = sum_a xi_{a,j} D4_a T,
+     d2 phi/dx_j dx_k = sum_{a,b} xi_{a,j} xi_{b,k} phi_ab + sum_a xi_{a,jk} phi_a,
+       phi_aa = D2_a phi (5-point 4th order), phi_ab = D4_a(D4_b phi) (a != b),
+     d tau_ij/d x_j = mu (lap u_i + (1/3) d_i div u) + sum_j (mu' g_j)(G_ij + G_ji - (2/3) delta_ij div u),
+     V_{1+i} = d tau_ij / d x_j,
+     V_4 = u_i d tau_ij/d x_j + tau_ij G_ij + kappa lap T + (c_p/Pr) mu' |g|^2,  V_0 = 0. */
+static void visc_expanded(const int64_t n[3], const oracle_phys *ph, const double *U,
+                          const double *met, const double *met2, double *V)
+{
+    obox b = make_box(n, OG);
+    const int64_t cs = b.cs;
+    int64_t st[3] = {1, b.p[0], b.p[0] * b.p[1]};
+    const double gm1 = ph->gamma - 1.0;
+    const double cp = ph->gamma * ph->R / gm1;
+    double *pr = (double *)malloc((size_t)(4 * cs) * sizeof(double)); /* u v w T */
+    for (int64_t p = 0; p < cs; p++) {
+        double rho = U[p];
+        double u = U[cs + p] / rho, v = U[2 * cs + p] / rho, w = U[3 * cs + p] / rho;
+        double pres = gm1 * (U[4 * cs + p] - 0.5 * rho * (u * u + v * v + w * w));
+        pr[p] = u;
+        pr[cs + p] = v;
+        pr[2 * cs + p] = w;
+        pr[3 * cs + p] = pres / (rho * ph->R);
+    }
+    /* first computational derivatives D4_b phi on the interior +-2 box (for the mixed ones) */
+    double *dphi = (double *)calloc((size_t)(12 * cs), sizeof(double)); /* [4 fields][3 dirs] */
+    for (int64_t k = -2; k < n[2] + 2; k++)
+        for (int64_t j = -2; j < n[1] + 2; j++)
+            for (int64_t i = -2; i < n[0] + 2; i++) {
+                int64_t p = IX(&b, i, j, k);
+                for (int f = 0; f < 4; f++)
+                    for (int d = 0; d < 3; d++)
+                        dphi[(3 * f + d) * cs + p] = d4(pr + f * cs, p, st[d]);
+            }
+#pragma omp parallel for OMP_THREADS
+    for (int64_t k = 0; k < n[2]; k++)
+        for (int64_t j = 0; j < n[1]; j++)
+            for (int64_t i = 0; i < n[0]; i++) {
+                int64_t p = IX(&b, i, j, k);
+                double xi[3][3], xi2[3][6];
+                for (int a = 0; a < 3; a++)
+                    for (int c = 0; c < 3; c++)
+                        xi[a][c] = met[p] * met[(1 + 3 * a + c) * cs + p];
+                for (int a = 0; a < 3; a++)
+                    for (int q = 0; q < 6; q++)
+                        xi2[a][q] = met2[(6 * a + q) * cs + p];
+                double ph1[4][3], ph2[4][3][3]; /* phi_a, phi_ab */
+                for (int f = 0; f < 4; f++) {
+                    for (int a = 0; a < 3; a++)
+                        ph1[f][a] = dphi[(3 * f + a) * cs + p];
+                    for (int a = 0; a < 3; a++)
+                        for (int c = 0; c < 3; c++) {
+                            if (a == c)
+                                ph2[f][a][c] = d2(pr + f * cs, p, st[a]);
+                            else {
+                                int lo = a < c ? a : c, hi = a < c ? c : a;
+                                ph2[f][a][c] = d4(dphi + (3 * f + lo) * cs, p, st[hi]);
+                            }
+                        }
+                }
+                /* physical first and second derivatives */
+                double gx[4][3], hx[4][3][3];
+                for (int f = 0; f < 4; f++) {
+                    for (int c = 0; c < 3; c++) {
+                        double s = 0.0;
+                        for (int a = 0; a < 3; a++)
+                            s = s + xi[a][c] * ph1[f][a];
+                        gx[f][c] = s;
+                    }
+                    for (int jj = 0; jj < 3; jj++)
+                        for (int kk = 0; kk < 3; kk++) {
+                            double s = 0.0;
+                            for (int a = 0; a < 3; a++)
+                                for (int c = 0; c < 3; c++)
+                                    s = s + xi[a][jj] * xi[c][kk] * ph2[f][a][c];
+                            for (int a = 0; a < 3; a++)
+                                s = s + xi2[a][pair_of(jj, kk)] * ph1[f][a];
+                            hx[f][jj][kk] = s;
+                        }
+                }
+                double T = pr[3 * cs + p];
+                double mu = mu_of_T(ph, T), mup = dmu_dT(ph, T);
+                double kap = mu * cp / ph->Pr;
+                double div = gx[0][0] + gx[1][1] + gx[2][2];
+                double dtau[3];
+                for (int a = 0; a < 3; a++) {
+                    double lap = hx[a][0][0] + hx[a][1][1] + hx[a][2][2];
+                    double gdiv = hx[0][0][a] + hx[1][1][a] + hx[2][2][a];
+                    double s = mu * (lap + gdiv / 3.0);
+                    for (int c = 0; c < 3; c++) {
+                        double sym = gx[a][c] + gx[c][a];
+                        if (a == c)
+                            sym = sym - 2.0 / 3.0 * div;
+                        s = s + mup * gx[3][c] * sym;
+                    }
+                    dtau[a] = s;
+                }
+                double work = 0.0;
+                for (int a = 0; a < 3; a++)
+                    work = work + pr[a * cs + p] * dtau[a];
+                double diss = 0.0;
+                for (int a = 0; a < 3; a++)
+                    for (int c = 0; c < 3; c++) {
+                        double tau = mu * (gx[a][c] + gx[c][a]);
+                        if (a == c)
+                            tau = tau - 2.0 / 3.0 * mu * div;
+                        diss = diss + tau * gx[a][c];
+                    }
+                double lapT = hx[3][0][0] + hx[3][1][1] + hx[3][2][2];
+                double gT2 = gx[3][0] * gx[3][0] + gx[3][1] * gx[3][1] + gx[3][2] * gx[3][2];
+                V[p] = 0.0;
+                for (int a = 0; a < 3; a++)
+                    V[(1 + a) * cs + p] = dtau[a];
+                V[4 * cs + p] = work + diss + kap * lapT + cp / ph->Pr * mup * gT2;
+            }
+    free(dphi);
+    free(pr);
 }
 
 /* ------------------------------------------------------------------ */
