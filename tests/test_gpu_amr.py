@@ -181,6 +181,31 @@ def test_two_level_ramp_wall_parity():
     F.close()
 
 
+@pytest.mark.slow
+def test_full_size_amr_bench_config_bitwise():
+    """bench.py --config amr at full size and in its launch configuration: 256^3 coarse TGV level,
+    256^3-node fine level at c0 = (64, 64, 64), C/F faces all round.  Every fine ghost after
+    FillPatchTwoLevels and every coarse interior point after AverageDown equal the oracle's."""
+    import math
+    nc, c0, nf = (256, 256, 256), (64, 64, 64), (256, 256, 256)
+    grid = synth.Wavy3D(L=(2 * math.pi,) * 3, N=nc, x0=(-math.pi,) * 3, k=2.0, A=0.15)
+    phys = dict(gamma=1.4, R=1.0, Pr=0.71, mu_ref=1.0 / 1600.0, terms=3)
+    tgv = lambda x: synth.tgv(x, noise=0.01, seed=5)
+    h = Hier(nc, c0, nf, ((CF, CF),) * 3, grid, phys, state=tgv)
+    C, F, A = h.gpu((1, 1, 1), (1, 1, 1))
+    Uc = synth.pad_state(h.Uc0)
+    oracle.fill(nc, PER, Uc)
+    Uf = synth.pad_state(h.Uf0)
+    oracle.fill_two_levels(nf, h.bcf, Uf, nc, c0, Uc)
+    A.fill_fine()
+    assert np.array_equal(F.get(F.U)[0], Uf)
+    oracle.average_down(nf, h.bcf, Uf, nc, c0, Uc)
+    A.average_down()
+    assert np.array_equal(C.get(C.U)[0][:, G:-G, G:-G, G:-G], Uc[:, G:-G, G:-G, G:-G])
+    C.close()
+    F.close()
+
+
 def test_amr_abi_refusals():
     from paper_conf_ipps_davissngmb23_b200 import crocco as cc
     from paper_conf_ipps_davissngmb23_b200.solver import AmrSolver, Solver

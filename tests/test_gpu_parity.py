@@ -296,7 +296,7 @@ def _block_points(bn, rng, k_random):
 
 
 @pytest.mark.slow
-@pytest.mark.parametrize("name", ["weak", "ramp", "tgv"])
+@pytest.mark.parametrize("name", ["weak", "ramp", "tgv", "dmr"])
 def test_full_size_config_sampled(name):
     """BASELINE.json full sizes in bench.py's launch configuration (crocco_rk_stage):
     weak = 512^3 periodic wavy TGV (configs[4]); ramp = 1024 x 512 x 256 Mach-6
@@ -308,7 +308,10 @@ def test_full_size_config_sampled(name):
     n = c.n_global
     from paper_conf_ipps_davissngmb23_b200 import crocco as cc
     from paper_conf_ipps_davissngmb23_b200.solver import Solver
-    S = Solver(n, c.n_blocks, c.bc, cc.make_phys(**c.phys))
+    bc, dirichlet, split = c.bc, None, None
+    if name == "dmr":  # the paper's case (NEXT-2): slip wall + moving-shock SPLIT faces
+        bc, dirichlet, split = synth.dmr_bc(1.0 / n[1])
+    S = Solver(n, c.n_blocks, bc, cc.make_phys(**c.phys), dirichlet=dirichlet, split=split)
     bn, blocks = block_slices(n, c.n_blocks)
     xyz = []
     U0 = []
