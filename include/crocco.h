@@ -125,6 +125,10 @@ typedef struct {
                               bit 1: max beta < weno_alpha_al (absolute limiter; beta of the
                               reconstructed characteristic flux (g +- lambda w)/2) */
     double weno_alpha_rl, weno_alpha_al;  /* thresholds, >= 0 */
+    int32_t visc_form;     /* viscous discretisation: 0 = conservative point-flux form (reading 12,
+                              default); 1 = expanded (non-conservative) form with the paper's
+                              27-component metrics (readings 27-28):
+                              needs crocco_init_metrics2 after crocco_init_metrics */
 } crocco_phys;
 
 typedef struct {
@@ -172,6 +176,16 @@ crocco_status crocco_scratch_bytes(crocco_ctx ctx, int64_t *bytes);
    padded box (interior +-4), then copy the periodic / inter-block ghost metrics
    from their owners (crocco_fill_boundary(METRIC)).  Collective. */
 crocco_status crocco_init_metrics(crocco_ctx ctx, double *const *xyz, double *const *metrics);
+/* The 18 second metrics of the paper's 27-component set (reading 27):
+   xi_{a,jk} = d2 xi_a / dx_j dx_k = sum_b xi_{b,k} D6_b(xi_{a,j}), xi_{a,j} = J m^a_j, j <= k,
+   component 6a + pair index of (00, 01, 02, 11, 12, 22), on interior points, computed from
+   `metrics` (filled by crocco_init_metrics) into LIBRARY-OWNED device memory (18 fp64 per
+   interior point; reported by crocco_scratch_bytes) used by the expanded viscous form
+   (visc_form = 1).  Call again after changing the metrics.  Not collective. */
+crocco_status crocco_init_metrics2(crocco_ctx ctx, double *const *metrics);
+/* Copy local block b's second metrics to dst (device memory, 18 x n0 n1 n2 fp64, component
+   q at q * n0 n1 n2 + i + n0 (j + n1 k)); tests.  CROCCO_ERR_STATE if not initialised. */
+crocco_status crocco_copy_metrics2(crocco_ctx ctx, int32_t local_block, double *dst);
 
 /* FillPatch + BC_Fill: in place on 4 ghost layers,
    phases xi -> eta (spanning xi ghosts) -> zeta (spanning xi, eta ghosts).

@@ -45,7 +45,7 @@ class PhysC(C.Structure):
                 ("mu_law", C.c_int32), ("mu_ref", C.c_double), ("T_ref", C.c_double),
                 ("S", C.c_double), ("weno_eps", C.c_double), ("terms", C.c_int32),
                 ("dir_mask", C.c_int32), ("weno_weights", C.c_int32), ("weno_limiter", C.c_int32),
-                ("weno_alpha_rl", C.c_double), ("weno_alpha_al", C.c_double)]
+                ("weno_alpha_rl", C.c_double), ("weno_alpha_al", C.c_double), ("visc_form", C.c_int32)]
 
 
 class BlockLayout(C.Structure):
@@ -93,6 +93,8 @@ _SIGS = {
     "crocco_compute_dt": [C.c_void_p, DPP, DPP, C.c_double, C.POINTER(C.c_double)],
     "crocco_rk3_step": [C.c_void_p, C.c_double, DPP, DPP, DPP, DPP, C.c_int32],
     "crocco_amr_link": [C.c_void_p, C.c_void_p, C.POINTER(C.c_int64)],
+    "crocco_init_metrics2": [C.c_void_p, DPP],
+    "crocco_copy_metrics2": [C.c_void_p, C.c_int32, C.c_void_p],
     "crocco_fill_patch_two_levels": [C.c_void_p, DPP, DPP, DPP],
     "crocco_amr_rk_stage": [C.c_void_p, C.c_int32, C.c_double, DPP, DPP, DPP, DPP, DPP],
     "crocco_average_down": [C.c_void_p, DPP, DPP],
@@ -178,9 +180,9 @@ def make_desc(n_global, n_blocks=(1, 1, 1), bc=((0, 0),) * 3, dirichlet=None, ra
 
 def make_phys(gamma=1.4, R=1.0, Pr=0.72, mu_law=MU_CONST, mu_ref=0.0, T_ref=1.0, S=0.0,
               weno_eps=1e-6, terms=TERM_INVISCID | TERM_VISCOUS, dir_mask=7, weno_weights=0,
-              weno_limiter=0, weno_alpha_rl=0.0, weno_alpha_al=0.0):
+              weno_limiter=0, weno_alpha_rl=0.0, weno_alpha_al=0.0, visc_form=0):
     return PhysC(gamma, R, Pr, mu_law, mu_ref, T_ref, S, weno_eps, terms, dir_mask, weno_weights,
-                 weno_limiter, weno_alpha_rl, weno_alpha_al)
+                 weno_limiter, weno_alpha_rl, weno_alpha_al, visc_form)
 
 
 def crocco_init_grid(desc: GridDesc, phys: PhysC):
@@ -347,3 +349,13 @@ def crocco_average_down(fine, Uf_ptrs, Uc_ptrs):
     a, ka = _ptrs(Uf_ptrs)
     b, kb = _ptrs(Uc_ptrs)
     _check(lib().crocco_average_down(fine, a, b), fine)
+
+
+# ---- 27-component metrics / expanded viscous form (readings 27-28) ----
+def crocco_init_metrics2(ctx, met_ptrs):
+    a, ka = _ptrs(met_ptrs)
+    _check(lib().crocco_init_metrics2(ctx, a), ctx)
+
+
+def crocco_copy_metrics2(ctx, b, dst_ptr):
+    _check(lib().crocco_copy_metrics2(ctx, int(b), C.c_void_p(int(dst_ptr))), ctx)

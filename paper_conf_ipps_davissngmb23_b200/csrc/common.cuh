@@ -20,6 +20,7 @@ struct Phys {
     int lim;       // WENO limiters (reading 23): bit 0 relative, bit 1 absolute
     double arl;    // relative threshold (scale-free)
     double aal_b;  // absolute threshold in the units of the kernels' b_k (weno.cuh)
+    int visc_form; // 0 conservative point-flux viscous form, 1 expanded form (viscexp.cuh)
 };
 
 struct Lay {  // padded block layout (elements)

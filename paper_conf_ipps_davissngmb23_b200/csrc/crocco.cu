@@ -20,6 +20,7 @@
 #include "metrics.cuh"
 #include "pointwise.cuh"
 #include "sweep.cuh"
+#include "viscexp.cuh"
 
 using namespace crocco;
 
@@ -45,6 +46,8 @@ struct LocalBlock {
     int64_t rcs = 0;
     double *fv = nullptr;
     double *rv = nullptr;    // viscous D4_zeta term (CROCCO_ZDIV_SWEEP != 0)
+    double *met2 = nullptr;  // expanded viscous form: 18 second metrics (compact interior, rcs)
+    double *p4 = nullptr;    // expanded viscous form: u v w T on the padded box
 };
 
 enum { K_PRIMS = 0, K_FLUX_X, K_FLUX_Y, K_FLUX_Z, K_VISC, K_UPDATE, K_FILL, K_METRICS, K_CFL, K_AMR,
@@ -414,6 +417,7 @@ static Phys to_phys(const crocco_phys *p) {
     // b_k of the kernels = (12/13) beta_k of the reconstructed values, which carry a factor 2
     // (LLF 1/2 folded, flux.cuh): b = (48/13) beta of (g +- lambda w)/2
     ph.aal_b = p->weno_alpha_al * (4.0 * WENO_BSCALE);
+    ph.visc_form = p->visc_form;
 #if CROCCO_WENO_FOLD
     // only the ratios C_k / C_0 enter W (weno.cuh); alpha_0 then needs no multiply
     const double c0 = ph.wC[0];
@@ -433,6 +437,7 @@ static crocco_status check_phys(const crocco_phys *p) {
     if (p->weno_limiter & ~3) return fail(nullptr, CROCCO_ERR_ARG, "bad weno_limiter mask");
     if (!(p->weno_alpha_rl >= 0) || !(p->weno_alpha_al >= 0))
         return fail(nullptr, CROCCO_ERR_ARG, "WENO limiter thresholds must be >= 0");
+    if (p->visc_form != 0 && p->visc_form != 1) return fail(nullptr, CROCCO_ERR_ARG, "bad visc_form");
     return CROCCO_OK;
 }
 
@@ -451,6 +456,8 @@ static void free_ctx(crocco_ctx c) {
         cudaFree(b.racc);
         cudaFree(b.fv);
         cudaFree(b.rv);
+        cudaFree(b.met2);
+        cudaFree(b.p4);
     }
     cudaFree(c->send_stage);
     cudaFree(c->dmax);
@@ -905,6 +912,41 @@ crocco_status crocco_init_metrics(crocco_ctx c, double *const *xyz, double *cons
     return fill_all(c, met, CROCCO_FIELD_METRIC, nullptr, 0.0);
 }
 
+crocco_status crocco_init_metrics2(crocco_ctx c, double *const *met) {
+    LIVE(c);
+    crocco_status st = check_ptrs(c, met, "metrics");
+    if (st) return st;
+    for (auto &b : c->loc) {
+        if (!b.met2) {
+            if (cudaMalloc((void **)&b.met2, (size_t)(18 * b.rcs) * sizeof(double)) != cudaSuccess ||
+                cudaMalloc((void **)&b.p4, (size_t)(4 * b.L.cs) * sizeof(double)) != cudaSuccess) {
+                cudaGetLastError();
+                return fail(c, CROCCO_ERR_NOMEM, "second-metric allocation failed");
+            }
+            CK(c, cudaMemsetAsync(b.p4, 0, (size_t)(4 * b.L.cs) * sizeof(double), c->stream));
+            c->scratch += (18 * b.rcs + 4 * b.L.cs) * (int64_t)sizeof(double);
+        }
+    }
+    for (size_t bi = 0; bi < c->loc.size(); bi++) {
+        const LocalBlock &b = c->loc[bi];
+        const int64_t ni = (int64_t)b.g.n[0] * b.g.n[1] * b.g.n[2];
+        LAUNCH(c, K_METRICS, k_metric2<<<cdiv(ni, 128), 128, 0, c->stream>>>(met[bi], b.met2, b.L, b.rcs));
+    }
+    return CROCCO_OK;
+}
+
+crocco_status crocco_copy_metrics2(crocco_ctx c, int32_t lb, double *dst) {
+    LIVE(c);
+    if (lb < 0 || lb >= (int)c->loc.size() || !dst) return fail(c, CROCCO_ERR_ARG, "bad local block / dst");
+    const LocalBlock &b = c->loc[lb];
+    if (!b.met2) return fail(c, CROCCO_ERR_STATE, "second metrics not initialised");
+    const int64_t ni = (int64_t)b.g.n[0] * b.g.n[1] * b.g.n[2];
+    for (int q = 0; q < 18; q++)
+        CK(c, cudaMemcpyAsync(dst + q * ni, b.met2 + q * b.rcs, (size_t)ni * sizeof(double),
+                              cudaMemcpyDeviceToDevice, c->stream));
+    return CROCCO_OK;
+}
+
 // ---------------------------------------------------------------------------
 // RHS / RK
 // ---------------------------------------------------------------------------
@@ -918,7 +960,7 @@ static const double RK_B[3] = {1.0 / 3.0, 15.0 / 16.0, 8.0 / 15.0};
 // ghost-free interior tiles of the viscous kernel (k_visc_tiled sel 1) of one block;
 // returns false if the block has none or the configuration has no such split
 static bool visc_overlap_possible(crocco_ctx c) {
-    const bool viscous = (c->ph.terms & CROCCO_TERM_VISCOUS) != 0;
+    const bool viscous = (c->ph.terms & CROCCO_TERM_VISCOUS) != 0 && c->ph.visc_form == 0;
     if (!(viscous && CROCCO_SWEEP_SMEM && !CROCCO_VISC_DIV && CROCCO_VISC_ZDIV && CROCCO_ZDIV_SWEEP == 0))
         return false;
     for (const auto &b : c->loc) {
@@ -941,7 +983,8 @@ static crocco_status rhs_block(crocco_ctx c, const LocalBlock &b, const double *
                                double *dU, int stage, double dt, int visc_sel = 0) {
     const Phys &ph = c->ph;
     const bool inviscid = (ph.terms & CROCCO_TERM_INVISCID) != 0;
-    const bool viscous = (ph.terms & CROCCO_TERM_VISCOUS) != 0;
+    const bool vexp = (ph.terms & CROCCO_TERM_VISCOUS) != 0 && ph.visc_form == 1;  // readings 27-28
+    const bool viscous = (ph.terms & CROCCO_TERM_VISCOUS) != 0 && !vexp;
     const int64_t np = (int64_t)(b.g.n[0] + 2 * G) * (b.g.n[1] + 2 * G) * (b.g.n[2] + 2 * G);
     if (!CROCCO_SWEEP_SMEM)  // the staged sweeps and the tiled viscous kernel compute their own primitives
         LAUNCH(c, K_PRIMS, k_prims<<<cdiv(np, 256), 256, 0, c->stream>>>(U, b.prim, b.L, ph));
@@ -952,7 +995,13 @@ static crocco_status rhs_block(crocco_ctx c, const LocalBlock &b, const double *
     // 1 / 2 -> separate buffer added by the eta / zeta sweep
     const int zsw = CROCCO_ZDIV_SWEEP;
     double *rvz = (zdiv && zsw != 0) ? b.rv : b.racc;
-    if (vdiv) {
+    if (vexp) {  // expanded viscous form: V / J -> R comps 1..4, the xi sweep adds (mode 4)
+        if (!b.met2 || !b.p4)
+            return fail(c, CROCCO_ERR_STATE, "visc_form = 1 needs crocco_init_metrics2");
+        LAUNCH(c, K_VISC, k_prims4<<<cdiv(b.L.cs, 256), 256, 0, c->stream>>>(U, b.p4, b.L, ph));
+        const int64_t ni = (int64_t)b.g.n[0] * b.g.n[1] * b.g.n[2];
+        LAUNCH(c, K_VISC, k_visc_exp<<<cdiv(ni, 128), 128, 0, c->stream>>>(b.p4, M, b.met2, b.racc, b.rcs, b.L, ph));
+    } else if (vdiv) {
         const unsigned nt = (unsigned)(((b.g.n[0] + DTX - 1) / DTX) * ((b.g.n[1] + DTY - 1) / DTY) *
                                        ((b.g.n[2] + DK - 1) / DK));
         LAUNCH(c, K_VISC, k_visc_div<<<nt, DNT, VDIV_SMEM, c->stream>>>(U, M, b.racc, b.rcs, b.L, ph));
@@ -988,7 +1037,7 @@ static crocco_status rhs_block(crocco_ctx c, const LocalBlock &b, const double *
         a.rcs = b.rcs;
         a.inv = inviscid && (ph.dir_mask >> d & 1);
         a.visc = viscous && !vdiv && !(zdiv && d == 2);
-        a.mode = d == 0 ? ((vdiv || (zdiv && zsw == 0)) ? 4 : 0) : (d == 1 ? 1 : final_mode);
+        a.mode = d == 0 ? ((vexp || vdiv || (zdiv && zsw == 0)) ? 4 : 0) : (d == 1 ? 1 : final_mode);
         a.RV = (zdiv && zsw != 0 && d == zsw) ? b.rv : nullptr;
         a.rhs = rhs;
         a.Uin = Uin;

@@ -82,8 +82,18 @@ class Solver:
 
     def _init_metrics(self):
         cc.crocco_init_metrics(self.ctx, self._ptrs(self._coords), self._ptrs(self.met))
+        if self.phys.visc_form == 1:     # expanded viscous form: the 18 second metrics
+            cc.crocco_init_metrics2(self.ctx, self._ptrs(self.met))
         self.sync()
         self._coords = None
+
+    def metrics2(self, b):
+        """(18, n2, n1, n0) second metrics of local block b (expanded viscous form; tests)."""
+        L = self.layouts[b]
+        out = torch.empty((18, L.n[2], L.n[1], L.n[0]), dtype=torch.float64, device=self.device)
+        cc.crocco_copy_metrics2(self.ctx, b, out.data_ptr())
+        self.sync()
+        return out
 
     def set_state(self, U_blocks, interior=True):
         """U_blocks[b]: numpy/torch conserved state, interior (5, n2, n1, n0) or padded."""
@@ -178,8 +188,11 @@ class Solver:
         return cc.crocco_compute_dt(self.ctx, self._ptrs(self.U), self._ptrs(self.met), cfl)
 
     def set_phys(self, phys):
+        switch = phys.visc_form == 1 and self.phys.visc_form != 1
         self.phys = phys
         cc.crocco_set_phys(self.ctx, phys)
+        if switch:
+            cc.crocco_init_metrics2(self.ctx, self._ptrs(self.met))
 
     def sync(self):
         cc.crocco_sync(self.ctx)
