@@ -210,31 +210,68 @@ class Solver:
 
 
 class AmrSolver:
-    """Two-level hierarchy (DESIGN readings 24-26): a coarse Solver and a fine
-    Solver whose faces inside the coarse domain are BC_COARSE_FINE, fine node 0 at coarse node
-    c0 (ratio 2, node-centred).  step() follows Algorithm 2: per stage the
-    coarse level, then the fine level with its C/F ghosts interpolated from the coarse stage
-    input, then AverageDown at the third stage.  Plumbing only -- the C ABI does every step."""
+    """Two-level hierarchy (DESIGN readings 24-26): a coarse Solver and one or
+    more fine patches (Solvers whose faces inside the coarse domain are BC_COARSE_FINE), patch p's
+    fine node 0 at coarse node c0[p] (ratio 2, node-centred).  step() follows Algorithm 2
+    (PAPER.md:102-119): per stage the coarse level, then every patch of the fine level with its
+    C/F ghosts interpolated from the coarse stage input, then AverageDown at the third stage.
+    Patches of the same level must be disjoint with no patch's ghost band (4 fine points)
+    reaching into another patch's interior: each patch's ghosts come from the coarse level only
+    (touching patches would need a same-level exchange between them, not built).  Plumbing only
+    -- the C ABI does every step."""
 
-    def __init__(self, coarse: Solver, fine: Solver, c0):
-        self.coarse, self.fine, self.c0 = coarse, fine, tuple(int(x) for x in c0)
-        cc.crocco_amr_link(fine.ctx, coarse.ctx, self.c0)
+    def __init__(self, coarse: Solver, fine, c0):
+        fines = list(fine) if isinstance(fine, (list, tuple)) else [fine]
+        c0s = [tuple(int(x) for x in c) for c in c0] if isinstance(fine, (list, tuple)) else \
+            [tuple(int(x) for x in c0)]
+        if len(fines) != len(c0s):
+            raise ValueError("one c0 per fine patch")
+        self.coarse = coarse
+        self.patches = list(zip(fines, c0s))
+        self.fine, self.c0 = self.patches[0]
+        self._check_disjoint()
+        for F, c in self.patches:
+            cc.crocco_amr_link(F.ctx, coarse.ctx, c)
+
+    def _box(self, F, c, grow):
+        """Fine-level index box [lo, hi) of a patch in the common fine index space (2x coarse);
+        a direction a PERIODIC patch spans is the whole axis (None)."""
+        out = []
+        for d in range(3):
+            if F.desc.bc[d][0] == cc.BC_PERIODIC:
+                out.append(None)
+            else:
+                out.append((2 * c[d] - grow, 2 * c[d] + F.desc.n_global[d] + grow))
+        return out
+
+    def _check_disjoint(self):
+        G4 = cc.GHOST
+        for a in range(len(self.patches)):
+            for b in range(len(self.patches)):
+                if a == b:
+                    continue
+                A = self._box(*self.patches[a], G4)
+                B = self._box(*self.patches[b], 0)
+                if all(x is None or y is None or (x[0] < y[1] and y[0] < x[1]) for x, y in zip(A, B)):
+                    raise ValueError(f"fine patches {a} and {b} overlap or touch within the ghost band")
 
     def fill_fine(self):
-        """FillPatchTwoLevels of the current fine state from the current coarse state."""
-        cc.crocco_fill_patch_two_levels(self.fine.ctx, self.fine._ptrs(self.fine.U),
-                                        self.fine._ptrs(self.fine.met), self.coarse._ptrs(self.coarse.U))
+        """FillPatchTwoLevels of every patch's current state from the current coarse state."""
+        for F, _ in self.patches:
+            cc.crocco_fill_patch_two_levels(F.ctx, F._ptrs(F.U), F._ptrs(F.met), self.coarse._ptrs(self.coarse.U))
 
     def average_down(self):
-        cc.crocco_average_down(self.fine.ctx, self.fine._ptrs(self.fine.U), self.coarse._ptrs(self.coarse.U))
+        for F, _ in self.patches:
+            cc.crocco_average_down(F.ctx, F._ptrs(F.U), self.coarse._ptrs(self.coarse.U))
 
     def stage(self, s, dt):
-        C, F = self.coarse, self.fine
+        C = self.coarse
         Uc_in = C.U
         C.stage(s, dt)                                   # fills Uc_in's ghosts, writes C.V; swaps
-        cc.crocco_amr_rk_stage(F.ctx, s, dt, F._ptrs(F.U), F._ptrs(F.V), F._ptrs(F.dU), F._ptrs(F.met),
-                               C._ptrs(Uc_in))
-        F.U, F.V = F.V, F.U
+        for F, _ in self.patches:
+            cc.crocco_amr_rk_stage(F.ctx, s, dt, F._ptrs(F.U), F._ptrs(F.V), F._ptrs(F.dU), F._ptrs(F.met),
+                                   C._ptrs(Uc_in))
+            F.U, F.V = F.V, F.U
         if s == 2:
             self.average_down()
 
@@ -243,8 +280,10 @@ class AmrSolver:
             for s in range(3):
                 self.stage(s, dt)
             self.coarse.set_time(self.coarse.time + dt)
-            self.fine.set_time(self.fine.time + dt)
+            for F, _ in self.patches:
+                F.set_time(F.time + dt)
 
     def sync(self):
         self.coarse.sync()
-        self.fine.sync()
+        for F, _ in self.patches:
+            F.sync()

@@ -206,6 +206,71 @@ def test_full_size_amr_bench_config_bitwise():
     F.close()
 
 
+def test_two_disjoint_fine_patches_parity():
+    """Same-level multi-patch (NEXT-4): two disjoint fine patches on one coarse level, each its
+    own ctx.  Reference: the pinned oracle functions composed in Algorithm 2's order (per stage
+    the coarse stage, then every patch's FillPatchTwoLevels + RHS + update, AverageDown of every
+    patch at the third stage)."""
+    from paper_conf_ipps_davissngmb23_b200 import crocco as cc
+    from paper_conf_ipps_davissngmb23_b200.solver import AmrSolver, Solver
+    nc = (32, 24, 16)
+    grid = synth.Wavy3D(L=(10.0,) * 3, N=nc)
+    phys = dict(terms=3, mu_ref=0.01)
+    ph = oracle.phys(**phys)
+    patches = [((2, 3, 2), (16, 16, 12), (1, 1, 1)), ((18, 6, 3), (20, 24, 16), (2, 2, 1))]
+    bcf = ((CF, CF),) * 3
+    st = lambda x: synth.vortex(x)
+    xc = grid.coords(nc, (0, 0, 0), oracle.GC)
+    metc = oracle.metrics(nc, PER, xc)
+    Uc = synth.pad_state(st(xc))
+    P = []
+    for c0, nf, _ in patches:
+        xf = synth.Refined(grid, c0).coords(nf, (0, 0, 0), oracle.GC)
+        P.append([c0, nf, oracle.metrics(nf, bcf, xf), synth.pad_state(st(xf))])
+    dt, nsteps = 0.01, 4
+    # oracle reference (composition of pinned functions, Alg. 2 order)
+    Vc, dUc = Uc.copy(), np.zeros_like(Uc)
+    ref = [[U.copy(), U.copy(), np.zeros_like(U)] for _, _, _, U in P]   # a, o, dU
+    ac, oc = Uc.copy(), Vc
+    for _ in range(nsteps):
+        for s in range(3):
+            oracle.rk_stage(nc, PER, ph, s, dt, ac, oc, dUc, metc)
+            for (c0, nf, metf, _), R in zip(P, ref):
+                oracle.fill_two_levels(nf, bcf, R[0], nc, c0, ac)
+                r = oracle.rhs(nf, ph, R[0], metf)
+                oracle.rk_update(nf, s, dt, R[0], R[1], R[2], r)
+                if s == 2:
+                    oracle.average_down(nf, bcf, R[1], nc, c0, oc)
+                R[0], R[1] = R[1], R[0]
+            ac, oc = oc, ac
+    # GPU
+    C = Solver(nc, (2, 2, 1), PER, cc.make_phys(**phys))
+    bn, blocks = block_slices(nc, (2, 2, 1))
+    C.set_coords([grid.coords(bn, o, oracle.GC) for o, _ in blocks])
+    C.set_state([np.ascontiguousarray(st(xc)[(slice(None),) + sl]) for _, sl in blocks])
+    Fs = []
+    for (c0, nf, nb), (_, _, _, U0) in zip(patches, P):
+        F = Solver(nf, nb, bcf, cc.make_phys(**phys))
+        bnf, bl = block_slices(nf, nb)
+        F.set_coords([synth.Refined(grid, c0).coords(bnf, o, oracle.GC) for o, _ in bl])
+        Ui = U0[:, G:-G, G:-G, G:-G]
+        F.set_state([np.ascontiguousarray(Ui[(slice(None),) + sl]) for _, sl in bl])
+        Fs.append(F)
+    A = AmrSolver(C, Fs, [p[0] for p in patches])
+    A.step(dt, nsteps)
+    A.sync()
+    for S, n, nb, r in [(C, nc, (2, 2, 1), ac)] + [(F, p[1], p[2], R[0]) for F, p, R in zip(Fs, patches, ref)]:
+        _, _, refs = _blocks_of(r, n, nb)
+        for g, rr in zip(S.get(S.U), refs):
+            ri = rr[:, G:-G, G:-G, G:-G]
+            assert rel_linf(g[:, G:-G, G:-G, G:-G], ri, state_scale(ri)) <= 1e-9
+    with pytest.raises(ValueError):               # patches touching within the ghost band
+        AmrSolver(C, Fs, [(2, 3, 2), (11, 6, 3)])
+    C.close()
+    for F in Fs:
+        F.close()
+
+
 def test_amr_abi_refusals():
     from paper_conf_ipps_davissngmb23_b200 import crocco as cc
     from paper_conf_ipps_davissngmb23_b200.solver import AmrSolver, Solver
