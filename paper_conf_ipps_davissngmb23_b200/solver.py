@@ -287,3 +287,55 @@ class AmrSolver:
         self.coarse.sync()
         for F, _ in self.patches:
             F.sync()
+
+
+class AmrHierarchy:
+    """Multi-level hierarchy (the paper's DMR runs "three-level curvilinear AMR", PAPER.md:195;
+    SURVEY NEXT-4; DESIGN readings 24-26, 29).  levels[0] is the base Solver; levels[k] (k >= 1)
+    is a list of (Solver, parent, c0): a patch of level k whose fine node 0 sits at node c0 of
+    patch `parent` of level k-1 (ratio 2 between consecutive levels; the base level has the
+    single "patch" 0).  A level-k patch is an ordinary fine ctx whose coarse level is its
+    parent -- crocco_amr_link composes, since the parent's ghosts (its own C/F faces included)
+    are filled by the parent's stage before the child interpolates from them.
+    stage() follows Algorithm 2 literally: for each level n = 0..nlevels in
+    ascending order, FillPatch + RHS + Update of every patch of level n, and at the third stage
+    AverageDown of level n onto level n-1 right after level n's update (reading 29)."""
+
+    def __init__(self, base: Solver, levels):
+        self.levels = [[(base, None, None)]] + [list(lv) for lv in levels]
+        for k in range(1, len(self.levels)):
+            for S, parent, c0 in self.levels[k]:
+                P = self.levels[k - 1][parent][0]
+                cc.crocco_amr_link(S.ctx, P.ctx, tuple(int(x) for x in c0))
+
+    def stage(self, s, dt):
+        prev_in = None
+        for k, lv in enumerate(self.levels):
+            cur_in = []
+            for S, parent, _ in lv:
+                U_in = S.U
+                if k == 0:
+                    S.stage(s, dt)                       # fills U_in's ghosts, writes S.V; swaps
+                else:
+                    cc.crocco_amr_rk_stage(S.ctx, s, dt, S._ptrs(S.U), S._ptrs(S.V), S._ptrs(S.dU),
+                                           S._ptrs(S.met), prev_in[parent])
+                    S.U, S.V = S.V, S.U
+                cur_in.append(S._ptrs(U_in))
+            if s == 2 and k >= 1:                        # AverageDown of level k onto level k-1
+                for S, parent, _ in lv:
+                    P = self.levels[k - 1][parent][0]
+                    cc.crocco_average_down(S.ctx, S._ptrs(S.U), P._ptrs(P.U))
+            prev_in = cur_in
+
+    def step(self, dt, nsteps=1):
+        for _ in range(nsteps):
+            for s in range(3):
+                self.stage(s, dt)
+            for lv in self.levels:
+                for S, _, _ in lv:
+                    S.set_time(S.time + dt)
+
+    def sync(self):
+        for lv in self.levels:
+            for S, _, _ in lv:
+                S.sync()

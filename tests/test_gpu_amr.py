@@ -271,6 +271,69 @@ def test_two_disjoint_fine_patches_parity():
         F.close()
 
 
+def test_three_level_hierarchy_parity():
+    """Three levels (the paper's DMR runs three-level AMR): level 2 is a patch of
+    level 1, which is a patch of level 0.  Reference: the pinned oracle functions composed in
+    Algorithm 2's literal order (reading 29): per stage, level by level, FillPatch + RHS + update,
+    and at the third stage AverageDown of level n onto n-1 right after level n's update."""
+    from paper_conf_ipps_davissngmb23_b200 import crocco as cc
+    from paper_conf_ipps_davissngmb23_b200.solver import AmrHierarchy, Solver
+    n0 = (24, 24, 16)
+    g0 = synth.Wavy3D(L=(10.0,) * 3, N=n0)
+    c01, n1 = (4, 5, 2), (28, 24, 20)           # level 1 in level-0 index space
+    c12, n2 = (6, 4, 5), (24, 24, 16)           # level 2 in level-1 index space
+    g1 = synth.Refined(g0, c01)
+    g2 = synth.Refined(g1, c12)
+    bcf = ((CF, CF),) * 3
+    phys = dict(terms=3, mu_ref=0.01)
+    ph = oracle.phys(**phys)
+    st = lambda x: synth.vortex(x)
+    lv = []
+    for n, g, bc in ((n0, g0, PER), (n1, g1, bcf), (n2, g2, bcf)):
+        x = g.coords(n, (0, 0, 0), oracle.GC)
+        lv.append([n, g, bc, oracle.metrics(n, bc, x), synth.pad_state(st(x))])
+    oracle.fill(n0, PER, lv[0][4])
+    dt, nsteps = 0.005, 3
+    A = [L[4].copy() for L in lv]
+    O = [L[4].copy() for L in lv]
+    D = [np.zeros_like(L[4]) for L in lv]
+    c0s = [None, c01, c12]
+    for _ in range(nsteps):
+        for s in range(3):
+            for k in range(3):
+                n, _, bc, met, _ = lv[k]
+                if k == 0:
+                    oracle.rk_stage(n, PER, ph, s, dt, A[0], O[0], D[0], met)
+                else:
+                    oracle.fill_two_levels(n, bc, A[k], lv[k - 1][0], c0s[k], A[k - 1])
+                    r = oracle.rhs(n, ph, A[k], met)
+                    oracle.rk_update(n, s, dt, A[k], O[k], D[k], r)
+                    if s == 2:
+                        oracle.average_down(n, bc, O[k], lv[k - 1][0], c0s[k], O[k - 1])
+            for k in range(3):
+                A[k], O[k] = O[k], A[k]
+    # GPU (multi-block levels)
+    nbs = [(2, 2, 1), (2, 1, 2), (1, 2, 1)]
+    S = []
+    for (n, g, bc, _, U0), nb in zip(lv, nbs):
+        X = Solver(n, nb, bc, cc.make_phys(**phys))
+        bn, bl = block_slices(n, nb)
+        X.set_coords([g.coords(bn, o, oracle.GC) for o, _ in bl])
+        Ui = U0[:, G:-G, G:-G, G:-G]
+        X.set_state([np.ascontiguousarray(Ui[(slice(None),) + sl]) for _, sl in bl])
+        S.append(X)
+    H = AmrHierarchy(S[0], [[(S[1], 0, c01)], [(S[2], 0, c12)]])
+    H.step(dt, nsteps)
+    H.sync()
+    for X, (n, *_), nb, ref in zip(S, lv, nbs, A):
+        _, _, refs = _blocks_of(ref, n, nb)
+        for gg, rr in zip(X.get(X.U), refs):
+            ri = rr[:, G:-G, G:-G, G:-G]
+            assert rel_linf(gg[:, G:-G, G:-G, G:-G], ri, state_scale(ri)) <= 1e-9
+    for X in S:
+        X.close()
+
+
 def test_amr_abi_refusals():
     from paper_conf_ipps_davissngmb23_b200 import crocco as cc
     from paper_conf_ipps_davissngmb23_b200.solver import AmrSolver, Solver
