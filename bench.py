@@ -296,10 +296,7 @@ def run_crocco(args, rank, world, local_rank):
     ms = float(t.item())
     value = pts_total * 3 * args.steps / (ms / 1e3)
     # state sanity (finite, positive density) -- not part of the timed region
-    finite = True
-    for bl in range(S.nloc):
-        Ui = S.view(S.U[bl], bl, 5)[:, 4:-4, 4:-4, 4:-4]
-        finite = finite and bool(torch.isfinite(Ui).all().item()) and float(Ui[0].min().item()) > 0
+    finite = S.check_state() == 0   # crocco_check_state: no non-finite value, rho, p > 0
 
     # ---------------- end-to-end through the public API with host buffers
     e2e = None
@@ -474,7 +471,7 @@ def run_amr(args):
     pts = nc[0] * nc[1] * nc[2] + nf[0] * nf[1] * nf[2]
     value = pts * 3 * args.steps / (ms / 1e3)
     amr_ms = sum(v["ms"] for k, v in kt.items() if k.endswith(":amr"))
-    finite = all(bool(torch.isfinite(S.view(S.U[0], 0, 5)[:, 4:-4, 4:-4, 4:-4]).all().item()) for S in (C, F))
+    finite = all(S.check_state() == 0 for S in (C, F))
     # C/F interpolation and AverageDown: HBM gathers; algorithmic bytes = 5 comps x 8 B written per
     # C/F ghost point (+ the coarse corners read once, 1/8 of that) and 27+1 fine/coarse values per
     # covered coarse point -- reported as a share of the step, not as a roofline (they are < 1 %)

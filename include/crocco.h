@@ -274,6 +274,11 @@ crocco_status crocco_amr_rk_stage(crocco_ctx fine, int32_t stage, double dt, dou
    points only) becomes the full-weighting (trapezoid) average of the fine data over its cell. */
 crocco_status crocco_average_down(crocco_ctx fine, double *const *U_fine, double *const *U_coarse);
 
+/* State check (SURVEY sec. 5 failure detection; test / bench utility): *n_bad = number of
+   interior points of all local blocks with a non-finite component, rho <= 0 or p <= 0
+   (p from the ctx's gamma).  n_bad: HOST pointer.  Synchronises the stream.  Not collective. */
+crocco_status crocco_check_state(crocco_ctx ctx, double *const *U, int64_t *n_bad);
+
 /* Block until all work of the ctx finished; surfaces asynchronous errors. */
 crocco_status crocco_sync(crocco_ctx ctx);
 const char *crocco_last_error(crocco_ctx ctx);

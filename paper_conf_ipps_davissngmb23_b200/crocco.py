@@ -94,6 +94,7 @@ _SIGS = {
     "crocco_rk3_step": [C.c_void_p, C.c_double, DPP, DPP, DPP, DPP, C.c_int32],
     "crocco_amr_link": [C.c_void_p, C.c_void_p, C.POINTER(C.c_int64)],
     "crocco_init_metrics2": [C.c_void_p, DPP],
+    "crocco_check_state": [C.c_void_p, DPP, C.POINTER(C.c_int64)],
     "crocco_copy_metrics2": [C.c_void_p, C.c_int32, C.c_void_p],
     "crocco_fill_patch_two_levels": [C.c_void_p, DPP, DPP, DPP],
     "crocco_amr_rk_stage": [C.c_void_p, C.c_int32, C.c_double, DPP, DPP, DPP, DPP, DPP],
@@ -359,3 +360,11 @@ def crocco_init_metrics2(ctx, met_ptrs):
 
 def crocco_copy_metrics2(ctx, b, dst_ptr):
     _check(lib().crocco_copy_metrics2(ctx, int(b), C.c_void_p(int(dst_ptr))), ctx)
+
+
+def crocco_check_state(ctx, U_ptrs) -> int:
+    """Interior points with a non-finite component, rho <= 0 or p <= 0 (synchronises)."""
+    a, ka = _ptrs(U_ptrs)
+    n = C.c_int64()
+    _check(lib().crocco_check_state(ctx, a, C.byref(n)), ctx)
+    return int(n.value)

@@ -6,6 +6,7 @@
 // numerical step runs in the CUDA kernels, never on the host.
 #include <cuda_runtime.h>
 #include <nccl.h>
+#include <nvtx3/nvToolsExt.h>
 
 #include <algorithm>
 #include <cstdarg>
@@ -56,6 +57,12 @@ const char *k_names[K_NCLASS] = {"prims", "sweep_xi", "sweep_eta", "sweep_zeta_u
                                  "update", "fill", "metrics", "compute_dt", "amr"};
 // internal fill kind: 5-component state, periodic / inter-block copies only (AverageDown)
 enum { FILL_STATE_COPIES = 100 };
+
+// NVTX range of a host-side region (tracing): visible in nsys / ncu --nvtx
+struct NvtxRange {
+    explicit NvtxRange(const char *name) { nvtxRangePushA(name); }
+    ~NvtxRange() { nvtxRangePop(); }
+};
 
 struct TimedLaunch {
     int cls;
@@ -814,6 +821,7 @@ static crocco_status fill_phase(crocco_ctx c, double *const *f, int kind, int D,
     }
     st = flush_ops(c, ops);
     if (st) return st;
+    NvtxRange nv("crocco:nccl_halo");
     NK(c, ncclGroupStart());
     for (size_t r = 0; r < remote.size(); r++) {
         const crocco_msg &m = *remote[r];
@@ -859,6 +867,7 @@ static crocco_status check_ptrs(crocco_ctx c, double *const *p, const char *what
 }
 
 static crocco_status fill_all(crocco_ctx c, double *const *f, int32_t kind, double *const *met, double t) {
+    NvtxRange nv(c->amr_Uc ? "crocco:fill_two_levels" : "crocco:fill");
     if (kind != CROCCO_FIELD_STATE && kind != CROCCO_FIELD_METRIC && kind != FILL_STATE_COPIES)
         return fail(c, CROCCO_ERR_ARG, "bad field kind");
     crocco_status st = check_ptrs(c, f, "field");
@@ -1080,6 +1089,7 @@ static crocco_status rhs_block(crocco_ctx c, const LocalBlock &b, const double *
 
 crocco_status crocco_rhs(crocco_ctx c, double *const *U, double *const *M, double *const *rhs) {
     LIVE(c);
+    NvtxRange nv("crocco:rhs");
     crocco_status st;
     if ((st = check_ptrs(c, U, "U")) || (st = check_ptrs(c, M, "metrics")) ||
         (st = check_ptrs(c, rhs, "rhs")))
@@ -1096,6 +1106,7 @@ crocco_status crocco_rhs(crocco_ctx c, double *const *U, double *const *M, doubl
 crocco_status crocco_rk_stage(crocco_ctx c, int32_t stage, double dt, double *const *Uin,
                               double *const *Uout, double *const *dU, double *const *M) {
     LIVE(c);
+    NvtxRange nv("crocco:rk_stage");
     crocco_status st;
     if (stage < 0 || stage > 2) return fail(c, CROCCO_ERR_ARG, "stage must be 0..2");
     if ((st = check_ptrs(c, Uin, "U_in")) || (st = check_ptrs(c, Uout, "U_out")) ||
@@ -1383,6 +1394,7 @@ crocco_status crocco_amr_rk_stage(crocco_ctx f, int32_t stage, double dt, double
 
 crocco_status crocco_average_down(crocco_ctx f, double *const *Uf, double *const *Uc) {
     LIVE(f);
+    NvtxRange nv("crocco:average_down");
     crocco_status st = amr_ready(f, Uc);
     if (st) return st;
     if ((st = check_ptrs(f, Uf, "U_fine"))) return st;
@@ -1426,6 +1438,26 @@ crocco_status crocco_average_down(crocco_ctx f, double *const *Uf, double *const
         if (ops.nops == CF_MAX_OPS && (st = flush())) return st;
     }
     return flush();
+}
+
+crocco_status crocco_check_state(crocco_ctx c, double *const *U, int64_t *n_bad) {
+    LIVE(c);
+    crocco_status st = check_ptrs(c, U, "U");
+    if (st) return st;
+    if (!n_bad) return fail(c, CROCCO_ERR_ARG, "null n_bad");
+    if (!c->dmax) CK(c, cudaMalloc((void **)&c->dmax, sizeof(unsigned long long)));
+    CK(c, cudaMemsetAsync(c->dmax, 0, sizeof(unsigned long long), c->stream));
+    for (size_t bi = 0; bi < c->loc.size(); bi++) {
+        const LocalBlock &b = c->loc[bi];
+        const int64_t tot = (int64_t)b.g.n[0] * b.g.n[1] * b.g.n[2];
+        const unsigned grid = (unsigned)std::min<int64_t>(cdiv(tot, 256), 148 * 8);
+        LAUNCH(c, K_CFL, k_check_state<<<grid, 256, 0, c->stream>>>(U[bi], b.L, c->ph, c->dmax));
+    }
+    unsigned long long h = 0;
+    CK(c, cudaMemcpyAsync(&h, c->dmax, sizeof h, cudaMemcpyDeviceToHost, c->stream));
+    CK(c, cudaStreamSynchronize(c->stream));
+    *n_bad = (int64_t)h;
+    return CROCCO_OK;
 }
 
 crocco_status crocco_sync(crocco_ctx c) {

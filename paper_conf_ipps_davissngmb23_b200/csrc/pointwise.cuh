@@ -773,6 +773,26 @@ __global__ void __launch_bounds__(256) k_cfl(const double *__restrict__ U, const
 }
 
 // Update alone, from a materialised rhs (crocco_rk_update).
+// state check (SURVEY sec. 5 failure detection, a test / bench utility): count interior
+// points with a non-finite component, rho <= 0 or p <= 0
+__global__ void __launch_bounds__(256) k_check_state(const double *__restrict__ U, Lay L, const Phys ph,
+                                                     unsigned long long *bad) {
+    const int64_t tot = (int64_t)L.n0 * L.n1 * L.n2;
+    unsigned cnt = 0;
+    for (int64_t t = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; t < tot; t += (int64_t)gridDim.x * blockDim.x) {
+        const int i = (int)(t % L.n0);
+        const int64_t r = t / L.n0;
+        const int64_t p = at(L, i, (int)(r % L.n1), (int)(r / L.n1));
+        const double rho = U[p], mx = U[L.cs + p], my = U[2 * L.cs + p], mz = U[3 * L.cs + p], E = U[4 * L.cs + p];
+        const double pr = ph.gm1 * (E - 0.5 * (mx * mx + my * my + mz * mz) / rho);
+        const bool ok = isfinite(rho) && isfinite(mx) && isfinite(my) && isfinite(mz) && isfinite(E) &&
+                        rho > 0.0 && pr > 0.0;
+        cnt += ok ? 0u : 1u;
+    }
+    for (int o = 16; o > 0; o >>= 1) cnt += __shfl_down_sync(0xffffffffu, cnt, o);
+    if ((threadIdx.x & 31) == 0 && cnt) atomicAdd(bad, (unsigned long long)cnt);
+}
+
 __global__ void __launch_bounds__(256) k_update(const double *__restrict__ Uin,
                                                 double *__restrict__ Uout, double *__restrict__ dU,
                                                 const double *__restrict__ rhs, Lay L, int stage,

@@ -183,6 +183,10 @@ class Solver:
                 ev_d[n].record(self._d2h)
         comp.wait_stream(self._d2h)
 
+    def check_state(self):
+        """Number of interior points with a non-finite value, rho <= 0 or p <= 0 (crocco_check_state)."""
+        return cc.crocco_check_state(self.ctx, self._ptrs(self.U))
+
     def compute_dt(self, cfl):
         """ComputeDt (Alg. 1 l.9): CFL time step of the current state (synchronises)."""
         return cc.crocco_compute_dt(self.ctx, self._ptrs(self.U), self._ptrs(self.met), cfl)

@@ -496,3 +496,19 @@ def test_compute_dt_sod_closed_form():
     S.close()
     expect = 0.9 / (3 * math.sqrt(1.4) * 200)
     assert abs(got - expect) < 1e-12 * expect
+
+
+# ------------------------------------------------------------------ state check
+
+def test_check_state_counts_bad_points():
+    n = (20, 16, 12)
+    pb = wavy_random(n, 9)
+    S = pb.solver((2, 1, 1))
+    assert S.check_state() == 0
+    v = S.view(S.U[0], 0, 5)
+    v[0, 4 + 3, 4 + 2, 4 + 1] = float("nan")          # non-finite
+    v[0, 4 + 5, 4 + 6, 4 + 7] = -1.0                  # rho <= 0
+    v[4, 4 + 1, 4 + 1, 4 + 1] = 0.0                   # E = 0 -> p < 0
+    v[1, 0, 0, 0] = float("inf")                      # a ghost point: not counted
+    assert S.check_state() == 3
+    S.close()
