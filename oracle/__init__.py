@@ -109,6 +109,8 @@ def lib():
         L.oracle_compute_dt.argtypes = [i64p, C.POINTER(Phys), dp, dp, C.c_double]
         L.oracle_compute_dt.restype = C.c_double
         L.oracle_fill_two_levels.argtypes = [i64p, i32p, dp, dp, dp, i64p, i64p, dp]
+        L.oracle_fill_two_levels_ex.argtypes = [i64p, i32p, dp, C.POINTER(Split), C.c_double, dp, dp, i64p,
+                                                i64p, dp]
         L.oracle_average_down.argtypes = [i64p, i32p, dp, dp, i64p, i64p, dp]
         L.oracle_amr_advance.argtypes = [i64p, i32p, dp, i64p, i32p, dp, i64p, C.POINTER(Phys),
                                          C.c_double, C.c_int32, dp, dp, dp, dp]
@@ -215,10 +217,12 @@ def rk_update(n, stage, dt, Uin, Uout, dU, r):
     lib().oracle_rk_update(_n(n), stage, dt, _dp(Uin), _dp(Uout), _dp(dU), _dp(r))
 
 
-def rk_stage(n, bc, ph, stage, dt, Uin, Uout, dU, met, dirichlet=None):
+def rk_stage(n, bc, ph, stage, dt, Uin, Uout, dU, met, dirichlet=None, split=None, t=0.0):
+    """One RK stage (fill at t + c_s dt, RHS, update); t = start of the step."""
     d = _dir(dirichlet)
-    lib().oracle_rk_stage(_n(n), _bc(bc), _dp(d), C.byref(ph), stage, dt, _dp(Uin), _dp(Uout),
-                          _dp(dU), _dp(met))
+    sp = split if split is not None else splits()
+    lib().oracle_rk_stage_ex(_n(n), _bc(bc), _dp(d), sp, float(t), C.byref(ph), stage, dt, _dp(Uin),
+                             _dp(Uout), _dp(dU), _dp(met))
 
 
 def advance(n, bc, ph, dt, nsteps, U, met, dirichlet=None, split=None, t0=0.0):
@@ -235,12 +239,15 @@ def compute_dt(n, ph: Phys, U, met, cfl):
 
 
 # ---- two-level AMR (oracle section 9, readings 24-26) ----
-def fill_two_levels(nf, bcf, Uf, nc, c0, Uc, dirichlet=None, met=None):
+def fill_two_levels(nf, bcf, Uf, nc, c0, Uc, dirichlet=None, met=None, split=None, t=0.0):
     """FillPatchTwoLevels in place on the fine state Uf: the three-phase fill with COARSE_FINE
-    faces interpolated (trilinear, ratio 2, node-centred) from the coarse state Uc (ghosts filled)."""
+    faces interpolated (trilinear, ratio 2, node-centred) from the coarse state Uc (ghosts filled);
+    the fine level's own physical faces (SPLIT data at time t, SLIPWALL with met) as in fill()."""
     d = _dir(dirichlet)
     mp = _dp(met) if met is not None else None
-    lib().oracle_fill_two_levels(_n(nf), _bc(bcf), _dp(d), mp, _dp(Uf), _n(nc), _n(c0), _dp(Uc))
+    sp = split if split is not None else splits()
+    lib().oracle_fill_two_levels_ex(_n(nf), _bc(bcf), _dp(d), sp, float(t), mp, _dp(Uf), _n(nc), _n(c0),
+                                    _dp(Uc))
     return Uf
 
 

@@ -1132,9 +1132,9 @@ static void cf_interp(const oracle_amr *a, const int64_t f[3], double v[5])
 
 /* FillPatch of a fine level (Alg. 2 l.3-4 at level 1): the three-phase fill of section 1
    with COARSE_FINE faces interpolated from the coarse state Uc (ghosts filled). */
-void oracle_fill_two_levels(const int64_t nf[3], const int32_t bcf[6], const double dirichlet[30],
-                            const double *metf, double *Uf, const int64_t nc[3],
-                            const int64_t c0[3], const double *Uc)
+void oracle_fill_two_levels_ex(const int64_t nf[3], const int32_t bcf[6], const double dirichlet[30],
+                               const oracle_split *split, double t, const double *metf, double *Uf,
+                               const int64_t nc[3], const int64_t c0[3], const double *Uc)
 {
     oracle_amr a;
     for (int d = 0; d < 3; d++) {
@@ -1142,7 +1142,14 @@ void oracle_fill_two_levels(const int64_t nf[3], const int32_t bcf[6], const dou
         a.c0[d] = c0[d];
     }
     a.Uc = Uc;
-    fill_core(nf, bcf, dirichlet, NULL, 0.0, metf, Uf, 5, O_FIELD_STATE, &a);
+    fill_core(nf, bcf, dirichlet, split, t, metf, Uf, 5, O_FIELD_STATE, &a);
+}
+
+void oracle_fill_two_levels(const int64_t nf[3], const int32_t bcf[6], const double dirichlet[30],
+                            const double *metf, double *Uf, const int64_t nc[3],
+                            const int64_t c0[3], const double *Uc)
+{
+    oracle_fill_two_levels_ex(nf, bcf, dirichlet, NULL, 0.0, metf, Uf, nc, c0, Uc);
 }
 
 /* AverageDown (Alg. 2 l.10-12; "sets covered coarse AMR cells to be equal to the

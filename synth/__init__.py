@@ -356,6 +356,33 @@ def dmr_bc(h, gamma=1.4):
     return bc, dirichlet, split
 
 
+def refine_bc(n_coarse, bc, dirichlet, split, c0, nf, cf=6):
+    """Boundary data of a ratio-2 fine patch (fine node f at coarse index c0 + f/2, DESIGN reading
+    24): a face on the domain boundary keeps the coarse kind and data, a face inside the domain is
+    COARSE_FINE (6), a periodic direction the patch spans (nf = 2 n) stays PERIODIC.  SPLIT data
+    along an axis move to the fine index space: the coarse rule g + 1/2 < s_c at position c0 + f/2
+    reads f + 1/2 < 2 (s_c - c0) - 1/2, so i0_f = 2 (i0 - c0_axis) - 1/2 and di_dt_f = 2 di_dt."""
+    bcf, spf = [], {}
+    dirf = np.zeros((3, 2, 5)) if dirichlet is None else np.array(dirichlet, dtype=float).copy()
+    for d in range(3):
+        if bc[d][0] == P:
+            if nf[d] != 2 * n_coarse[d] or c0[d] != 0:
+                raise ValueError("a patch in a periodic direction must span it (nf = 2 n, c0 = 0)")
+            bcf.append((P, P))
+            continue
+        lo = bc[d][0] if c0[d] == 0 else cf
+        hi = bc[d][1] if 2 * c0[d] + nf[d] - 1 == 2 * (n_coarse[d] - 1) else cf
+        bcf.append((lo, hi))
+        for side, kind in ((0, lo), (1, hi)):
+            if kind == SPL:
+                sp = dict(split[(d, side)])
+                ax = sp["axis"]
+                sp["i0"] = 2.0 * (sp["i0"] - c0[ax]) - 0.5
+                sp["di_dt"] = 2.0 * sp["di_dt"]
+                spf[(d, side)] = sp
+    return tuple(bcf), dirf, spf
+
+
 def case(name: str, scale: int = 1) -> Case:
     """Configs of BASELINE.json; ``scale`` divides the grid for parity runs."""
     if name == "sod":

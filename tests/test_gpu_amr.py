@@ -334,6 +334,77 @@ def test_three_level_hierarchy_parity():
         X.close()
 
 
+def _dmr_hierarchy(scale, patches):
+    """The paper's DMR with a three-level hierarchy: base grid of
+    synth.case("dmr", scale), then patches (c0, nf, nblocks) of levels 1, 2 (each inside the
+    previous one) with their boundary data from synth.refine_bc."""
+    c = synth.case("dmr", scale=scale)
+    n0 = c.n_global
+    h = 1.0 / n0[1]
+    bc0, dv0, sp0 = synth.dmr_bc(h)
+    levels = [dict(n=n0, grid=c.grid, bc=bc0, dir=dv0, split=sp0, nb=c.n_blocks, c0=None)]
+    for c0, nf, nb in patches:
+        up = levels[-1]
+        bcf, dvf, spf = synth.refine_bc(up["n"], up["bc"], up["dir"], up["split"], c0, nf)
+        levels.append(dict(n=nf, grid=synth.Refined(up["grid"], c0), bc=bcf, dir=dvf, split=spf, nb=nb, c0=c0))
+    return c, levels
+
+
+def test_three_level_dmr_parity():
+    """DMR with three levels on the GPU (SLIPWALL and moving SPLIT faces on the fine patches at the
+    wall, C/F faces elsewhere) against the oracle functions composed in Alg. 2's order."""
+    from paper_conf_ipps_davissngmb23_b200 import crocco as cc
+    from paper_conf_ipps_davissngmb23_b200.solver import AmrHierarchy, Solver
+    c, L = _dmr_hierarchy(16, [((2, 0, 0), (128, 24, 16), (2, 1, 2)), ((4, 0, 0), (64, 16, 32), (1, 1, 2))])
+    ph = oracle.phys(**c.phys)
+    h2 = 1.0 / c.n_global[1] / 4
+    dt, nsteps = 0.2 * h2 / 13.0, 4
+    for lv in L:
+        x = lv["grid"].coords(lv["n"], (0, 0, 0), oracle.GC)
+        lv["met"] = oracle.metrics(lv["n"], lv["bc"], x)
+        lv["U0"] = synth.dmr_state(x)
+        lv["sp"] = oracle.splits(lv["split"])
+    A = [synth.pad_state(lv["U0"]) for lv in L]
+    O = [a.copy() for a in A]
+    D = [np.zeros_like(a) for a in A]
+    t = 0.0
+    for _ in range(nsteps):
+        for s in range(3):
+            ts = t + (0.0, 1.0 / 3.0, 3.0 / 4.0)[s] * dt
+            for k, lv in enumerate(L):
+                if k == 0:
+                    oracle.rk_stage(lv["n"], lv["bc"], ph, s, dt, A[0], O[0], D[0], lv["met"],
+                                    dirichlet=lv["dir"], split=lv["sp"], t=t)
+                else:
+                    oracle.fill_two_levels(lv["n"], lv["bc"], A[k], L[k - 1]["n"], lv["c0"], A[k - 1],
+                                           dirichlet=lv["dir"], met=lv["met"], split=lv["sp"], t=ts)
+                    r = oracle.rhs(lv["n"], ph, A[k], lv["met"])
+                    oracle.rk_update(lv["n"], s, dt, A[k], O[k], D[k], r)
+                    if s == 2:
+                        oracle.average_down(lv["n"], lv["bc"], O[k], L[k - 1]["n"], lv["c0"], O[k - 1])
+            for k in range(len(L)):
+                A[k], O[k] = O[k], A[k]
+        t = t + dt
+    S = []
+    for lv in L:
+        X = Solver(lv["n"], lv["nb"], lv["bc"], cc.make_phys(**c.phys), dirichlet=lv["dir"], split=lv["split"])
+        bn, bl = block_slices(lv["n"], lv["nb"])
+        X.set_coords([lv["grid"].coords(bn, o, oracle.GC) for o, _ in bl])
+        X.set_state([np.ascontiguousarray(lv["U0"][(slice(None),) + sl]) for _, sl in bl])
+        S.append(X)
+    H = AmrHierarchy(S[0], [[(S[1], 0, L[1]["c0"])], [(S[2], 0, L[2]["c0"])]])
+    H.step(dt, nsteps)
+    H.sync()
+    for X, lv, ref in zip(S, L, A):
+        _, _, refs = _blocks_of(ref, lv["n"], lv["nb"])
+        for gg, rr in zip(X.get(X.U), refs):
+            ri = rr[:, G:-G, G:-G, G:-G]
+            assert rel_linf(gg[:, G:-G, G:-G, G:-G], ri, state_scale(ri)) <= 1e-9
+        assert X.check_state() == 0
+    for X in S:
+        X.close()
+
+
 def test_amr_abi_refusals():
     from paper_conf_ipps_davissngmb23_b200 import crocco as cc
     from paper_conf_ipps_davissngmb23_b200.solver import AmrSolver, Solver

@@ -208,3 +208,33 @@ def test_two_level_vortex_more_accurate_on_fine_patch():
     assert exf[fsl].shape == exc[csl].shape
     assert err_fine < 0.5 * err_coarse, (err_fine, err_coarse)
     assert err_comp < err_coarse, (err_comp, err_coarse)
+
+
+def test_refined_dmr_split_faces_follow_the_physical_rule():
+    """DMR boundary data on a fine patch at the bottom wall (synth.refine_bc, reading 20 + 24): the
+    fine bottom ghosts take the post-shock state exactly where the ghost's physical x < 1/6 (the
+    coarse rule re-expressed in the fine index space), slip-wall reflections elsewhere; the top
+    face inside the domain is C/F."""
+    n = (96, 32, 4)
+    h = 1.0 / n[1]
+    bc, dv, spec = synth.dmr_bc(h)
+    grid = synth.Cartesian(h=(h,) * 3)
+    c0, nf = (2, 0, 0), (40, 20, 8)
+    bcf, dirf, splf = synth.refine_bc(n, bc, dv, spec, c0, nf)
+    assert bcf == ((CF, CF), (synth.SPL, CF), (0, 0))
+    xf = synth.Refined(grid, c0).coords(nf, (0, 0, 0), oracle.GC)
+    metf = oracle.metrics(nf, bcf, xf)
+    Uf = synth.pad_state(synth.random_state(nf, seed=12))
+    Uc = synth.pad_state(synth.random_state(n, seed=13))
+    oracle.fill(n, bc, Uc, dirichlet=dv, split=oracle.splits(spec), met=oracle.metrics(n, bc, grid.coords(n, (0, 0, 0), oracle.GC)))
+    oracle.fill_two_levels(nf, bcf, Uf, n, c0, Uc, dirichlet=dirf, met=metf, split=oracle.splits(splf), t=0.0)
+    post = np.array(synth.prim_to_cons(*[np.float64(a) for a in synth.DMR_POST]))
+    x = (c0[0] + 0.5 * np.arange(-G, nf[0] + G) + 0.5) * h      # physical x of the fine columns
+    for g in range(1, G + 1):                                      # bottom ghost rows j = -g
+        row = Uf[:, G:-G, G - g, :]                                # (5, k, i)
+        is_post = np.all(np.isclose(row, post[:, None, None], rtol=0, atol=0), axis=(0, 1))
+        assert np.array_equal(is_post[G:-G], x[G:-G] < 1.0 / 6.0)
+        mirror = Uf[:, G:-G, G + g - 1, :]
+        slip = ~(x < 1.0 / 6.0)
+        assert np.array_equal(row[0][:, slip], mirror[0][:, slip])                 # rho mirrored
+        assert np.array_equal(row[2][:, slip], -mirror[2][:, slip])                # v reflected
