@@ -50,6 +50,9 @@ WORKLOADS = {
     "sod": "sod: Sod shock tube 200x4x4, inviscid (configs[0])",
     "dmr": "dmr: double Mach reflection 2048x512x128 in 2x2x1 blocks, slip wall + moving shock BCs "
            "(the paper's case, PAPER.md:183-185; SURVEY NEXT-2)",
+    "dmr_amr": "dmr_amr: the paper's DMR on a three-level hierarchy (PAPER.md:185, 195): base 1024x256x64 "
+               "(2x2x1 blocks) + level-1 patch 1280x128x128 along the wall + level-2 patch 1280x128x256 "
+               "around the reflection, ratio 2, slip wall / moving-shock SPLIT faces on every level",
     "amr": "amr: two-level hierarchy (SURVEY NEXT-4): TGV 256^3 coarse level on the wavy grid + a "
            "256^3-node fine level (ratio 2) over its central 128^3 region, C/F faces all round, viscous",
 }
@@ -490,6 +493,89 @@ def run_amr(args):
     return 0
 
 
+def run_dmr_amr(args):
+    """--config dmr_amr (one GPU): Algorithm 2 over three levels (AmrHierarchy): per stage the base
+    DMR grid, the level-1 and level-2 patches (C/F ghosts from the parent's stage input, DMR
+    boundary data on the wall faces), AverageDown of each level after its third-stage update.
+    value = (all levels' interior points) x 3 x steps / time.  Also reports the point count of the
+    equivalent uniform finest grid (the paper's AMR-savings measure)."""
+    import torch
+
+    import synth
+    from paper_conf_ipps_davissngmb23_b200 import crocco as cc
+    from paper_conf_ipps_davissngmb23_b200.solver import AmrHierarchy, Solver
+
+    dev = torch.device("cuda", 0)
+    torch.cuda.set_device(dev)
+    c = synth.case("dmr", scale=2)
+    n0 = c.n_global
+    h = 1.0 / n0[1]
+    bc0, dv0, sp0 = synth.dmr_bc(h)
+    specs = [(n0, c.grid, bc0, dv0, sp0, c.n_blocks, None)]
+    for c0, nf, nb in (((128, 0, 0), (1280, 128, 128), (2, 1, 1)), ((320, 0, 0), (1280, 128, 256), (2, 1, 2))):
+        n_up, g_up, bc_up, dv_up, sp_up = specs[-1][:5]
+        bcf, dvf, spf = synth.refine_bc(n_up, bc_up, dv_up, sp_up, c0, nf)
+        specs.append((nf, synth.Refined(g_up, c0), bcf, dvf, spf, nb, c0))
+    phys = cc.make_phys(**c.phys)
+    S = []
+    for n, g, bc, dv, sp, nb, _ in specs:
+        X = Solver(n, nb, bc, phys, dirichlet=dv, split=sp, device=dev)
+        for bl in range(X.nloc):
+            L = X.layouts[bl]
+            xyz = g.coords(tuple(L.n), tuple(L.origin), cc.GHOST_COORDS)
+            X.set_coords_block(bl, xyz)
+            X.set_state_block(bl, synth.dmr_state(xyz))
+        S.append(X)
+    H = AmrHierarchy(S[0], [[(S[1], 0, specs[1][6])], [(S[2], 0, specs[2][6])]])
+    dt = 0.2 * (h / 4) / 13.0
+    for _ in range(args.warmup):
+        H.step(dt)
+    torch.cuda.synchronize()
+    for X in S:
+        cc.crocco_set_timing(X.ctx, True)
+        cc.crocco_kernel_times(X.ctx)
+        cc.crocco_launch_count(X.ctx, reset=True)
+    clk = ClockSampler(0) if not args.no_clocks else None
+    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    torch.cuda.synchronize()
+    e0.record(S[0].stream)
+    H.step(dt, args.steps)
+    e1.record(S[0].stream)
+    torch.cuda.synchronize()
+    ms = e0.elapsed_time(e1)
+    clocks = clk.stop() if clk else None
+    launches = sum(cc.crocco_launch_count(X.ctx) for X in S)
+    kt = {}
+    for lv, X in enumerate(S):
+        for k, (nl, kms) in cc.crocco_kernel_times(X.ctx).items():
+            if nl:
+                kt[f"level{lv}:{k}"] = {"launches": nl, "ms": kms}
+    ktot = sum(v["ms"] for v in kt.values())
+    for v in kt.values():
+        v["share_of_kernel_time"] = v["ms"] / max(ktot, 1e-9)
+    pts = [n[0] * n[1] * n[2] for n, *_ in specs]
+    uniform = n0[0] * n0[1] * n0[2] * 64                      # finest spacing h/4 everywhere
+    value = sum(pts) * 3 * args.steps / (ms / 1e3)
+    finite = all(X.check_state() == 0 for X in S)
+    out = {"metric": METRIC, "value": value, "unit": UNIT, "n_gpus": 1, "steps": args.steps,
+           "warmup": args.warmup, "ms_per_step": ms / args.steps, "higher_is_better": True,
+           "scaling": "strong", "vs_baseline": None, "dtype": "f64",
+           "data": "synthetic (Woodward-Colella DMR initial state on every level, DESIGN.md sec. 4)",
+           "config": {"workload": WORKLOADS["dmr_amr"] + "; step = 1 RK3 step (3 stages x 3 levels + AverageDown)",
+                      "levels": [{"n": list(n), "c0": list(c0) if c0 else None, "blocks": list(nb), "points": p}
+                                 for (n, _, _, _, _, nb, c0), p in zip(specs, pts)],
+                      "points": sum(pts), "uniform_finest_points": uniform,
+                      "amr_point_saving": 1.0 - sum(pts) / uniform, "dt": dt,
+                      "l2": "inputs larger than L2", "parallelism": "1 GPU"},
+           "amr_kernels_share": sum(v["ms"] for k, v in kt.items() if k.endswith(":amr")) / max(ktot, 1e-9),
+           "kernel_breakdown": kt, "gpu_launches": launches, "clocks": clocks, "state_finite": finite,
+           "impl": "crocco"}
+    for X in S:
+        X.close()
+    print(json.dumps(out), flush=True)
+    return 0
+
+
 def _profiled_traffic(kname):
     """dram bytes per launch of the dominant kernel from the committed ncu summary, if any."""
     p = os.path.join(ROOT, "profiles", "ncu_summary.json")
@@ -510,7 +596,8 @@ def main():
     ap.add_argument("--steps", type=int, default=5)
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--impl", choices=["crocco", "reference"], default="crocco")
-    ap.add_argument("--config", choices=["weak", "ramp", "tgv", "vortex", "sod", "dmr", "amr"], default="weak",
+    ap.add_argument("--config", choices=["weak", "ramp", "tgv", "vortex", "sod", "dmr", "amr", "dmr_amr"],
+                    default="weak",
                     help="weak (default, the north_star 512^3/GPU workload) or a fixed BASELINE config")
     ap.add_argument("--e2e-steps", type=int, default=16,
                     help="independent jobs streamed through host memory for e2e (pipeline fill + drain amortised)")
@@ -523,10 +610,10 @@ def main():
     local_rank = int(os.environ.get("LOCAL_RANK", "0"))
     if args.impl == "reference":
         return run_reference(args, rank, world)
-    if args.config == "amr":
+    if args.config in ("amr", "dmr_amr"):
         if world > 1:
-            raise SystemExit("--config amr runs on one GPU")
-        return run_amr(args)
+            raise SystemExit(f"--config {args.config} runs on one GPU")
+        return run_amr(args) if args.config == "amr" else run_dmr_amr(args)
     if world > 1:
         import torch
         import torch.distributed as dist
