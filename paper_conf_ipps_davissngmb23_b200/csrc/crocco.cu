@@ -1317,7 +1317,12 @@ crocco_status crocco_amr_link(crocco_ctx f, crocco_ctx c, const int64_t c0[3]) {
             return fail(f, CROCCO_ERR_ARG, "direction %d: a physical hi face must lie on the domain boundary", d);
         if (nf < 3) return fail(f, CROCCO_ERR_ARG, "direction %d: fine level needs >= 3 points", d);
     }
-    for (int d = 0; d < 3; d++) f->amr_c0[d] = c0[d];
+    int64_t c0_prev[3];
+    for (int d = 0; d < 3; d++) {
+        c0_prev[d] = f->amr_c0[d];
+        f->amr_c0[d] = c0[d];  // covered_range() reads it; restored below on failure
+    }
+    crocco_status st = CROCCO_OK;
     // locality: every coarse block a fine ghost interpolates from, and every fine block a
     // covered coarse node averages, lives on this rank (no inter-level communication)
     for (const LocalBlock &b : f->loc) {
@@ -1331,9 +1336,9 @@ crocco_status crocco_amr_link(crocco_ctx f, crocco_ctx c, const int64_t c0[3]) {
         for (int64_t z = lo[2]; z <= hi[2]; z++)
             for (int64_t y = lo[1]; y <= hi[1]; y++)
                 for (int64_t x = lo[0]; x <= hi[0]; x++)
-                    if (c->gid_to_local[x + c->nb[0] * (y + c->nb[1] * z)] < 0)
-                        return fail(f, CROCCO_ERR_ARG,
-                                    "fine block %d interpolates from a coarse block on another rank", b.g.gid);
+                    if (st == CROCCO_OK && c->gid_to_local[x + c->nb[0] * (y + c->nb[1] * z)] < 0)
+                        st = fail(f, CROCCO_ERR_ARG,
+                                  "fine block %d interpolates from a coarse block on another rank", b.g.gid);
     }
     for (const LocalBlock &b : c->loc) {
         int64_t lo[3], hi[3];
@@ -1352,9 +1357,13 @@ crocco_status crocco_amr_link(crocco_ctx f, crocco_ctx c, const int64_t c0[3]) {
         for (int64_t z = lo[2]; z <= hi[2]; z++)
             for (int64_t y = lo[1]; y <= hi[1]; y++)
                 for (int64_t x = lo[0]; x <= hi[0]; x++)
-                    if (f->gid_to_local[x + f->nb[0] * (y + f->nb[1] * z)] < 0)
-                        return fail(f, CROCCO_ERR_ARG,
-                                    "coarse block %d averages down from a fine block on another rank", b.g.gid);
+                    if (st == CROCCO_OK && f->gid_to_local[x + f->nb[0] * (y + f->nb[1] * z)] < 0)
+                        st = fail(f, CROCCO_ERR_ARG,
+                                  "coarse block %d averages down from a fine block on another rank", b.g.gid);
+    }
+    if (st != CROCCO_OK) {
+        for (int d = 0; d < 3; d++) f->amr_c0[d] = c0_prev[d];
+        return st;
     }
     f->amr_coarse = c;
     return CROCCO_OK;

@@ -69,6 +69,7 @@ def test_invalid_desc_is_err_arg(kw, frag):
     (dict(weno_limiter=4), "weno_limiter"),
     (dict(weno_limiter=1, weno_alpha_rl=-1.0), "thresholds"),
     (dict(weno_weights=2), "weno_weights"),
+    (dict(visc_form=2), "visc_form"),
 ])
 def test_invalid_phys_is_err_arg(kw, frag):
     d = cc.make_desc((8, 8, 8))
@@ -136,3 +137,33 @@ def test_plan_is_identical_across_ranks_for_shared_messages():
                 if m.kind == 0:
                     assert m.src_rank == br[m.src_block]
                     assert r in (m.src_rank, m.dst_rank)
+
+
+def test_plan_marks_coarse_fine_faces_physical():
+    """A fine AMR level (CROCCO_BC_COARSE_FINE faces, NEXT-4) gets no copy message across a C/F
+    face: those ghosts belong to the two-level fill (host plan, no GPU needed)."""
+    CF = cc.BC_COARSE_FINE
+    d = cc.make_desc((16, 8, 8), (2, 1, 1), ((CF, CF), (CF, CF), (0, 0)))
+    xi = cc.crocco_exchange_plan(d, 0)
+    outer = [m for m in xi if (m.dst_block == 0 and m.side == 0) or (m.dst_block == 1 and m.side == 1)]
+    inner = [m for m in xi if m not in outer]
+    assert len(outer) == 2 and all(m.kind == 1 and m.src_block == -1 and m.bc_kind == CF for m in outer)
+    assert len(inner) == 2 and all(m.kind == 0 for m in inner)      # same-level copy between blocks
+    for m in cc.crocco_exchange_plan(d, 1):                         # eta: both faces C/F, no copies
+        assert m.kind == 1 and m.src_block == -1
+
+
+def test_amr_patch_separation_check_host_logic():
+    """AmrSolver refuses same-level patches whose ghost band reaches another patch (host logic)."""
+    from types import SimpleNamespace as NS
+    from paper_conf_ipps_davissngmb23_b200.solver import AmrSolver
+    CF = cc.BC_COARSE_FINE
+
+    def patch(n):
+        return NS(desc=NS(bc=((CF, CF), (CF, CF), (0, 0)), n_global=n))
+    A = AmrSolver.__new__(AmrSolver)
+    A.patches = [(patch((16, 16, 8)), (2, 2, 0)), (patch((16, 16, 8)), (14, 2, 0))]
+    A._check_disjoint()                                      # x: [4,20)+-4 vs [28,44): apart
+    A.patches[1] = (patch((16, 16, 8)), (11, 2, 0))          # [22,38) within 4 of [4,20)
+    with pytest.raises(ValueError):
+        A._check_disjoint()
