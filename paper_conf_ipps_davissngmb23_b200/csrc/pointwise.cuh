@@ -300,11 +300,21 @@ __global__ void __launch_bounds__(VTX * VTY, CROCCO_VISC_MINB) k_visc_tiled(cons
     ld_own(k0 + 2, cO);
     ld_halo(k0, cH);
     ld_met(k0, cM);
+#if CROCCO_VISC_PREFETCH >= 2
+    // distance 2: the operands of plane k+1 are already in flight when plane k starts
+    double mO[5], mH[5], mM[10];
+    {
+        const int k1n = min(k0 + 1, k1 - 1);
+        ld_own(k1n + 2, mO);
+        ld_halo(k1n, mH);
+        ld_met(k1n, mM);
+    }
+#endif
 #endif
     for (int k = k0; k < k1; k++) {
 #if CROCCO_VISC_PREFETCH
         double nO[5], nH[5], nM[10];
-        const int kn = min(k + 1, k1 - 1);  // clamp: the last step reloads its own plane
+        const int kn = min(k + CROCCO_VISC_PREFETCH, k1 - 1);  // clamp: the last steps reload
         ld_own(kn + 2, nO);
         ld_halo(kn, nH);
         ld_met(kn, nM);
@@ -435,7 +445,20 @@ __global__ void __launch_bounds__(VTX * VTY, CROCCO_VISC_MINB) k_visc_tiled(cons
             }
 #endif
         }
-#if CROCCO_VISC_PREFETCH
+#if CROCCO_VISC_PREFETCH >= 2
+#pragma unroll
+        for (int c = 0; c < 5; c++) {
+            cO[c] = mO[c];
+            cH[c] = mH[c];
+            mO[c] = nO[c];
+            mH[c] = nH[c];
+        }
+#pragma unroll
+        for (int c = 0; c < 10; c++) {
+            cM[c] = mM[c];
+            mM[c] = nM[c];
+        }
+#elif CROCCO_VISC_PREFETCH
 #pragma unroll
         for (int c = 0; c < 5; c++) {
             cO[c] = nO[c];

@@ -89,9 +89,10 @@ def _check_padded(S, bufs, ref_glob, n, nb, exact=True, tol=0.0, floor=0.0):
             assert rel_linf(g[:, G:-G, G:-G, G:-G], r[:, G:-G, G:-G, G:-G], floor) <= tol
 
 
-@pytest.mark.parametrize("nbc,nbf", [((1, 1, 1), (1, 1, 1)), ((2, 2, 2), (2, 2, 1)), ((3, 1, 2), (1, 2, 3))])
-def test_fill_patch_two_levels_bitwise(nbc, nbf):
-    nc, c0, nf = (24, 20, 16), (3, 4, 2), (20, 16, 12)
+@pytest.mark.parametrize("nbc,nbf,nf", [((1, 1, 1), (1, 1, 1), (20, 16, 12)), ((2, 2, 2), (2, 2, 1), (20, 16, 12)),
+                                        ((3, 1, 2), (1, 2, 3), (20, 16, 12)), ((2, 2, 1), (1, 1, 1), (17, 13, 11))])
+def test_fill_patch_two_levels_bitwise(nbc, nbf, nf):
+    nc, c0 = (24, 20, 16), (3, 4, 2)
     h = Hier(nc, c0, nf, ((CF, CF),) * 3, synth.Wavy3D(L=(10.0,) * 3, N=nc), dict(terms=3, mu_ref=0.02))
     metc, Uc, metf, Uf = h.oracle()
     oracle.fill_two_levels(nf, h.bcf, Uf, nc, c0, Uc)
@@ -118,14 +119,15 @@ def test_fill_patch_two_levels_mixed_faces_bitwise():
     F.close()
 
 
-@pytest.mark.parametrize("bcf,nf,c0", [(((CF, CF),) * 3, (18, 14, 12), (2, 3, 1)),
-                                       (((CF, CF), (CF, CF), (0, 0)), (18, 14, 16), (2, 3, 0))])
-def test_average_down_bitwise(bcf, nf, c0):
+@pytest.mark.parametrize("bcf,nf,c0,nbf", [(((CF, CF),) * 3, (18, 14, 12), (2, 3, 1), (2, 1, 2)),
+                                           (((CF, CF), (CF, CF), (0, 0)), (18, 14, 16), (2, 3, 0), (2, 1, 2)),
+                                           (((CF, CF),) * 3, (17, 13, 12), (3, 2, 1), (1, 1, 3))])
+def test_average_down_bitwise(bcf, nf, c0, nbf):
     nc = (16, 12, 8)
     h = Hier(nc, c0, nf, bcf, synth.Wavy3D(L=(10.0,) * 3, N=nc), dict(terms=3, mu_ref=0.02))
     metc, Uc, metf, Uf = h.oracle()
     oracle.average_down(nf, bcf, Uf, nc, c0, Uc)
-    C, F, A = h.gpu((2, 2, 1), (2, 1, 2))
+    C, F, A = h.gpu((2, 2, 1), nbf)
     A.average_down()
     bn, blocks, refs = _blocks_of(Uc, nc, (2, 2, 1))
     for g, r in zip(C.get(C.U), refs):
