@@ -339,6 +339,11 @@ class AmrHierarchy:
                 for S, _, _ in lv:
                     S.set_time(S.time + dt)
 
+    def compute_dt(self, cfl):
+        """ComputeDt over the whole hierarchy (Alg. 1 l.9; every patch iterates with the same dt,
+        PAPER.md:131): the minimum of every patch's crocco_compute_dt."""
+        return min(S.compute_dt(cfl) for lv in self.levels for S, _, _ in lv)
+
     def sync(self):
         for lv in self.levels:
             for S, _, _ in lv:

@@ -395,6 +395,10 @@ def test_three_level_dmr_parity():
         X.set_state([np.ascontiguousarray(lv["U0"][(slice(None),) + sl]) for _, sl in bl])
         S.append(X)
     H = AmrHierarchy(S[0], [[(S[1], 0, L[1]["c0"])], [(S[2], 0, L[2]["c0"])]])
+    # ComputeDt over the hierarchy = min over levels (the finest level binds: spacing h/4)
+    dts = [oracle.compute_dt(lv["n"], ph, synth.pad_state(lv["U0"]), lv["met"], 0.5) for lv in L]
+    assert abs(H.compute_dt(0.5) - min(dts)) <= 1e-13 * min(dts)
+    assert min(dts) == dts[2]
     H.step(dt, nsteps)
     H.sync()
     for X, lv, ref in zip(S, L, A):
