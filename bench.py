@@ -386,7 +386,10 @@ def run_crocco(args, rank, world, local_rank):
                 "flops_per_unit": FLUX_FLOPS_PER_IFACE, "unit_of_work": "interface flux",
                 "units_per_launch": ifaces, "avg_launch_ms": avg_ms,
                 "traffic": _profiled_traffic(f"k_sweep_s<{d},"),
-                "traffic_source": "profiles/ncu_summary.json (ncu --set full, dram__bytes_read+write per launch)"}
+                "fp64_pipe_active_pct": _profiled_traffic(f"k_sweep_s<{d},", "fp64_pipe_pct"),
+                "achieved_occupancy_pct": _profiled_traffic(f"k_sweep_s<{d},", "achieved_occupancy_pct"),
+                "traffic_source": "profiles/ncu_summary.json (ncu --set full, dram__bytes_read+write per launch; "
+                                  "sm__pipe_fp64_cycles_active and achieved occupancy of the same capture)"}
     peaks = measured_peaks()
     hbm = peaks.get("hbm_gbs", 6650.0)
     stage_gbs = value / world * HBM_BYTES_PER_PT_STAGE / 1e9
@@ -576,15 +579,16 @@ def run_dmr_amr(args):
     return 0
 
 
-def _profiled_traffic(kname):
-    """dram bytes per launch of the dominant kernel from the committed ncu summary, if any."""
+def _profiled_traffic(kname, key="dram_bytes_per_launch"):
+    """A per-launch ncu figure (default: dram bytes) of the dominant kernel from the committed
+    ncu summary (profiles/ncu_summary.json), if any."""
     p = os.path.join(ROOT, "profiles", "ncu_summary.json")
     try:
         with open(p) as f:
             ks = json.load(f).get("kernels", {})
         for k, v in ks.items():  # kname: full kernel name or a prefix of it
-            if k.startswith(kname) and "dram_bytes_per_launch" in v:
-                return v["dram_bytes_per_launch"]
+            if k.startswith(kname) and key in v:
+                return v[key]
         return None
     except Exception:
         return None
