@@ -411,6 +411,27 @@ def test_three_level_dmr_parity():
         X.close()
 
 
+def test_two_level_overlapped_stage_equals_serial_bitwise():
+    """The fine level's C/F interpolation also runs inside the overlapped stage (fill on the
+    comm stream beside the ghost-free viscous tiles): forcing the overlap on gives the serial
+    result bit for bit."""
+    from paper_conf_ipps_davissngmb23_b200 import crocco as cc
+    nc, c0, nf = (32, 24, 80), (4, 5, 2), (40, 20, 136)   # fine level has ghost-free viscous tiles
+    outs = []
+    for ov in (0, 1):
+        h = Hier(nc, c0, nf, ((CF, CF),) * 3, synth.Wavy3D(L=(10.0,) * 3, N=nc), dict(terms=3, mu_ref=0.01),
+                 state="vortex")
+        C, F, A = h.gpu((1, 1, 1), (1, 1, 1))
+        cc.crocco_set_overlap(F.ctx, ov)
+        cc.crocco_set_overlap(C.ctx, ov)
+        A.step(0.005, 2)
+        A.sync()
+        outs.append([C.get(C.U)[0], F.get(F.U)[0]])
+        C.close()
+        F.close()
+    assert np.array_equal(outs[0][0], outs[1][0]) and np.array_equal(outs[0][1], outs[1][1])
+
+
 def test_amr_abi_refusals():
     from paper_conf_ipps_davissngmb23_b200 import crocco as cc
     from paper_conf_ipps_davissngmb23_b200.solver import AmrSolver, Solver
