@@ -55,6 +55,9 @@ def test_version():
     (dict(n_global=(8, 8, 8), bc=((0, 1), (0, 0), (0, 0))), "PERIODIC must be paired"),
     (dict(n_global=(8, 8, 8), nranks=2, rank=0), "block_rank"),
     (dict(n_global=(8, 8, 8), block_rank=[3], nranks=2), "out of range"),
+    (dict(n_global=(0, 8, 8)), "bad n_global"),                                   # empty domain
+    (dict(n_global=(70000, 8, 8)), "65535"),                                      # beyond the grid limits
+    (dict(n_global=(8, 8, 8), bc=((7, 7), (0, 0), (0, 0))), "bad bc kind"),
 ])
 def test_invalid_desc_is_err_arg(kw, frag):
     d = cc.make_desc(**kw)

@@ -512,3 +512,19 @@ def test_check_state_counts_bad_points():
     v[1, 0, 0, 0] = float("inf")                      # a ghost point: not counted
     assert S.check_state() == 3
     S.close()
+
+
+def test_degenerate_no_terms_is_exactly_stationary():
+    """terms = 0 (no inviscid, no viscous flux): the RHS is exactly zero and an RK stage
+    returns U_in bit for bit (dU = 0) -- the degenerate case of the method."""
+    n = (19, 13, 11)
+    pb = wavy_random(n, 4, phys=dict(terms=0))
+    S = pb.solver((1, 1, 1))
+    S.fill()
+    r = S.get(S.rhs())[0][:, 4:-4, 4:-4, 4:-4]
+    assert np.all(r == 0.0)
+    U0 = S.get(S.U)[0][:, 4:-4, 4:-4, 4:-4]
+    S.stage(0, 1e-2)
+    S.sync()
+    assert np.array_equal(S.get(S.U)[0][:, 4:-4, 4:-4, 4:-4], U0)
+    S.close()
