@@ -352,12 +352,17 @@ def _dmr_hierarchy(scale, patches):
     return c, levels
 
 
-def test_three_level_dmr_parity():
-    """DMR with three levels on the GPU (SLIPWALL and moving SPLIT faces on the fine patches at the
-    wall, C/F faces elsewhere) against the oracle functions composed in Alg. 2's order."""
+@pytest.mark.parametrize("patches", [
+    [((2, 0, 0), (128, 24, 16), (2, 1, 2)), ((4, 0, 0), (64, 16, 32), (1, 1, 2))],       # on the wall
+    [((6, 16, 0), (96, 31, 16), (2, 1, 1)), ((20, 14, 0), (80, 33, 32), (1, 1, 2))],     # under the moving top
+])
+def test_three_level_dmr_parity(patches):
+    """DMR with three levels on the GPU (SLIPWALL and the static / moving SPLIT faces of the bottom /
+    top boundary on the fine patches that touch them, C/F faces elsewhere) against the oracle
+    functions composed in Alg. 2's order."""
     from paper_conf_ipps_davissngmb23_b200 import crocco as cc
     from paper_conf_ipps_davissngmb23_b200.solver import AmrHierarchy, Solver
-    c, L = _dmr_hierarchy(16, [((2, 0, 0), (128, 24, 16), (2, 1, 2)), ((4, 0, 0), (64, 16, 32), (1, 1, 2))])
+    c, L = _dmr_hierarchy(16, patches)
     ph = oracle.phys(**c.phys)
     h2 = 1.0 / c.n_global[1] / 4
     dt, nsteps = 0.2 * h2 / 13.0, 4
