@@ -332,6 +332,7 @@ static void build_plan(const crocco_grid_desc *d, const int nb[3], const int bn[
 #ifndef CROCCO_ZDIV_SWEEP
 #define CROCCO_ZDIV_SWEEP 0  // 0: k_visc_tiled writes R, the xi sweep adds (measured equal to 1 / 2, no extra buffer)
 #endif
+static_assert(!CROCCO_VISC_XDIV || CROCCO_ZDIV_SWEEP == 0, "XDIV writes R from k_visc_tiled (ZDIV_SWEEP 0)");
 #ifndef CROCCO_SWEEP_SMEM
 #define CROCCO_SWEEP_SMEM 1  // shared-memory staged sweeps (k_sweep_s); 0: global-load sweeps
 #endif
@@ -542,8 +543,9 @@ crocco_status crocco_init_grid(const crocco_grid_desc *desc, const crocco_phys *
         ok = ok && alloc(&b.racc, 5 * b.rcs);
         ok = ok && (!(CROCCO_SWEEP_SMEM && !CROCCO_VISC_DIV && CROCCO_VISC_ZDIV && CROCCO_ZDIV_SWEEP) ||
                     alloc(&b.rv, 5 * b.rcs));
+        // point viscous fluxes kept in HBM: xi and eta (ZDIV), eta only (ZDIV + XDIV), all three otherwise
         ok = ok && ((CROCCO_SWEEP_SMEM && CROCCO_VISC_DIV) ||
-                    alloc(&b.fv, (CROCCO_SWEEP_SMEM && CROCCO_VISC_ZDIV ? 8 : 12) * b.V.cs));
+                    alloc(&b.fv, (CROCCO_SWEEP_SMEM && CROCCO_VISC_ZDIV ? (CROCCO_VISC_XDIV ? 4 : 8) : 12) * b.V.cs));
         if (!ok) {
             cudaGetLastError();
             free_ctx(c);
@@ -1018,7 +1020,7 @@ static crocco_status rhs_block(crocco_ctx c, const LocalBlock &b, const double *
 #if CROCCO_SWEEP_SMEM
         if (visc_sel != 1) {  // sel 1 (interior tiles) was launched by visc_interior() beside the fill
             const int nz = zdiv ? b.g.n[2] : b.V.b2;
-            int64_t nt = (int64_t)((b.V.b0 + VTX - 1) / VTX) * ((b.V.b1 + VTY - 1) / VTY) * ((nz + VK - 1) / VK);
+            int64_t nt = (int64_t)visc_tiles_x(b.L, b.V) * ((b.V.b1 + VTY - 1) / VTY) * ((nz + VK - 1) / VK);
             if (visc_sel == 2) {
                 const VTiles t = visc_interior_tiles(b.L);
                 nt -= (int64_t)(t.x1 - t.x0) * (t.y1 - t.y0) * (t.z1 - t.z0);
@@ -1038,14 +1040,16 @@ static crocco_status rhs_block(crocco_ctx c, const LocalBlock &b, const double *
         a.in.U = U;
         a.in.P = b.prim;
         a.in.M = M;
-        a.in.FV = b.fv + (int64_t)4 * d * b.V.cs;
+        // FV holds (xi, eta) point fluxes, or eta only with XDIV (the xi sweep then reads none)
+        const int fvd = (CROCCO_SWEEP_SMEM && CROCCO_VISC_ZDIV && CROCCO_VISC_XDIV) ? (d > 0 ? d - 1 : 0) : d;
+        a.in.FV = b.fv + (int64_t)4 * fvd * b.V.cs;
         a.in.cs = b.L.cs;
         a.in.vcs = b.V.cs;
         a.V = b.V;
         a.R = b.racc;
         a.rcs = b.rcs;
         a.inv = inviscid && (ph.dir_mask >> d & 1);
-        a.visc = viscous && !vdiv && !(zdiv && d == 2);
+        a.visc = viscous && !vdiv && !(zdiv && d == 2) && !(zdiv && CROCCO_VISC_XDIV && d == 0);
         a.mode = d == 0 ? ((vexp || vdiv || (zdiv && zsw == 0)) ? 4 : 0) : (d == 1 ? 1 : final_mode);
         a.RV = (zdiv && zsw != 0 && d == zsw) ? b.rv : nullptr;
         a.rhs = rhs;

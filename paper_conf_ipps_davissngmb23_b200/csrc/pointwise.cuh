@@ -125,17 +125,33 @@ __global__ void __launch_bounds__(256) k_visc(const double *__restrict__ Pm,
 #ifndef CROCCO_VISC_ZDIV
 #define CROCCO_VISC_ZDIV 1  // 1: D4_zeta of F^_v^zeta folded into k_visc_tiled (own-column queue) -> R
 #endif
+#ifndef CROCCO_VISC_XDIV
+#define CROCCO_VISC_XDIV 1  // 1: D4_xi of F^_v^xi also taken here (tiles overlap by 2-column arms), the xi sweep
+                            //    carries no viscous term and F^_v^xi never goes to HBM (requires ZDIV);
+                            //    measured -1.0..-1.5 ms per 512^3 stage with 32 x 8 tiles
+#endif
 #ifndef CROCCO_VISC_TX
-#define CROCCO_VISC_TX 16  // 16 x 8 tiles: two 4-warp CTAs per SM (measured 3 % faster than 32 x 8)
+// XDIV: 32 x 8 tiles (arms cost 4/28 = 14 %; 16 x 8 with 33 % arms measured slower, 24 x 8 slower still);
+// without XDIV: 16 x 8 tiles, two 4-warp CTAs per SM (measured 3 % faster than 32 x 8)
+#define CROCCO_VISC_TX (CROCCO_VISC_XDIV ? 32 : 16)
+#endif
+#ifndef CROCCO_VISC_TY
+#define CROCCO_VISC_TY 8
 #endif
 #ifndef CROCCO_VISC_VK
 #define CROCCO_VISC_VK (CROCCO_VISC_ZDIV ? 64 : 32)  // slab depth (ZDIV recomputes 4 planes per slab)
 #endif
-constexpr int VTX = CROCCO_VISC_TX, VTY = 8, VK = CROCCO_VISC_VK;  // tile and slab
+constexpr int VTX = CROCCO_VISC_TX, VTY = CROCCO_VISC_TY, VK = CROCCO_VISC_VK;  // tile and slab
+constexpr int VSX = CROCCO_VISC_XDIV ? VTX - 4 : VTX;  // tile stride in i (XDIV: 2-column arms each side)
 constexpr int VHX = VTX + 4, VHY = VTY + 4;          // with halo
 constexpr int VPL = VHX * VHY;                       // points per staged plane
 constexpr int VHALO = VPL - VTX * VTY;               // halo points per plane
-constexpr size_t VISC_SMEM = (size_t)2 * 4 * VPL * sizeof(double);
+constexpr size_t VISC_SMEM = (size_t)2 * 4 * VPL * sizeof(double) +
+                              (CROCCO_VISC_XDIV ? (size_t)2 * 4 * VTX * VTY * sizeof(double) : 0);
+// tiles in i of the viscous box (XDIV: central columns tile the interior [0, n0) with stride VSX)
+__host__ __device__ inline int visc_tiles_x(const Lay &L, const VLay &V) {
+    return CROCCO_VISC_XDIV ? (L.n0 + VSX - 1) / VSX : (V.b0 + VTX - 1) / VTX;
+}
 
 __device__ __forceinline__ void prim4(const double *__restrict__ U, int64_t cs, int64_t p, double gm1,
                                       double iR, double out[4]) {
@@ -157,9 +173,9 @@ struct VTiles {
 };
 __host__ __device__ inline VTiles visc_interior_tiles(const Lay &L) {
     VTiles t;
-    // x: loads i0-2 .. i0+VTX+1 with i0 = bx VTX - 2; y likewise; z: planes z0-4 .. z1+3
-    t.x0 = (4 + VTX - 1) / VTX;
-    t.x1 = (L.n0 - VTX) >= 0 ? (L.n0 - VTX) / VTX + 1 : 0;
+    // x: loads i0-2 .. i0+VTX+1 with i0 = bx VSX - 2; y likewise (stride VTY); z: planes z0-4 .. z1+3
+    t.x0 = (4 + VSX - 1) / VSX;
+    t.x1 = (L.n0 - VTX) >= 0 ? (L.n0 - VTX) / VSX + 1 : 0;
     t.y0 = (4 + VTY - 1) / VTY;
     t.y1 = (L.n1 - VTY) >= 0 ? (L.n1 - VTY) / VTY + 1 : 0;
     t.z0 = (4 + VK - 1) / VK;
@@ -179,7 +195,7 @@ __global__ void __launch_bounds__(VTX * VTY, CROCCO_VISC_MINB) k_visc_tiled(cons
     extern __shared__ double vsm[];  // [buffer 2][value 4][VPL]
     const int tid = threadIdx.x;
     const int tx = tid % VTX, ty = tid / VTX;
-    const int tilesx = (V.b0 + VTX - 1) / VTX, tilesy = (V.b1 + VTY - 1) / VTY;
+    const int tilesx = visc_tiles_x(L, V), tilesy = (V.b1 + VTY - 1) / VTY;
     int b = blockIdx.x;
     int bx, by, bz;
     const VTiles it = visc_interior_tiles(L);
@@ -225,7 +241,11 @@ __global__ void __launch_bounds__(VTX * VTY, CROCCO_VISC_MINB) k_visc_tiled(cons
         by = b % tilesy;
         bz = b / tilesy;
     }
-    const int i0 = bx * VTX - 2, j0 = by * VTY - 2;      // first output point of the tile
+    const int i0 = bx * VSX - 2, j0 = by * VTY - 2;      // first output point of the tile
+#if CROCCO_VISC_XDIV
+    double *fxs = vsm + 2 * 4 * VPL;  // [buffer 2][comp 4][VTX * VTY]: F^xi of the computed columns
+    double xq[4] = {0.0, 0.0, 0.0, 0.0};  // D4_xi F^xi of plane k-2 (computed in the previous step)
+#endif
 #if CROCCO_VISC_ZDIV
     // slab of interior output planes [z0, z1); gradients / point fluxes on planes z0-2 .. z1+1
     const int z0 = bz * VK, z1 = min(z0 + VK, L.n2);
@@ -242,6 +262,8 @@ __global__ void __launch_bounds__(VTX * VTY, CROCCO_VISC_MINB) k_visc_tiled(cons
     // own column (clamped into the padded box for the idle threads of edge tiles)
     const int i = i0 + tx, j = j0 + ty;
     const bool own = i < V.b0 - 2 && j < V.b1 - 2;
+    // the column whose outputs (F^eta, R) this thread writes: XDIV -> central columns only
+    const bool central = CROCCO_VISC_XDIV ? (tx >= 2 && tx < VTX - 2 && i < L.n0) : true;
     const int gi = min(i, L.n0 + G - 1), gj = min(j, L.n1 + G - 1);
     // halo point handled by this thread (tid < VHALO): rows j0-2, j0-1, j0+8, j0+9 (36 each),
     // then columns i0-2, i0-1, i0+32, i0+33 of rows j0..j0+7
@@ -359,6 +381,17 @@ __global__ void __launch_bounds__(VTX * VTY, CROCCO_VISC_MINB) k_visc_tiled(cons
         }
 #endif
         __syncthreads();
+#if CROCCO_VISC_XDIV
+        double xn[4] = {0.0, 0.0, 0.0, 0.0};  // D4_xi F^xi of plane k-1 (staged in the previous step)
+        if (central && k > k0) {
+            const double *fb = fxs + ((k - 1) & 1) * 4 * VTX * VTY + ty * VTX + tx;
+#pragma unroll
+            for (int q = 0; q < 4; q++) {
+                const double *c = fb + q * VTX * VTY;
+                xn[q] = fma(8.0, c[1] - c[-1], -(c[2] - c[-2])) * (1.0 / 12.0);
+            }
+        }
+#endif
         if (own) {
             double gc[4][3];
 #pragma unroll
@@ -412,6 +445,21 @@ __global__ void __launch_bounds__(VTX * VTY, CROCCO_VISC_MINB) k_visc_tiled(cons
 #if CROCCO_VISC_ZDIV
             // F^xi, F^eta of the interior planes to HBM (the xi / eta sweeps difference them);
             // F^zeta stays in the own column's queue and is differenced here (D4_zeta)
+#if CROCCO_VISC_XDIV
+            {   // F^xi of this column for the xi-divergence of the next step (shared memory only)
+                double *fb = fxs + (k & 1) * 4 * VTX * VTY + ty * VTX + tx;
+#pragma unroll
+                for (int a = 0; a < 3; a++)
+                    fb[a * VTX * VTY] = fma(m[0][0], tau[a][0], fma(m[0][1], tau[a][1], m[0][2] * tau[a][2]));
+                fb[3 * VTX * VTY] = fma(m[0][0], hb[0], fma(m[0][1], hb[1], m[0][2] * hb[2]));
+            }
+            if (k >= z0 && k < z1 && central) {  // F^eta only (the eta sweep differences it)
+#pragma unroll
+                for (int a = 0; a < 3; a++)
+                    FV[a * V.cs + o] = fma(m[1][0], tau[a][0], fma(m[1][1], tau[a][1], m[1][2] * tau[a][2]));
+                FV[3 * V.cs + o] = fma(m[1][0], hb[0], fma(m[1][1], hb[1], m[1][2] * hb[2]));
+            }
+#else
             if (k >= z0 && k < z1) {
 #pragma unroll
                 for (int d = 0; d < 2; d++) {
@@ -421,6 +469,7 @@ __global__ void __launch_bounds__(VTX * VTY, CROCCO_VISC_MINB) k_visc_tiled(cons
                     FV[(4 * d + 3) * V.cs + o] = fma(m[d][0], hb[0], fma(m[d][1], hb[1], m[d][2] * hb[2]));
                 }
             }
+#endif
 #pragma unroll
             for (int oq = 0; oq < 4; oq++)
 #pragma unroll
@@ -428,12 +477,17 @@ __global__ void __launch_bounds__(VTX * VTY, CROCCO_VISC_MINB) k_visc_tiled(cons
 #pragma unroll
             for (int a = 0; a < 3; a++) zq[4][a] = fma(m[2][0], tau[a][0], fma(m[2][1], tau[a][1], m[2][2] * tau[a][2]));
             zq[4][3] = fma(m[2][0], hb[0], fma(m[2][1], hb[1], m[2][2] * hb[2]));
-            if (k - 2 >= z0 && i >= 0 && i < L.n0 && j >= 0 && j < L.n1) {
+            if (k - 2 >= z0 && central && i >= 0 && i < L.n0 && j >= 0 && j < L.n1) {
                 const int64_t r = (int64_t)i + (int64_t)L.n0 * (j + (int64_t)L.n1 * (k - 2));
 #pragma unroll
-                for (int q = 0; q < 4; q++)
-                    R[(1 + q) * rcs + r] =
-                        fma(8.0, zq[3][q] - zq[1][q], -(zq[4][q] - zq[0][q])) * (1.0 / 12.0);
+                for (int q = 0; q < 4; q++) {
+                    const double zd = fma(8.0, zq[3][q] - zq[1][q], -(zq[4][q] - zq[0][q])) * (1.0 / 12.0);
+#if CROCCO_VISC_XDIV
+                    R[(1 + q) * rcs + r] = zd + xq[q];
+#else
+                    R[(1 + q) * rcs + r] = zd;
+#endif
+                }
             }
 #else
 #pragma unroll
@@ -445,6 +499,10 @@ __global__ void __launch_bounds__(VTX * VTY, CROCCO_VISC_MINB) k_visc_tiled(cons
             }
 #endif
         }
+#if CROCCO_VISC_XDIV
+#pragma unroll
+        for (int q = 0; q < 4; q++) xq[q] = xn[q];  // plane k-1 -> written with plane k-1's zeta term next step
+#endif
 #if CROCCO_VISC_PREFETCH >= 2
 #pragma unroll
         for (int c = 0; c < 5; c++) {
