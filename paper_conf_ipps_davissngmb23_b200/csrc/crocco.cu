@@ -333,6 +333,9 @@ static void build_plan(const crocco_grid_desc *d, const int nb[3], const int bn[
 #define CROCCO_ZDIV_SWEEP 0  // 0: k_visc_tiled writes R, the xi sweep adds (measured equal to 1 / 2, no extra buffer)
 #endif
 static_assert(!CROCCO_VISC_XDIV || CROCCO_ZDIV_SWEEP == 0, "XDIV writes R from k_visc_tiled (ZDIV_SWEEP 0)");
+#ifndef CROCCO_FILL_GATHER
+#define CROCCO_FILL_GATHER 1  // single-pass gather fill where it applies (0: always the 3-phase box ops)
+#endif
 #ifndef CROCCO_SWEEP_SMEM
 #define CROCCO_SWEEP_SMEM 1  // shared-memory staged sweeps (k_sweep_s); 0: global-load sweeps
 #endif
@@ -868,12 +871,47 @@ static crocco_status check_ptrs(crocco_ctx c, double *const *p, const char *what
     return CROCCO_OK;
 }
 
+// single-pass gather fill (fill.cuh k_fill_gather): state fills whose faces are all PERIODIC,
+// EXTRAP, WALL or DIRICHLET with every block on this rank (bitwise equal to the 3 phases)
+static bool gather_fill_ok(const crocco_ctx_s *c, int32_t kind) {
+    if (kind != CROCCO_FIELD_STATE || CROCCO_FILL_GATHER == 0) return false;
+    if (c->loc.size() != c->all.size() || c->loc.size() > AMR_MAX_LOCAL || c->all.size() > AMR_MAX_BLOCKS)
+        return false;
+    for (int d = 0; d < 3; d++)
+        for (int sd = 0; sd < 2; sd++) {
+            const int k = c->desc.bc[d][sd];
+            if (k != CROCCO_BC_PERIODIC && k != CROCCO_BC_EXTRAP && k != CROCCO_BC_WALL && k != CROCCO_BC_DIRICHLET)
+                return false;
+        }
+    return true;
+}
+
+static crocco_status fill_gather(crocco_ctx c, double *const *f) {
+    GatherArgs ga;
+    memset(&ga, 0, sizeof ga);
+    level_tab(c, f, ga.t);
+    for (size_t b = 0; b < c->loc.size(); b++)
+        for (int d = 0; d < 3; d++) ga.org[b][d] = c->loc[b].g.origin[d];
+    for (int d = 0; d < 3; d++)
+        for (int sd = 0; sd < 2; sd++) {
+            ga.bc[d][sd] = c->desc.bc[d][sd];
+            for (int q = 0; q < 5; q++) ga.dir[d][sd][q] = c->desc.dirichlet[d][sd][q];
+        }
+    const int64_t n0 = c->bn[0], n1 = c->bn[1], n2 = c->bn[2];
+    const int64_t shell = (int64_t)2 * G * (n0 + 2 * G) * (n1 + 2 * G) + (int64_t)2 * G * n2 * (n0 + 2 * G) +
+                          (int64_t)2 * G * n2 * n1;
+    dim3 grid(std::min<int64_t>(cdiv(shell, 256), 4096), (unsigned)c->loc.size());
+    LAUNCH(c, K_FILL, k_fill_gather<<<grid, 256, 0, c->stream>>>(ga));
+    return CROCCO_OK;
+}
+
 static crocco_status fill_all(crocco_ctx c, double *const *f, int32_t kind, double *const *met, double t) {
     NvtxRange nv(c->amr_Uc ? "crocco:fill_two_levels" : "crocco:fill");
     if (kind != CROCCO_FIELD_STATE && kind != CROCCO_FIELD_METRIC && kind != FILL_STATE_COPIES)
         return fail(c, CROCCO_ERR_ARG, "bad field kind");
     crocco_status st = check_ptrs(c, f, "field");
     if (st) return st;
+    if (gather_fill_ok(c, kind)) return fill_gather(c, f);
     for (int d = 0; d < 3; d++) {
         st = fill_phase(c, f, kind, d, met, t);
         if (st) return st;
