@@ -333,6 +333,12 @@ static void build_plan(const crocco_grid_desc *d, const int nb[3], const int bn[
 #define CROCCO_ZDIV_SWEEP 0  // 0: k_visc_tiled writes R, the xi sweep adds (measured equal to 1 / 2, no extra buffer)
 #endif
 static_assert(!CROCCO_VISC_XDIV || CROCCO_ZDIV_SWEEP == 0, "XDIV writes R from k_visc_tiled (ZDIV_SWEEP 0)");
+#ifndef CROCCO_SEG_MIN
+#define CROCCO_SEG_MIN 32       // shortest march segment of a sweep line (small blocks split lines into segments)
+#endif
+#ifndef CROCCO_SEG_WARPS
+#define CROCCO_SEG_WARPS 16384  // lines are split until at least this many warps march
+#endif
 #ifndef CROCCO_FILL_GATHER
 #define CROCCO_FILL_GATHER 1  // single-pass gather fill where it applies (0: always the 3-phase box ops)
 #endif
@@ -1104,7 +1110,10 @@ static crocco_status rhs_block(crocco_ctx c, const LocalBlock &b, const double *
         const int64_t lines = d == 0 ? ((int64_t)b.g.n[1] * b.g.n[2] + 3) / 4
                                      : (int64_t)((b.g.n[0] + 7) / 8) * (d == 1 ? b.g.n[2] : b.g.n[1]);
         int64_t seg = nd;
-        while (lines * ((nd + seg - 1) / seg) < 16384 && seg > 32) seg = (seg + 1) / 2;
+        // fewer lines than SMs (e.g. Sod's 4 xi lines): segments down to 8 points (measured 8.6e7 -> 1.1e8
+        // point-stages/s on Sod); otherwise >= 32 (shorter segments measured slower on the 64^3 vortex)
+        const int64_t segmin = lines < 148 ? 8 : CROCCO_SEG_MIN;
+        while (lines * ((nd + seg - 1) / seg) < CROCCO_SEG_WARPS && seg > segmin) seg = (seg + 1) / 2;
         a.seg = (int)seg;
         const int64_t warps = lines * ((nd + seg - 1) / seg);
         const unsigned grid = cdiv(warps * 32, SWEEP_THREADS);
