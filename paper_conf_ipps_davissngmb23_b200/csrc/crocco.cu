@@ -1019,17 +1019,18 @@ static bool visc_overlap_possible(crocco_ctx c) {
     if (!(viscous && CROCCO_SWEEP_SMEM && !CROCCO_VISC_DIV && CROCCO_VISC_ZDIV && CROCCO_ZDIV_SWEEP == 0))
         return false;
     for (const auto &b : c->loc) {
-        const VTiles t = visc_interior_tiles(b.L);
+        const VTiles t = visc_interior_tiles(b.L, visc_slab(b.L, b.V));
         if (t.x1 > t.x0 && t.y1 > t.y0 && t.z1 > t.z0) return true;
     }
     return false;
 }
 static crocco_status visc_interior(crocco_ctx c, const LocalBlock &b, const double *U, const double *M) {
-    const VTiles t = visc_interior_tiles(b.L);
+    const int vk = visc_slab(b.L, b.V);
+    const VTiles t = visc_interior_tiles(b.L, vk);
     const int64_t nt = (int64_t)(t.x1 - t.x0) * (t.y1 - t.y0) * (t.z1 - t.z0);
     if (nt == 0) return CROCCO_OK;
     LAUNCH(c, K_VISC, k_visc_tiled<<<(unsigned)nt, VTX * VTY, VISC_SMEM, c->stream>>>(U, M, b.fv, b.L, b.V,
-                                                                                     c->ph, b.racc, b.rcs, 1));
+                                                                                     c->ph, b.racc, b.rcs, 1, vk));
     return CROCCO_OK;
 }
 
@@ -1064,14 +1065,15 @@ static crocco_status rhs_block(crocco_ctx c, const LocalBlock &b, const double *
 #if CROCCO_SWEEP_SMEM
         if (visc_sel != 1) {  // sel 1 (interior tiles) was launched by visc_interior() beside the fill
             const int nz = zdiv ? b.g.n[2] : b.V.b2;
-            int64_t nt = (int64_t)visc_tiles_x(b.L, b.V) * ((b.V.b1 + VTY - 1) / VTY) * ((nz + VK - 1) / VK);
+            const int vk = visc_slab(b.L, b.V);
+            int64_t nt = (int64_t)visc_tiles_x(b.L, b.V) * ((b.V.b1 + VTY - 1) / VTY) * ((nz + vk - 1) / vk);
             if (visc_sel == 2) {
-                const VTiles t = visc_interior_tiles(b.L);
+                const VTiles t = visc_interior_tiles(b.L, vk);
                 nt -= (int64_t)(t.x1 - t.x0) * (t.y1 - t.y0) * (t.z1 - t.z0);
             }
             if (nt > 0)
                 LAUNCH(c, K_VISC, k_visc_tiled<<<(unsigned)nt, VTX * VTY, VISC_SMEM, c->stream>>>(
-                                      U, M, b.fv, b.L, b.V, ph, rvz, b.rcs, visc_sel));
+                                      U, M, b.fv, b.L, b.V, ph, rvz, b.rcs, visc_sel, vk));
         }
 #else
         const int64_t nv = (int64_t)b.V.b0 * b.V.b1 * b.V.b2;

@@ -153,6 +153,20 @@ constexpr int VPL = VHX * VHY;                       // points per staged plane
 constexpr int VHALO = VPL - VTX * VTY;               // halo points per plane
 constexpr size_t VISC_SMEM = (size_t)2 * 4 * VPL * sizeof(double) +
                               (CROCCO_VISC_XDIV && !CROCCO_VISC_XSHFL ? (size_t)2 * 4 * VTX * VTY * sizeof(double) : 0);
+// slab depth of k_visc_tiled (runtime): the longest of CROCCO_VISC_VKMAX / ... / 128 planes that still gives >= 8
+// waves of one-CTA-per-SM tiles (each slab recomputes 4 boundary planes; 64 -> 256 measured
+// 6.47 -> 6.22 ms per 512^3 launch), else CROCCO_VISC_VK
+#ifndef CROCCO_VISC_VKMAX
+#define CROCCO_VISC_VKMAX 256  // 512 measured slower at 512^3 (one slab per column: 8.3 waves, tail)
+#endif
+__host__ __device__ inline int visc_tiles_x(const Lay &L, const VLay &V);
+inline int visc_slab(const Lay &L, const VLay &V) {
+    const int nz = CROCCO_VISC_ZDIV ? L.n2 : V.b2;
+    const int64_t txy = (int64_t)visc_tiles_x(L, V) * ((V.b1 + VTY - 1) / VTY);
+    for (int vk = CROCCO_VISC_VKMAX; vk > VK; vk /= 2)
+        if (txy * ((nz + vk - 1) / vk) >= 8 * 148) return vk;
+    return VK;
+}
 // tiles in i of the viscous box (XDIV: central columns tile the interior [0, n0) with stride VSX)
 __host__ __device__ inline int visc_tiles_x(const Lay &L, const VLay &V) {
     return CROCCO_VISC_XDIV ? (L.n0 + VSX - 1) / VSX : (V.b0 + VTX - 1) / VTX;
@@ -176,15 +190,15 @@ __device__ __forceinline__ void prim4(const double *__restrict__ U, int64_t cs, 
 struct VTiles {
     int x0, x1, y0, y1, z0, z1;
 };
-__host__ __device__ inline VTiles visc_interior_tiles(const Lay &L) {
+__host__ __device__ inline VTiles visc_interior_tiles(const Lay &L, int vk) {
     VTiles t;
     // x: loads i0-2 .. i0+VTX+1 with i0 = bx VSX - 2; y likewise (stride VTY); z: planes z0-4 .. z1+3
     t.x0 = (4 + VSX - 1) / VSX;
     t.x1 = (L.n0 - VTX) >= 0 ? (L.n0 - VTX) / VSX + 1 : 0;
     t.y0 = (4 + VTY - 1) / VTY;
     t.y1 = (L.n1 - VTY) >= 0 ? (L.n1 - VTY) / VTY + 1 : 0;
-    t.z0 = (4 + VK - 1) / VK;
-    t.z1 = (L.n2 - 4) / VK;
+    t.z0 = (4 + vk - 1) / vk;
+    t.z1 = (L.n2 - 4) / vk;
     if (t.x1 < t.x0) t.x1 = t.x0;
     if (t.y1 < t.y0) t.y1 = t.y0;
     if (t.z1 < t.z0) t.z1 = t.z0;
@@ -196,14 +210,14 @@ __global__ void __launch_bounds__(VTX * VTY, CROCCO_VISC_MINB) k_visc_tiled(cons
                                                           const double *__restrict__ M,
                                                           double *__restrict__ FV, Lay L, VLay V,
                                                           Phys ph, double *__restrict__ R, int64_t rcs,
-                                                          int sel) {
+                                                          int sel, int vk) {
     extern __shared__ double vsm[];  // [buffer 2][value 4][VPL]
     const int tid = threadIdx.x;
     const int tx = tid % VTX, ty = tid / VTX;
     const int tilesx = visc_tiles_x(L, V), tilesy = (V.b1 + VTY - 1) / VTY;
     int b = blockIdx.x;
     int bx, by, bz;
-    const VTiles it = visc_interior_tiles(L);
+    const VTiles it = visc_interior_tiles(L, vk);
     if (sel == 1) {
         const int nx = it.x1 - it.x0, ny = it.y1 - it.y0;
         bx = it.x0 + b % nx;
@@ -215,7 +229,7 @@ __global__ void __launch_bounds__(VTX * VTY, CROCCO_VISC_MINB) k_visc_tiled(cons
         // slabs outside [z0, z1), then the xy ring around [x0, x1) x [y0, y1) of the others
         const int nx = it.x1 - it.x0, ny = it.y1 - it.y0, nzi = it.z1 - it.z0;
         const int plane = tilesx * tilesy;
-        const int tz = (L.n2 + VK - 1) / VK;
+        const int tz = (L.n2 + vk - 1) / vk;
         const int nzs = tz - nzi;
         if (b < nzs * plane) {
             const int sl = b / plane, r = b % plane;
@@ -258,7 +272,7 @@ __global__ void __launch_bounds__(VTX * VTY, CROCCO_VISC_MINB) k_visc_tiled(cons
 #endif
 #if CROCCO_VISC_ZDIV
     // slab of interior output planes [z0, z1); gradients / point fluxes on planes z0-2 .. z1+1
-    const int z0 = bz * VK, z1 = min(z0 + VK, L.n2);
+    const int z0 = bz * vk, z1 = min(z0 + vk, L.n2);
     const int k0 = z0 - 2, k1 = z1 + 2;
     double zq[5][4];  // F^zeta of the own column, planes k-4 .. k
 #pragma unroll
@@ -266,7 +280,7 @@ __global__ void __launch_bounds__(VTX * VTY, CROCCO_VISC_MINB) k_visc_tiled(cons
 #pragma unroll
         for (int q = 0; q < 4; q++) zq[o][q] = 0.0;
 #else
-    const int k0 = bz * VK - 2, k1 = min(k0 + VK, V.b2 - 2);
+    const int k0 = bz * vk - 2, k1 = min(k0 + vk, V.b2 - 2);
 #endif
     const double iR = 1.0 / ph.R;
     // own column (clamped into the padded box for the idle threads of edge tiles)
