@@ -94,6 +94,7 @@ def lib():
         L.oracle_eigvecs.argtypes = [dp, C.c_double, C.c_double, C.c_double, C.c_double,
                                      C.c_double, C.c_double, dp, dp]
         L.oracle_interface_flux.argtypes = [C.POINTER(Phys), dp, dp, dp]
+        L.oracle_roe_state.argtypes = [dp, dp, C.c_double, dp]
         L.oracle_rhs.argtypes = [i64p, C.POINTER(Phys), dp, dp, dp]
         L.oracle_rk_update.argtypes = [i64p, C.c_int32, C.c_double, dp, dp, dp, dp]
         L.oracle_rk_stage.argtypes = [i64p, i32p, dp, C.POINTER(Phys), C.c_int32, C.c_double,
@@ -188,6 +189,15 @@ def eigvecs(nrm, rho, u, v, w, c, gamma=1.4):
     a = np.ascontiguousarray(nrm, dtype=np.float64)
     lib().oracle_eigvecs(_dp(a), rho, u, v, w, c, gamma, _dp(T), _dp(Ti))
     return T.reshape(5, 5), Ti.reshape(5, 5)
+
+
+def roe_state(UL, UR, gamma=1.4):
+    """Roe average (rho~, u~, v~, w~, c~) of the conserved states at points i, i+1 (reading 9)."""
+    a = np.ascontiguousarray(UL, dtype=np.float64)
+    b = np.ascontiguousarray(UR, dtype=np.float64)
+    out = np.zeros(5)
+    lib().oracle_roe_state(_dp(a), _dp(b), float(gamma), _dp(out))
+    return out
 
 
 def interface_flux(ph: Phys, Ul, ml):

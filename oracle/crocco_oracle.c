@@ -482,6 +482,34 @@ void oracle_eigvecs(const double nrm[3], double rho, double u, double v, double 
 }
 
 /* ------------------------------------------------------------------ */
+/* 4b. Roe average of the states at points i (UL) and i+1 (UR)         */
+/*     (reading 9; [lit] Roe 1981, J. Comput. Phys. 43:357):            */
+/*     r = sqrt(rho_R/rho_L), (u,v,w,H)~ = (q_L + r q_R)/(1+r),          */
+/*     rho~ = r rho_L, c~ = sqrt((gamma-1)(H~ - |u~|^2/2)).             */
+/*     out = (rho~, u~, v~, w~, c~).                                    */
+/* ------------------------------------------------------------------ */
+void oracle_roe_state(const double UL[5], const double UR[5], double gamma, double out[5])
+{
+    const double gm1 = gamma - 1.0;
+    const double *U2 = UL, *U3 = UR;
+    double uL = U2[1] / U2[0], vL = U2[2] / U2[0], wL = U2[3] / U2[0];
+    double uR = U3[1] / U3[0], vR = U3[2] / U3[0], wR = U3[3] / U3[0];
+    double pL = gm1 * (U2[4] - 0.5 * U2[0] * (uL * uL + vL * vL + wL * wL));
+    double pR = gm1 * (U3[4] - 0.5 * U3[0] * (uR * uR + vR * vR + wR * wR));
+    double HL = (U2[4] + pL) / U2[0], HR = (U3[4] + pR) / U3[0];
+    double r = sqrt(U3[0] / U2[0]);
+    double ut = (uL + r * uR) / (1.0 + r);
+    double vt = (vL + r * vR) / (1.0 + r);
+    double wt = (wL + r * wR) / (1.0 + r);
+    double Ht = (HL + r * HR) / (1.0 + r);
+    out[0] = r * U2[0];
+    out[1] = ut;
+    out[2] = vt;
+    out[3] = wt;
+    out[4] = sqrt(gm1 * (Ht - 0.5 * (ut * ut + vt * vt + wt * wt)));
+}
+
+/* ------------------------------------------------------------------ */
 /* 5. Characteristic WENO interface flux (PAPER.md:50, 110-112;        */
 /*    readings 8-11).  Inputs: the 6 conserved states U_{i-2..i+3} and */
 /*    the metric row m^d at the same 6 points.  Output F^_{i+1/2}.     */
@@ -499,7 +527,7 @@ void oracle_interface_flux(const oracle_phys *ph, const double Ul[30], const dou
     double nrm[3] = {mh[0] / mag, mh[1] / mag, mh[2] / mag};
 
     /* primitive variables at the 6 points */
-    double rho[6], u[6], v[6], w[6], p[6], c[6], H[6];
+    double rho[6], u[6], v[6], w[6], p[6], c[6];
     for (int l = 0; l < 6; l++) {
         const double *U = Ul + 5 * l;
         rho[l] = U[0];
@@ -508,18 +536,12 @@ void oracle_interface_flux(const oracle_phys *ph, const double Ul[30], const dou
         w[l] = U[3] / U[0];
         p[l] = gm1 * (U[4] - 0.5 * rho[l] * (u[l] * u[l] + v[l] * v[l] + w[l] * w[l]));
         c[l] = sqrt(gam * p[l] / rho[l]);
-        H[l] = (U[4] + p[l]) / rho[l];
     }
-    /* Roe average of points i (l=2) and i+1 (l=3) */
-    double r = sqrt(rho[3] / rho[2]);
-    double ut = (u[2] + r * u[3]) / (1.0 + r);
-    double vt = (v[2] + r * v[3]) / (1.0 + r);
-    double wt = (w[2] + r * w[3]) / (1.0 + r);
-    double Ht = (H[2] + r * H[3]) / (1.0 + r);
-    double rhot = r * rho[2];
-    double ct = sqrt(gm1 * (Ht - 0.5 * (ut * ut + vt * vt + wt * wt)));
+    /* Roe average of points i (l=2) and i+1 (l=3), section 4b */
+    double roe[5];
+    oracle_roe_state(Ul + 5 * 2, Ul + 5 * 3, gam, roe);
     double T[25], Ti[25];
-    oracle_eigvecs(nrm, rhot, ut, vt, wt, ct, gam, T, Ti);
+    oracle_eigvecs(nrm, roe[0], roe[1], roe[2], roe[3], roe[4], gam, T, Ti);
 
     /* projected fluxes and states, characteristic speeds */
     double g[5][6], wv[5][6], lam[5];

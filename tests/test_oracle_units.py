@@ -139,6 +139,120 @@ def test_eigvecs_inverse_and_diagonalise():
         assert np.abs(A @ T - T * lam).max() < 1e-12 * scale
 
 
+def _cons(rho, vel, p, gamma=1.4):
+    return np.array([rho, *(rho * np.asarray(vel)), p / (gamma - 1) + 0.5 * rho * np.dot(vel, vel)])
+
+
+def test_roe_state_satisfies_roe_property():
+    """Roe (1981): the flux Jacobian at the Roe-averaged state maps the jump of the states
+    onto the jump of the fluxes, A(U~)(U_R - U_L) = F_n(U_R) - F_n(U_L), for any normal n.
+    A comes from a complex-step derivative of Eq. 1's flux (not from the oracle), and also
+    as T Lambda T^-1 from the (separately pinned) eigenvectors.  Inverted Roe weights or an
+    arithmetic mean fail it (next test, so the pin has teeth).  rho~ does not enter A;
+    it is pinned by its definition rho~^2 = rho_L rho_R (reading 9)."""
+    rng = np.random.default_rng(21)
+    gamma = 1.4
+    worst = worst_eig = 0.0
+    for _ in range(200):
+        n = rng.normal(size=3)
+        n /= np.linalg.norm(n)
+        UL = _cons(rng.uniform(0.1, 5), rng.normal(size=3) * 2, rng.uniform(0.1, 5), gamma)
+        UR = _cons(rng.uniform(0.1, 5), rng.normal(size=3) * 2, rng.uniform(0.1, 5), gamma)
+        rt, ut, vt, wt, ct = oracle.roe_state(UL, UR, gamma)
+        assert abs(rt * rt - UL[0] * UR[0]) < 1e-13 * UL[0] * UR[0]
+        vel = np.array([ut, vt, wt])
+        Ut = _cons(rt, vel, rt * ct * ct / gamma, gamma)
+        A = _jacobian_complex_step(Ut, n, gamma)
+        jump = _flux_n(UR, n, gamma) - _flux_n(UL, n, gamma)
+        scale = np.abs(jump).max() + np.abs(A).max() * np.abs(UR - UL).max()
+        worst = max(worst, np.abs(A @ (UR - UL) - jump).max() / scale)
+        T, Ti = oracle.eigvecs(n, rt, ut, vt, wt, ct, gamma)
+        th = n @ vel
+        lam = np.array([th, th, th, th + ct, th - ct])
+        worst_eig = max(worst_eig, np.abs(T @ (lam * (Ti @ (UR - UL))) - jump).max() / scale)
+    assert worst < 1e-13, worst
+    assert worst_eig < 1e-12, worst_eig
+
+
+def test_roe_wrong_averages_violate_property_typically():
+    """Teeth of the pin above: on a generic pair the arithmetic mean / inverted weights miss
+    Roe's property by many orders of magnitude more than rounding."""
+    gamma = 1.4
+    n = np.array([0.6, 0.0, 0.8])
+    UL = _cons(1.0, [0.3, -0.2, 0.5], 1.0, gamma)
+    UR = _cons(3.0, [-0.4, 0.6, 0.1], 2.5, gamma)
+    jump = _flux_n(UR, n, gamma) - _flux_n(UL, n, gamma)
+    r = math.sqrt(UR[0] / UL[0])
+    vL, vR = UL[1:4] / UL[0], UR[1:4] / UR[0]
+    pL = (gamma - 1) * (UL[4] - 0.5 * UL[0] * vL @ vL)
+    pR = (gamma - 1) * (UR[4] - 0.5 * UR[0] * vR @ vR)
+    HL, HR = (UL[4] + pL) / UL[0], (UR[4] + pR) / UR[0]
+    for wl, wr in ((0.5, 0.5), (r / (1 + r), 1 / (1 + r))):
+        v2 = wl * vL + wr * vR
+        c2 = (gamma - 1) * (wl * HL + wr * HR - 0.5 * v2 @ v2)
+        A2 = _jacobian_complex_step(_cons(1.7, v2, 1.7 * c2 / gamma, gamma), n, gamma)
+        assert np.abs(A2 @ (UR - UL) - jump).max() > 1e-3 * np.abs(jump).max()
+    rt, ut, vt, wt, ct = oracle.roe_state(UL, UR, gamma)
+    A = _jacobian_complex_step(_cons(rt, [ut, vt, wt], rt * ct * ct / gamma, gamma), n, gamma)
+    assert np.abs(A @ (UR - UL) - jump).max() < 1e-13 * np.abs(jump).max()
+
+
+def _linear_weno_coeffs():
+    C = _gold_weights()
+    c = np.zeros(6)
+    for k, (start, coef) in enumerate(SHU_STENCILS):
+        c[start:start + 3] += C[k] * np.array(coef)
+    return c / C.sum()
+
+
+def _flux_linear_mode(U6, m, points, gamma=1.4):
+    """Interface flux of readings 8-11 in linear-weight mode, composed from independently
+    pinned pieces (Roe state, eigenvectors, linear SYMBO stencil from the golden weights,
+    Eq. 1's flux), with the LLF speed lambda_s = max over the stencil points `points`."""
+    c = _linear_weno_coeffs()
+    mag = np.linalg.norm(m)
+    n = m / mag
+    rt, ut, vt, wt, ct = oracle.roe_state(U6[2], U6[3], gamma)
+    T, Ti = oracle.eigvecs(n, rt, ut, vt, wt, ct, gamma)
+    g = np.array([Ti @ _flux_n(U6[l], n, gamma) for l in range(6)]).T   # (s, l)
+    w = np.array([Ti @ U6[l] for l in range(6)]).T
+    eig = np.zeros((5, 6))
+    for l in range(6):
+        vel = U6[l, 1:4] / U6[l, 0]
+        p = (gamma - 1) * (U6[l, 4] - 0.5 * U6[l, 0] * vel @ vel)
+        th, cl = n @ vel, math.sqrt(gamma * p / U6[l, 0])
+        eig[:, l] = np.abs([th, th, th, th + cl, th - cl])
+    lam = eig[:, points].max(1)
+    gp = 0.5 * (g + lam[:, None] * w)
+    gm = 0.5 * (g - lam[:, None] * w)
+    gh = gp @ c + gm @ c[::-1]          # W(g+) + W(mirror of g-)
+    return mag * (T @ gh)
+
+
+def test_llf_speed_is_max_over_all_six_stencil_points():
+    """Reading 10: lambda_s = max over the 6 stencil points i-2..i+3.  A stencil whose fastest
+    point is l = 0 (i-2) only: the oracle's linear-mode flux equals the composition with the
+    6-point maximum and differs clearly from the (i, i+1) maximum."""
+    gamma = 1.4
+    ph = _ph(terms=1, weno_linear=1)
+    rng = np.random.default_rng(22)
+    for trial in range(20):
+        U6 = np.array([_cons(rng.uniform(0.8, 1.2), rng.normal(size=3) * 0.1, rng.uniform(0.8, 1.2), gamma)
+                       for _ in range(6)])
+        m = rng.normal(size=3) + np.array([2.0, 0, 0])
+        n = m / np.linalg.norm(m)
+        fast = 3.0 + trial * 0.1
+        U6[0] = _cons(1.0, fast * n, 1.0, gamma)   # |theta + c| largest at l = 0 only
+        F = oracle.interface_flux(ph, U6, np.tile(m, (6, 1)))
+        F6 = _flux_linear_mode(U6, m, [0, 1, 2, 3, 4, 5], gamma)
+        F2 = _flux_linear_mode(U6, m, [2, 3], gamma)
+        F5 = _flux_linear_mode(U6, m, [1, 2, 3, 4, 5], gamma)
+        sc = np.abs(F6).max()
+        assert np.abs(F - F6).max() < 1e-12 * sc, (trial, F, F6)
+        assert np.abs(F - F2).max() > 1e-3 * sc
+        assert np.abs(F - F5).max() > 1e-3 * sc
+
+
 # ------------------------------------------------------------------ interface flux (readings 8-11)
 
 def _ph(**kw):
