@@ -594,6 +594,30 @@ def _profiled_traffic(kname, key="dram_bytes_per_launch"):
         return None
 
 
+def relaunch(ngpus):
+    """`python bench.py --gpus N` without torchrun: check that N GPUs are visible, then run
+    the same command line as N ranks (one process per GPU) under torch.distributed.run on
+    127.0.0.1, with NCCL's INIT lines on stderr.  Fails loudly (exit 2) with fewer GPUs:
+    N ranks on one device is not a multi-GPU run (NCCL refuses it anyway)."""
+    import socket
+
+    import torch
+    have = torch.cuda.device_count()
+    if have < ngpus:
+        print(f"bench.py: --gpus {ngpus} needs {ngpus} visible CUDA devices, found {have}", file=sys.stderr)
+        return 2
+    with socket.socket() as so:
+        so.bind(("127.0.0.1", 0))
+        port = so.getsockname()[1]
+    env = dict(os.environ)
+    env.setdefault("NCCL_DEBUG", "INFO")
+    env.setdefault("NCCL_DEBUG_SUBSYS", "INIT")
+    cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", f"--nproc-per-node={ngpus}",
+           "--master-addr=127.0.0.1", f"--master-port={port}", os.path.abspath(__file__), *sys.argv[1:]]
+    print("bench.py: relaunching as " + " ".join(cmd), file=sys.stderr, flush=True)
+    return subprocess.call(cmd, env=env)
+
+
 def main():
     ap = argparse.ArgumentParser(description=__doc__, formatter_class=argparse.RawDescriptionHelpFormatter)
     ap.add_argument("--gpus", type=int, default=1)
@@ -609,11 +633,19 @@ def main():
     ap.add_argument("--no-clocks", action="store_true")
     ap.add_argument("--ref-n", type=int, default=64)
     args = ap.parse_args()
+    launched = "WORLD_SIZE" in os.environ
     rank = int(os.environ.get("RANK", "0"))
     world = int(os.environ.get("WORLD_SIZE", "1"))
     local_rank = int(os.environ.get("LOCAL_RANK", "0"))
+    if args.gpus < 1:
+        raise SystemExit("--gpus must be >= 1")
     if args.impl == "reference":
+        # the CPU oracle arm: rank 0 alone runs (under torchrun the other ranks exit 0)
         return run_reference(args, rank, world)
+    if not launched and args.gpus > 1:
+        return relaunch(args.gpus)
+    if world != args.gpus:
+        raise SystemExit(f"bench.py: --gpus {args.gpus} but WORLD_SIZE={world}: one rank per GPU required")
     if args.config in ("amr", "dmr_amr"):
         if world > 1:
             raise SystemExit(f"--config {args.config} runs on one GPU")
@@ -621,6 +653,10 @@ def main():
     if world > 1:
         import torch
         import torch.distributed as dist
+        os.environ.setdefault("NCCL_DEBUG", "INFO")        # INIT lines (transport, NVLS) on stderr
+        os.environ.setdefault("NCCL_DEBUG_SUBSYS", "INIT")
+        if torch.cuda.device_count() < world:
+            raise SystemExit(f"bench.py: {world} ranks but {torch.cuda.device_count()} visible GPUs")
         torch.cuda.set_device(local_rank)
         dist.init_process_group("nccl", device_id=torch.device("cuda", local_rank))
     try:

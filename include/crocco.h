@@ -166,6 +166,8 @@ crocco_status crocco_init_grid(const crocco_grid_desc *desc, const crocco_phys *
 crocco_status crocco_num_local_blocks(crocco_ctx ctx, int32_t *n_local);
 crocco_status crocco_get_block_layout(crocco_ctx ctx, int32_t local_block,
                                       crocco_block_layout *out);
+/* Replace the gas / scheme constants (validated like crocco_init_grid).  Drops every cached
+   RK3 step graph (crocco_rk3_step): a graph bakes in the kernel arguments and variants. */
 crocco_status crocco_set_phys(crocco_ctx ctx, const crocco_phys *phys);
 crocco_status crocco_scratch_bytes(crocco_ctx ctx, int64_t *bytes);
 
@@ -181,7 +183,8 @@ crocco_status crocco_init_metrics(crocco_ctx ctx, double *const *xyz, double *co
    component 6a + pair index of (00, 01, 02, 11, 12, 22), on interior points, computed from
    `metrics` (filled by crocco_init_metrics) into LIBRARY-OWNED device memory (18 fp64 per
    interior point; reported by crocco_scratch_bytes) used by the expanded viscous form
-   (visc_form = 1).  Call again after changing the metrics.  Not collective. */
+   (visc_form = 1).  Call again after changing the metrics.  Drops the cached RK3 step
+   graphs.  Not collective. */
 crocco_status crocco_init_metrics2(crocco_ctx ctx, double *const *metrics);
 /* Copy local block b's second metrics to dst (device memory, 18 x n0 n1 n2 fp64, component
    q at q * n0 n1 n2 + i + n0 (j + n1 k)); tests.  CROCCO_ERR_STATE if not initialised. */
@@ -235,7 +238,9 @@ crocco_status crocco_rk_update(crocco_ctx ctx, int32_t stage, double dt, double 
    *dt = cfl / max_i sum_d J_i (|m^d_i . u_i| + c_i |m^d_i|) over the interior points of
    all blocks of all ranks (global reduction with ncclAllReduce(max) when nranks > 1).
    U: conserved state (ghosts not read); metrics from crocco_init_metrics; dt: HOST
-   pointer.  Synchronises the stream.  Collective. */
+   pointer.  Synchronises the stream.  Collective.  A non-finite local radius (NaN
+   component, negative pressure) is not dropped by the maximum: CROCCO_ERR_ARG with
+   "non-finite spectral radius". */
 crocco_status crocco_compute_dt(crocco_ctx ctx, double *const *U, double *const *metrics,
                                 double cfl, double *dt);
 
@@ -289,13 +294,27 @@ crocco_status crocco_finalize(crocco_ctx ctx);
    the fill has NCCL faces; a purely local fill is too short to hide and the split
    viscous launch costs more than it saves -- measured on one B200).  Results are
    bitwise identical either way: the fill writes only ghost points, the overlapped
-   tiles read only interior points.  CROCCO_ERR_ARG for other values. */
+   tiles read only interior points.  CROCCO_ERR_ARG for other values.  Changing it
+   drops the cached RK3 step graphs (the stage structure differs).  With overlap the
+   viscous slab depth is capped so that an interior slab exists ((n2 - 4)/vk >= 2). */
 crocco_status crocco_set_overlap(crocco_ctx ctx, int32_t enable);
 
 /* ---- instrumentation (bench / tests) ---------------------------------------- */
 
 /* Number of kernels this ctx launched since init (or the last reset). */
 crocco_status crocco_launch_count(crocco_ctx ctx, int64_t *count, int32_t reset);
+/* Debug / hardware check of the NCCL halo path on ONE GPU (nranks == 1 only): with enable != 0
+   the library creates a 1-rank NCCL communicator and routes every same-rank inter-block and
+   periodic ghost copy of crocco_fill_boundary / crocco_rk_stage through the multi-rank code path
+   -- pack kernel -> ncclGroupStart; ncclSend + ncclRecv to itself; ncclGroupEnd -> unpack kernel
+   -- and crocco_compute_dt through ncclAllReduce(max) on that communicator.  Results are bitwise
+   those of the local copies.  Steps launch eagerly (no graphs) while a communicator exists.
+   enable = 0 destroys the communicator.  CROCCO_ERR_ARG when nranks > 1. */
+crocco_status crocco_set_nccl_loopback(crocco_ctx ctx, int32_t enable);
+/* Number of RK stages that ran overlapped (fill on the comm stream beside the ghost-free
+   viscous tiles) since init (or the last reset); graph replays count their captured stages.
+   Lets tests assert that the overlap path really ran. */
+crocco_status crocco_overlap_count(crocco_ctx ctx, int64_t *count, int32_t reset);
 /* Kernel-class timing with CUDA events recorded on the launching stream.
    When enabled, every launch of class k is bracketed by events; crocco_kernel_times
    returns, per class, the number of launches and the summed milliseconds

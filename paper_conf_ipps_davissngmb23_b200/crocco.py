@@ -85,6 +85,8 @@ _SIGS = {
     "crocco_launch_count": [C.c_void_p, C.POINTER(C.c_int64), C.c_int32],
     "crocco_set_timing": [C.c_void_p, C.c_int32],
     "crocco_set_overlap": [C.c_void_p, C.c_int32],
+    "crocco_overlap_count": [C.c_void_p, C.POINTER(C.c_int64), C.c_int32],
+    "crocco_set_nccl_loopback": [C.c_void_p, C.c_int32],
     "crocco_kernel_times": [C.c_void_p, C.c_int32, C.POINTER(C.c_int64), C.POINTER(C.c_double),
                             C.POINTER(C.c_int32)],
     "crocco_exchange_plan": [C.POINTER(GridDesc), C.c_int32, C.POINTER(Msg), C.c_int32,
@@ -273,6 +275,18 @@ def crocco_finalize(ctx):
 def crocco_launch_count(ctx, reset=False) -> int:
     v = C.c_int64()
     _check(lib().crocco_launch_count(ctx, C.byref(v), int(reset)), ctx)
+    return v.value
+
+
+def crocco_set_nccl_loopback(ctx, enable=True):
+    """Single-rank debug: same-rank ghost copies through ncclSend/ncclRecv to self, ComputeDt
+    through ncclAllReduce on a 1-rank communicator (bitwise equal to the local path)."""
+    _check(lib().crocco_set_nccl_loopback(ctx, int(enable)), ctx)
+
+
+def crocco_overlap_count(ctx, reset=False) -> int:
+    v = C.c_int64()
+    _check(lib().crocco_overlap_count(ctx, C.byref(v), int(reset)), ctx)
     return v.value
 
 

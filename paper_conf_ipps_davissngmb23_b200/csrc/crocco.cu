@@ -9,6 +9,7 @@
 #include <nvtx3/nvToolsExt.h>
 
 #include <algorithm>
+#include <cmath>
 #include <cstdarg>
 #include <cstdio>
 #include <cstring>
@@ -90,6 +91,7 @@ struct crocco_ctx_s {
     std::vector<crocco_msg> plan[3];
     // NCCL
     ncclComm_t comm = nullptr;
+    bool loopback = false;  // debug: same-rank copies through ncclSend/ncclRecv to self (crocco_set_nccl_loopback)
     double *send_stage = nullptr, *recv_stage = nullptr;
     unsigned long long *dmax = nullptr;  // ComputeDt reduction cell
     // CUDA graphs of full RK3 steps, keyed by (buffers, dt)
@@ -98,11 +100,13 @@ struct crocco_ctx_s {
         double dt;
         cudaGraphExec_t exec;
         int64_t nodes;
+        int64_t ov_stages;  // overlapped stages inside the captured step
     };
     std::vector<StepGraph> graphs;
     cudaStream_t cap_stream = nullptr;
     // overlapped stage: ghost fill / exchange on comm_stream beside the interior viscous tiles
     int overlap = -1;  // -1 auto (on when the fill has remote faces, nranks > 1), 0 off, 1 on
+    int64_t overlapped_stages = 0;  // stages that ran the fill beside the ghost-free tiles
     cudaStream_t comm_stream = nullptr;
     cudaEvent_t ev_fork = nullptr, ev_join = nullptr;
     double time = 0.0;  // start of the current step (time-dependent SPLIT faces)
@@ -458,12 +462,20 @@ static crocco_status check_phys(const crocco_phys *p) {
     return CROCCO_OK;
 }
 
+// cached RK3 step graphs bake in the kernel arguments (Phys), the kernel variants (limiter,
+// viscous form) and the scratch pointers of the capture: any change of those drops them
+static void drop_graphs(crocco_ctx c) {
+    for (auto &g : c->graphs) cudaGraphExecDestroy(g.exec);
+    c->graphs.clear();
+}
+
 crocco_status crocco_set_phys(crocco_ctx c, const crocco_phys *p) {
     LIVE(c);
     crocco_status st = check_phys(p);
     if (st) return fail(c, st, "%s", g_err.c_str());
     c->phys_in = *p;
     c->ph = to_phys(p);
+    drop_graphs(c);
     return CROCCO_OK;
 }
 
@@ -484,7 +496,7 @@ static void free_ctx(crocco_ctx c) {
         cudaEventDestroy(t.e1);
     }
     for (auto e : c->pool) cudaEventDestroy(e);
-    for (auto &g : c->graphs) cudaGraphExecDestroy(g.exec);
+    drop_graphs(c);
     if (c->cap_stream) cudaStreamDestroy(c->cap_stream);
     if (c->comm_stream) cudaStreamDestroy(c->comm_stream);
     if (c->ev_fork) cudaEventDestroy(c->ev_fork);
@@ -685,7 +697,7 @@ static void level_tab(const crocco_ctx_s *lv, double *const *ptr, LevelTab &t) {
     for (size_t b = 0; b < lv->loc.size(); b++) t.p[b] = ptr[b];
     for (int g = 0; g < AMR_MAX_BLOCKS; g++)
         t.g2l[g] = g < (int)lv->gid_to_local.size() ? (int16_t)lv->gid_to_local[g] : (int16_t)-1;
-    t.L = lv->loc[0].L;
+    if (!lv->loc.empty()) t.L = lv->loc[0].L;  // a rank may own no block of a level
     for (int d = 0; d < 3; d++) {
         t.bn[d] = lv->bn[d];
         t.nb[d] = lv->nb[d];
@@ -711,7 +723,7 @@ static crocco_status fill_phase(crocco_ctx c, double *const *f, int kind, int D,
     }
     std::vector<const crocco_msg *> remote;
     for (const crocco_msg &m : c->plan[D]) {
-        if (m.kind == 0 && (m.src_rank != m.dst_rank)) {
+        if (m.kind == 0 && (m.src_rank != m.dst_rank || c->loopback)) {
             remote.push_back(&m);
             continue;
         }
@@ -798,12 +810,16 @@ static crocco_status fill_phase(crocco_ctx c, double *const *f, int kind, int D,
     if (interp && (st = flush_cf(c, cf, ct))) return st;
     if (remote.empty()) return CROCCO_OK;
     if (!c->comm) return fail(c, CROCCO_ERR_STATE, "remote halo without communicator");
-    // pack sends
+    // pack sends (a loopback message is both sent and received by this rank)
     int64_t soff = 0, roff = 0;
-    std::vector<int64_t> offs(remote.size());
+    std::vector<int64_t> offs(remote.size()), roffs(remote.size());
     for (size_t r = 0; r < remote.size(); r++) {
         const crocco_msg &m = *remote[r];
         const int64_t vol = m.ext[0] * m.ext[1] * m.ext[2];
+        if (m.dst_rank == c->desc.rank) {
+            roffs[r] = roff;
+            roff += vol * ncomp;
+        }
         if (m.src_rank == c->desc.rank) {
             const int sl = c->gid_to_local[m.src_block];
             const LocalBlock &sb = c->loc[sl];
@@ -825,9 +841,6 @@ static crocco_status fill_phase(crocco_ctx c, double *const *f, int kind, int D,
             soff += vol * ncomp;
             st = push_op(c, ops, o);
             if (st) return st;
-        } else {
-            offs[r] = roff;
-            roff += vol * ncomp;
         }
     }
     st = flush_ops(c, ops);
@@ -839,8 +852,8 @@ static crocco_status fill_phase(crocco_ctx c, double *const *f, int kind, int D,
         const size_t cnt = (size_t)(m.ext[0] * m.ext[1] * m.ext[2] * ncomp);
         if (m.src_rank == c->desc.rank)
             NK(c, ncclSend(c->send_stage + offs[r], cnt, ncclDouble, m.dst_rank, c->comm, c->stream));
-        else
-            NK(c, ncclRecv(c->recv_stage + offs[r], cnt, ncclDouble, m.src_rank, c->comm, c->stream));
+        if (m.dst_rank == c->desc.rank)
+            NK(c, ncclRecv(c->recv_stage + roffs[r], cnt, ncclDouble, m.src_rank, c->comm, c->stream));
     }
     NK(c, ncclGroupEnd());
     // unpack receives
@@ -852,7 +865,7 @@ static crocco_status fill_phase(crocco_ctx c, double *const *f, int kind, int D,
         const int64_t vol = m.ext[0] * m.ext[1] * m.ext[2];
         BoxOp o;
         memset(&o, 0, sizeof o);
-        o.src = c->recv_stage + offs[r];
+        o.src = c->recv_stage + roffs[r];
         o.sst[0] = 1;
         o.sst[1] = m.ext[0];
         o.sst[2] = m.ext[0] * m.ext[1];
@@ -880,7 +893,7 @@ static crocco_status check_ptrs(crocco_ctx c, double *const *p, const char *what
 // single-pass gather fill (fill.cuh k_fill_gather): state fills whose faces are all PERIODIC,
 // EXTRAP, WALL or DIRICHLET with every block on this rank (bitwise equal to the 3 phases)
 static bool gather_fill_ok(const crocco_ctx_s *c, int32_t kind) {
-    if (kind != CROCCO_FIELD_STATE || CROCCO_FILL_GATHER == 0) return false;
+    if (kind != CROCCO_FIELD_STATE || CROCCO_FILL_GATHER == 0 || c->loopback) return false;
     if (c->loc.size() != c->all.size() || c->loc.size() > AMR_MAX_LOCAL || c->all.size() > AMR_MAX_BLOCKS)
         return false;
     for (int d = 0; d < 3; d++)
@@ -971,6 +984,7 @@ crocco_status crocco_init_metrics2(crocco_ctx c, double *const *met) {
     LIVE(c);
     crocco_status st = check_ptrs(c, met, "metrics");
     if (st) return st;
+    drop_graphs(c);  // new scratch pointers / kernel variant of the expanded viscous form
     for (auto &b : c->loc) {
         if (!b.met2) {
             if (cudaMalloc((void **)&b.met2, (size_t)(18 * b.rcs) * sizeof(double)) != cudaSuccess ||
@@ -1019,13 +1033,13 @@ static bool visc_overlap_possible(crocco_ctx c) {
     if (!(viscous && CROCCO_SWEEP_SMEM && !CROCCO_VISC_DIV && CROCCO_VISC_ZDIV && CROCCO_ZDIV_SWEEP == 0))
         return false;
     for (const auto &b : c->loc) {
-        const VTiles t = visc_interior_tiles(b.L, visc_slab(b.L, b.V));
+        const VTiles t = visc_interior_tiles(b.L, visc_slab(b.L, b.V, true));
         if (t.x1 > t.x0 && t.y1 > t.y0 && t.z1 > t.z0) return true;
     }
     return false;
 }
 static crocco_status visc_interior(crocco_ctx c, const LocalBlock &b, const double *U, const double *M) {
-    const int vk = visc_slab(b.L, b.V);
+    const int vk = visc_slab(b.L, b.V, true);
     const VTiles t = visc_interior_tiles(b.L, vk);
     const int64_t nt = (int64_t)(t.x1 - t.x0) * (t.y1 - t.y0) * (t.z1 - t.z0);
     if (nt == 0) return CROCCO_OK;
@@ -1065,7 +1079,7 @@ static crocco_status rhs_block(crocco_ctx c, const LocalBlock &b, const double *
 #if CROCCO_SWEEP_SMEM
         if (visc_sel != 1) {  // sel 1 (interior tiles) was launched by visc_interior() beside the fill
             const int nz = zdiv ? b.g.n[2] : b.V.b2;
-            const int vk = visc_slab(b.L, b.V);
+            const int vk = visc_slab(b.L, b.V, visc_sel != 0);
             int64_t nt = (int64_t)visc_tiles_x(b.L, b.V) * ((b.V.b1 + VTY - 1) / VTY) * ((nz + vk - 1) / vk);
             if (visc_sel == 2) {
                 const VTiles t = visc_interior_tiles(b.L, vk);
@@ -1199,6 +1213,7 @@ crocco_status crocco_rk_stage(crocco_ctx c, int32_t stage, double dt, double *co
         if (st) return st;
     }
     CK(c, cudaEventRecord(c->ev_join, c->comm_stream));
+    c->overlapped_stages++;
     for (size_t bi = 0; bi < c->loc.size(); bi++)
         if ((st = visc_interior(c, c->loc[bi], Uin[bi], M[bi]))) return st;
     CK(c, cudaStreamWaitEvent(c->stream, c->ev_join, 0));
@@ -1231,7 +1246,7 @@ crocco_status crocco_rk3_step(crocco_ctx c, double dt, double *const *U, double 
     for (int d = 0; d < 3; d++)
         for (int sd = 0; sd < 2; sd++)
             moving = moving || (c->desc.bc[d][sd] == CROCCO_BC_SPLIT && c->desc.split[d][sd].di_dt != 0.0);
-    if (!use_graph || c->timing || c->desc.nranks > 1 || c->stream == nullptr || moving) {
+    if (!use_graph || c->timing || c->desc.nranks > 1 || c->comm || moving) {
         st = rk3_eager(c, dt, U, V, dU, M);
         if (st == CROCCO_OK) c->time = c->time + dt;
         return st;
@@ -1254,7 +1269,7 @@ crocco_status crocco_rk3_step(crocco_ctx c, double dt, double *const *U, double 
         CK(c, cudaEventRecord(ev, c->stream));
         CK(c, cudaStreamWaitEvent(c->cap_stream, ev, 0));
         cudaStream_t orig = c->stream;
-        const int64_t l0 = c->launches;
+        const int64_t l0 = c->launches, o0 = c->overlapped_stages;
         c->stream = c->cap_stream;
         CK(c, cudaStreamBeginCapture(c->cap_stream, cudaStreamCaptureModeThreadLocal));
         st = rk3_eager(c, dt, U, V, dU, M);
@@ -1272,12 +1287,14 @@ crocco_status crocco_rk3_step(crocco_ctx c, double dt, double *const *U, double 
             cudaGraphExecDestroy(c->graphs.front().exec);
             c->graphs.erase(c->graphs.begin());
         }
-        c->graphs.push_back({key, dt, exec, c->launches - l0});
+        c->graphs.push_back({key, dt, exec, c->launches - l0, c->overlapped_stages - o0});
         c->launches = l0;  // captured, not launched
+        c->overlapped_stages = o0;
         g = &c->graphs.back();
     }
     CK(c, cudaGraphLaunch(g->exec, c->stream));
     c->launches += g->nodes;
+    c->overlapped_stages += g->ov_stages;
     c->time = c->time + dt;
     return CROCCO_OK;
 }
@@ -1321,6 +1338,8 @@ crocco_status crocco_compute_dt(crocco_ctx c, double *const *U, double *const *M
     double lam;
     memcpy(&lam, &h, sizeof lam);
     if (!(lam > 0)) return fail(c, CROCCO_ERR_ARG, "non-positive spectral radius (state not set?)");
+    if (!(lam < INFINITY))
+        return fail(c, CROCCO_ERR_ARG, "non-finite spectral radius: NaN or negative pressure in the state");
     *dt = cfl / lam;
     return CROCCO_OK;
 }
@@ -1546,7 +1565,55 @@ crocco_status crocco_launch_count(crocco_ctx c, int64_t *count, int32_t reset) {
 crocco_status crocco_set_overlap(crocco_ctx c, int32_t enable) {
     LIVE(c);
     if (enable < -1 || enable > 1) return fail(c, CROCCO_ERR_ARG, "overlap must be -1, 0 or 1");
+    if (enable != c->overlap) drop_graphs(c);  // the captured stage structure changes
     c->overlap = enable;
+    return CROCCO_OK;
+}
+
+crocco_status crocco_set_nccl_loopback(crocco_ctx c, int32_t enable) {
+    LIVE(c);
+    if (c->desc.nranks != 1) return fail(c, CROCCO_ERR_ARG, "NCCL loopback is a single-rank debug mode");
+    drop_graphs(c);
+    if (!enable) {
+        c->loopback = false;
+        if (c->comm) ncclCommDestroy(c->comm);
+        c->comm = nullptr;
+        return CROCCO_OK;
+    }
+    // staging for every same-rank copy of a phase, sent and received by this rank
+    int64_t maxe = 0;
+    for (int d = 0; d < 3; d++) {
+        int64_t v = 0;
+        for (auto &m : c->plan[d])
+            if (m.kind == 0) v += m.ext[0] * m.ext[1] * m.ext[2] * 10;
+        maxe = std::max(maxe, v);
+    }
+    if (maxe > c->stage_elems) {
+        cudaFree(c->send_stage);
+        cudaFree(c->recv_stage);
+        c->send_stage = c->recv_stage = nullptr;
+        if (cudaMalloc((void **)&c->send_stage, (size_t)maxe * sizeof(double)) != cudaSuccess ||
+            cudaMalloc((void **)&c->recv_stage, (size_t)maxe * sizeof(double)) != cudaSuccess) {
+            cudaGetLastError();
+            c->stage_elems = 0;
+            return fail(c, CROCCO_ERR_NOMEM, "loopback staging allocation failed");
+        }
+        c->scratch += 2 * (maxe - c->stage_elems) * (int64_t)sizeof(double);
+        c->stage_elems = maxe;
+    }
+    if (!c->comm) {
+        ncclUniqueId id;
+        NK(c, ncclGetUniqueId(&id));
+        NK(c, ncclCommInitRank(&c->comm, 1, id, 0));
+    }
+    c->loopback = true;
+    return CROCCO_OK;
+}
+
+crocco_status crocco_overlap_count(crocco_ctx c, int64_t *count, int32_t reset) {
+    if (!c) return fail(nullptr, CROCCO_ERR_ARG, "null ctx");
+    if (count) *count = c->overlapped_stages;
+    if (reset) c->overlapped_stages = 0;
     return CROCCO_OK;
 }
 

@@ -160,11 +160,13 @@ constexpr size_t VISC_SMEM = (size_t)2 * 4 * VPL * sizeof(double) +
 #define CROCCO_VISC_VKMAX 256  // 512 measured slower at 512^3 (one slab per column: 8.3 waves, tail)
 #endif
 __host__ __device__ inline int visc_tiles_x(const Lay &L, const VLay &V);
-inline int visc_slab(const Lay &L, const VLay &V) {
+// overlap: the stage runs the ghost-free tiles beside the fill (crocco_rk_stage), so the slab
+// depth must leave at least one interior slab, (n2 - 4)/vk >= 2 (visc_interior_tiles)
+inline int visc_slab(const Lay &L, const VLay &V, bool overlap = false) {
     const int nz = CROCCO_VISC_ZDIV ? L.n2 : V.b2;
     const int64_t txy = (int64_t)visc_tiles_x(L, V) * ((V.b1 + VTY - 1) / VTY);
     for (int vk = CROCCO_VISC_VKMAX; vk > VK; vk /= 2)
-        if (txy * ((nz + vk - 1) / vk) >= 8 * 148) return vk;
+        if (txy * ((nz + vk - 1) / vk) >= 8 * 148 && (!overlap || (L.n2 - 4) / vk >= 2)) return vk;
     return VK;
 }
 // tiles in i of the viscous box (XDIV: central columns tile the interior [0, n0) with stride VSX)
@@ -887,7 +889,10 @@ __global__ void __launch_bounds__(256) k_cfl(const double *__restrict__ U, const
                          mz = M[(3 + 3 * d) * L.cs + p];
             sum += fabs(fma(mx, u, fma(my, v, mz * w))) + c * sqrt(fma(mx, mx, fma(my, my, mz * mz)));
         }
-        lmax = fmax(lmax, M[p] * sum);
+        // a non-finite local radius (NaN state, negative pressure -> NaN c) poisons the maximum
+        // (+inf) instead of being dropped by fmax; the host then reports the blow-up
+        const double lp = M[p] * sum;
+        lmax = lp <= 1.7976931348623157e308 ? fmax(lmax, lp) : __longlong_as_double(0x7ff0000000000000LL);
     }
 #pragma unroll
     for (int o = 16; o > 0; o >>= 1) lmax = fmax(lmax, __shfl_xor_sync(0xffffffffu, lmax, o));

@@ -87,6 +87,14 @@ class Solver:
         self.sync()
         self._coords = None
 
+    def set_phys(self, phys):
+        """Replace the gas / scheme constants (crocco_set_phys drops the cached step graphs);
+        switching to the expanded viscous form computes the second metrics."""
+        cc.crocco_set_phys(self.ctx, phys)
+        self.phys = phys
+        if phys.visc_form == 1:
+            cc.crocco_init_metrics2(self.ctx, self._ptrs(self.met))
+
     def metrics2(self, b):
         """(18, n2, n1, n0) second metrics of local block b (expanded viscous form; tests)."""
         L = self.layouts[b]

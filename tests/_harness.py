@@ -91,13 +91,13 @@ class Problem:
         return oracle.phys(**self.phys_kw)
 
     # ---------------- GPU side
-    def solver(self, n_blocks=(1, 1, 1)):
+    def solver(self, n_blocks=(1, 1, 1), stream=None):
         from paper_conf_ipps_davissngmb23_b200 import crocco as cc
         from paper_conf_ipps_davissngmb23_b200.solver import Solver
         kw = dict(self.phys_kw)
         kw.pop("weno_linear", None)  # oracle-only test flag
         S = Solver(self.n, n_blocks, self.bc, cc.make_phys(**kw), dirichlet=self.dirichlet,
-                   split=self.split)
+                   split=self.split, stream=stream)
         bn, blocks = block_slices(self.n, n_blocks)
         xyz = [self.grid.coords(bn, o, oracle.GC) for o, _ in blocks]
         S.set_coords(xyz)

@@ -31,3 +31,24 @@ def test_reference_arm_non_zero_rank_is_silent():
                                    "--steps", "1", "--warmup", "0", "--ref-n", "12"], cwd=ROOT, env=env,
                                   timeout=300)
     assert out.decode().strip() == ""
+
+
+def test_gpus_beyond_visible_devices_fails_loudly():
+    """`bench.py --gpus N` without torchrun re-executes itself as N ranks only when N GPUs are
+    visible; otherwise it exits non-zero (never silently runs one GPU)."""
+    import torch
+    n = torch.cuda.device_count() + 1
+    env = {k: v for k, v in os.environ.items() if k not in ("WORLD_SIZE", "RANK", "LOCAL_RANK")}
+    r = subprocess.run([sys.executable, os.path.join(ROOT, "bench.py"), "--gpus", str(max(n, 2)),
+                        "--steps", "1", "--warmup", "3"], cwd=ROOT, env=env, timeout=300,
+                       capture_output=True)
+    assert r.returncode != 0
+    assert b"visible CUDA devices" in r.stderr
+    assert not [l for l in r.stdout.decode().splitlines() if l.strip().startswith("{")]
+
+
+def test_world_size_must_match_gpus():
+    env = dict(os.environ, RANK="0", WORLD_SIZE="1", LOCAL_RANK="0")
+    r = subprocess.run([sys.executable, os.path.join(ROOT, "bench.py"), "--gpus", "2", "--steps", "1"],
+                       cwd=ROOT, env=env, timeout=300, capture_output=True)
+    assert r.returncode != 0 and b"one rank per GPU" in r.stderr

@@ -421,7 +421,7 @@ def test_two_level_overlapped_stage_equals_serial_bitwise():
     comm stream beside the ghost-free viscous tiles): forcing the overlap on gives the serial
     result bit for bit."""
     from paper_conf_ipps_davissngmb23_b200 import crocco as cc
-    nc, c0, nf = (32, 24, 80), (4, 5, 2), (40, 20, 136)   # fine level has ghost-free viscous tiles
+    nc, c0, nf = (48, 24, 80), (4, 5, 2), (72, 20, 136)   # fine level has ghost-free viscous tiles
     outs = []
     for ov in (0, 1):
         h = Hier(nc, c0, nf, ((CF, CF),) * 3, synth.Wavy3D(L=(10.0,) * 3, N=nc), dict(terms=3, mu_ref=0.01),
@@ -431,6 +431,7 @@ def test_two_level_overlapped_stage_equals_serial_bitwise():
         cc.crocco_set_overlap(C.ctx, ov)
         A.step(0.005, 2)
         A.sync()
+        assert cc.crocco_overlap_count(F.ctx) == (6 if ov else 0)
         outs.append([C.get(C.U)[0], F.get(F.U)[0]])
         C.close()
         F.close()

@@ -284,6 +284,38 @@ def test_rk3_100_steps_parity(name):
     assert rel_linf(got, inner(U), state_scale(inner(U))) < 1e-9
 
 
+@pytest.mark.parametrize("name", ["weak64", "ramp_down"])
+def test_rk3_100_steps_viscous_parity(name):
+    """The north_star's "<= 1e-9 after 100 RK steps" on the default VISCOUS path (reading 12,
+    PAPER.md:50): the weak recipe (wavy periodic TGV + 1 % noise, Re 1600) at
+    64^3 in 2 x 2 x 1 blocks, and the Mach-6 ramp at 64 x 32 x 16 in 2 x 2 x 2 blocks (no-slip
+    wall, extrapolation faces, Sutherland viscosity).  100 RK3 steps through crocco_rk3_step
+    (CUDA graph) against oracle.advance on the same seeded inputs; floor of reading 30."""
+    if name == "weak64":
+        c = synth.case("weak", scale=8)
+        nb = (2, 2, 1)
+        xyz = c.grid.coords(c.n_global, (0, 0, 0), oracle.GC)
+        U0 = synth.tgv(xyz, noise=0.01, seed=5)
+    else:
+        c = synth.case("ramp", scale=16)
+        nb = (2, 2, 2)
+        xyz = c.grid.coords(c.n_global, (0, 0, 0), oracle.GC)
+        U0 = synth.ramp_state(xyz, c.grid)
+    n = c.n_global
+    pb = Problem(n, c.grid, c.bc, U0, c.phys)
+    _, met, U = pb.oracle_inputs()
+    oracle.advance(n, c.bc, pb.oracle_phys(), c.dt, 100, U, met)
+    S = pb.solver(nb)
+    S.step(c.dt, 100)
+    S.sync()
+    got = pb.gather(S, S.get(S.U))
+    S.close()
+    ref = inner(U)
+    assert np.isfinite(ref).all()
+    err = rel_linf(got, ref, state_scale(ref))
+    assert err < 1e-9, (name, err)
+
+
 # ------------------------------------------------------------------ full size, sampled
 
 def _block_points(bn, rng, k_random):
@@ -302,7 +334,11 @@ def test_full_size_config_sampled(name):
     weak = 512^3 periodic wavy TGV (configs[4]); ramp = 1024 x 512 x 256 Mach-6
     ramp in 2 x 2 x 2 blocks with walls (configs[3]).  Stages 0 and 1; sampled
     points recomputed by the oracle one by one from the GPU's filled 9^3
-    neighbourhood of U and metrics (plus the stage-1 dU)."""
+    neighbourhood of U (plus the stage-1 dU) and the ORACLE's metrics of that
+    neighbourhood, computed from the generator's coordinates around the point
+    (a 1-point block with non-periodic faces, so every window value is computed,
+    none copied); the GPU's metric arrays are compared with those windows at the
+    full size (1.4e9 elements at 512^3: 64-bit offsets)."""
     _torch_cuda()
     c = synth.case(name)
     n = c.n_global
@@ -326,6 +362,27 @@ def test_full_size_config_sampled(name):
     per_block = max(8, 64 // len(blocks))
     pts = [(b, p) for b in range(len(blocks)) for p in _block_points(bn, rng, per_block)]
     ph = oracle.phys(**c.phys)
+    EXT = ((E, E),) * 3
+    Mo = {}
+    worst_m = 0.0
+    for b, p in pts:
+        o = blocks[b][0]
+        gp = (o[0] + p[0], o[1] + p[1], o[2] + p[2])
+        Mo[(b, p)] = oracle.metrics((1, 1, 1), EXT, c.grid.coords((1, 1, 1), gp, oracle.GC))
+        sl = (slice(None), slice(p[2], p[2] + 9), slice(p[1], p[1] + 9), slice(p[0], p[0] + 9))
+        Mg = S.view(S.met[b], b, 10)[sl].cpu().numpy()
+        ref = Mo[(b, p)]
+        # centre point: computed on both sides from the same coordinates (<= 1e-13, SURVEY 8(c)
+        # metrics pin); window: ghost metrics across periodic / inter-block faces are copies of
+        # the owner's (reading 6), equal to the computed value up to coordinate rounding
+        # floor: the largest metric of the window (components that vanish analytically, e.g.
+        # m^zeta_x on the ramp, are compared on the scale of the metric tensor)
+        fl = np.abs(ref[1:]).max()
+        worst_m = max(worst_m, rel_linf(Mg[:1, 4, 4, 4][:, None], ref[:1, 4, 4, 4][:, None]),
+                      rel_linf(Mg[1:, 4, 4, 4][:, None], ref[1:, 4, 4, 4][:, None], fl))
+        assert rel_linf(Mg[:1].reshape(1, -1), ref[:1].reshape(1, -1)) < 1e-11, (name, b, p)
+        assert rel_linf(Mg[1:].reshape(9, -1), ref[1:].reshape(9, -1), fl) < 1e-11, (name, b, p)
+    assert worst_m < 1e-13, (name, worst_m)
     for stage in (0, 1):
         Uin_bufs, dU_bufs = list(S.U), list(S.dU)
         dU_before = {(b, p): S.view(dU_bufs[b], b, 5)[:, p[2] + 4, p[1] + 4, p[0] + 4].cpu().numpy()
@@ -337,10 +394,9 @@ def test_full_size_config_sampled(name):
             Uin = S.view(Uin_bufs[b], b, 5)
             Uout = S.view(S.U[b], b, 5)
             dUv = S.view(dU_bufs[b], b, 5)
-            M = S.view(S.met[b], b, 10)
             sl = (slice(None), slice(p[2], p[2] + 9), slice(p[1], p[1] + 9), slice(p[0], p[0] + 9))
             Uw = np.ascontiguousarray(Uin[sl].cpu().numpy())
-            Mw = np.ascontiguousarray(M[sl].cpu().numpy())
+            Mw = Mo[(b, p)]
             r = oracle.rhs((1, 1, 1), ph, Uw, Mw)
             Uo = np.zeros_like(Uw)
             dUo = np.zeros_like(Uw)
@@ -423,10 +479,12 @@ def test_rk3_step_graph_equals_eager_bitwise():
     assert np.array_equal(outs[0], outs[1])
 
 
-@pytest.mark.parametrize("nb,n", [((1, 1, 1), (40, 40, 140)), ((2, 1, 2), (72, 36, 264))])
+@pytest.mark.parametrize("nb,n", [((1, 1, 1), (72, 40, 140)), ((2, 1, 2), (144, 36, 280))])
 def test_overlapped_stage_equals_serial_bitwise(nb, n):
     """crocco_rk_stage with the ghost fill on the comm stream beside the ghost-free viscous
-    tiles equals the serial stage bit for bit; sizes with interior tiles."""
+    tiles equals the serial stage bit for bit.  Blocks >= 60 wide in x (a
+    ghost-free 32-column tile advancing by 28) and >= 132 deep in z (an interior slab), and
+    crocco_overlap_count proves the overlapped path ran (eager and graph-captured steps)."""
     from paper_conf_ipps_davissngmb23_b200 import crocco as cc
     pb = wavy_random(n, 37, dict(terms=3, mu_law=1, mu_ref=0.02, S=0.3))
     outs = []
@@ -435,10 +493,58 @@ def test_overlapped_stage_equals_serial_bitwise(nb, n):
         cc.crocco_set_overlap(S.ctx, ov)
         S.step(1e-3, 2, graph=False)
         S.step(1e-3, 1, graph=True)
+        S.step(1e-3, 1, graph=True)           # replay
+        S.sync()
+        outs.append(pb.gather(S, S.get(S.U)))
+        assert cc.crocco_overlap_count(S.ctx) == (12 if ov else 0)
+        S.close()
+    assert np.array_equal(outs[0], outs[1])
+
+
+@pytest.mark.parametrize("change", ["limiter", "visc_form", "gamma"])
+def test_graph_dropped_on_set_phys(change):
+    """crocco_set_phys drops the cached RK3 step graphs (they bake in Phys and the kernel
+    variants): graph step -> set_phys -> graph step equals the same sequence taken eagerly,
+    bit for bit, and differs from keeping the old physics."""
+    from paper_conf_ipps_davissngmb23_b200 import crocco as cc
+    n = (32, 24, 20)
+    base = dict(terms=3, mu_ref=0.02)
+    new = dict(base)
+    if change == "limiter":
+        new.update(weno_limiter=1, weno_alpha_rl=5.0)
+    elif change == "visc_form":
+        new.update(visc_form=1)
+    else:
+        new.update(gamma=1.3)
+    pb = wavy_random(n, 47, base)
+    outs = []
+    for graph, switch in ((True, True), (False, True), (True, False)):
+        S = pb.solver((2, 1, 1))
+        S.step(1e-3, 2, graph=graph)
+        if switch:
+            S.set_phys(cc.make_phys(**new))
+        S.step(1e-3, 2, graph=graph)
         S.sync()
         outs.append(pb.gather(S, S.get(S.U)))
         S.close()
     assert np.array_equal(outs[0], outs[1])
+    assert not np.array_equal(outs[0], outs[2])
+
+
+def test_compute_dt_reports_non_finite_state():
+    """A NaN / negative-pressure point is not dropped by the CFL maximum: ComputeDt
+    fails instead of returning a dt from the healthy points."""
+    from paper_conf_ipps_davissngmb23_b200 import crocco as cc
+    n = (16, 12, 8)
+    pb = wavy_random(n, 48)
+    S = pb.solver()
+    dt = cc.crocco_compute_dt(S.ctx, S._ptrs(S.U), S._ptrs(S.met), 0.5)
+    assert dt > 0
+    v = S.view(S.U[0], 0, 5)
+    v[4, 6, 7, 8] = -1.0                     # negative energy -> negative pressure -> NaN c
+    with pytest.raises(cc.CroccoError, match="non-finite"):
+        cc.crocco_compute_dt(S.ctx, S._ptrs(S.U), S._ptrs(S.met), 0.5)
+    S.close()
 
 
 def test_steps_from_host_equals_resident_steps_bitwise():
@@ -528,3 +634,42 @@ def test_degenerate_no_terms_is_exactly_stationary():
     S.sync()
     assert np.array_equal(S.get(S.U)[0][:, 4:-4, 4:-4, 4:-4], U0)
     S.close()
+
+
+# ------------------------------------------------------------------ NCCL halo path on one GPU
+
+@pytest.mark.parametrize("bc,nb,ov", [(PER, (2, 2, 2), 0), (((E, E), (W, E), (P, P)), (2, 1, 2), 0),
+                                      (PER, (2, 1, 1), 1)])
+def test_nccl_loopback_equals_local_and_oracle(bc, nb, ov):
+    """The multi-rank exchange code (pack -> ncclSend/ncclRecv -> unpack, PAPER.md:129-131
+    FillBoundary) and ComputeDt's ncclAllReduce run on hardware through a 1-rank
+    communicator (crocco_set_nccl_loopback): the fill is bitwise the local fill and the oracle's,
+    RK3 steps (also with the overlapped stage) are bitwise the local steps, dt is identical."""
+    from paper_conf_ipps_davissngmb23_b200 import crocco as cc
+    n = (144, 24, 280) if ov else (24, 20, 16)
+    g = synth.Wavy3D(L=(10.0,) * 3, N=n) if bc == PER else synth.Cartesian(h=(0.1, 0.07, 0.05))
+    pb = Problem(n, g, bc, synth.random_state(n, seed=51, amp=0.2), dict(terms=3, mu_ref=0.02))
+    _, met, Uref = pb.oracle_inputs()
+    outs, dts = [], []
+    for loop in (False, True):
+        S = pb.solver(nb)
+        if loop:
+            cc.crocco_set_nccl_loopback(S.ctx, True)
+            S.fill(S.met, cc.FIELD_METRIC)       # metric ghosts through NCCL too
+        cc.crocco_set_overlap(S.ctx, ov)
+        S.fill()
+        S.sync()
+        got = S.get(S.U)
+        bn, blocks = block_slices(n, nb)
+        for b, (o, _) in enumerate(blocks):
+            ref = Uref[:, o[2]:o[2] + bn[2] + 8, o[1]:o[1] + bn[1] + 8, o[0]:o[0] + bn[0] + 8]
+            assert np.array_equal(got[b], ref), (loop, b)
+        dts.append(cc.crocco_compute_dt(S.ctx, S._ptrs(S.U), S._ptrs(S.met), 0.5))
+        S.step(2e-3, 2)
+        S.sync()
+        if ov:
+            assert cc.crocco_overlap_count(S.ctx) == 6
+        outs.append(pb.gather(S, S.get(S.U)))
+        S.close()
+    assert np.array_equal(outs[0], outs[1])
+    assert dts[0] == dts[1]
