@@ -43,18 +43,16 @@ struct LocalBlock {
     Lay L;       // state/metric layout
     Lay C;       // coordinate layout
     VLay V;      // viscous-flux box
-    double *prim = nullptr;
     double *racc = nullptr;  // RHS accumulator R (5 comps, compact interior)
     int64_t rcs = 0;
-    double *fv = nullptr;
-    double *rv = nullptr;    // viscous D4_zeta term (CROCCO_ZDIV_SWEEP != 0)
+    double *fv = nullptr;    // viscous point flux F^_v^eta (4 comps, interior +-2 box)
     double *met2 = nullptr;  // expanded viscous form: 18 second metrics (compact interior, rcs)
     double *p4 = nullptr;    // expanded viscous form: u v w T on the padded box
 };
 
-enum { K_PRIMS = 0, K_FLUX_X, K_FLUX_Y, K_FLUX_Z, K_VISC, K_UPDATE, K_FILL, K_METRICS, K_CFL, K_AMR,
+enum { K_RESERVED = 0, K_FLUX_X, K_FLUX_Y, K_FLUX_Z, K_VISC, K_UPDATE, K_FILL, K_METRICS, K_CFL, K_AMR,
        K_NCLASS };
-const char *k_names[K_NCLASS] = {"prims", "sweep_xi", "sweep_eta", "sweep_zeta_update", "viscous",
+const char *k_names[K_NCLASS] = {"unused", "sweep_xi", "sweep_eta", "sweep_zeta_update", "viscous",
                                  "update", "fill", "metrics", "compute_dt", "amr"};
 // internal fill kind: 5-component state, periodic / inter-block copies only (AverageDown)
 enum { FILL_STATE_COPIES = 100 };
@@ -333,22 +331,8 @@ static void build_plan(const crocco_grid_desc *d, const int nb[3], const int bn[
     }
 }
 
-#ifndef CROCCO_ZDIV_SWEEP
-#define CROCCO_ZDIV_SWEEP 0  // 0: k_visc_tiled writes R, the xi sweep adds (measured equal to 1 / 2, no extra buffer)
-#endif
-static_assert(!CROCCO_VISC_XDIV || CROCCO_ZDIV_SWEEP == 0, "XDIV writes R from k_visc_tiled (ZDIV_SWEEP 0)");
-#ifndef CROCCO_SEG_MIN
-#define CROCCO_SEG_MIN 32       // shortest march segment of a sweep line (small blocks split lines into segments)
-#endif
-#ifndef CROCCO_SEG_WARPS
-#define CROCCO_SEG_WARPS 16384  // lines are split until at least this many warps march
-#endif
-#ifndef CROCCO_FILL_GATHER
-#define CROCCO_FILL_GATHER 1  // single-pass gather fill where it applies (0: always the 3-phase box ops)
-#endif
-#ifndef CROCCO_SWEEP_SMEM
-#define CROCCO_SWEEP_SMEM 1  // shared-memory staged sweeps (k_sweep_s); 0: global-load sweeps
-#endif
+constexpr int SEG_MIN = 32;        // shortest march segment of a sweep line (small blocks split lines)
+constexpr int SEG_WARPS = 16384;   // lines are split until at least this many warps march
 template <int D>
 static constexpr size_t sweep_smem_bytes() {
     return (size_t)(SWEEP_THREADS / 32) * RingGeom<D>::PER_WARP * sizeof(double);
@@ -363,16 +347,13 @@ static cudaError_t sweep_attr1() {
     return e;
 }
 static cudaError_t sweep_attrs() {
+    // the variants rhs_block launches: only the eta sweep carries a viscous interface term
     cudaError_t e = sweep_attr1<0, false>();
     if (e == cudaSuccess) e = sweep_attr1<1, false>();
     if (e == cudaSuccess) e = sweep_attr1<2, false>();
-    if (e == cudaSuccess) e = sweep_attr1<0, true>();
     if (e == cudaSuccess) e = sweep_attr1<1, true>();
-    if (e == cudaSuccess) e = sweep_attr1<2, true>();
     if (e == cudaSuccess)
         e = cudaFuncSetAttribute(k_visc_tiled, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)VISC_SMEM);
-    if (e == cudaSuccess)
-        e = cudaFuncSetAttribute(k_visc_div, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)VDIV_SMEM);
     return e;
 }
 
@@ -439,11 +420,9 @@ static Phys to_phys(const crocco_phys *p) {
     // (LLF 1/2 folded, flux.cuh): b = (48/13) beta of (g +- lambda w)/2
     ph.aal_b = p->weno_alpha_al * (4.0 * WENO_BSCALE);
     ph.visc_form = p->visc_form;
-#if CROCCO_WENO_FOLD
     // only the ratios C_k / C_0 enter W (weno.cuh); alpha_0 then needs no multiply
     const double c0 = ph.wC[0];
     for (int k = 0; k < 4; k++) ph.wC[k] = k == 0 ? 1.0 : ph.wC[k] / c0;
-#endif
     return ph;
 }
 
@@ -481,10 +460,8 @@ crocco_status crocco_set_phys(crocco_ctx c, const crocco_phys *p) {
 
 static void free_ctx(crocco_ctx c) {
     for (auto &b : c->loc) {
-        cudaFree(b.prim);
         cudaFree(b.racc);
         cudaFree(b.fv);
-        cudaFree(b.rv);
         cudaFree(b.met2);
         cudaFree(b.p4);
     }
@@ -557,16 +534,11 @@ crocco_status crocco_init_grid(const crocco_grid_desc *desc, const crocco_phys *
         return true;
     };
     for (auto &b : c->loc) {
-        // primitives are only materialised by the global-load sweeps; point viscous fluxes only
-        // when the divergence is not fused (k_visc_div keeps them on chip)
-        bool ok = CROCCO_SWEEP_SMEM || alloc(&b.prim, NPRIM * b.L.cs);
+        // R accumulator; of the viscous point fluxes only F^_v^eta goes to HBM (k_visc_tiled
+        // differences the xi and zeta ones on chip)
         b.rcs = rup((int64_t)b.g.n[0] * b.g.n[1] * b.g.n[2], 32);
-        ok = ok && alloc(&b.racc, 5 * b.rcs);
-        ok = ok && (!(CROCCO_SWEEP_SMEM && !CROCCO_VISC_DIV && CROCCO_VISC_ZDIV && CROCCO_ZDIV_SWEEP) ||
-                    alloc(&b.rv, 5 * b.rcs));
-        // point viscous fluxes kept in HBM: xi and eta (ZDIV), eta only (ZDIV + XDIV), all three otherwise
-        ok = ok && ((CROCCO_SWEEP_SMEM && CROCCO_VISC_DIV) ||
-                    alloc(&b.fv, (CROCCO_SWEEP_SMEM && CROCCO_VISC_ZDIV ? (CROCCO_VISC_XDIV ? 4 : 8) : 12) * b.V.cs));
+        bool ok = alloc(&b.racc, 5 * b.rcs);
+        ok = ok && alloc(&b.fv, 4 * b.V.cs);
         if (!ok) {
             cudaGetLastError();
             free_ctx(c);
@@ -893,7 +865,7 @@ static crocco_status check_ptrs(crocco_ctx c, double *const *p, const char *what
 // single-pass gather fill (fill.cuh k_fill_gather): state fills whose faces are all PERIODIC,
 // EXTRAP, WALL or DIRICHLET with every block on this rank (bitwise equal to the 3 phases)
 static bool gather_fill_ok(const crocco_ctx_s *c, int32_t kind) {
-    if (kind != CROCCO_FIELD_STATE || CROCCO_FILL_GATHER == 0 || c->loopback) return false;
+    if (kind != CROCCO_FIELD_STATE || c->loopback) return false;
     if (c->loc.size() != c->all.size() || c->loc.size() > AMR_MAX_LOCAL || c->all.size() > AMR_MAX_BLOCKS)
         return false;
     for (int d = 0; d < 3; d++)
@@ -1030,8 +1002,7 @@ static const double RK_B[3] = {1.0 / 3.0, 15.0 / 16.0, 8.0 / 15.0};
 // returns false if the block has none or the configuration has no such split
 static bool visc_overlap_possible(crocco_ctx c) {
     const bool viscous = (c->ph.terms & CROCCO_TERM_VISCOUS) != 0 && c->ph.visc_form == 0;
-    if (!(viscous && CROCCO_SWEEP_SMEM && !CROCCO_VISC_DIV && CROCCO_VISC_ZDIV && CROCCO_ZDIV_SWEEP == 0))
-        return false;
+    if (!viscous) return false;
     for (const auto &b : c->loc) {
         const VTiles t = visc_interior_tiles(b.L, visc_slab(b.L, b.V, true));
         if (t.x1 > t.x0 && t.y1 > t.y0 && t.z1 > t.z0) return true;
@@ -1055,63 +1026,40 @@ static crocco_status rhs_block(crocco_ctx c, const LocalBlock &b, const double *
     const bool inviscid = (ph.terms & CROCCO_TERM_INVISCID) != 0;
     const bool vexp = (ph.terms & CROCCO_TERM_VISCOUS) != 0 && ph.visc_form == 1;  // readings 27-28
     const bool viscous = (ph.terms & CROCCO_TERM_VISCOUS) != 0 && !vexp;
-    const int64_t np = (int64_t)(b.g.n[0] + 2 * G) * (b.g.n[1] + 2 * G) * (b.g.n[2] + 2 * G);
-    if (!CROCCO_SWEEP_SMEM)  // the staged sweeps and the tiled viscous kernel compute their own primitives
-        LAUNCH(c, K_PRIMS, k_prims<<<cdiv(np, 256), 256, 0, c->stream>>>(U, b.prim, b.L, ph));
-    const bool vdiv = viscous && CROCCO_SWEEP_SMEM && CROCCO_VISC_DIV;  // fused viscous divergence -> R
-    // D4_zeta of the zeta point flux inside k_visc_tiled -> R (the zeta sweep carries no viscous term)
-    const bool zdiv = viscous && CROCCO_SWEEP_SMEM && !CROCCO_VISC_DIV && CROCCO_VISC_ZDIV;
-    // where the D4_zeta term is added: 0 -> k_visc_tiled writes R and the xi sweep adds to it;
-    // 1 / 2 -> separate buffer added by the eta / zeta sweep
-    const int zsw = CROCCO_ZDIV_SWEEP;
-    double *rvz = (zdiv && zsw != 0) ? b.rv : b.racc;
     if (vexp) {  // expanded viscous form: V / J -> R comps 1..4, the xi sweep adds (mode 4)
         if (!b.met2 || !b.p4)
             return fail(c, CROCCO_ERR_STATE, "visc_form = 1 needs crocco_init_metrics2");
         LAUNCH(c, K_VISC, k_prims4<<<cdiv(b.L.cs, 256), 256, 0, c->stream>>>(U, b.p4, b.L, ph));
         const int64_t ni = (int64_t)b.g.n[0] * b.g.n[1] * b.g.n[2];
         LAUNCH(c, K_VISC, k_visc_exp<<<cdiv(ni, 128), 128, 0, c->stream>>>(b.p4, M, b.met2, b.racc, b.rcs, b.L, ph));
-    } else if (vdiv) {
-        const unsigned nt = (unsigned)(((b.g.n[0] + DTX - 1) / DTX) * ((b.g.n[1] + DTY - 1) / DTY) *
-                                       ((b.g.n[2] + DK - 1) / DK));
-        LAUNCH(c, K_VISC, k_visc_div<<<nt, DNT, VDIV_SMEM, c->stream>>>(U, M, b.racc, b.rcs, b.L, ph));
-    } else if (viscous) {
-#if CROCCO_SWEEP_SMEM
-        if (visc_sel != 1) {  // sel 1 (interior tiles) was launched by visc_interior() beside the fill
-            const int nz = zdiv ? b.g.n[2] : b.V.b2;
-            const int vk = visc_slab(b.L, b.V, visc_sel != 0);
-            int64_t nt = (int64_t)visc_tiles_x(b.L, b.V) * ((b.V.b1 + VTY - 1) / VTY) * ((nz + vk - 1) / vk);
-            if (visc_sel == 2) {
-                const VTiles t = visc_interior_tiles(b.L, vk);
-                nt -= (int64_t)(t.x1 - t.x0) * (t.y1 - t.y0) * (t.z1 - t.z0);
-            }
-            if (nt > 0)
-                LAUNCH(c, K_VISC, k_visc_tiled<<<(unsigned)nt, VTX * VTY, VISC_SMEM, c->stream>>>(
-                                      U, M, b.fv, b.L, b.V, ph, rvz, b.rcs, visc_sel, vk));
+    } else if (viscous && visc_sel != 1) {
+        // k_visc_tiled: R comps 1..4 = D4_xi + D4_zeta of the point fluxes, F^_v^eta -> HBM
+        // (sel 1, the ghost-free tiles, was launched by visc_interior() beside the fill)
+        const int vk = visc_slab(b.L, b.V, visc_sel != 0);
+        int64_t nt = (int64_t)visc_tiles_x(b.L) * ((b.V.b1 + VTY - 1) / VTY) * ((b.g.n[2] + vk - 1) / vk);
+        if (visc_sel == 2) {
+            const VTiles t = visc_interior_tiles(b.L, vk);
+            nt -= (int64_t)(t.x1 - t.x0) * (t.y1 - t.y0) * (t.z1 - t.z0);
         }
-#else
-        const int64_t nv = (int64_t)b.V.b0 * b.V.b1 * b.V.b2;
-        LAUNCH(c, K_VISC, k_visc<<<cdiv(nv, 256), 256, 0, c->stream>>>(b.prim, M, b.fv, b.L, b.V, ph));
-#endif
+        if (nt > 0)
+            LAUNCH(c, K_VISC, k_visc_tiled<<<(unsigned)nt, VTX * VTY, VISC_SMEM, c->stream>>>(
+                                  U, M, b.fv, b.L, b.V, ph, b.racc, b.rcs, visc_sel, vk));
     }
     for (int d = 0; d < 3; d++) {
         SweepArgs a;
         memset(&a, 0, sizeof a);
         a.in.U = U;
-        a.in.P = b.prim;
         a.in.M = M;
-        // FV holds (xi, eta) point fluxes, or eta only with XDIV (the xi sweep then reads none)
-        const int fvd = (CROCCO_SWEEP_SMEM && CROCCO_VISC_ZDIV && CROCCO_VISC_XDIV) ? (d > 0 ? d - 1 : 0) : d;
-        a.in.FV = b.fv + (int64_t)4 * fvd * b.V.cs;
+        a.in.FV = b.fv;  // F^_v^eta: only the eta sweep has a viscous interface term
         a.in.cs = b.L.cs;
         a.in.vcs = b.V.cs;
         a.V = b.V;
         a.R = b.racc;
         a.rcs = b.rcs;
         a.inv = inviscid && (ph.dir_mask >> d & 1);
-        a.visc = viscous && !vdiv && !(zdiv && d == 2) && !(zdiv && CROCCO_VISC_XDIV && d == 0);
-        a.mode = d == 0 ? ((vexp || vdiv || (zdiv && zsw == 0)) ? 4 : 0) : (d == 1 ? 1 : final_mode);
-        a.RV = (zdiv && zsw != 0 && d == zsw) ? b.rv : nullptr;
+        a.visc = viscous && d == 1;
+        // R: the viscous kernel wrote comps 1..4 (xi sweep adds, mode 4), else the xi sweep writes
+        a.mode = d == 0 ? ((ph.terms & CROCCO_TERM_VISCOUS) ? 4 : 0) : (d == 1 ? 1 : final_mode);
         a.rhs = rhs;
         a.Uin = Uin;
         a.Uout = Uout;
@@ -1128,12 +1076,11 @@ static crocco_status rhs_block(crocco_ctx c, const LocalBlock &b, const double *
         int64_t seg = nd;
         // fewer lines than SMs (e.g. Sod's 4 xi lines): segments down to 8 points (measured 8.6e7 -> 1.1e8
         // point-stages/s on Sod); otherwise >= 32 (shorter segments measured slower on the 64^3 vortex)
-        const int64_t segmin = lines < 148 ? 8 : CROCCO_SEG_MIN;
-        while (lines * ((nd + seg - 1) / seg) < CROCCO_SEG_WARPS && seg > segmin) seg = (seg + 1) / 2;
+        const int64_t segmin = lines < 148 ? 8 : SEG_MIN;
+        while (lines * ((nd + seg - 1) / seg) < SEG_WARPS && seg > segmin) seg = (seg + 1) / 2;
         a.seg = (int)seg;
         const int64_t warps = lines * ((nd + seg - 1) / seg);
         const unsigned grid = cdiv(warps * 32, SWEEP_THREADS);
-#if CROCCO_SWEEP_SMEM
 #define SWEEP_LAUNCH(DD, VV)                                                                              \
     do {                                                                                                  \
         if (ph.lim)                                                                                       \
@@ -1141,15 +1088,10 @@ static crocco_status rhs_block(crocco_ctx c, const LocalBlock &b, const double *
         else                                                                                              \
             k_sweep_s<DD, VV, false><<<grid, SWEEP_THREADS, sweep_smem_bytes<DD>(), c->stream>>>(a, b.L, ph); \
     } while (0)
-        if (d == 0) LAUNCH(c, K_FLUX_X, if (a.visc) SWEEP_LAUNCH(0, true); else SWEEP_LAUNCH(0, false));
+        if (d == 0) LAUNCH(c, K_FLUX_X, SWEEP_LAUNCH(0, false));
         else if (d == 1) LAUNCH(c, K_FLUX_Y, if (a.visc) SWEEP_LAUNCH(1, true); else SWEEP_LAUNCH(1, false));
-        else LAUNCH(c, K_FLUX_Z, if (a.visc) SWEEP_LAUNCH(2, true); else SWEEP_LAUNCH(2, false));
+        else LAUNCH(c, K_FLUX_Z, SWEEP_LAUNCH(2, false));
 #undef SWEEP_LAUNCH
-#else
-        if (d == 0) LAUNCH(c, K_FLUX_X, k_sweep<0><<<grid, SWEEP_THREADS, 0, c->stream>>>(a, b.L, ph));
-        else if (d == 1) LAUNCH(c, K_FLUX_Y, k_sweep<1><<<grid, SWEEP_THREADS, 0, c->stream>>>(a, b.L, ph));
-        else LAUNCH(c, K_FLUX_Z, k_sweep<2><<<grid, SWEEP_THREADS, 0, c->stream>>>(a, b.L, ph));
-#endif
     }
     return CROCCO_OK;
 }

@@ -21,57 +21,24 @@
 
 namespace crocco {
 
-#ifndef CROCCO_FIELD_ROLLED
-#define CROCCO_FIELD_ROLLED 0  // 1: keep the characteristic-field loop rolled (fewer live registers)
-#endif
-#ifndef CROCCO_PL_SMEM
-#define CROCCO_PL_SMEM 0  // 1: stencil pressures re-read from the ring per field (fewer live registers)
-#endif
-#ifndef CROCCO_DEFER_DIV
-#define CROCCO_DEFER_DIV 1  // 1: the five WENO-pair divisions after the field loop (independent chains)
-#endif
-#ifndef CROCCO_LAM_TREE
 // bit D: the three 6-point maxima of direction D as depth-3 trees instead of 6-deep chains (bitwise
 // equal); measured: zeta -0.2 ms, xi +0.3 ms per 512^3 launch -> zeta only
-#define CROCCO_LAM_TREE 4
-#endif
-#ifndef CROCCO_SWEEP_UREG
-#define CROCCO_SWEEP_UREG 0  // 1: hold the 6x5 stencil states in registers; 0: re-read per field
-#endif
+constexpr int LAM_TREE = 4;
 
 struct FluxIn {
     const double *__restrict__ U;
-    const double *__restrict__ P;
     const double *__restrict__ M;
     const double *__restrict__ FV;  // point viscous fluxes of this direction (4 comps) or null
-    int64_t cs;                     // component stride of U / P / M
+    int64_t cs;                     // component stride of U / M
     int64_t vcs;                    // component stride of FV
 };
 
-// Stencil accessors: conserved state U(l, c), primitives P(l, k) (k = PU..PH),
+// Stencil accessor (SAcc): conserved state U(l, c), primitives P(l, k) (k = PU..PH),
 // the metric row m^d M(l, a) and the point viscous flux of direction d FV(l, q)
 // (q = momentum x, y, z, energy) at stencil point l = 0..5 (points i-2..i+3).
-template <int D>
-struct GAcc {  // straight from the global arrays (L1/L2 cached)
-    const double *__restrict__ u;
-    const double *__restrict__ p;
-    const double *__restrict__ m;   // metric component 1+3D
-    const double *__restrict__ fv;  // FV of direction D
-    int64_t cs, p0, s, vcs, v0, vs; // v0: FV index of point i-2
-    __device__ __forceinline__ double U(int l, int c) const { return u[c * cs + p0 + l * s]; }
-    __device__ __forceinline__ double P(int l, int k) const { return p[k * cs + p0 + l * s]; }
-    __device__ __forceinline__ double M(int l, int a) const { return m[a * cs + p0 + l * s]; }
-    __device__ __forceinline__ double FV(int l, int q) const { return fv[q * vcs + v0 + l * vs]; }
-    __device__ __forceinline__ double SR(int l) const { return P(l, PSR); }  // sqrt(rho)
-    __device__ __forceinline__ double H(int l) const { return P(l, PH); }    // total enthalpy
-};
-
 // shared-memory ring of a warp: value v of ring point q in column col at
 // sv[v * VS + (q & (NR-1)) * PS + col]
-#ifndef CROCCO_RING_LEAN
-#define CROCCO_RING_LEAN 0  // 1: stage u v w p c only; sqrt(rho), H derived per interface
-#endif
-enum { SV_U = 0, SV_M = 5, SV_FV = 8, SV_P = 12, SV_N = CROCCO_RING_LEAN ? 17 : 19 };
+enum { SV_U = 0, SV_M = 5, SV_FV = 8, SV_P = 12, SV_N = 19 };
 template <int NR, int PS>
 struct SAcc {
     const double *sv;
@@ -84,17 +51,12 @@ struct SAcc {
     __device__ __forceinline__ double P(int l, int k) const { return at_(SV_P + k, l); }
     __device__ __forceinline__ double M(int l, int a) const { return at_(SV_M + a, l); }
     __device__ __forceinline__ double FV(int l, int q) const { return at_(SV_FV + q, l); }
-#if CROCCO_RING_LEAN
-    __device__ __forceinline__ double SR(int l) const { return U(l, 0) * rsqrt_nr(U(l, 0)); }
-    __device__ __forceinline__ double H(int l) const { return (U(l, 4) + P(l, PP)) * rcp_nr(U(l, 0)); }
-#else
-    __device__ __forceinline__ double SR(int l) const { return P(l, PSR); }
-    __device__ __forceinline__ double H(int l) const { return P(l, PH); }
-#endif
+    __device__ __forceinline__ double SR(int l) const { return P(l, PSR); }  // sqrt(rho)
+    __device__ __forceinline__ double H(int l) const { return P(l, PH); }    // total enthalpy
 };
 
 // Total interface flux F = F^_inv - h_v of direction D at interface i+1/2.
-// A: stencil accessor (flux.cuh GAcc / SAcc).
+// A: stencil accessor (SAcc).
 template <int D, class Acc, bool LIM = false>
 __device__ __forceinline__ void total_flux(const Acc &A, bool inv, bool visc, const Phys &ph,
                                            double F[5]) {
@@ -132,29 +94,19 @@ __device__ __forceinline__ void total_flux(const Acc &A, bool inv, bool visc, co
         const double alph = rt * ict * SQ12;   // rho/(sqrt2 c)
         const double beta = irt * ict * SQ12;  // 1/(sqrt2 rho c)
 
-        // stencil points
-#if CROCCO_SWEEP_UREG
-        double Ul[6][5];
-#define UL(l, c) Ul[l][c]
-#else
+        // stencil points (the states are re-read from the ring per field: holding the 6 x 5
+        // states in registers measured slower)
 #define UL(l, c) A.U(l, c)
-#endif
         double th[6], pl[6];
         double lam0 = 0.0, lam3 = 0.0, lam4 = 0.0;
-        constexpr bool lam_tree = (CROCCO_LAM_TREE >> D) & 1;
+        constexpr bool lam_tree = (LAM_TREE >> D) & 1;
         double a0[6], a3[6], a4[6];
 #pragma unroll
         for (int l = 0; l < 6; l++) {
-#if CROCCO_SWEEP_UREG
-#pragma unroll
-            for (int c = 0; c < 5; c++) Ul[l][c] = A.U(l, c);
-#endif
             const double t = fma(nx, A.P(l, PU), fma(ny, A.P(l, PV), nz * A.P(l, PW)));
             const double cl = A.P(l, PC);
             th[l] = t;
-#if !CROCCO_PL_SMEM
             pl[l] = A.P(l, PP);
-#endif
             if constexpr (lam_tree) {
                 a0[l] = fabs(t);
                 a3[l] = fabs(t + cl);
@@ -176,14 +128,10 @@ __device__ __forceinline__ void total_flux(const Acc &A, bool inv, bool visc, co
         const double cx = ny * wt - nz * vt, cy = nz * ut - nx * wt, cz = nx * vt - ny * ut;
         const double ph1 = phi2 * ph.igm1;
         double f0 = 0.0, f1 = 0.0, f2 = 0.0, f3 = 0.0, f4 = 0.0;
-#if CROCCO_DEFER_DIV
+        // the five WENO-pair divisions are issued after the field loop (independent chains;
+        // inside the loop measured slower); the loop is unrolled (rolled: +14 %)
         double gb[5], gn[5], gd[5];
-#endif
-#if CROCCO_FIELD_ROLLED
-#pragma unroll 1
-#else
 #pragma unroll
-#endif
         for (int sf = 0; sf < 5; sf++) {
             double L0, L1, L2, L3, L4, R0, R1, R2, R3, R4, lam, kA, kB;
             if (sf < 3) {
@@ -243,15 +191,10 @@ __device__ __forceinline__ void total_flux(const Acc &A, bool inv, bool visc, co
             for (int l = 0; l < 6; l++) {
                 const double w =
                     fma(L0, UL(l, 0), fma(L1, UL(l, 1), fma(L2, UL(l, 2), fma(L3, UL(l, 3), L4 * UL(l, 4)))));
-#if CROCCO_PL_SMEM
-                const double g = fma(th[l], w, A.P(l, PP) * fma(kB, th[l], kA));
-#else
                 const double g = fma(th[l], w, pl[l] * fma(kB, th[l], kA));
-#endif
                 gp[l] = fma(lam, w, g);
                 gm[l] = fma(-lam, w, g);
             }
-#if CROCCO_DEFER_DIV
             const WenoFrac wf = weno_pair_frac<LIM>(gp, gm, eps_b, ph.wC, &ph);
             gb[sf] = wf.base;
             gn[sf] = wf.num;
@@ -289,9 +232,6 @@ __device__ __forceinline__ void total_flux(const Acc &A, bool inv, bool visc, co
                 R3 = alph * fma(sc, nz, wt);
                 R4 = alph * fma(phi2 + c2, ph.igm1, sc * tht);
             }
-#else
-            const double gh = weno_pair<LIM>(gp, gm, eps_b, ph.wC, &ph);
-#endif
             f0 = fma(R0, gh, f0);
             f1 = fma(R1, gh, f1);
             f2 = fma(R2, gh, f2);

@@ -22,20 +22,10 @@
 
 namespace crocco {
 
-#ifndef CROCCO_SWEEP_MINB
-#define CROCCO_SWEEP_MINB 1  // min CTAs/SM (register cap); the staged ring allows 2 CTAs x 4 warps
-#endif
-#ifndef CROCCO_CARRY_SMEM
-#define CROCCO_CARRY_SMEM 2  // bit D: sweep D passes neighbour / carried interface fluxes through shared
-                             // memory instead of a register carry (measured: eta -4 %, xi +16 %, zeta 0)
-#endif
-#ifndef CROCCO_PRIMS_LATE
-#define CROCCO_PRIMS_LATE 0  // 1: next chunk's primitives computed at the end of the step (registers)
-#endif
-#ifndef CROCCO_SWEEP_THREADS
-#define CROCCO_SWEEP_THREADS 128
-#endif
-constexpr int SWEEP_THREADS = CROCCO_SWEEP_THREADS;
+// bit D: sweep D passes neighbour / carried interface fluxes through shared memory instead of a
+// register carry (measured: eta -4 %, xi +16 %, zeta 0)
+constexpr int CARRY_SMEM = 2;
+constexpr int SWEEP_THREADS = 128;  // 4 warps, 2 CTAs per SM (register file: 8 warps x 255 registers)
 
 struct SweepArgs {
     FluxIn in;
@@ -44,135 +34,14 @@ struct SweepArgs {
     int64_t rcs;        // its component stride
     int inv, visc;      // terms evaluated in this direction
     int mode;           // 0 write R, 1 add to R, 2 rhs = J R, 3 RK update,
-                        // 4 add to the viscous divergence in R comps 1..4 (k_visc_div), write comp 0
-    int seg;            // march segment (D = 1, 2)
-    const double *RV;   // viscous D4_zeta term (comps 1..4, R layout) added by this sweep, or null
+                        // 4 add to the viscous divergence in R comps 1..4 (k_visc_tiled), write comp 0
+    int seg;            // march segment
     double *rhs;        // mode 2 (padded layout)
     const double *Uin;  // mode 3 (padded layout)
     double *Uout, *dU;
     double A, B, dt;
     int stage;
 };
-
-// finish / accumulate the contribution dF = F_{i-1/2} - F_{i+1/2} at interior point (i,j,k)
-__device__ __forceinline__ void contribute(const SweepArgs &a, const Lay &L, int i, int j, int k,
-                                           const double dF[5]) {
-    const int64_t r = (int64_t)i + (int64_t)L.n0 * (j + (int64_t)L.n1 * k);
-    if (a.mode == 0) {
-#pragma unroll
-        for (int c = 0; c < 5; c++) a.R[c * a.rcs + r] = dF[c];
-        return;
-    }
-    double Rt[5];
-#pragma unroll
-    for (int c = 0; c < 5; c++) Rt[c] = a.R[c * a.rcs + r] + dF[c];
-    if (a.mode == 1) {
-#pragma unroll
-        for (int c = 0; c < 5; c++) a.R[c * a.rcs + r] = Rt[c];
-        return;
-    }
-    const int64_t p = at(L, i, j, k);
-    const double J = a.in.M[p];
-    if (a.mode == 2) {
-#pragma unroll
-        for (int c = 0; c < 5; c++) a.rhs[c * L.cs + p] = J * Rt[c];
-        return;
-    }
-#pragma unroll
-    for (int c = 0; c < 5; c++) {
-        const int64_t q = c * L.cs + p;
-        const double rr = J * Rt[c];
-        const double du = (a.stage == 0) ? a.dt * rr : fma(a.A, a.dU[q], a.dt * rr);
-        a.dU[q] = du;
-        a.Uout[q] = fma(a.B, du, a.Uin[q]);
-    }
-}
-
-template <int D>
-__global__ void __launch_bounds__(SWEEP_THREADS, CROCCO_SWEEP_MINB) k_sweep(const __grid_constant__ SweepArgs a,
-                                                                        const Lay L, const Phys ph) {
-    // warp tile: D = 0: 4 lines x 8 consecutive interfaces (lane = 8*line + offset);
-    //            D = 1, 2: 8 consecutive i x 4 consecutive interfaces (lane = 8*offset + i).
-    constexpr int WS = (D == 0) ? 8 : 4;  // interfaces per step along the sweep
-    constexpr int WT = 32 / WS;           // transverse lines per warp
-    const int lane = threadIdx.x & 31;
-    const int ls = (D == 0) ? (lane & 7) : (lane >> 3);  // sweep offset
-    const int lt = (D == 0) ? (lane >> 3) : (lane & 7);  // transverse offset
-    const int64_t gw = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
-    const bool inv = a.inv != 0, visc = a.visc != 0;
-    // swept extent and segments of the march
-    const int nd = D == 0 ? L.n0 : (D == 1 ? L.n1 : L.n2);
-    const int nseg = (nd + a.seg - 1) / a.seg;
-    bool lvalid;
-    int ci = 0, cj = 0, ck = 0;  // point coordinates of the line (swept one unused)
-    int sg;
-    if (D == 0) {
-        const int64_t ntl = ((int64_t)L.n1 * L.n2 + WT - 1) / WT;
-        if (gw >= ntl * nseg) return;
-        sg = (int)(gw / ntl);
-        const int64_t tline = (gw % ntl) * WT + lt;  // j + n1 k
-        lvalid = tline < (int64_t)L.n1 * L.n2;
-        if (lvalid) {
-            cj = (int)(tline % L.n1);
-            ck = (int)(tline / L.n1);
-        }
-    } else {
-        const int tiles = (L.n0 + WT - 1) / WT;
-        const int nother = (D == 1) ? L.n2 : L.n1;
-        const int64_t ntl = (int64_t)tiles * nother;
-        if (gw >= ntl * nseg) return;
-        sg = (int)(gw / ntl);
-        const int64_t r = gw % ntl;
-        const int iv = (int)(r % tiles) * WT + lt;
-        const int oo = (int)(r / tiles);
-        lvalid = iv < L.n0;
-        if (lvalid) {
-            ci = iv;
-            if (D == 1) ck = oo;
-            else cj = oo;
-        }
-    }
-    const int e0 = sg * a.seg, e1 = min(nd, e0 + a.seg);
-    const int64_t s = (D == 0) ? 1 : (D == 1 ? L.py : L.pz);
-    const int64_t vs = (D == 0) ? 1 : (D == 1 ? a.V.py : a.V.pz);
-    const int nsteps = (e1 - e0 + 1 + WS - 1) / WS;  // interfaces e0-1 .. e1-1
-    double F[5], Fc[5];
-#pragma unroll
-    for (int c = 0; c < 5; c++) Fc[c] = 0.0;
-    for (int st = 0; st < nsteps; st++) {
-        const int e = e0 - 1 + WS * st + ls;  // this lane's interface e+1/2
-        const bool act = lvalid && e <= e1 - 1;
-        const int pi = D == 0 ? e : ci, pj = D == 1 ? e : cj, pk = D == 2 ? e : ck;
-        if (act) {
-            // the single call site of the flux for every interface (bitwise decomposition invariance)
-            const int qi = D == 0 ? e - 2 : pi, qj = D == 1 ? e - 2 : pj, qk = D == 2 ? e - 2 : pk;
-            const int vi = D == 0 ? e - 1 : pi, vj = D == 1 ? e - 1 : pj, vk = D == 2 ? e - 1 : pk;
-            const GAcc<D> A{a.in.U, a.in.P, a.in.M + (int64_t)(1 + 3 * D) * a.in.cs, a.in.FV,
-                            a.in.cs, at(L, qi, qj, qk), s, a.in.vcs, vat(a.V, vi, vj, vk) - vs, vs};
-            if (ph.lim) total_flux<D, GAcc<D>, true>(A, inv, visc, ph, F);
-            else total_flux<D, GAcc<D>, false>(A, inv, visc, ph, F);
-        } else {
-#pragma unroll
-            for (int c = 0; c < 5; c++) F[c] = 0.0;
-        }
-        double dF[5];
-#pragma unroll
-        for (int c = 0; c < 5; c++) {
-            double Fm;
-            if (D == 0) {
-                Fm = __shfl_up_sync(0xffffffffu, F[c], 1, 8);
-                if (ls == 0) Fm = Fc[c];
-                Fc[c] = __shfl_sync(0xffffffffu, F[c], 7, 8);
-            } else {
-                Fm = __shfl_up_sync(0xffffffffu, F[c], 8);
-                if (ls == 0) Fm = Fc[c];
-                Fc[c] = __shfl_sync(0xffffffffu, F[c], 24 + lt);
-            }
-            dF[c] = Fm - F[c];
-        }
-        if (act && e >= e0) contribute(a, L, pi, pj, pk, dF);
-    }
-}
 
 // ---------------------------------------------------------------------------
 // Shared-memory staged sweep (same tiles and arithmetic as k_sweep): each warp
@@ -198,14 +67,14 @@ struct RingGeom {
     static constexpr int C = 32 / WS;              // columns (lines) per warp
     static constexpr int LA = (D == 0) ? 1 : 2;    // chunks ahead needed by a step
     static constexpr int NR = (D == 0) ? 32 : 16;  // ring points (>= (LA + 2) * WS, power of 2)
-    static constexpr int NCB = 20;                 // prefetched accumulate/update operands per lane
-    static constexpr bool CARRY = (CROCCO_CARRY_SMEM >> D) & 1;
+    static constexpr int NCB = 16;                 // prefetched accumulate/update operands per lane
+    static constexpr bool CARRY = (CARRY_SMEM >> D) & 1;
     static constexpr int NFC = CARRY ? 2 * 5 * 32 : 0;  // interface fluxes of two steps
     static constexpr int PER_WARP = SV_N * NR * C + NCB * 32 + NFC;  // doubles
 };
 
 template <int D, bool VISC, bool LIM>
-__global__ void __launch_bounds__(SWEEP_THREADS, CROCCO_SWEEP_MINB) k_sweep_s(const __grid_constant__ SweepArgs a,
+__global__ void __launch_bounds__(SWEEP_THREADS, 1) k_sweep_s(const __grid_constant__ SweepArgs a,
                                                                           const Lay L, const Phys ph) {
     using RG = RingGeom<D>;
     constexpr int WS = RG::WS, C = RG::C, LA = RG::LA, NR = RG::NR;
@@ -326,16 +195,13 @@ __global__ void __launch_bounds__(SWEEP_THREADS, CROCCO_SWEEP_MINB) k_sweep_s(co
         if (q > qmax) return;
         double *bq = sv + (q & (NR - 1)) * C + lt;
 #pragma unroll
-        for (int k = 0; k < (CROCCO_RING_LEAN ? 5 : 7); k++) bq[(SV_P + k) * VS] = pv[k];
+        for (int k = 0; k < 7; k++) bq[(SV_P + k) * VS] = pv[k];
     };
     auto prims = [&](int ch) {
         double pv[7];
         prim_calc(ch, pv);
         prim_store(ch, pv);
     };
-#if CROCCO_PRIMS_LATE
-    double pnext[7];  // primitives of chunk st+LA, computed at the end of step st-1
-#endif
 
     // prologue: chunks 0 .. LA staged with primitives
     for (int ch = 0; ch <= LA; ch++) issue(ch);
@@ -359,14 +225,10 @@ __global__ void __launch_bounds__(SWEEP_THREADS, CROCCO_SWEEP_MINB) k_sweep_s(co
     for (int c = 0; c < 5; c++) Fc[c] = 0.0;
     for (int st = 0; st < nsteps; st++, rr += rstep, pp += pstep) {
         if (st > 0) {
-#if CROCCO_PRIMS_LATE
-            prim_store(st + LA, pnext);
-#else
             // chunk st+LA landed -> primitives
             cp_async_wait_all();
             __syncwarp();
             prims(st + LA);
-#endif
             __syncwarp();
         }
         const int e = e0 - 1 + WS * st + ls;  // this lane's interface e+1/2
@@ -376,10 +238,6 @@ __global__ void __launch_bounds__(SWEEP_THREADS, CROCCO_SWEEP_MINB) k_sweep_s(co
 #pragma unroll
             for (int c = 0; c < 5; c++)
                 if (c > 0 || a.mode != 4) cp_async8(cb + 32 * c, a.R + c * a.rcs + rr);
-            if (a.RV) {
-#pragma unroll
-                for (int c = 1; c < 5; c++) cp_async8(cb + 32 * (15 + c), a.RV + c * a.rcs + rr);
-            }
             if (a.mode >= 2) {
                 cp_async8(cb + 32 * 5, a.in.M + pp);
                 if (a.mode == 3) {
@@ -441,10 +299,6 @@ __global__ void __launch_bounds__(SWEEP_THREADS, CROCCO_SWEEP_MINB) k_sweep_s(co
                 double Rt[5];
 #pragma unroll
                 for (int c = 0; c < 5; c++) Rt[c] = (c == 0 && a.mode == 4) ? dF[0] : cb[32 * c] + dF[c];
-                if (a.RV) {
-#pragma unroll
-                    for (int c = 1; c < 5; c++) Rt[c] += cb[32 * (15 + c)];
-                }
                 if (a.mode == 1 || a.mode == 4) {
 #pragma unroll
                     for (int c = 0; c < 5; c++) a.R[c * a.rcs + rr] = Rt[c];
@@ -464,15 +318,7 @@ __global__ void __launch_bounds__(SWEEP_THREADS, CROCCO_SWEEP_MINB) k_sweep_s(co
                 }
             }
         }
-#if CROCCO_PRIMS_LATE
-        // chunk st+LA+1 (issued at the top of this step) landed -> its primitives, kept in
-        // registers so their latency chain overlaps the tail of this step's flux
-        cp_async_wait_all();
         __syncwarp();
-        if (st + 1 < nsteps) prim_calc(st + 1 + LA, pnext);
-#else
-        __syncwarp();
-#endif
     }
     cp_async_wait_all();
 }

@@ -24,11 +24,7 @@ struct WenoFrac {
     double base, num, den;  // W = base + num/(6 den)
 };
 
-#ifndef CROCCO_WENO_FOLD
-#define CROCCO_WENO_FOLD 1  // eps folded into the smoothness-indicator FMAs; C normalised to C0 = 1
-#endif
-
-// With CROCCO_WENO_FOLD the host passes C / C0 (the weights' ratios are all that
+// The host passes C / C0 (the weights' ratios are all that
 // enter W), so alpha_0 needs no multiply, and e_k = eps + b_k is formed inside the
 // FMA chain of b_k; max_k(eps + b_k) = eps + max_k b_k (monotone), so the
 // downwind-stencil rule is unchanged.
@@ -66,22 +62,13 @@ __device__ __forceinline__ WenoFrac weno_symbo_frac(double v0, double v1, double
         e2 = eps_b + b2;
         e3 = eps_b + b3;
     } else {
-#if CROCCO_WENO_FOLD
-    e0 = fma(s0, s0, fma(K3 * f0, f0, eps_b));
-    e1 = fma(s1, s1, fma(K3 * f1, f1, eps_b));
-    e2 = fma(s2, s2, fma(K3 * f2, f2, eps_b));
-    e3 = fma(s3, s3, fma(K3 * f3, f3, eps_b));
-    // downwind stencil never preferred (continuous max, parity-safe)
-    e3 = maxnn(maxnn(e0, e1), maxnn(e2, e3));
-#else
-    const double b0 = fma(K3 * f0, f0, s0 * s0);
-    const double b1 = fma(K3 * f1, f1, s1 * s1);
-    const double b2 = fma(K3 * f2, f2, s2 * s2);
-    double b3 = fma(K3 * f3, f3, s3 * s3);
-    // downwind stencil never preferred (continuous max, parity-safe)
-    b3 = maxnn(maxnn(b0, b1), maxnn(b2, b3));
-    e0 = eps_b + b0, e1 = eps_b + b1, e2 = eps_b + b2, e3 = eps_b + b3;
-#endif
+        // eps folded into the FMA chain of the smoothness indicators
+        e0 = fma(s0, s0, fma(K3 * f0, f0, eps_b));
+        e1 = fma(s1, s1, fma(K3 * f1, f1, eps_b));
+        e2 = fma(s2, s2, fma(K3 * f2, f2, eps_b));
+        e3 = fma(s3, s3, fma(K3 * f3, f3, eps_b));
+        // downwind stencil never preferred (continuous max, parity-safe)
+        e3 = maxnn(maxnn(e0, e1), maxnn(e2, e3));
     }
     e0 *= e0;
     e1 *= e1;
@@ -89,11 +76,7 @@ __device__ __forceinline__ WenoFrac weno_symbo_frac(double v0, double v1, double
     e3 *= e3;
     // alpha_0 = C0 e1 e2 e3, alpha_1 = C1 e0 e2 e3, alpha_2 = C2 e0 e1 e3, alpha_3 = C3 e0 e1 e2
     double e01 = e0 * e1, e23 = e2 * e3;
-#if CROCCO_WENO_FOLD
-    double x0 = e1;  // C0 = 1
-#else
-    double x0 = C0 * e1;
-#endif
+    double x0 = e1;  // C0 = 1 (the host normalises C)
     double x1 = C1 * e0, x2 = C2 * e3, x3 = C3 * e2;
     if constexpr (LIM) {
         if (lin) {  // linear optimal weights: alpha_k = C_k
