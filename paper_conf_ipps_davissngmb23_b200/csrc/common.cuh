@@ -42,17 +42,17 @@ __host__ __device__ inline int64_t vat(const VLay &V, int i, int j, int k) {
 }
 
 // Branch-free reciprocal / reciprocal square root: hardware approximation
-// (MUFU.RCP64H / MUFU.RSQ64H) + 2 Newton steps + (for x/y) one residual
-// correction -- within ~1 ulp for the positive, normal-range operands of this
-// path (densities, sound speeds, metric norms, WENO weight sums); used instead
-// of the IEEE div/sqrt sequences, whose slow-path branches cost issue slots.
+// (MUFU.RCP64H / MUFU.RSQ64H, relative error <= 2^-20, profiles/r01_approx.txt) + one
+// third-order correction (error ~ e^3 <= 2^-60, i.e. rounding level) + (for x/y) one
+// residual correction -- used instead of the IEEE div/sqrt sequences, whose slow-path
+// branches cost issue slots, and shorter than two Newton steps (3 / 5 dependent FP64
+// operations instead of 4 / 6) for the positive, normal-range operands of this path
+// (densities, sound speeds, metric norms, WENO weight sums).
 __device__ __forceinline__ double rcp_nr(double y) {
     double r;
     asm("rcp.approx.ftz.f64 %0, %1;" : "=d"(r) : "d"(y));
-    double e = fma(-y, r, 1.0);
-    r = fma(r, e, r);
-    e = fma(-y, r, 1.0);
-    return fma(r, e, r);
+    const double e = fma(-y, r, 1.0);   // y r = 1 - e
+    return fma(r, fma(e, e, e), r);     // r (1 + e + e^2) = (1 - e^3)/y
 }
 // x/y: one Newton step on the 2^-20 hardware reciprocal (2^-40) then the residual
 // correction q + r (x - y q), which is (near) correctly rounded -- measured exact on
@@ -67,9 +67,8 @@ __device__ __forceinline__ double div_nr(double x, double y) {
 __device__ __forceinline__ double rsqrt_nr(double x) {
     double r;
     asm("rsqrt.approx.ftz.f64 %0, %1;" : "=d"(r) : "d"(x));
-    const double h = 0.5 * x;
-    r = r * fma(-h * r, r, 1.5);
-    return r * fma(-h * r, r, 1.5);
+    const double e = fma(-x * r, r, 1.0);           // x r^2 = 1 - e
+    return fma(r * e, fma(0.375, e, 0.5), r);       // r (1 + e/2 + 3 e^2/8) = x^-1/2 (1 + O(e^3))
 }
 __device__ __forceinline__ double sqrt_nr(double x) {  // x > 0
     const double r = rsqrt_nr(x);
@@ -89,6 +88,7 @@ __device__ __forceinline__ double minnn(double a, double b) {
 }
 
 // primitive buffer components (k_prims)
-enum { PU = 0, PV = 1, PW = 2, PP = 3, PC = 4, PSR = 5, PH = 6, PT = 7, NPRIM = 8 };
+// (PIS = 1/sqrt(rho): the Roe weights use sqrt(rho) = rho / sqrt(rho), 1/rho~ = PIS_L PIS_R)
+enum { PU = 0, PV = 1, PW = 2, PP = 3, PC = 4, PIS = 5, PH = 6 };
 
 }  // namespace crocco

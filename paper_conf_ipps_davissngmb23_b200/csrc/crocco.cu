@@ -333,17 +333,17 @@ static void build_plan(const crocco_grid_desc *d, const int nb[3], const int bn[
 
 constexpr int SEG_MIN = 32;        // shortest march segment of a sweep line (small blocks split lines)
 constexpr int SEG_WARPS = 16384;   // lines are split until at least this many warps march
-template <int D>
+template <int D, bool V>
 static constexpr size_t sweep_smem_bytes() {
-    return (size_t)(SWEEP_THREADS / 32) * RingGeom<D>::PER_WARP * sizeof(double);
+    return (size_t)(sweep_threads(D) / 32) * RingGeom<D, V>::PER_WARP * sizeof(double);
 }
 template <int D, bool V>
 static cudaError_t sweep_attr1() {
     cudaError_t e = cudaFuncSetAttribute(k_sweep_s<D, V, false>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                         (int)sweep_smem_bytes<D>());
+                                         (int)sweep_smem_bytes<D, V>());
     if (e == cudaSuccess)
         e = cudaFuncSetAttribute(k_sweep_s<D, V, true>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                 (int)sweep_smem_bytes<D>());
+                                 (int)sweep_smem_bytes<D, V>());
     return e;
 }
 static cudaError_t sweep_attrs() {
@@ -1080,13 +1080,13 @@ static crocco_status rhs_block(crocco_ctx c, const LocalBlock &b, const double *
         while (lines * ((nd + seg - 1) / seg) < SEG_WARPS && seg > segmin) seg = (seg + 1) / 2;
         a.seg = (int)seg;
         const int64_t warps = lines * ((nd + seg - 1) / seg);
-        const unsigned grid = cdiv(warps * 32, SWEEP_THREADS);
+        const unsigned grid = cdiv(warps * 32, sweep_threads(d));
 #define SWEEP_LAUNCH(DD, VV)                                                                              \
     do {                                                                                                  \
         if (ph.lim)                                                                                       \
-            k_sweep_s<DD, VV, true><<<grid, SWEEP_THREADS, sweep_smem_bytes<DD>(), c->stream>>>(a, b.L, ph);  \
+            k_sweep_s<DD, VV, true><<<grid, sweep_threads(DD), sweep_smem_bytes<DD, VV>(), c->stream>>>(a, b.L, ph);  \
         else                                                                                              \
-            k_sweep_s<DD, VV, false><<<grid, SWEEP_THREADS, sweep_smem_bytes<DD>(), c->stream>>>(a, b.L, ph); \
+            k_sweep_s<DD, VV, false><<<grid, sweep_threads(DD), sweep_smem_bytes<DD, VV>(), c->stream>>>(a, b.L, ph); \
     } while (0)
         if (d == 0) LAUNCH(c, K_FLUX_X, SWEEP_LAUNCH(0, false));
         else if (d == 1) LAUNCH(c, K_FLUX_Y, if (a.visc) SWEEP_LAUNCH(1, true); else SWEEP_LAUNCH(1, false));

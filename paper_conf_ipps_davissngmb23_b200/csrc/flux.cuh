@@ -37,12 +37,30 @@ struct FluxIn {
 // the metric row m^d M(l, a) and the point viscous flux of direction d FV(l, q)
 // (q = momentum x, y, z, energy) at stencil point l = 0..5 (points i-2..i+3).
 // shared-memory ring of a warp: value v of ring point q in column col at
-// sv[v * VS + (q & (NR-1)) * PS + col]
-enum { SV_U = 0, SV_M = 5, SV_FV = 8, SV_P = 12, SV_N = 19 };
-template <int NR, int PS>
+// sv[v * VS + (q & (NR-1)) * PS + col]; values: U (5), metric row (3), [F^_v (4) when the
+// sweep carries a viscous term], primitives (7)
+enum { SV_U = 0, SV_M = 5, SV_FV = 8 };
+__host__ __device__ constexpr int sv_p(bool visc) { return visc ? 12 : 8; }   // first primitive
+__host__ __device__ constexpr int sv_n(bool visc) { return sv_p(visc) + 7; }  // values per point
+#ifndef CROCCO_FLUX_SCR
+#define CROCCO_FLUX_SCR 0  // bit 0: deferred WENO fractions in shared scratch; bit 1: theta_l, p_l there
+#endif
+constexpr int FLUX_SCR = CROCCO_FLUX_SCR;
+constexpr int flux_scr_values() { return (FLUX_SCR & 5 ? 15 : 0) + (FLUX_SCR & 2 ? 12 : 0); }
+// shared-memory load the compiler may not hoist or merge (keeps a value out of the registers
+// between its uses)
+__device__ __forceinline__ double lds_keep(const double *p) {
+    double v;
+    asm volatile("ld.shared.f64 %0, [%1];" : "=d"(v) : "r"((unsigned)__cvta_generic_to_shared(p)));
+    return v;
+}
+
+template <int NR, int PS, bool VISC>
 struct SAcc {
+    static constexpr int SV_P = sv_p(VISC);
     const double *sv;
     int q0, col;
+    double *scr;  // this lane's scratch (stride 32), FLUX_SCR
     static constexpr int VS = NR * PS;
     __device__ __forceinline__ double at_(int v, int l) const {
         return sv[v * VS + ((q0 + l) & (NR - 1)) * PS + col];
@@ -51,7 +69,7 @@ struct SAcc {
     __device__ __forceinline__ double P(int l, int k) const { return at_(SV_P + k, l); }
     __device__ __forceinline__ double M(int l, int a) const { return at_(SV_M + a, l); }
     __device__ __forceinline__ double FV(int l, int q) const { return at_(SV_FV + q, l); }
-    __device__ __forceinline__ double SR(int l) const { return P(l, PSR); }  // sqrt(rho)
+    __device__ __forceinline__ double IS(int l) const { return P(l, PIS); }  // 1/sqrt(rho)
     __device__ __forceinline__ double H(int l) const { return P(l, PH); }    // total enthalpy
 };
 
@@ -74,7 +92,8 @@ __device__ __forceinline__ void total_flux(const Acc &A, bool inv, bool visc, co
         const double nx = mh[0] * imag, ny = mh[1] * imag, nz = mh[2] * imag;
 
         // Roe average of points i (l=2), i+1 (l=3), sqrt(rho) weights
-        const double srL = A.SR(2), srR = A.SR(3);
+        const double isL = A.IS(2), isR = A.IS(3);
+        const double srL = A.U(2, 0) * isL, srR = A.U(3, 0) * isR;
         const double iden = rcp_nr(srL + srR);
         const double wL = srL * iden, wR = srR * iden;
         const double ut = fma(wL, A.P(2, PU), wR * A.P(3, PU));
@@ -87,7 +106,7 @@ __device__ __forceinline__ void total_flux(const Acc &A, bool inv, bool visc, co
         const double ict = rsqrt_nr(c2);
         const double ct = c2 * ict;
         const double ic2 = ict * ict;
-        const double irt = rcp_nr(rt);
+        const double irt = isL * isR;  // 1/rho~
         const double tht = fma(nx, ut, fma(ny, vt, nz * wt));
         const double phi2 = 0.5 * gm1 * q2;
         constexpr double SQ12 = 0.70710678118654752440;
@@ -107,6 +126,10 @@ __device__ __forceinline__ void total_flux(const Acc &A, bool inv, bool visc, co
             const double cl = A.P(l, PC);
             th[l] = t;
             pl[l] = A.P(l, PP);
+            if constexpr ((FLUX_SCR & 2) != 0) {
+                A.scr[32 * (15 + l)] = t;
+                A.scr[32 * (21 + l)] = pl[l];
+            }
             if constexpr (lam_tree) {
                 a0[l] = fabs(t);
                 a3[l] = fabs(t + cl);
@@ -191,19 +214,41 @@ __device__ __forceinline__ void total_flux(const Acc &A, bool inv, bool visc, co
             for (int l = 0; l < 6; l++) {
                 const double w =
                     fma(L0, UL(l, 0), fma(L1, UL(l, 1), fma(L2, UL(l, 2), fma(L3, UL(l, 3), L4 * UL(l, 4)))));
-                const double g = fma(th[l], w, pl[l] * fma(kB, th[l], kA));
+                double thl = th[l], pll = pl[l];
+                if constexpr ((FLUX_SCR & 2) != 0) {
+                    thl = lds_keep(A.scr + 32 * (15 + l));
+                    pll = lds_keep(A.scr + 32 * (21 + l));
+                }
+                const double g = fma(thl, w, pll * fma(kB, thl, kA));
                 gp[l] = fma(lam, w, g);
                 gm[l] = fma(-lam, w, g);
             }
             const WenoFrac wf = weno_pair_frac<LIM>(gp, gm, eps_b, ph.wC, &ph);
-            gb[sf] = wf.base;
-            gn[sf] = wf.num;
-            gd[sf] = wf.den;
+            if constexpr ((FLUX_SCR & 5) != 0) {
+                A.scr[32 * sf] = wf.base;
+                A.scr[32 * (5 + sf)] = wf.num;
+                A.scr[32 * (10 + sf)] = wf.den;
+            } else {
+                gb[sf] = wf.base;
+                gn[sf] = wf.num;
+                gd[sf] = wf.den;
+            }
             (void)R0; (void)R1; (void)R2; (void)R3; (void)R4;
         }
+        if constexpr ((FLUX_SCR & 4) != 0) __syncwarp();  // the fractions come back from shared memory
 #pragma unroll
         for (int sf = 0; sf < 5; sf++) {
-            const double gh = gb[sf] + div_nr(gn[sf], gd[sf]);
+            double ghb = gb[sf], ghn = gn[sf], ghd = gd[sf];
+            if constexpr ((FLUX_SCR & 4) != 0) {
+                ghb = A.scr[32 * sf];
+                ghn = A.scr[32 * (5 + sf)];
+                ghd = A.scr[32 * (10 + sf)];
+            } else if constexpr ((FLUX_SCR & 1) != 0) {
+                ghb = lds_keep(A.scr + 32 * sf);
+                ghn = lds_keep(A.scr + 32 * (5 + sf));
+                ghd = lds_keep(A.scr + 32 * (10 + sf));
+            }
+            const double gh = ghb + div_nr(ghn, ghd);
             double R0, R1, R2, R3, R4;
             if (sf < 3) {
                 const double na = sf == 0 ? nx : (sf == 1 ? ny : nz);

@@ -24,8 +24,35 @@ namespace crocco {
 
 // bit D: sweep D passes neighbour / carried interface fluxes through shared memory instead of a
 // register carry (measured: eta -4 %, xi +16 %, zeta 0)
-constexpr int CARRY_SMEM = 2;
-constexpr int SWEEP_THREADS = 128;  // 4 warps, 2 CTAs per SM (register file: 8 warps x 255 registers)
+#ifndef CROCCO_CARRY_SMEM
+#define CROCCO_CARRY_SMEM 2
+#endif
+#ifndef CROCCO_SWEEP_WARPS
+#define CROCCO_SWEEP_WARPS 4
+#endif
+#ifndef CROCCO_SWEEP_MINB
+#define CROCCO_SWEEP_MINB 1
+#endif
+#ifndef CROCCO_SWEEP_WARPS_X
+#define CROCCO_SWEEP_WARPS_X CROCCO_SWEEP_WARPS
+#endif
+#ifndef CROCCO_SWEEP_MINB_X
+#define CROCCO_SWEEP_MINB_X CROCCO_SWEEP_MINB
+#endif
+#ifndef CROCCO_SWEEP_WARPS_Z
+#define CROCCO_SWEEP_WARPS_Z CROCCO_SWEEP_WARPS
+#endif
+#ifndef CROCCO_SWEEP_MINB_Z
+#define CROCCO_SWEEP_MINB_Z CROCCO_SWEEP_MINB
+#endif
+constexpr int CARRY_SMEM = CROCCO_CARRY_SMEM;
+// threads per CTA and min CTAs per SM of sweep D
+__host__ __device__ constexpr int sweep_threads(int D) {
+    return 32 * (D == 0 ? CROCCO_SWEEP_WARPS_X : (D == 2 ? CROCCO_SWEEP_WARPS_Z : CROCCO_SWEEP_WARPS));
+}
+__host__ __device__ constexpr int sweep_minb(int D) {
+    return D == 0 ? CROCCO_SWEEP_MINB_X : (D == 2 ? CROCCO_SWEEP_MINB_Z : CROCCO_SWEEP_MINB);
+}
 
 struct SweepArgs {
     FluxIn in;
@@ -61,28 +88,33 @@ __device__ __forceinline__ void cp_async16(double *dst, const double *src) {
 __device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commit_group;\n" ::: "memory"); }
 __device__ __forceinline__ void cp_async_wait_all() { asm volatile("cp.async.wait_group 0;\n" ::: "memory"); }
 
-template <int D>
+template <int D, bool VISC>
 struct RingGeom {
     static constexpr int WS = (D == 0) ? 8 : 4;    // interfaces per step
     static constexpr int C = 32 / WS;              // columns (lines) per warp
     static constexpr int LA = (D == 0) ? 1 : 2;    // chunks ahead needed by a step
     static constexpr int NR = (D == 0) ? 32 : 16;  // ring points (>= (LA + 2) * WS, power of 2)
-    static constexpr int NCB = 16;                 // prefetched accumulate/update operands per lane
+    static constexpr int SVN = sv_n(VISC);         // staged values per ring point
+    // prefetched accumulate / update operands per lane: xi (mode 0 / 4) and eta (mode 1) read R;
+    // zeta finishes the point (mode 2: R, J; mode 3: R, J, dU, U_in)
+    static constexpr int NCB = D == 2 ? 16 : 5;
     static constexpr bool CARRY = (CARRY_SMEM >> D) & 1;
     static constexpr int NFC = CARRY ? 2 * 5 * 32 : 0;  // interface fluxes of two steps
-    static constexpr int PER_WARP = SV_N * NR * C + NCB * 32 + NFC;  // doubles
+    static constexpr int NSC = flux_scr_values() * 32;  // per-lane flux scratch (FLUX_SCR)
+    static constexpr int PER_WARP = SVN * NR * C + NCB * 32 + NFC + NSC;  // doubles
 };
 
 template <int D, bool VISC, bool LIM>
-__global__ void __launch_bounds__(SWEEP_THREADS, 1) k_sweep_s(const __grid_constant__ SweepArgs a,
+__global__ void __launch_bounds__(sweep_threads(D), sweep_minb(D)) k_sweep_s(const __grid_constant__ SweepArgs a,
                                                                           const Lay L, const Phys ph) {
-    using RG = RingGeom<D>;
+    using RG = RingGeom<D, VISC>;
     constexpr int WS = RG::WS, C = RG::C, LA = RG::LA, NR = RG::NR;
     constexpr int VS = NR * C;
+    constexpr int SV_P = sv_p(VISC);
     extern __shared__ double smem_dyn[];
     const int lane = threadIdx.x & 31;
     double *sv = smem_dyn + (threadIdx.x >> 5) * RG::PER_WARP;
-    double *cb = sv + SV_N * VS + lane;  // this lane's prefetched operands
+    double *cb = sv + RG::SVN * VS + lane;  // this lane's prefetched operands
     const int ls = (D == 0) ? (lane & 7) : (lane >> 3);  // sweep offset of this lane
     const int lt = (D == 0) ? (lane >> 3) : (lane & 7);  // column of this lane
     const int64_t gw = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
@@ -187,7 +219,7 @@ __global__ void __launch_bounds__(SWEEP_THREADS, 1) k_sweep_s(const __grid_const
         pv[PW] = w;
         pv[PP] = pr;
         pv[PC] = sqrt_nr(ph.gamma * pr * ir);
-        pv[PSR] = sqrt_nr(rho);
+        pv[PIS] = rsqrt_nr(rho);
         pv[PH] = (E + pr) * ir;
     };
     auto prim_store = [&](int ch, const double pv[7]) {
@@ -238,7 +270,7 @@ __global__ void __launch_bounds__(SWEEP_THREADS, 1) k_sweep_s(const __grid_const
 #pragma unroll
             for (int c = 0; c < 5; c++)
                 if (c > 0 || a.mode != 4) cp_async8(cb + 32 * c, a.R + c * a.rcs + rr);
-            if (a.mode >= 2) {
+            if (a.mode == 2 || a.mode == 3) {  // J (the zeta sweep finishes the point)
                 cp_async8(cb + 32 * 5, a.in.M + pp);
                 if (a.mode == 3) {
 #pragma unroll
@@ -252,8 +284,9 @@ __global__ void __launch_bounds__(SWEEP_THREADS, 1) k_sweep_s(const __grid_const
         cp_async_commit();
         issue(st + LA + 1);                   // group B: chunk st+LA+1 (slot of chunk st-1)
         if (act) {
-            const SAcc<NR, C> A{sv, WS * st + ls, lt};  // ring point of stencil point i-2
-            total_flux<D, SAcc<NR, C>, LIM>(A, inv, VISC, ph, F);
+            const SAcc<NR, C, VISC> A{sv, WS * st + ls, lt,  // ring point of stencil point i-2
+                                      sv + RG::SVN * VS + RG::NCB * 32 + RG::NFC + lane};
+            total_flux<D, SAcc<NR, C, VISC>, LIM>(A, inv, VISC, ph, F);
         } else {
 #pragma unroll
             for (int c = 0; c < 5; c++) F[c] = 0.0;
@@ -262,7 +295,7 @@ __global__ void __launch_bounds__(SWEEP_THREADS, 1) k_sweep_s(const __grid_const
         if constexpr (RG::CARRY) {
             // fluxes of step st in slot (st & 1); the left neighbour interface is lane-1 (xi) /
             // lane-8 (eta, zeta) of this step, or the last interface of the line in the last step
-            double *fs = sv + SV_N * VS + RG::NCB * 32;
+            double *fs = sv + RG::SVN * VS + RG::NCB * 32;
             double *cur = fs + (st & 1) * 160, *prv = fs + ((st & 1) ^ 1) * 160;
 #pragma unroll
             for (int c = 0; c < 5; c++) cur[32 * c + lane] = F[c];
