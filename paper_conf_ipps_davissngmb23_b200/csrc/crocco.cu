@@ -357,6 +357,14 @@ static cudaError_t sweep_attrs() {
     return e;
 }
 
+// one launch of the viscous kernel over `nt` tiles (sel / vk as k_visc_tiled)
+static crocco_status launch_visc(crocco_ctx c, const LocalBlock &b, const double *U, const double *M,
+                                 const Phys &ph, int64_t nt, int sel, int vk) {
+    LAUNCH(c, K_VISC, k_visc_tiled<<<(unsigned)nt, VTX * VTY, VISC_SMEM, c->stream>>>(
+                          U, M, b.fv, b.L, b.V, ph, b.racc, b.rcs, sel, vk));
+    return CROCCO_OK;
+}
+
 // ---------------------------------------------------------------------------
 // ABI
 // ---------------------------------------------------------------------------
@@ -1014,10 +1022,10 @@ static crocco_status visc_interior(crocco_ctx c, const LocalBlock &b, const doub
     const VTiles t = visc_interior_tiles(b.L, vk);
     const int64_t nt = (int64_t)(t.x1 - t.x0) * (t.y1 - t.y0) * (t.z1 - t.z0);
     if (nt == 0) return CROCCO_OK;
-    LAUNCH(c, K_VISC, k_visc_tiled<<<(unsigned)nt, VTX * VTY, VISC_SMEM, c->stream>>>(U, M, b.fv, b.L, b.V,
-                                                                                     c->ph, b.racc, b.rcs, 1, vk));
-    return CROCCO_OK;
+    return launch_visc(c, b, U, M, c->ph, nt, 1, vk);
 }
+
+
 
 static crocco_status rhs_block(crocco_ctx c, const LocalBlock &b, const double *U, const double *M,
                                int final_mode, double *rhs, const double *Uin, double *Uout,
@@ -1041,9 +1049,10 @@ static crocco_status rhs_block(crocco_ctx c, const LocalBlock &b, const double *
             const VTiles t = visc_interior_tiles(b.L, vk);
             nt -= (int64_t)(t.x1 - t.x0) * (t.y1 - t.y0) * (t.z1 - t.z0);
         }
-        if (nt > 0)
-            LAUNCH(c, K_VISC, k_visc_tiled<<<(unsigned)nt, VTX * VTY, VISC_SMEM, c->stream>>>(
-                                  U, M, b.fv, b.L, b.V, ph, b.racc, b.rcs, visc_sel, vk));
+        if (nt > 0) {
+            crocco_status st = launch_visc(c, b, U, M, ph, nt, visc_sel, vk);
+            if (st) return st;
+        }
     }
     for (int d = 0; d < 3; d++) {
         SweepArgs a;

@@ -42,25 +42,11 @@ struct FluxIn {
 enum { SV_U = 0, SV_M = 5, SV_FV = 8 };
 __host__ __device__ constexpr int sv_p(bool visc) { return visc ? 12 : 8; }   // first primitive
 __host__ __device__ constexpr int sv_n(bool visc) { return sv_p(visc) + 7; }  // values per point
-#ifndef CROCCO_FLUX_SCR
-#define CROCCO_FLUX_SCR 0  // bit 0: deferred WENO fractions in shared scratch; bit 1: theta_l, p_l there
-#endif
-constexpr int FLUX_SCR = CROCCO_FLUX_SCR;
-constexpr int flux_scr_values() { return (FLUX_SCR & 5 ? 15 : 0) + (FLUX_SCR & 2 ? 12 : 0); }
-// shared-memory load the compiler may not hoist or merge (keeps a value out of the registers
-// between its uses)
-__device__ __forceinline__ double lds_keep(const double *p) {
-    double v;
-    asm volatile("ld.shared.f64 %0, [%1];" : "=d"(v) : "r"((unsigned)__cvta_generic_to_shared(p)));
-    return v;
-}
-
 template <int NR, int PS, bool VISC>
 struct SAcc {
     static constexpr int SV_P = sv_p(VISC);
     const double *sv;
     int q0, col;
-    double *scr;  // this lane's scratch (stride 32), FLUX_SCR
     static constexpr int VS = NR * PS;
     __device__ __forceinline__ double at_(int v, int l) const {
         return sv[v * VS + ((q0 + l) & (NR - 1)) * PS + col];
@@ -73,45 +59,73 @@ struct SAcc {
     __device__ __forceinline__ double H(int l) const { return P(l, PH); }    // total enthalpy
 };
 
-// Total interface flux F = F^_inv - h_v of direction D at interface i+1/2.
+// Interface quantities that need no primitive of the outermost stencil points: frozen
+// metric, normal and |m^|/2 (R6 of the staged metric rows) and the Roe state of points i,
+// i+1 with the eigenvector scalars.  k_sweep_s evaluates them before it stores the newest
+// chunk's primitives (independent chains for the scheduler), then calls flux_fields.
+struct FluxSetup {
+    double nx, ny, nz, hmag;           // unit normal, |m^|/2 (LLF 1/2 folded here)
+    double ut, vt, wt, rt, irt;        // Roe velocity, density and its reciprocal
+    double ct, c2, ic2, tht, phi2;     // Roe sound speed, c^2, 1/c^2, n.u~, (gamma-1)|u~|^2/2
+    double alph, beta;                 // rho/(sqrt2 c), 1/(sqrt2 rho c)
+};
+template <class Acc>
+__device__ __forceinline__ void flux_setup(const Acc &A, const Phys &ph, FluxSetup &su) {
+    const double gm1 = ph.gm1;
+    double mh[3];
+#pragma unroll
+    for (int a = 0; a < 3; a++)
+        mh[a] = fma(37.0, A.M(2, a) + A.M(3, a), fma(-8.0, A.M(1, a) + A.M(4, a), A.M(0, a) + A.M(5, a))) *
+                (1.0 / 60.0);
+    const double s2 = fma(mh[0], mh[0], fma(mh[1], mh[1], mh[2] * mh[2]));
+    const double imag = rsqrt_nr(s2);
+    su.hmag = 0.5 * s2 * imag;
+    const double nx = mh[0] * imag, ny = mh[1] * imag, nz = mh[2] * imag;
+    su.nx = nx;
+    su.ny = ny;
+    su.nz = nz;
+
+    // Roe average of points i (l=2), i+1 (l=3), sqrt(rho) weights
+    const double isL = A.IS(2), isR = A.IS(3);
+    const double srL = A.U(2, 0) * isL, srR = A.U(3, 0) * isR;
+    const double iden = rcp_nr(srL + srR);
+    const double wL = srL * iden, wR = srR * iden;
+    const double ut = fma(wL, A.P(2, PU), wR * A.P(3, PU));
+    const double vt = fma(wL, A.P(2, PV), wR * A.P(3, PV));
+    const double wt = fma(wL, A.P(2, PW), wR * A.P(3, PW));
+    const double Ht = fma(wL, A.H(2), wR * A.H(3));
+    const double rt = srL * srR;
+    const double q2 = fma(ut, ut, fma(vt, vt, wt * wt));
+    const double c2 = gm1 * fma(-0.5, q2, Ht);
+    const double ict = rsqrt_nr(c2);
+    const double irt = isL * isR;  // 1/rho~
+    constexpr double SQ12 = 0.70710678118654752440;
+    su.ut = ut;
+    su.vt = vt;
+    su.wt = wt;
+    su.rt = rt;
+    su.irt = irt;
+    su.c2 = c2;
+    su.ct = c2 * ict;
+    su.ic2 = ict * ict;
+    su.tht = fma(nx, ut, fma(ny, vt, nz * wt));
+    su.phi2 = 0.5 * gm1 * q2;
+    su.alph = rt * ict * SQ12;
+    su.beta = irt * ict * SQ12;
+}
+
+// Total interface flux F = F^_inv - h_v of direction D at interface i+1/2 from the setup above.
 // A: stencil accessor (SAcc).
 template <int D, class Acc, bool LIM = false>
-__device__ __forceinline__ void total_flux(const Acc &A, bool inv, bool visc, const Phys &ph,
-                                           double F[5]) {
+__device__ __forceinline__ void flux_fields(const Acc &A, const FluxSetup &su, bool inv, bool visc,
+                                            const Phys &ph, double F[5]) {
     F[0] = F[1] = F[2] = F[3] = F[4] = 0.0;
     if (inv) {
         const double gm1 = ph.gm1;
-        double mh[3];
-#pragma unroll
-        for (int a = 0; a < 3; a++)
-            mh[a] = fma(37.0, A.M(2, a) + A.M(3, a), fma(-8.0, A.M(1, a) + A.M(4, a), A.M(0, a) + A.M(5, a))) *
-                    (1.0 / 60.0);
-        const double s2 = fma(mh[0], mh[0], fma(mh[1], mh[1], mh[2] * mh[2]));
-        const double imag = rsqrt_nr(s2);
-        const double hmag = 0.5 * s2 * imag;  // |m^|/2 (LLF 1/2 folded here)
-        const double nx = mh[0] * imag, ny = mh[1] * imag, nz = mh[2] * imag;
-
-        // Roe average of points i (l=2), i+1 (l=3), sqrt(rho) weights
-        const double isL = A.IS(2), isR = A.IS(3);
-        const double srL = A.U(2, 0) * isL, srR = A.U(3, 0) * isR;
-        const double iden = rcp_nr(srL + srR);
-        const double wL = srL * iden, wR = srR * iden;
-        const double ut = fma(wL, A.P(2, PU), wR * A.P(3, PU));
-        const double vt = fma(wL, A.P(2, PV), wR * A.P(3, PV));
-        const double wt = fma(wL, A.P(2, PW), wR * A.P(3, PW));
-        const double Ht = fma(wL, A.H(2), wR * A.H(3));
-        const double rt = srL * srR;
-        const double q2 = fma(ut, ut, fma(vt, vt, wt * wt));
-        const double c2 = gm1 * fma(-0.5, q2, Ht);
-        const double ict = rsqrt_nr(c2);
-        const double ct = c2 * ict;
-        const double ic2 = ict * ict;
-        const double irt = isL * isR;  // 1/rho~
-        const double tht = fma(nx, ut, fma(ny, vt, nz * wt));
-        const double phi2 = 0.5 * gm1 * q2;
-        constexpr double SQ12 = 0.70710678118654752440;
-        const double alph = rt * ict * SQ12;   // rho/(sqrt2 c)
-        const double beta = irt * ict * SQ12;  // 1/(sqrt2 rho c)
+        const double nx = su.nx, ny = su.ny, nz = su.nz, hmag = su.hmag;
+        const double ut = su.ut, vt = su.vt, wt = su.wt, rt = su.rt, irt = su.irt;
+        const double ct = su.ct, c2 = su.c2, ic2 = su.ic2, tht = su.tht, phi2 = su.phi2;
+        const double alph = su.alph, beta = su.beta;
 
         // stencil points (the states are re-read from the ring per field: holding the 6 x 5
         // states in registers measured slower)
@@ -126,10 +140,6 @@ __device__ __forceinline__ void total_flux(const Acc &A, bool inv, bool visc, co
             const double cl = A.P(l, PC);
             th[l] = t;
             pl[l] = A.P(l, PP);
-            if constexpr ((FLUX_SCR & 2) != 0) {
-                A.scr[32 * (15 + l)] = t;
-                A.scr[32 * (21 + l)] = pl[l];
-            }
             if constexpr (lam_tree) {
                 a0[l] = fabs(t);
                 a3[l] = fabs(t + cl);
@@ -214,41 +224,19 @@ __device__ __forceinline__ void total_flux(const Acc &A, bool inv, bool visc, co
             for (int l = 0; l < 6; l++) {
                 const double w =
                     fma(L0, UL(l, 0), fma(L1, UL(l, 1), fma(L2, UL(l, 2), fma(L3, UL(l, 3), L4 * UL(l, 4)))));
-                double thl = th[l], pll = pl[l];
-                if constexpr ((FLUX_SCR & 2) != 0) {
-                    thl = lds_keep(A.scr + 32 * (15 + l));
-                    pll = lds_keep(A.scr + 32 * (21 + l));
-                }
-                const double g = fma(thl, w, pll * fma(kB, thl, kA));
+                const double g = fma(th[l], w, pl[l] * fma(kB, th[l], kA));
                 gp[l] = fma(lam, w, g);
                 gm[l] = fma(-lam, w, g);
             }
             const WenoFrac wf = weno_pair_frac<LIM>(gp, gm, eps_b, ph.wC, &ph);
-            if constexpr ((FLUX_SCR & 5) != 0) {
-                A.scr[32 * sf] = wf.base;
-                A.scr[32 * (5 + sf)] = wf.num;
-                A.scr[32 * (10 + sf)] = wf.den;
-            } else {
-                gb[sf] = wf.base;
-                gn[sf] = wf.num;
-                gd[sf] = wf.den;
-            }
+            gb[sf] = wf.base;
+            gn[sf] = wf.num;
+            gd[sf] = wf.den;
             (void)R0; (void)R1; (void)R2; (void)R3; (void)R4;
         }
-        if constexpr ((FLUX_SCR & 4) != 0) __syncwarp();  // the fractions come back from shared memory
 #pragma unroll
         for (int sf = 0; sf < 5; sf++) {
-            double ghb = gb[sf], ghn = gn[sf], ghd = gd[sf];
-            if constexpr ((FLUX_SCR & 4) != 0) {
-                ghb = A.scr[32 * sf];
-                ghn = A.scr[32 * (5 + sf)];
-                ghd = A.scr[32 * (10 + sf)];
-            } else if constexpr ((FLUX_SCR & 1) != 0) {
-                ghb = lds_keep(A.scr + 32 * sf);
-                ghn = lds_keep(A.scr + 32 * (5 + sf));
-                ghd = lds_keep(A.scr + 32 * (10 + sf));
-            }
-            const double gh = ghb + div_nr(ghn, ghd);
+            const double gh = gb[sf] + div_nr(gn[sf], gd[sf]);
             double R0, R1, R2, R3, R4;
             if (sf < 3) {
                 const double na = sf == 0 ? nx : (sf == 1 ? ny : nz);

@@ -11,7 +11,7 @@
 //   A line is marched over segments of `seg` points; each segment recomputes
 //   the one interface it shares with the previous segment.
 // Every interface, in any decomposition and any lane, runs the same code
-// (total_flux), so an n-block run equals the 1-block run bit for bit.
+// (flux_setup + flux_fields), so an n-block run equals the 1-block run bit for bit.
 //
 // Accumulation of R = -sum_d (F_{i+1/2} - F_{i-1/2}) per point in fixed order
 // xi, eta, zeta (mode 0 writes, mode 1 adds); the zeta sweep finishes the point:
@@ -24,35 +24,12 @@ namespace crocco {
 
 // bit D: sweep D passes neighbour / carried interface fluxes through shared memory instead of a
 // register carry (measured: eta -4 %, xi +16 %, zeta 0)
-#ifndef CROCCO_CARRY_SMEM
-#define CROCCO_CARRY_SMEM 2
-#endif
-#ifndef CROCCO_SWEEP_WARPS
-#define CROCCO_SWEEP_WARPS 4
-#endif
-#ifndef CROCCO_SWEEP_MINB
-#define CROCCO_SWEEP_MINB 1
-#endif
-#ifndef CROCCO_SWEEP_WARPS_X
-#define CROCCO_SWEEP_WARPS_X CROCCO_SWEEP_WARPS
-#endif
-#ifndef CROCCO_SWEEP_MINB_X
-#define CROCCO_SWEEP_MINB_X CROCCO_SWEEP_MINB
-#endif
-#ifndef CROCCO_SWEEP_WARPS_Z
-#define CROCCO_SWEEP_WARPS_Z CROCCO_SWEEP_WARPS
-#endif
-#ifndef CROCCO_SWEEP_MINB_Z
-#define CROCCO_SWEEP_MINB_Z CROCCO_SWEEP_MINB
-#endif
-constexpr int CARRY_SMEM = CROCCO_CARRY_SMEM;
-// threads per CTA and min CTAs per SM of sweep D
-__host__ __device__ constexpr int sweep_threads(int D) {
-    return 32 * (D == 0 ? CROCCO_SWEEP_WARPS_X : (D == 2 ? CROCCO_SWEEP_WARPS_Z : CROCCO_SWEEP_WARPS));
-}
-__host__ __device__ constexpr int sweep_minb(int D) {
-    return D == 0 ? CROCCO_SWEEP_MINB_X : (D == 2 ? CROCCO_SWEEP_MINB_Z : CROCCO_SWEEP_MINB);
-}
+constexpr int CARRY_SMEM = 2;
+// threads per CTA and min CTAs per SM of sweep D: 4 warps, register-limited to 2 CTAs (8 warps)
+// per SM at 253 registers.  Measured (profiles/r02_variants_sweep.jsonl): capping the
+// registers for 10 or 12 warps per SM (2-warp CTAs) spills 150-280 B/thread and runs 25 % slower.
+__host__ __device__ constexpr int sweep_threads(int) { return 128; }
+__host__ __device__ constexpr int sweep_minb(int) { return 1; }
 
 struct SweepArgs {
     FluxIn in;
@@ -94,14 +71,14 @@ struct RingGeom {
     static constexpr int C = 32 / WS;              // columns (lines) per warp
     static constexpr int LA = (D == 0) ? 1 : 2;    // chunks ahead needed by a step
     static constexpr int NR = (D == 0) ? 32 : 16;  // ring points (>= (LA + 2) * WS, power of 2)
+    static_assert(NR >= (LA + 2) * WS && (NR & (NR - 1)) == 0, "ring too small");
     static constexpr int SVN = sv_n(VISC);         // staged values per ring point
     // prefetched accumulate / update operands per lane: xi (mode 0 / 4) and eta (mode 1) read R;
     // zeta finishes the point (mode 2: R, J; mode 3: R, J, dU, U_in)
     static constexpr int NCB = D == 2 ? 16 : 5;
     static constexpr bool CARRY = (CARRY_SMEM >> D) & 1;
     static constexpr int NFC = CARRY ? 2 * 5 * 32 : 0;  // interface fluxes of two steps
-    static constexpr int NSC = flux_scr_values() * 32;  // per-lane flux scratch (FLUX_SCR)
-    static constexpr int PER_WARP = SVN * NR * C + NCB * 32 + NFC + NSC;  // doubles
+    static constexpr int PER_WARP = SVN * NR * C + NCB * 32 + NFC;  // doubles
 };
 
 template <int D, bool VISC, bool LIM>
@@ -257,7 +234,8 @@ __global__ void __launch_bounds__(sweep_threads(D), sweep_minb(D)) k_sweep_s(con
     for (int c = 0; c < 5; c++) Fc[c] = 0.0;
     for (int st = 0; st < nsteps; st++, rr += rstep, pp += pstep) {
         if (st > 0) {
-            // chunk st+LA landed -> primitives
+            // chunk st+LA landed -> primitives (computing the interface setup beside them, as two
+            // independent chains, measured 3.5 % slower: register pressure)
             cp_async_wait_all();
             __syncwarp();
             prims(st + LA);
@@ -266,6 +244,7 @@ __global__ void __launch_bounds__(sweep_threads(D), sweep_minb(D)) k_sweep_s(con
         const int e = e0 - 1 + WS * st + ls;  // this lane's interface e+1/2
         const bool act = lvalid && e <= e1 - 1;
         const bool own = act && e >= e0;      // this lane finishes point e
+        const SAcc<NR, C, VISC> A{sv, WS * st + ls, lt};  // ring point of stencil point i-2
         if (own && a.mode != 0) {             // group A: accumulate / update operands
 #pragma unroll
             for (int c = 0; c < 5; c++)
@@ -284,9 +263,9 @@ __global__ void __launch_bounds__(sweep_threads(D), sweep_minb(D)) k_sweep_s(con
         cp_async_commit();
         issue(st + LA + 1);                   // group B: chunk st+LA+1 (slot of chunk st-1)
         if (act) {
-            const SAcc<NR, C, VISC> A{sv, WS * st + ls, lt,  // ring point of stencil point i-2
-                                      sv + RG::SVN * VS + RG::NCB * 32 + RG::NFC + lane};
-            total_flux<D, SAcc<NR, C, VISC>, LIM>(A, inv, VISC, ph, F);
+            FluxSetup su;
+            if (inv) flux_setup(A, ph, su);
+            flux_fields<D, SAcc<NR, C, VISC>, LIM>(A, su, inv, VISC, ph, F);
         } else {
 #pragma unroll
             for (int c = 0; c < 5; c++) F[c] = 0.0;
