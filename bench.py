@@ -170,6 +170,49 @@ def oracle_rate(max_seconds=12.0, n=64, max_steps=100, steps=None, warmup=0):
                       f"{el:.2f} s wall", "seconds": el, "steps": done, "per_step_s": per_step}
 
 
+def oracle_suite(max_total=60.0):
+    """BASELINE.md sec. 4's CPU baseline: the oracle (as it stands) on the paper-shaped configs at
+    1 host core and at all host cores -- Sod 200x4x4 for 100 RK3 steps (wall seconds), the
+    isentropic vortex on the 64^3 wavy grid (100 steps on all cores, a bounded number on one
+    core), and one RK3 step (3 stages) of a 128^3 TGV box; each as point-stages/s."""
+    import oracle
+    import synth
+    oracle.build()
+    cores = os.cpu_count() or 1
+    out = []
+    t_start = time.perf_counter()
+
+    def run(name, n, bc, grid, U0, ph, dt, steps, threads, note):
+        oracle.set_threads(threads)
+        xyz = grid.coords(n, (0, 0, 0), oracle.GC)
+        met = oracle.metrics(n, bc, xyz)
+        U = synth.pad_state(U0(xyz))
+        t0 = time.perf_counter()
+        oracle.advance(n, bc, ph, dt, steps, U, met)
+        el = time.perf_counter() - t0
+        pts = n[0] * n[1] * n[2] * 3 * steps
+        out.append({"config": name, "cores": oracle.get_threads(), "steps": steps, "seconds": round(el, 4),
+                    "value": pts / el, "unit": UNIT, "note": note})
+
+    sod = synth.case("sod")
+    vtx = synth.case("vortex")
+    tgv = synth.case("tgv", scale=2)  # 128^3
+    ph_inv = oracle.phys(gamma=1.4, R=1.0, terms=1)
+    ph_tgv = oracle.phys(**tgv.phys)
+    for threads in (1, cores):
+        run("sod 200x4x4 (configs[0])", sod.n_global, sod.bc, sod.grid, synth.sod, ph_inv, sod.dt, 100, threads,
+            "100 RK3 steps, wall seconds")
+        vsteps = 100 if threads == cores else 4
+        run("vortex 64^3 wavy (configs[1])", vtx.n_global, vtx.bc, vtx.grid, synth.vortex, ph_inv, vtx.dt, vsteps,
+            threads, "100 RK3 steps" if vsteps == 100 else f"bounded sample: {vsteps} RK3 steps on one core")
+        run("tgv 128^3 wavy, viscous (configs[2] at half resolution)", tgv.n_global, tgv.bc, tgv.grid,
+            synth.tgv, ph_tgv, tgv.dt, 1, threads, "3 RK stages (one RK3 step)")
+        if time.perf_counter() - t_start > max_total:
+            break
+    oracle.set_threads(cores)
+    return out
+
+
 # ------------------------------------------------------------------ reference arm
 def run_reference(args, rank, world):
     if rank != 0:
@@ -417,6 +460,8 @@ def run_crocco(args, rank, world, local_rank):
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
         r = oracle_rate()
         out["cpu_baseline"] = {k: r[k] for k in ("value", "unit", "cores", "kind", "sample")}
+        # 1 core and all cores on Sod / vortex / TGV (same run, same host)
+        out["cpu_baseline"]["suite"] = oracle_suite()
     S.close()
     if rank == 0:
         print(json.dumps(out), flush=True)
