@@ -113,6 +113,9 @@ def lib():
         L.oracle_fill_two_levels_ex.argtypes = [i64p, i32p, dp, C.POINTER(Split), C.c_double, dp, dp, i64p,
                                                 i64p, dp]
         L.oracle_average_down.argtypes = [i64p, i32p, dp, dp, i64p, i64p, dp]
+        dpp = C.POINTER(dp)
+        L.oracle_fill_two_levels_sib.argtypes = [i64p, i32p, dp, dp, dp, i64p, i64p, dp, C.c_int32, i64p, i64p, dpp]
+        L.oracle_average_down_sib.argtypes = [i64p, i32p, dp, dp, i64p, i64p, dp, C.c_int32, i64p, i64p, dpp]
         L.oracle_amr_advance.argtypes = [i64p, i32p, dp, i64p, i32p, dp, i64p, C.POINTER(Phys),
                                          C.c_double, C.c_int32, dp, dp, dp, dp]
         L.oracle_metrics2.argtypes = [i64p, dp, dp]
@@ -266,6 +269,35 @@ def average_down(nf, bcf, Uf, nc, c0, Uc, dirichlet=None):
     the coarse cell); refills the same-level ghosts of Uf first."""
     d = _dir(dirichlet)
     lib().oracle_average_down(_n(nf), _bc(bcf), _dp(d), _dp(Uf), _n(nc), _n(c0), _dp(Uc))
+    return Uc
+
+
+def _sibs(sibs):
+    """[(offset (3), n (3), padded state)] -> ctypes arrays (offset = fine index of the sibling's
+    node 0 in this patch's fine index space, 2 (c0_sibling - c0))."""
+    k = len(sibs)
+    so = (C.c_int64 * (3 * max(k, 1)))(*[int(x) for o, _, _ in sibs for x in o])
+    sn = (C.c_int64 * (3 * max(k, 1)))(*[int(x) for _, n, _ in sibs for x in n])
+    su = (C.POINTER(C.c_double) * max(k, 1))(*[_dp(U) for _, _, U in sibs])
+    return k, so, sn, su
+
+
+def fill_two_levels_sib(nf, bcf, Uf, nc, c0, Uc, sibs, dirichlet=None, met=None):
+    """FillPatchTwoLevels with same-level siblings (reading 31): C/F ghosts inside a sibling's
+    interior take the sibling's value, the others are interpolated from the coarse level."""
+    k, so, sn, su = _sibs(sibs)
+    mp = _dp(met) if met is not None else None
+    lib().oracle_fill_two_levels_sib(_n(nf), _bc(bcf), _dp(_dir(dirichlet)), mp, _dp(Uf), _n(nc), _n(c0),
+                                     _dp(Uc), k, so, sn, su)
+    return Uf
+
+
+def average_down_sib(nf, bcf, Uf, nc, c0, Uc, sibs, dirichlet=None):
+    """AverageDown with same-level siblings (reading 31): nodes whose central fine node this patch
+    owns and whose 27 fine nodes lie in the level's patch interiors."""
+    k, so, sn, su = _sibs(sibs)
+    lib().oracle_average_down_sib(_n(nf), _bc(bcf), _dp(_dir(dirichlet)), _dp(Uf), _n(nc), _n(c0), _dp(Uc),
+                                  k, so, sn, su)
     return Uc
 
 

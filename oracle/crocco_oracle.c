@@ -129,12 +129,19 @@ typedef struct {
    face inside the coarse domain are interpolated from the coarse level (FillPatchTwoLevels,
    PAPER.md:83, 129).  Without a coarse level (amr == NULL) they are left untouched. */
 enum { O_COARSE_FINE = 6 };
+#define O_MAX_SIB 8
 typedef struct {
     int64_t nc[3];    /* coarse-level interior size (one global box, ghost width 4) */
     int64_t c0[3];    /* coarse node index of fine node 0 (refinement ratio 2) */
     const double *Uc; /* coarse state, padded, ghosts filled */
+    /* same-level sibling patches (reading 31): sibling s has interior size sn[s], its node 0 at
+       fine index so[s] of this patch (so = 2 (c0_s - c0)), state sU[s] (padded); NULL sU: none */
+    int32_t nsib;
+    int64_t so[O_MAX_SIB][3], sn[O_MAX_SIB][3];
+    const double *sU[O_MAX_SIB];
 } oracle_amr;
 static void cf_interp(const oracle_amr *a, const int64_t f[3], double v[5]);
+static void cf_value(const oracle_amr *a, const int64_t f[3], double v[5]);
 
 static void fill_core(const int64_t n[3], const int32_t bc[6], const double dirichlet[30],
                       const oracle_split *split, double t, const double *met, double *f,
@@ -200,7 +207,7 @@ static void fill_core(const int64_t n[3], const int32_t bc[6], const double diri
                         }
                         double v[5];
                         if (k == O_COARSE_FINE) {
-                            cf_interp(amr, id, v);
+                            cf_value(amr, id, v);
                             for (int c = 0; c < 5; c++)
                                 f[c * b.cs + pd] = v[c];
                             continue;
@@ -1152,6 +1159,52 @@ static void cf_interp(const oracle_amr *a, const int64_t f[3], double v[5])
     }
 }
 
+/* sibling s of the patch whose interior holds fine point f (patch-local fine index), or -1 */
+static int sibling_of(const oracle_amr *a, const int64_t f[3])
+{
+    for (int s = 0; s < a->nsib; s++) {
+        int in = 1;
+        for (int d = 0; d < 3; d++) {
+            int64_t q = f[d] - a->so[s][d];
+            if (q < 0 || q >= a->sn[s][d])
+                in = 0;
+        }
+        if (in)
+            return s;
+    }
+    return -1;
+}
+
+/* value of a ghost point on a COARSE_FINE face (reading 31): a point inside another patch of
+   the same level takes that patch's value (FillPatchSingleLevel -> FillBoundary),
+   every other point is interpolated from the coarse level (FillPatchTwoLevels) */
+static void cf_value(const oracle_amr *a, const int64_t f[3], double v[5])
+{
+    int s = sibling_of(a, f);
+    if (s < 0) {
+        cf_interp(a, f, v);
+        return;
+    }
+    int64_t ns[3] = {a->sn[s][0], a->sn[s][1], a->sn[s][2]};
+    obox sb = make_box(ns, OG);
+    int64_t p = IX(&sb, f[0] - a->so[s][0], f[1] - a->so[s][1], f[2] - a->so[s][2]);
+    for (int c = 0; c < 5; c++)
+        v[c] = a->sU[s][c * sb.cs + p];
+}
+
+static void set_siblings(oracle_amr *a, int32_t nsib, const int64_t *so, const int64_t *sn,
+                         const double *const *sU)
+{
+    a->nsib = nsib < O_MAX_SIB ? nsib : O_MAX_SIB;
+    for (int s = 0; s < a->nsib; s++) {
+        for (int d = 0; d < 3; d++) {
+            a->so[s][d] = so[3 * s + d];
+            a->sn[s][d] = sn[3 * s + d];
+        }
+        a->sU[s] = sU[s];
+    }
+}
+
 /* FillPatch of a fine level (Alg. 2 l.3-4 at level 1): the three-phase fill of section 1
    with COARSE_FINE faces interpolated from the coarse state Uc (ghosts filled). */
 void oracle_fill_two_levels_ex(const int64_t nf[3], const int32_t bcf[6], const double dirichlet[30],
@@ -1164,7 +1217,24 @@ void oracle_fill_two_levels_ex(const int64_t nf[3], const int32_t bcf[6], const 
         a.c0[d] = c0[d];
     }
     a.Uc = Uc;
+    a.nsib = 0;
     fill_core(nf, bcf, dirichlet, split, t, metf, Uf, 5, O_FIELD_STATE, &a);
+}
+
+/* the same with same-level siblings (reading 31): so/sn: 3 x nsib offsets / sizes, sU their states */
+void oracle_fill_two_levels_sib(const int64_t nf[3], const int32_t bcf[6], const double dirichlet[30],
+                                const double *metf, double *Uf, const int64_t nc[3], const int64_t c0[3],
+                                const double *Uc, int32_t nsib, const int64_t *so, const int64_t *sn,
+                                const double *const *sU)
+{
+    oracle_amr a;
+    for (int d = 0; d < 3; d++) {
+        a.nc[d] = nc[d];
+        a.c0[d] = c0[d];
+    }
+    a.Uc = Uc;
+    set_siblings(&a, nsib, so, sn, sU);
+    fill_core(nf, bcf, dirichlet, NULL, 0.0, metf, Uf, 5, O_FIELD_STATE, &a);
 }
 
 void oracle_fill_two_levels(const int64_t nf[3], const int32_t bcf[6], const double dirichlet[30],
@@ -1209,6 +1279,79 @@ void oracle_average_down(const int64_t nf[3], const int32_t bcf[6], const double
                             for (int a = -1; a <= 1; a++) {
                                 double w = wt[a + 1] * wt[bb + 1] * wt[c + 1];
                                 int64_t pf = IX(&fb, fc[0] + a, fc[1] + bb, fc[2] + c);
+                                s = s + w * Uf[q * fb.cs + pf];
+                            }
+                    Uc[q * cb.cs + pc] = s;
+                }
+            }
+}
+
+/* AverageDown with same-level siblings (reading 31): the fine ghosts that lie inside a sibling
+   are first set to the sibling's values (with the periodic copies); a coarse node I is averaged
+   by the patch whose interior holds its central fine node 2(I - c0) when all 27 fine nodes of its
+   cell lie in the interiors of the level's patches (directions the patch spans periodically
+   always qualify) -- without siblings exactly oracle_average_down's covered set.  Same formula
+   and summation order. */
+void oracle_average_down_sib(const int64_t nf[3], const int32_t bcf[6], const double dirichlet[30],
+                             double *Uf, const int64_t nc[3], const int64_t c0[3], double *Uc,
+                             int32_t nsib, const int64_t *so, const int64_t *sn, const double *const *sU)
+{
+    static const double wt[3] = {0.25, 0.5, 0.25};
+    obox fb = make_box(nf, OG), cb = make_box(nc, OG);
+    oracle_amr a;
+    for (int d = 0; d < 3; d++) {
+        a.nc[d] = nc[d];
+        a.c0[d] = c0[d];
+    }
+    a.Uc = NULL;
+    set_siblings(&a, nsib, so, sn, sU);
+    fill_core(nf, bcf, dirichlet, NULL, 0.0, NULL, Uf, 5, O_FIELD_METRIC, NULL);
+    /* sibling copies into the ghost band */
+    for (int64_t k = -OG; k < nf[2] + OG; k++)
+        for (int64_t j = -OG; j < nf[1] + OG; j++)
+            for (int64_t i = -OG; i < nf[0] + OG; i++) {
+                int64_t f[3] = {i, j, k};
+                if (i >= 0 && i < nf[0] && j >= 0 && j < nf[1] && k >= 0 && k < nf[2])
+                    continue;
+                if (sibling_of(&a, f) < 0)
+                    continue;
+                double v[5];
+                cf_value(&a, f, v);
+                int64_t p = IX(&fb, i, j, k);
+                for (int c = 0; c < 5; c++)
+                    Uf[c * fb.cs + p] = v[c];
+            }
+    for (int64_t k = 0; k < nc[2]; k++)
+        for (int64_t j = 0; j < nc[1]; j++)
+            for (int64_t i = 0; i < nc[0]; i++) {
+                int64_t I[3] = {i, j, k}, fc[3];
+                int covered = 1;
+                for (int d = 0; d < 3; d++) {
+                    fc[d] = 2 * (I[d] - c0[d]);
+                    if (bcf[2 * d] != O_PERIODIC && (fc[d] < 0 || fc[d] > nf[d] - 1))
+                        covered = 0; /* central node not in this patch */
+                }
+                for (int c = -1; c <= 1 && covered; c++)
+                    for (int bb = -1; bb <= 1 && covered; bb++)
+                        for (int aa = -1; aa <= 1 && covered; aa++) {
+                            int64_t f[3] = {fc[0] + aa, fc[1] + bb, fc[2] + c};
+                            int inside = 1;
+                            for (int d = 0; d < 3; d++)
+                                if (bcf[2 * d] != O_PERIODIC && (f[d] < 0 || f[d] > nf[d] - 1))
+                                    inside = 0;
+                            if (!inside && sibling_of(&a, f) < 0)
+                                covered = 0;
+                        }
+                if (!covered)
+                    continue;
+                int64_t pc = IX(&cb, i, j, k);
+                for (int q = 0; q < 5; q++) {
+                    double s = 0.0;
+                    for (int c = -1; c <= 1; c++)
+                        for (int bb = -1; bb <= 1; bb++)
+                            for (int aa = -1; aa <= 1; aa++) {
+                                double w = wt[aa + 1] * wt[bb + 1] * wt[c + 1];
+                                int64_t pf = IX(&fb, fc[0] + aa, fc[1] + bb, fc[2] + c);
                                 s = s + w * Uf[q * fb.cs + pf];
                             }
                     Uc[q * cb.cs + pc] = s;

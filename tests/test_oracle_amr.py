@@ -238,3 +238,131 @@ def test_refined_dmr_split_faces_follow_the_physical_rule():
         slip = ~(x < 1.0 / 6.0)
         assert np.array_equal(row[0][:, slip], mirror[0][:, slip])                 # rho mirrored
         assert np.array_equal(row[2][:, slip], -mirror[2][:, slip])                # v reflected
+
+
+# ------------------------------------------------------------------ same-level siblings (reading 31)
+
+def advance_level(nc, metc, Uc, patches, ph, dt, nsteps):
+    """Algorithm 2 on a periodic coarse level + one fine level of patches,
+    composed from the oracle functions: per stage the coarse stage, every patch's FillPatch (C/F
+    ghosts inside a sibling patch copied from the sibling's stage input -- FillBoundary,
+    PAPER.md:129 -- the others interpolated), RHS, update; AverageDown of every patch at the third
+    stage.  patches: list of dicts c0, nf, metf, U (padded, updated in place).  Test helper; the
+    arithmetic is the oracle's."""
+    bcf = ((CF, CF),) * 3
+    ac, oc, dUc = Uc, Uc.copy(), np.zeros_like(Uc)
+    st = [dict(a=p["U"], o=p["U"].copy(), dU=np.zeros_like(p["U"])) for p in patches]
+
+    def sibs(i, key):
+        p = patches[i]
+        return [(tuple(2 * (q["c0"][d] - p["c0"][d]) for d in range(3)), q["nf"], st[j][key])
+                for j, q in enumerate(patches) if j != i]
+
+    for _ in range(nsteps):
+        for s in range(3):
+            oracle.rk_stage(nc, PER, ph, s, dt, ac, oc, dUc, metc)
+            for i, p in enumerate(patches):
+                oracle.fill_two_levels_sib(p["nf"], bcf, st[i]["a"], nc, p["c0"], ac, sibs(i, "a"))
+            for i, p in enumerate(patches):
+                r = oracle.rhs(p["nf"], ph, st[i]["a"], p["metf"])
+                oracle.rk_update(p["nf"], s, dt, st[i]["a"], st[i]["o"], st[i]["dU"], r)
+            if s == 2:
+                for i, p in enumerate(patches):
+                    oracle.average_down_sib(p["nf"], bcf, st[i]["o"], nc, p["c0"], oc, sibs(i, "o"))
+            for x in st:
+                x["a"], x["o"] = x["o"], x["a"]
+            ac, oc = oc, ac
+    for p, x in zip(patches, st):
+        p["U"][...] = x["a"]
+    Uc[...] = ac
+    return Uc
+
+
+def _level_setup(nc, grid, specs, state):
+    bcf = ((CF, CF),) * 3
+    xc = grid.coords(nc, (0, 0, 0), oracle.GC)
+    metc = oracle.metrics(nc, PER, xc)
+    Uc = synth.pad_state(state(xc))
+    P = []
+    for c0, nf in specs:
+        xf = synth.Refined(grid, c0).coords(nf, (0, 0, 0), oracle.GC)
+        P.append(dict(c0=c0, nf=nf, metf=oracle.metrics(nf, bcf, xf), U=synth.pad_state(state(xf))))
+    return metc, Uc, P
+
+
+@pytest.mark.parametrize("axis", [0, 1, 2])
+def test_abutting_patches_equal_their_union_bitwise(axis):
+    """Reading 31: two abutting fine patches (each other's siblings) advance exactly like the one
+    patch covering their union -- fine states on the union and the coarse state bit for bit, over
+    3 RK3 steps of a viscous vortex flow -- because a C/F ghost inside the sibling takes the
+    sibling's value (the union's interior value), every other C/F ghost is interpolated at the
+    same position, and AverageDown covers exactly the union's covered set."""
+    nc = (16, 16, 16)
+    grid = synth.Wavy3D(L=(10.0,) * 3, N=nc)
+    ph = oracle.phys(terms=3, mu_ref=0.01)
+    c0, nu = (3, 4, 2), [16, 16, 12]   # halves even: a patch starts at an even fine index
+    half = [nu[d] // 2 if d == axis else nu[d] for d in range(3)]
+    c0b = tuple(c0[d] + (half[d] // 2 if d == axis else 0) for d in range(3))
+    metc, Uu, Pu = _level_setup(nc, grid, [(c0, tuple(nu))], lambda x: synth.vortex(x))
+    metc2, Us, Ps = _level_setup(nc, grid, [(c0, tuple(half)), (c0b, tuple(half))], lambda x: synth.vortex(x))
+    assert np.array_equal(metc, metc2)
+    # the two halves' fine metrics are the union's (same coordinates)
+    sl = [slice(G, -G)] * 3
+    su = list(sl)
+    su[2 - axis] = slice(G, G + half[axis])
+    assert np.array_equal(Pu[0]["metf"][(slice(None),) + tuple(su)], Ps[0]["metf"][:, G:-G, G:-G, G:-G])
+    advance_level(nc, metc, Uu, Pu, ph, 0.01, 3)
+    advance_level(nc, metc, Us, Ps, ph, 0.01, 3)
+    assert np.array_equal(Uu, Us)
+    union = Pu[0]["U"][:, G:-G, G:-G, G:-G]
+    parts = [P["U"][:, G:-G, G:-G, G:-G] for P in Ps]
+    assert np.array_equal(np.concatenate(parts, axis=3 - axis), union)
+
+
+def test_sibling_ghosts_are_copies_and_covered_set():
+    """The C/F ghosts of patch A that lie in sibling B's interior equal B's values exactly (the
+    others keep the trilinear value), and AverageDown with the sibling covers the coarse nodes
+    whose 27 fine nodes lie in A or B, each written by the patch owning the central node."""
+    nc = (14, 12, 13)
+    c0a, nfa, c0b, nfb = (2, 2, 2), (10, 12, 8), (7, 3, 2), (8, 10, 8)   # B abuts A's hi-x face
+    bcf = ((CF, CF),) * 3
+    Uc = _coarse_field(nc, lambda q, X, Y, Z: (q + 1) * (1 + 0.1 * X - 0.2 * Y + 0.05 * Z * X))
+    rng = np.random.default_rng(31)
+    Ua = rng.uniform(1, 2, (5, nfa[2] + 2 * G, nfa[1] + 2 * G, nfa[0] + 2 * G))
+    Ub = rng.uniform(1, 2, (5, nfb[2] + 2 * G, nfb[1] + 2 * G, nfb[0] + 2 * G))
+    Ua0 = Ua.copy()
+    oracle.fill_two_levels_sib(nfa, bcf, Ua, nc, c0a, Uc, [((10, 2, 0), nfb, Ub)])
+    ref = oracle.fill_two_levels(nfa, bcf, Ua0.copy(), nc, c0a, Uc)
+    assert np.array_equal(Ua[:, G:-G, G:-G, G:-G], Ua0[:, G:-G, G:-G, G:-G])
+    n_copied = 0
+    for k in range(-G, nfa[2] + G):
+        for j in range(-G, nfa[1] + G):
+            for i in range(-G, nfa[0] + G):
+                if 0 <= i < nfa[0] and 0 <= j < nfa[1] and 0 <= k < nfa[2]:
+                    continue
+                ib, jb, kb = i - 10, j - 2, k
+                got = Ua[:, k + G, j + G, i + G]
+                if 0 <= ib < nfb[0] and 0 <= jb < nfb[1] and 0 <= kb < nfb[2]:
+                    assert np.array_equal(got, Ub[:, kb + G, jb + G, ib + G])
+                    n_copied += 1
+                else:
+                    assert np.array_equal(got, ref[:, k + G, j + G, i + G])
+    assert n_copied == G * nfb[1] * nfa[2] - G * 0  # the hi-x ghost slab over B's j-range
+    # AverageDown: mark coarse nodes
+    Ca = np.full_like(Uc, -7.0)
+    Cb = Ca.copy()
+    oracle.average_down_sib(nfa, bcf, Ua.copy(), nc, c0a, Ca, [((10, 2, 0), nfb, Ub)])
+    oracle.average_down_sib(nfb, bcf, Ub.copy(), nc, c0b, Cb, [((-10, -2, 0), nfa, Ua)])
+    for K in range(nc[2]):
+        for J in range(nc[1]):
+            for I in range(nc[0]):
+                fa = (2 * (I - c0a[0]), 2 * (J - c0a[1]), 2 * (K - c0a[2]))
+                fb = (2 * (I - c0b[0]), 2 * (J - c0b[1]), 2 * (K - c0b[2]))
+                ina = lambda f: all(0 <= f[d] < nfa[d] for d in range(3))
+                inb = lambda f: all(0 <= f[d] < nfb[d] for d in range(3))
+                allin = all(ina((fa[0] + a, fa[1] + b, fa[2] + c)) or inb((fb[0] + a, fb[1] + b, fb[2] + c))
+                            for a in (-1, 0, 1) for b in (-1, 0, 1) for c in (-1, 0, 1))
+                wa = Ca[0, K + G, J + G, I + G] != -7.0
+                wb = Cb[0, K + G, J + G, I + G] != -7.0
+                assert wa == (allin and ina(fa)) and wb == (allin and inb(fb)), (I, J, K)
+    assert (Ca[0] != -7.0).sum() + (Cb[0] != -7.0).sum() > 0
