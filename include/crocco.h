@@ -253,7 +253,8 @@ crocco_status crocco_compute_dt(crocco_ctx ctx, double *const *U, double *const 
    inside the stage loop), then the fine level with its C/F ghosts interpolated from the coarse
    stage INPUT, then at stage 2 (the third) AverageDown.  Both ctx must enqueue on the same
    stream (or the caller orders them).  No inter-level communication: every coarse block a fine
-   block reads (and every fine block a covered coarse node reads) must be local to the rank. */
+   block reads (and every fine block a covered coarse node reads) must be local to the rank.
+   Several patches of one level: see the sibling calls below. */
 
 /* Declare `fine` a refinement of `coarse` with fine node 0 at coarse node c0[3].  Checks:
    per direction either the fine level is PERIODIC and spans the periodic coarse domain
@@ -278,6 +279,29 @@ crocco_status crocco_amr_rk_stage(crocco_ctx fine, int32_t stage, double dt, dou
    (periodic / inter-block copies only), then every covered coarse node of U_coarse (interior
    points only) becomes the full-weighting (trapezoid) average of the fine data over its cell. */
 crocco_status crocco_average_down(crocco_ctx fine, double *const *U_fine, double *const *U_coarse);
+
+/* ---- same-level sibling patches (NEXT-4 completion; a level is a union of
+   patches, FillPatchSingleLevel -> FillBoundary exchanges their ghosts; reading 31) ---
+   Declare two fine patches of the same level (both crocco_amr_link'ed to the same coarse ctx,
+   interiors disjoint, even fine offset 2 (c0_g - c0_f), single-rank) siblings of each other;
+   symmetric, idempotent; <= 8 siblings / 16 sibling blocks per patch; CROCCO_ERR_ARG otherwise.
+   With siblings, the _level calls below replace the two-level calls; `sib` holds, for each
+   sibling in link order, the pointer array of its local blocks (caller-owned, device):
+   - C/F ghosts lying inside a sibling's interior take the sibling's value (the stage INPUT of
+     the sibling for crocco_amr_rk_stage_level), all others are interpolated as before;
+   - AverageDown averages the coarse nodes whose central fine node lies in this patch and whose
+     27 fine nodes lie in the interiors of this patch or its siblings (`sib` = the siblings'
+     updated states), so each covered node of the level is written by exactly one patch.
+   Two abutting patches then advance exactly like the one patch covering their union (oracle
+   pin tests/test_oracle_amr.py; GPU parity tests/test_gpu_amr.py). */
+crocco_status crocco_amr_link_sibling(crocco_ctx fine, crocco_ctx sibling);
+crocco_status crocco_fill_patch_level(crocco_ctx fine, double *const *U_fine, double *const *metrics_fine,
+                                      double *const *U_coarse, double *const *const *sib);
+crocco_status crocco_amr_rk_stage_level(crocco_ctx fine, int32_t stage, double dt, double *const *U_in,
+                                        double *const *U_out, double *const *dU, double *const *metrics,
+                                        double *const *U_coarse_in, double *const *const *sib_in);
+crocco_status crocco_average_down_level(crocco_ctx fine, double *const *U_fine, double *const *U_coarse,
+                                        double *const *const *sib);
 
 /* State check (SURVEY sec. 5 failure detection; test / bench utility): *n_bad = number of
    interior points of all local blocks with a non-finite component, rho <= 0 or p <= 0

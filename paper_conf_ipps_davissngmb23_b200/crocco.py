@@ -101,6 +101,10 @@ _SIGS = {
     "crocco_fill_patch_two_levels": [C.c_void_p, DPP, DPP, DPP],
     "crocco_amr_rk_stage": [C.c_void_p, C.c_int32, C.c_double, DPP, DPP, DPP, DPP, DPP],
     "crocco_average_down": [C.c_void_p, DPP, DPP],
+    "crocco_amr_link_sibling": [C.c_void_p, C.c_void_p],
+    "crocco_fill_patch_level": [C.c_void_p, DPP, DPP, DPP, C.POINTER(DPP)],
+    "crocco_amr_rk_stage_level": [C.c_void_p, C.c_int32, C.c_double, DPP, DPP, DPP, DPP, DPP, C.POINTER(DPP)],
+    "crocco_average_down_level": [C.c_void_p, DPP, DPP, C.POINTER(DPP)],
 }
 _STR = {"crocco_last_error": [C.c_void_p], "crocco_version": [],
         "crocco_kernel_class_name": [C.c_int32]}
@@ -364,6 +368,42 @@ def crocco_average_down(fine, Uf_ptrs, Uc_ptrs):
     a, ka = _ptrs(Uf_ptrs)
     b, kb = _ptrs(Uc_ptrs)
     _check(lib().crocco_average_down(fine, a, b), fine)
+
+
+def crocco_amr_link_sibling(fine, sibling):
+    _check(lib().crocco_amr_link_sibling(fine, sibling), fine)
+
+
+def _sib_table(sib_ptr_lists):
+    """[[block pointers of sibling 0], ...] -> (double **)[] plus the arrays keeping it alive."""
+    keep = [_ptrs(pl) for pl in sib_ptr_lists]
+    tab = (DPP * max(len(keep), 1))(*[k[0] for k in keep])
+    return tab, keep
+
+
+def crocco_fill_patch_level(fine, Uf_ptrs, metf_ptrs, Uc_ptrs, sib_ptr_lists):
+    a, ka = _ptrs(Uf_ptrs)
+    b, kb = _ptrs(metf_ptrs) if metf_ptrs is not None else (None, None)
+    c, kc = _ptrs(Uc_ptrs)
+    t, kt = _sib_table(sib_ptr_lists)
+    _check(lib().crocco_fill_patch_level(fine, a, b, c, t), fine)
+
+
+def crocco_amr_rk_stage_level(fine, stage, dt, Uin_ptrs, Uout_ptrs, dU_ptrs, met_ptrs, Uc_in_ptrs, sib_in_lists):
+    a, ka = _ptrs(Uin_ptrs)
+    b, kb = _ptrs(Uout_ptrs)
+    c, kc = _ptrs(dU_ptrs)
+    d, kd = _ptrs(met_ptrs)
+    e, ke = _ptrs(Uc_in_ptrs)
+    t, kt = _sib_table(sib_in_lists)
+    _check(lib().crocco_amr_rk_stage_level(fine, stage, dt, a, b, c, d, e, t), fine)
+
+
+def crocco_average_down_level(fine, Uf_ptrs, Uc_ptrs, sib_ptr_lists):
+    a, ka = _ptrs(Uf_ptrs)
+    b, kb = _ptrs(Uc_ptrs)
+    t, kt = _sib_table(sib_ptr_lists)
+    _check(lib().crocco_average_down_level(fine, a, b, t), fine)
 
 
 # ---- 27-component metrics / expanded viscous form (SURVEY NEXT-3; readings 27-28) ----

@@ -27,6 +27,24 @@ struct LevelTab {
 
 __device__ __forceinline__ int64_t floor_half(int64_t h) { return h >= 0 ? h / 2 : -((-h + 1) / 2); }
 
+// Blocks of the same-level sibling patches of a fine level (reading 31): box [lo, hi) of the
+// block's interior in this level's fine index space, its state array and layout.
+constexpr int SIB_MAX_BLOCKS = 16;
+struct SibTab {
+    int n;
+    int64_t lo[SIB_MAX_BLOCKS][3], hi[SIB_MAX_BLOCKS][3];
+    const double *p[SIB_MAX_BLOCKS];
+    Lay L[SIB_MAX_BLOCKS];
+};
+// sibling block holding fine point f (this level's fine index), or -1
+__device__ __forceinline__ int sib_find(const SibTab &sb, const int64_t f[3]) {
+    for (int s = 0; s < sb.n; s++)
+        if (f[0] >= sb.lo[s][0] && f[0] < sb.hi[s][0] && f[1] >= sb.lo[s][1] && f[1] < sb.hi[s][1] &&
+            f[2] >= sb.lo[s][2] && f[2] < sb.hi[s][2])
+            return s;
+    return -1;
+}
+
 // One ghost box of a fine block on a COARSE_FINE face.
 struct CFOp {
     double *dst;
@@ -38,6 +56,7 @@ constexpr int CF_MAX_OPS = 16;
 struct CFOps {
     CFOp op[CF_MAX_OPS];
     int nops;
+    int interp;     // 1: points outside the siblings interpolated; 0: sibling copies only
     Lay Lf;         // fine block layout
     int64_t c0[3];  // coarse index of fine node 0
 };
@@ -46,8 +65,11 @@ struct CFOps {
 // 8 coarse nodes around c0 + f/2 (weights 1, 1/2 or 0 per direction, corner order
 // e0 fastest).  The coarse state's ghosts must be filled (they supply corners
 // beyond block faces and outside the domain).
+// A point inside a same-level sibling takes the sibling's value instead (FillBoundary between
+// the level's patches, reading 31).
 __global__ void __launch_bounds__(256) k_cf_interp(const __grid_constant__ CFOps ops,
-                                                   const __grid_constant__ LevelTab ct) {
+                                                   const __grid_constant__ LevelTab ct,
+                                                   const __grid_constant__ SibTab sb) {
     const CFOp &o = ops.op[blockIdx.y];
     const int64_t tot = (int64_t)o.ext[0] * o.ext[1] * o.ext[2];
     const Lay &Lc = ct.L;
@@ -58,6 +80,19 @@ __global__ void __launch_bounds__(256) k_cf_interp(const __grid_constant__ CFOps
         const int b = (int)(r % o.ext[1]);
         const int c = (int)(r / o.ext[1]);
         const int loc[3] = {a, b, c};
+        const int64_t dp = o.dbase + a + b * ops.Lf.py + c * ops.Lf.pz;
+        if (sb.n > 0) {
+            const int64_t f[3] = {o.fo[0] + a, o.fo[1] + b, o.fo[2] + c};
+            const int s = sib_find(sb, f);
+            if (s >= 0) {
+                const Lay &Ls = sb.L[s];
+                const int64_t ps = at(Ls, (int)(f[0] - sb.lo[s][0]), (int)(f[1] - sb.lo[s][1]), (int)(f[2] - sb.lo[s][2]));
+#pragma unroll
+                for (int q = 0; q < 5; q++) o.dst[q * ops.Lf.cs + dp] = sb.p[s][q * Ls.cs + ps];
+                continue;
+            }
+        }
+        if (!ops.interp) continue;
         int64_t I[3];
         double tt[3];
         int bx[3];
@@ -84,7 +119,6 @@ __global__ void __launch_bounds__(256) k_cf_interp(const __grid_constant__ CFOps
 #pragma unroll
             for (int q = 0; q < 5; q++) v[q] = v[q] + w * src[q * Lc.cs + p];
         }
-        const int64_t dp = o.dbase + a + b * ops.Lf.py + c * ops.Lf.pz;
 #pragma unroll
         for (int q = 0; q < 5; q++) o.dst[q * ops.Lf.cs + dp] = v[q];
     }
@@ -105,10 +139,27 @@ struct ADOps {
     int nops;
     Lay Lc;
     int64_t c0[3];
+    int64_t Nf[3];   // fine level interior size
+    int per[3];      // fine level spans direction d periodically
 };
+// With siblings (reading 31) the boxes hold the nodes whose central fine node lies in this level;
+// a node is averaged when its 27 fine nodes lie in this level's interior or a sibling's.
+__device__ __forceinline__ bool ad_covered(const ADOps &ops, const SibTab &sb, const int64_t f[3]) {
+    if (sb.n == 0) return true;  // the host boxes are the covered set
+    for (int cz = -1; cz <= 1; cz++)
+        for (int cy = -1; cy <= 1; cy++)
+            for (int cx = -1; cx <= 1; cx++) {
+                const int64_t g[3] = {f[0] + cx, f[1] + cy, f[2] + cz};
+                bool in = true;
+                for (int d = 0; d < 3; d++) in = in && (ops.per[d] || (g[d] >= 0 && g[d] < ops.Nf[d]));
+                if (!in && sib_find(sb, g) < 0) return false;
+            }
+    return true;
+}
 
 __global__ void __launch_bounds__(256) k_average_down(const __grid_constant__ ADOps ops,
-                                                      const __grid_constant__ LevelTab ft) {
+                                                      const __grid_constant__ LevelTab ft,
+                                                      const __grid_constant__ SibTab sb) {
     const ADOp &o = ops.op[blockIdx.y];
     const int64_t tot = (int64_t)o.ext[0] * o.ext[1] * o.ext[2];
     const Lay &Lf = ft.L;
@@ -120,14 +171,16 @@ __global__ void __launch_bounds__(256) k_average_down(const __grid_constant__ AD
         const int b = (int)(r % o.ext[1]);
         const int c = (int)(r / o.ext[1]);
         const int loc[3] = {a, b, c};
-        int64_t fc[3];
+        int64_t fc[3], fg[3];
         int bx[3];
 #pragma unroll
         for (int d = 0; d < 3; d++) {
             const int64_t f = 2 * (o.Io[d] + loc[d] - ops.c0[d]);  // inside [0, N_f) by coverage
+            fg[d] = f;
             bx[d] = (int)(f / ft.bn[d]);
             fc[d] = f - (int64_t)bx[d] * ft.bn[d];
         }
+        if (!ad_covered(ops, sb, fg)) continue;
         const double *src = ft.p[ft.g2l[bx[0] + ft.nb[0] * (bx[1] + ft.nb[1] * bx[2])]];
         const int64_t pc = at(Lf, (int)fc[0], (int)fc[1], (int)fc[2]);
         const int64_t dp = o.dbase + a + b * ops.Lc.py + c * ops.Lc.pz;

@@ -113,6 +113,8 @@ struct crocco_ctx_s {
     crocco_ctx amr_coarse = nullptr;     // set by crocco_amr_link
     int64_t amr_c0[3] = {0, 0, 0};       // coarse index of fine node 0
     double *const *amr_Uc = nullptr;     // coarse state of the current two-level call only
+    std::vector<crocco_ctx> sibs;        // same-level sibling patches (crocco_amr_link_sibling)
+    double *const *const *amr_sibU = nullptr;  // their states for the current call only
     int64_t stage_elems = 0;
     // timing
     bool timing = false;
@@ -660,13 +662,13 @@ static void op_strides(const Lay &L, int64_t st[3]) {
     st[2] = L.pz;
 }
 
-static crocco_status flush_cf(crocco_ctx c, CFOps &cf, const LevelTab &ct) {
+static crocco_status flush_cf(crocco_ctx c, CFOps &cf, const LevelTab &ct, const SibTab &sb) {
     if (cf.nops == 0) return CROCCO_OK;
     int64_t mx = 0;
     for (int i = 0; i < cf.nops; i++)
         mx = std::max(mx, (int64_t)cf.op[i].ext[0] * cf.op[i].ext[1] * cf.op[i].ext[2]);
     dim3 grid(std::min<int64_t>(cdiv(mx, 256), 4096), cf.nops);
-    LAUNCH(c, K_AMR, k_cf_interp<<<grid, 256, 0, c->stream>>>(cf, ct));
+    LAUNCH(c, K_AMR, k_cf_interp<<<grid, 256, 0, c->stream>>>(cf, ct, sb));
     cf.nops = 0;
     return CROCCO_OK;
 }
@@ -685,6 +687,25 @@ static void level_tab(const crocco_ctx_s *lv, double *const *ptr, LevelTab &t) {
     }
 }
 
+// the blocks of f's same-level siblings in f's fine index space, with the states of this call
+static void sib_tab(const crocco_ctx_s *f, SibTab &t) {
+    memset(&t, 0, sizeof t);
+    if (!f->amr_sibU) return;
+    for (size_t s = 0; s < f->sibs.size(); s++) {
+        const crocco_ctx_s *g = f->sibs[s];
+        for (size_t b = 0; b < g->loc.size() && t.n < SIB_MAX_BLOCKS; b++) {
+            const LocalBlock &lb = g->loc[b];
+            for (int d = 0; d < 3; d++) {
+                t.lo[t.n][d] = 2 * (g->amr_c0[d] - f->amr_c0[d]) + lb.g.origin[d];
+                t.hi[t.n][d] = t.lo[t.n][d] + lb.g.n[d];
+            }
+            t.p[t.n] = f->amr_sibU[s][b];
+            t.L[t.n] = lb.L;
+            t.n++;
+        }
+    }
+}
+
 static crocco_status fill_phase(crocco_ctx c, double *const *f, int kind, int D,
                                 double *const *met, double t) {
     const bool copies_only = kind == FILL_STATE_COPIES;
@@ -695,7 +716,18 @@ static crocco_status fill_phase(crocco_ctx c, double *const *f, int kind, int D,
     CFOps cf;
     cf.nops = 0;
     LevelTab ct;
+    memset(&ct, 0, sizeof ct);
     const bool interp = kind == CROCCO_FIELD_STATE && !copies_only && c->amr_Uc && c->amr_coarse;
+    // C/F faces: interpolation (+ sibling copies), or -- copies-only fills of AverageDown with
+    // siblings -- the sibling copies alone
+    const bool cfface = interp || (copies_only && c->amr_sibU && !c->sibs.empty());
+    SibTab sb;
+    sib_tab(c, sb);
+    cf.interp = interp ? 1 : 0;
+    if (cfface) {
+        cf.Lf = c->loc.empty() ? Lay{} : c->loc[0].L;
+        for (int e = 0; e < 3; e++) cf.c0[e] = c->amr_c0[e];
+    }
     if (interp) {
         level_tab(c->amr_coarse, c->amr_Uc, ct);
         cf.Lf = c->loc.empty() ? Lay{} : c->loc[0].L;
@@ -727,10 +759,11 @@ static crocco_status fill_phase(crocco_ctx c, double *const *f, int kind, int D,
             o.sbase = at(sb.L, (int)m.src_lo[0], (int)m.src_lo[1], (int)m.src_lo[2]);
             o.mode = BOX_COPY;
         } else {
-            if (kind == CROCCO_FIELD_METRIC || copies_only) continue;  // physical faces keep computed metrics
             const int bc = m.bc_kind;
+            if (kind == CROCCO_FIELD_METRIC || (copies_only && !(bc == CROCCO_BC_COARSE_FINE && cfface)))
+                continue;  // physical faces keep computed metrics; copies-only fills skip BCs
             if (bc == CROCCO_BC_COARSE_FINE) {  // FillPatchTwoLevels (reading 25); untouched without a coarse level
-                if (!interp) continue;
+                if (!cfface) continue;
                 CFOp q;
                 q.dst = f[dl];
                 q.dbase = o.dbase;
@@ -740,7 +773,7 @@ static crocco_status fill_phase(crocco_ctx c, double *const *f, int kind, int D,
                 }
                 cf.op[cf.nops++] = q;
                 if (cf.nops == CF_MAX_OPS) {
-                    crocco_status s2 = flush_cf(c, cf, ct);
+                    crocco_status s2 = flush_cf(c, cf, ct, sb);
                     if (s2) return s2;
                 }
                 continue;
@@ -787,7 +820,7 @@ static crocco_status fill_phase(crocco_ctx c, double *const *f, int kind, int D,
     }
     crocco_status st = flush_ops(c, ops);
     if (st) return st;
-    if (interp && (st = flush_cf(c, cf, ct))) return st;
+    if (cfface && (st = flush_cf(c, cf, ct, sb))) return st;
     if (remote.empty()) return CROCCO_OK;
     if (!c->comm) return fail(c, CROCCO_ERR_STATE, "remote halo without communicator");
     // pack sends (a loopback message is both sent and received by this rank)
@@ -1435,15 +1468,21 @@ crocco_status crocco_average_down(crocco_ctx f, double *const *Uf, double *const
     const crocco_ctx_s *c = f->amr_coarse;
     LevelTab ft;
     level_tab(f, Uf, ft);
+    SibTab sb;
+    sib_tab(f, sb);
     ADOps ops;
     memset(&ops, 0, sizeof ops);
     ops.Lc = c->loc.empty() ? Lay{} : c->loc[0].L;
-    for (int d = 0; d < 3; d++) ops.c0[d] = f->amr_c0[d];
+    for (int d = 0; d < 3; d++) {
+        ops.c0[d] = f->amr_c0[d];
+        ops.Nf[d] = f->desc.n_global[d];
+        ops.per[d] = f->desc.bc[d][0] == CROCCO_BC_PERIODIC;
+    }
     int64_t mx = 0;
     auto flush = [&]() -> crocco_status {
         if (ops.nops == 0) return CROCCO_OK;
         dim3 grid(std::min<int64_t>(cdiv(mx, 256), 4096), ops.nops);
-        LAUNCH(f, K_AMR, k_average_down<<<grid, 256, 0, f->stream>>>(ops, ft));
+        LAUNCH(f, K_AMR, k_average_down<<<grid, 256, 0, f->stream>>>(ops, ft, sb));
         ops.nops = 0;
         mx = 0;
         return CROCCO_OK;
@@ -1454,6 +1493,10 @@ crocco_status crocco_average_down(crocco_ctx f, double *const *Uf, double *const
         bool empty = false;
         for (int d = 0; d < 3; d++) {
             covered_range(f, d, lo[d], hi[d]);
+            if (sb.n > 0 && f->desc.bc[d][0] != CROCCO_BC_PERIODIC) {  // nodes whose central fine node
+                lo[d] = f->amr_c0[d];                                   // is ours; k_average_down
+                hi[d] = f->amr_c0[d] + (f->desc.n_global[d] - 1) / 2;    // checks the 27 nodes
+            }
             lo[d] = std::max<int64_t>(lo[d], b.g.origin[d]);
             hi[d] = std::min<int64_t>(hi[d], b.g.origin[d] + b.g.n[d] - 1);
             empty = empty || lo[d] > hi[d];
@@ -1470,6 +1513,83 @@ crocco_status crocco_average_down(crocco_ctx f, double *const *Uf, double *const
         if (ops.nops == CF_MAX_OPS && (st = flush())) return st;
     }
     return flush();
+}
+
+crocco_status crocco_amr_link_sibling(crocco_ctx f, crocco_ctx g) {
+    LIVE(f);
+    LIVE(g);
+    if (f == g) return fail(f, CROCCO_ERR_ARG, "a patch is not its own sibling");
+    if (!f->amr_coarse || f->amr_coarse != g->amr_coarse)
+        return fail(f, CROCCO_ERR_ARG, "siblings must be linked (crocco_amr_link) to the same coarse level");
+    if (f->desc.nranks != 1 || g->desc.nranks != 1)
+        return fail(f, CROCCO_ERR_ARG, "same-level siblings: single-rank levels only");
+    for (auto s : f->sibs)
+        if (s == g) return CROCCO_OK;
+    if (f->sibs.size() >= 8 || g->sibs.size() >= 8) return fail(f, CROCCO_ERR_ARG, "at most 8 siblings per patch");
+    int nb = 0;
+    for (auto s : f->sibs) nb += (int)s->loc.size();
+    int ng = 0;
+    for (auto s : g->sibs) ng += (int)s->loc.size();
+    if (nb + (int)g->loc.size() > SIB_MAX_BLOCKS || ng + (int)f->loc.size() > SIB_MAX_BLOCKS)
+        return fail(f, CROCCO_ERR_ARG, "at most %d sibling blocks per patch", SIB_MAX_BLOCKS);
+    // interiors disjoint (in the common fine index space 2 c0 + f); a periodic direction spans all
+    bool overlap = true;
+    for (int d = 0; d < 3; d++) {
+        if (f->desc.bc[d][0] == CROCCO_BC_PERIODIC || g->desc.bc[d][0] == CROCCO_BC_PERIODIC) continue;
+        const int64_t a0 = 2 * f->amr_c0[d], a1 = a0 + f->desc.n_global[d];
+        const int64_t b0 = 2 * g->amr_c0[d], b1 = b0 + g->desc.n_global[d];
+        overlap = overlap && a0 < b1 && b0 < a1;
+        if (((b0 - a0) & 1) != 0) return fail(f, CROCCO_ERR_ARG, "sibling offset must be even in direction %d", d);
+    }
+    if (overlap) return fail(f, CROCCO_ERR_ARG, "sibling patches overlap");
+    f->sibs.push_back(g);
+    g->sibs.push_back(f);
+    return CROCCO_OK;
+}
+
+static crocco_status sib_ready(crocco_ctx f, double *const *const *sibU) {
+    if (f->sibs.empty()) return CROCCO_OK;
+    if (!sibU) return fail(f, CROCCO_ERR_ARG, "null sibling pointer table");
+    for (size_t s = 0; s < f->sibs.size(); s++) {
+        if (!sibU[s]) return fail(f, CROCCO_ERR_ARG, "null sibling %zu pointer array", s);
+        for (size_t b = 0; b < f->sibs[s]->loc.size(); b++)
+            if (!sibU[s][b]) return fail(f, CROCCO_ERR_ARG, "null sibling %zu block %zu pointer", s, b);
+    }
+    return CROCCO_OK;
+}
+
+crocco_status crocco_fill_patch_level(crocco_ctx f, double *const *Uf, double *const *Mf, double *const *Uc,
+                                      double *const *const *sibU) {
+    LIVE(f);
+    crocco_status st = sib_ready(f, sibU);
+    if (st) return st;
+    f->amr_sibU = sibU;
+    st = crocco_fill_patch_two_levels(f, Uf, Mf, Uc);
+    f->amr_sibU = nullptr;
+    return st;
+}
+
+crocco_status crocco_amr_rk_stage_level(crocco_ctx f, int32_t stage, double dt, double *const *Uin,
+                                        double *const *Uout, double *const *dU, double *const *M,
+                                        double *const *Uc_in, double *const *const *sib_in) {
+    LIVE(f);
+    crocco_status st = sib_ready(f, sib_in);
+    if (st) return st;
+    f->amr_sibU = sib_in;
+    st = crocco_amr_rk_stage(f, stage, dt, Uin, Uout, dU, M, Uc_in);
+    f->amr_sibU = nullptr;
+    return st;
+}
+
+crocco_status crocco_average_down_level(crocco_ctx f, double *const *Uf, double *const *Uc,
+                                        double *const *const *sibU) {
+    LIVE(f);
+    crocco_status st = sib_ready(f, sibU);
+    if (st) return st;
+    f->amr_sibU = sibU;
+    st = crocco_average_down(f, Uf, Uc);
+    f->amr_sibU = nullptr;
+    return st;
 }
 
 crocco_status crocco_check_state(crocco_ctx c, double *const *U, int64_t *n_bad) {

@@ -227,10 +227,11 @@ class AmrSolver:
     fine node 0 at coarse node c0[p] (ratio 2, node-centred).  step() follows Algorithm 2
     (PAPER.md:102-119): per stage the coarse level, then every patch of the fine level with its
     C/F ghosts interpolated from the coarse stage input, then AverageDown at the third stage.
-    Patches of the same level must be disjoint with no patch's ghost band (4 fine points)
-    reaching into another patch's interior: each patch's ghosts come from the coarse level only
-    (touching patches would need a same-level exchange between them, not built).  Plumbing only
-    -- the C ABI does every step."""
+    Patches of the same level must have disjoint interiors; patches whose 4-point ghost band
+    reaches into another patch's interior (abutting or nearby patches) are linked as siblings
+    (crocco_amr_link_sibling, reading 31): their C/F ghosts inside a sibling take the sibling's
+    stage input, and AverageDown covers the nodes whose cell lies in the union of the level's
+    patches.  Plumbing only -- the C ABI does every step."""
 
     def __init__(self, coarse: Solver, fine, c0):
         fines = list(fine) if isinstance(fine, (list, tuple)) else [fine]
@@ -241,9 +242,14 @@ class AmrSolver:
         self.coarse = coarse
         self.patches = list(zip(fines, c0s))
         self.fine, self.c0 = self.patches[0]
-        self._check_disjoint()
+        pairs = self._sibling_pairs()
         for F, c in self.patches:
             cc.crocco_amr_link(F.ctx, coarse.ctx, c)
+        self.sibs = [[] for _ in self.patches]   # per patch, sibling indices in link order
+        for a, b in pairs:
+            cc.crocco_amr_link_sibling(self.patches[a][0].ctx, self.patches[b][0].ctx)
+            self.sibs[a].append(b)
+            self.sibs[b].append(a)
 
     def _box(self, F, c, grow):
         """Fine-level index box [lo, hi) of a patch in the common fine index space (2x coarse);
@@ -256,33 +262,50 @@ class AmrSolver:
                 out.append((2 * c[d] - grow, 2 * c[d] + F.desc.n_global[d] + grow))
         return out
 
-    def _check_disjoint(self):
+    def _sibling_pairs(self):
+        """Pairs of patches whose ghost bands reach into each other's interior (siblings);
+        overlapping interiors are refused."""
         G4 = cc.GHOST
+
+        def meets(A, B):
+            return all(x is None or y is None or (x[0] < y[1] and y[0] < x[1]) for x, y in zip(A, B))
+
+        pairs = []
         for a in range(len(self.patches)):
-            for b in range(len(self.patches)):
-                if a == b:
-                    continue
-                A = self._box(*self.patches[a], G4)
-                B = self._box(*self.patches[b], 0)
-                if all(x is None or y is None or (x[0] < y[1] and y[0] < x[1]) for x, y in zip(A, B)):
-                    raise ValueError(f"fine patches {a} and {b} overlap or touch within the ghost band")
+            for b in range(a + 1, len(self.patches)):
+                if meets(self._box(*self.patches[a], 0), self._box(*self.patches[b], 0)):
+                    raise ValueError(f"fine patches {a} and {b} overlap")
+                if meets(self._box(*self.patches[a], G4), self._box(*self.patches[b], 0)) or \
+                        meets(self._box(*self.patches[b], G4), self._box(*self.patches[a], 0)):
+                    pairs.append((a, b))
+        return pairs
+
+    def _sib_ptrs(self, i, states):
+        return [states[j] for j in self.sibs[i]]
 
     def fill_fine(self):
-        """FillPatchTwoLevels of every patch's current state from the current coarse state."""
-        for F, _ in self.patches:
-            cc.crocco_fill_patch_two_levels(F.ctx, F._ptrs(F.U), F._ptrs(F.met), self.coarse._ptrs(self.coarse.U))
+        """FillPatchTwoLevels of every patch's current state from the current coarse state
+        (and its siblings' current states)."""
+        cur = [F._ptrs(F.U) for F, _ in self.patches]
+        for i, (F, _) in enumerate(self.patches):
+            cc.crocco_fill_patch_level(F.ctx, F._ptrs(F.U), F._ptrs(F.met), self.coarse._ptrs(self.coarse.U),
+                                       self._sib_ptrs(i, cur))
 
     def average_down(self):
-        for F, _ in self.patches:
-            cc.crocco_average_down(F.ctx, F._ptrs(F.U), self.coarse._ptrs(self.coarse.U))
+        cur = [F._ptrs(F.U) for F, _ in self.patches]
+        for i, (F, _) in enumerate(self.patches):
+            cc.crocco_average_down_level(F.ctx, F._ptrs(F.U), self.coarse._ptrs(self.coarse.U),
+                                         self._sib_ptrs(i, cur))
 
     def stage(self, s, dt):
         C = self.coarse
         Uc_in = C.U
         C.stage(s, dt)                                   # fills Uc_in's ghosts, writes C.V; swaps
+        ins = [F._ptrs(F.U) for F, _ in self.patches]    # every patch's stage input
+        for i, (F, _) in enumerate(self.patches):
+            cc.crocco_amr_rk_stage_level(F.ctx, s, dt, F._ptrs(F.U), F._ptrs(F.V), F._ptrs(F.dU),
+                                         F._ptrs(F.met), C._ptrs(Uc_in), self._sib_ptrs(i, ins))
         for F, _ in self.patches:
-            cc.crocco_amr_rk_stage(F.ctx, s, dt, F._ptrs(F.U), F._ptrs(F.V), F._ptrs(F.dU), F._ptrs(F.met),
-                                   C._ptrs(Uc_in))
             F.U, F.V = F.V, F.U
         if s == 2:
             self.average_down()

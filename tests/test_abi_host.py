@@ -156,8 +156,9 @@ def test_plan_marks_coarse_fine_faces_physical():
         assert m.kind == 1 and m.src_block == -1
 
 
-def test_amr_patch_separation_check_host_logic():
-    """AmrSolver refuses same-level patches whose ghost band reaches another patch (host logic)."""
+def test_amr_patch_sibling_detection_host_logic():
+    """AmrSolver links same-level patches whose ghost band reaches another patch as siblings
+    (reading 31) and refuses overlapping interiors (host logic)."""
     from types import SimpleNamespace as NS
     from paper_conf_ipps_davissngmb23_b200.solver import AmrSolver
     CF = cc.BC_COARSE_FINE
@@ -166,7 +167,11 @@ def test_amr_patch_separation_check_host_logic():
         return NS(desc=NS(bc=((CF, CF), (CF, CF), (0, 0)), n_global=n))
     A = AmrSolver.__new__(AmrSolver)
     A.patches = [(patch((16, 16, 8)), (2, 2, 0)), (patch((16, 16, 8)), (14, 2, 0))]
-    A._check_disjoint()                                      # x: [4,20)+-4 vs [28,44): apart
+    assert A._sibling_pairs() == []                          # x: [4,20)+-4 vs [28,44): apart
     A.patches[1] = (patch((16, 16, 8)), (11, 2, 0))          # [22,38) within 4 of [4,20)
+    assert A._sibling_pairs() == [(0, 1)]
+    A.patches[1] = (patch((16, 16, 8)), (10, 2, 0))          # [20,36): abutting
+    assert A._sibling_pairs() == [(0, 1)]
+    A.patches[1] = (patch((16, 16, 8)), (9, 2, 0))           # [18,34): interiors overlap
     with pytest.raises(ValueError):
-        A._check_disjoint()
+        A._sibling_pairs()

@@ -266,8 +266,8 @@ def test_two_disjoint_fine_patches_parity():
         for g, rr in zip(S.get(S.U), refs):
             ri = rr[:, G:-G, G:-G, G:-G]
             assert rel_linf(g[:, G:-G, G:-G, G:-G], ri, state_scale(ri)) <= 1e-9
-    with pytest.raises(ValueError):               # patches touching within the ghost band
-        AmrSolver(C, Fs, [(2, 3, 2), (11, 6, 3)])
+    with pytest.raises(ValueError):               # patches with overlapping interiors
+        AmrSolver(C, Fs, [(2, 3, 2), (9, 6, 3)])
     C.close()
     for F in Fs:
         F.close()
@@ -466,3 +466,78 @@ def test_amr_abi_refusals():
     A.sync()
     C.close()
     F.close()
+
+
+def _gpu_level(nc, grid, nbc, specs, state, phys):
+    from paper_conf_ipps_davissngmb23_b200 import crocco as cc
+    from paper_conf_ipps_davissngmb23_b200.solver import AmrSolver, Solver
+    bcf = ((CF, CF),) * 3
+    xc = grid.coords(nc, (0, 0, 0), oracle.GC)
+    C = Solver(nc, nbc, PER, cc.make_phys(**phys))
+    bn, blocks = block_slices(nc, nbc)
+    C.set_coords([grid.coords(bn, o, oracle.GC) for o, _ in blocks])
+    C.set_state([np.ascontiguousarray(state(xc)[(slice(None),) + sl]) for _, sl in blocks])
+    Fs = []
+    for c0, nf, nb in specs:
+        F = Solver(nf, nb, bcf, cc.make_phys(**phys))
+        bnf, bl = block_slices(nf, nb)
+        xf = synth.Refined(grid, c0).coords(nf, (0, 0, 0), oracle.GC)
+        F.set_coords([synth.Refined(grid, c0).coords(bnf, o, oracle.GC) for o, _ in bl])
+        U0 = state(xf)
+        F.set_state([np.ascontiguousarray(U0[(slice(None),) + sl]) for _, sl in bl])
+        Fs.append(F)
+    return C, Fs, AmrSolver(C, Fs, [s[0] for s in specs])
+
+
+@pytest.mark.parametrize("axis", [0, 1])
+def test_abutting_patches_parity_and_union(axis):
+    """NEXT-4 completion (reading 31): two abutting fine patches of one level,
+    siblings exchanging their ghosts (crocco_amr_rk_stage_level / crocco_average_down_level),
+    multi-block on both levels.  (a) parity <= 1e-9 with the oracle functions composed in
+    Algorithm 2's order (tests/test_oracle_amr.py advance_level) after 3 RK3 steps; (b) bitwise
+    equal to the GPU run of the single patch covering their union."""
+    from test_oracle_amr import advance_level, _level_setup
+    nc = (24, 20, 16)
+    grid = synth.Wavy3D(L=(10.0,) * 3, N=nc)
+    phys = dict(terms=3, mu_ref=0.01)
+    c0, nu = (3, 4, 2), [24, 16, 12]
+    half = [nu[d] // 2 if d == axis else nu[d] for d in range(3)]
+    c0b = tuple(c0[d] + (half[d] // 2 if d == axis else 0) for d in range(3))
+    st = lambda x: synth.vortex(x)
+    specs = [(c0, tuple(half), (2, 1, 1) if axis == 1 else (1, 2, 1)), (c0b, tuple(half), (1, 1, 2))]
+    dt, nsteps = 0.01, 3
+    metc, Uc, P = _level_setup(nc, grid, [(s[0], s[1]) for s in specs], st)
+    advance_level(nc, metc, Uc, P, oracle.phys(**phys), dt, nsteps)
+    C, Fs, A = _gpu_level(nc, grid, (2, 1, 1), specs, st, phys)
+    assert A.sibs == [[1], [0]]
+    A.step(dt, nsteps)
+    A.sync()
+    _, _, refs = _blocks_of(Uc, nc, (2, 1, 1))
+    for g, rr in zip(C.get(C.U), refs):
+        ri = rr[:, G:-G, G:-G, G:-G]
+        assert rel_linf(g[:, G:-G, G:-G, G:-G], ri, state_scale(ri)) <= 1e-9
+    got_parts = []
+    for F, (c0p, nf, nb), p in zip(Fs, specs, P):
+        _, _, refs = _blocks_of(p["U"], nf, nb)
+        gl = F.get(F.U)
+        for g, rr in zip(gl, refs):
+            ri = rr[:, G:-G, G:-G, G:-G]
+            assert rel_linf(g[:, G:-G, G:-G, G:-G], ri, state_scale(ri)) <= 1e-9
+        glob = np.zeros((5, nf[2], nf[1], nf[0]))
+        bnf, bl = block_slices(nf, nb)
+        for (o, sl), g in zip(bl, gl):
+            glob[(slice(None),) + sl] = g[:, G:-G, G:-G, G:-G]
+        got_parts.append(glob)
+    coarse_two = [g.copy() for g in C.get(C.U)]
+    for S in [C] + Fs:
+        S.close()
+    # the union patch on the GPU
+    Cu, Fu, Au = _gpu_level(nc, grid, (2, 1, 1), [(c0, tuple(nu), (1, 1, 1))], st, phys)
+    Au.step(dt, nsteps)
+    Au.sync()
+    union = Fu[0].get(Fu[0].U)[0][:, G:-G, G:-G, G:-G]
+    assert np.array_equal(np.concatenate(got_parts, axis=3 - axis), union)
+    for a, b in zip(coarse_two, Cu.get(Cu.U)):
+        assert np.array_equal(a, b)
+    for S in [Cu] + Fu:
+        S.close()
