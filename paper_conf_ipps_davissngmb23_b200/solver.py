@@ -338,28 +338,44 @@ class AmrHierarchy:
 
     def __init__(self, base: Solver, levels):
         self.levels = [[(base, None, None)]] + [list(lv) for lv in levels]
+        self.sibs = [[[]]]
         for k in range(1, len(self.levels)):
             for S, parent, c0 in self.levels[k]:
                 P = self.levels[k - 1][parent][0]
                 cc.crocco_amr_link(S.ctx, P.ctx, tuple(int(x) for x in c0))
+            # patches of one level under the same parent whose ghost bands meet: siblings (reading 31)
+            lv = self.levels[k]
+            sib = [[] for _ in lv]
+            for parent in sorted({p for _, p, _ in lv}):
+                idx = [i for i, (_, p, _) in enumerate(lv) if p == parent]
+                tmp = AmrSolver.__new__(AmrSolver)
+                tmp.patches = [(lv[i][0], tuple(int(x) for x in lv[i][2])) for i in idx]
+                for a, b in tmp._sibling_pairs():
+                    cc.crocco_amr_link_sibling(lv[idx[a]][0].ctx, lv[idx[b]][0].ctx)
+                    sib[idx[a]].append(idx[b])
+                    sib[idx[b]].append(idx[a])
+            self.sibs.append(sib)
 
     def stage(self, s, dt):
         prev_in = None
         for k, lv in enumerate(self.levels):
-            cur_in = []
-            for S, parent, _ in lv:
-                U_in = S.U
+            cur_in = [S._ptrs(S.U) for S, _, _ in lv]     # every patch's stage input
+            for i, (S, parent, _) in enumerate(lv):
                 if k == 0:
                     S.stage(s, dt)                       # fills U_in's ghosts, writes S.V; swaps
                 else:
-                    cc.crocco_amr_rk_stage(S.ctx, s, dt, S._ptrs(S.U), S._ptrs(S.V), S._ptrs(S.dU),
-                                           S._ptrs(S.met), prev_in[parent])
+                    cc.crocco_amr_rk_stage_level(S.ctx, s, dt, S._ptrs(S.U), S._ptrs(S.V), S._ptrs(S.dU),
+                                                 S._ptrs(S.met), prev_in[parent],
+                                                 [cur_in[j] for j in self.sibs[k][i]])
+            if k >= 1:
+                for S, _, _ in lv:
                     S.U, S.V = S.V, S.U
-                cur_in.append(S._ptrs(U_in))
             if s == 2 and k >= 1:                        # AverageDown of level k onto level k-1
-                for S, parent, _ in lv:
+                cur = [S._ptrs(S.U) for S, _, _ in lv]
+                for i, (S, parent, _) in enumerate(lv):
                     P = self.levels[k - 1][parent][0]
-                    cc.crocco_average_down(S.ctx, S._ptrs(S.U), P._ptrs(P.U))
+                    cc.crocco_average_down_level(S.ctx, S._ptrs(S.U), P._ptrs(P.U),
+                                                 [cur[j] for j in self.sibs[k][i]])
             prev_in = cur_in
 
     def step(self, dt, nsteps=1):
