@@ -602,7 +602,6 @@ def run_dmr_amr(args):
     for v in kt.values():
         v["share_of_kernel_time"] = v["ms"] / max(ktot, 1e-9)
     pts = [n[0] * n[1] * n[2] for n, *_ in specs]
-    uniform = n0[0] * n0[1] * n0[2] * 64                      # finest spacing h/4 everywhere
     value = sum(pts) * 3 * args.steps / (ms / 1e3)
     finite = all(X.check_state() == 0 for X in S)
     out = {"metric": METRIC, "value": value, "unit": UNIT, "n_gpus": 1, "steps": args.steps,
@@ -612,8 +611,7 @@ def run_dmr_amr(args):
            "config": {"workload": WORKLOADS["dmr_amr"] + "; step = 1 RK3 step (3 stages x 3 levels + AverageDown)",
                       "levels": [{"n": list(n), "c0": list(c0) if c0 else None, "blocks": list(nb), "points": p}
                                  for (n, _, _, _, _, nb, c0), p in zip(specs, pts)],
-                      "points": sum(pts), "uniform_finest_points": uniform,
-                      "amr_point_saving": 1.0 - sum(pts) / uniform, "dt": dt,
+                      "points": sum(pts), "dt": dt,
                       "l2": "inputs larger than L2", "parallelism": "1 GPU"},
            "amr_kernels_share": sum(v["ms"] for k, v in kt.items() if k.endswith(":amr")) / max(ktot, 1e-9),
            "kernel_breakdown": kt, "gpu_launches": launches, "clocks": clocks, "state_finite": finite,

@@ -673,3 +673,31 @@ def test_nccl_loopback_equals_local_and_oracle(bc, nb, ov):
         S.close()
     assert np.array_equal(outs[0], outs[1])
     assert dts[0] == dts[1]
+
+
+@pytest.mark.slow
+def test_overlap_has_interior_slabs_at_bench_depth():
+    """with the run-time slab depth of 256 planes (chosen when the block is large) no
+    viscous tile was ghost-free and the overlapped stage silently ran serially.  With overlap the
+    depth is capped so an interior slab exists: a 512 x 512 x 264 block (slab 256 without the cap)
+    runs every stage overlapped, bitwise equal to the serial stage."""
+    from paper_conf_ipps_davissngmb23_b200 import crocco as cc
+    n = (512, 512, 264)
+    g = synth.Wavy3D(L=(2 * math.pi,) * 3, N=n, x0=(-math.pi,) * 3, k=2.0, A=0.15)
+    import torch
+    outs = []
+    for ov in (0, 1):
+        from paper_conf_ipps_davissngmb23_b200.solver import Solver
+        S = Solver(n, (1, 1, 1), PER, cc.make_phys(gamma=1.4, R=1.0, Pr=0.71, mu_ref=1 / 1600))
+        xyz = torch.from_numpy(g.coords(n, (0, 0, 0), oracle.GC)).cuda()
+        S.set_coords([xyz])
+        S.set_state([synth.tgv(xyz, noise=0.01, seed=5)])
+        del xyz
+        cc.crocco_set_overlap(S.ctx, ov)
+        S.step(2e-4, 1)
+        S.sync()
+        assert cc.crocco_overlap_count(S.ctx) == (3 if ov else 0)
+        outs.append(S.view(S.U[0], 0, 5)[:, 4:-4, 4:-4, 4:-4].cpu().numpy())
+        S.close()
+        torch.cuda.empty_cache()
+    assert np.array_equal(outs[0], outs[1])
