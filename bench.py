@@ -545,8 +545,7 @@ def run_dmr_amr(args):
     """--config dmr_amr (one GPU): Algorithm 2 over three levels (AmrHierarchy): per stage the base
     DMR grid, the level-1 and level-2 patches (C/F ghosts from the parent's stage input, DMR
     boundary data on the wall faces), AverageDown of each level after its third-stage update.
-    value = (all levels' interior points) x 3 x steps / time.  Also reports the point count of the
-    equivalent uniform finest grid (the paper's AMR-savings measure)."""
+    value = (all levels' interior points) x 3 x steps / time."""
     import torch
 
     import synth
