@@ -1104,6 +1104,7 @@ static crocco_status rhs_block(crocco_ctx c, const LocalBlock &b, const double *
         a.mode = d == 0 ? ((ph.terms & CROCCO_TERM_VISCOUS) ? 4 : 0) : (d == 1 ? 1 : final_mode);
         a.rhs = rhs;
         a.Uin = Uin;
+        if (final_mode == 3 && Uin != U) return fail(c, CROCCO_ERR_ARG, "RK stage: U_in must be the swept state");
         a.Uout = Uout;
         a.dU = dU;
         a.stage = stage;

@@ -41,7 +41,7 @@ struct SweepArgs {
                         // 4 add to the viscous divergence in R comps 1..4 (k_visc_tiled), write comp 0
     int seg;            // march segment
     double *rhs;        // mode 2 (padded layout)
-    const double *Uin;  // mode 3 (padded layout)
+    const double *Uin;  // mode 3 (padded layout): must be the swept state in.U (its values are read from the ring)
     double *Uout, *dU;
     double A, B, dt;
     int stage;
@@ -74,8 +74,8 @@ struct RingGeom {
     static_assert(NR >= (LA + 2) * WS && (NR & (NR - 1)) == 0, "ring too small");
     static constexpr int SVN = sv_n(VISC);         // staged values per ring point
     // prefetched accumulate / update operands per lane: xi (mode 0 / 4) and eta (mode 1) read R;
-    // zeta finishes the point (mode 2: R, J; mode 3: R, J, dU, U_in)
-    static constexpr int NCB = D == 2 ? 16 : 5;
+    // zeta finishes the point (mode 2: R, J; mode 3: R, J, dU -- U_in comes from the ring)
+    static constexpr int NCB = D == 2 ? 11 : 5;
     static constexpr bool CARRY = (CARRY_SMEM >> D) & 1;
     static constexpr int NFC = CARRY ? 2 * 5 * 32 : 0;  // interface fluxes of two steps
     static constexpr int PER_WARP = SVN * NR * C + NCB * 32 + NFC;  // doubles
@@ -255,7 +255,6 @@ __global__ void __launch_bounds__(sweep_threads(D), sweep_minb(D)) k_sweep_s(con
 #pragma unroll
                     for (int c = 0; c < 5; c++) {
                         if (a.stage != 0) cp_async8(cb + 32 * (6 + c), a.dU + c * L.cs + pp);
-                        cp_async8(cb + 32 * (11 + c), a.Uin + c * L.cs + pp);
                     }
                 }
             }
@@ -325,7 +324,9 @@ __global__ void __launch_bounds__(sweep_threads(D), sweep_minb(D)) k_sweep_s(con
                         const double rv = J * Rt[c];
                         const double du = (a.stage == 0) ? a.dt * rv : fma(a.A, cb[32 * (6 + c)], a.dt * rv);
                         a.dU[c * L.cs + pp] = du;
-                        a.Uout[c * L.cs + pp] = fma(a.B, du, cb[32 * (11 + c)]);
+                        // U_in of the finished point = stencil point i of the ring (U_in is the
+                        // swept state): no second read of U_in
+                        a.Uout[c * L.cs + pp] = fma(a.B, du, A.U(2, c));
                     }
                 }
             }
