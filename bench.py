@@ -669,7 +669,7 @@ def main():
     ap.add_argument("--config", choices=["weak", "ramp", "tgv", "vortex", "sod", "dmr", "amr", "dmr_amr"],
                     default="weak",
                     help="weak (default, the north_star 512^3/GPU workload) or a fixed BASELINE config")
-    ap.add_argument("--e2e-steps", type=int, default=16,
+    ap.add_argument("--e2e-steps", type=int, default=48,
                     help="independent jobs streamed through host memory for e2e (pipeline fill + drain amortised)")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-clocks", action="store_true")
