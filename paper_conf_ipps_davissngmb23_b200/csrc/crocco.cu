@@ -47,7 +47,6 @@ struct LocalBlock {
     int64_t rcs = 0;
     double *fv = nullptr;    // viscous point flux F^_v^eta (4 comps, interior +-2 box)
     double *met2 = nullptr;  // expanded viscous form: 18 second metrics (compact interior, rcs)
-    double *p4 = nullptr;    // expanded viscous form: u v w T on the padded box
 };
 
 enum { K_RESERVED = 0, K_FLUX_X, K_FLUX_Y, K_FLUX_Z, K_VISC, K_UPDATE, K_FILL, K_METRICS, K_CFL, K_AMR,
@@ -356,6 +355,8 @@ static cudaError_t sweep_attrs() {
     if (e == cudaSuccess) e = sweep_attr1<1, true>();
     if (e == cudaSuccess)
         e = cudaFuncSetAttribute(k_visc_tiled, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)VISC_SMEM);
+    if (e == cudaSuccess)
+        e = cudaFuncSetAttribute(k_visc_exp_tiled, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)VISC_EXP_SMEM);
     return e;
 }
 
@@ -473,7 +474,6 @@ static void free_ctx(crocco_ctx c) {
         cudaFree(b.racc);
         cudaFree(b.fv);
         cudaFree(b.met2);
-        cudaFree(b.p4);
     }
     cudaFree(c->send_stage);
     cudaFree(c->dmax);
@@ -1000,13 +1000,11 @@ crocco_status crocco_init_metrics2(crocco_ctx c, double *const *met) {
     drop_graphs(c);  // new scratch pointers / kernel variant of the expanded viscous form
     for (auto &b : c->loc) {
         if (!b.met2) {
-            if (cudaMalloc((void **)&b.met2, (size_t)(18 * b.rcs) * sizeof(double)) != cudaSuccess ||
-                cudaMalloc((void **)&b.p4, (size_t)(4 * b.L.cs) * sizeof(double)) != cudaSuccess) {
+            if (cudaMalloc((void **)&b.met2, (size_t)(18 * b.rcs) * sizeof(double)) != cudaSuccess) {
                 cudaGetLastError();
                 return fail(c, CROCCO_ERR_NOMEM, "second-metric allocation failed");
             }
-            CK(c, cudaMemsetAsync(b.p4, 0, (size_t)(4 * b.L.cs) * sizeof(double), c->stream));
-            c->scratch += (18 * b.rcs + 4 * b.L.cs) * (int64_t)sizeof(double);
+            c->scratch += 18 * b.rcs * (int64_t)sizeof(double);
         }
     }
     for (size_t bi = 0; bi < c->loc.size(); bi++) {
@@ -1068,11 +1066,12 @@ static crocco_status rhs_block(crocco_ctx c, const LocalBlock &b, const double *
     const bool vexp = (ph.terms & CROCCO_TERM_VISCOUS) != 0 && ph.visc_form == 1;  // readings 27-28
     const bool viscous = (ph.terms & CROCCO_TERM_VISCOUS) != 0 && !vexp;
     if (vexp) {  // expanded viscous form: V / J -> R comps 1..4, the xi sweep adds (mode 4)
-        if (!b.met2 || !b.p4)
+        if (!b.met2)
             return fail(c, CROCCO_ERR_STATE, "visc_form = 1 needs crocco_init_metrics2");
-        LAUNCH(c, K_VISC, k_prims4<<<cdiv(b.L.cs, 256), 256, 0, c->stream>>>(U, b.p4, b.L, ph));
-        const int64_t ni = (int64_t)b.g.n[0] * b.g.n[1] * b.g.n[2];
-        LAUNCH(c, K_VISC, k_visc_exp<<<cdiv(ni, 128), 128, 0, c->stream>>>(b.p4, M, b.met2, b.racc, b.rcs, b.L, ph));
+        const unsigned nt = (unsigned)(((b.g.n[0] + XTX - 1) / XTX) * ((b.g.n[1] + XTY - 1) / XTY) *
+                                       ((b.g.n[2] + XVK - 1) / XVK));
+        LAUNCH(c, K_VISC, k_visc_exp_tiled<<<nt, XTX * XTY, VISC_EXP_SMEM, c->stream>>>(U, M, b.met2, b.racc,
+                                                                                       b.rcs, b.L, ph));
     } else if (viscous && visc_sel != 1) {
         // k_visc_tiled: R comps 1..4 = D4_xi + D4_zeta of the point fluxes, F^_v^eta -> HBM
         // (sel 1, the ghost-free tiles, was launched by visc_interior() beside the fill)
