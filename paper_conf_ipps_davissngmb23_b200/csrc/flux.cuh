@@ -42,14 +42,18 @@ struct FluxIn {
 enum { SV_U = 0, SV_M = 5, SV_FV = 8 };
 __host__ __device__ constexpr int sv_p(bool visc) { return visc ? 12 : 8; }   // first primitive
 __host__ __device__ constexpr int sv_n(bool visc) { return sv_p(visc) + 7; }  // values per point
-template <int NR, int PS, bool VISC>
+// CS = 0: point-major slots (q & (NR-1)) * PS + col (eta / zeta: a chunk of points is contiguous per
+// column row); CS > 0: column-major col * CS + (q & (NR-1)) (xi: consecutive points of a line
+// contiguous, CS padded so a warp's 32 reads take the minimum two wavefronts)
+template <int NR, int PS, bool VISC, int CS = 0>
 struct SAcc {
     static constexpr int SV_P = sv_p(VISC);
     const double *sv;
     int q0, col;
-    static constexpr int VS = NR * PS;
+    static constexpr int VS = CS ? PS * CS : NR * PS;
     __device__ __forceinline__ double at_(int v, int l) const {
-        return sv[v * VS + ((q0 + l) & (NR - 1)) * PS + col];
+        if constexpr (CS != 0) return sv[v * VS + col * CS + ((q0 + l) & (NR - 1))];
+        else return sv[v * VS + ((q0 + l) & (NR - 1)) * PS + col];
     }
     __device__ __forceinline__ double U(int l, int c) const { return at_(SV_U + c, l); }
     __device__ __forceinline__ double P(int l, int k) const { return at_(SV_P + k, l); }

@@ -73,12 +73,19 @@ struct RingGeom {
     static constexpr int NR = (D == 0) ? 32 : 16;  // ring points (>= (LA + 2) * WS, power of 2)
     static_assert(NR >= (LA + 2) * WS && (NR & (NR - 1)) == 0, "ring too small");
     static constexpr int SVN = sv_n(VISC);         // staged values per ring point
+    // xi: column-major ring (16-B copies of point pairs along the line); column stride padded 32 -> 40
+    static constexpr int CS = D == 0 ? NR + 8 : 0;
+    static constexpr int VS = CS ? C * CS : NR * C;  // doubles per staged value
+    static constexpr int QOFF = D == 0 ? 1 : 0;      // xi: ring point 0 is swept index e0 - 4 (even)
+    __host__ __device__ static constexpr int slot(int q, int col) {
+        return CS ? col * CS + (q & (NR - 1)) : (q & (NR - 1)) * C + col;
+    }
     // prefetched accumulate / update operands per lane: xi (mode 0 / 4) and eta (mode 1) read R;
     // zeta finishes the point (mode 2: R, J; mode 3: R, J, dU -- U_in comes from the ring)
     static constexpr int NCB = D == 2 ? 11 : 5;
     static constexpr bool CARRY = (CARRY_SMEM >> D) & 1;
     static constexpr int NFC = CARRY ? 2 * 5 * 32 : 0;  // interface fluxes of two steps
-    static constexpr int PER_WARP = SVN * NR * C + NCB * 32 + NFC;  // doubles
+    static constexpr int PER_WARP = SVN * VS + NCB * 32 + NFC;  // doubles
 };
 
 template <int D, bool VISC, bool LIM>
@@ -86,8 +93,9 @@ __global__ void __launch_bounds__(sweep_threads(D), sweep_minb(D)) k_sweep_s(con
                                                                           const Lay L, const Phys ph) {
     using RG = RingGeom<D, VISC>;
     constexpr int WS = RG::WS, C = RG::C, LA = RG::LA, NR = RG::NR;
-    constexpr int VS = NR * C;
+    constexpr int VS = RG::VS;
     constexpr int SV_P = sv_p(VISC);
+    static_assert(D != 0 || !VISC, "the xi sweep carries no viscous interface term");
     extern __shared__ double smem_dyn[];
     const int lane = threadIdx.x & 31;
     double *sv = smem_dyn + (threadIdx.x >> 5) * RG::PER_WARP;
@@ -105,7 +113,7 @@ __global__ void __launch_bounds__(sweep_threads(D), sweep_minb(D)) k_sweep_s(con
     const int sg = (int)(gw / ntl);
     const int64_t r = gw % ntl;
     const int e0 = sg * a.seg, e1 = min(nd, e0 + a.seg);
-    const int qbase = e0 - 3;                        // swept index of ring point q = 0
+    const int qbase = e0 - 3 - RG::QOFF;             // swept index of ring point q = 0
     const int nsteps = (e1 - e0 + 1 + WS - 1) / WS;  // interfaces e0-1 .. e1-1
     const int qmax = nd + G - 1 - qbase;             // last ring point inside the padded box
     const int64_t sst = D == 0 ? 1 : (D == 1 ? L.py : L.pz);  // swept strides
@@ -139,23 +147,36 @@ __global__ void __launch_bounds__(sweep_threads(D), sweep_minb(D)) k_sweep_s(con
         cpv = D == 1 ? vat(a.V, gi, 0, oo) : vat(a.V, gi, oo, 0);
     }
     const double *Mrow = a.in.M + (int64_t)(1 + 3 * D) * L.cs;
+    // xi copies: line (column) lane & 3 of this warp
+    bool xcv = false;
+    int64_t xco = 0;
+    if (D == 0) {
+        const int64_t t = r * C + (lane & 3);
+        xcv = t < (int64_t)L.n1 * L.n2;
+        if (xcv) xco = at(L, 0, (int)(t % L.n1), (int)(t / L.n1));
+    }
 
     // issue the copies of chunk `ch`: U (5) + metric row (3) [+ FV (4)] of WS points x C columns
     auto issue = [&](int ch) {
         if (D == 0) {
-            // lane: point lane&7 of column lane>>3, all values, 8-B copies
-            const int q = ch * WS + (lane & 7), gq = qbase + q;
-            if (cvalid && q <= qmax) {
-                double *dst = sv + (q & (NR - 1)) * C + lt;
-                const int64_t o = cpo + gq;
+            // xi, column-major ring: 16-B copies of point pairs (2p, 2p+1) -- lane: column lane&3,
+            // pair (lane>>2)&3, values 4 (lane>>4) .. 4 (lane>>4) + 3 (U 0-4, metric row 5-7);
+            // 8-B copies when the segment start is odd (16-B source alignment)
+            const int col = lane & 3, pr = (lane >> 2) & 3, vg = lane >> 4;
+            const int q = ch * WS + 2 * pr, gq = qbase + q;
+            if (xcv && q <= qmax) {
+                const int64_t co = xco;
+                double *dst = sv + RG::slot(q, col);
 #pragma unroll
-                for (int v = 0; v < 5; v++) cp_async8(dst + v * VS, a.in.U + v * L.cs + o);
-#pragma unroll
-                for (int v = 0; v < 3; v++) cp_async8(dst + (SV_M + v) * VS, Mrow + v * L.cs + o);
-                if (VISC && gq >= -2 && gq <= nd + 1) {
-                    const int64_t ov = cpv + gq;
-#pragma unroll
-                    for (int v = 0; v < 4; v++) cp_async8(dst + (SV_FV + v) * VS, a.in.FV + v * a.in.vcs + ov);
+                for (int t = 0; t < 4; t++) {
+                    const int v = 4 * vg + t;
+                    const double *src = (v < 5 ? a.in.U + v * L.cs : Mrow + (v - 5) * L.cs) + co + gq;
+                    if ((e0 & 1) == 0) {
+                        cp_async16(dst + v * VS, src);
+                    } else {
+                        cp_async8(dst + v * VS, src);
+                        if (q + 1 <= qmax) cp_async8(dst + v * VS + 1, src + 1);
+                    }
                 }
             }
         } else {
@@ -186,7 +207,7 @@ __global__ void __launch_bounds__(sweep_threads(D), sweep_minb(D)) k_sweep_s(con
     auto prim_calc = [&](int ch, double pv[7]) {
         const int q = ch * WS + ls;
         if (q > qmax) return;
-        const double *bq = sv + (q & (NR - 1)) * C + lt;
+        const double *bq = sv + RG::slot(q, lt);
         const double rho = bq[0], ru = bq[VS], rv = bq[2 * VS], rw = bq[3 * VS], E = bq[4 * VS];
         const double ir = rcp_nr(rho);
         const double u = ru * ir, v = rv * ir, w = rw * ir;
@@ -202,7 +223,7 @@ __global__ void __launch_bounds__(sweep_threads(D), sweep_minb(D)) k_sweep_s(con
     auto prim_store = [&](int ch, const double pv[7]) {
         const int q = ch * WS + ls;
         if (q > qmax) return;
-        double *bq = sv + (q & (NR - 1)) * C + lt;
+        double *bq = sv + RG::slot(q, lt);
 #pragma unroll
         for (int k = 0; k < 7; k++) bq[(SV_P + k) * VS] = pv[k];
     };
@@ -244,7 +265,7 @@ __global__ void __launch_bounds__(sweep_threads(D), sweep_minb(D)) k_sweep_s(con
         const int e = e0 - 1 + WS * st + ls;  // this lane's interface e+1/2
         const bool act = lvalid && e <= e1 - 1;
         const bool own = act && e >= e0;      // this lane finishes point e
-        const SAcc<NR, C, VISC> A{sv, WS * st + ls, lt};  // ring point of stencil point i-2
+        const SAcc<NR, C, VISC, RG::CS> A{sv, WS * st + ls + RG::QOFF, lt};  // ring point of stencil point i-2
         if (own && a.mode != 0) {             // group A: accumulate / update operands
 #pragma unroll
             for (int c = 0; c < 5; c++)
@@ -264,7 +285,7 @@ __global__ void __launch_bounds__(sweep_threads(D), sweep_minb(D)) k_sweep_s(con
         if (act) {
             FluxSetup su;
             if (inv) flux_setup(A, ph, su);
-            flux_fields<D, SAcc<NR, C, VISC>, LIM>(A, su, inv, VISC, ph, F);
+            flux_fields<D, SAcc<NR, C, VISC, RG::CS>, LIM>(A, su, inv, VISC, ph, F);
         } else {
 #pragma unroll
             for (int c = 0; c < 5; c++) F[c] = 0.0;
