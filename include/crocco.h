@@ -252,16 +252,31 @@ crocco_status crocco_compute_dt(crocco_ctx ctx, double *const *U, double *const 
    All levels take the same dt; per RK stage the coarse level runs first (Alg. 2 l.2 level loop
    inside the stage loop), then the fine level with its C/F ghosts interpolated from the coarse
    stage INPUT, then at stage 2 (the third) AverageDown.  Both ctx must enqueue on the same
-   stream (or the caller orders them).  No inter-level communication: every coarse block a fine
-   block reads (and every fine block a covered coarse node reads) must be local to the rank.
-   Several patches of one level: see the sibling calls below. */
+   stream (or the caller orders them).
+   The levels may be decomposed independently over the ranks (each level is
+   distributed and load-balanced on its own).  Inter-level data then moves as NCCL p2p boxes on
+   the fine ctx's communicator (plan: crocco_amr_plan, fixed at link time):
+     - FillPatch: every coarse box a fine block's C/F ghosts interpolate from (the 8-corner
+       stencils of its ghost boxes, coarse ghosts included) goes from the coarse block's rank to
+       the fine block's rank, into a mirror of that coarse block; the interpolation reads the
+       mirror (bitwise the values it would read from the coarse block itself);
+     - AverageDown: the covered coarse nodes whose central fine node lies in a fine block are
+       averaged on the fine block's rank (into a mirror of the coarse block) and sent to the
+       coarse block's rank, which writes them into U_coarse.
+   Boxes whose coarse and fine blocks share a rank are read / written in place (or through
+   ncclSend/ncclRecv to self under crocco_set_nccl_loopback on the FINE ctx).  So the two-level
+   calls are collective over the fine ctx's communicator: every rank calls them, also a rank
+   that owns no fine block (it may still own coarse blocks that others read).
+   Several patches of one level: see the sibling calls below (single-rank). */
 
 /* Declare `fine` a refinement of `coarse` with fine node 0 at coarse node c0[3].  Checks:
    per direction either the fine level is PERIODIC and spans the periodic coarse domain
    (N_f = 2 N_c, c0 = 0), or 0 <= c0 and 2 c0 + N_f - 1 <= 2 (N_c - 1) with physical (non-C/F)
-   faces only on the domain boundary; <= 64 local / 512 blocks per level; locality as above.
-   CROCCO_ERR_ARG otherwise.  The ctx keep no reference beyond the pair (finalize the fine
-   level first or relink). */
+   faces only on the domain boundary; <= 512 blocks per level; local coarse blocks + coarse
+   mirrors of this rank <= 64; both ctx on the same ranks; a communicator on the fine ctx when
+   the plan has inter-rank boxes.  CROCCO_ERR_ARG otherwise.  Allocates the coarse-block
+   mirrors and the staging buffers of the plan (crocco_scratch_bytes counts them).  The ctx keep
+   no reference beyond the pair (finalize the fine level first or relink). */
 crocco_status crocco_amr_link(crocco_ctx fine, crocco_ctx coarse, const int64_t c0[3]);
 /* FillPatch of the fine level (FillPatchTwoLevels + BC_Fill; reading 25):
    the 3-phase fill of U_fine in place, COARSE_FINE ghosts = trilinear interpolation from the
@@ -331,8 +346,9 @@ crocco_status crocco_launch_count(crocco_ctx ctx, int64_t *count, int32_t reset)
    the library creates a 1-rank NCCL communicator and routes every same-rank inter-block and
    periodic ghost copy of crocco_fill_boundary / crocco_rk_stage through the multi-rank code path
    -- pack kernel -> ncclGroupStart; ncclSend + ncclRecv to itself; ncclGroupEnd -> unpack kernel
-   -- and crocco_compute_dt through ncclAllReduce(max) on that communicator.  Results are bitwise
-   those of the local copies.  Steps launch eagerly (no graphs) while a communicator exists.
+   -- and crocco_compute_dt through ncclAllReduce(max) on that communicator; on a fine AMR level
+   also every inter-level box of crocco_amr_plan (coarse mirrors filled / averaged values
+   returned through ncclSend + ncclRecv to itself).  Results are bitwise those of the local copies.  Steps launch eagerly (no graphs) while a communicator exists.
    enable = 0 destroys the communicator.  CROCCO_ERR_ARG when nranks > 1. */
 crocco_status crocco_set_nccl_loopback(crocco_ctx ctx, int32_t enable);
 /* Number of RK stages that ran overlapped (fill on the comm stream beside the ghost-free
@@ -356,6 +372,30 @@ const char *crocco_kernel_class_name(int32_t cls);
    *n_out = total count. */
 crocco_status crocco_exchange_plan(const crocco_grid_desc *desc, int32_t phase, crocco_msg *out,
                                    int32_t cap, int32_t *n_out);
+/* One inter-level box of a two-level AMR pair (crocco_amr_link; ratio 2, node-centred). */
+typedef struct {
+    int32_t kind;          /* 0 = FillPatch: coarse values to the fine block's rank (its C/F ghosts
+                              interpolate from them); 1 = AverageDown: averaged coarse values from
+                              the fine block's rank to the coarse block's rank */
+    int32_t coarse_block;  /* global id of the coarse block (the box is in its local indices) */
+    int32_t fine_block;    /* global id of the fine block the box serves */
+    int32_t src_rank, dst_rank;
+    int64_t lo[3];         /* coarse-block-local box [lo, lo+ext); kind 0 may reach into the
+                              coarse ghosts, kind 1 lies in the interior */
+    int64_t ext[3];
+} crocco_amr_msg;
+/* The inter-level plan of fine level `fine` linked at coarse node c0 to `coarse`, for rank
+   fine->rank: every box it sends or receives (src_rank or dst_rank = rank; both for boxes
+   local to the rank), kind 0 first, each kind in the canonical order both sides use for NCCL
+   matching (fine block id, then phase / side of the C/F ghost box, then coarse block id).
+   Kind 0: for each C/F ghost box of a fine block, per coarse block, the coarse nodes I and I+1
+   per direction of the corners its trilinear stencils read, I = floor((2 c0 + f)/2), with the
+   owner block of I chosen by clamping I into the domain (k_cf_interp).  Kind 1: per fine block
+   and coarse block, the covered nodes (reading 26) whose central fine node 2 (I - c0) lies in
+   the fine block.  Writes up to cap entries, *n_out = total count; CROCCO_ERR_ARG for
+   descriptors crocco_amr_link would refuse (no sibling semantics: siblings are single-rank). */
+crocco_status crocco_amr_plan(const crocco_grid_desc *fine, const crocco_grid_desc *coarse, const int64_t c0[3],
+                              crocco_amr_msg *out, int32_t cap, int32_t *n_out);
 /* Generate an ncclUniqueId (128 bytes written to out, size >= 128) on the rank
    that bootstraps the communicator; the caller broadcasts it (torch.distributed)
    and passes it as desc.nccl_unique_id on every rank. */

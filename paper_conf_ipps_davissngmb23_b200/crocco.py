@@ -63,6 +63,12 @@ class Msg(C.Structure):
                 ("src_lo", C.c_int64 * 3), ("ext", C.c_int64 * 3)]
 
 
+class AmrMsg(C.Structure):
+    _fields_ = [("kind", C.c_int32), ("coarse_block", C.c_int32), ("fine_block", C.c_int32),
+                ("src_rank", C.c_int32), ("dst_rank", C.c_int32), ("lo", C.c_int64 * 3),
+                ("ext", C.c_int64 * 3)]
+
+
 _lib = None
 
 DPP = C.POINTER(C.c_void_p)  # double *const * (array of device pointers)
@@ -91,6 +97,8 @@ _SIGS = {
                             C.POINTER(C.c_int32)],
     "crocco_exchange_plan": [C.POINTER(GridDesc), C.c_int32, C.POINTER(Msg), C.c_int32,
                              C.POINTER(C.c_int32)],
+    "crocco_amr_plan": [C.POINTER(GridDesc), C.POINTER(GridDesc), C.POINTER(C.c_int64), C.POINTER(AmrMsg),
+                        C.c_int32, C.POINTER(C.c_int32)],
     "crocco_nccl_unique_id": [C.c_void_p, C.c_int32],
     "crocco_compute_dt": [C.c_void_p, DPP, DPP, C.c_double, C.POINTER(C.c_double)],
     "crocco_rk3_step": [C.c_void_p, C.c_double, DPP, DPP, DPP, DPP, C.c_int32],
@@ -317,6 +325,16 @@ def crocco_exchange_plan(desc: GridDesc, phase: int):
     _check(lib().crocco_exchange_plan(C.byref(desc), phase, None, 0, C.byref(n)))
     arr = (Msg * max(n.value, 1))()
     _check(lib().crocco_exchange_plan(C.byref(desc), phase, arr, n.value, C.byref(n)))
+    return [arr[i] for i in range(n.value)]
+
+
+def crocco_amr_plan(fine: GridDesc, coarse: GridDesc, c0):
+    """Inter-level boxes of a two-level pair for rank fine.rank (host only, no GPU)."""
+    c = (C.c_int64 * 3)(*[int(x) for x in c0])
+    n = C.c_int32()
+    _check(lib().crocco_amr_plan(C.byref(fine), C.byref(coarse), c, None, 0, C.byref(n)))
+    arr = (AmrMsg * max(n.value, 1))()
+    _check(lib().crocco_amr_plan(C.byref(fine), C.byref(coarse), c, arr, n.value, C.byref(n)))
     return [arr[i] for i in range(n.value)]
 
 

@@ -13,6 +13,7 @@
 #include <cstdarg>
 #include <cstdio>
 #include <cstring>
+#include <functional>
 #include <string>
 #include <vector>
 
@@ -114,6 +115,14 @@ struct crocco_ctx_s {
     double *const *amr_Uc = nullptr;     // coarse state of the current two-level call only
     std::vector<crocco_ctx> sibs;        // same-level sibling patches (crocco_amr_link_sibling)
     double *const *const *amr_sibU = nullptr;  // their states for the current call only
+    // inter-level boxes touching this rank (crocco_amr_plan), the coarse-block mirrors they fill
+    // (allocated on first use) and their NCCL staging
+    std::vector<crocco_amr_msg> amr_plan;
+    std::vector<int> amr_mirror_gid;
+    std::vector<double *> amr_mirror;
+    std::vector<int> amr_cf_gids;        // coarse blocks read from mirrors by the current fill
+    double *amr_send = nullptr, *amr_recv = nullptr;
+    int64_t amr_stage_elems = 0;
     int64_t stage_elems = 0;
     // timing
     bool timing = false;
@@ -478,6 +487,9 @@ static void free_ctx(crocco_ctx c) {
     cudaFree(c->send_stage);
     cudaFree(c->dmax);
     cudaFree(c->recv_stage);
+    for (double *m : c->amr_mirror) cudaFree(m);
+    cudaFree(c->amr_send);
+    cudaFree(c->amr_recv);
     for (auto &t : c->pending) {
         cudaEventDestroy(t.e0);
         cudaEventDestroy(t.e1);
@@ -679,7 +691,7 @@ static void level_tab(const crocco_ctx_s *lv, double *const *ptr, LevelTab &t) {
     for (size_t b = 0; b < lv->loc.size(); b++) t.p[b] = ptr[b];
     for (int g = 0; g < AMR_MAX_BLOCKS; g++)
         t.g2l[g] = g < (int)lv->gid_to_local.size() ? (int16_t)lv->gid_to_local[g] : (int16_t)-1;
-    if (!lv->loc.empty()) t.L = lv->loc[0].L;  // a rank may own no block of a level
+    t.L = make_layout(lv->bn, G);  // equal blocks (also when this rank owns none of the level)
     for (int d = 0; d < 3; d++) {
         t.bn[d] = lv->bn[d];
         t.nb[d] = lv->nb[d];
@@ -706,6 +718,8 @@ static void sib_tab(const crocco_ctx_s *f, SibTab &t) {
     }
 }
 
+static crocco_status amr_fill_exchange(crocco_ctx f);  // two-level AMR section below
+static double *amr_mirror(crocco_ctx f, int gid);
 static crocco_status fill_phase(crocco_ctx c, double *const *f, int kind, int D,
                                 double *const *met, double t) {
     const bool copies_only = kind == FILL_STATE_COPIES;
@@ -730,6 +744,12 @@ static crocco_status fill_phase(crocco_ctx c, double *const *f, int kind, int D,
     }
     if (interp) {
         level_tab(c->amr_coarse, c->amr_Uc, ct);
+        // coarse blocks whose boxes came through NCCL (other rank / loopback): read the mirrors
+        int slot = (int)c->amr_coarse->loc.size();
+        for (int gid : c->amr_cf_gids) {
+            ct.p[slot] = amr_mirror(c, gid);
+            ct.g2l[gid] = (int16_t)slot++;
+        }
         cf.Lf = c->loc.empty() ? Lay{} : c->loc[0].L;
         for (int e = 0; e < 3; e++) cf.c0[e] = c->amr_c0[e];
     }
@@ -943,6 +963,8 @@ static crocco_status fill_all(crocco_ctx c, double *const *f, int32_t kind, doub
         return fail(c, CROCCO_ERR_ARG, "bad field kind");
     crocco_status st = check_ptrs(c, f, "field");
     if (st) return st;
+    // FillPatchTwoLevels: the inter-level boxes first (collective over the fine level)
+    if (kind == CROCCO_FIELD_STATE && c->amr_Uc && c->amr_coarse && (st = amr_fill_exchange(c))) return st;
     if (gather_fill_ok(c, kind)) return fill_gather(c, f);
     for (int d = 0; d < 3; d++) {
         st = fill_phase(c, f, kind, d, met, t);
@@ -1334,95 +1356,335 @@ crocco_status crocco_compute_dt(crocco_ctx c, double *const *U, double *const *M
 static int64_t floor_half_h(int64_t h) { return h >= 0 ? h / 2 : -((-h + 1) / 2); }
 
 // coarse nodes I in [lo, hi] along d of the covered set (reading 26); empty when lo > hi
-static void covered_range(const crocco_ctx_s *f, int d, int64_t &lo, int64_t &hi) {
-    const int64_t nf = f->desc.n_global[d], c0 = f->amr_c0[d];
-    if (f->desc.bc[d][0] == CROCCO_BC_PERIODIC) {
+static void covered_range_of(const crocco_grid_desc *fd, const int64_t c0[3], int d, int64_t &lo, int64_t &hi) {
+    const int64_t nf = fd->n_global[d];
+    if (fd->bc[d][0] == CROCCO_BC_PERIODIC) {
         lo = 0;
         hi = nf / 2 - 1;
     } else {
-        lo = c0 + 1;
-        hi = c0 + (nf - 2) / 2;
+        lo = c0[d] + 1;
+        hi = c0[d] + (nf - 2) / 2;
     }
+}
+static void covered_range(const crocco_ctx_s *f, int d, int64_t &lo, int64_t &hi) {
+    covered_range_of(&f->desc, f->amr_c0, d, lo, hi);
+}
+
+// geometry of a two-level pair (crocco_amr_link's checks; reading 24)
+static crocco_status amr_geom_check(crocco_ctx ec, const crocco_grid_desc *fd, const crocco_grid_desc *cd,
+                                    const int fnb[3], const int cnb[3], const int64_t c0[3]) {
+    if (fd->nranks != cd->nranks || fd->rank != cd->rank)
+        return fail(ec, CROCCO_ERR_ARG, "fine and coarse levels must share the process group");
+    if ((int64_t)fnb[0] * fnb[1] * fnb[2] > AMR_MAX_BLOCKS || (int64_t)cnb[0] * cnb[1] * cnb[2] > AMR_MAX_BLOCKS)
+        return fail(ec, CROCCO_ERR_ARG, "two-level AMR: at most %d blocks per level", AMR_MAX_BLOCKS);
+    for (int d = 0; d < 3; d++) {
+        const int64_t nf = fd->n_global[d], nc = cd->n_global[d];
+        const int *bf = fd->bc[d], *bcc = cd->bc[d];
+        if (bf[0] == CROCCO_BC_PERIODIC) {
+            if (bcc[0] != CROCCO_BC_PERIODIC || nf != 2 * nc || c0[d] != 0)
+                return fail(ec, CROCCO_ERR_ARG,
+                            "direction %d: a PERIODIC fine level must span the periodic coarse domain "
+                            "(N_f = 2 N_c, c0 = 0)", d);
+            continue;
+        }
+        if (c0[d] < 0 || 2 * c0[d] + nf - 1 > 2 * (nc - 1))
+            return fail(ec, CROCCO_ERR_ARG, "direction %d: fine level outside the coarse domain", d);
+        if (bf[0] != CROCCO_BC_COARSE_FINE && c0[d] != 0)
+            return fail(ec, CROCCO_ERR_ARG, "direction %d: a physical lo face must lie on the domain boundary", d);
+        if (bf[1] != CROCCO_BC_COARSE_FINE && 2 * c0[d] + nf - 1 != 2 * (nc - 1))
+            return fail(ec, CROCCO_ERR_ARG, "direction %d: a physical hi face must lie on the domain boundary", d);
+        if (nf < 3) return fail(ec, CROCCO_ERR_ARG, "direction %d: fine level needs >= 3 points", d);
+    }
+    return CROCCO_OK;
+}
+
+// The inter-level plan (crocco_amr_plan, include/crocco.h): every box of the pair touching rank
+// `me` (me < 0: all), kind 0 then kind 1, canonical order.
+static void build_amr_plan(const crocco_grid_desc *fd, const int fnb[3], const int fbn[3],
+                           const std::vector<BlockGeom> &fall, const crocco_grid_desc *cd, const int cnb[3],
+                           const int cbn[3], const std::vector<BlockGeom> &call, const int64_t c0[3], int me,
+                           std::vector<crocco_amr_msg> &out) {
+    out.clear();
+    auto keep = [&](const crocco_amr_msg &m) {
+        if (me < 0 || m.src_rank == me || m.dst_rank == me) out.push_back(m);
+    };
+    // kind 0: per C/F ghost box of a fine block, the coarse corners of its trilinear stencils
+    for (const BlockGeom &fb : fall)
+        for (int D = 0; D < 3; D++)
+            for (int side = 0; side < 2; side++) {
+                if (fd->bc[D][side] != CROCCO_BC_COARSE_FINE) continue;
+                if (fb.bidx[D] != (side == 0 ? 0 : fnb[D] - 1)) continue;  // not a domain face
+                int64_t Ilo[3], Ihi[3];
+                for (int e = 0; e < 3; e++) {
+                    int64_t lo, ext;  // the ghost box of phase D (build_plan)
+                    if (e == D) {
+                        lo = side == 0 ? -G : fbn[e];
+                        ext = G;
+                    } else if (e < D) {
+                        lo = -G;
+                        ext = fbn[e] + 2 * G;
+                    } else {
+                        lo = 0;
+                        ext = fbn[e];
+                    }
+                    Ilo[e] = floor_half_h(2 * c0[e] + fb.origin[e] + lo);
+                    Ihi[e] = floor_half_h(2 * c0[e] + fb.origin[e] + lo + ext - 1);
+                }
+                for (const BlockGeom &cb : call) {
+                    crocco_amr_msg m;
+                    memset(&m, 0, sizeof m);
+                    bool empty = false;
+                    for (int e = 0; e < 3; e++) {
+                        // nodes I whose clamped owner block is cb (k_cf_interp), corners I and I+1
+                        const int64_t o = cb.origin[e];
+                        const int64_t own_lo = cb.bidx[e] == 0 ? INT64_MIN / 4 : o;
+                        const int64_t own_hi = cb.bidx[e] == cnb[e] - 1 ? INT64_MAX / 4 : o + cbn[e] - 1;
+                        const int64_t a = std::max(Ilo[e], own_lo), b2 = std::min(Ihi[e], own_hi);
+                        if (a > b2) {
+                            empty = true;
+                            break;
+                        }
+                        m.lo[e] = a - o;
+                        m.ext[e] = b2 + 1 - a + 1;
+                    }
+                    if (empty) continue;
+                    m.kind = 0;
+                    m.coarse_block = cb.gid;
+                    m.fine_block = fb.gid;
+                    m.src_rank = cb.rank;
+                    m.dst_rank = fb.rank;
+                    keep(m);
+                }
+            }
+    // kind 1: covered nodes whose central fine node lies in the fine block, per coarse block
+    for (const BlockGeom &fb : fall)
+        for (const BlockGeom &cb : call) {
+            crocco_amr_msg m;
+            memset(&m, 0, sizeof m);
+            bool empty = false;
+            for (int e = 0; e < 3 && !empty; e++) {
+                int64_t lo, hi;
+                covered_range_of(fd, c0, e, lo, hi);
+                // 2 (I - c0) in [origin, origin + n - 1]
+                lo = std::max(lo, c0[e] + (fb.origin[e] + 1) / 2);
+                hi = std::min(hi, c0[e] + (fb.origin[e] + fbn[e] - 1) / 2);
+                lo = std::max<int64_t>(lo, cb.origin[e]);
+                hi = std::min<int64_t>(hi, cb.origin[e] + cbn[e] - 1);
+                empty = lo > hi;
+                m.lo[e] = lo - cb.origin[e];
+                m.ext[e] = hi - lo + 1;
+            }
+            if (empty) continue;
+            m.kind = 1;
+            m.coarse_block = cb.gid;
+            m.fine_block = fb.gid;
+            m.src_rank = fb.rank;
+            m.dst_rank = cb.rank;
+            keep(m);
+        }
+}
+
+crocco_status crocco_amr_plan(const crocco_grid_desc *fine, const crocco_grid_desc *coarse, const int64_t c0[3],
+                              crocco_amr_msg *out, int32_t cap, int32_t *n_out) {
+    int fnb[3], fbn[3], cnb[3], cbn[3];
+    crocco_status st = validate(fine, fnb, fbn);
+    if (!st) st = validate(coarse, cnb, cbn);
+    if (st) return st;
+    if (!c0) return fail(nullptr, CROCCO_ERR_ARG, "null c0");
+    if ((st = amr_geom_check(nullptr, fine, coarse, fnb, cnb, c0))) return st;
+    std::vector<BlockGeom> fall, call;
+    build_blocks(fine, fnb, fbn, fall);
+    build_blocks(coarse, cnb, cbn, call);
+    std::vector<crocco_amr_msg> plan;
+    build_amr_plan(fine, fnb, fbn, fall, coarse, cnb, cbn, call, c0, fine->rank, plan);
+    if (n_out) *n_out = (int32_t)plan.size();
+    for (int i = 0; i < (int)plan.size() && i < cap; i++) out[i] = plan[i];
+    return CROCCO_OK;
+}
+
+static void amr_release(crocco_ctx f) {
+    for (double *m : f->amr_mirror) cudaFree(m);
+    f->amr_mirror.clear();
+    f->amr_mirror_gid.clear();
+    cudaFree(f->amr_send);
+    cudaFree(f->amr_recv);
+    f->amr_send = f->amr_recv = nullptr;
+    f->amr_stage_elems = 0;
+    f->amr_plan.clear();
 }
 
 crocco_status crocco_amr_link(crocco_ctx f, crocco_ctx c, const int64_t c0[3]) {
     LIVE(f);
     LIVE(c);
     if (!c0 || f == c) return fail(f, CROCCO_ERR_ARG, "need distinct fine / coarse ctx and c0");
-    if (f->desc.nranks != c->desc.nranks || f->desc.rank != c->desc.rank)
-        return fail(f, CROCCO_ERR_ARG, "fine and coarse levels must share the process group");
-    if (f->loc.size() > AMR_MAX_LOCAL || c->loc.size() > AMR_MAX_LOCAL || f->all.size() > AMR_MAX_BLOCKS ||
-        c->all.size() > AMR_MAX_BLOCKS)
-        return fail(f, CROCCO_ERR_ARG, "two-level AMR: at most %d local / %d blocks per level", AMR_MAX_LOCAL,
-                    AMR_MAX_BLOCKS);
-    for (int d = 0; d < 3; d++) {
-        const int64_t nf = f->desc.n_global[d], nc = c->desc.n_global[d];
-        const int *bf = f->desc.bc[d], *bcc = c->desc.bc[d];
-        if (bf[0] == CROCCO_BC_PERIODIC) {
-            if (bcc[0] != CROCCO_BC_PERIODIC || nf != 2 * nc || c0[d] != 0)
-                return fail(f, CROCCO_ERR_ARG,
-                            "direction %d: a PERIODIC fine level must span the periodic coarse domain "
-                            "(N_f = 2 N_c, c0 = 0)", d);
-            continue;
-        }
-        if (c0[d] < 0 || 2 * c0[d] + nf - 1 > 2 * (nc - 1))
-            return fail(f, CROCCO_ERR_ARG, "direction %d: fine level outside the coarse domain", d);
-        if (bf[0] != CROCCO_BC_COARSE_FINE && c0[d] != 0)
-            return fail(f, CROCCO_ERR_ARG, "direction %d: a physical lo face must lie on the domain boundary", d);
-        if (bf[1] != CROCCO_BC_COARSE_FINE && 2 * c0[d] + nf - 1 != 2 * (nc - 1))
-            return fail(f, CROCCO_ERR_ARG, "direction %d: a physical hi face must lie on the domain boundary", d);
-        if (nf < 3) return fail(f, CROCCO_ERR_ARG, "direction %d: fine level needs >= 3 points", d);
-    }
-    int64_t c0_prev[3];
-    for (int d = 0; d < 3; d++) {
-        c0_prev[d] = f->amr_c0[d];
-        f->amr_c0[d] = c0[d];  // covered_range() reads it; restored below on failure
-    }
-    crocco_status st = CROCCO_OK;
-    // locality: every coarse block a fine ghost interpolates from, and every fine block a
-    // covered coarse node averages, lives on this rank (no inter-level communication)
-    for (const LocalBlock &b : f->loc) {
-        int64_t lo[3], hi[3];
-        for (int d = 0; d < 3; d++) {
-            lo[d] = floor_half_h(2 * c0[d] + b.g.origin[d] - G);
-            hi[d] = floor_half_h(2 * c0[d] + b.g.origin[d] + b.g.n[d] + G - 1);
-            lo[d] = std::min<int64_t>(std::max<int64_t>(lo[d], 0), c->desc.n_global[d] - 1) / c->bn[d];
-            hi[d] = std::min<int64_t>(std::max<int64_t>(hi[d], 0), c->desc.n_global[d] - 1) / c->bn[d];
-        }
-        for (int64_t z = lo[2]; z <= hi[2]; z++)
-            for (int64_t y = lo[1]; y <= hi[1]; y++)
-                for (int64_t x = lo[0]; x <= hi[0]; x++)
-                    if (st == CROCCO_OK && c->gid_to_local[x + c->nb[0] * (y + c->nb[1] * z)] < 0)
-                        st = fail(f, CROCCO_ERR_ARG,
-                                  "fine block %d interpolates from a coarse block on another rank", b.g.gid);
-    }
-    for (const LocalBlock &b : c->loc) {
-        int64_t lo[3], hi[3];
-        bool empty = false;
-        for (int d = 0; d < 3; d++) {
-            covered_range(f, d, lo[d], hi[d]);
-            lo[d] = std::max<int64_t>(lo[d], b.g.origin[d]);
-            hi[d] = std::min<int64_t>(hi[d], b.g.origin[d] + b.g.n[d] - 1);
-            empty = empty || lo[d] > hi[d];
-            if (!empty) {
-                lo[d] = 2 * (lo[d] - c0[d]) / f->bn[d];
-                hi[d] = 2 * (hi[d] - c0[d]) / f->bn[d];
-            }
-        }
-        if (empty) continue;
-        for (int64_t z = lo[2]; z <= hi[2]; z++)
-            for (int64_t y = lo[1]; y <= hi[1]; y++)
-                for (int64_t x = lo[0]; x <= hi[0]; x++)
-                    if (st == CROCCO_OK && f->gid_to_local[x + f->nb[0] * (y + f->nb[1] * z)] < 0)
-                        st = fail(f, CROCCO_ERR_ARG,
-                                  "coarse block %d averages down from a fine block on another rank", b.g.gid);
-    }
-    if (st != CROCCO_OK) {
-        for (int d = 0; d < 3; d++) f->amr_c0[d] = c0_prev[d];
-        return st;
-    }
+    crocco_status st = amr_geom_check(f, &f->desc, &c->desc, f->nb, c->nb, c0);
+    if (st) return st;
+    if (f->loc.size() > (size_t)AMR_MAX_LOCAL)
+        return fail(f, CROCCO_ERR_ARG, "two-level AMR: at most %d local fine blocks", AMR_MAX_LOCAL);
+    std::vector<crocco_amr_msg> plan;
+    build_amr_plan(&f->desc, f->nb, f->bn, f->all, &c->desc, c->nb, c->bn, c->all, c0, f->desc.rank, plan);
+    // slots of the coarse-level table: the local coarse blocks plus the mirrors this rank may use
+    std::vector<int> mg;
+    for (const crocco_amr_msg &m : plan)
+        if ((m.kind == 0 && m.dst_rank == f->desc.rank) || (m.kind == 1 && m.src_rank == f->desc.rank))
+            if (std::find(mg.begin(), mg.end(), m.coarse_block) == mg.end()) mg.push_back(m.coarse_block);
+    if (c->loc.size() + mg.size() > (size_t)AMR_MAX_LOCAL)
+        return fail(f, CROCCO_ERR_ARG, "two-level AMR: %zu local coarse blocks + %zu mirrors > %d", c->loc.size(),
+                    mg.size(), AMR_MAX_LOCAL);
+    for (const crocco_amr_msg &m : plan)
+        if (m.src_rank != m.dst_rank && !f->comm)
+            return fail(f, CROCCO_ERR_ARG, "inter-rank AMR boxes need the fine level's communicator");
+    amr_release(f);
+    f->amr_plan = std::move(plan);
+    for (int d = 0; d < 3; d++) f->amr_c0[d] = c0[d];
     f->amr_coarse = c;
     return CROCCO_OK;
+}
+
+// a box of the plan goes through ncclSend / ncclRecv (other rank, or loopback)
+static bool amr_routed(const crocco_ctx_s *f, const crocco_amr_msg &m) {
+    return m.src_rank != m.dst_rank || f->loopback;
+}
+
+// mirror of coarse block gid (coarse block layout, 5 comps), allocated zeroed on first use
+static double *amr_mirror(crocco_ctx f, int gid) {
+    for (size_t i = 0; i < f->amr_mirror_gid.size(); i++)
+        if (f->amr_mirror_gid[i] == gid) return f->amr_mirror[i];
+    const crocco_ctx_s *c = f->amr_coarse;
+    const Lay L = make_layout(c->bn, G);
+    double *p = nullptr;
+    if (cudaMalloc((void **)&p, (size_t)(5 * L.cs) * sizeof(double)) != cudaSuccess ||
+        cudaMemset(p, 0, (size_t)(5 * L.cs) * sizeof(double)) != cudaSuccess) {
+        cudaGetLastError();
+        cudaFree(p);
+        return nullptr;
+    }
+    f->scratch += 5 * L.cs * (int64_t)sizeof(double);
+    f->amr_mirror_gid.push_back(gid);
+    f->amr_mirror.push_back(p);
+    return p;
+}
+
+// box [lo, lo+ext) of a 5-component array in layout L <-> a contiguous staging slice
+static BoxOp amr_box_op(double *arr, const Lay &L, const crocco_amr_msg &m, double *stage, bool pack) {
+    BoxOp o;
+    memset(&o, 0, sizeof o);
+    const int64_t vol = m.ext[0] * m.ext[1] * m.ext[2];
+    int64_t st[3];
+    op_strides(L, st);
+    const int64_t base = at(L, (int)m.lo[0], (int)m.lo[1], (int)m.lo[2]);
+    const int64_t cst[3] = {1, m.ext[0], m.ext[0] * m.ext[1]};
+    if (pack) {
+        o.src = arr;
+        for (int e = 0; e < 3; e++) o.sst[e] = st[e];
+        o.scs = L.cs;
+        o.sbase = base;
+        o.dst = stage;
+        for (int e = 0; e < 3; e++) o.dst_[e] = cst[e];
+        o.dcs = vol;
+        o.dbase = 0;
+    } else {
+        o.src = stage;
+        for (int e = 0; e < 3; e++) o.sst[e] = cst[e];
+        o.scs = vol;
+        o.sbase = 0;
+        o.dst = arr;
+        for (int e = 0; e < 3; e++) o.dst_[e] = st[e];
+        o.dcs = L.cs;
+        o.dbase = base;
+    }
+    for (int e = 0; e < 3; e++) o.ext[e] = (int)m.ext[e];
+    o.ncomp = 5;
+    o.mode = BOX_COPY;
+    return o;
+}
+
+// The routed boxes of one kind: pack (src arrays) -> grouped ncclSend / ncclRecv -> unpack (dst
+// arrays).  src_arr / dst_arr give the array of a box on the sending / receiving side.
+typedef std::function<double *(const crocco_amr_msg &)> AmrArr;
+static crocco_status amr_exchange(crocco_ctx f, int kind, const AmrArr &src_arr, const AmrArr &dst_arr) {
+    const int me = f->desc.rank;
+    std::vector<const crocco_amr_msg *> r;
+    int64_t ns = 0, nr = 0;
+    for (const crocco_amr_msg &m : f->amr_plan)
+        if (m.kind == kind && amr_routed(f, m)) {
+            r.push_back(&m);
+            const int64_t v = 5 * m.ext[0] * m.ext[1] * m.ext[2];
+            if (m.src_rank == me) ns += v;
+            if (m.dst_rank == me) nr += v;
+        }
+    if (r.empty()) return CROCCO_OK;
+    if (!f->comm) return fail(f, CROCCO_ERR_STATE, "inter-level boxes without communicator");
+    const int64_t need = std::max(ns, nr);
+    if (need > f->amr_stage_elems) {
+        cudaStreamSynchronize(f->stream);  // the old staging may still be read
+        cudaFree(f->amr_send);
+        cudaFree(f->amr_recv);
+        f->amr_send = f->amr_recv = nullptr;
+        if (cudaMalloc((void **)&f->amr_send, (size_t)need * sizeof(double)) != cudaSuccess ||
+            cudaMalloc((void **)&f->amr_recv, (size_t)need * sizeof(double)) != cudaSuccess) {
+            cudaGetLastError();
+            f->amr_stage_elems = 0;
+            return fail(f, CROCCO_ERR_NOMEM, "AMR staging allocation failed");
+        }
+        f->scratch += 2 * (need - f->amr_stage_elems) * (int64_t)sizeof(double);
+        f->amr_stage_elems = need;
+    }
+    const Lay Lc = make_layout(f->amr_coarse->bn, G);
+    BoxOps ops;
+    ops.nops = 0;
+    crocco_status st;
+    std::vector<int64_t> so(r.size()), ro(r.size());
+    int64_t s = 0, q = 0;
+    for (size_t i = 0; i < r.size(); i++) {
+        const int64_t v = 5 * r[i]->ext[0] * r[i]->ext[1] * r[i]->ext[2];
+        if (r[i]->dst_rank == me) {
+            ro[i] = q;
+            q += v;
+        }
+        if (r[i]->src_rank != me) continue;
+        so[i] = s;
+        double *a = src_arr(*r[i]);
+        if (!a) return fail(f, CROCCO_ERR_NOMEM, "AMR mirror allocation failed");
+        if ((st = push_op(f, ops, amr_box_op(a, Lc, *r[i], f->amr_send + s, true)))) return st;
+        s += v;
+    }
+    if ((st = flush_ops(f, ops))) return st;
+    {
+        NvtxRange nv("crocco:nccl_amr");
+        NK(f, ncclGroupStart());
+        for (size_t i = 0; i < r.size(); i++) {
+            const size_t cnt = (size_t)(5 * r[i]->ext[0] * r[i]->ext[1] * r[i]->ext[2]);
+            if (r[i]->src_rank == me)
+                NK(f, ncclSend(f->amr_send + so[i], cnt, ncclDouble, r[i]->dst_rank, f->comm, f->stream));
+            if (r[i]->dst_rank == me)
+                NK(f, ncclRecv(f->amr_recv + ro[i], cnt, ncclDouble, r[i]->src_rank, f->comm, f->stream));
+        }
+        NK(f, ncclGroupEnd());
+    }
+    for (size_t i = 0; i < r.size(); i++) {
+        if (r[i]->dst_rank != me) continue;
+        double *a = dst_arr(*r[i]);
+        if (!a) return fail(f, CROCCO_ERR_NOMEM, "AMR mirror allocation failed");
+        if ((st = push_op(f, ops, amr_box_op(a, Lc, *r[i], f->amr_recv + ro[i], false)))) return st;
+    }
+    return flush_ops(f, ops);
+}
+
+// FillPatch, inter-level part: the coarse boxes the C/F interpolation of this rank's fine blocks
+// reads from other ranks (or through the loopback) land in the coarse-block mirrors;
+// fill_phase then maps those coarse blocks to their mirrors (amr_cf_gids).
+static crocco_status amr_fill_exchange(crocco_ctx f) {
+    f->amr_cf_gids.clear();
+    const crocco_ctx_s *c = f->amr_coarse;
+    for (const crocco_amr_msg &m : f->amr_plan)
+        if (m.kind == 0 && m.dst_rank == f->desc.rank && amr_routed(f, m) &&
+            std::find(f->amr_cf_gids.begin(), f->amr_cf_gids.end(), m.coarse_block) == f->amr_cf_gids.end())
+            f->amr_cf_gids.push_back(m.coarse_block);
+    double *const *Uc = f->amr_Uc;
+    return amr_exchange(
+        f, 0, [&](const crocco_amr_msg &m) { return Uc[c->gid_to_local[m.coarse_block]]; },
+        [&](const crocco_amr_msg &m) { return amr_mirror(f, m.coarse_block); });
 }
 
 static crocco_status amr_ready(crocco_ctx f, double *const *Uc) {
@@ -1472,7 +1734,7 @@ crocco_status crocco_average_down(crocco_ctx f, double *const *Uf, double *const
     sib_tab(f, sb);
     ADOps ops;
     memset(&ops, 0, sizeof ops);
-    ops.Lc = c->loc.empty() ? Lay{} : c->loc[0].L;
+    ops.Lc = make_layout(c->bn, G);
     for (int d = 0; d < 3; d++) {
         ops.c0[d] = f->amr_c0[d];
         ops.Nf[d] = f->desc.n_global[d];
@@ -1487,32 +1749,57 @@ crocco_status crocco_average_down(crocco_ctx f, double *const *Uf, double *const
         mx = 0;
         return CROCCO_OK;
     };
-    for (size_t bi = 0; bi < c->loc.size(); bi++) {
-        const LocalBlock &b = c->loc[bi];
-        int64_t lo[3], hi[3];
-        bool empty = false;
-        for (int d = 0; d < 3; d++) {
-            covered_range(f, d, lo[d], hi[d]);
-            if (sb.n > 0 && f->desc.bc[d][0] != CROCCO_BC_PERIODIC) {  // nodes whose central fine node
-                lo[d] = f->amr_c0[d];                                   // is ours; k_average_down
-                hi[d] = f->amr_c0[d] + (f->desc.n_global[d] - 1) / 2;    // checks the 27 nodes
-            }
-            lo[d] = std::max<int64_t>(lo[d], b.g.origin[d]);
-            hi[d] = std::min<int64_t>(hi[d], b.g.origin[d] + b.g.n[d] - 1);
-            empty = empty || lo[d] > hi[d];
-        }
-        if (empty) continue;
+    auto push = [&](double *dst, const Lay &Lb, const int64_t org[3], const int64_t lo[3],
+                    const int64_t hi[3]) -> crocco_status {
         ADOp &o = ops.op[ops.nops++];
-        o.dst = Uc[bi];
-        o.dbase = at(b.L, (int)(lo[0] - b.g.origin[0]), (int)(lo[1] - b.g.origin[1]), (int)(lo[2] - b.g.origin[2]));
+        o.dst = dst;
+        o.dbase = at(Lb, (int)(lo[0] - org[0]), (int)(lo[1] - org[1]), (int)(lo[2] - org[2]));
         for (int d = 0; d < 3; d++) {
             o.ext[d] = (int)(hi[d] - lo[d] + 1);
             o.Io[d] = lo[d];
         }
         mx = std::max<int64_t>(mx, (int64_t)o.ext[0] * o.ext[1] * o.ext[2]);
-        if (ops.nops == CF_MAX_OPS && (st = flush())) return st;
+        return ops.nops == CF_MAX_OPS ? flush() : CROCCO_OK;
+    };
+    if (sb.n > 0) {
+        // siblings (single-rank, reading 31): per local coarse block the nodes whose central fine
+        // node is ours; k_average_down checks their 27 nodes
+        for (size_t bi = 0; bi < c->loc.size(); bi++) {
+            const LocalBlock &b = c->loc[bi];
+            int64_t lo[3], hi[3];
+            bool empty = false;
+            for (int d = 0; d < 3; d++) {
+                covered_range(f, d, lo[d], hi[d]);
+                if (f->desc.bc[d][0] != CROCCO_BC_PERIODIC) {
+                    lo[d] = f->amr_c0[d];
+                    hi[d] = f->amr_c0[d] + (f->desc.n_global[d] - 1) / 2;
+                }
+                lo[d] = std::max<int64_t>(lo[d], b.g.origin[d]);
+                hi[d] = std::min<int64_t>(hi[d], b.g.origin[d] + b.g.n[d] - 1);
+                empty = empty || lo[d] > hi[d];
+            }
+            if (!empty && (st = push(Uc[bi], b.L, b.g.origin, lo, hi))) return st;
+        }
+        return flush();
     }
-    return flush();
+    // the plan's kind-1 boxes computed on this rank: in place when the coarse block is ours,
+    // else (or under the loopback) into its mirror, then sent to the coarse block's rank
+    for (const crocco_amr_msg &m : f->amr_plan) {
+        if (m.kind != 1 || m.src_rank != f->desc.rank) continue;
+        const BlockGeom &cb = c->all[m.coarse_block];
+        double *dst = amr_routed(f, m) ? amr_mirror(f, m.coarse_block) : Uc[c->gid_to_local[m.coarse_block]];
+        if (!dst) return fail(f, CROCCO_ERR_NOMEM, "AMR mirror allocation failed");
+        int64_t lo[3], hi[3];
+        for (int d = 0; d < 3; d++) {
+            lo[d] = cb.origin[d] + m.lo[d];
+            hi[d] = lo[d] + m.ext[d] - 1;
+        }
+        if ((st = push(dst, ops.Lc, cb.origin, lo, hi))) return st;
+    }
+    if ((st = flush())) return st;
+    return amr_exchange(
+        f, 1, [&](const crocco_amr_msg &m) { return amr_mirror(f, m.coarse_block); },
+        [&](const crocco_amr_msg &m) { return Uc[c->gid_to_local[m.coarse_block]]; });
 }
 
 crocco_status crocco_amr_link_sibling(crocco_ctx f, crocco_ctx g) {

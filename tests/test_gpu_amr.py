@@ -438,6 +438,38 @@ def test_two_level_overlapped_stage_equals_serial_bitwise():
     assert np.array_equal(outs[0][0], outs[1][0]) and np.array_equal(outs[0][1], outs[1][1])
 
 
+@pytest.mark.parametrize("nbc,nbf,c0,nf,bcf", [
+    ((1, 1, 1), (1, 1, 1), (5, 6, 3), (24, 20, 16), ((CF, CF),) * 3),
+    ((2, 2, 1), (2, 1, 2), (5, 6, 3), (24, 20, 16), ((CF, CF),) * 3),
+    ((2, 1, 2), (2, 2, 1), (0, 4, 3), (48, 20, 16), ((0, 0), (CF, CF), (CF, CF)))])
+def test_inter_level_boxes_through_nccl_loopback_bitwise(nbc, nbf, c0, nf, bcf):
+    """Multi-rank AMR on one GPU (each level decomposed on its own; include/
+    crocco.h crocco_amr_plan): with the NCCL loopback on the fine ctx every inter-level box --
+    the coarse corners of the C/F interpolation into the coarse-block mirrors, the averaged
+    coarse nodes back from the mirrors -- goes pack -> ncclSend/ncclRecv -> unpack, the code a
+    fine block on another rank than its coarse footprint runs.  3 RK3 steps are bitwise those of
+    the in-place path, which the oracle pins (test_two_level_rk3_parity)."""
+    from paper_conf_ipps_davissngmb23_b200 import crocco as cc
+    nc = (24, 24, 16)
+    outs = []
+    for lb in (0, 1):
+        h = Hier(nc, c0, nf, bcf, synth.Wavy3D(L=(10.0,) * 3, N=nc), dict(terms=3, mu_ref=0.01), state="random")
+        C, F, A = h.gpu(nbc, nbf)
+        if lb:
+            cc.crocco_set_nccl_loopback(F.ctx, 1)
+        s0 = cc.crocco_scratch_bytes(F.ctx)
+        A.step(0.01, 3)
+        A.sync()
+        if lb:   # the coarse-block mirrors and the AMR staging were allocated by the exchange
+            assert cc.crocco_scratch_bytes(F.ctx) > s0
+        outs.append([C.get(C.U), F.get(F.U)])
+        C.close()
+        F.close()
+    for a, b in zip(outs[0], outs[1]):
+        for x, y in zip(a, b):
+            assert np.array_equal(x, y)
+
+
 def test_amr_abi_refusals():
     from paper_conf_ipps_davissngmb23_b200 import crocco as cc
     from paper_conf_ipps_davissngmb23_b200.solver import AmrSolver, Solver
