@@ -267,7 +267,7 @@ crocco_status crocco_compute_dt(crocco_ctx ctx, double *const *U, double *const 
    ncclSend/ncclRecv to self under crocco_set_nccl_loopback on the FINE ctx).  So the two-level
    calls are collective over the fine ctx's communicator: every rank calls them, also a rank
    that owns no fine block (it may still own coarse blocks that others read).
-   Several patches of one level: see the sibling calls below (single-rank). */
+   Several patches of one level: see the sibling calls below. */
 
 /* Declare `fine` a refinement of `coarse` with fine node 0 at coarse node c0[3].  Checks:
    per direction either the fine level is PERIODIC and spans the periodic coarse domain
@@ -298,8 +298,11 @@ crocco_status crocco_average_down(crocco_ctx fine, double *const *U_fine, double
 /* ---- same-level sibling patches (NEXT-4 completion; a level is a union of
    patches, FillPatchSingleLevel -> FillBoundary exchanges their ghosts; reading 31) ---
    Declare two fine patches of the same level (both crocco_amr_link'ed to the same coarse ctx,
-   interiors disjoint, even fine offset 2 (c0_g - c0_f), single-rank) siblings of each other;
-   symmetric, idempotent; <= 8 siblings / 16 sibling blocks per patch; CROCCO_ERR_ARG otherwise.
+   interiors disjoint, even fine offset 2 (c0_g - c0_f), the same ranks) siblings of each other;
+   symmetric, idempotent; <= 8 siblings / 16 sibling blocks (all ranks) per patch; CROCCO_ERR_ARG
+   otherwise.  Sibling blocks on other ranks (or all of them under the loopback) reach the patch
+   as kind-2 boxes of its plan (crocco_amr_sibling_plan) through NCCL p2p into sibling-block
+   mirrors, so the _level calls are collective over the patch's communicator.
    With siblings, the _level calls below replace the two-level calls; `sib` holds, for each
    sibling in link order, the pointer array of its local blocks (caller-owned, device):
    - C/F ghosts lying inside a sibling's interior take the sibling's value (the stage INPUT of
@@ -376,12 +379,16 @@ crocco_status crocco_exchange_plan(const crocco_grid_desc *desc, int32_t phase, 
 typedef struct {
     int32_t kind;          /* 0 = FillPatch: coarse values to the fine block's rank (its C/F ghosts
                               interpolate from them); 1 = AverageDown: averaged coarse values from
-                              the fine block's rank to the coarse block's rank */
+                              the fine block's rank to the coarse block's rank; 2 = sibling ghosts:
+                              interior values of a same-level sibling block to the fine block's
+                              rank (its C/F ghosts inside the sibling copy them) */
     int32_t coarse_block;  /* global id of the coarse block (the box is in its local indices) */
     int32_t fine_block;    /* global id of the fine block the box serves */
+    int32_t sibling;       /* kind 2: index of the sibling patch in link order; -1 otherwise */
     int32_t src_rank, dst_rank;
     int64_t lo[3];         /* coarse-block-local box [lo, lo+ext); kind 0 may reach into the
-                              coarse ghosts, kind 1 lies in the interior */
+                              coarse ghosts, kind 1 lies in the interior; kind 2: box of the
+                              sibling block (coarse_block = its global id in the sibling patch) */
     int64_t ext[3];
 } crocco_amr_msg;
 /* The inter-level plan of fine level `fine` linked at coarse node c0 to `coarse`, for rank
@@ -396,6 +403,15 @@ typedef struct {
    descriptors crocco_amr_link would refuse (no sibling semantics: siblings are single-rank). */
 crocco_status crocco_amr_plan(const crocco_grid_desc *fine, const crocco_grid_desc *coarse, const int64_t c0[3],
                               crocco_amr_msg *out, int32_t cap, int32_t *n_out);
+/* Kind-2 boxes (sibling index `sibling`) of fine patch `fine` at coarse node c0 with its sibling
+   patch `sib` at coarse node c0s, for rank fine->rank: per fine block (id order), per C/F ghost
+   box (phase, side), per sibling block (id order), the part of the ghost box inside the sibling
+   block's interior, in the sibling block's local indices.  crocco_amr_link_sibling adds these to
+   both patches' plans (and then computes the kind-1 boxes over the nodes whose central fine node
+   is the patch's, which k_average_down filters by the 27-node rule).  Host only. */
+crocco_status crocco_amr_sibling_plan(const crocco_grid_desc *fine, const int64_t c0[3], const crocco_grid_desc *sib,
+                                      const int64_t c0s[3], int32_t sibling, crocco_amr_msg *out, int32_t cap,
+                                      int32_t *n_out);
 /* Generate an ncclUniqueId (128 bytes written to out, size >= 128) on the rank
    that bootstraps the communicator; the caller broadcasts it (torch.distributed)
    and passes it as desc.nccl_unique_id on every rank. */

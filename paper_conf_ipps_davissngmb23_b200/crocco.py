@@ -65,7 +65,7 @@ class Msg(C.Structure):
 
 class AmrMsg(C.Structure):
     _fields_ = [("kind", C.c_int32), ("coarse_block", C.c_int32), ("fine_block", C.c_int32),
-                ("src_rank", C.c_int32), ("dst_rank", C.c_int32), ("lo", C.c_int64 * 3),
+                ("sibling", C.c_int32), ("src_rank", C.c_int32), ("dst_rank", C.c_int32), ("lo", C.c_int64 * 3),
                 ("ext", C.c_int64 * 3)]
 
 
@@ -99,6 +99,9 @@ _SIGS = {
                              C.POINTER(C.c_int32)],
     "crocco_amr_plan": [C.POINTER(GridDesc), C.POINTER(GridDesc), C.POINTER(C.c_int64), C.POINTER(AmrMsg),
                         C.c_int32, C.POINTER(C.c_int32)],
+    "crocco_amr_sibling_plan": [C.POINTER(GridDesc), C.POINTER(C.c_int64), C.POINTER(GridDesc),
+                                C.POINTER(C.c_int64), C.c_int32, C.POINTER(AmrMsg), C.c_int32,
+                                C.POINTER(C.c_int32)],
     "crocco_nccl_unique_id": [C.c_void_p, C.c_int32],
     "crocco_compute_dt": [C.c_void_p, DPP, DPP, C.c_double, C.POINTER(C.c_double)],
     "crocco_rk3_step": [C.c_void_p, C.c_double, DPP, DPP, DPP, DPP, C.c_int32],
@@ -335,6 +338,17 @@ def crocco_amr_plan(fine: GridDesc, coarse: GridDesc, c0):
     _check(lib().crocco_amr_plan(C.byref(fine), C.byref(coarse), c, None, 0, C.byref(n)))
     arr = (AmrMsg * max(n.value, 1))()
     _check(lib().crocco_amr_plan(C.byref(fine), C.byref(coarse), c, arr, n.value, C.byref(n)))
+    return [arr[i] for i in range(n.value)]
+
+
+def crocco_amr_sibling_plan(fine: GridDesc, c0, sib: GridDesc, c0s, sibling=0):
+    """Kind-2 (sibling ghost) boxes of patch `fine` from sibling patch `sib` (host only)."""
+    a = (C.c_int64 * 3)(*[int(x) for x in c0])
+    b = (C.c_int64 * 3)(*[int(x) for x in c0s])
+    n = C.c_int32()
+    _check(lib().crocco_amr_sibling_plan(C.byref(fine), a, C.byref(sib), b, sibling, None, 0, C.byref(n)))
+    arr = (AmrMsg * max(n.value, 1))()
+    _check(lib().crocco_amr_sibling_plan(C.byref(fine), a, C.byref(sib), b, sibling, arr, n.value, C.byref(n)))
     return [arr[i] for i in range(n.value)]
 
 

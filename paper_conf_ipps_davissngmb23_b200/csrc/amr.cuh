@@ -133,6 +133,8 @@ struct ADOp {
     int64_t dbase;   // element of the box origin
     int ext[3];
     int64_t Io[3];   // coarse global index of the box origin
+    const double *buf;  // non-null: averages received from the fine block's rank (box order, 5
+                        // comps) -- the covered nodes of the box take them (the others keep dst)
 };
 struct ADOps {
     ADOp op[CF_MAX_OPS];
@@ -181,9 +183,14 @@ __global__ void __launch_bounds__(256) k_average_down(const __grid_constant__ AD
             fc[d] = f - (int64_t)bx[d] * ft.bn[d];
         }
         if (!ad_covered(ops, sb, fg)) continue;
+        const int64_t dp = o.dbase + a + b * ops.Lc.py + c * ops.Lc.pz;
+        if (o.buf) {
+#pragma unroll
+            for (int q = 0; q < 5; q++) o.dst[q * ops.Lc.cs + dp] = o.buf[q * tot + t];
+            continue;
+        }
         const double *src = ft.p[ft.g2l[bx[0] + ft.nb[0] * (bx[1] + ft.nb[1] * bx[2])]];
         const int64_t pc = at(Lf, (int)fc[0], (int)fc[1], (int)fc[2]);
-        const int64_t dp = o.dbase + a + b * ops.Lc.py + c * ops.Lc.pz;
 #pragma unroll
         for (int q = 0; q < 5; q++) {
             const double *s = src + q * Lf.cs + pc;

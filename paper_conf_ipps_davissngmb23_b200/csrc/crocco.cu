@@ -121,6 +121,8 @@ struct crocco_ctx_s {
     std::vector<int> amr_mirror_gid;
     std::vector<double *> amr_mirror;
     std::vector<int> amr_cf_gids;        // coarse blocks read from mirrors by the current fill
+    std::vector<int> amr_smirror_key;    // sibling-block mirrors: key sibling * AMR_MAX_BLOCKS + gid
+    std::vector<double *> amr_smirror;
     double *amr_send = nullptr, *amr_recv = nullptr;
     int64_t amr_stage_elems = 0;
     int64_t stage_elems = 0;
@@ -488,6 +490,7 @@ static void free_ctx(crocco_ctx c) {
     cudaFree(c->dmax);
     cudaFree(c->recv_stage);
     for (double *m : c->amr_mirror) cudaFree(m);
+    for (double *m : c->amr_smirror) cudaFree(m);
     cudaFree(c->amr_send);
     cudaFree(c->amr_recv);
     for (auto &t : c->pending) {
@@ -699,27 +702,33 @@ static void level_tab(const crocco_ctx_s *lv, double *const *ptr, LevelTab &t) {
     }
 }
 
+static crocco_status amr_fill_exchange(crocco_ctx f);  // two-level AMR section below
+static crocco_status amr_sib_exchange(crocco_ctx f);
+static double *amr_mirror(crocco_ctx f, int gid);
+static double *amr_sib_mirror_if(crocco_ctx f, int s, int gid);
 // the blocks of f's same-level siblings in f's fine index space, with the states of this call
-static void sib_tab(const crocco_ctx_s *f, SibTab &t) {
+// (every block of every sibling, on any rank: the geometry decides which ghost points copy and
+// which coarse nodes are covered; the data of a block on another rank -- or of every block under
+// the loopback -- is read from its mirror, filled by the kind-2 boxes of amr_sib_exchange)
+static void sib_tab(crocco_ctx f, SibTab &t) {
     memset(&t, 0, sizeof t);
     if (!f->amr_sibU) return;
     for (size_t s = 0; s < f->sibs.size(); s++) {
         const crocco_ctx_s *g = f->sibs[s];
-        for (size_t b = 0; b < g->loc.size() && t.n < SIB_MAX_BLOCKS; b++) {
-            const LocalBlock &lb = g->loc[b];
+        for (size_t b = 0; b < g->all.size() && t.n < SIB_MAX_BLOCKS; b++) {
+            const BlockGeom &bg = g->all[b];
             for (int d = 0; d < 3; d++) {
-                t.lo[t.n][d] = 2 * (g->amr_c0[d] - f->amr_c0[d]) + lb.g.origin[d];
-                t.hi[t.n][d] = t.lo[t.n][d] + lb.g.n[d];
+                t.lo[t.n][d] = 2 * (g->amr_c0[d] - f->amr_c0[d]) + bg.origin[d];
+                t.hi[t.n][d] = t.lo[t.n][d] + bg.n[d];
             }
-            t.p[t.n] = f->amr_sibU[s][b];
-            t.L[t.n] = lb.L;
+            const int l = g->gid_to_local[bg.gid];
+            t.p[t.n] = (l >= 0 && !f->loopback) ? f->amr_sibU[s][l] : amr_sib_mirror_if(f, (int)s, bg.gid);
+            t.L[t.n] = make_layout(bg.n, G);
             t.n++;
         }
     }
 }
 
-static crocco_status amr_fill_exchange(crocco_ctx f);  // two-level AMR section below
-static double *amr_mirror(crocco_ctx f, int gid);
 static crocco_status fill_phase(crocco_ctx c, double *const *f, int kind, int D,
                                 double *const *met, double t) {
     const bool copies_only = kind == FILL_STATE_COPIES;
@@ -965,6 +974,9 @@ static crocco_status fill_all(crocco_ctx c, double *const *f, int32_t kind, doub
     if (st) return st;
     // FillPatchTwoLevels: the inter-level boxes first (collective over the fine level)
     if (kind == CROCCO_FIELD_STATE && c->amr_Uc && c->amr_coarse && (st = amr_fill_exchange(c))) return st;
+    if (((kind == CROCCO_FIELD_STATE && c->amr_Uc) || kind == FILL_STATE_COPIES) && c->amr_sibU && !c->sibs.empty() &&
+        (st = amr_sib_exchange(c)))
+        return st;
     if (gather_fill_ok(c, kind)) return fill_gather(c, f);
     for (int d = 0; d < 3; d++) {
         st = fill_phase(c, f, kind, d, met, t);
@@ -1366,9 +1378,6 @@ static void covered_range_of(const crocco_grid_desc *fd, const int64_t c0[3], in
         hi = c0[d] + (nf - 2) / 2;
     }
 }
-static void covered_range(const crocco_ctx_s *f, int d, int64_t &lo, int64_t &hi) {
-    covered_range_of(&f->desc, f->amr_c0, d, lo, hi);
-}
 
 // geometry of a two-level pair (crocco_amr_link's checks; reading 24)
 static crocco_status amr_geom_check(crocco_ctx ec, const crocco_grid_desc *fd, const crocco_grid_desc *cd,
@@ -1398,12 +1407,14 @@ static crocco_status amr_geom_check(crocco_ctx ec, const crocco_grid_desc *fd, c
     return CROCCO_OK;
 }
 
+static bool cf_ghost_box(const crocco_grid_desc *fd, const int fnb[3], const int fbn[3], const BlockGeom &fb, int D,
+                         int side, int64_t lo[3], int64_t ext[3]);
 // The inter-level plan (crocco_amr_plan, include/crocco.h): every box of the pair touching rank
 // `me` (me < 0: all), kind 0 then kind 1, canonical order.
 static void build_amr_plan(const crocco_grid_desc *fd, const int fnb[3], const int fbn[3],
                            const std::vector<BlockGeom> &fall, const crocco_grid_desc *cd, const int cnb[3],
                            const int cbn[3], const std::vector<BlockGeom> &call, const int64_t c0[3], int me,
-                           std::vector<crocco_amr_msg> &out) {
+                           bool sib_mode, std::vector<crocco_amr_msg> &out) {
     out.clear();
     auto keep = [&](const crocco_amr_msg &m) {
         if (me < 0 || m.src_rank == me || m.dst_rank == me) out.push_back(m);
@@ -1412,23 +1423,12 @@ static void build_amr_plan(const crocco_grid_desc *fd, const int fnb[3], const i
     for (const BlockGeom &fb : fall)
         for (int D = 0; D < 3; D++)
             for (int side = 0; side < 2; side++) {
-                if (fd->bc[D][side] != CROCCO_BC_COARSE_FINE) continue;
-                if (fb.bidx[D] != (side == 0 ? 0 : fnb[D] - 1)) continue;  // not a domain face
+                int64_t lo[3], ext[3];  // the ghost box of phase D (build_plan)
+                if (!cf_ghost_box(fd, fnb, fbn, fb, D, side, lo, ext)) continue;
                 int64_t Ilo[3], Ihi[3];
                 for (int e = 0; e < 3; e++) {
-                    int64_t lo, ext;  // the ghost box of phase D (build_plan)
-                    if (e == D) {
-                        lo = side == 0 ? -G : fbn[e];
-                        ext = G;
-                    } else if (e < D) {
-                        lo = -G;
-                        ext = fbn[e] + 2 * G;
-                    } else {
-                        lo = 0;
-                        ext = fbn[e];
-                    }
-                    Ilo[e] = floor_half_h(2 * c0[e] + fb.origin[e] + lo);
-                    Ihi[e] = floor_half_h(2 * c0[e] + fb.origin[e] + lo + ext - 1);
+                    Ilo[e] = floor_half_h(2 * c0[e] + fb.origin[e] + lo[e]);
+                    Ihi[e] = floor_half_h(2 * c0[e] + fb.origin[e] + lo[e] + ext[e] - 1);
                 }
                 for (const BlockGeom &cb : call) {
                     crocco_amr_msg m;
@@ -1451,6 +1451,7 @@ static void build_amr_plan(const crocco_grid_desc *fd, const int fnb[3], const i
                     m.kind = 0;
                     m.coarse_block = cb.gid;
                     m.fine_block = fb.gid;
+                    m.sibling = -1;
                     m.src_rank = cb.rank;
                     m.dst_rank = fb.rank;
                     keep(m);
@@ -1465,6 +1466,10 @@ static void build_amr_plan(const crocco_grid_desc *fd, const int fnb[3], const i
             for (int e = 0; e < 3 && !empty; e++) {
                 int64_t lo, hi;
                 covered_range_of(fd, c0, e, lo, hi);
+                if (sib_mode && fd->bc[e][0] != CROCCO_BC_PERIODIC) {  // central fine node ours;
+                    lo = c0[e];                                         // k_average_down checks
+                    hi = c0[e] + (fd->n_global[e] - 1) / 2;             // the 27 nodes
+                }
                 // 2 (I - c0) in [origin, origin + n - 1]
                 lo = std::max(lo, c0[e] + (fb.origin[e] + 1) / 2);
                 hi = std::min(hi, c0[e] + (fb.origin[e] + fbn[e] - 1) / 2);
@@ -1478,10 +1483,86 @@ static void build_amr_plan(const crocco_grid_desc *fd, const int fnb[3], const i
             m.kind = 1;
             m.coarse_block = cb.gid;
             m.fine_block = fb.gid;
+            m.sibling = -1;
             m.src_rank = fb.rank;
             m.dst_rank = cb.rank;
             keep(m);
         }
+}
+
+// C/F ghost box (phase D, side) of block fb, [lo, lo+ext) in fine-block-local indices; false when
+// the face is not a C/F domain face
+static bool cf_ghost_box(const crocco_grid_desc *fd, const int fnb[3], const int fbn[3], const BlockGeom &fb, int D,
+                         int side, int64_t lo[3], int64_t ext[3]) {
+    if (fd->bc[D][side] != CROCCO_BC_COARSE_FINE || fb.bidx[D] != (side == 0 ? 0 : fnb[D] - 1)) return false;
+    for (int e = 0; e < 3; e++) {
+        if (e == D) {
+            lo[e] = side == 0 ? -G : fbn[e];
+            ext[e] = G;
+        } else if (e < D) {
+            lo[e] = -G;
+            ext[e] = fbn[e] + 2 * G;
+        } else {
+            lo[e] = 0;
+            ext[e] = fbn[e];
+        }
+    }
+    return true;
+}
+
+// kind 2 (crocco_amr_sibling_plan): the parts of the C/F ghost boxes of f's blocks inside the
+// interiors of sibling g's blocks, in the common fine index space 2 c0 + f
+static void build_sib_plan(const crocco_grid_desc *fd, const int fnb[3], const int fbn[3],
+                           const std::vector<BlockGeom> &fall, const int64_t c0f[3], const int gbn[3],
+                           const std::vector<BlockGeom> &gall, const int64_t c0g[3], int sidx, int me,
+                           std::vector<crocco_amr_msg> &out) {
+    for (const BlockGeom &fb : fall)
+        for (int D = 0; D < 3; D++)
+            for (int side = 0; side < 2; side++) {
+                int64_t lo[3], ext[3];
+                if (!cf_ghost_box(fd, fnb, fbn, fb, D, side, lo, ext)) continue;
+                for (const BlockGeom &gb : gall) {
+                    crocco_amr_msg m;
+                    memset(&m, 0, sizeof m);
+                    bool empty = false;
+                    for (int e = 0; e < 3 && !empty; e++) {
+                        const int64_t a0 = 2 * c0f[e] + fb.origin[e] + lo[e], a1 = a0 + ext[e];
+                        const int64_t b0 = 2 * c0g[e] + gb.origin[e], b1 = b0 + gbn[e];
+                        const int64_t x0 = std::max(a0, b0), x1 = std::min(a1, b1);
+                        empty = x0 >= x1;
+                        m.lo[e] = x0 - b0;
+                        m.ext[e] = x1 - x0;
+                    }
+                    if (empty) continue;
+                    m.kind = 2;
+                    m.coarse_block = gb.gid;
+                    m.fine_block = fb.gid;
+                    m.sibling = sidx;
+                    m.src_rank = gb.rank;
+                    m.dst_rank = fb.rank;
+                    if (me < 0 || m.src_rank == me || m.dst_rank == me) out.push_back(m);
+                }
+            }
+}
+
+crocco_status crocco_amr_sibling_plan(const crocco_grid_desc *fine, const int64_t c0[3], const crocco_grid_desc *sib,
+                                      const int64_t c0s[3], int32_t sibling, crocco_amr_msg *out, int32_t cap,
+                                      int32_t *n_out) {
+    int fnb[3], fbn[3], gnb[3], gbn[3];
+    crocco_status st = validate(fine, fnb, fbn);
+    if (!st) st = validate(sib, gnb, gbn);
+    if (st) return st;
+    if (!c0 || !c0s) return fail(nullptr, CROCCO_ERR_ARG, "null c0");
+    if (fine->nranks != sib->nranks || fine->rank != sib->rank)
+        return fail(nullptr, CROCCO_ERR_ARG, "sibling patches must share the process group");
+    std::vector<BlockGeom> fall, gall;
+    build_blocks(fine, fnb, fbn, fall);
+    build_blocks(sib, gnb, gbn, gall);
+    std::vector<crocco_amr_msg> plan;
+    build_sib_plan(fine, fnb, fbn, fall, c0, gbn, gall, c0s, sibling, fine->rank, plan);
+    if (n_out) *n_out = (int32_t)plan.size();
+    for (int i = 0; i < (int)plan.size() && i < cap; i++) out[i] = plan[i];
+    return CROCCO_OK;
 }
 
 crocco_status crocco_amr_plan(const crocco_grid_desc *fine, const crocco_grid_desc *coarse, const int64_t c0[3],
@@ -1496,7 +1577,7 @@ crocco_status crocco_amr_plan(const crocco_grid_desc *fine, const crocco_grid_de
     build_blocks(fine, fnb, fbn, fall);
     build_blocks(coarse, cnb, cbn, call);
     std::vector<crocco_amr_msg> plan;
-    build_amr_plan(fine, fnb, fbn, fall, coarse, cnb, cbn, call, c0, fine->rank, plan);
+    build_amr_plan(fine, fnb, fbn, fall, coarse, cnb, cbn, call, c0, fine->rank, false, plan);
     if (n_out) *n_out = (int32_t)plan.size();
     for (int i = 0; i < (int)plan.size() && i < cap; i++) out[i] = plan[i];
     return CROCCO_OK;
@@ -1522,7 +1603,7 @@ crocco_status crocco_amr_link(crocco_ctx f, crocco_ctx c, const int64_t c0[3]) {
     if (f->loc.size() > (size_t)AMR_MAX_LOCAL)
         return fail(f, CROCCO_ERR_ARG, "two-level AMR: at most %d local fine blocks", AMR_MAX_LOCAL);
     std::vector<crocco_amr_msg> plan;
-    build_amr_plan(&f->desc, f->nb, f->bn, f->all, &c->desc, c->nb, c->bn, c->all, c0, f->desc.rank, plan);
+    build_amr_plan(&f->desc, f->nb, f->bn, f->all, &c->desc, c->nb, c->bn, c->all, c0, f->desc.rank, false, plan);
     // slots of the coarse-level table: the local coarse blocks plus the mirrors this rank may use
     std::vector<int> mg;
     for (const crocco_amr_msg &m : plan)
@@ -1602,7 +1683,10 @@ static BoxOp amr_box_op(double *arr, const Lay &L, const crocco_amr_msg &m, doub
 // The routed boxes of one kind: pack (src arrays) -> grouped ncclSend / ncclRecv -> unpack (dst
 // arrays).  src_arr / dst_arr give the array of a box on the sending / receiving side.
 typedef std::function<double *(const crocco_amr_msg &)> AmrArr;
-static crocco_status amr_exchange(crocco_ctx f, int kind, const AmrArr &src_arr, const AmrArr &dst_arr) {
+typedef std::vector<std::pair<const crocco_amr_msg *, int64_t>> AmrRecv;
+// recv_out non-null: the received boxes are not unpacked; (box, offset in amr_recv) are returned
+static crocco_status amr_exchange(crocco_ctx f, int kind, const AmrArr &src_arr, const AmrArr &dst_arr,
+                                  AmrRecv *recv_out = nullptr) {
     const int me = f->desc.rank;
     std::vector<const crocco_amr_msg *> r;
     int64_t ns = 0, nr = 0;
@@ -1631,6 +1715,7 @@ static crocco_status amr_exchange(crocco_ctx f, int kind, const AmrArr &src_arr,
         f->amr_stage_elems = need;
     }
     const Lay Lc = make_layout(f->amr_coarse->bn, G);
+    auto lay = [&](const crocco_amr_msg &m) { return m.kind == 2 ? make_layout(f->sibs[m.sibling]->bn, G) : Lc; };
     BoxOps ops;
     ops.nops = 0;
     crocco_status st;
@@ -1646,7 +1731,7 @@ static crocco_status amr_exchange(crocco_ctx f, int kind, const AmrArr &src_arr,
         so[i] = s;
         double *a = src_arr(*r[i]);
         if (!a) return fail(f, CROCCO_ERR_NOMEM, "AMR mirror allocation failed");
-        if ((st = push_op(f, ops, amr_box_op(a, Lc, *r[i], f->amr_send + s, true)))) return st;
+        if ((st = push_op(f, ops, amr_box_op(a, lay(*r[i]), *r[i], f->amr_send + s, true)))) return st;
         s += v;
     }
     if ((st = flush_ops(f, ops))) return st;
@@ -1664,9 +1749,13 @@ static crocco_status amr_exchange(crocco_ctx f, int kind, const AmrArr &src_arr,
     }
     for (size_t i = 0; i < r.size(); i++) {
         if (r[i]->dst_rank != me) continue;
+        if (recv_out) {
+            recv_out->push_back({r[i], ro[i]});
+            continue;
+        }
         double *a = dst_arr(*r[i]);
         if (!a) return fail(f, CROCCO_ERR_NOMEM, "AMR mirror allocation failed");
-        if ((st = push_op(f, ops, amr_box_op(a, Lc, *r[i], f->amr_recv + ro[i], false)))) return st;
+        if ((st = push_op(f, ops, amr_box_op(a, lay(*r[i]), *r[i], f->amr_recv + ro[i], false)))) return st;
     }
     return flush_ops(f, ops);
 }
@@ -1687,9 +1776,47 @@ static crocco_status amr_fill_exchange(crocco_ctx f) {
         [&](const crocco_amr_msg &m) { return amr_mirror(f, m.coarse_block); });
 }
 
+// mirror of block gid of sibling s (the sibling's block layout), allocated zeroed on first use;
+// amr_sib_mirror_if: the existing one or null (a block no routed box of this rank lands in)
+static double *amr_sib_mirror(crocco_ctx f, int s, int gid) {
+    const int key = s * AMR_MAX_BLOCKS + gid;
+    for (size_t i = 0; i < f->amr_smirror_key.size(); i++)
+        if (f->amr_smirror_key[i] == key) return f->amr_smirror[i];
+    const Lay L = make_layout(f->sibs[s]->bn, G);
+    double *p = nullptr;
+    if (cudaMalloc((void **)&p, (size_t)(5 * L.cs) * sizeof(double)) != cudaSuccess ||
+        cudaMemset(p, 0, (size_t)(5 * L.cs) * sizeof(double)) != cudaSuccess) {
+        cudaGetLastError();
+        cudaFree(p);
+        return nullptr;
+    }
+    f->scratch += 5 * L.cs * (int64_t)sizeof(double);
+    f->amr_smirror_key.push_back(key);
+    f->amr_smirror.push_back(p);
+    return p;
+}
+static double *amr_sib_mirror_if(crocco_ctx f, int s, int gid) {
+    const int key = s * AMR_MAX_BLOCKS + gid;
+    for (size_t i = 0; i < f->amr_smirror_key.size(); i++)
+        if (f->amr_smirror_key[i] == key) return f->amr_smirror[i];
+    return nullptr;
+}
+
+// same-level part of the C/F fill with siblings: the sibling interior boxes this rank's ghost
+// bands copy from other ranks (or through the loopback) land in the sibling-block mirrors
+static crocco_status amr_sib_exchange(crocco_ctx f) {
+    double *const *const *sU = f->amr_sibU;
+    return amr_exchange(
+        f, 2,
+        [&](const crocco_amr_msg &m) { return sU[m.sibling][f->sibs[m.sibling]->gid_to_local[m.coarse_block]]; },
+        [&](const crocco_amr_msg &m) { return amr_sib_mirror(f, m.sibling, m.coarse_block); });
+}
+
 static crocco_status amr_ready(crocco_ctx f, double *const *Uc) {
     if (!f->amr_coarse) return fail(f, CROCCO_ERR_ARG, "fine level not linked (crocco_amr_link)");
     if (f->amr_coarse->poisoned) return CROCCO_ERR_STATE;
+    if (!f->sibs.empty() && !f->amr_sibU)
+        return fail(f, CROCCO_ERR_ARG, "patch has siblings: use the _level calls with their states");
     if (!Uc) return fail(f, CROCCO_ERR_ARG, "null coarse pointer array");
     for (size_t b = 0; b < f->amr_coarse->loc.size(); b++)
         if (!Uc[b]) return fail(f, CROCCO_ERR_ARG, "null coarse pointer for local block %zu", b);
@@ -1749,10 +1876,11 @@ crocco_status crocco_average_down(crocco_ctx f, double *const *Uf, double *const
         mx = 0;
         return CROCCO_OK;
     };
-    auto push = [&](double *dst, const Lay &Lb, const int64_t org[3], const int64_t lo[3],
-                    const int64_t hi[3]) -> crocco_status {
+    auto push = [&](double *dst, const Lay &Lb, const int64_t org[3], const int64_t lo[3], const int64_t hi[3],
+                    const double *buf) -> crocco_status {
         ADOp &o = ops.op[ops.nops++];
         o.dst = dst;
+        o.buf = buf;
         o.dbase = at(Lb, (int)(lo[0] - org[0]), (int)(lo[1] - org[1]), (int)(lo[2] - org[2]));
         for (int d = 0; d < 3; d++) {
             o.ext[d] = (int)(hi[d] - lo[d] + 1);
@@ -1761,29 +1889,10 @@ crocco_status crocco_average_down(crocco_ctx f, double *const *Uf, double *const
         mx = std::max<int64_t>(mx, (int64_t)o.ext[0] * o.ext[1] * o.ext[2]);
         return ops.nops == CF_MAX_OPS ? flush() : CROCCO_OK;
     };
-    if (sb.n > 0) {
-        // siblings (single-rank, reading 31): per local coarse block the nodes whose central fine
-        // node is ours; k_average_down checks their 27 nodes
-        for (size_t bi = 0; bi < c->loc.size(); bi++) {
-            const LocalBlock &b = c->loc[bi];
-            int64_t lo[3], hi[3];
-            bool empty = false;
-            for (int d = 0; d < 3; d++) {
-                covered_range(f, d, lo[d], hi[d]);
-                if (f->desc.bc[d][0] != CROCCO_BC_PERIODIC) {
-                    lo[d] = f->amr_c0[d];
-                    hi[d] = f->amr_c0[d] + (f->desc.n_global[d] - 1) / 2;
-                }
-                lo[d] = std::max<int64_t>(lo[d], b.g.origin[d]);
-                hi[d] = std::min<int64_t>(hi[d], b.g.origin[d] + b.g.n[d] - 1);
-                empty = empty || lo[d] > hi[d];
-            }
-            if (!empty && (st = push(Uc[bi], b.L, b.g.origin, lo, hi))) return st;
-        }
-        return flush();
-    }
     // the plan's kind-1 boxes computed on this rank: in place when the coarse block is ours,
-    // else (or under the loopback) into its mirror, then sent to the coarse block's rank
+    // else (or under the loopback) into its mirror, then sent to the coarse block's rank; with
+    // siblings the boxes hold the nodes whose central fine node is ours and k_average_down keeps
+    // those whose 27 fine nodes lie in the level's patch interiors (reading 31)
     for (const crocco_amr_msg &m : f->amr_plan) {
         if (m.kind != 1 || m.src_rank != f->desc.rank) continue;
         const BlockGeom &cb = c->all[m.coarse_block];
@@ -1794,12 +1903,47 @@ crocco_status crocco_average_down(crocco_ctx f, double *const *Uf, double *const
             lo[d] = cb.origin[d] + m.lo[d];
             hi[d] = lo[d] + m.ext[d] - 1;
         }
-        if ((st = push(dst, ops.Lc, cb.origin, lo, hi))) return st;
+        if ((st = push(dst, ops.Lc, cb.origin, lo, hi, nullptr))) return st;
     }
     if ((st = flush())) return st;
-    return amr_exchange(
-        f, 1, [&](const crocco_amr_msg &m) { return amr_mirror(f, m.coarse_block); },
-        [&](const crocco_amr_msg &m) { return Uc[c->gid_to_local[m.coarse_block]]; });
+    // the boxes averaged on other ranks: their covered nodes (the same 27-node rule, evaluated
+    // here) take the received values -- the others of a sibling-mode box were not averaged
+    AmrRecv got;
+    if ((st = amr_exchange(
+             f, 1, [&](const crocco_amr_msg &m) { return amr_mirror(f, m.coarse_block); },
+             [&](const crocco_amr_msg &) { return (double *)nullptr; }, &got)))
+        return st;
+    for (auto &g : got) {
+        const crocco_amr_msg &m = *g.first;
+        const BlockGeom &cb = c->all[m.coarse_block];
+        int64_t lo[3], hi[3];
+        for (int d = 0; d < 3; d++) {
+            lo[d] = cb.origin[d] + m.lo[d];
+            hi[d] = lo[d] + m.ext[d] - 1;
+        }
+        if ((st = push(Uc[c->gid_to_local[m.coarse_block]], ops.Lc, cb.origin, lo, hi, f->amr_recv + g.second)))
+            return st;
+    }
+    return flush();
+}
+
+// f's plan with its siblings: kind-1 boxes over the nodes whose central fine node is f's, plus the
+// kind-2 boxes of every sibling in link order
+static crocco_status amr_rebuild_plan(crocco_ctx f) {
+    const crocco_ctx_s *c = f->amr_coarse;
+    std::vector<crocco_amr_msg> plan;
+    build_amr_plan(&f->desc, f->nb, f->bn, f->all, &c->desc, c->nb, c->bn, c->all, f->amr_c0, f->desc.rank,
+                   !f->sibs.empty(), plan);
+    for (size_t i = 0; i < f->sibs.size(); i++) {
+        const crocco_ctx_s *g = f->sibs[i];
+        build_sib_plan(&f->desc, f->nb, f->bn, f->all, f->amr_c0, g->bn, g->all, g->amr_c0, (int)i, f->desc.rank,
+                       plan);
+    }
+    for (const crocco_amr_msg &m : plan)
+        if (m.src_rank != m.dst_rank && !f->comm)
+            return fail(f, CROCCO_ERR_ARG, "inter-rank AMR boxes need the patch's communicator");
+    f->amr_plan = std::move(plan);
+    return CROCCO_OK;
 }
 
 crocco_status crocco_amr_link_sibling(crocco_ctx f, crocco_ctx g) {
@@ -1808,16 +1952,16 @@ crocco_status crocco_amr_link_sibling(crocco_ctx f, crocco_ctx g) {
     if (f == g) return fail(f, CROCCO_ERR_ARG, "a patch is not its own sibling");
     if (!f->amr_coarse || f->amr_coarse != g->amr_coarse)
         return fail(f, CROCCO_ERR_ARG, "siblings must be linked (crocco_amr_link) to the same coarse level");
-    if (f->desc.nranks != 1 || g->desc.nranks != 1)
-        return fail(f, CROCCO_ERR_ARG, "same-level siblings: single-rank levels only");
+    if (f->desc.nranks != g->desc.nranks || f->desc.rank != g->desc.rank)
+        return fail(f, CROCCO_ERR_ARG, "sibling patches must share the process group");
     for (auto s : f->sibs)
         if (s == g) return CROCCO_OK;
     if (f->sibs.size() >= 8 || g->sibs.size() >= 8) return fail(f, CROCCO_ERR_ARG, "at most 8 siblings per patch");
     int nb = 0;
-    for (auto s : f->sibs) nb += (int)s->loc.size();
+    for (auto s : f->sibs) nb += (int)s->all.size();
     int ng = 0;
-    for (auto s : g->sibs) ng += (int)s->loc.size();
-    if (nb + (int)g->loc.size() > SIB_MAX_BLOCKS || ng + (int)f->loc.size() > SIB_MAX_BLOCKS)
+    for (auto s : g->sibs) ng += (int)s->all.size();
+    if (nb + (int)g->all.size() > SIB_MAX_BLOCKS || ng + (int)f->all.size() > SIB_MAX_BLOCKS)
         return fail(f, CROCCO_ERR_ARG, "at most %d sibling blocks per patch", SIB_MAX_BLOCKS);
     // interiors disjoint (in the common fine index space 2 c0 + f); a periodic direction spans all
     bool overlap = true;
@@ -1831,7 +1975,15 @@ crocco_status crocco_amr_link_sibling(crocco_ctx f, crocco_ctx g) {
     if (overlap) return fail(f, CROCCO_ERR_ARG, "sibling patches overlap");
     f->sibs.push_back(g);
     g->sibs.push_back(f);
-    return CROCCO_OK;
+    crocco_status st = amr_rebuild_plan(f);
+    if (!st) st = amr_rebuild_plan(g);
+    if (st) {
+        f->sibs.pop_back();
+        g->sibs.pop_back();
+        amr_rebuild_plan(f);
+        amr_rebuild_plan(g);
+    }
+    return st;
 }
 
 static crocco_status sib_ready(crocco_ctx f, double *const *const *sibU) {

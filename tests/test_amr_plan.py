@@ -163,3 +163,60 @@ def test_plan_refuses_what_link_refuses():
     cd2 = cc.make_desc((24, 24, 16), (1, 1, 1), ((PER, PER),) * 3, rank=1, nranks=2, block_rank=[0])
     with pytest.raises(RuntimeError):
         cc.crocco_amr_plan(fd2, cd2, (1, 1, 1))             # different ranks of one process
+
+
+SIB = [  # two patches of one level in the common fine index space 2 c0 + f (reading 31)
+    dict(nf=(16, 16, 12), nbf=(2, 1, 1), c0=(3, 4, 2), ng=(16, 16, 12), nbg=(1, 2, 2), c0g=(11, 4, 2)),   # abut in x
+    dict(nf=(16, 12, 12), nbf=(1, 2, 1), c0=(3, 4, 2), ng=(12, 16, 8), nbg=(2, 1, 2), c0g=(5, 11, 3)),    # gap of 2 in y
+]
+
+
+@pytest.mark.parametrize("sc", SIB, ids=["abutting", "nearby"])
+@pytest.mark.parametrize("nranks", [1, 2, 3])
+def test_sibling_boxes_cover_the_ghost_points_inside_the_sibling(sc, nranks):
+    """Kind-2 boxes (crocco_amr_sibling_plan): a C/F ghost point of a patch block lying in a sibling
+    block's interior is in exactly the box routed from that sibling block to that patch block;
+    boxes hold no other point; sends and receives of every rank pair match in order."""
+    bcf = ((CF, CF),) * 3
+    rng = np.random.default_rng(nranks)
+    rf = rng.integers(0, nranks, int(np.prod(sc["nbf"]))).tolist()
+    rg = rng.integers(0, nranks, int(np.prod(sc["nbg"]))).tolist()
+    plans = []
+    for r in range(nranks):
+        fd = cc.make_desc(sc["nf"], sc["nbf"], bcf, rank=r, nranks=nranks, block_rank=rf)
+        gd = cc.make_desc(sc["ng"], sc["nbg"], bcf, rank=r, nranks=nranks, block_rank=rg)
+        plans.append(cc.crocco_amr_sibling_plan(fd, sc["c0"], gd, sc["c0g"], 1))
+    for r, s in itertools.product(range(nranks), repeat=2):
+        if r != s:
+            assert [_t(m) for m in plans[r] if m.src_rank == r and m.dst_rank == s] == \
+                   [_t(m) for m in plans[s] if m.src_rank == r and m.dst_rank == s]
+    allm = {_t(m) + (m.sibling,) for p in plans for m in p}
+    assert allm and all(m[0] == 2 and m[7] == 1 for m in allm)
+    # sibling blocks in the common index space
+    gbl = {gid: [2 * sc["c0g"][d] + org[d] for d in range(3)] for gid, _, org, _ in _blocks(sc["ng"], sc["nbg"])}
+    bng = [sc["ng"][d] // sc["nbg"][d] for d in range(3)]
+    want = set()
+    for gid, bidx, org, bn in _blocks(sc["nf"], sc["nbf"]):
+        for D, side in itertools.product(range(3), range(2)):
+            if bidx[D] != (0 if side == 0 else sc["nbf"][D] - 1):
+                continue
+            rngs = []
+            for e in range(3):
+                if e == D:
+                    lo, ext = (-G if side == 0 else bn[e]), G
+                elif e < D:
+                    lo, ext = -G, bn[e] + 2 * G
+                else:
+                    lo, ext = 0, bn[e]
+                rngs.append(range(lo, lo + ext))
+            for f in itertools.product(*rngs):
+                p = [2 * sc["c0"][d] + org[d] + f[d] for d in range(3)]
+                for sg, o in gbl.items():
+                    if all(o[d] <= p[d] < o[d] + bng[d] for d in range(3)):
+                        want.add((sg, gid, tuple(p[d] - o[d] for d in range(3))))
+    got = set()
+    for kind, sg, fg, src, dst, lo, ext, _ in allm:
+        assert src == rg[sg] and dst == rf[fg]
+        for q in itertools.product(*[range(lo[d], lo[d] + ext[d]) for d in range(3)]):
+            got.add((sg, fg, q))
+    assert got == want and want

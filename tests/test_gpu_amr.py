@@ -573,3 +573,38 @@ def test_abutting_patches_parity_and_union(axis):
         assert np.array_equal(a, b)
     for S in [Cu] + Fu:
         S.close()
+
+
+@pytest.mark.parametrize("axis", [0, 1])
+def test_sibling_boxes_through_nccl_loopback_bitwise(axis):
+    """Sibling patches on different ranks (include/crocco.h crocco_amr_link_sibling, kind-2 boxes
+    of crocco_amr_sibling_plan) on one GPU: with the NCCL loopback on both patch ctx every
+    sibling ghost box and every inter-level box goes pack -> ncclSend/ncclRecv -> unpack into the
+    mirrors; 3 RK3 steps of two abutting multi-block patches are bitwise those of the in-place
+    run, which test_abutting_patches_parity_and_union pins to the oracle and to the union patch."""
+    from paper_conf_ipps_davissngmb23_b200 import crocco as cc
+    nc = (24, 20, 16)
+    grid = synth.Wavy3D(L=(10.0,) * 3, N=nc)
+    phys = dict(terms=3, mu_ref=0.01)
+    c0, nu = (3, 4, 2), [24, 16, 12]
+    half = [nu[d] // 2 if d == axis else nu[d] for d in range(3)]
+    c0b = tuple(c0[d] + (half[d] // 2 if d == axis else 0) for d in range(3))
+    specs = [(c0, tuple(half), (2, 1, 1) if axis == 1 else (1, 2, 1)), (c0b, tuple(half), (1, 1, 2))]
+    outs = []
+    for lb in (0, 1):
+        C, Fs, A = _gpu_level(nc, grid, (2, 1, 1), specs, lambda x: synth.vortex(x), phys)
+        assert A.sibs == [[1], [0]]
+        if lb:
+            for F in Fs:
+                cc.crocco_set_nccl_loopback(F.ctx, 1)
+        s0 = [cc.crocco_scratch_bytes(F.ctx) for F in Fs]
+        A.step(0.01, 3)
+        A.sync()
+        if lb:
+            assert all(cc.crocco_scratch_bytes(F.ctx) > s for F, s in zip(Fs, s0))
+        outs.append([C.get(C.U)] + [F.get(F.U) for F in Fs])
+        for S in [C] + Fs:
+            S.close()
+    for a, b in zip(outs[0], outs[1]):
+        for x, y in zip(a, b):
+            assert np.array_equal(x, y)
