@@ -621,6 +621,86 @@ def run_dmr_amr(args):
     return 0
 
 
+def run_size_sweep(args):
+    """The paper's Fig. 3 analogue (sec. VI-A): time per RK3 step spent in the
+    WENOx and Viscous work over a range of problem sizes, on the GPU (this library: the xi sweep
+    class and the viscous kernel class, CUDA events per launch) and on the host CPU (the oracle as
+    it stands, at 1 core and all cores: its RHS with only the xi inviscid flux, and with only the
+    viscous terms).  The GPU viscous class holds the point fluxes and the xi / zeta divergences
+    (the eta divergence rides in the eta sweep); the oracle's viscous RHS holds all three.
+    Weak-recipe boxes (periodic wavy grid, TGV + noise), one block, one GPU."""
+    import torch
+
+    import synth
+    from paper_conf_ipps_davissngmb23_b200 import crocco as cc
+    from paper_conf_ipps_davissngmb23_b200.solver import Solver
+
+    phys = dict(gamma=1.4, R=1.0, Pr=0.71, mu_ref=1.0 / 1600.0, terms=3)
+    dt = 2e-4
+    gpu = []
+    for N in (32, 64, 96, 128, 192, 256, 384, 512):
+        n = (N, N, N)
+        grid = synth.Wavy3D(L=(2 * math.pi,) * 3, N=n, x0=(-math.pi,) * 3, k=2.0, A=0.15)
+        S = Solver(n, (1, 1, 1), ((0, 0),) * 3, cc.make_phys(**phys))
+        dev = S.device
+        xyz = torch.from_numpy(grid.coords(n, (0, 0, 0), cc.GHOST_COORDS)).to(dev)
+        S.set_coords_block(0, xyz)
+        S.set_state_block(0, synth.tgv(xyz, noise=0.01, seed=5))
+        del xyz
+        for _ in range(max(args.warmup, 1)):
+            S.step(dt, graph=False)
+        reps = max(2, min(50, int(2e8 // N ** 3)))
+        cc.crocco_set_timing(S.ctx, True)
+        cc.crocco_kernel_times(S.ctx)
+        torch.cuda.synchronize()
+        for _ in range(reps):
+            S.step(dt, graph=False)
+        kt = cc.crocco_kernel_times(S.ctx)
+        S.close()
+        row = {"n": N, "points": N ** 3, "rk3_steps": reps}
+        for cls, key in (("sweep_xi", "wenox_ms_per_step"), ("viscous", "viscous_ms_per_step")):
+            row[key] = kt[cls][1] / reps
+        row["all_kernels_ms_per_step"] = sum(v[1] for v in kt.values()) / reps
+        gpu.append(row)
+    cpu = []
+    if not args.no_cpu_baseline:
+        import oracle
+        oracle.build()
+        cores = os.cpu_count() or 1
+        t_start = time.perf_counter()
+        for threads in (1, cores):
+            oracle.set_threads(threads)
+            for N in (16, 24, 32, 48, 64):
+                n = (N, N, N)
+                grid = synth.Wavy3D(L=(2 * math.pi,) * 3, N=n, x0=(-math.pi,) * 3, k=2.0, A=0.15)
+                xyz = grid.coords(n, (0, 0, 0), oracle.GC)
+                met = oracle.metrics(n, ((0, 0),) * 3, xyz)
+                U = synth.pad_state(synth.tgv(xyz, noise=0.01, seed=5))
+                oracle.fill(n, ((0, 0),) * 3, U)
+                row = {"n": N, "points": N ** 3, "cores": oracle.get_threads()}
+                for key, kw in (("wenox_ms_per_step", dict(terms=1, dir_mask=1)), ("viscous_ms_per_step", dict(terms=2))):
+                    ph = oracle.phys(**dict(phys, **kw))
+                    t0 = time.perf_counter()
+                    k = 0
+                    while True:
+                        oracle.rhs(n, ph, U, met)
+                        k += 1
+                        if time.perf_counter() - t0 > 0.5 or k >= 20:
+                            break
+                    row[key] = 3e3 * (time.perf_counter() - t0) / k   # 3 RHS evaluations per RK3 step
+                cpu.append(row)
+                if time.perf_counter() - t_start > 120:
+                    break
+        oracle.set_threads(cores)
+    out = {"metric": "WENOx / Viscous time per RK3 step vs problem size (PAPER.md Fig. 3 analogue)",
+           "unit": "ms per RK3 step", "dtype": "f64", "data": "synthetic",
+           "config": {"workload": "size sweep: weak-recipe boxes N^3 (periodic wavy grid, TGV + noise, viscous), "
+                                  "one block, one GPU; CPU = the oracle at 1 core and all cores"},
+           "gpu": gpu, "cpu": cpu}
+    print(json.dumps(out), flush=True)
+    return 0
+
+
 def _profiled_traffic(kname, key="dram_bytes_per_launch"):
     """A per-launch ncu figure (default: dram bytes) of the dominant kernel from the committed
     ncu summary (profiles/ncu_summary.json), if any."""
@@ -666,7 +746,8 @@ def main():
     ap.add_argument("--steps", type=int, default=5)
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--impl", choices=["crocco", "reference"], default="crocco")
-    ap.add_argument("--config", choices=["weak", "ramp", "tgv", "vortex", "sod", "dmr", "amr", "dmr_amr"],
+    ap.add_argument("--config", choices=["weak", "ramp", "tgv", "vortex", "sod", "dmr", "amr", "dmr_amr",
+                                         "size_sweep"],
                     default="weak",
                     help="weak (default, the north_star 512^3/GPU workload) or a fixed BASELINE config")
     ap.add_argument("--e2e-steps", type=int, default=48,
@@ -688,6 +769,10 @@ def main():
         return relaunch(args.gpus)
     if world != args.gpus:
         raise SystemExit(f"bench.py: --gpus {args.gpus} but WORLD_SIZE={world}: one rank per GPU required")
+    if args.config == "size_sweep":
+        if world > 1:
+            raise SystemExit("--config size_sweep runs on one GPU")
+        return run_size_sweep(args)
     if args.config in ("amr", "dmr_amr"):
         if world > 1:
             raise SystemExit(f"--config {args.config} runs on one GPU")

@@ -50,11 +50,16 @@ constexpr int VISC_VKMAX = 256;
 __host__ __device__ inline int visc_tiles_x(const Lay &L) { return (L.n0 + VSX - 1) / VSX; }
 // overlap: the stage runs the ghost-free tiles beside the fill (crocco_rk_stage), so the slab
 // depth must leave at least one interior slab, (n2 - 4)/vk >= 2 (visc_interior_tiles)
+// Small boxes (fewer than two waves of tiles at VK): shorter slabs down to VISC_VKMIN planes, so
+// the marching chains shorten and more SMs take part (64^3: 27 tiles of 68 planes -> 216 of 12).
+constexpr int VISC_VKMIN = 8;
 inline int visc_slab(const Lay &L, const VLay &V, bool overlap = false) {
     const int64_t txy = (int64_t)visc_tiles_x(L) * ((V.b1 + VTY - 1) / VTY);
     for (int vk = VISC_VKMAX; vk > VK; vk /= 2)
         if (txy * ((L.n2 + vk - 1) / vk) >= 8 * 148 && (!overlap || (L.n2 - 4) / vk >= 2)) return vk;
-    return VK;
+    int vk = VK;
+    while (vk > VISC_VKMIN && txy * ((L.n2 + vk - 1) / vk) < 2 * 148) vk /= 2;
+    return vk;
 }
 
 // Tiles of k_visc_tiled whose loads stay inside the interior [0, n) in every
