@@ -608,3 +608,42 @@ def test_sibling_boxes_through_nccl_loopback_bitwise(axis):
     for a, b in zip(outs[0], outs[1]):
         for x, y in zip(a, b):
             assert np.array_equal(x, y)
+
+
+def test_three_level_hierarchy_through_nccl_loopback_bitwise():
+    """Every inter-level box of a three-level hierarchy (level 1 is the fine level of level 0 and
+    the coarse level of level 2) through ncclSend/ncclRecv to self: 2 RK3 steps bitwise equal to
+    the in-place run (which test_three_level_hierarchy_parity pins to the oracle)."""
+    from paper_conf_ipps_davissngmb23_b200 import crocco as cc
+    from paper_conf_ipps_davissngmb23_b200.solver import AmrHierarchy, Solver
+    n0 = (24, 24, 16)
+    g0 = synth.Wavy3D(L=(10.0,) * 3, N=n0)
+    c01, n1 = (4, 5, 2), (28, 24, 20)
+    c12, n2 = (6, 4, 5), (24, 24, 16)
+    g1 = synth.Refined(g0, c01)
+    g2 = synth.Refined(g1, c12)
+    bcf = ((CF, CF),) * 3
+    phys = dict(terms=3, mu_ref=0.01)
+    outs = []
+    for lb in (0, 1):
+        S = []
+        for n, g, bc, nb in ((n0, g0, PER, (2, 2, 1)), (n1, g1, bcf, (2, 1, 2)), (n2, g2, bcf, (1, 2, 1))):
+            X = Solver(n, nb, bc, cc.make_phys(**phys))
+            bn, bl = block_slices(n, nb)
+            X.set_coords([g.coords(bn, o, oracle.GC) for o, _ in bl])
+            x = g.coords(n, (0, 0, 0), oracle.GC)
+            U0 = synth.vortex(x)
+            X.set_state([np.ascontiguousarray(U0[(slice(None),) + sl]) for _, sl in bl])
+            S.append(X)
+        H = AmrHierarchy(S[0], [[(S[1], 0, c01)], [(S[2], 0, c12)]])
+        if lb:
+            cc.crocco_set_nccl_loopback(S[1].ctx, 1)
+            cc.crocco_set_nccl_loopback(S[2].ctx, 1)
+        H.step(0.005, 2)
+        H.sync()
+        outs.append([X.get(X.U) for X in S])
+        for X in S:
+            X.close()
+    for a, b in zip(outs[0], outs[1]):
+        for x, y in zip(a, b):
+            assert np.array_equal(x, y)
