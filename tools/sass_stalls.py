@@ -4,7 +4,11 @@ import csv, collections, sys
 def load(path):
     rows = list(csv.reader(open(path)))
     h = rows[1]; ix = {n: i for i, n in enumerate(h)}
-    data = [r for r in rows[2:] if len(r) == len(h) and r[0] != 'Address']
+    data, seen = [], set()
+    for r in rows[2:]:  # ncu may print the kernel's listing twice: keep one row per address
+        if len(r) == len(h) and r[0] != 'Address' and r[0] not in seen:
+            seen.add(r[0])
+            data.append(r)
     return h, ix, data
 
 def num(x):
