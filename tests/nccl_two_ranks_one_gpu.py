@@ -1,4 +1,6 @@
-"""Exercise the library's NCCL halo path with 2 ranks on ONE GPU (if NCCL allows it):
+"""(Round-1 diagnostic, kept under tests/ because it calls the oracle; NCCL refuses two ranks on one
+GPU, profiles/r01s2_nccl_two_ranks_one_gpu.log -- the loopback tests replace it.)
+Exercise the library's NCCL halo path with 2 ranks on ONE GPU (if NCCL allows it):
 gloo broadcasts the ncclUniqueId, each rank owns one block, and the filled state must
 equal the oracle's global fill bit for bit; then RK steps are compared with the oracle."""
 import os, sys, json

@@ -1,7 +1,7 @@
 # round-1 session-2 evidence: NCCL 2-ranks-on-1-GPU probe, bench (default + reference arm),
 # launch list, full ncu of sweeps / viscous / fill, SASS source page of the sweeps
 cd "${GRAFT_REPO_ROOT:-/root/repo}"; mkdir -p gpurun_out
-timeout 240 python -m torch.distributed.run --nnodes=1 --nproc-per-node 2 --master-addr 127.0.0.1 --master-port 29511 tools/nccl_two_ranks_one_gpu.py > gpurun_out/nccl2.log 2>&1
+timeout 240 python -m torch.distributed.run --nnodes=1 --nproc-per-node 2 --master-addr 127.0.0.1 --master-port 29511 tests/nccl_two_ranks_one_gpu.py > gpurun_out/nccl2.log 2>&1
 echo "nccl2 exit $?" >> gpurun_out/nccl2.log
 timeout 900 python bench.py --steps 5 --warmup 3 > gpurun_out/bench.log 2>&1
 echo "bench exit $?" >> gpurun_out/bench.log
