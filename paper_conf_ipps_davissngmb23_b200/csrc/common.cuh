@@ -87,6 +87,18 @@ __device__ __forceinline__ double minnn(double a, double b) {
     return __longlong_as_double(x < y ? x : y);
 }
 
+// asynchronous global -> shared copies (sm_80+ cp.async; the sweeps' rings, the viscous kernels' staging)
+__device__ __forceinline__ void cp_async8(double *dst, const double *src) {
+    const unsigned d = (unsigned)__cvta_generic_to_shared(dst);
+    asm volatile("cp.async.ca.shared.global [%0], [%1], 8;\n" ::"r"(d), "l"(src) : "memory");
+}
+__device__ __forceinline__ void cp_async16(double *dst, const double *src) {
+    const unsigned d = (unsigned)__cvta_generic_to_shared(dst);
+    asm volatile("cp.async.cg.shared.global [%0], [%1], 16;\n" ::"r"(d), "l"(src) : "memory");
+}
+__device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commit_group;\n" ::: "memory"); }
+__device__ __forceinline__ void cp_async_wait_all() { asm volatile("cp.async.wait_group 0;\n" ::: "memory"); }
+
 // primitive buffer components (k_prims)
 // (PIS = 1/sqrt(rho): the Roe weights use sqrt(rho) = rho / sqrt(rho), 1/rho~ = PIS_L PIS_R)
 enum { PU = 0, PV = 1, PW = 2, PP = 3, PC = 4, PIS = 5, PH = 6 };

@@ -54,16 +54,6 @@ struct SweepArgs {
 // once per point when it enters the ring -- so the characteristic WENO reads
 // only shared memory.  Warps are independent (no block barriers).
 // ---------------------------------------------------------------------------
-__device__ __forceinline__ void cp_async8(double *dst, const double *src) {
-    const unsigned d = (unsigned)__cvta_generic_to_shared(dst);
-    asm volatile("cp.async.ca.shared.global [%0], [%1], 8;\n" ::"r"(d), "l"(src) : "memory");
-}
-__device__ __forceinline__ void cp_async16(double *dst, const double *src) {
-    const unsigned d = (unsigned)__cvta_generic_to_shared(dst);
-    asm volatile("cp.async.cg.shared.global [%0], [%1], 16;\n" ::"r"(d), "l"(src) : "memory");
-}
-__device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commit_group;\n" ::: "memory"); }
-__device__ __forceinline__ void cp_async_wait_all() { asm volatile("cp.async.wait_group 0;\n" ::: "memory"); }
 
 template <int D, bool VISC>
 struct RingGeom {
