@@ -400,7 +400,8 @@ typedef struct {
    owner block of I chosen by clamping I into the domain (k_cf_interp).  Kind 1: per fine block
    and coarse block, the covered nodes (reading 26) whose central fine node 2 (I - c0) lies in
    the fine block.  Writes up to cap entries, *n_out = total count; CROCCO_ERR_ARG for
-   descriptors crocco_amr_link would refuse (no sibling semantics: siblings are single-rank). */
+   descriptors crocco_amr_link would refuse.  Without sibling semantics: a patch with siblings
+   gets the kind-1 boxes of the sibling rule and its kind-2 boxes from crocco_amr_link_sibling. */
 crocco_status crocco_amr_plan(const crocco_grid_desc *fine, const crocco_grid_desc *coarse, const int64_t c0[3],
                               crocco_amr_msg *out, int32_t cap, int32_t *n_out);
 /* Kind-2 boxes (sibling index `sibling`) of fine patch `fine` at coarse node c0 with its sibling
