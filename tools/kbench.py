@@ -7,16 +7,20 @@ import synth
 from paper_conf_ipps_davissngmb23_b200 import crocco as cc
 from paper_conf_ipps_davissngmb23_b200.solver import Solver
 N = int(os.environ.get("KB_N", "512"))
-n = (N, N, N)
-grid = synth.Wavy3D(L=(2 * math.pi,) * 3, N=n, x0=(-math.pi,) * 3, k=2.0, A=0.15)
-S = Solver(n, (1, 1, 1), ((0, 0),) * 3, cc.make_phys(gamma=1.4, R=1.0, Pr=0.71, mu_ref=1 / 1600, terms=int(os.environ.get("KB_TERMS", "3")),
+NB = tuple(int(x) for x in os.environ.get("KB_BLOCKS", "1,1,1").split(","))   # N^3 per block
+n = (N * NB[0], N * NB[1], N * NB[2])
+grid = synth.Wavy3D(L=(2 * math.pi * NB[0], 2 * math.pi * NB[1], 2 * math.pi * NB[2]), N=n, x0=(-math.pi,) * 3,
+                    k=2.0, A=0.15)
+S = Solver(n, NB, ((0, 0),) * 3, cc.make_phys(gamma=1.4, R=1.0, Pr=0.71, mu_ref=1 / 1600, terms=int(os.environ.get("KB_TERMS", "3")),
                                                   weno_limiter=int(os.environ.get("KB_LIM", "0")), weno_alpha_rl=5.0, weno_alpha_al=1e-4,
                                                   visc_form=int(os.environ.get("KB_VISC_FORM", "0"))))
 cc.crocco_set_overlap(S.ctx, int(os.environ.get("KB_OVERLAP", "1")))
 if int(os.environ.get("KB_LOOPBACK", "0")):   # same-rank copies through NCCL (multi-rank exchange code)
     cc.crocco_set_nccl_loopback(S.ctx, True)
-xyz = torch.from_numpy(grid.coords(n, (0, 0, 0), 10)).cuda()
-S.set_coords([xyz]); S.set_state([synth.tgv(xyz, noise=0.01, seed=5)]); del xyz
+for b in range(S.nloc):
+    L = S.layouts[b]
+    xyz = torch.from_numpy(grid.coords(tuple(L.n), tuple(L.origin), 10)).cuda()
+    S.set_coords_block(b, xyz); S.set_state_block(b, synth.tgv(xyz, noise=0.01, seed=5)); del xyz
 for s in range(3): S.stage(s, 2e-4)
 torch.cuda.synchronize()
 REPS = int(os.environ.get("KB_REPS", "3"))
@@ -36,8 +40,7 @@ for rep in range(REPS):
         if v[0]:
             best_k[k] = min(best_k.get(k, 1e30), v[1] / v[0])
 tot = best
-out = {"lib": os.path.basename(cc.LIB_PATH), "overlap": os.environ.get("KB_OVERLAP", "1"), "loopback": os.environ.get("KB_LOOPBACK", "0"), "weno_limiter": os.environ.get("KB_LIM", "0"), "visc_form": os.environ.get("KB_VISC_FORM", "0"), "ms_per_stage": tot, "pts_stage_per_s": N ** 3 / tot * 1e3,
+out = {"lib": os.path.basename(cc.LIB_PATH), "overlap": os.environ.get("KB_OVERLAP", "1"), "loopback": os.environ.get("KB_LOOPBACK", "0"), "weno_limiter": os.environ.get("KB_LIM", "0"), "visc_form": os.environ.get("KB_VISC_FORM", "0"), "blocks": NB, "ms_per_stage": tot, "pts_stage_per_s": n[0] * n[1] * n[2] / tot * 1e3,
        "kernels_ms": {k: round(v, 3) for k, v in best_k.items()}}
-U = S.view(S.U[0], 0, 5)[:, 4:-4, 4:-4, 4:-4]
-out["finite"] = bool(torch.isfinite(U).all().item())
+out["finite"] = all(bool(torch.isfinite(S.view(S.U[b], b, 5)[:, 4:-4, 4:-4, 4:-4]).all().item()) for b in range(S.nloc))
 print(json.dumps(out), flush=True)
