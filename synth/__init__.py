@@ -26,14 +26,23 @@ GC = 10
 
 # ---------------------------------------------------------------- grids
 
-def _index_grids(n, origin, g):
+def _index_grids(n, origin, g, device=None):
     """Global index arrays (float64) for the padded box of a block, as mutually
-    broadcastable arrays I (1,1,P0), J (1,P1,1), K (P2,1,1)."""
-    ax = [np.arange(origin[d] - g, origin[d] + n[d] + g, dtype=np.float64) for d in range(3)]
+    broadcastable arrays I (1,1,P0), J (1,P1,1), K (P2,1,1); torch tensors on
+    ``device`` when given (device-side generation of very large blocks)."""
+    if device is not None:
+        import torch
+        ax = [torch.arange(origin[d] - g, origin[d] + n[d] + g, dtype=torch.float64, device=device)
+              for d in range(3)]
+    else:
+        ax = [np.arange(origin[d] - g, origin[d] + n[d] + g, dtype=np.float64) for d in range(3)]
     return ax[0][None, None, :], ax[1][None, :, None], ax[2][:, None, None]
 
 
 def _stack3(a, b, c):
+    if type(a).__module__.startswith("torch"):
+        import torch
+        return torch.stack(torch.broadcast_tensors(a, b, c))
     shape = np.broadcast_shapes(np.shape(a), np.shape(b), np.shape(c))
     out = np.empty((3,) + shape)
     out[0], out[1], out[2] = a, b, c
@@ -68,17 +77,18 @@ class Wavy3D:
     k: float = 2 * math.pi * 2 / 10.0
     A: float = 0.3 / (2 * math.pi * 2 / 10.0)
 
-    def coords(self, n, origin=(0, 0, 0), g=GC):
-        return self.map(*_index_grids(n, origin, g))
+    def coords(self, n, origin=(0, 0, 0), g=GC, device=None):
+        return self.map(*_index_grids(n, origin, g, device))
 
     def map(self, I, J, K):
+        xp = _xp(I)
         xi = self.x0[0] + I * self.L[0] / self.N[0]
         et = self.x0[1] + J * self.L[1] / self.N[1]
         ze = self.x0[2] + K * self.L[2] / self.N[2]
         k, A = self.k, self.A
-        return _stack3(xi + A * np.sin(k * et) * np.sin(k * ze),
-                       et + A * np.sin(k * ze) * np.sin(k * xi),
-                       ze + A * np.sin(k * xi) * np.sin(k * et))
+        return _stack3(xi + A * xp.sin(k * et) * xp.sin(k * ze),
+                       et + A * xp.sin(k * ze) * xp.sin(k * xi),
+                       ze + A * xp.sin(k * xi) * xp.sin(k * et))
 
 
 @dataclass
@@ -413,9 +423,12 @@ def case(name: str, scale: int = 1) -> Case:
         bc, _, _ = dmr_bc(h)
         return Case("dmr", N, (2, 2, 1) if scale < 8 else (1, 1, 1), bc, Cartesian(h=(h, h, h)), "dmr",
                     dict(gamma=1.4, R=1.0, terms=1), dt=0.2 * h / 13.0, steps=100)
-    if name == "weak":
-        N = 512 // scale
-        return Case("weak", (N, N, N), (1, 1, 1), ((P, P),) * 3,
+    if name in ("weak", "weak_max"):
+        # weak_max: the largest weak-recipe cube tested in one block (768^3, 139 GB of device
+        # buffers): its state arrays hold 2.3e9 and its metric arrays 4.7e9 elements, so element
+        # offsets pass 2^31 (int64 indexing); a parity case, not a bench line
+        N = (512 if name == "weak" else 768) // scale
+        return Case(name, (N, N, N), (1, 1, 1), ((P, P),) * 3,
                     Wavy3D(L=(2 * math.pi,) * 3, N=(N, N, N), x0=(-math.pi,) * 3, k=2.0, A=0.3 / 2.0),
                     "tgv_noise", dict(gamma=1.4, R=1.0, Pr=0.71, mu_ref=1.0 / 1600.0),
                     dt=2e-4 * scale, steps=100)

@@ -328,11 +328,13 @@ def _block_points(bn, rng, k_random):
 
 
 @pytest.mark.slow
-@pytest.mark.parametrize("name", ["weak", "ramp", "tgv", "dmr"])
+@pytest.mark.parametrize("name", ["weak", "ramp", "tgv", "dmr", "weak_max"])
 def test_full_size_config_sampled(name):
     """BASELINE.json full sizes in bench.py's launch configuration (crocco_rk_stage):
     weak = 512^3 periodic wavy TGV (configs[4]); ramp = 1024 x 512 x 256 Mach-6
-    ramp in 2 x 2 x 2 blocks with walls (configs[3]).  Stages 0 and 1; sampled
+    ramp in 2 x 2 x 2 blocks with walls (configs[3]); weak_max = the weak recipe at 768^3
+    in one block, the maximum-size case (element offsets past 2^31 in every state and
+    metric array; corners and faces of the block are among the sampled points).  Stages 0 and 1; sampled
     points recomputed by the oracle one by one from the GPU's filled 9^3
     neighbourhood of U (plus the stage-1 dU) and the ORACLE's metrics of that
     neighbourhood, computed from the generator's coordinates around the point
@@ -349,15 +351,32 @@ def test_full_size_config_sampled(name):
         bc, dirichlet, split = synth.dmr_bc(1.0 / n[1])
     S = Solver(n, c.n_blocks, bc, cc.make_phys(**c.phys), dirichlet=dirichlet, split=split)
     bn, blocks = block_slices(n, c.n_blocks)
-    xyz = []
-    U0 = []
-    for o, _ in blocks:
-        x, u = synth.block_inputs(c, o, bn)
-        xyz.append(x)
-        U0.append(u)
-    S.set_coords(xyz)
-    S.set_state(U0)
-    del xyz, U0
+    # weak, weak_max (one block each): coordinates and state generated on the device (the same
+    # generator formulas through torch; numpy takes minutes at 768^3); the oracle's metric
+    # windows below then come from the same device path, so both sides see identical coordinates
+    dev = "cuda" if name in ("weak", "weak_max") else None
+    if dev:
+        import torch
+        x = c.grid.coords(bn, blocks[0][0], oracle.GC, device=dev).cpu()  # host copy: InitGridMetrics
+        torch.cuda.empty_cache()                                             # needs 35 GB of scratch
+        S.set_coords_block(0, x)
+        del x
+        Uv = S.view(S.U[0], 0, 5)
+        for k0 in range(0, bn[2], 64):  # the state in k slabs (pointwise in the coordinates)
+            ks = min(64, bn[2] - k0)
+            xs = c.grid.coords((bn[0], bn[1], ks), (0, 0, k0), oracle.GC, device=dev)
+            Uv[:, 4 + k0:4 + k0 + ks, 4:-4, 4:-4].copy_(synth.tgv(xs, noise=0.01, seed=5))
+        del xs, Uv
+    else:
+        xyz = []
+        U0 = []
+        for o, _ in blocks:
+            x, u = synth.block_inputs(c, o, bn)
+            xyz.append(x)
+            U0.append(u)
+        S.set_coords(xyz)
+        S.set_state(U0)
+        del xyz, U0
     rng = np.random.default_rng(0)
     per_block = max(8, 64 // len(blocks))
     pts = [(b, p) for b in range(len(blocks)) for p in _block_points(bn, rng, per_block)]
@@ -368,7 +387,9 @@ def test_full_size_config_sampled(name):
     for b, p in pts:
         o = blocks[b][0]
         gp = (o[0] + p[0], o[1] + p[1], o[2] + p[2])
-        Mo[(b, p)] = oracle.metrics((1, 1, 1), EXT, c.grid.coords((1, 1, 1), gp, oracle.GC))
+        xw = c.grid.coords((1, 1, 1), gp, oracle.GC, device=dev).cpu().numpy() if dev else \
+            c.grid.coords((1, 1, 1), gp, oracle.GC)
+        Mo[(b, p)] = oracle.metrics((1, 1, 1), EXT, xw)
         sl = (slice(None), slice(p[2], p[2] + 9), slice(p[1], p[1] + 9), slice(p[0], p[0] + 9))
         Mg = S.view(S.met[b], b, 10)[sl].cpu().numpy()
         ref = Mo[(b, p)]
