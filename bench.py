@@ -278,7 +278,10 @@ def run_crocco(args, rank, world, local_rank):
         origin, bn = tuple(L.origin), tuple(L.n)
         if case.state in ("tgv", "tgv_noise"):
             # generated on the device (torch ops on the synth formulas) -- input setup only
-            xyz = torch.from_numpy(grid.coords(bn, origin, cc.GHOST_COORDS)).to(dev)
+            if isinstance(grid, synth.Wavy3D):
+                xyz = grid.coords(bn, origin, cc.GHOST_COORDS, device=dev)
+            else:
+                xyz = torch.from_numpy(grid.coords(bn, origin, cc.GHOST_COORDS)).to(dev)
             U0 = synth.tgv(xyz, noise=0.01 if case.state == "tgv_noise" else 0.0, seed=5)
         else:
             xyz, U0 = synth.block_inputs(case, origin, bn)
