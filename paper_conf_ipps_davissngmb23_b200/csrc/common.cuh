@@ -96,7 +96,7 @@ __device__ __forceinline__ void cp_async16(double *dst, const double *src) {
 __device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commit_group;\n" ::: "memory"); }
 __device__ __forceinline__ void cp_async_wait_all() { asm volatile("cp.async.wait_group 0;\n" ::: "memory"); }
 
-// primitive buffer components (k_prims)
+// primitive components staged per ring point by the sweeps (sweep.cuh)
 // (PIS = 1/sqrt(rho): the Roe weights use sqrt(rho) = rho / sqrt(rho), 1/rho~ = PIS_L PIS_R)
 enum { PU = 0, PV = 1, PW = 2, PP = 3, PC = 4, PIS = 5, PH = 6 };
 

@@ -48,7 +48,7 @@ struct SweepArgs {
 };
 
 // ---------------------------------------------------------------------------
-// Shared-memory staged sweep (same tiles and arithmetic as k_sweep): each warp
+// Shared-memory staged sweep: each warp
 // keeps a ring of its stencil window in shared memory -- conserved state and
 // metric row copied with cp.async one step ahead of use, primitives computed
 // once per point when it enters the ring -- so the characteristic WENO reads
