@@ -203,11 +203,29 @@ __global__ void __launch_bounds__(WS_THREADS, 1) k_sweep_ws(const __grid_constan
         double *sv0 = smem_dyn + (size_t)p * RG::PER_WARP, *sv1 = smem_dyn + (size_t)(p + WS_PROD) * RG::PER_WARP;
         uint64_t *b0 = bars + p * 2 * NSLOT, *b1 = bars + (p + WS_PROD) * 2 * NSLOT;
         const int nm = max(n0, n1);
-        if (0 < n0) ws_issue<D, VISC>(a, L, g0, sv0, lane, 0);
-        if (0 < n1) ws_issue<D, VISC>(a, L, g1, sv1, lane, 0);
-        cp_async_commit();
+        // second version: K chunks in flight; the primitives of chunk ch are published BEFORE
+        // waiting for the slot of chunk ch + K (released by consumer step ch + K - NSLOT <= ch - LA - 1)
+        constexpr int K = NSLOT - LA - 1;
+        static_assert(K >= 1 && K <= 2, "lookahead");
+#pragma unroll
+        for (int c = 0; c < K; c++) {
+            if (c < n0) ws_issue<D, VISC>(a, L, g0, sv0, lane, c);
+            if (c < n1) ws_issue<D, VISC>(a, L, g1, sv1, lane, c);
+            cp_async_commit();
+        }
         for (int ch = 0; ch < nm; ch++) {
-            const int nx = ch + 1, s = nx % NSLOT;
+            if constexpr (K == 1) asm volatile("cp.async.wait_group 0;\n" ::: "memory");  // chunk ch landed
+            else asm volatile("cp.async.wait_group 1;\n" ::: "memory");
+            __syncwarp();
+            if (ch < n0) {
+                ws_prims<D, VISC>(ph, g0, sv0, lane, ch);
+                mbar_arrive(b0 + ch % NSLOT);
+            }
+            if (ch < n1) {
+                ws_prims<D, VISC>(ph, g1, sv1, lane, ch);
+                mbar_arrive(b1 + ch % NSLOT);
+            }
+            const int nx = ch + K, s = nx % NSLOT;
             const unsigned par = ((unsigned)(nx / NSLOT) + 1u) & 1u;  // completion nx/NSLOT - 1 of empty[s]
             if (nx < n0) {
                 if (nx >= NSLOT) mbar_wait(b0 + NSLOT + s, par);
@@ -218,16 +236,6 @@ __global__ void __launch_bounds__(WS_THREADS, 1) k_sweep_ws(const __grid_constan
                 ws_issue<D, VISC>(a, L, g1, sv1, lane, nx);
             }
             cp_async_commit();
-            asm volatile("cp.async.wait_group 1;\n" ::: "memory");  // chunk ch landed
-            __syncwarp();
-            if (ch < n0) {
-                ws_prims<D, VISC>(ph, g0, sv0, lane, ch);
-                mbar_arrive(b0 + ch % NSLOT);
-            }
-            if (ch < n1) {
-                ws_prims<D, VISC>(ph, g1, sv1, lane, ch);
-                mbar_arrive(b1 + ch % NSLOT);
-            }
         }
         cp_async_wait_all();
         return;
