@@ -11,7 +11,9 @@
 //   folded: W(v/2; eps) = W(v; 4 eps)/2, so the sum is halved at the end],
 //   F^ = |m^| T g^.
 // L_s.F_n(U_l) is evaluated as theta_l (L_s.U_l) + p_l k_{s,l} using the exact
-// identity F_n(U) = theta U + p (0, n, theta).
+// identity F_n(U) = theta U + p (0, n, theta); for the entropy / vorticity fields
+// (k = ng (theta~ - theta_l)) the per-point products pm_l = p_l (theta~ - theta_l) are formed once
+// and shared by the three fields (acoustic fields first in the field loop).
 // Viscous part: with the point fluxes f = F^_v^d (k_visc),
 //   h_{i+1/2} = [7(f_i + f_{i+1}) - (f_{i-1} + f_{i+2})]/12,
 //   h_{i+1/2} - h_{i-1/2} = D4 f_i  (exactly, in exact arithmetic).
@@ -169,7 +171,14 @@ __device__ __forceinline__ void flux_fields(const Acc &A, const FluxSetup &su, b
         // inside the loop measured slower); the loop is unrolled (rolled: +14 %)
         double gb[5], gn[5], gd[5];
 #pragma unroll
-        for (int sf = 0; sf < 5; sf++) {
+        for (int it = 0; it < 5; it++) {
+            // acoustic fields first; then p_l becomes pm_l = p_l (theta~ - theta_l), so the
+            // entropy / vorticity fields' p_l (kB theta_l + kA) = ng pm_l (kA = ng theta~, kB = -ng)
+            const int sf = it < 2 ? it + 3 : it - 2;
+            if (it == 2) {
+#pragma unroll
+                for (int l = 0; l < 6; l++) pl[l] *= tht - th[l];
+            }
             double L0, L1, L2, L3, L4, R0, R1, R2, R3, R4, lam, kA, kB;
             if (sf < 3) {
                 const double na = sf == 0 ? nx : (sf == 1 ? ny : nz);
@@ -228,7 +237,7 @@ __device__ __forceinline__ void flux_fields(const Acc &A, const FluxSetup &su, b
             for (int l = 0; l < 6; l++) {
                 const double w =
                     fma(L0, UL(l, 0), fma(L1, UL(l, 1), fma(L2, UL(l, 2), fma(L3, UL(l, 3), L4 * UL(l, 4)))));
-                const double g = fma(th[l], w, pl[l] * fma(kB, th[l], kA));
+                const double g = sf < 3 ? fma(th[l], w, -kB * pl[l]) : fma(th[l], w, pl[l] * fma(kB, th[l], kA));
                 gp[l] = fma(lam, w, g);
                 gm[l] = fma(-lam, w, g);
             }
@@ -240,7 +249,7 @@ __device__ __forceinline__ void flux_fields(const Acc &A, const FluxSetup &su, b
         }
 #pragma unroll
         for (int sf = 0; sf < 5; sf++) {
-            const double gh = gb[sf] + div_nr(gn[sf], gd[sf]);
+            const double gh = fma(div_nr(gn[sf], gd[sf]), 1.0 / 6.0, gb[sf]);
             double R0, R1, R2, R3, R4;
             if (sf < 3) {
                 const double na = sf == 0 ? nx : (sf == 1 ? ny : nz);

@@ -95,7 +95,8 @@ __device__ __forceinline__ WenoFrac weno_symbo_frac(double v0, double v1, double
 }
 
 // W^+ of (vp0..vp5) plus W^- of the mirrored (vm5..vm0), as one fraction:
-// (b+ + b-) + (n+ d- + n- d+)/(6 d+ d-)  -- one division per characteristic field.
+// (b+ + b-) + [(n+ d- + n- d+)/(d+ d-)]/6  -- one division per characteristic field; the pair's
+// den is d+ d- (the 1/6 enters the caller's final FMA, one multiply less than 6 (d+ d-)).
 // Range: the alpha products stay inside fp64 for |v| up to ~1e9.
 template <bool LIM = false>
 __device__ __forceinline__ WenoFrac weno_pair_frac(const double vp[6], const double vm[6], double eps_b,
@@ -105,14 +106,14 @@ __device__ __forceinline__ WenoFrac weno_pair_frac(const double vp[6], const dou
     WenoFrac w;
     w.base = a.base + b.base;
     w.num = fma(a.num, b.den, b.num * a.den);
-    w.den = 6.0 * (a.den * b.den);
+    w.den = a.den * b.den;  // the 1/6 is applied by the caller: W = base + (num/den)/6
     return w;
 }
 template <bool LIM = false>
 __device__ __forceinline__ double weno_pair(const double vp[6], const double vm[6], double eps_b,
                                             const double C[4], const Phys *lp = nullptr) {
     const WenoFrac w = weno_pair_frac<LIM>(vp, vm, eps_b, C, lp);
-    return w.base + div_nr(w.num, w.den);
+    return fma(div_nr(w.num, w.den), 1.0 / 6.0, w.base);
 }
 
 }  // namespace crocco
