@@ -247,42 +247,29 @@ __device__ __forceinline__ void flux_fields(const Acc &A, const FluxSetup &su, b
             gd[sf] = wf.den;
             (void)R0; (void)R1; (void)R2; (void)R3; (void)R4;
         }
+        double gh[5];
 #pragma unroll
-        for (int sf = 0; sf < 5; sf++) {
-            const double gh = fma(div_nr(gn[sf], gd[sf]), 1.0 / 6.0, gb[sf]);
-            double R0, R1, R2, R3, R4;
-            if (sf < 3) {
-                const double na = sf == 0 ? nx : (sf == 1 ? ny : nz);
-                R0 = na;
-                if (sf == 0) {
-                    R1 = na * ut;
-                    R2 = fma(na, vt, nz * rt);
-                    R3 = fma(na, wt, -ny * rt);
-                    R4 = fma(na, ph1, rt * (nz * vt - ny * wt));
-                } else if (sf == 1) {
-                    R1 = fma(na, ut, -nz * rt);
-                    R2 = na * vt;
-                    R3 = fma(na, wt, nx * rt);
-                    R4 = fma(na, ph1, rt * (nx * wt - nz * ut));
-                } else {
-                    R1 = fma(na, ut, ny * rt);
-                    R2 = fma(na, vt, -nx * rt);
-                    R3 = na * wt;
-                    R4 = fma(na, ph1, rt * (ny * ut - nx * vt));
-                }
-            } else {
-                const double sc = (sf == 3) ? ct : -ct;
-                R0 = alph;
-                R1 = alph * fma(sc, nx, ut);
-                R2 = alph * fma(sc, ny, vt);
-                R3 = alph * fma(sc, nz, wt);
-                R4 = alph * fma(phi2 + c2, ph.igm1, sc * tht);
-            }
-            f0 = fma(R0, gh, f0);
-            f1 = fma(R1, gh, f1);
-            f2 = fma(R2, gh, f2);
-            f3 = fma(R3, gh, f3);
-            f4 = fma(R4, gh, f4);
+        for (int sf = 0; sf < 5; sf++) gh[sf] = fma(div_nr(gn[sf], gd[sf]), 1.0 / 6.0, gb[sf]);
+        // back projection F^/|m^| = sum_s gh_s R_s in closed form (the right eigenvectors R_s of
+        // the columns written out above, summed symbolically):
+        //   entropy / vorticity fields, G = (gh_0, gh_1, gh_2), s = n.G, c = rho~ (n x G):
+        //     (s, u~ s + c, |u~|^2/2 s + u~.c)
+        //   acoustic pair, S = alpha (gh_3 + gh_4), Dd = alpha c~ (gh_3 - gh_4):
+        //     S (1, u~, H~) + Dd (0, n, n.u~),  H~ = (phi2 + c~^2)/(gamma-1)
+        {
+            const double sG = fma(nx, gh[0], fma(ny, gh[1], nz * gh[2]));
+            const double cgx = rt * fma(ny, gh[2], -nz * gh[1]);
+            const double cgy = rt * fma(nz, gh[0], -nx * gh[2]);
+            const double cgz = rt * fma(nx, gh[1], -ny * gh[0]);
+            const double S = alph * (gh[3] + gh[4]);
+            const double Dd = (alph * ct) * (gh[3] - gh[4]);
+            const double Ht = (phi2 + c2) * ph.igm1;
+            const double sS = sG + S;
+            f0 = sS;
+            f1 = fma(ut, sS, fma(Dd, nx, cgx));
+            f2 = fma(vt, sS, fma(Dd, ny, cgy));
+            f3 = fma(wt, sS, fma(Dd, nz, cgz));
+            f4 = fma(ph1, sG, fma(ut, cgx, fma(vt, cgy, fma(wt, cgz, fma(S, Ht, Dd * tht)))));
         }
 #undef UL
         F[0] = hmag * f0;
