@@ -72,8 +72,7 @@ struct SAcc {
 struct FluxSetup {
     double nx, ny, nz, hmag;           // unit normal, |m^|/2 (LLF 1/2 folded here)
     double ut, vt, wt, rt, irt;        // Roe velocity, density and its reciprocal
-    double ct, c2, ic2, tht, phi2;     // Roe sound speed, c^2, 1/c^2, n.u~, (gamma-1)|u~|^2/2
-    double alph, beta;                 // rho/(sqrt2 c), 1/(sqrt2 rho c)
+    double ct, c2, ic2, ict, tht, phi2;  // Roe sound speed, c^2, 1/c^2, 1/c, n.u~, (gamma-1)|u~|^2/2
 };
 template <class Acc>
 __device__ __forceinline__ void flux_setup(const Acc &A, const Phys &ph, FluxSetup &su) {
@@ -105,7 +104,6 @@ __device__ __forceinline__ void flux_setup(const Acc &A, const Phys &ph, FluxSet
     const double c2 = gm1 * fma(-0.5, q2, Ht);
     const double ict = rsqrt_nr(c2);
     const double irt = isL * isR;  // 1/rho~
-    constexpr double SQ12 = 0.70710678118654752440;
     su.ut = ut;
     su.vt = vt;
     su.wt = wt;
@@ -116,8 +114,7 @@ __device__ __forceinline__ void flux_setup(const Acc &A, const Phys &ph, FluxSet
     su.ic2 = ict * ict;
     su.tht = fma(nx, ut, fma(ny, vt, nz * wt));
     su.phi2 = 0.5 * gm1 * q2;
-    su.alph = rt * ict * SQ12;
-    su.beta = irt * ict * SQ12;
+    su.ict = ict;
 }
 
 // Total interface flux F = F^_inv - h_v of direction D at interface i+1/2 from the setup above.
@@ -130,8 +127,7 @@ __device__ __forceinline__ void flux_fields(const Acc &A, const FluxSetup &su, b
         const double gm1 = ph.gm1;
         const double nx = su.nx, ny = su.ny, nz = su.nz, hmag = su.hmag;
         const double ut = su.ut, vt = su.vt, wt = su.wt, rt = su.rt, irt = su.irt;
-        const double ct = su.ct, c2 = su.c2, ic2 = su.ic2, tht = su.tht, phi2 = su.phi2;
-        const double alph = su.alph, beta = su.beta;
+        const double ct = su.ct, c2 = su.c2, ic2 = su.ic2, ict = su.ict, tht = su.tht, phi2 = su.phi2;
 
         // stencil points (the states are re-read from the ring per field: holding the 6 x 5
         // states in registers measured slower)
@@ -162,6 +158,11 @@ __device__ __forceinline__ void flux_fields(const Acc &A, const FluxSetup &su, b
             lam4 = maxnn(maxnn(maxnn(a4[0], a4[1]), maxnn(a4[2], a4[3])), maxnn(a4[4], a4[5]));
         }
         const double eps_b = 4.0 * WENO_BSCALE * ph.eps;  // b-units (weno.cuh) x 4 (folded 1/2)
+        // acoustic rows are used as L_s / beta, beta = 1/(sqrt2 rho~ c~): W is homogeneous,
+        // W(v; eps) = beta W(v / beta; eps / beta^2), so those fields take eps (and the absolute
+        // limiter threshold) times 1/beta^2 = 2 rho~^2 c~^2; the factor beta returns in the back projection
+        const double ib2 = (2.0 * rt * rt) * c2;
+        const double epsA = eps_b * ib2;
         const double onemp = fma(-phi2, ic2, 1.0);
         const double gic2 = gm1 * ic2;
         const double cx = ny * wt - nz * vt, cy = nz * ut - nx * wt, cz = nx * vt - ny * ut;
@@ -179,7 +180,7 @@ __device__ __forceinline__ void flux_fields(const Acc &A, const FluxSetup &su, b
 #pragma unroll
                 for (int l = 0; l < 6; l++) pl[l] *= tht - th[l];
             }
-            double L0, L1, L2, L3, L4, R0, R1, R2, R3, R4, lam, kA, kB;
+            double L0, L1, L2, L3, L4, lam, kA, kB;
             if (sf < 3) {
                 const double na = sf == 0 ? nx : (sf == 1 ? ny : nz);
                 const double cr = sf == 0 ? cx : (sf == 1 ? cy : cz);
@@ -189,48 +190,29 @@ __device__ __forceinline__ void flux_fields(const Acc &A, const FluxSetup &su, b
                     L1 = ng * ut;
                     L2 = fma(nz, irt, ng * vt);
                     L3 = fma(-ny, irt, ng * wt);
-                    R1 = na * ut;
-                    R2 = fma(na, vt, nz * rt);
-                    R3 = fma(na, wt, -ny * rt);
-                    R4 = fma(na, ph1, rt * (nz * vt - ny * wt));
                 } else if (sf == 1) {
                     L1 = fma(-nz, irt, ng * ut);
                     L2 = ng * vt;
                     L3 = fma(nx, irt, ng * wt);
-                    R1 = fma(na, ut, -nz * rt);
-                    R2 = na * vt;
-                    R3 = fma(na, wt, nx * rt);
-                    R4 = fma(na, ph1, rt * (nx * wt - nz * ut));
                 } else {
                     L1 = fma(ny, irt, ng * ut);
                     L2 = fma(-nx, irt, ng * vt);
                     L3 = ng * wt;
-                    R1 = fma(na, ut, ny * rt);
-                    R2 = fma(na, vt, -nx * rt);
-                    R3 = na * wt;
-                    R4 = fma(na, ph1, rt * (ny * ut - nx * vt));
                 }
                 L4 = -ng;
-                R0 = na;
                 lam = lam0;
                 kA = ng * tht;
                 kB = -ng;
             } else {
-                const double sg = (sf == 3) ? 1.0 : -1.0;
-                const double sc = sg * ct;
-                L0 = beta * fma(-sc, tht, phi2);
-                L1 = beta * fma(sc, nx, -gm1 * ut);
-                L2 = beta * fma(sc, ny, -gm1 * vt);
-                L3 = beta * fma(sc, nz, -gm1 * wt);
-                L4 = beta * gm1;
-                R0 = alph;
-                R1 = alph * fma(sc, nx, ut);
-                R2 = alph * fma(sc, ny, vt);
-                R3 = alph * fma(sc, nz, wt);
-                R4 = alph * fma(phi2 + c2, ph.igm1, sc * tht);
+                const double sc = (sf == 3) ? ct : -ct;
+                L0 = fma(-sc, tht, phi2);
+                L1 = fma(sc, nx, -gm1 * ut);
+                L2 = fma(sc, ny, -gm1 * vt);
+                L3 = fma(sc, nz, -gm1 * wt);
+                L4 = gm1;
                 lam = (sf == 3) ? lam3 : lam4;
-                kA = beta * fma(-gm1, tht, sc);
-                kB = beta * gm1;
+                kA = fma(-gm1, tht, sc);
+                kB = gm1;
             }
             double gp[6], gm[6];
 #pragma unroll
@@ -241,11 +223,11 @@ __device__ __forceinline__ void flux_fields(const Acc &A, const FluxSetup &su, b
                 gp[l] = fma(lam, w, g);
                 gm[l] = fma(-lam, w, g);
             }
-            const WenoFrac wf = weno_pair_frac<LIM>(gp, gm, eps_b, ph.wC, &ph);
+            const WenoFrac wf = sf < 3 ? weno_pair_frac<LIM>(gp, gm, eps_b, ph.wC, &ph, ph.aal_b)
+                                       : weno_pair_frac<LIM>(gp, gm, epsA, ph.wC, &ph, ph.aal_b * ib2);
             gb[sf] = wf.base;
             gn[sf] = wf.num;
             gd[sf] = wf.den;
-            (void)R0; (void)R1; (void)R2; (void)R3; (void)R4;
         }
         double gh[5];
 #pragma unroll
@@ -254,15 +236,16 @@ __device__ __forceinline__ void flux_fields(const Acc &A, const FluxSetup &su, b
         // the columns written out above, summed symbolically):
         //   entropy / vorticity fields, G = (gh_0, gh_1, gh_2), s = n.G, c = rho~ (n x G):
         //     (s, u~ s + c, |u~|^2/2 s + u~.c)
-        //   acoustic pair, S = alpha (gh_3 + gh_4), Dd = alpha c~ (gh_3 - gh_4):
+        //   acoustic pair, S = alpha (gh_3 + gh_4), Dd = alpha c~ (gh_3 - gh_4), with alpha = rho~/(sqrt2 c~)
+        //   and gh_{3,4} = beta x (the values computed from L_s / beta): alpha beta = 1/(2 c~^2):
         //     S (1, u~, H~) + Dd (0, n, n.u~),  H~ = (phi2 + c~^2)/(gamma-1)
         {
             const double sG = fma(nx, gh[0], fma(ny, gh[1], nz * gh[2]));
             const double cgx = rt * fma(ny, gh[2], -nz * gh[1]);
             const double cgy = rt * fma(nz, gh[0], -nx * gh[2]);
             const double cgz = rt * fma(nx, gh[1], -ny * gh[0]);
-            const double S = alph * (gh[3] + gh[4]);
-            const double Dd = (alph * ct) * (gh[3] - gh[4]);
+            const double S = (0.5 * ic2) * (gh[3] + gh[4]);
+            const double Dd = (0.5 * ict) * (gh[3] - gh[4]);
             const double Ht = (phi2 + c2) * ph.igm1;
             const double sS = sG + S;
             f0 = sS;

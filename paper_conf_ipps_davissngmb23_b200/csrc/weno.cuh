@@ -30,11 +30,13 @@ struct WenoFrac {
 // downwind-stencil rule is unchanged.
 // LIM: the limiters of reading 23 (ph.lim / ph.arl / ph.aal_b, common.cuh): linear weights
 // alpha_k = C_k when max b < arl min b (bit 0) or max b < aal_b (bit 1), b after the
-// downwind substitution
+// downwind substitution; aal: the absolute threshold in the units of b of the values passed (the
+// caller scales it with the values, see flux.cuh)
 template <bool LIM = false>
 __device__ __forceinline__ WenoFrac weno_symbo_frac(double v0, double v1, double v2, double v3,
                                                     double v4, double v5, double eps_b,
-                                                    const double C[4], const Phys *lp = nullptr) {
+                                                    const double C[4], const Phys *lp = nullptr,
+                                                    double aal = 0.0) {
     const double C0 = C[0], C1 = C[1], C2 = C[2], C3 = C[3];
     constexpr double K3 = 3.0 / 13.0;
     const double d0 = v1 - v0, d1 = v2 - v1, d2 = v3 - v2, d3 = v4 - v3, d4 = v5 - v4;
@@ -56,7 +58,7 @@ __device__ __forceinline__ WenoFrac weno_symbo_frac(double v0, double v1, double
         double b3 = fma(K3 * f3, f3, s3 * s3);
         b3 = maxnn(maxnn(b0, b1), maxnn(b2, b3));
         const double bmin = minnn(minnn(b0, b1), b2);  // b3 is the maximum
-        lin = ((lp->lim & 1) && b3 < lp->arl * bmin) || ((lp->lim & 2) && b3 < lp->aal_b);
+        lin = ((lp->lim & 1) && b3 < lp->arl * bmin) || ((lp->lim & 2) && b3 < aal);
         e0 = eps_b + b0;
         e1 = eps_b + b1;
         e2 = eps_b + b2;
@@ -100,20 +102,13 @@ __device__ __forceinline__ WenoFrac weno_symbo_frac(double v0, double v1, double
 // Range: the alpha products stay inside fp64 for |v| up to ~1e9.
 template <bool LIM = false>
 __device__ __forceinline__ WenoFrac weno_pair_frac(const double vp[6], const double vm[6], double eps_b,
-                                                   const double C[4], const Phys *lp = nullptr) {
-    const WenoFrac a = weno_symbo_frac<LIM>(vp[0], vp[1], vp[2], vp[3], vp[4], vp[5], eps_b, C, lp);
-    const WenoFrac b = weno_symbo_frac<LIM>(vm[5], vm[4], vm[3], vm[2], vm[1], vm[0], eps_b, C, lp);
+                                                   const double C[4], const Phys *lp = nullptr, double aal = 0.0) {
+    const WenoFrac a = weno_symbo_frac<LIM>(vp[0], vp[1], vp[2], vp[3], vp[4], vp[5], eps_b, C, lp, aal);
+    const WenoFrac b = weno_symbo_frac<LIM>(vm[5], vm[4], vm[3], vm[2], vm[1], vm[0], eps_b, C, lp, aal);
     WenoFrac w;
     w.base = a.base + b.base;
     w.num = fma(a.num, b.den, b.num * a.den);
     w.den = a.den * b.den;  // the 1/6 is applied by the caller: W = base + (num/den)/6
     return w;
 }
-template <bool LIM = false>
-__device__ __forceinline__ double weno_pair(const double vp[6], const double vm[6], double eps_b,
-                                            const double C[4], const Phys *lp = nullptr) {
-    const WenoFrac w = weno_pair_frac<LIM>(vp, vm, eps_b, C, lp);
-    return fma(div_nr(w.num, w.den), 1.0 / 6.0, w.base);
-}
-
 }  // namespace crocco
