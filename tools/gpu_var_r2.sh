@@ -3,7 +3,7 @@ cd "${GRAFT_REPO_ROOT:-/root/repo}"; mkdir -p gpurun_out
 OUT=gpurun_out/${VAR_OUT:-variants_r2}.jsonl
 : > $OUT
 export KB_OVERLAP=0
-for r in 1 2; do
+for r in ${VAR_REPS:-1 2}; do
 for v in build/variants/libcrocco_*.so; do
   CROCCO_LIB=$PWD/$v timeout 300 python tools/kbench.py >> $OUT 2>> gpurun_out/variants.err
 done
