@@ -349,21 +349,24 @@ template <int D, bool V>
 static constexpr size_t sweep_smem_bytes() {
     return (size_t)(sweep_threads(D) / 32) * RingGeom<D, V>::PER_WARP * sizeof(double);
 }
-template <int D, bool V>
+template <int D, bool V, int MODE>
 static cudaError_t sweep_attr1() {
-    cudaError_t e = cudaFuncSetAttribute(k_sweep_s<D, V, false>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+    cudaError_t e = cudaFuncSetAttribute(k_sweep_s<D, V, false, MODE>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                          (int)sweep_smem_bytes<D, V>());
     if (e == cudaSuccess)
-        e = cudaFuncSetAttribute(k_sweep_s<D, V, true>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+        e = cudaFuncSetAttribute(k_sweep_s<D, V, true, MODE>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                  (int)sweep_smem_bytes<D, V>());
     return e;
 }
 static cudaError_t sweep_attrs() {
-    // the variants rhs_block launches: only the eta sweep carries a viscous interface term
-    cudaError_t e = sweep_attr1<0, false>();
-    if (e == cudaSuccess) e = sweep_attr1<1, false>();
-    if (e == cudaSuccess) e = sweep_attr1<2, false>();
-    if (e == cudaSuccess) e = sweep_attr1<1, true>();
+    // the variants rhs_block launches: only the eta sweep carries a viscous interface term; modes:
+    // xi 0 (write R) or 4 (add to the viscous divergence), eta 1 (add), zeta 2 (rhs) or 3 (RK update)
+    cudaError_t e = sweep_attr1<0, false, 0>();
+    if (e == cudaSuccess) e = sweep_attr1<0, false, 4>();
+    if (e == cudaSuccess) e = sweep_attr1<1, false, 1>();
+    if (e == cudaSuccess) e = sweep_attr1<1, true, 1>();
+    if (e == cudaSuccess) e = sweep_attr1<2, false, 2>();
+    if (e == cudaSuccess) e = sweep_attr1<2, false, 3>();
     if (e == cudaSuccess)
         e = cudaFuncSetAttribute(k_visc_tiled, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)VISC_SMEM);
     if (e == cudaSuccess)
@@ -1157,16 +1160,16 @@ static crocco_status rhs_block(crocco_ctx c, const LocalBlock &b, const double *
         a.seg = (int)seg;
         const int64_t warps = lines * ((nd + seg - 1) / seg);
         const unsigned grid = cdiv(warps * 32, sweep_threads(d));
-#define SWEEP_LAUNCH(DD, VV)                                                                              \
+#define SWEEP_LAUNCH(DD, VV, MM)                                                                          \
     do {                                                                                                  \
         if (ph.lim)                                                                                       \
-            k_sweep_s<DD, VV, true><<<grid, sweep_threads(DD), sweep_smem_bytes<DD, VV>(), c->stream>>>(a, b.L, ph);  \
+            k_sweep_s<DD, VV, true, MM><<<grid, sweep_threads(DD), sweep_smem_bytes<DD, VV>(), c->stream>>>(a, b.L, ph);  \
         else                                                                                              \
-            k_sweep_s<DD, VV, false><<<grid, sweep_threads(DD), sweep_smem_bytes<DD, VV>(), c->stream>>>(a, b.L, ph); \
+            k_sweep_s<DD, VV, false, MM><<<grid, sweep_threads(DD), sweep_smem_bytes<DD, VV>(), c->stream>>>(a, b.L, ph); \
     } while (0)
-        if (d == 0) LAUNCH(c, K_FLUX_X, SWEEP_LAUNCH(0, false));
-        else if (d == 1) LAUNCH(c, K_FLUX_Y, if (a.visc) SWEEP_LAUNCH(1, true); else SWEEP_LAUNCH(1, false));
-        else LAUNCH(c, K_FLUX_Z, SWEEP_LAUNCH(2, false));
+        if (d == 0) LAUNCH(c, K_FLUX_X, if (a.mode == 4) SWEEP_LAUNCH(0, false, 4); else SWEEP_LAUNCH(0, false, 0));
+        else if (d == 1) LAUNCH(c, K_FLUX_Y, if (a.visc) SWEEP_LAUNCH(1, true, 1); else SWEEP_LAUNCH(1, false, 1));
+        else LAUNCH(c, K_FLUX_Z, if (a.mode == 3) SWEEP_LAUNCH(2, false, 3); else SWEEP_LAUNCH(2, false, 2));
 #undef SWEEP_LAUNCH
     }
     return CROCCO_OK;

@@ -78,7 +78,9 @@ struct RingGeom {
     static constexpr int PER_WARP = SVN * VS + NCB * 32 + NFC;  // doubles
 };
 
-template <int D, bool VISC, bool LIM>
+// MODE = MODE as a template parameter: each launch compiles only its own accumulate / update
+// path (a run-time mode let every direction's kernel carry all five, and their register allocation)
+template <int D, bool VISC, bool LIM, int MODE>
 __global__ void __launch_bounds__(sweep_threads(D), sweep_minb(D)) k_sweep_s(const __grid_constant__ SweepArgs a,
                                                                           const Lay L, const Phys ph) {
     using RG = RingGeom<D, VISC>;
@@ -256,13 +258,13 @@ __global__ void __launch_bounds__(sweep_threads(D), sweep_minb(D)) k_sweep_s(con
         const bool act = lvalid && e <= e1 - 1;
         const bool own = act && e >= e0;      // this lane finishes point e
         const SAcc<NR, C, VISC, RG::CS> A{sv, WS * st + ls + RG::QOFF, lt};  // ring point of stencil point i-2
-        if (own && a.mode != 0) {             // group A: accumulate / update operands
+        if (own && MODE != 0) {             // group A: accumulate / update operands
 #pragma unroll
             for (int c = 0; c < 5; c++)
-                if (c > 0 || a.mode != 4) cp_async8(cb + 32 * c, a.R + c * a.rcs + rr);
-            if (a.mode == 2 || a.mode == 3) {  // J (the zeta sweep finishes the point)
+                if (c > 0 || MODE != 4) cp_async8(cb + 32 * c, a.R + c * a.rcs + rr);
+            if (MODE == 2 || MODE == 3) {  // J (the zeta sweep finishes the point)
                 cp_async8(cb + 32 * 5, a.in.M + pp);
-                if (a.mode == 3) {
+                if (MODE == 3) {
 #pragma unroll
                     for (int c = 0; c < 5; c++) {
                         if (a.stage != 0) cp_async8(cb + 32 * (6 + c), a.dU + c * L.cs + pp);
@@ -314,17 +316,17 @@ __global__ void __launch_bounds__(sweep_threads(D), sweep_minb(D)) k_sweep_s(con
         }
         asm volatile("cp.async.wait_group 1;\n" ::: "memory");  // group A landed (own data)
         if (own) {
-            if (a.mode == 0) {
+            if (MODE == 0) {
 #pragma unroll
                 for (int c = 0; c < 5; c++) a.R[c * a.rcs + rr] = dF[c];
             } else {
                 double Rt[5];
 #pragma unroll
-                for (int c = 0; c < 5; c++) Rt[c] = (c == 0 && a.mode == 4) ? dF[0] : cb[32 * c] + dF[c];
-                if (a.mode == 1 || a.mode == 4) {
+                for (int c = 0; c < 5; c++) Rt[c] = (c == 0 && MODE == 4) ? dF[0] : cb[32 * c] + dF[c];
+                if (MODE == 1 || MODE == 4) {
 #pragma unroll
                     for (int c = 0; c < 5; c++) a.R[c * a.rcs + rr] = Rt[c];
-                } else if (a.mode == 2) {
+                } else if (MODE == 2) {
                     const double J = cb[32 * 5];
 #pragma unroll
                     for (int c = 0; c < 5; c++) a.rhs[c * L.cs + pp] = J * Rt[c];
