@@ -354,7 +354,10 @@ static cudaError_t sweep_attr1() {
     cudaError_t e = cudaFuncSetAttribute(k_sweep_s<D, V, false, MODE>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                          (int)sweep_smem_bytes<D, V>());
     if (e == cudaSuccess)
-        e = cudaFuncSetAttribute(k_sweep_s<D, V, true, MODE>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+        e = cudaFuncSetAttribute(k_sweep_s<D, V, true, MODE, 2>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                 (int)sweep_smem_bytes<D, V>());
+    if (e == cudaSuccess)  // no inviscid term in this direction (dir_mask / terms): the limiter is moot
+        e = cudaFuncSetAttribute(k_sweep_s<D, V, false, MODE, 0>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                  (int)sweep_smem_bytes<D, V>());
     return e;
 }
@@ -1162,8 +1165,10 @@ static crocco_status rhs_block(crocco_ctx c, const LocalBlock &b, const double *
         const unsigned grid = cdiv(warps * 32, sweep_threads(d));
 #define SWEEP_LAUNCH(DD, VV, MM)                                                                          \
     do {                                                                                                  \
-        if (ph.lim)                                                                                       \
-            k_sweep_s<DD, VV, true, MM><<<grid, sweep_threads(DD), sweep_smem_bytes<DD, VV>(), c->stream>>>(a, b.L, ph);  \
+        if (!a.inv)                                                                                       \
+            k_sweep_s<DD, VV, false, MM, 0><<<grid, sweep_threads(DD), sweep_smem_bytes<DD, VV>(), c->stream>>>(a, b.L, ph); \
+        else if (ph.lim)                                                                                  \
+            k_sweep_s<DD, VV, true, MM, 2><<<grid, sweep_threads(DD), sweep_smem_bytes<DD, VV>(), c->stream>>>(a, b.L, ph);  \
         else                                                                                              \
             k_sweep_s<DD, VV, false, MM><<<grid, sweep_threads(DD), sweep_smem_bytes<DD, VV>(), c->stream>>>(a, b.L, ph); \
     } while (0)

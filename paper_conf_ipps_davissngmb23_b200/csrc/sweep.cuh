@@ -80,7 +80,9 @@ struct RingGeom {
 
 // MODE = MODE as a template parameter: each launch compiles only its own accumulate / update
 // path (a run-time mode let every direction's kernel carry all five, and their register allocation)
-template <int D, bool VISC, bool LIM, int MODE>
+// INV: 1 inviscid flux on, 0 off (dir_mask / terms), 2 decided at run time by a.inv (the limiter
+// variants: a compile-time 1 makes ptxas spill their eta sweep, measured 19.1 vs 13.3 ms per 512^3 launch)
+template <int D, bool VISC, bool LIM, int MODE, int INV = 1>
 __global__ void __launch_bounds__(sweep_threads(D), sweep_minb(D)) k_sweep_s(const __grid_constant__ SweepArgs a,
                                                                           const Lay L, const Phys ph) {
     using RG = RingGeom<D, VISC>;
@@ -95,7 +97,7 @@ __global__ void __launch_bounds__(sweep_threads(D), sweep_minb(D)) k_sweep_s(con
     const int ls = (D == 0) ? (lane & 7) : (lane >> 3);  // sweep offset of this lane
     const int lt = (D == 0) ? (lane >> 3) : (lane & 7);  // column of this lane
     const int64_t gw = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
-    const bool inv = a.inv != 0;
+    const bool inv = INV == 2 ? a.inv != 0 : INV == 1;
     const int nd = D == 0 ? L.n0 : (D == 1 ? L.n1 : L.n2);
     const int nseg = (nd + a.seg - 1) / a.seg;
     int64_t ntl;
