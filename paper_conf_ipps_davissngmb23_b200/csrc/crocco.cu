@@ -371,7 +371,9 @@ static cudaError_t sweep_attrs() {
     if (e == cudaSuccess) e = sweep_attr1<2, false, 2>();
     if (e == cudaSuccess) e = sweep_attr1<2, false, 3>();
     if (e == cudaSuccess)
-        e = cudaFuncSetAttribute(k_visc_tiled, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)VISC_SMEM);
+        e = cudaFuncSetAttribute(k_visc_tiled<0>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)VISC_SMEM);
+    if (e == cudaSuccess)
+        e = cudaFuncSetAttribute(k_visc_tiled<1>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)VISC_SMEM);
     if (e == cudaSuccess)
         e = cudaFuncSetAttribute(k_visc_exp_tiled, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)VISC_EXP_SMEM);
     return e;
@@ -380,8 +382,12 @@ static cudaError_t sweep_attrs() {
 // one launch of the viscous kernel over `nt` tiles (sel / vk as k_visc_tiled)
 static crocco_status launch_visc(crocco_ctx c, const LocalBlock &b, const double *U, const double *M,
                                  const Phys &ph, int64_t nt, int sel, int vk) {
-    LAUNCH(c, K_VISC, k_visc_tiled<<<(unsigned)nt, VTX * VTY, VISC_SMEM, c->stream>>>(
-                          U, M, b.fv, b.L, b.V, ph, b.racc, b.rcs, sel, vk));
+    if (ph.mu_law == 1)
+        LAUNCH(c, K_VISC, k_visc_tiled<1><<<(unsigned)nt, VTX * VTY, VISC_SMEM, c->stream>>>(
+                              U, M, b.fv, b.L, b.V, ph, b.racc, b.rcs, sel, vk));
+    else
+        LAUNCH(c, K_VISC, k_visc_tiled<0><<<(unsigned)nt, VTX * VTY, VISC_SMEM, c->stream>>>(
+                              U, M, b.fv, b.L, b.V, ph, b.racc, b.rcs, sel, vk));
     return CROCCO_OK;
 }
 

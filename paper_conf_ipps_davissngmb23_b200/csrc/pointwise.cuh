@@ -84,6 +84,9 @@ __host__ __device__ inline VTiles visc_interior_tiles(const Lay &L, int vk) {
 }
 
 // sel: 0 every tile, 1 the ghost-free interior tiles only, 2 every other tile
+// MUL: the viscosity law (ph.mu_law) as a template parameter (the Sutherland branch's sqrt and division
+// otherwise sit in every launch's code)
+template <int MUL>
 __global__ void __launch_bounds__(VTX * VTY, 1) k_visc_tiled(const double *__restrict__ U,
                                                           const double *__restrict__ M,
                                                           double *__restrict__ FV, Lay L, VLay V,
@@ -263,7 +266,7 @@ __global__ void __launch_bounds__(VTX * VTY, 1) k_visc_tiled(const double *__res
                 for (int a = 0; a < 3; a++)
                     gx[f][a] = J * fma(m[0][a], gc[f][0], fma(m[1][a], gc[f][1], m[2][a] * gc[f][2]));
             const double T = win[3][2];
-            const double mu = mu_of_T(ph, T);
+            const double mu = MUL == 1 ? mu_of_T(ph, T) : ph.mu_ref;
             const double kap = mu * ph.cp_over_Pr;
             const double div = gx[0][0] + gx[1][1] + gx[2][2];
             double tau[3][3];

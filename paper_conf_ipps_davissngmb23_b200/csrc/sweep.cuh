@@ -78,7 +78,7 @@ struct RingGeom {
     static constexpr int PER_WARP = SVN * VS + NCB * 32 + NFC;  // doubles
 };
 
-// MODE = MODE as a template parameter: each launch compiles only its own accumulate / update
+// MODE = SweepArgs::mode as a template parameter: each launch compiles only its own accumulate / update
 // path (a run-time mode let every direction's kernel carry all five, and their register allocation)
 // INV: 1 inviscid flux on, 0 off (dir_mask / terms), 2 decided at run time by a.inv (the limiter
 // variants: a compile-time 1 makes ptxas spill their eta sweep, measured 19.1 vs 13.3 ms per 512^3 launch)
