@@ -4,7 +4,7 @@ import json, sys
 def main(md="profiles/r02_ncu.md", summ="profiles/ncu_summary.json", tag=None):
     d = json.load(open(summ))
     ll = {k.replace("crocco::", ""): v for k, v in d["launch_list"].items()
-          if k.startswith("crocco::k_sweep_s") or k in ("crocco::k_visc_tiled", "crocco::k_fill_gather")}
+          if k.startswith(("crocco::k_sweep_s", "crocco::k_visc_tiled", "crocco::k_fill_gather"))}
     tot = sum(v["n"] * v["avg_ms"] for v in ll.values())
     rows = ["| kernel | launches | avg ms | share of step kernels |", "|---|---|---|---|"]
     for k, v in sorted(ll.items(), key=lambda kv: -kv[1]["avg_ms"]):
