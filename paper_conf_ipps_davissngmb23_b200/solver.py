@@ -149,13 +149,23 @@ class Solver:
                                self._ptrs(self.dU), self._ptrs(self.met), graph)
             self.U, self.V = self.V, self.U
 
-    def steps_from_host(self, h_in, h_out, dt):
+    def steps_from_host(self, h_in, h_out, dt, interior=False):
         """Independent RK3 steps streamed through pinned host memory: job n's padded state is
         uploaded from h_in[n] (list over local blocks of flat pinned float64 tensors sized like
         the state arrays), advanced one RK3 step and downloaded into h_out[n].  Uploads and
         downloads run on their own copy streams, so job n's download and job n+1's upload
         overlap the compute of the neighbouring jobs (two device state pairs alternate).
+        interior=True: the host tensors hold only the interior points, (5, n2, n1, n0) per
+        block (the ghosts are the step's own fill), 9 % fewer bytes over the host link at 512^3;
+        the copies go through contiguous device staging (torch).
         Plumbing only: the step itself is crocco_rk3_step."""
+        def dev_view(buf, b):
+            v = self.view(buf, b, 5)
+            return v[:, G:-G, G:-G, G:-G] if interior else buf
+
+        def host_view(h, b):
+            n = self.layouts[b].n
+            return h.view(5, n[2], n[1], n[0]) if interior else h
         if not hasattr(self, "_pairs"):
             self._pairs = [(self.U, self.V), ([self._alloc(L, 5) for L in self.layouts],
                                               [self._alloc(L, 5) for L in self.layouts])]
@@ -172,8 +182,8 @@ class Solver:
             with torch.cuda.stream(self._h2d):
                 if n - 2 in ev_c:
                     self._h2d.wait_event(ev_c[n - 2])          # X clobbered by job n-2's stages
-                for h, x in zip(h_in[n], X):
-                    x.copy_(h, non_blocking=True)
+                for b, (h, x) in enumerate(zip(h_in[n], X)):
+                    dev_view(x, b).copy_(host_view(h, b), non_blocking=True)
                 eh = torch.cuda.Event()
                 eh.record(self._h2d)
             comp.wait_event(eh)
@@ -185,8 +195,8 @@ class Solver:
             ev_c[n].record(comp)
             with torch.cuda.stream(self._d2h):
                 self._d2h.wait_event(ev_c[n])
-                for h, y in zip(h_out[n], Y):
-                    h.copy_(y, non_blocking=True)
+                for b, (h, y) in enumerate(zip(h_out[n], Y)):
+                    host_view(h, b).copy_(dev_view(y, b), non_blocking=True)
                 ev_d[n] = torch.cuda.Event()
                 ev_d[n].record(self._d2h)
         comp.wait_stream(self._d2h)

@@ -568,31 +568,44 @@ def test_compute_dt_reports_non_finite_state():
     S.close()
 
 
-def test_steps_from_host_equals_resident_steps_bitwise():
+@pytest.mark.parametrize("interior", [False, True])
+def test_steps_from_host_equals_resident_steps_bitwise(interior):
     """Solver.steps_from_host (bench e2e: independent jobs through pinned host memory, copies
-    overlapped with compute on two streams) gives each job exactly the resident RK3 step."""
+    overlapped with compute on two streams) gives each job exactly the resident RK3 step;
+    interior=True moves only the interior points (the step's fill makes every ghost it reads)."""
     import torch
     n = (32, 16, 12)
     pb = wavy_random(n, 31, dict(terms=3, mu_ref=0.02))
     S = pb.solver((2, 1, 1))
     jobs = []
     for j in range(5):                           # 5 distinct inputs: state after j resident steps
-        jobs.append([u.detach().cpu().pin_memory() for u in S.U])
+        if interior:
+            jobs.append([S.view(u, b, 5)[:, 4:-4, 4:-4, 4:-4].contiguous().cpu().pin_memory()
+                         for b, u in enumerate(S.U)])
+        else:
+            jobs.append([u.detach().cpu().pin_memory() for u in S.U])
         S.step(1e-3)
     S.sync()
     ref = []
     for j in range(5):                           # resident reference: one step from each input
-        for u, h in zip(S.U, jobs[j]):
-            u.copy_(h)
+        for b, (u, h) in enumerate(zip(S.U, jobs[j])):
+            if interior:
+                S.view(u, b, 5)[:, 4:-4, 4:-4, 4:-4].copy_(h)
+            else:
+                u.copy_(h)
         S.step(1e-3)
         S.sync()
         ref.append([u.detach().cpu().clone() for u in S.U])
     outs = [[torch.empty_like(h).pin_memory() for h in jobs[0]] for _ in range(5)]
-    S.steps_from_host(jobs, outs, 1e-3)
+    # stale ghosts in the device buffers (interior mode must not depend on them)
+    if interior:
+        for buf in S.U + S.V:
+            buf.fill_(float("nan"))
+    S.steps_from_host(jobs, outs, 1e-3, interior=interior)
     torch.cuda.synchronize()
     for j in range(5):
         for b in range(S.nloc):
-            v = S.view(outs[j][b], b, 5)[:, 4:-4, 4:-4, 4:-4]
+            v = outs[j][b] if interior else S.view(outs[j][b], b, 5)[:, 4:-4, 4:-4, 4:-4]
             r = S.view(ref[j][b], b, 5)[:, 4:-4, 4:-4, 4:-4]
             assert torch.equal(v, r), (j, b)
     S.close()
