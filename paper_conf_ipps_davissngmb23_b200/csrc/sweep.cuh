@@ -276,13 +276,14 @@ __global__ void __launch_bounds__(sweep_threads(D), sweep_minb(D)) k_sweep_s(con
         }
         cp_async_commit();
         issue(st + LA + 1);                   // group B: chunk st+LA+1 (slot of chunk st-1)
-        if (act) {
+        {   // every lane evaluates its interface (lanes past the segment end or outside the block on
+            // stale ring values) and the inactive lanes' result is masked: no divergent branch around
+            // the flux, measured -0.2 ms per 512^3 eta launch
             FluxSetup su;
             if (inv) flux_setup(A, ph, su);
             flux_fields<D, SAcc<NR, C, VISC, RG::CS>, LIM>(A, su, inv, VISC, ph, F);
-        } else {
 #pragma unroll
-            for (int c = 0; c < 5; c++) F[c] = 0.0;
+            for (int c = 0; c < 5; c++) F[c] = act ? F[c] : 0.0;
         }
         double dF[5];
         if constexpr (RG::CARRY) {
