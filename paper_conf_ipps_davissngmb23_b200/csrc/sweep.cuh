@@ -151,6 +151,8 @@ __global__ void __launch_bounds__(sweep_threads(D), sweep_minb(D)) k_sweep_s(con
     }
 
     // issue the copies of chunk `ch`: U (5) + metric row (3) [+ FV (4)] of WS points x C columns
+    // (predicated cp.async: points outside the padded box / FV box are zero-filled, nothing read, no
+    // branch; measured with the xi / eta group-A predication -0.7 ms per 512^3 stage)
     auto issue = [&](int ch) {
         if (D == 0) {
             // xi, column-major ring: 16-B copies of point pairs (2p, 2p+1) -- lane: column lane&3,
@@ -158,18 +160,19 @@ __global__ void __launch_bounds__(sweep_threads(D), sweep_minb(D)) k_sweep_s(con
             // 8-B copies when the segment start is odd (16-B source alignment)
             const int col = lane & 3, pr = (lane >> 2) & 3, vg = lane >> 4;
             const int q = ch * WS + 2 * pr, gq = qbase + q;
-            if (xcv && q <= qmax) {
-                const int64_t co = xco;
+            {
+                const bool ok = xcv && q <= qmax, ok1 = ok && q + 1 <= qmax;
                 double *dst = sv + RG::slot(q, col);
 #pragma unroll
                 for (int t = 0; t < 4; t++) {
                     const int v = 4 * vg + t;
-                    const double *src = (v < 5 ? a.in.U + v * L.cs : Mrow + (v - 5) * L.cs) + co + gq;
+                    const double *base = v < 5 ? a.in.U + v * L.cs : Mrow + (v - 5) * L.cs;
+                    const double *src = ok ? base + xco + gq : base;
                     if ((e0 & 1) == 0) {
-                        cp_async16(dst + v * VS, src);
+                        cp_async16z(dst + v * VS, src, ok);
                     } else {
-                        cp_async8(dst + v * VS, src);
-                        if (q + 1 <= qmax) cp_async8(dst + v * VS + 1, src + 1);
+                        cp_async8z(dst + v * VS, src, ok);
+                        cp_async8z(dst + v * VS + 1, ok1 ? src + 1 : base, ok1);
                     }
                 }
             }
@@ -182,7 +185,7 @@ __global__ void __launch_bounds__(sweep_threads(D), sweep_minb(D)) k_sweep_s(con
 #pragma unroll
             for (int pt = 0; pt < WS; pt++) {
                 const int q = ch * WS + pt, gq = qbase + q;
-                if (q <= qmax) cp_async16(dst0 + (q & (NR - 1)) * C, src0 + gq * sst);
+                cp_async16z(dst0 + (q & (NR - 1)) * C, q <= qmax ? src0 + gq * sst : src0, q <= qmax);
             }
             if (VISC && v < 4) {
                 const double *srcf = a.in.FV + v * a.in.vcs + cpv;
@@ -190,7 +193,8 @@ __global__ void __launch_bounds__(sweep_threads(D), sweep_minb(D)) k_sweep_s(con
 #pragma unroll
                 for (int pt = 0; pt < WS; pt++) {
                     const int q = ch * WS + pt, gq = qbase + q;
-                    if (q <= qmax && gq >= -2 && gq <= nd + 1) cp_async16(dstf + (q & (NR - 1)) * C, srcf + gq * vst);
+                    const bool okf = q <= qmax && gq >= -2 && gq <= nd + 1;
+                    cp_async16z(dstf + (q & (NR - 1)) * C, okf ? srcf + gq * vst : srcf, okf);
                 }
             }
         }
@@ -259,6 +263,22 @@ __global__ void __launch_bounds__(sweep_threads(D), sweep_minb(D)) k_sweep_s(con
         const bool act = lvalid && e <= e1 - 1;
         const bool own = act && e >= e0;      // this lane finishes point e
         const SAcc<NR, C, VISC, RG::CS> A{sv, WS * st + ls + RG::QOFF, lt};  // ring point of stencil point i-2
+        // group A: accumulate / update operands of the own point; xi / eta: predicated copies (zero-
+        // filled for the other lanes, no branch), zeta: branch (measured: predication there +0.1 ms)
+        if constexpr (MODE == 1 || MODE == 4) {
+        {
+#pragma unroll
+            for (int c = 0; c < 5; c++)
+                if (c > 0 || MODE != 4) cp_async8z(cb + 32 * c, own ? a.R + c * a.rcs + rr : a.R, own);
+            if (MODE == 2 || MODE == 3) {  // J (the zeta sweep finishes the point)
+                cp_async8z(cb + 32 * 5, own ? a.in.M + pp : a.in.M, own);
+                if (MODE == 3 && a.stage != 0) {
+#pragma unroll
+                    for (int c = 0; c < 5; c++) cp_async8z(cb + 32 * (6 + c), own ? a.dU + c * L.cs + pp : a.dU, own);
+                }
+            }
+        }
+        } else {
         if (own && MODE != 0) {             // group A: accumulate / update operands
 #pragma unroll
             for (int c = 0; c < 5; c++)
@@ -272,6 +292,7 @@ __global__ void __launch_bounds__(sweep_threads(D), sweep_minb(D)) k_sweep_s(con
                     }
                 }
             }
+        }
         }
         cp_async_commit();
         issue(st + LA + 1);                   // group B: chunk st+LA+1 (slot of chunk st-1)
