@@ -24,8 +24,9 @@
 namespace crocco {
 
 // bit D: the three 6-point maxima of direction D as depth-3 trees instead of 6-deep chains (bitwise
-// equal); measured: zeta -0.2 ms, xi +0.3 ms per 512^3 launch -> zeta only
-constexpr int LAM_TREE = 4;
+// equal); round 1: zeta only (zeta -0.2 ms, xi +0.3 ms); on the final round-2 kernels all three
+// directions (with the shared-memory flux carry, sweep.cuh)
+constexpr int LAM_TREE = 7;
 
 struct FluxIn {
     const double *__restrict__ U;

@@ -23,8 +23,10 @@
 namespace crocco {
 
 // bit D: sweep D passes neighbour / carried interface fluxes through shared memory instead of a
-// register carry (measured: eta -4 %, xi +16 %, zeta 0)
-constexpr int CARRY_SMEM = 2;
+// register carry (round 1: eta -4 %, xi +16 %, zeta 0; re-measured at the end of round 2 on the final
+// kernels together with the lambda trees of flux.cuh: all three directions, -0.45 ms per 512^3 stage,
+// profiles/r02_variants_retune_final.jsonl)
+constexpr int CARRY_SMEM = 7;
 // threads per CTA and min CTAs per SM of sweep D: 4 warps, register-limited to 2 CTAs (8 warps)
 // per SM at 253 registers.  Measured (profiles/r02_variants_sweep.jsonl): capping the
 // registers for 10 or 12 warps per SM (2-warp CTAs) spills 150-280 B/thread and runs 25 % slower.
